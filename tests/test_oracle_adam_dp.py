@@ -1,0 +1,74 @@
+"""Pins: oracle Adam vs torch.optim.Adam (reading 17); data-parallel
+linearity with a 2-rank gloo process group (reading 19)."""
+import os
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import synth
+from oracle import StepConfig, adam_update, train_step
+
+
+def test_adam_matches_torch():
+    rng = np.random.default_rng(0)
+    w0 = rng.standard_normal((5, 7))
+    p = torch.tensor(w0.copy(), dtype=torch.float64, requires_grad=True)
+    opt = torch.optim.Adam([p], lr=1e-3, betas=(0.9, 0.999), eps=1e-8)
+    w, m, v = w0.copy(), np.zeros_like(w0), np.zeros_like(w0)
+    for step in range(1, 6):
+        g = rng.standard_normal(w0.shape) * 10 ** rng.uniform(-4, 1)
+        p.grad = torch.tensor(g)
+        opt.step()
+        w, m, v = adam_update(w, g, m, v, step)
+        np.testing.assert_allclose(w, p.detach().numpy(), rtol=1e-14, atol=1e-15)
+
+
+def _dp_worker(rank, world, port, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    T, B = 10, 4
+    x, y = synth.make_inputs(net, T, B)
+    shard = slice(rank * B // world, (rank + 1) * B // world)
+    xs, ys = x[:, shard], y[shard]
+    # phase 1: local first pass gives the local s; allreduce it (int64 sum)
+    r0 = train_step(net, W, xs, ys, StepConfig(T=T, C=2, mode="ckpt", global_batch=B))
+    s = torch.tensor(r0.s)
+    dist.all_reduce(s)
+    r = train_step(net, W, xs, ys, StepConfig(T=T, C=2, mode="skip", p=50.0, global_batch=B,
+                                              s_global=s.numpy()))
+    grads = [torch.tensor(g) for g in r.dW]
+    for g in grads:
+        dist.all_reduce(g)
+    loss = torch.tensor([r.loss], dtype=torch.float64)
+    dist.all_reduce(loss)
+    if rank == 0:
+        out.put((float(loss[0]), [g.numpy() for g in grads], r.keep.copy(), s.numpy()))
+    dist.destroy_process_group()
+
+
+def test_data_parallel_sharding_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29500 + os.getpid() % 1000
+    procs = [ctx.Process(target=_dp_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    loss, grads, keep, s = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, 10, 4)
+    ref = train_step(net, W, x, y, StepConfig(T=10, C=2, mode="skip", p=50.0))
+    np.testing.assert_array_equal(s, ref.s)
+    np.testing.assert_array_equal(keep, ref.keep)
+    assert loss == pytest.approx(ref.loss, rel=1e-12)
+    for a, b in zip(grads, ref.dW):
+        np.testing.assert_allclose(a, b, rtol=1e-10, atol=1e-14)

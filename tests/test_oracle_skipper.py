@@ -1,0 +1,138 @@
+"""Pins for SAM / SST / keep mask (Eq.4-5), the checkpoint schedule (Fig. 5/6)
+and the memory laws (Eq.3, Eq.6, Eq.7)."""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import StepConfig, train_step, keep_mask, spike_sum_threshold, kept_lists
+from oracle.skipper import eq7_p_max, ledger_model
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def test_sst_hand_examples():
+    for case in json.load(open(os.path.join(GOLD, "sst_hand_examples.json")))["cases"]:
+        s = np.array(case["s"])
+        keep = keep_mask(s, case["T"], case["C"], case["p"])
+        assert keep.astype(int).tolist() == case["keep"], case
+        if case["sst"] is not None:
+            np.testing.assert_allclose(spike_sum_threshold(s, case["T"], case["C"], case["p"]),
+                                       case["sst"], rtol=0, atol=1e-12)
+
+
+def test_kept_count_order_statistics():
+    """With distinct spike sums, exactly S-1-floor((S-1)p/100) values of a segment
+    exceed the linear-interpolated percentile (order statistics)."""
+    rng = np.random.default_rng(11)
+    for _ in range(200):
+        C = int(rng.integers(1, 5))
+        S = int(rng.integers(2, 30))
+        T = C * S
+        p = float(rng.uniform(1, 99))
+        s = rng.permutation(10 * T)[:T]
+        keep = keep_mask(s, T, C, p)
+        sst = spike_sum_threshold(s, T, C, p)
+        for c in range(C):
+            seg = s[c * S:(c + 1) * S]
+            n_gt = S - 1 - math.floor((S - 1) * p / 100)
+            expect = 1 + n_gt - int(seg[0] > sst[c])
+            assert keep[c * S:(c + 1) * S].sum() == expect
+
+
+def test_sam_brute_force():
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    T = 10
+    x, y = synth.make_inputs(net, T, 3)
+    r = train_step(net, W, x, y, StepConfig(T=T, mode="full", record=True))
+    for t in range(T):
+        brute = int(x[t].astype(np.int64).sum())
+        for o in r.first_o:
+            brute += int(np.count_nonzero(o[t]))
+        assert r.s[t] == brute
+
+
+def _events(trace, kind):
+    return [t for k, t in trace if k == kind]
+
+
+def test_fig5_schedule_T20_C2():
+    g = json.load(open(os.path.join(GOLD, "fig5_schedule_T20_C2.json")))
+    net = synth.net_config("tiny_fc")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, g["T"], 2)
+    r = train_step(net, W, x, y, StepConfig(T=g["T"], C=g["C"], mode="ckpt", trace=True))
+    assert _events(r.trace, "ckpt") == g["checkpoints"]
+    assert _events(r.trace, "first") == list(range(g["T"]))
+    assert _events(r.trace, "loss") == [g["loss_at"]]
+    # split the backward part of the trace per release
+    seq = r.trace[r.trace.index(("loss", g["loss_at"])) + 1:]
+    segs, cur = [], []
+    for ev in seq:
+        if ev[0] == "release":
+            segs.append((ev[1], cur))
+            cur = []
+        else:
+            cur.append(ev)
+    assert len(segs) == len(g["segments_in_backward_order"])
+    for (c, evs), ref in zip(segs, g["segments_in_backward_order"]):
+        assert c == ref["segment"]
+        assert _events(evs, "recompute") == ref["recompute"]
+        assert _events(evs, "bptt") == ref["bptt"]
+    # "the recomputation for each time step happens only once"
+    rec = _events(r.trace, "recompute")
+    assert len(rec) == len(set(rec)) == g["T"] - g["C"]
+
+
+def test_fig6_skip_eligibility():
+    g = json.load(open(os.path.join(GOLD, "fig5_schedule_T20_C2.json")))
+    rng = np.random.default_rng(0)
+    for p in [10.0, 50.0, 90.0]:
+        s = rng.integers(0, 1000, g["T"])
+        keep = keep_mask(s, g["T"], g["C"], p)
+        assert keep[0] and keep[10]
+        skipped = set(np.nonzero(~keep)[0].tolist())
+        assert skipped <= set(sum(g["skipper_eligible"], []))
+
+
+def test_ledger_matches_eq3_eq6_and_sqrtT():
+    net = synth.net_config("tiny_fc")
+    W = synth.make_weights(net)
+    B = 2
+    N = sum(L["cout"] for L in net["layers"] if L["kind"] != "readout")
+    T = 36
+    x, y = synth.make_inputs(net, T, B)
+    per = 5  # U float32 + o uint8 per stored neuron-step
+    rf = train_step(net, W, x, y, StepConfig(T=T, mode="full"))
+    assert rf.ledger_peak == ledger_model("full", T, 1, per, B * N)
+    peaks = {}
+    for C in [2, 3, 4, 6, 9, 12, 18]:
+        rc = train_step(net, W, x, y, StepConfig(T=T, C=C, mode="ckpt"))
+        assert rc.ledger_peak == ledger_model("ckpt", T, C, per, B * N)
+        rs = train_step(net, W, x, y, StepConfig(T=T, C=C, mode="skip", p=50.0))
+        kmax = max(len(k) for k in rs.kept)
+        assert rs.ledger_peak == ledger_model("skip", T, C, per, B * N, kept_max=kmax)
+        assert rs.ledger_peak <= rc.ledger_peak < rf.ledger_peak
+        peaks[C] = rc.ledger_peak
+    assert min(peaks, key=peaks.get) == 6          # C* = sqrt(T)
+
+
+def test_memory_sublinear_in_T():
+    """Eq.3 at C = sqrt(T): ActCost ~ 2 sqrt(T) - quadrupling T doubles memory; FULL is linear."""
+    for T in [16, 64, 256]:
+        C = int(math.isqrt(T))
+        full = ledger_model("full", T, 1, 5, 100)
+        ck = ledger_model("ckpt", T, C, 5, 100)
+        assert full == T * 500
+        assert ck == 2 * C * 500
+    assert ledger_model("ckpt", 256, 16, 5, 1) / ledger_model("ckpt", 64, 8, 5, 1) == 2
+
+
+def test_eq7_bounds_for_workloads():
+    assert eq7_p_max(100, 10, 6) == pytest.approx(40.0)    # cfg 2 -> p=40
+    assert eq7_p_max(200, 5, 11) == pytest.approx(72.5)    # cfg 3
+    assert eq7_p_max(20, 2, 2) == pytest.approx(80.0)      # cfg 1
