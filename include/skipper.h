@@ -1,0 +1,181 @@
+/*
+ * skipper.h - C ABI of the B200 (sm_100a) Skipper SNN training hot path.
+ *
+ * Paper: Singh et al., "Skipper: Enabling efficient SNN training through
+ * activation-checkpointing and time-skipping", MICRO 2022.  Citations P:<n>
+ * are lines of the paper text; SURVEY.md §8 is the scope contract.
+ *
+ * What one training iteration computes (skipper_step):
+ *   FIRST forward pass over t = 0..T-1 (Fig. 5/6 Step 1):
+ *     LIF dynamics, Eq.1:  U_t = lam*U_{t-1} + W o^{l-1}_t - theta*o_{t-1},
+ *     o_t = [U_t > theta]; the state (U, o) of every spiking layer is stored only at
+ *     the segment starts t = cS (the checkpoints); SAM spike sums s_t, Eq.4.
+ *   readout + loss at t = T-1 (readout reading 5 of SURVEY.md §8(c)).
+ *   SST_c, Eq.5, keep t iff s_t > SST_c [mode SKIP].
+ *   for c = C-1..0: RECOMPUTE the kept steps of segment c from its checkpoint
+ *     (P:742-748), then BACKWARD through them with the surrogate
+ *     gradient, Eq.2, carrying dL/dU of the segment start to c-1
+ *     (P:750-753); segment memory is released.
+ *   data-parallel gradient allreduce and Adam.
+ *
+ * Conventions
+ *   - Pointers named *_dev are CUDA device pointers, *_host are host pointers.
+ *   - Every call is stream-ordered on the stream given to skipper_create, except
+ *     the calls documented as synchronising (they say "host sync").
+ *   - Layouts are row-major, NHWC for images.  Input spikes x are uint8 {0,1}
+ *     of shape [T][B][H][W][C] (conv first layer) or [T][B][D] (fc first layer),
+ *     B = cfg.batch (the per-rank batch).  Labels are int32 [B].
+ *   - Weights are float32, per layer:  fc [cout][cin];  conv [cout][3][3][cin];
+ *     readout [classes][cin].  fc layers read the previous conv output flattened
+ *     in (h, w, c) order.
+ *   - Ownership: the caller owns x, labels and any output buffer and keeps them
+ *     alive until the stream reaches the call.  The context owns all state and
+ *     workspace and allocates device memory through the allocator given at
+ *     creation (NULL -> cudaMallocAsync on the context stream).
+ *   - Errors: every call returns a skipper_status; skipper_last_error() gives the
+ *     message.  A CUDA or NCCL error poisons the context (later calls return
+ *     SKIPPER_EFAILED).  Argument or call-order errors leave the weights untouched.
+ *   - A context is not thread-safe; use one per rank / per thread.
+ */
+#ifndef SKIPPER_H
+#define SKIPPER_H
+
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct skipper_ctx skipper_ctx;
+
+typedef enum {
+    SKIPPER_OK = 0,
+    SKIPPER_EINVAL = 1,       /* invalid argument / configuration                  */
+    SKIPPER_ENOMEM = 2,       /* allocator returned NULL                            */
+    SKIPPER_ECUDA = 3,        /* CUDA error (context poisoned)                      */
+    SKIPPER_ENCCL = 4,        /* NCCL error (context poisoned)                      */
+    SKIPPER_EORDER = 5,       /* segment calls out of the order Fig. 5/6 require    */
+    SKIPPER_EFAILED = 6,      /* context previously poisoned                        */
+    SKIPPER_EUNSUPPORTED = 7  /* layer geometry this build has no kernel for        */
+} skipper_status;
+
+typedef enum { SKIPPER_MODE_FULL = 0, SKIPPER_MODE_CKPT = 1, SKIPPER_MODE_SKIP = 2 } skipper_mode;
+typedef enum { SKIPPER_PASS_FIRST = 0, SKIPPER_PASS_RECOMPUTE = 1, SKIPPER_PASS_RECORD = 2 } skipper_pass;
+typedef enum { SKIPPER_LAYER_FC = 0, SKIPPER_LAYER_CONV3X3 = 1, SKIPPER_LAYER_READOUT = 2 } skipper_layer_kind;
+typedef enum { SKIPPER_SURR_TRIANGLE = 0, SKIPPER_SURR_FAST_SIGMOID = 1 } skipper_surrogate;
+
+/* One layer.  conv3x3: stride 1, zero pad 1, input and output h x w, optional 2x2
+ * average pooling of the output spikes (pool = 2).  fc: h = w = 1.  The last layer
+ * must be the (non-spiking) readout; lambda/theta are ignored for it. */
+typedef struct {
+    int kind;        /* skipper_layer_kind */
+    int cin, cout;
+    int h, w;
+    int pool;        /* 0 or 2 */
+    float lambda;    /* leak, Eq.1 (lambda < 1; 1 = integrate-and-fire) */
+    float theta;     /* firing threshold, Eq.1 */
+} skipper_layer;
+
+typedef struct {
+    int T;                 /* timesteps */
+    int C;                 /* checkpoints = segments; T % C == 0, C < T/L_n */
+    double p;              /* SST percentile in [0, 100); 0 => no skipping (Eq.5) */
+    int mode;              /* skipper_mode (FULL ignores C and p) */
+    int batch;             /* per-rank batch B */
+    int global_batch;      /* loss normaliser (sum over ranks of batch); 0 => batch */
+    int surrogate;         /* skipper_surrogate */
+    float surr_gamma;      /* triangle: peak; fast sigmoid: slope */
+    float lr, beta1, beta2, eps;   /* Adam */
+    int debug_record;      /* 1: keep per-step states for skipper_debug_copy (tests) */
+} skipper_config;
+
+/* Device-memory allocator used for every context allocation. */
+typedef struct {
+    void *(*alloc)(size_t bytes, void *stream, void *user);
+    void (*free)(void *ptr, size_t bytes, void *stream, void *user);
+    void *user;
+} skipper_allocator;
+
+/* Create a context: validates the network and configuration (EINVAL with a
+ * message on failure; a p above the Eq.7 bound is accepted and
+ * reported by skipper_last_error as a warning), allocates weights, optimizer
+ * moments, checkpoint store and persistent buffers.  Weights start at zero:
+ * call skipper_set_weights for every layer.  cuda_stream may be NULL (legacy
+ * default stream).  On failure *out is NULL and the message is available from
+ * skipper_last_error(NULL). */
+skipper_status skipper_create(const skipper_layer *layers, int n_layers, const skipper_config *cfg,
+                              const skipper_allocator *alloc, void *cuda_stream, skipper_ctx **out);
+void skipper_destroy(skipper_ctx *ctx);
+const char *skipper_last_error(const skipper_ctx *ctx);   /* ctx may be NULL */
+
+/* Weights, float32 on the device, layout per the conventions above.  set copies
+ * into the fp32 master and refreshes the bf16 shadows used by the tensor cores;
+ * it resets nothing else.  get_grads returns dL/dW of the last completed
+ * backward (summed over ranks after skipper_optimizer_step / skipper_step). */
+skipper_status skipper_set_weights(skipper_ctx *ctx, int layer, const float *w_dev);
+skipper_status skipper_get_weights(skipper_ctx *ctx, int layer, float *w_dev);
+skipper_status skipper_get_grads(skipper_ctx *ctx, int layer, float *dw_dev);
+size_t skipper_weight_count(const skipper_ctx *ctx, int layer);
+
+/* ---- segment-level calls (the pieces skipper_step composes) ----------------
+ * Order (EORDER otherwise):
+ *   CKPT/SKIP: forward_segment(c, FIRST) for c = 0..C-1 (the call for c = C-1
+ *              takes labels_dev, computes the loss and dL/dz, allreduces s over
+ *              ranks and fixes the keep mask - one host sync);
+ *              then for c = C-1..0: forward_segment(c, RECOMPUTE), backward_segment(c);
+ *              then optimizer_step.
+ *   FULL:      forward_segment(0, RECORD) (all T steps stored, takes labels_dev),
+ *              backward_segment(0), optimizer_step.
+ * x_dev is the whole input [T][B][...] (uint8) and must be the same pointer
+ * contents for every call of one iteration. */
+skipper_status skipper_forward_segment(skipper_ctx *ctx, int seg, int pass,
+                                       const unsigned char *x_dev, const int *labels_dev);
+skipper_status skipper_backward_segment(skipper_ctx *ctx, int seg);
+/* Allreduce dW over ranks (if skipper_comm_init was called) and apply Adam. */
+skipper_status skipper_optimizer_step(skipper_ctx *ctx);
+
+/* One full training iteration on device-resident inputs.  loss_host may be NULL
+ * (then the only host sync of the step is the one that fixes the keep mask). */
+skipper_status skipper_step(skipper_ctx *ctx, const unsigned char *x_dev, const int *labels_dev,
+                            float *loss_host);
+/* Same, end to end from host memory: copies x [T][B][...] and labels to the
+ * device inside the call (pinned host memory gives asynchronous copies), runs
+ * the step and copies the loss back (host sync). */
+skipper_status skipper_step_host(skipper_ctx *ctx, const unsigned char *x_host, const int *labels_host,
+                                 float *loss_host);
+
+/* ---- data parallelism (batch-sharded) ---------- */
+skipper_status skipper_comm_unique_id(unsigned char id_out[128]);
+skipper_status skipper_comm_init(skipper_ctx *ctx, const unsigned char id[128], int rank, int world);
+
+/* ---- introspection (host sync) ----------------------------------------------- */
+skipper_status skipper_get_loss(skipper_ctx *ctx, float *loss_host);
+skipper_status skipper_get_spike_sums(skipper_ctx *ctx, long long *s_host);      /* [T], global */
+skipper_status skipper_get_keep_mask(skipper_ctx *ctx, unsigned char *keep_host); /* [T] */
+skipper_status skipper_get_sst(skipper_ctx *ctx, double *sst_host);               /* [C]; NaN if p == 0 */
+skipper_status skipper_mem_stats(skipper_ctx *ctx, size_t *current_bytes, size_t *peak_bytes);
+skipper_status skipper_reset_peak(skipper_ctx *ctx);
+
+/* Debug copies (require cfg.debug_record = 1), device to device:
+ *   which 0: first-pass U   float32 [T][B*N_l]
+ *   which 1: first-pass o   uint8   [T][B*N_l]
+ *   which 2: recomputed U   float32 [T][B*N_l]  (rows of kept t; others 0)
+ *   which 3: recomputed o   uint8   [T][B*N_l]
+ * N_l is the un-pooled neuron count of spiking layer `layer` (0-based). */
+skipper_status skipper_debug_copy(skipper_ctx *ctx, int which, int layer, void *dst_dev, size_t bytes);
+
+/* Pure host functions (no GPU needed). */
+/* Eq.5 for one segment: p-th percentile of n int64 values, numpy 'linear' method. */
+double skipper_sst_host(const long long *s, int n, double p);
+/* Stored neuron-state bytes at the peak for a mode (the Eq.3 / Eq.6 model with
+ * this build's storage: fp32 U + bf16 output per stored step, fp32 U + u8 o per
+ * checkpoint); kept_max < 0 means T/C. */
+size_t skipper_workspace_bytes(const skipper_layer *layers, int n_layers, const skipper_config *cfg,
+                               int kept_max);
+const char *skipper_status_string(int status);
+const char *skipper_build_info(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SKIPPER_H */

@@ -1,0 +1,42 @@
+/*
+ * skipper_kernels.h - kernel-level entry points of the sm_100a library, for
+ * per-kernel parity tests and micro-benchmarks.  They launch exactly the
+ * kernels skipper_step uses (same launchers), stream-ordered on `stream`.
+ * All pointers are device pointers; bf16 tensors are passed as uint16 bit
+ * patterns.  Return value: a skipper_status (0 = OK); on a CUDA error the
+ * message is in skipper_last_error(NULL).
+ *
+ * Contractions (the synaptic GEMMs of Eq.1 forward and Eq.2 backward),
+ * all bf16 x bf16 -> fp32 on the tcgen05 tensor cores:
+ *   fc_fwd     C[M][N]  = A[M][K] . B[N][K]^T                 (I = P(o) W^T; dgrad g = delta Wt^T)
+ *   fc_wgrad   dW[N][K] (+)= D[M][N]^T . X[M][K]              (dW = sum_rows delta^T a)
+ *   conv_fwd   Y[nb,y,x,co] = sum_{dy,dx,ci} Wk[co][dy*3+dx][ci] X[nb,y+dy-1,x+dx-1,ci]   (pad 1)
+ *   conv_dgrad G[nb,y,x,ci] = sum_{dy,dx,co} Wt[ci][dy*3+dx][co] D[nb,y-dy+1,x-dx+1,co]
+ *   conv_wgrad dW[co][dy*3+dx][ci] (+)= sum_{nb,y,x} D[nb,y,x,co] X[nb,y+dy-1,x+dx-1,ci]
+ * Shape limits: K, N, cin, cout multiples of 8 (16-byte rows); conv h*w*... see DESIGN.md.
+ */
+#ifndef SKIPPER_KERNELS_H
+#define SKIPPER_KERNELS_H
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+int skipper_k_fc_fwd(const unsigned short *A, const unsigned short *B, float *C,
+                     int M, int N, int K, void *stream);
+int skipper_k_fc_wgrad(const unsigned short *D, const unsigned short *X, float *dW,
+                       int M, int N, int K, int accumulate, void *stream);
+int skipper_k_conv_fwd(const unsigned short *X, const unsigned short *Wk, float *Y,
+                       int nb, int h, int w, int cin, int cout, void *stream);
+int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, float *G,
+                         int nb, int h, int w, int cin, int cout, void *stream);
+int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float *dW,
+                         int nb, int h, int w, int cin, int cout, int accumulate, void *stream);
+
+/* Number of SMs the persistent kernels size their grids for (148 on B200). */
+int skipper_k_num_sms(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

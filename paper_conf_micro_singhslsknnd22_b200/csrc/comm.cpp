@@ -1,0 +1,97 @@
+// comm.cpp - NCCL entry points resolved at run time (see comm.h).
+#include "comm.h"
+
+#include <dlfcn.h>
+#include <cstring>
+#include <mutex>
+
+#include <nccl.h>
+
+namespace sk {
+namespace {
+
+struct Nccl {
+    void *h = nullptr;
+    decltype(&ncclGetUniqueId) getUniqueId = nullptr;
+    decltype(&ncclCommInitRank) commInitRank = nullptr;
+    decltype(&ncclAllReduce) allReduce = nullptr;
+    decltype(&ncclCommDestroy) commDestroy = nullptr;
+    decltype(&ncclGetErrorString) errStr = nullptr;
+    bool ok = false;
+};
+
+Nccl &nccl() {
+    static Nccl n;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        const char *names[] = {"libnccl.so.2", "libnccl.so"};
+        for (const char *nm : names) {
+            n.h = dlopen(nm, RTLD_NOW | RTLD_GLOBAL);
+            if (n.h) break;
+        }
+        if (!n.h) return;
+        n.getUniqueId = reinterpret_cast<decltype(n.getUniqueId)>(dlsym(n.h, "ncclGetUniqueId"));
+        n.commInitRank = reinterpret_cast<decltype(n.commInitRank)>(dlsym(n.h, "ncclCommInitRank"));
+        n.allReduce = reinterpret_cast<decltype(n.allReduce)>(dlsym(n.h, "ncclAllReduce"));
+        n.commDestroy = reinterpret_cast<decltype(n.commDestroy)>(dlsym(n.h, "ncclCommDestroy"));
+        n.errStr = reinterpret_cast<decltype(n.errStr)>(dlsym(n.h, "ncclGetErrorString"));
+        n.ok = n.getUniqueId && n.commInitRank && n.allReduce && n.commDestroy && n.errStr;
+    });
+    return n;
+}
+
+bool check(ncclResult_t r, const char *what, std::string *err) {
+    if (r == ncclSuccess) return true;
+    if (err) *err = std::string(what) + ": " + (nccl().errStr ? nccl().errStr(r) : "nccl error");
+    return false;
+}
+
+}  // namespace
+
+bool Comm::unique_id(unsigned char id[128], std::string *err) {
+    Nccl &n = nccl();
+    if (!n.ok) {
+        if (err) *err = "libnccl.so.2 not found (dlopen)";
+        return false;
+    }
+    ncclUniqueId u;
+    if (!check(n.getUniqueId(&u), "ncclGetUniqueId", err)) return false;
+    static_assert(sizeof(u) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(id, &u, 128);
+    return true;
+}
+
+bool Comm::init(const unsigned char id[128], int r, int w, std::string *err) {
+    Nccl &n = nccl();
+    if (!n.ok) {
+        if (err) *err = "libnccl.so.2 not found (dlopen)";
+        return false;
+    }
+    ncclUniqueId u;
+    std::memcpy(&u, id, 128);
+    ncclComm_t c = nullptr;
+    if (!check(n.commInitRank(&c, w, u, r), "ncclCommInitRank", err)) return false;
+    comm = c;
+    rank = r;
+    world = w;
+    return true;
+}
+
+bool Comm::allreduce_i64(long long *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    return check(nccl().allReduce(buf, buf, cnt, ncclInt64, ncclSum, static_cast<ncclComm_t>(comm), s),
+                 "ncclAllReduce(s)", err);
+}
+
+bool Comm::allreduce_f32(float *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    return check(nccl().allReduce(buf, buf, cnt, ncclFloat32, ncclSum, static_cast<ncclComm_t>(comm), s),
+                 "ncclAllReduce(dW)", err);
+}
+
+void Comm::destroy() {
+    if (comm && nccl().ok) nccl().commDestroy(static_cast<ncclComm_t>(comm));
+    comm = nullptr;
+    world = 1;
+    rank = 0;
+}
+
+}  // namespace sk

@@ -1,0 +1,1271 @@
+// engine.cpp - the C ABI of include/skipper.h: context, validation, memory plan and the
+// segment schedule of checkpointed / Skipper BPTT (Sec. V Fig. 5, Sec. VI-A Fig. 6).
+//
+// Per iteration (SKIP mode):
+//   stage input (SAM l=0) -> FIRST pass over segments 0..C-1 (layer-major inside a segment:
+//   GEMM over all S timesteps, then the LIF scan walks t; checkpoint (U,o) at t=cS) ->
+//   readout + loss -> [allreduce s] -> host SST_c (Eq.5) and keep lists (one host sync) ->
+//   for c = C-1..0 { RECOMPUTE kept rows from checkpoint c ; BACKWARD: K4 scan, wgrad, dgrad }
+//   -> [allreduce dW] -> Adam.
+#include "../../include/skipper.h"
+#include "gemm.h"
+#include "kernels.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "comm.h"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+struct Layer {
+    skipper_layer d{};
+    bool fc = false, conv = false, pool = false, direct = false, readout = false;
+    int H = 1, W = 1, Cin = 0, Cout = 0, PH = 1, PW = 1;
+    long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
+    size_t wcount = 0;
+    float *w = nullptr, *dw = nullptr, *m = nullptr, *v = nullptr;
+    uint16_t *wb = nullptr, *wt = nullptr;
+    float *U_run = nullptr, *ckU = nullptr, *carry = nullptr;
+    uint8_t *o_run = nullptr, *cko = nullptr;
+    uint16_t *Po = nullptr;    // arena rows
+    float *Useg = nullptr;     // arena rows
+    float *dbg[2] = {nullptr, nullptr};     // first / recompute U
+    uint8_t *dbgo[2] = {nullptr, nullptr};  // first / recompute o
+};
+
+enum Phase { PH_IDLE = 0, PH_FIRST, PH_READY_BWD, PH_RECOMPUTED, PH_BWD_DONE };
+
+}  // namespace
+
+struct skipper_ctx {
+    std::vector<Layer> L;  // spiking layers then readout (L.back())
+    int Ls = 0;            // number of spiking layers
+    skipper_config cfg{};
+    skipper_allocator alloc{};
+    bool own_alloc = true;
+    cudaStream_t st = nullptr;
+    int T = 0, C = 1, S = 0, B = 0, Bg = 0;
+    int num_sms = 148;
+    bool input_direct = false;  // first layer is the fused direct conv
+    int in_h = 1, in_w = 1, in_c = 0;
+    long long in_elems = 0;     // per sample
+    // persistent
+    uint32_t *xmask = nullptr;
+    uint16_t *xb = nullptr;
+    unsigned *s_part = nullptr;
+    long long *s_dev = nullptr;
+    float *cnt = nullptr, *cnt_kept = nullptr, *z = nullptr, *dz = nullptr, *loss_dev = nullptr, *g_last = nullptr;
+    int *kept_dev = nullptr;
+    float *dw_all = nullptr;
+    size_t dw_total = 0;
+    unsigned char *x_stage = nullptr;
+    int *y_stage = nullptr;
+    // host-side step state
+    std::vector<long long> s_host;
+    std::vector<unsigned char> keep;
+    std::vector<double> sst;
+    std::vector<std::vector<int>> kept;
+    std::vector<int> kept_flat;
+    int Kmax = 0;
+    // arenas
+    void *arena = nullptr;
+    size_t arena_bytes = 0;
+    float *I_buf = nullptr;     // currents (fwd) and gradients wrt spikes (dgrad)
+    uint16_t *d_buf = nullptr;  // delta (bf16)
+    uint16_t *P2[2] = {nullptr, nullptr};
+    uint16_t *xg = nullptr;     // gathered fc-first input rows
+    // schedule state
+    int phase = PH_IDLE;
+    int next_seg = 0;
+    bool grads_ready = false;
+    long long adam_step = 0;
+    const unsigned char *x_cur = nullptr;
+    // memory accounting
+    size_t cur_bytes = 0, peak_bytes = 0;
+    std::string err;
+    bool poisoned = false;
+    // comm
+    sk::Comm comm;
+    // profiling (per kernel class: launches, device ms, algorithmic bytes and flops)
+    bool prof_on = false;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    struct ProfRec { int cls; cudaEvent_t a, b; double bytes, flops; };
+    std::vector<ProfRec> prof_recs;
+    long long prof_n[16] = {0};
+    double prof_ms[16] = {0}, prof_bytes[16] = {0}, prof_flops[16] = {0};
+    long long launches = 0;
+};
+
+enum KClass {
+    K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_DIRECT_FWD, K_READOUT, K_SCAN_BWD, K_DIRECT_BWD,
+    K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_GATHER, K_NCLASS
+};
+static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "direct_conv_lif_fwd",
+                                               "readout_loss", "lif_bwd_scan", "direct_conv_bwd_wgrad",
+                                               "gemm_wgrad", "gemm_dgrad", "adam", "gather"};
+
+static cudaEvent_t ev_get(skipper_ctx *c) {
+    if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    c->ev_pool.push_back(e);
+    c->ev_used++;
+    return e;
+}
+
+// One kernel launch: counts it and, when profiling, brackets it with CUDA events on the
+// context stream together with its algorithmic bytes / flops.
+struct ProfScope {
+    skipper_ctx *c;
+    int rec = -1;
+    ProfScope(skipper_ctx *c_, int cls, double bytes, double flops) : c(c_) {
+        c->launches++;
+        if (!c->prof_on) return;
+        cudaEvent_t a = ev_get(c), b = ev_get(c);
+        cudaEventRecord(a, c->st);
+        c->prof_recs.push_back({cls, a, b, bytes, flops});
+        rec = (int)c->prof_recs.size() - 1;
+    }
+    ~ProfScope() {
+        if (rec >= 0) cudaEventRecord(c->prof_recs[rec].b, c->st);
+    }
+};
+
+static void prof_resolve(skipper_ctx *c) {
+    if (c->prof_recs.empty()) return;
+    cudaEventSynchronize(c->prof_recs.back().b);
+    for (auto &r : c->prof_recs) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, r.a, r.b) == cudaSuccess) {
+            c->prof_n[r.cls] += 1;
+            c->prof_ms[r.cls] += ms;
+            c->prof_bytes[r.cls] += r.bytes;
+            c->prof_flops[r.cls] += r.flops;
+        }
+    }
+    c->prof_recs.clear();
+    c->ev_used = 0;
+}
+
+// ------------------------------------------------------------------------------------ helpers
+static skipper_status fail(skipper_ctx *c, skipper_status s, const char *fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) {
+        c->err = buf;
+        if (s == SKIPPER_ECUDA || s == SKIPPER_ENCCL) c->poisoned = true;
+    }
+    g_last_error = buf;
+    return s;
+}
+
+#define CK(call)                                                                                     \
+    do {                                                                                             \
+        cudaError_t e_ = (call);                                                                     \
+        if (e_ != cudaSuccess)                                                                       \
+            return fail(c, SKIPPER_ECUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_)); \
+    } while (0)
+
+#define CKS(expr)                            \
+    do {                                     \
+        skipper_status s_ = (expr);          \
+        if (s_ != SKIPPER_OK) return s_;     \
+    } while (0)
+
+static size_t al256(size_t n) { return (n + 255) & ~size_t(255); }
+
+static void *dev_alloc(skipper_ctx *c, size_t bytes) {
+    if (bytes == 0) return nullptr;
+    bytes = al256(bytes);
+    void *p = nullptr;
+    if (c->own_alloc) {
+        if (cudaMallocAsync(&p, bytes, c->st) != cudaSuccess) p = nullptr;
+    } else {
+        p = c->alloc.alloc(bytes, c->st, c->alloc.user);
+    }
+    if (p) {
+        c->cur_bytes += bytes;
+        c->peak_bytes = std::max(c->peak_bytes, c->cur_bytes);
+    }
+    return p;
+}
+
+static void dev_free(skipper_ctx *c, void *p, size_t bytes) {
+    if (!p) return;
+    bytes = al256(bytes);
+    if (c->own_alloc)
+        cudaFreeAsync(p, c->st);
+    else
+        c->alloc.free(p, bytes, c->st, c->alloc.user);
+    c->cur_bytes -= bytes;
+}
+
+template <typename T>
+static skipper_status alloc_arr(skipper_ctx *c, T **p, size_t n) {
+    *p = static_cast<T *>(dev_alloc(c, n * sizeof(T)));
+    if (n && !*p) return fail(c, SKIPPER_ENOMEM, "device allocation of %zu bytes failed", n * sizeof(T));
+    return SKIPPER_OK;
+}
+template <typename T>
+static void free_arr(skipper_ctx *c, T *&p, size_t n) {
+    dev_free(c, p, n * sizeof(T));
+    p = nullptr;
+}
+
+// ------------------------------------------------------------------------------------ SST (Eq.5)
+// numpy.percentile(a, p) with the default 'linear' method, replicated operation by operation:
+// q = p / 100; vi = (n-1)*q; lo = floor(vi); g = vi - lo;
+// lerp(a, b, g) = a + (b-a)*g, or b - (b-a)*(1-g) when g >= 0.5.
+extern "C" double skipper_sst_host(const long long *s, int n, double p) {
+    if (n <= 0) return NAN;
+    std::vector<long long> v(s, s + n);
+    std::sort(v.begin(), v.end());
+    const double q = p / 100.0;
+    const double vi = (double)(n - 1) * q;
+    double lo_d = std::floor(vi);
+    long long lo = (long long)lo_d;
+    if (lo < 0) lo = 0;
+    if (lo > n - 1) lo = n - 1;
+    long long hi = std::min<long long>(lo + 1, n - 1);
+    const double g = vi - lo_d;
+    const long long diff = v[hi] - v[lo];
+    const double a = (double)v[lo], b = (double)v[hi];
+    if (g >= 0.5) return b - (double)diff * (1.0 - g);
+    return a + (double)diff * g;
+}
+
+// ------------------------------------------------------------------------------------ create
+static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *layers, int n) {
+    if (!layers || n < 2) return fail(c, SKIPPER_EINVAL, "need at least one spiking layer and a readout");
+    if (layers[n - 1].kind != SKIPPER_LAYER_READOUT) return fail(c, SKIPPER_EINVAL, "last layer must be the readout");
+    c->L.resize(n);
+    c->Ls = n - 1;
+    for (int i = 0; i < n; ++i) {
+        Layer &l = c->L[i];
+        l.d = layers[i];
+        const skipper_layer &d = layers[i];
+        if (d.cin <= 0 || d.cout <= 0) return fail(c, SKIPPER_EINVAL, "layer %d: cin/cout must be positive", i);
+        if (i < n - 1 && d.kind == SKIPPER_LAYER_READOUT) return fail(c, SKIPPER_EINVAL, "layer %d: readout must be last", i);
+        if (d.kind == SKIPPER_LAYER_CONV3X3) {
+            l.conv = true;
+            l.H = d.h;
+            l.W = d.w;
+            l.Cin = d.cin;
+            l.Cout = d.cout;
+            l.pool = d.pool == 2;
+            if (d.pool != 0 && d.pool != 2) return fail(c, SKIPPER_EINVAL, "layer %d: pool must be 0 or 2", i);
+            if (l.pool && (d.h % 2 || d.w % 2)) return fail(c, SKIPPER_EINVAL, "layer %d: pooled size must be even", i);
+            l.PH = l.pool ? d.h / 2 : d.h;
+            l.PW = l.pool ? d.w / 2 : d.w;
+            l.N = (long long)d.h * d.w * d.cout;
+            l.Nout = (long long)l.PH * l.PW * d.cout;
+            l.Nin = (long long)d.h * d.w * d.cin;
+            l.wcount = (size_t)d.cout * 9 * d.cin;
+        } else if (d.kind == SKIPPER_LAYER_FC || d.kind == SKIPPER_LAYER_READOUT) {
+            l.fc = d.kind == SKIPPER_LAYER_FC;
+            l.readout = d.kind == SKIPPER_LAYER_READOUT;
+            l.Cin = d.cin;
+            l.Cout = d.cout;
+            l.N = l.Nout = d.cout;
+            l.Nin = d.cin;
+            l.wcount = (size_t)d.cout * d.cin;
+        } else {
+            return fail(c, SKIPPER_EINVAL, "layer %d: unknown kind %d", i, d.kind);
+        }
+        if (!l.readout) {
+            if (!(d.theta > 0.f) || !(d.lambda > 0.f) || d.lambda > 1.f)
+                return fail(c, SKIPPER_EINVAL, "layer %d: need theta > 0 and 0 < lambda <= 1 (Eq.1)", i);
+            if (d.cout % 4) return fail(c, SKIPPER_EINVAL, "layer %d: cout must be a multiple of 4", i);
+        }
+    }
+    // chaining
+    const Layer &f = c->L[0];
+    if (f.conv) {
+        c->in_h = f.H;
+        c->in_w = f.W;
+        c->in_c = f.Cin;
+    } else {
+        c->in_h = c->in_w = 1;
+        c->in_c = f.Cin;
+    }
+    c->in_elems = (long long)c->in_h * c->in_w * c->in_c;
+    for (int i = 1; i < n; ++i) {
+        const Layer &p = c->L[i - 1];
+        const Layer &l = c->L[i];
+        if (l.conv) {
+            if (!p.conv || l.H != p.PH || l.W != p.PW || l.Cin != p.Cout)
+                return fail(c, SKIPPER_EINVAL, "layer %d: conv input must be the %dx%dx%d output of layer %d", i, p.PH, p.PW,
+                            p.Cout, i - 1);
+        } else if (l.Cin != p.Nout) {
+            return fail(c, SKIPPER_EINVAL, "layer %d: cin %d != %lld outputs of layer %d", i, l.Cin, p.Nout, i - 1);
+        }
+    }
+    // kernel support per layer
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        if (l.conv && i == 0 && 9 * l.Cin <= 32) {
+            l.direct = true;
+            if (256 % l.Cout) return fail(c, SKIPPER_EUNSUPPORTED, "layer 0: direct conv needs cout | 256");
+            c->input_direct = true;
+            continue;
+        }
+        if (l.conv) {
+            if (l.Cin % 64) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: tensor-core conv needs cin %% 64 == 0", i);
+            if (l.Cout % 64 && i > 0) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: conv dgrad needs cout %% 64 == 0", i);
+            auto boxok = [](int h, int w, int rows) {
+                if (w > rows || rows % w) return false;
+                int by = rows / w;
+                if (by <= h) return h % by == 0;
+                return by % h == 0;
+            };
+            if (!boxok(l.H, l.W, 128) || !boxok(l.H, l.W, 64))
+                return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: %dx%d image does not tile 64/128-row TMA boxes", i, l.H, l.W);
+        } else {
+            if (l.Cin % 8 || l.Cout % 8) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: fc needs cin, cout %% 8 == 0", i);
+        }
+    }
+    if (c->L.back().readout && c->L.back().Cout > 1024) return fail(c, SKIPPER_EUNSUPPORTED, "readout classes <= 1024");
+    return SKIPPER_OK;
+}
+
+static skipper_status zero_dev(skipper_ctx *c, void *p, size_t bytes) {
+    if (p && bytes) CK(cudaMemsetAsync(p, 0, bytes, c->st));
+    return SKIPPER_OK;
+}
+
+static long long max_nout(const skipper_ctx *c) {
+    long long m = 0;
+    for (int i = 0; i < c->Ls; ++i) m = std::max(m, c->L[i].Nout);
+    return m;
+}
+static long long max_n(const skipper_ctx *c) {
+    long long m = 0;
+    for (int i = 0; i < c->Ls; ++i) m = std::max(m, c->L[i].N);
+    return m;
+}
+static long long max_gemm_io(const skipper_ctx *c) {  // fp32 I (fwd) and g (dgrad) per sample-row
+    long long m = 0;
+    for (int i = 0; i < c->Ls; ++i) {
+        if (!c->L[i].direct) m = std::max(m, c->L[i].N);
+        if (i > 0) m = std::max(m, c->L[i].Nin);
+    }
+    return std::max(m, 4LL);
+}
+
+extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_layers, const skipper_config *cfg,
+                                         const skipper_allocator *alloc, void *cuda_stream, skipper_ctx **out) {
+    if (out) *out = nullptr;
+    if (!cfg || !out) return fail(nullptr, SKIPPER_EINVAL, "null config or output pointer");
+    skipper_ctx *c = new skipper_ctx();
+    auto bail = [&](skipper_status s) {
+        g_last_error = c->err.empty() ? g_last_error : c->err;
+        skipper_destroy(c);
+        return s;
+    };
+    c->cfg = *cfg;
+    c->st = static_cast<cudaStream_t>(cuda_stream);
+    if (alloc && alloc->alloc && alloc->free) {
+        c->alloc = *alloc;
+        c->own_alloc = false;
+    }
+    skipper_status s = validate_and_shape(c, layers, n_layers);
+    if (s != SKIPPER_OK) return bail(s);
+    c->T = cfg->T;
+    c->B = cfg->batch;
+    c->Bg = cfg->global_batch > 0 ? cfg->global_batch : cfg->batch;
+    if (c->T <= 0 || c->B <= 0) return bail(fail(c, SKIPPER_EINVAL, "T and batch must be positive"));
+    if (cfg->mode < 0 || cfg->mode > 2) return bail(fail(c, SKIPPER_EINVAL, "unknown mode %d", cfg->mode));
+    if (cfg->surrogate != SKIPPER_SURR_TRIANGLE && cfg->surrogate != SKIPPER_SURR_FAST_SIGMOID)
+        return bail(fail(c, SKIPPER_EINVAL, "unknown surrogate %d", cfg->surrogate));
+    if (cfg->mode == SKIPPER_MODE_FULL) {
+        c->C = 1;
+    } else {
+        c->C = cfg->C;
+        if (c->C <= 0 || c->T % c->C)
+            return bail(fail(c, SKIPPER_EINVAL, "C=%d must divide T=%d (P:1779-1781)", c->C, c->T));
+        const int Ln = n_layers;
+        if (c->T / c->C <= Ln)
+            return bail(fail(c, SKIPPER_EINVAL, "segment length T/C=%d must exceed the %d layers (P:840-853)", c->T / c->C, Ln));
+        if (!(cfg->p >= 0.0 && cfg->p < 100.0))
+            return bail(fail(c, SKIPPER_EINVAL, "p=%g outside [0, 100) (Eq.5)", cfg->p));
+        if (cfg->mode == SKIPPER_MODE_SKIP && cfg->p / 100.0 > 1.0 - (double)c->C * Ln / c->T) {
+            char buf[256];
+            snprintf(buf, sizeof buf, "warning: p=%g exceeds the Eq.7 rule of thumb p_max=%g (P:1082-1091)", cfg->p,
+                     100.0 * (1.0 - (double)c->C * Ln / c->T));
+            c->err = buf;
+        }
+    }
+    c->S = c->T / c->C;
+    c->num_sms = sk::device_num_sms();
+
+    // ---- persistent allocations
+    c->dw_total = 0;
+    for (auto &l : c->L) c->dw_total += l.wcount;
+#define AL(ptr, n)                                  \
+    do {                                            \
+        s = alloc_arr(c, &(ptr), (size_t)(n));      \
+        if (s != SKIPPER_OK) return bail(s);        \
+    } while (0)
+    AL(c->dw_all, c->dw_total);
+    size_t off = 0;
+    for (int i = 0; i < (int)c->L.size(); ++i) {
+        Layer &l = c->L[i];
+        AL(l.w, l.wcount);
+        AL(l.m, l.wcount);
+        AL(l.v, l.wcount);
+        AL(l.wb, l.wcount);
+        l.dw = c->dw_all + off;
+        off += l.wcount;
+        if (!l.readout) {
+            if (i > 0 && !l.direct) AL(l.wt, l.wcount);
+            const size_t bn = (size_t)c->B * l.N;
+            AL(l.U_run, bn);
+            AL(l.o_run, bn);
+            AL(l.carry, bn);
+            if (cfg->mode != SKIPPER_MODE_FULL) {
+                AL(l.ckU, bn * c->C);
+                AL(l.cko, bn * c->C);
+            }
+            if (cfg->debug_record) {
+                for (int k = 0; k < 2; ++k) {
+                    AL(l.dbg[k], bn * c->T);
+                    AL(l.dbgo[k], bn * c->T);
+                }
+            }
+        }
+    }
+    if (c->input_direct)
+        AL(c->xmask, (size_t)c->T * c->B * c->in_h * c->in_w);
+    else
+        AL(c->xb, (size_t)c->T * c->B * c->in_elems);
+    AL(c->s_part, (size_t)c->T * 32);
+    AL(c->s_dev, (size_t)c->T);
+    const Layer &last = c->L[c->Ls - 1];
+    const Layer &ro = c->L.back();
+    AL(c->cnt, (size_t)c->B * last.Nout);
+    AL(c->cnt_kept, (size_t)c->B * last.Nout);
+    AL(c->g_last, (size_t)c->B * last.Nout);
+    AL(c->z, (size_t)c->B * ro.Cout);
+    AL(c->dz, (size_t)c->B * ro.Cout);
+    AL(c->loss_dev, 1);
+    AL(c->kept_dev, (size_t)c->T);
+#undef AL
+    for (auto &l : c->L) {
+        s = zero_dev(c, l.w, l.wcount * 4);
+        if (s == SKIPPER_OK) s = zero_dev(c, l.m, l.wcount * 4);
+        if (s == SKIPPER_OK) s = zero_dev(c, l.v, l.wcount * 4);
+        if (s == SKIPPER_OK) s = zero_dev(c, l.wb, l.wcount * 2);
+        if (s == SKIPPER_OK && l.wt) s = zero_dev(c, l.wt, l.wcount * 2);
+        if (s != SKIPPER_OK) return bail(s);
+    }
+    s = zero_dev(c, c->dw_all, c->dw_total * 4);
+    if (s != SKIPPER_OK) return bail(s);
+    if (cudaStreamSynchronize(c->st) != cudaSuccess) return bail(fail(c, SKIPPER_ECUDA, "stream sync failed at create"));
+    c->s_host.assign(c->T, 0);
+    c->keep.assign(c->T, 1);
+    c->sst.assign(c->C, NAN);
+    *out = c;
+    return SKIPPER_OK;
+}
+
+extern "C" void skipper_destroy(skipper_ctx *c) {
+    if (!c) return;
+    if (c->st) cudaStreamSynchronize(c->st);
+    if (c->arena) dev_free(c, c->arena, c->arena_bytes);
+    for (auto &l : c->L) {
+        dev_free(c, l.w, l.wcount * 4);
+        dev_free(c, l.m, l.wcount * 4);
+        dev_free(c, l.v, l.wcount * 4);
+        dev_free(c, l.wb, l.wcount * 2);
+        dev_free(c, l.wt, l.wcount * 2);
+        if (!l.readout) {
+            const size_t bn = (size_t)c->B * l.N;
+            dev_free(c, l.U_run, bn * 4);
+            dev_free(c, l.o_run, bn);
+            dev_free(c, l.carry, bn * 4);
+            dev_free(c, l.ckU, bn * c->C * 4);
+            dev_free(c, l.cko, bn * c->C);
+            for (int k = 0; k < 2; ++k) {
+                dev_free(c, l.dbg[k], bn * c->T * 4);
+                dev_free(c, l.dbgo[k], bn * c->T);
+            }
+        }
+    }
+    dev_free(c, c->dw_all, c->dw_total * 4);
+    if (!c->L.empty() && c->Ls > 0) {
+        const Layer &last = c->L[c->Ls - 1];
+        const Layer &ro = c->L.back();
+        dev_free(c, c->xmask, (size_t)c->T * c->B * c->in_h * c->in_w * 4);
+        dev_free(c, c->xb, (size_t)c->T * c->B * c->in_elems * 2);
+        dev_free(c, c->s_part, (size_t)c->T * 32 * 4);
+        dev_free(c, c->s_dev, (size_t)c->T * 8);
+        dev_free(c, c->cnt, (size_t)c->B * last.Nout * 4);
+        dev_free(c, c->cnt_kept, (size_t)c->B * last.Nout * 4);
+        dev_free(c, c->g_last, (size_t)c->B * last.Nout * 4);
+        dev_free(c, c->z, (size_t)c->B * ro.Cout * 4);
+        dev_free(c, c->dz, (size_t)c->B * ro.Cout * 4);
+        dev_free(c, c->loss_dev, 4);
+        dev_free(c, c->kept_dev, (size_t)c->T * 4);
+        dev_free(c, c->x_stage, (size_t)c->T * c->B * c->in_elems);
+        dev_free(c, c->y_stage, (size_t)c->B * 4);
+    }
+    if (c->st) cudaStreamSynchronize(c->st);
+    for (auto e : c->ev_pool) cudaEventDestroy(e);
+    c->comm.destroy();
+    delete c;
+}
+
+extern "C" const char *skipper_last_error(const skipper_ctx *c) {
+    if (c) return c->err.c_str();
+    return g_last_error.c_str();
+}
+
+extern "C" const char *skipper_status_string(int s) {
+    switch (s) {
+        case SKIPPER_OK: return "ok";
+        case SKIPPER_EINVAL: return "invalid argument";
+        case SKIPPER_ENOMEM: return "out of device memory";
+        case SKIPPER_ECUDA: return "CUDA error";
+        case SKIPPER_ENCCL: return "NCCL error";
+        case SKIPPER_EORDER: return "call order violation";
+        case SKIPPER_EFAILED: return "context failed earlier";
+        case SKIPPER_EUNSUPPORTED: return "unsupported geometry";
+    }
+    return "unknown";
+}
+
+extern "C" const char *skipper_build_info(void) {
+    return "skipper-b200: sm_100a tcgen05/TMA GEMMs, fused LIF scans; built " __DATE__ " " __TIME__;
+}
+
+// ------------------------------------------------------------------------------------ weights
+static skipper_status check_ctx(skipper_ctx *c) {
+    if (!c) return fail(nullptr, SKIPPER_EINVAL, "null context");
+    if (c->poisoned) return SKIPPER_EFAILED;
+    return SKIPPER_OK;
+}
+
+static skipper_status refresh_shadows(skipper_ctx *c, int i) {
+    Layer &l = c->L[i];
+    CK(sk::launch_cast_bf16(l.w, l.wb, l.wcount, c->st));
+    if (l.wt) {
+        if (l.conv)  // wt[ci][tap][co] = wb[co][tap][ci]
+            CK(sk::launch_transpose_bf16(l.wb, l.wt, l.Cout, 9, l.Cin, c->st));
+        else  // wt[k][n] = wb[n][k]
+            CK(sk::launch_transpose_bf16(l.wb, l.wt, l.Cout, 1, l.Cin, c->st));
+    }
+    return SKIPPER_OK;
+}
+
+extern "C" size_t skipper_weight_count(const skipper_ctx *c, int layer) {
+    if (!c || layer < 0 || layer >= (int)c->L.size()) return 0;
+    return c->L[layer].wcount;
+}
+
+extern "C" skipper_status skipper_set_weights(skipper_ctx *c, int layer, const float *w_dev) {
+    CKS(check_ctx(c));
+    if (layer < 0 || layer >= (int)c->L.size() || !w_dev) return fail(c, SKIPPER_EINVAL, "bad layer or pointer");
+    Layer &l = c->L[layer];
+    CK(cudaMemcpyAsync(l.w, w_dev, l.wcount * 4, cudaMemcpyDeviceToDevice, c->st));
+    return refresh_shadows(c, layer);
+}
+
+extern "C" skipper_status skipper_get_weights(skipper_ctx *c, int layer, float *w_dev) {
+    CKS(check_ctx(c));
+    if (layer < 0 || layer >= (int)c->L.size() || !w_dev) return fail(c, SKIPPER_EINVAL, "bad layer or pointer");
+    CK(cudaMemcpyAsync(w_dev, c->L[layer].w, c->L[layer].wcount * 4, cudaMemcpyDeviceToDevice, c->st));
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_get_grads(skipper_ctx *c, int layer, float *dw_dev) {
+    CKS(check_ctx(c));
+    if (layer < 0 || layer >= (int)c->L.size() || !dw_dev) return fail(c, SKIPPER_EINVAL, "bad layer or pointer");
+    CK(cudaMemcpyAsync(dw_dev, c->L[layer].dw, c->L[layer].wcount * 4, cudaMemcpyDeviceToDevice, c->st));
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ arenas
+// FIRST pass: two ping-pong output buffers of S rows and the fp32 current buffer.
+// RECOMPUTE/RECORD (R rows): per-layer U and output rows, fp32 I/g, bf16 delta, gathered input.
+static skipper_status arena_free(skipper_ctx *c) {
+    if (c->arena) dev_free(c, c->arena, c->arena_bytes);
+    c->arena = nullptr;
+    c->arena_bytes = 0;
+    for (auto &l : c->L) {
+        l.Po = nullptr;
+        l.Useg = nullptr;
+    }
+    c->I_buf = nullptr;
+    c->d_buf = nullptr;
+    c->P2[0] = c->P2[1] = nullptr;
+    c->xg = nullptr;
+    return SKIPPER_OK;
+}
+
+static skipper_status arena_first(skipper_ctx *c) {
+    arena_free(c);
+    const size_t rowsB = (size_t)c->S * c->B;
+    const size_t pbytes = al256(rowsB * max_nout(c) * 2);
+    const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
+    c->arena_bytes = 2 * pbytes + ibytes;
+    c->arena = dev_alloc(c, c->arena_bytes);
+    if (!c->arena) return fail(c, SKIPPER_ENOMEM, "first-pass arena of %zu bytes", c->arena_bytes);
+    char *p = static_cast<char *>(c->arena);
+    c->P2[0] = reinterpret_cast<uint16_t *>(p);
+    c->P2[1] = reinterpret_cast<uint16_t *>(p + pbytes);
+    c->I_buf = reinterpret_cast<float *>(p + 2 * pbytes);
+    return SKIPPER_OK;
+}
+
+static skipper_status arena_rows(skipper_ctx *c, int R) {
+    arena_free(c);
+    const size_t rowsB = (size_t)R * c->B;
+    size_t bytes = 0;
+    for (int i = 0; i < c->Ls; ++i) bytes += al256(rowsB * c->L[i].Nout * 2) + al256(rowsB * c->L[i].N * 4);
+    const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
+    const size_t dbytes = al256(rowsB * max_n(c) * 2);
+    const size_t xbytes = c->input_direct ? 0 : al256(rowsB * c->in_elems * 2);
+    bytes += ibytes + dbytes + xbytes;
+    c->arena_bytes = bytes;
+    c->arena = dev_alloc(c, bytes);
+    if (!c->arena) return fail(c, SKIPPER_ENOMEM, "segment arena of %zu bytes (%d rows)", bytes, R);
+    char *p = static_cast<char *>(c->arena);
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        l.Po = reinterpret_cast<uint16_t *>(p);
+        p += al256(rowsB * l.Nout * 2);
+        l.Useg = reinterpret_cast<float *>(p);
+        p += al256(rowsB * l.N * 4);
+    }
+    c->I_buf = reinterpret_cast<float *>(p);
+    p += ibytes;
+    c->d_buf = reinterpret_cast<uint16_t *>(p);
+    p += dbytes;
+    if (xbytes) c->xg = reinterpret_cast<uint16_t *>(p);
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ GEMM dispatch
+static skipper_status run_gemm(skipper_ctx *c, const sk::GemmLaunch &g, bool ok, const char *what, int layer,
+                               int cls, double bytes, double flops) {
+    if (!ok) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: cannot plan %s GEMM (tensor map)", layer, what);
+    ProfScope ps(c, cls, bytes, flops);
+    CK(sk::gemm_run(g, c->st, c->num_sms));
+    return SKIPPER_OK;
+}
+
+// I rows = input rows x W^T for spiking layer i over `rows` timestep rows.
+static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, float *I, int rows) {
+    Layer &l = c->L[i];
+    if (rows <= 0) return SKIPPER_OK;
+    sk::GemmLaunch g;
+    const int nb = rows * c->B;
+    bool ok;
+    if (l.conv)
+        ok = sk::plan_conv(&g, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
+    else
+        ok = sk::plan_fc(&g, in, l.wb, I, nb, l.Cout, l.Cin);
+    const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
+    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4;
+    return run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, bytes, 2.0 * M * l.Cout * K);
+}
+
+// ------------------------------------------------------------------------------------ step pieces
+static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
+    if (c->prof_on) prof_resolve(c);
+    CKS(zero_dev(c, c->s_part, (size_t)c->T * 32 * 4));
+    CKS(zero_dev(c, c->cnt, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
+    CKS(zero_dev(c, c->cnt_kept, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
+    CKS(zero_dev(c, c->loss_dev, 4));
+    CKS(zero_dev(c, c->dw_all, c->dw_total * 4));
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        const size_t bn = (size_t)c->B * l.N;
+        CKS(zero_dev(c, l.U_run, bn * 4));
+        CKS(zero_dev(c, l.o_run, bn));
+        CKS(zero_dev(c, l.carry, bn * 4));
+        if (c->cfg.debug_record)
+            for (int k = 0; k < 2; ++k) {
+                CKS(zero_dev(c, l.dbg[k], bn * c->T * 4));
+                CKS(zero_dev(c, l.dbgo[k], bn * c->T));
+            }
+    }
+    {
+        const double xbytes = (double)c->T * c->B * c->in_elems;
+        if (c->input_direct) {
+            ProfScope ps(c, K_STAGE, xbytes + (double)c->T * c->B * c->in_h * c->in_w * 4, 0);
+            CK(sk::launch_stage_bits(x, c->xmask, c->s_part, c->T, c->B, c->in_h, c->in_w, c->in_c, c->st));
+        } else {
+            ProfScope ps(c, K_STAGE, xbytes * 3, 0);
+            CK(sk::launch_stage_bf16(x, c->xb, c->s_part, c->T, c->B, (int)c->in_elems, c->st));
+        }
+    }
+    c->x_cur = x;
+    c->grads_ready = false;
+    return SKIPPER_OK;
+}
+
+// Algorithmic HBM bytes of one scan launch: every operand read or written once.
+static double scan_fwd_bytes(const skipper_ctx *c, const Layer &l, const sk::ScanFwdArgs &a) {
+    const double rows = a.R, comp = a.R - (a.restore ? 1 : 0), bn = (double)c->B * l.N, bno = (double)c->B * l.Nout;
+    double b = rows * bno * 2;                                        // layer output (bf16)
+    b += a.I ? comp * bn * 4 : comp * (double)c->B * l.H * l.W * 4;  // currents, or input bit masks
+    if (a.U_out) b += rows * bn * 4;                                  // stored membranes
+    b += bn * 5 * (a.restore ? 1 : 2);                                // state / checkpoint in (and out)
+    if (a.ckU) b += bn * 5;
+    return b;
+}
+static double scan_bwd_bytes(const skipper_ctx *c, const Layer &l, const sk::ScanBwdArgs &a) {
+    const double rows = a.R, bn = (double)c->B * l.N, bno = (double)c->B * l.Nout;
+    double b = rows * bn * 4;                                         // U
+    b += a.g_broadcast ? bno * 4 : rows * bno * 4;                    // g (pooled resolution when pooled)
+    if (a.delta) b += rows * bn * 2;                                  // delta (bf16)
+    if (a.xmask) b += rows * (double)c->B * l.H * l.W * 4 + (double)l.wcount * 4;
+    b += bn * 8;                                                      // carry in/out
+    return b;
+}
+
+// Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
+static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        const uint16_t *in;
+        uint16_t *out;
+        if (record) {
+            in = i == 0 ? (c->xb ? c->xb : nullptr) : c->L[i - 1].Po;
+            out = l.Po;
+        } else {
+            in = i == 0 ? (c->xb ? c->xb + (size_t)t0 * c->B * c->in_elems : nullptr) : c->P2[(i - 1) & 1];
+            out = c->P2[i & 1];
+        }
+        if (!l.direct) CKS(gemm_forward(c, i, in, c->I_buf, R));
+        sk::ScanFwdArgs a{};
+        a.I = l.direct ? nullptr : c->I_buf;
+        a.R = R;
+        a.restore = 0;
+        a.U_state = l.U_run;
+        a.o_state = l.o_run;
+        a.U_out = record ? l.Useg : nullptr;
+        a.Po_out = out;
+        a.ckU = record ? nullptr : l.ckU + (size_t)seg * c->B * l.N;
+        a.cko = record ? nullptr : l.cko + (size_t)seg * c->B * l.N;
+        a.s_part = c->s_part;
+        a.row_t = nullptr;
+        a.t0 = t0;
+        a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
+        a.dbg_U = c->cfg.debug_record ? l.dbg[0] : nullptr;
+        a.dbg_o = c->cfg.debug_record ? l.dbgo[0] : nullptr;
+        a.B = c->B;
+        a.H = l.H;
+        a.W = l.W;
+        a.C = l.Cout;
+        a.pool = l.pool ? 1 : 0;
+        a.lam = l.d.lambda;
+        a.theta = l.d.theta;
+        if (l.direct) {
+            a.xmask = c->xmask;
+            a.w_direct = l.wb;
+            a.kbits = 9 * l.Cin;
+        }
+        {
+            ProfScope ps(c, l.direct ? K_DIRECT_FWD : K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
+            CK(sk::launch_lif_fwd(a, c->st));
+        }
+    }
+    return SKIPPER_OK;
+}
+
+static skipper_status comm_allreduce_s(skipper_ctx *c) {
+    if (c->comm.world > 1) {
+        std::string e;
+        if (!c->comm.allreduce_i64(c->s_dev, c->T, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    }
+    return SKIPPER_OK;
+}
+
+// After the last FIRST segment: loss, SAM totals, SST and keep lists (Eq.4, Eq.5).
+static skipper_status finish_first(skipper_ctx *c, const int *labels) {
+    const Layer &last = c->L[c->Ls - 1];
+    const Layer &ro = c->L.back();
+    ProfScope ps0(c, K_READOUT, (double)c->T * 32 * 4, 0);
+    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, c->T, c->st));
+    ProfScope ps1(c, K_READOUT, (double)c->B * last.Nout * 8 + (double)ro.wcount * 2, 4.0 * c->B * last.Nout * ro.Cout);
+    CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
+                               ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+    CKS(comm_allreduce_s(c));
+    CK(cudaMemcpyAsync(c->s_host.data(), c->s_dev, (size_t)c->T * 8, cudaMemcpyDeviceToHost, c->st));
+    CK(cudaStreamSynchronize(c->st));  // the one host sync of the step
+    const int C = c->C, S = c->S;
+    c->kept.assign(C, {});
+    c->keep.assign(c->T, 1);
+    c->sst.assign(C, NAN);
+    const bool skip = c->cfg.mode == SKIPPER_MODE_SKIP && c->cfg.p != 0.0;
+    for (int seg = 0; seg < C; ++seg) {
+        if (skip) c->sst[seg] = skipper_sst_host(c->s_host.data() + (size_t)seg * S, S, c->cfg.p);
+        for (int t = seg * S; t < (seg + 1) * S; ++t) {
+            bool k = true;
+            if (skip && t != seg * S) k = (double)c->s_host[t] > c->sst[seg];
+            c->keep[t] = k ? 1 : 0;
+            if (k) c->kept[seg].push_back(t);
+        }
+    }
+    c->kept_flat.assign((size_t)C * S, 0);
+    c->Kmax = 0;
+    for (int seg = 0; seg < C; ++seg) {
+        std::copy(c->kept[seg].begin(), c->kept[seg].end(), c->kept_flat.begin() + (size_t)seg * S);
+        c->Kmax = std::max<int>(c->Kmax, (int)c->kept[seg].size());
+    }
+    CK(cudaMemcpyAsync(c->kept_dev, c->kept_flat.data(), (size_t)C * S * 4, cudaMemcpyHostToDevice, c->st));
+    return SKIPPER_OK;
+}
+
+static skipper_status recompute_segment(skipper_ctx *c, int seg) {
+    const int R = (int)c->kept[seg].size();
+    const int *row_t = c->kept_dev + (size_t)seg * c->S;
+    if (!c->input_direct) {
+        ProfScope ps(c, K_GATHER, 4.0 * R * c->B * c->in_elems, 0);
+        CK(sk::launch_gather_rows(c->xb, c->xg, row_t, R, (size_t)c->B * c->in_elems, c->st));
+    }
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        const uint16_t *in = i == 0 ? c->xg : c->L[i - 1].Po;
+        const size_t in_row = (size_t)c->B * (i == 0 ? c->in_elems : c->L[i - 1].Nout);
+        if (!l.direct && R > 1)  // rows 1..R-1 (row 0 is the checkpoint)
+            CKS(gemm_forward(c, i, in + in_row, c->I_buf + (size_t)c->B * l.N, R - 1));
+        sk::ScanFwdArgs a{};
+        a.I = l.direct ? nullptr : c->I_buf;
+        a.R = R;
+        a.restore = 1;
+        a.U_state = l.ckU + (size_t)seg * c->B * l.N;
+        a.o_state = l.cko + (size_t)seg * c->B * l.N;
+        a.U_out = l.Useg;
+        a.Po_out = l.Po;
+        a.s_part = nullptr;
+        a.row_t = row_t;
+        a.cnt = (i == c->Ls - 1) ? c->cnt_kept : nullptr;
+        a.dbg_U = c->cfg.debug_record ? l.dbg[1] : nullptr;
+        a.dbg_o = c->cfg.debug_record ? l.dbgo[1] : nullptr;
+        a.B = c->B;
+        a.H = l.H;
+        a.W = l.W;
+        a.C = l.Cout;
+        a.pool = l.pool ? 1 : 0;
+        a.lam = l.d.lambda;
+        a.theta = l.d.theta;
+        if (l.direct) {
+            a.xmask = c->xmask;
+            a.w_direct = l.wb;
+            a.kbits = 9 * l.Cin;
+        }
+        {
+            ProfScope ps(c, l.direct ? K_DIRECT_FWD : K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
+            CK(sk::launch_lif_fwd(a, c->st));
+        }
+    }
+    return SKIPPER_OK;
+}
+
+// Eq.2 backward over the R stored rows of a segment (layer-major, reverse t inside the scan).
+static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
+    for (int i = c->Ls - 1; i >= 0; --i) {
+        Layer &l = c->L[i];
+        sk::ScanBwdArgs a{};
+        a.g = (i == c->Ls - 1) ? c->g_last : c->I_buf;
+        a.g_broadcast = (i == c->Ls - 1) ? 1 : 0;
+        a.g_pooled = l.pool ? 1 : 0;
+        a.U = l.Useg;
+        a.carry = l.carry;
+        a.delta = l.direct ? nullptr : c->d_buf;
+        a.R = R;
+        a.B = c->B;
+        a.H = l.H;
+        a.W = l.W;
+        a.C = l.Cout;
+        a.pool = l.pool ? 1 : 0;
+        a.lam = l.d.lambda;
+        a.theta = l.d.theta;
+        a.surr = c->cfg.surrogate;
+        a.gamma = c->cfg.surr_gamma;
+        if (l.direct) {
+            a.xmask = c->xmask;
+            a.row_t = row_t;
+            a.dW_direct = l.dw;
+            a.kbits = 9 * l.Cin;
+        }
+        {
+            ProfScope ps(c, l.direct ? K_DIRECT_BWD : K_SCAN_BWD, scan_bwd_bytes(c, l, a), 0);
+            CK(sk::launch_lif_bwd(a, c->st));
+        }
+        if (l.direct) continue;
+        const int nb = R * c->B;
+        const uint16_t *X = i == 0 ? (c->xg ? c->xg : c->xb) : c->L[i - 1].Po;
+        sk::GemmLaunch g;
+        bool ok;
+        if (l.conv)
+            ok = sk::plan_conv_wgrad(&g, c->d_buf, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
+        else
+            ok = sk::plan_fc_wgrad(&g, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
+        {
+            const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
+            const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
+            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K));
+        }
+        if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
+            if (l.conv)
+                ok = sk::plan_conv(&g, c->d_buf, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
+            else
+                ok = sk::plan_fc(&g, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout);
+            const double M = (double)nb * l.H * l.W, K = (double)l.Cout * (l.conv ? 9 : 1);
+            const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4;
+            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * (l.Nin / (l.H * l.W)) * K));
+        }
+    }
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ public schedule
+extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int pass, const unsigned char *x_dev,
+                                                  const int *labels_dev) {
+    CKS(check_ctx(c));
+    if (!x_dev) return fail(c, SKIPPER_EINVAL, "null input");
+    const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
+    if (pass == SKIPPER_PASS_RECORD) {
+        if (!full || seg != 0) return fail(c, SKIPPER_EORDER, "RECORD is the single pass of FULL mode (seg 0)");
+        if (!labels_dev) return fail(c, SKIPPER_EINVAL, "RECORD needs labels");
+        CKS(begin_step(c, x_dev));
+        CKS(arena_rows(c, c->T));
+        CKS(forward_rows_first(c, 0, c->T, 0, true));
+        CKS(finish_first(c, labels_dev));
+        c->phase = PH_RECOMPUTED;
+        c->next_seg = 0;
+        return SKIPPER_OK;
+    }
+    if (full) return fail(c, SKIPPER_EORDER, "FULL mode uses the RECORD pass");
+    if (pass == SKIPPER_PASS_FIRST) {
+        if (seg == 0) {
+            if (c->phase != PH_IDLE && c->phase != PH_BWD_DONE && c->phase != PH_FIRST)
+                return fail(c, SKIPPER_EORDER, "FIRST(0) while an iteration is in flight");
+            CKS(begin_step(c, x_dev));
+            CKS(arena_first(c));
+            c->phase = PH_FIRST;
+            c->next_seg = 0;
+        }
+        if (c->phase != PH_FIRST || seg != c->next_seg)
+            return fail(c, SKIPPER_EORDER, "FIRST segments must run 0..C-1 in order (expected %d)", c->next_seg);
+        if (x_dev != c->x_cur) return fail(c, SKIPPER_EINVAL, "x_dev changed within an iteration");
+        CKS(forward_rows_first(c, seg, c->S, seg * c->S, false));
+        c->next_seg = seg + 1;
+        if (seg == c->C - 1) {
+            if (!labels_dev) return fail(c, SKIPPER_EINVAL, "the last FIRST segment needs labels");
+            CKS(finish_first(c, labels_dev));
+            CKS(arena_rows(c, c->Kmax));
+            c->phase = PH_READY_BWD;
+            c->next_seg = c->C - 1;
+        }
+        return SKIPPER_OK;
+    }
+    if (pass == SKIPPER_PASS_RECOMPUTE) {
+        if (c->phase != PH_READY_BWD || seg != c->next_seg)
+            return fail(c, SKIPPER_EORDER, "RECOMPUTE must follow FIRST / the previous BACKWARD (expected seg %d)",
+                        c->next_seg);
+        if (x_dev != c->x_cur) return fail(c, SKIPPER_EINVAL, "x_dev changed within an iteration");
+        CKS(recompute_segment(c, seg));
+        c->phase = PH_RECOMPUTED;
+        return SKIPPER_OK;
+    }
+    return fail(c, SKIPPER_EINVAL, "unknown pass %d", pass);
+}
+
+extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
+    CKS(check_ctx(c));
+    if (c->phase != PH_RECOMPUTED || seg != c->next_seg)
+        return fail(c, SKIPPER_EORDER, "BACKWARD(%d) must follow RECOMPUTE(%d)", seg, c->next_seg);
+    const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
+    const int R = full ? c->T : (int)c->kept[seg].size();
+    const int *row_t = full ? nullptr : c->kept_dev + (size_t)seg * c->S;
+    if (full) c->xg = nullptr;  // layer-0 fc wgrad reads the staged input directly
+    CKS(backward_rows(c, R, row_t));
+    if (seg == 0) {
+        const Layer &last = c->L[c->Ls - 1];
+        const Layer &ro = c->L.back();
+        ProfScope ps(c, K_READOUT, (double)c->B * (last.Nout + ro.Cout) * 4 + (double)ro.wcount * 4,
+                     2.0 * c->B * last.Nout * ro.Cout);
+        CK(sk::launch_readout_wgrad(c->dz, full ? c->cnt : c->cnt_kept, ro.dw, c->B, (int)last.Nout, ro.Cout,
+                                    1.0f / c->T, c->st));
+        if (c->cfg.debug_record && full)
+            for (int i = 0; i < c->Ls; ++i) {
+                const size_t bn = (size_t)c->B * c->L[i].N * c->T;
+                CK(cudaMemcpyAsync(c->L[i].dbg[1], c->L[i].dbg[0], bn * 4, cudaMemcpyDeviceToDevice, c->st));
+                CK(cudaMemcpyAsync(c->L[i].dbgo[1], c->L[i].dbgo[0], bn, cudaMemcpyDeviceToDevice, c->st));
+            }
+        c->phase = PH_BWD_DONE;
+        c->grads_ready = true;
+        CKS(arena_free(c));
+    } else {
+        c->phase = PH_READY_BWD;
+        c->next_seg = seg - 1;
+    }
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_optimizer_step(skipper_ctx *c) {
+    CKS(check_ctx(c));
+    if (c->phase != PH_BWD_DONE || !c->grads_ready)
+        return fail(c, SKIPPER_EORDER, "optimizer_step needs a completed backward");
+    if (c->comm.world > 1) {
+        std::string e;
+        if (!c->comm.allreduce_f32(c->dw_all, c->dw_total, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    }
+    c->adam_step += 1;
+    const double b1 = c->cfg.beta1, b2 = c->cfg.beta2;
+    const float bc1 = (float)(1.0 - std::pow(b1, (double)c->adam_step));
+    const float bc2s = (float)std::sqrt(1.0 - std::pow(b2, (double)c->adam_step));
+    for (int i = 0; i < (int)c->L.size(); ++i) {
+        Layer &l = c->L[i];
+        {
+            ProfScope ps(c, K_ADAM, (double)l.wcount * 26, 0);
+            CK(sk::launch_adam(l.w, l.dw, l.m, l.v, l.wb, l.wcount, c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps,
+                               bc1, bc2s, c->st));
+        }
+        if (l.wt) {
+            ProfScope ps(c, K_ADAM, (double)l.wcount * 4, 0);
+            if (l.conv)
+                CK(sk::launch_transpose_bf16(l.wb, l.wt, l.Cout, 9, l.Cin, c->st));
+            else
+                CK(sk::launch_transpose_bf16(l.wb, l.wt, l.Cout, 1, l.Cin, c->st));
+        }
+    }
+    c->grads_ready = false;
+    c->phase = PH_IDLE;
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_step(skipper_ctx *c, const unsigned char *x_dev, const int *labels_dev,
+                                       float *loss_host) {
+    CKS(check_ctx(c));
+    if (!x_dev || !labels_dev) return fail(c, SKIPPER_EINVAL, "null input or labels");
+    if (c->cfg.mode == SKIPPER_MODE_FULL) {
+        CKS(skipper_forward_segment(c, 0, SKIPPER_PASS_RECORD, x_dev, labels_dev));
+        CKS(skipper_backward_segment(c, 0));
+    } else {
+        c->phase = PH_IDLE;
+        for (int seg = 0; seg < c->C; ++seg)
+            CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_FIRST, x_dev, seg == c->C - 1 ? labels_dev : nullptr));
+        for (int seg = c->C - 1; seg >= 0; --seg) {
+            CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_RECOMPUTE, x_dev, nullptr));
+            CKS(skipper_backward_segment(c, seg));
+        }
+    }
+    CKS(skipper_optimizer_step(c));
+    if (loss_host) {
+        CK(cudaMemcpyAsync(loss_host, c->loss_dev, 4, cudaMemcpyDeviceToHost, c->st));
+        CK(cudaStreamSynchronize(c->st));
+    }
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_step_host(skipper_ctx *c, const unsigned char *x_host, const int *labels_host,
+                                            float *loss_host) {
+    CKS(check_ctx(c));
+    if (!x_host || !labels_host) return fail(c, SKIPPER_EINVAL, "null host input");
+    const size_t xbytes = (size_t)c->T * c->B * c->in_elems;
+    if (!c->x_stage) {
+        CKS(alloc_arr(c, &c->x_stage, xbytes));
+        CKS(alloc_arr(c, &c->y_stage, (size_t)c->B));
+    }
+    CK(cudaMemcpyAsync(c->x_stage, x_host, xbytes, cudaMemcpyHostToDevice, c->st));
+    CK(cudaMemcpyAsync(c->y_stage, labels_host, (size_t)c->B * 4, cudaMemcpyHostToDevice, c->st));
+    float loss = 0.f;
+    CKS(skipper_step(c, c->x_stage, c->y_stage, &loss));
+    if (loss_host) *loss_host = loss;
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ introspection
+extern "C" skipper_status skipper_get_loss(skipper_ctx *c, float *loss_host) {
+    CKS(check_ctx(c));
+    CK(cudaMemcpyAsync(loss_host, c->loss_dev, 4, cudaMemcpyDeviceToHost, c->st));
+    CK(cudaStreamSynchronize(c->st));
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_get_spike_sums(skipper_ctx *c, long long *s_host) {
+    CKS(check_ctx(c));
+    CK(cudaStreamSynchronize(c->st));
+    std::copy(c->s_host.begin(), c->s_host.end(), s_host);
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_get_keep_mask(skipper_ctx *c, unsigned char *keep_host) {
+    CKS(check_ctx(c));
+    std::copy(c->keep.begin(), c->keep.end(), keep_host);
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_get_sst(skipper_ctx *c, double *sst_host) {
+    CKS(check_ctx(c));
+    std::copy(c->sst.begin(), c->sst.end(), sst_host);
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_mem_stats(skipper_ctx *c, size_t *cur, size_t *peak) {
+    CKS(check_ctx(c));
+    if (cur) *cur = c->cur_bytes;
+    if (peak) *peak = c->peak_bytes;
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_reset_peak(skipper_ctx *c) {
+    CKS(check_ctx(c));
+    c->peak_bytes = c->cur_bytes;
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_debug_copy(skipper_ctx *c, int which, int layer, void *dst, size_t bytes) {
+    CKS(check_ctx(c));
+    if (!c->cfg.debug_record) return fail(c, SKIPPER_EINVAL, "debug_record is off");
+    if (layer < 0 || layer >= c->Ls || which < 0 || which > 3 || !dst)
+        return fail(c, SKIPPER_EINVAL, "bad debug request");
+    const Layer &l = c->L[layer];
+    const size_t n = (size_t)c->T * c->B * l.N;
+    const bool isU = which == 0 || which == 2;
+    const size_t need = n * (isU ? 4 : 1);
+    if (bytes < need) return fail(c, SKIPPER_EINVAL, "debug buffer too small (%zu < %zu)", bytes, need);
+    const void *src = isU ? (const void *)l.dbg[which / 2] : (const void *)l.dbgo[which / 2];
+    CK(cudaMemcpyAsync(dst, src, need, cudaMemcpyDeviceToDevice, c->st));
+    return SKIPPER_OK;
+}
+
+extern "C" size_t skipper_workspace_bytes(const skipper_layer *layers, int n, const skipper_config *cfg, int kept_max) {
+    if (!layers || !cfg || n < 2) return 0;
+    long long Nsum = 0, Nout_sum = 0;
+    for (int i = 0; i < n - 1; ++i) {
+        const skipper_layer &d = layers[i];
+        long long N, No;
+        if (d.kind == SKIPPER_LAYER_CONV3X3) {
+            N = (long long)d.h * d.w * d.cout;
+            No = d.pool == 2 ? N / 4 : N;
+        } else {
+            N = No = d.cout;
+        }
+        Nsum += N;
+        Nout_sum += No;
+    }
+    const long long B = cfg->batch;
+    const long long per_step = B * (Nsum * 4 + Nout_sum * 2);  // stored U fp32 + layer output bf16
+    const long long per_ckpt = B * Nsum * 5;                   // checkpoint U fp32 + o u8
+    if (cfg->mode == SKIPPER_MODE_FULL) return (size_t)(cfg->T * per_step);
+    const int C = cfg->C > 0 ? cfg->C : 1;
+    const int rows = kept_max >= 0 ? kept_max : cfg->T / C;
+    return (size_t)(C * per_ckpt + (long long)rows * per_step);
+}
+
+extern "C" skipper_status skipper_comm_unique_id(unsigned char id_out[128]) {
+    std::string e;
+    if (!sk::Comm::unique_id(id_out, &e)) return fail(nullptr, SKIPPER_ENCCL, "%s", e.c_str());
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_comm_init(skipper_ctx *c, const unsigned char id[128], int rank, int world) {
+    CKS(check_ctx(c));
+    if (world < 1 || rank < 0 || rank >= world) return fail(c, SKIPPER_EINVAL, "bad rank/world");
+    if (world == 1) return SKIPPER_OK;
+    std::string e;
+    if (!c->comm.init(id, rank, world, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ kernel-level API
+// (include/skipper_kernels.h) - the same launchers skipper_step uses, for per-kernel parity tests.
+static int kapi_run(const sk::GemmLaunch &g, bool ok, void *stream, const char *what) {
+    if (!ok) {
+        g_last_error = std::string(what) + ": unsupported shape or tensor-map failure";
+        return SKIPPER_EUNSUPPORTED;
+    }
+    cudaError_t e = sk::gemm_run(g, static_cast<cudaStream_t>(stream), sk::device_num_sms());
+    if (e != cudaSuccess) {
+        g_last_error = std::string(what) + ": " + cudaGetErrorString(e);
+        return SKIPPER_ECUDA;
+    }
+    return SKIPPER_OK;
+}
+
+extern "C" int skipper_k_fc_fwd(const unsigned short *A, const unsigned short *B, float *C, int M, int N, int K,
+                                void *stream) {
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_fc(&g, A, B, C, M, N, K);
+    return kapi_run(g, ok, stream, "fc_fwd");
+}
+
+extern "C" int skipper_k_fc_wgrad(const unsigned short *D, const unsigned short *X, float *dW, int M, int N, int K,
+                                  int accumulate, void *stream) {
+    if (!accumulate && cudaMemsetAsync(dW, 0, (size_t)N * K * 4, static_cast<cudaStream_t>(stream)) != cudaSuccess)
+        return SKIPPER_ECUDA;
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_fc_wgrad(&g, D, X, dW, M, N, K, sk::device_num_sms());
+    return kapi_run(g, ok, stream, "fc_wgrad");
+}
+
+extern "C" int skipper_k_conv_fwd(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w,
+                                  int cin, int cout, void *stream) {
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_conv(&g, X, Wk, Y, nb, h, w, cin, cout, +1);
+    return kapi_run(g, ok, stream, "conv_fwd");
+}
+
+extern "C" int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, float *G, int nb, int h, int w,
+                                    int cin, int cout, void *stream) {
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_conv(&g, D, Wt, G, nb, h, w, cout, cin, -1);
+    return kapi_run(g, ok, stream, "conv_dgrad");
+}
+
+extern "C" int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float *dW, int nb, int h, int w,
+                                    int cin, int cout, int accumulate, void *stream) {
+    if (!accumulate && cudaMemsetAsync(dW, 0, (size_t)cout * 9 * cin * 4, static_cast<cudaStream_t>(stream)) != cudaSuccess)
+        return SKIPPER_ECUDA;
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_conv_wgrad(&g, D, X, dW, nb, h, w, cin, cout, sk::device_num_sms());
+    return kapi_run(g, ok, stream, "conv_wgrad");
+}
+
+extern "C" int skipper_k_num_sms(void) { return sk::device_num_sms(); }
+
+// ------------------------------------------------------------------------------------ profiling API
+extern "C" skipper_status skipper_profile(skipper_ctx *c, int enable) {
+    CKS(check_ctx(c));
+    prof_resolve(c);
+    c->prof_on = enable != 0;
+    for (int k = 0; k < 16; ++k) {
+        c->prof_n[k] = 0;
+        c->prof_ms[k] = c->prof_bytes[k] = c->prof_flops[k] = 0;
+    }
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_profile_read(skipper_ctx *c, int cls, long long *launches, double *ms, double *bytes,
+                                               double *flops) {
+    CKS(check_ctx(c));
+    if (cls < 0 || cls >= K_NCLASS) return fail(c, SKIPPER_EINVAL, "kernel class %d out of range", cls);
+    prof_resolve(c);
+    if (launches) *launches = c->prof_n[cls];
+    if (ms) *ms = c->prof_ms[cls];
+    if (bytes) *bytes = c->prof_bytes[cls];
+    if (flops) *flops = c->prof_flops[cls];
+    return SKIPPER_OK;
+}
+
+extern "C" const char *skipper_profile_class_name(int cls) {
+    if (cls < 0 || cls >= K_NCLASS) return nullptr;
+    return k_class_names[cls];
+}
+
+extern "C" int skipper_profile_num_classes(void) { return K_NCLASS; }
+
+extern "C" long long skipper_launch_count(const skipper_ctx *c) { return c ? c->launches : 0; }

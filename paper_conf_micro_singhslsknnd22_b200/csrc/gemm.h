@@ -1,0 +1,67 @@
+// gemm.h - host-side description of one synaptic contraction on the tcgen05 tensor cores.
+//
+// The synaptic GEMMs of Eq.1 (I = W o) and Eq.2 (W^T delta and
+// sum_t delta o^T), layer-major over all (kept) timesteps of a segment:
+// the M dimension is (t, b, h, w), so T*L tiny per-step products become L GEMMs.
+#pragma once
+#include <cstdint>
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+namespace sk {
+
+enum OperandKind {
+    OP_K2D = 0,     // K-major 2D matrix [rows][K], TMA box {64, rows}
+    OP_KCONV = 1,   // K-major implicit im2col of an NHWC image, one 3x3 tap per K block
+    OP_MN2D = 2,    // MN-major 2D matrix [K rows][MN], TMA boxes {64, 64}
+    OP_MNCONV = 3,  // MN-major shifted NHWC image (wgrad input operand), boxes {64, W, bh, bn}
+};
+
+enum StoreMode { STORE_OVERWRITE = 0, STORE_ATOMIC_ADD = 1 };
+
+// Passed by value to the kernel.
+struct GemmDev {
+    int m_tiles, n_tiles, taps, splits;
+    int num_kb, kb_per_split;
+    int a_kind, b_kind;
+    int conv_cb;        // channel blocks of 64 per tap (A = OP_KCONV)
+    int conv_hw, conv_w;  // image H*W and W (row -> (image, y) decode)
+    int conv_sign;      // +1 forward / wgrad, -1 dgrad (flipped taps)
+    int cols_per_tap;   // wgrad conv: output column offset per tap (= Cin)
+    float *C;
+    long long ldc;
+    int M, N;           // valid output extent (rows, columns of one tap block)
+    int store_mode;
+};
+
+struct GemmLaunch {
+    GemmDev d;
+    CUtensorMap ta, tb;
+    int bn;             // 64, 128 or 256
+    int mn_major;       // 0: both operands K-major; 1: both MN-major (wgrad)
+};
+
+// Tensor-map builders (bf16, 128-byte swizzle, OOB -> zero).
+bool make_map_2d(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                 uint32_t box_outer);
+bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint64_t H, uint64_t NB,
+                   uint32_t box_w, uint32_t box_h, uint32_t box_n);
+
+// Plans (return false on unsupported geometry).  All pointers are device pointers.
+// C[M][N] = A[M][K] . B[N][K]^T
+bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K);
+// dW[N][K] (+)= D[M][N]^T . X[M][K]   (reduction over the M rows)
+bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms);
+// conv forward / dgrad: Y[nb,h,w,cout] from X[nb,h,w,cin] and Wk[cout][9][cin];
+// dgrad: G[nb,h,w,cin] from D[nb,h,w,cout] and Wt[cin][9][cout]
+bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
+               int sign);
+// conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
+bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
+                     int num_sms);
+
+cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms);
+
+int device_num_sms();
+
+}  // namespace sk

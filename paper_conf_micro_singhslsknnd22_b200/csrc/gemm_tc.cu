@@ -1,0 +1,448 @@
+// gemm_tc.cu - K2: synaptic contractions on the 5th-generation tensor cores (sm_100a).
+//
+// One persistent, warp-specialised kernel family:
+//   warp 0      TMA producer  (cp.async.bulk.tensor -> 128B-swizzled smem ring, mbarrier complete_tx)
+//   warp 1      MMA issuer    (one thread: tcgen05.mma.cta_group::1.kind::f16, M=128, N=BN, K=16,
+//                              accumulators in TMEM, tcgen05.commit frees smem stages)
+//               + TMEM allocator (2 accumulator buffers so the epilogue of tile i overlaps tile i+1)
+//   warps 2-5   epilogue      (tcgen05.ld 32x32b -> registers -> fp32 store or red.add into global)
+// Operands are bf16 (exact for spikes and grid weights), accumulation fp32.
+// Convolutions are implicit GEMMs: each K block is one 3x3 tap x 64 channels, loaded by a 4D TMA
+// box shifted by the tap offset; the zero padding is TMA's out-of-bounds fill.
+#include "common.cuh"
+#include "gemm.h"
+
+#include <cstdio>
+#include <mutex>
+
+namespace sk {
+
+static constexpr int BM = 128;
+static constexpr int BK = 64;        // bf16 elements per K block = one 128-byte swizzle row
+static constexpr int NUM_THREADS = 192;
+
+template <int BN>
+struct GemmCfg {
+    static constexpr uint32_t A_BYTES = BM * BK * 2;
+    static constexpr uint32_t B_BYTES = BN * BK * 2;
+    static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int STAGES = (BN == 64) ? 8 : (BN == 128 ? 6 : 4);
+    static constexpr uint32_t TMEM_COLS = (2 * BN <= 128) ? 128 : (2 * BN <= 256 ? 256 : 512);
+    static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+struct TileCoord {
+    int m_t, n_t, tap, split, kb0, kb1;
+};
+
+SK_DEV TileCoord decode_tile(const GemmDev &g, int tile) {
+    TileCoord c;
+    c.m_t = tile % g.m_tiles;
+    int r = tile / g.m_tiles;
+    c.n_t = r % g.n_tiles;
+    r /= g.n_tiles;
+    c.tap = r % g.taps;
+    c.split = r / g.taps;
+    c.kb0 = c.split * g.kb_per_split;
+    c.kb1 = min(g.num_kb, c.kb0 + g.kb_per_split);
+    return c;
+}
+
+template <int BN, int MN>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const GemmDev g) {
+    using Cfg = GemmCfg<BN>;
+    constexpr int STAGES = Cfg::STAGES;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023u) & ~1023u;
+    const uint32_t bars = base + STAGES * Cfg::STAGE_BYTES;
+    auto full_bar = [&](int s) { return bars + 8u * s; };
+    auto empty_bar = [&](int s) { return bars + 8u * (STAGES + s); };
+    auto tfull_bar = [&](int a) { return bars + 8u * (2 * STAGES + a); };
+    auto tempty_bar = [&](int a) { return bars + 8u * (2 * STAGES + 2 + a); };
+    const uint32_t tmem_slot = bars + 8u * (2 * STAGES + 4);
+    uint32_t *tmem_slot_ptr = reinterpret_cast<uint32_t *>(smem_raw + (tmem_slot - raw));
+
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+
+    if (warp == 0 && lane == 0) {
+        tma_prefetch(&ta);
+        tma_prefetch(&tb);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(full_bar(s), 1);
+            mbar_init(empty_bar(s), 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(tfull_bar(a), 1);
+            mbar_init(tempty_bar(a), 4);
+        }
+        fence_mbar_init();
+    }
+    if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(tmem_slot_ptr);
+
+    const int total = g.m_tiles * g.n_tiles * g.taps * g.splits;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ TMA producer
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
+                const TileCoord tc = decode_tile(g, tile);
+                const int tdy = tc.tap / 3 - 1, tdx = tc.tap % 3 - 1;
+                for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
+                    mbar_wait(empty_bar(stage), phase ^ 1u);
+                    const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
+                    const uint32_t sb = sa + Cfg::A_BYTES;
+                    const uint32_t fb = full_bar(stage);
+                    mbar_expect_tx(fb, Cfg::STAGE_BYTES);
+                    // ---- A
+                    if (g.a_kind == OP_K2D) {
+                        tma_load_2d(sa, &ta, fb, kb * BK, tc.m_t * BM);
+                    } else if (g.a_kind == OP_KCONV) {
+                        const int tap = kb / g.conv_cb, cblk = kb % g.conv_cb;
+                        const int dy = tap / 3 - 1, dx = tap % 3 - 1;
+                        const int m0 = tc.m_t * BM;
+                        const int n0 = m0 / g.conv_hw;
+                        const int y0 = (m0 % g.conv_hw) / g.conv_w;
+                        tma_load_4d(sa, &ta, fb, cblk * BK, g.conv_sign * dx, y0 + g.conv_sign * dy, n0);
+                    } else {  // OP_MN2D: two 64-wide MN chunks
+                        tma_load_2d(sa, &ta, fb, tc.m_t * BM, kb * BK);
+                        tma_load_2d(sa + 8192u, &ta, fb, tc.m_t * BM + 64, kb * BK);
+                    }
+                    // ---- B
+                    if (g.b_kind == OP_K2D) {
+                        tma_load_2d(sb, &tb, fb, kb * BK, tc.n_t * BN);
+                    } else if (g.b_kind == OP_MN2D) {
+#pragma unroll
+                        for (int i = 0; i < BN / 64; ++i)
+                            tma_load_2d(sb + 8192u * i, &tb, fb, tc.n_t * BN + 64 * i, kb * BK);
+                    } else {  // OP_MNCONV: K rows kb*64.. of the image, shifted by the tile's tap
+                        const int m0 = kb * BK;
+                        const int n0 = m0 / g.conv_hw;
+                        const int y0 = (m0 % g.conv_hw) / g.conv_w;
+#pragma unroll
+                        for (int i = 0; i < BN / 64; ++i)
+                            tma_load_4d(sb + 8192u * i, &tb, fb, tc.n_t * BN + 64 * i, tdx, y0 + tdy, n0);
+                    }
+                    if (++stage == STAGES) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ MMA issuer
+            constexpr uint32_t idesc = umma_idesc_bf16(BM, BN, MN, MN);
+            int stage = 0;
+            uint32_t phase = 0;
+            int acc = 0;
+            uint32_t acc_phase = 0;
+            for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
+                const TileCoord tc = decode_tile(g, tile);
+                mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + acc * BN;
+                for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
+                    mbar_wait(full_bar(stage), phase);
+                    tc_fence_after();
+                    const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
+                    const uint32_t sb = sa + Cfg::A_BYTES;
+#pragma unroll
+                    for (int k = 0; k < BK / 16; ++k) {
+                        uint64_t ad, bd;
+                        if (MN) {
+                            ad = umma_desc_sw128(sa + k * 2048u, 8192u, 1024u);
+                            bd = umma_desc_sw128(sb + k * 2048u, 8192u, 1024u);
+                        } else {
+                            ad = umma_desc_sw128(sa + k * 32u, 16u, 1024u);
+                            bd = umma_desc_sw128(sb + k * 32u, 16u, 1024u);
+                        }
+                        tc_mma_f16(d_tmem, ad, bd, idesc, (kb > tc.kb0 || k > 0) ? 1u : 0u);
+                    }
+                    tc_commit(empty_bar(stage));
+                    if (++stage == STAGES) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                }
+                tc_commit(tfull_bar(acc));
+                acc ^= 1;
+                if (acc == 0) acc_phase ^= 1u;
+            }
+        }
+    } else {
+        // ---------------------------------------------------------------- epilogue
+        const int q = warp & 3;  // TMEM lane quadrant this warp may access
+        const int row = q * 32 + lane;
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
+            const TileCoord tc = decode_tile(g, tile);
+            mbar_wait(tfull_bar(acc), acc_phase);
+            tc_fence_after();
+            const int grow = tc.m_t * BM + row;
+            const bool row_ok = grow < g.M;
+            float *crow = g.C + (long long)grow * g.ldc + (long long)tc.tap * g.cols_per_tap;
+#pragma unroll 1
+            for (int c = 0; c < BN / 32; ++c) {
+                uint32_t r[32];
+                tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, r);
+                tmem_ld_wait();
+                const int col0 = tc.n_t * BN + c * 32;
+                if (row_ok) {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        const int col = col0 + 4 * j;
+                        if (col < g.N) {
+                            float *p = crow + col;
+                            const float a = __uint_as_float(r[4 * j]), b = __uint_as_float(r[4 * j + 1]);
+                            const float cc = __uint_as_float(r[4 * j + 2]), d = __uint_as_float(r[4 * j + 3]);
+                            if (g.store_mode == STORE_ATOMIC_ADD)
+                                red_add_v4(p, a, b, cc, d);
+                            else
+                                *reinterpret_cast<float4 *>(p) = make_float4(a, b, cc, d);
+                        }
+                    }
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(tempty_bar(acc));
+            acc ^= 1;
+            if (acc == 0) acc_phase ^= 1u;
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    if (warp == 1) tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+}
+
+// ------------------------------------------------------------------------------------ host side
+typedef CUresult (*PFN_encodeTiled_t)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                      const cuuint64_t *, const cuuint32_t *, const cuuint32_t *,
+                                      CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion,
+                                      CUtensorMapFloatOOBfill);
+
+static PFN_encodeTiled_t encode_fn() {
+    static PFN_encodeTiled_t fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void *p = nullptr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_encodeTiled_t>(p);
+    });
+    return fn;
+}
+
+bool make_map_2d(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                 uint32_t box_outer) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    if ((inner * 2) % 16 != 0 || (reinterpret_cast<uintptr_t>(ptr) & 15)) return false;
+    cuuint64_t dims[2] = {inner, outer};
+    cuuint64_t strides[1] = {inner * 2};
+    cuuint32_t box[2] = {box_inner, box_outer};
+    cuuint32_t es[2] = {1, 1};
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint64_t H, uint64_t NB,
+                   uint32_t box_w, uint32_t box_h, uint32_t box_n) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    if ((C * 2) % 16 != 0 || (reinterpret_cast<uintptr_t>(ptr) & 15)) return false;
+    cuuint64_t dims[4] = {C, W, H, NB};
+    cuuint64_t strides[3] = {C * 2, W * C * 2, H * W * C * 2};
+    cuuint32_t box[4] = {64, box_w, box_h, box_n};
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void *>(ptr), dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+static int pick_bn(int N) { return N <= 64 ? 64 : (N <= 128 ? 128 : 256); }
+static int cdiv(long long a, long long b) { return (int)((a + b - 1) / b); }
+
+// box geometry covering `rows` consecutive flat rows of an [nb][h][w] image stack
+static bool conv_box(int h, int w, int rows, uint32_t *bw, uint32_t *bh, uint32_t *bn) {
+    if (w > rows || rows % w) return false;
+    int by = rows / w;
+    if (by <= h) {
+        if (h % by) return false;
+        *bw = w; *bh = by; *bn = 1;
+        return true;
+    }
+    if (by % h) return false;
+    *bw = w; *bh = h; *bn = by / h;
+    return *bn <= 256;
+}
+
+bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K) {
+    if (M <= 0 || N <= 0 || K <= 0 || N % 4 || K % 8) return false;
+    GemmDev &d = g->d;
+    d = GemmDev{};
+    g->bn = pick_bn(N);
+    g->mn_major = 0;
+    d.m_tiles = cdiv(M, BM);
+    d.n_tiles = cdiv(N, g->bn);
+    d.taps = 1;
+    d.splits = 1;
+    d.num_kb = cdiv(K, BK);
+    d.kb_per_split = d.num_kb;
+    d.a_kind = OP_K2D;
+    d.b_kind = OP_K2D;
+    d.C = C;
+    d.ldc = N;
+    d.M = M;
+    d.N = N;
+    d.store_mode = STORE_OVERWRITE;
+    d.cols_per_tap = 0;
+    return make_map_2d(&g->ta, A, K, M, BK, BM) && make_map_2d(&g->tb, B, K, N, BK, g->bn);
+}
+
+static void choose_splits(GemmDev &d, int base_tiles, int num_sms) {
+    int target = 2 * num_sms;
+    int splits = base_tiles >= target ? 1 : cdiv(target, base_tiles);
+    if (splits > d.num_kb) splits = d.num_kb;
+    if (splits < 1) splits = 1;
+    d.kb_per_split = cdiv(d.num_kb, splits);
+    d.splits = cdiv(d.num_kb, d.kb_per_split);
+}
+
+bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms) {
+    // GEMM rows = N (output neurons), GEMM cols = K (inputs), reduction over M rows.
+    if (M <= 0 || N <= 0 || K <= 0 || N % 8 || K % 8) return false;
+    GemmDev &d = g->d;
+    d = GemmDev{};
+    g->bn = pick_bn(K);
+    g->mn_major = 1;
+    d.m_tiles = cdiv(N, BM);
+    d.n_tiles = cdiv(K, g->bn);
+    d.taps = 1;
+    d.num_kb = cdiv(M, BK);
+    choose_splits(d, d.m_tiles * d.n_tiles, num_sms);
+    d.a_kind = OP_MN2D;
+    d.b_kind = OP_MN2D;
+    d.C = dW;
+    d.ldc = K;
+    d.M = N;
+    d.N = K;
+    d.store_mode = STORE_ATOMIC_ADD;
+    return make_map_2d(&g->ta, D, N, M, 64, BK) && make_map_2d(&g->tb, X, K, M, 64, BK);
+}
+
+bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
+               int sign) {
+    // forward: A = X (cin channels), B = Wk [cout][9*cin], out channels cout.
+    // dgrad (sign = -1): caller passes X = D (cout channels of the layer) as "cin" and Wt as Wk.
+    if (cin % 64 || cout % 8) return false;
+    uint32_t bw, bh, bnn;
+    if (!conv_box(h, w, BM, &bw, &bh, &bnn)) return false;
+    const long long M = (long long)nb * h * w;
+    GemmDev &d = g->d;
+    d = GemmDev{};
+    g->bn = pick_bn(cout);
+    g->mn_major = 0;
+    d.m_tiles = cdiv(M, BM);
+    d.n_tiles = cdiv(cout, g->bn);
+    d.taps = 1;
+    d.splits = 1;
+    d.conv_cb = cin / 64;
+    d.num_kb = 9 * d.conv_cb;
+    d.kb_per_split = d.num_kb;
+    d.a_kind = OP_KCONV;
+    d.b_kind = OP_K2D;
+    d.conv_hw = h * w;
+    d.conv_w = w;
+    d.conv_sign = sign;
+    d.C = Y;
+    d.ldc = cout;
+    d.M = (int)M;
+    d.N = cout;
+    d.store_mode = STORE_OVERWRITE;
+    return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn);
+}
+
+bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
+                     int num_sms) {
+    if (cin % 64 || cout % 8) return false;
+    uint32_t bw, bh, bnn;
+    if (!conv_box(h, w, BK, &bw, &bh, &bnn)) return false;
+    const long long M = (long long)nb * h * w;
+    GemmDev &d = g->d;
+    d = GemmDev{};
+    g->bn = pick_bn(cin);
+    g->mn_major = 1;
+    d.m_tiles = cdiv(cout, BM);
+    d.n_tiles = cdiv(cin, g->bn);
+    d.taps = 9;
+    d.num_kb = cdiv(M, BK);
+    choose_splits(d, d.m_tiles * d.n_tiles * 9, num_sms);
+    d.a_kind = OP_MN2D;
+    d.b_kind = OP_MNCONV;
+    d.conv_hw = h * w;
+    d.conv_w = w;
+    d.conv_sign = 1;
+    d.cols_per_tap = cin;
+    d.C = dW;
+    d.ldc = 9ll * cin;
+    d.M = cout;
+    d.N = cin;
+    d.store_mode = STORE_ATOMIC_ADD;
+    return make_map_2d(&g->ta, D, cout, M, 64, BK) && make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn);
+}
+
+template <int BN, int MN>
+static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
+    using Cfg = GemmCfg<BN>;
+    static bool attr_done = false;
+    if (!attr_done) {
+        cudaError_t e = cudaFuncSetAttribute(gemm_tc_kernel<BN, MN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)Cfg::SMEM_BYTES);
+        if (e != cudaSuccess) return e;
+        attr_done = true;
+    }
+    const int total = g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
+    const int grid = total < num_sms ? total : num_sms;
+    gemm_tc_kernel<BN, MN><<<grid, NUM_THREADS, Cfg::SMEM_BYTES, stream>>>(g.ta, g.tb, g.d);
+    return cudaGetLastError();
+}
+
+cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
+    const int total = g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
+    if (total <= 0) return cudaSuccess;
+    if (g.mn_major) {
+        if (g.bn == 64) return launch_t<64, 1>(g, stream, num_sms);
+        if (g.bn == 128) return launch_t<128, 1>(g, stream, num_sms);
+        return launch_t<256, 1>(g, stream, num_sms);
+    }
+    if (g.bn == 64) return launch_t<64, 0>(g, stream, num_sms);
+    if (g.bn == 128) return launch_t<128, 0>(g, stream, num_sms);
+    return launch_t<256, 0>(g, stream, num_sms);
+}
+
+int device_num_sms() {
+    static int n = 0;
+    if (n == 0) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+    }
+    return n;
+}
+
+}  // namespace sk

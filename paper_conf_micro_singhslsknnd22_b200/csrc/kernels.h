@@ -1,0 +1,82 @@
+// kernels.h - launchers for the non-GEMM kernels of the hot path (all sm_100a CUDA cores).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace sk {
+
+enum { SURR_TRIANGLE = 0, SURR_FAST_SIGMOID = 1 };
+
+// K1: forward LIF temporal scan over the rows (timesteps) of one segment, Eq.1.
+// Neuron layout NHWC per row: row r holds B*H*W*C neurons (fc: H = W = 1).
+struct ScanFwdArgs {
+    const float *I;        // currents [R][B*N] (null for the direct conv kernel)
+    int R;                 // rows in the segment buffer
+    int restore;           // RECOMPUTE: row 0 is the checkpoint (U_state/o_state), rows 1.. recomputed
+    float *U_state;        // FIRST/RECORD: running U [B*N] (in/out); RECOMPUTE: checkpoint U (in)
+    uint8_t *o_state;      // same for spikes
+    float *U_out;          // [R][B*N] stored membranes (RECOMPUTE/RECORD) or null
+    uint16_t *Po_out;      // [R][B*Nout] bf16 layer output (pooled if pool) - next GEMM operand
+    float *ckU;            // FIRST: checkpoint slot written after row 0, else null
+    uint8_t *cko;
+    unsigned *s_part;      // SAM partials [T][32] or null (FIRST/RECORD only)
+    const int *row_t;      // absolute t of each row (device) or null -> t0 + r
+    int t0;
+    float *cnt;            // readout accumulation [B*Nout] or null (last spiking layer)
+    float *dbg_U;          // debug [T][B*N] or null
+    uint8_t *dbg_o;
+    int B, H, W, C, pool;
+    float lam, theta;
+    // direct conv (first layer, Cin*9 <= 32): input bit masks [T][B*H*W], weights bf16 [C][9*Cin]
+    const uint32_t *xmask;
+    const uint16_t *w_direct;
+    int kbits;             // 9*Cin
+};
+cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s);
+
+// K4: reverse surrogate-gradient scan, Eq.2: delta_t = sigma'(U_t) g_t + lam delta_{next}.
+struct ScanBwdArgs {
+    const float *g;        // gradient wrt the layer's output spikes
+    int g_pooled;          // g is at pooled resolution (x 0.25 spread, pool2^T)
+    int g_broadcast;       // g is [B*Nout] for every row (readout gradient, same at each t)
+    const float *U;        // [R][B*N]
+    float *carry;          // [B*N] delta at the first row of the next segment (in) / of this one (out)
+    uint16_t *delta;       // [R][B*N] bf16 (dgrad / wgrad operand) or null
+    int R;
+    int B, H, W, C, pool;
+    float lam, theta;
+    int surr;
+    float gamma;
+    // direct conv: fused weight gradient dW[C][kbits] += sum delta_bf16 * input bit
+    const uint32_t *xmask;
+    const int *row_t;
+    float *dW_direct;
+    int kbits;
+};
+cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s);
+
+// Input staging (once per step): SAM term l = 0 (Eq.4) and the first layer's operand.
+cudaError_t launch_stage_bits(const uint8_t *x, uint32_t *xmask, unsigned *s_part, int T, int B, int H, int W,
+                              int C0, cudaStream_t s);
+cudaError_t launch_stage_bf16(const uint8_t *x, uint16_t *xb, unsigned *s_part, int T, int B, int D,
+                              cudaStream_t s);
+cudaError_t launch_gather_rows(const uint16_t *src, uint16_t *dst, const int *rows, int R, size_t row_elems,
+                               cudaStream_t s);
+cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);
+
+// Readout integrator + softmax cross-entropy (reading 5) and its gradients.
+cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int *labels, float *z, float *dz,
+                                float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
+                                cudaStream_t s);
+cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K,
+                                 float invT, cudaStream_t s);
+
+// Adam + bf16 shadow; transposed bf16 shadow for the dgrad GEMMs.
+cudaError_t launch_adam(float *w, const float *g, float *m, float *v, uint16_t *wb, size_t n, float lr, float b1,
+                        float b2, float eps, float bc1, float bc2_sqrt, cudaStream_t s);
+cudaError_t launch_cast_bf16(const float *w, uint16_t *wb, size_t n, cudaStream_t s);
+// dst[c][t][a] = src[a][t][c]   (src viewed [A][Tp][Cc])
+cudaError_t launch_transpose_bf16(const uint16_t *src, uint16_t *dst, int A, int Tp, int Cc, cudaStream_t s);
+
+}  // namespace sk

@@ -1,0 +1,624 @@
+// lif_kernels.cu - K1 (forward LIF scan), K4 (reverse surrogate scan), the fused direct first-layer
+// conv kernels, input staging / SAM, readout + loss, Adam.  sm_100a CUDA cores; HBM-bound streams.
+//
+// Eq.1:  U_t = lam*U_{t-1} + W o^{l-1}_t - theta*o^l_{t-1};  o_t = [U_t > theta]
+//   evaluated without FMA in the order ((lam*U) + I) - theta*o so that spikes are bit-identical to
+//   the oracle.
+// Eq.2:  delta^l_t = sigma'(U^l_t) * g^l_t + lam * delta^l_{t+1}, reset detached.
+// Eq.4:  s_t = sum_l sum(o^l_t), accumulated in [T][32] partial counters.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace sk {
+
+SK_DEV float lif_update(float U, float I, float o, float lam, float th) {
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+}
+
+SK_DEV float surrogate(float U, float th, int kind, float gamma) {
+    if (kind == SURR_TRIANGLE) {
+        const float v = 1.0f - fabsf(U - th) / th;
+        return v > 0.0f ? gamma * v : 0.0f;
+    }
+    const float d = 1.0f + gamma * fabsf(U - th);
+    return 1.0f / (d * d);
+}
+
+SK_DEV uint2 pack_bf16x4(float a, float b, float c, float d) {
+    uint2 r;
+    r.x = (uint32_t)f2bf_bits(a) | ((uint32_t)f2bf_bits(b) << 16);
+    r.y = (uint32_t)f2bf_bits(c) | ((uint32_t)f2bf_bits(d) << 16);
+    return r;
+}
+
+SK_DEV float4 ldg4(const float *p) { return __ldg(reinterpret_cast<const float4 *>(p)); }
+
+// ============================================================================ K1 forward scan
+// One thread owns 4 consecutive channels of NP pixels (NP = 4 for a 2x2 pooled window).
+template <int POOL, int DIRECT, int CH>
+__global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
+    constexpr int NP = POOL ? 4 : 1;
+    extern __shared__ float ws[];  // DIRECT: fp32 copy of bf16 weights, [kbits][C]
+    __shared__ unsigned red[8][CH];
+    const int C = a.C;
+    const int C4 = C >> 2;
+    const long long HW = (long long)a.H * a.W;
+    const long long P = POOL ? (long long)a.B * (a.H / 2) * (a.W / 2) * C4 : (long long)a.B * HW * C4;
+    const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool active = p < P;
+    const long long rs = (long long)a.B * HW * C;  // neurons per row
+    const long long ors = POOL ? rs / 4 : rs;       // outputs per row
+    const long long npix_row = (long long)a.B * HW;
+
+    long long nidx[NP], pix[NP], oidx = 0;
+    int c4 = 0;
+    if (active) {
+        c4 = (int)(p % C4);
+        long long rest = p / C4;
+        if (POOL) {
+            const int PW = a.W / 2, PH = a.H / 2;
+            const int px = (int)(rest % PW);
+            rest /= PW;
+            const int py = (int)(rest % PH);
+            const long long b = rest / PH;
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                const int y = 2 * py + (k >> 1), x = 2 * px + (k & 1);
+                pix[k] = (b * a.H + y) * a.W + x;
+                nidx[k] = pix[k] * C + 4 * c4;
+            }
+            oidx = ((b * PH + py) * PW + px) * C + 4 * c4;
+        } else {
+            pix[0] = rest;
+            nidx[0] = rest * C + 4 * c4;
+            oidx = nidx[0];
+        }
+    } else {
+#pragma unroll
+        for (int k = 0; k < NP; ++k) nidx[k] = pix[k] = 0;
+    }
+    if (DIRECT) {
+        for (int i = threadIdx.x; i < a.kbits * C; i += blockDim.x) {
+            const int k = i / C, c = i % C;
+            ws[k * C + c] = bf_bits2f(a.w_direct[c * a.kbits + k]);
+        }
+        __syncthreads();
+    }
+
+    float U[NP][4], O[NP][4];
+#pragma unroll
+    for (int k = 0; k < NP; ++k) {
+        if (active) {
+            const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nidx[k]);
+            const uchar4 ob = *reinterpret_cast<const uchar4 *>(a.o_state + nidx[k]);
+            U[k][0] = u.x; U[k][1] = u.y; U[k][2] = u.z; U[k][3] = u.w;
+            O[k][0] = ob.x; O[k][1] = ob.y; O[k][2] = ob.z; O[k][3] = ob.w;
+        } else {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) U[k][i] = O[k][i] = 0.f;
+        }
+    }
+    float cacc[4] = {0.f, 0.f, 0.f, 0.f};
+
+    auto emit_row = [&](int r) {  // write outputs of row r from the current (U, O)
+        float out[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            float sum = 0.f;
+#pragma unroll
+            for (int k = 0; k < NP; ++k) sum += O[k][i];
+            out[i] = POOL ? sum * 0.25f : sum;
+            cacc[i] += out[i];
+        }
+        *reinterpret_cast<uint2 *>(a.Po_out + (long long)r * ors + oidx) = pack_bf16x4(out[0], out[1], out[2], out[3]);
+        if (a.U_out) {
+#pragma unroll
+            for (int k = 0; k < NP; ++k)
+                *reinterpret_cast<float4 *>(a.U_out + (long long)r * rs + nidx[k]) =
+                    make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
+        }
+        if (a.dbg_U) {
+            const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                *reinterpret_cast<float4 *>(a.dbg_U + t * rs + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
+                *reinterpret_cast<uchar4 *>(a.dbg_o + t * rs + nidx[k]) =
+                    make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+            }
+        }
+    };
+
+    int r0 = 0;
+    if (a.restore) {
+        if (active) emit_row(0);
+        r0 = 1;
+    }
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int nwarps = blockDim.x >> 5;
+    for (int rb = r0; rb < a.R; rb += CH) {
+        float4 Iv[CH][NP];
+        uint32_t mk[CH][NP];
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb + j;
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                if (active && r < a.R) {
+                    if (DIRECT) {
+                        const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+                        mk[j][k] = __ldg(a.xmask + t * npix_row + pix[k]);
+                    } else {
+                        Iv[j][k] = ldg4(a.I + (long long)r * rs + nidx[k]);
+                    }
+                } else {
+                    mk[j][k] = 0;
+                    Iv[j][k] = make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+            }
+        }
+        unsigned nspk[CH];
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb + j;
+            nspk[j] = 0;
+            if (active && r < a.R) {
+#pragma unroll
+                for (int k = 0; k < NP; ++k) {
+                    float4 Ik;
+                    if (DIRECT) {
+                        Ik = make_float4(0.f, 0.f, 0.f, 0.f);
+                        const uint32_t m = mk[j][k];
+                        for (int kb = 0; kb < a.kbits; ++kb) {
+                            if ((m >> kb) & 1u) {
+                                const float4 w = *reinterpret_cast<const float4 *>(&ws[kb * C + 4 * c4]);
+                                Ik.x += w.x; Ik.y += w.y; Ik.z += w.z; Ik.w += w.w;
+                            }
+                        }
+                    } else {
+                        Ik = Iv[j][k];
+                    }
+                    const float Ii[4] = {Ik.x, Ik.y, Ik.z, Ik.w};
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        U[k][i] = lif_update(U[k][i], Ii[i], O[k][i], a.lam, a.theta);
+                        O[k][i] = U[k][i] > a.theta ? 1.f : 0.f;
+                        nspk[j] += (unsigned)O[k][i];
+                    }
+                }
+                emit_row(r);
+                if (a.ckU && r == 0) {
+#pragma unroll
+                    for (int k = 0; k < NP; ++k) {
+                        *reinterpret_cast<float4 *>(a.ckU + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
+                        *reinterpret_cast<uchar4 *>(a.cko + nidx[k]) =
+                            make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+                    }
+                }
+            }
+        }
+        if (a.s_part) {  // block-uniform
+#pragma unroll
+            for (int j = 0; j < CH; ++j) {
+                const unsigned v = __reduce_add_sync(0xffffffffu, nspk[j]);
+                if (lane == 0) red[warp][j] = v;
+            }
+            __syncthreads();
+            if (threadIdx.x < CH && rb + (int)threadIdx.x < a.R) {
+                unsigned tot = 0;
+                for (int w = 0; w < nwarps; ++w) tot += red[w][threadIdx.x];
+                const int r = rb + threadIdx.x;
+                const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+                if (tot) atomicAdd(a.s_part + t * 32 + (blockIdx.x & 31), tot);
+            }
+            __syncthreads();
+        }
+    }
+    if (active) {
+        if (!a.restore) {
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                *reinterpret_cast<float4 *>(a.U_state + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
+                *reinterpret_cast<uchar4 *>(a.o_state + nidx[k]) =
+                    make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+            }
+        }
+        if (a.cnt) {
+            float4 *cp = reinterpret_cast<float4 *>(a.cnt + oidx);
+            float4 cv = *cp;
+            cv.x += cacc[0]; cv.y += cacc[1]; cv.z += cacc[2]; cv.w += cacc[3];
+            *cp = cv;
+        }
+    }
+}
+
+cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
+    if (a.C % 4) return cudaErrorInvalidValue;
+    const long long HW = (long long)a.H * a.W;
+    const long long P = a.pool ? (long long)a.B * (a.H / 2) * (a.W / 2) * (a.C / 4) : (long long)a.B * HW * (a.C / 4);
+    const int threads = 256;
+    const long long blocks = (P + threads - 1) / threads;
+    if (blocks == 0) return cudaSuccess;
+    const bool direct = a.xmask != nullptr;
+    const size_t smem = direct ? (size_t)a.kbits * a.C * sizeof(float) : 0;
+    if (a.pool) {
+        if (direct) lif_fwd_kernel<1, 1, 4><<<(unsigned)blocks, threads, smem, s>>>(a);
+        else lif_fwd_kernel<1, 0, 4><<<(unsigned)blocks, threads, smem, s>>>(a);
+    } else {
+        if (direct) lif_fwd_kernel<0, 1, 8><<<(unsigned)blocks, threads, smem, s>>>(a);
+        else lif_fwd_kernel<0, 0, 8><<<(unsigned)blocks, threads, smem, s>>>(a);
+    }
+    return cudaGetLastError();
+}
+
+// ============================================================================ K4 reverse scan
+template <int CH>
+__global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
+    const int C = a.C;
+    const long long HW = (long long)a.H * a.W;
+    const long long rs = (long long)a.B * HW * C;
+    const long long P = rs / 4;
+    const long long p = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (p >= P) return;
+    const long long n0 = 4 * p;
+    long long gi = n0, grs = rs;
+    if (a.g_pooled) {
+        const int c = (int)(n0 % C);
+        const long long pixel = n0 / C;
+        const int x = (int)(pixel % a.W);
+        const int y = (int)((pixel / a.W) % a.H);
+        const long long b = pixel / HW;
+        gi = ((b * (a.H / 2) + y / 2) * (a.W / 2) + x / 2) * C + c;
+        grs = rs / 4;
+    }
+    if (a.g_broadcast) grs = 0;
+    const float gs = a.g_pooled ? 0.25f : 1.0f;
+    float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
+    for (int rb = a.R - 1; rb >= 0; rb -= CH) {
+        float4 gv[CH], uv[CH];
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb - j;
+            if (r >= 0) {
+                gv[j] = ldg4(a.g + (long long)r * grs + gi);
+                uv[j] = ldg4(a.U + (long long)r * rs + n0);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb - j;
+            if (r >= 0) {
+                d.x = surrogate(uv[j].x, a.theta, a.surr, a.gamma) * (gs * gv[j].x) + a.lam * d.x;
+                d.y = surrogate(uv[j].y, a.theta, a.surr, a.gamma) * (gs * gv[j].y) + a.lam * d.y;
+                d.z = surrogate(uv[j].z, a.theta, a.surr, a.gamma) * (gs * gv[j].z) + a.lam * d.z;
+                d.w = surrogate(uv[j].w, a.theta, a.surr, a.gamma) * (gs * gv[j].w) + a.lam * d.w;
+                if (a.delta)
+                    *reinterpret_cast<uint2 *>(a.delta + (long long)r * rs + n0) = pack_bf16x4(d.x, d.y, d.z, d.w);
+            }
+        }
+    }
+    *reinterpret_cast<float4 *>(a.carry + n0) = d;
+}
+
+// Direct first layer: reverse scan fused with its weight gradient (the input is a 27-bit mask per
+// pixel, so dW[c][k] += bf16(delta) wherever input bit k is set).  One thread per (pixel, channel);
+// the mask is warp-uniform for C >= 32, so the per-bit branches do not diverge.
+template <int CH>
+__global__ void __launch_bounds__(256) lif_bwd_direct_kernel(const ScanBwdArgs a) {
+    __shared__ float red[256 * 32];
+    const int C = a.C;
+    const int c = threadIdx.x % C;
+    const int slot = threadIdx.x / C;
+    const int spb = blockDim.x / C;
+    const long long HW = (long long)a.H * a.W;
+    const long long npix = (long long)a.B * HW;
+    const long long rs = npix * C;
+    const float gs = a.g_pooled ? 0.25f : 1.0f;
+    float acc[32];
+#pragma unroll
+    for (int k = 0; k < 32; ++k) acc[k] = 0.f;
+    for (long long pixel = (long long)blockIdx.x * spb + slot; pixel < npix; pixel += (long long)gridDim.x * spb) {
+        const long long n = pixel * C + c;
+        long long gi = n, grs = rs;
+        if (a.g_pooled) {
+            const int x = (int)(pixel % a.W);
+            const int y = (int)((pixel / a.W) % a.H);
+            const long long b = pixel / HW;
+            gi = ((b * (a.H / 2) + y / 2) * (a.W / 2) + x / 2) * C + c;
+            grs = rs / 4;
+        }
+        if (a.g_broadcast) grs = 0;
+        float d = a.carry[n];
+        for (int rb = a.R - 1; rb >= 0; rb -= CH) {
+            float gv[CH], uv[CH];
+            uint32_t mk[CH];
+#pragma unroll
+            for (int j = 0; j < CH; ++j) {
+                const int r = rb - j;
+                if (r >= 0) {
+                    gv[j] = __ldg(a.g + (long long)r * grs + gi);
+                    uv[j] = __ldg(a.U + (long long)r * rs + n);
+                    const long long t = a.row_t ? a.row_t[r] : r;
+                    mk[j] = __ldg(a.xmask + t * npix + pixel);
+                } else {
+                    gv[j] = uv[j] = 0.f;
+                    mk[j] = 0;
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < CH; ++j) {
+                const int r = rb - j;
+                if (r >= 0) {
+                    d = surrogate(uv[j], a.theta, a.surr, a.gamma) * (gs * gv[j]) + a.lam * d;
+                    const float db = bf_bits2f(f2bf_bits(d));
+                    if (a.delta) a.delta[(long long)r * rs + n] = f2bf_bits(d);
+                    const uint32_t m = mk[j];
+#pragma unroll
+                    for (int k = 0; k < 32; ++k)
+                        if ((m >> k) & 1u) acc[k] += db;
+                }
+            }
+        }
+        a.carry[n] = d;
+    }
+#pragma unroll
+    for (int k = 0; k < 32; ++k) red[threadIdx.x * 32 + k] = acc[k];
+    __syncthreads();
+    for (int i = threadIdx.x; i < C * a.kbits; i += blockDim.x) {
+        const int cc = i / a.kbits, k = i % a.kbits;
+        float sum = 0.f;
+        for (int sl = 0; sl < spb; ++sl) sum += red[(sl * C + cc) * 32 + k];
+        if (sum != 0.f) atomicAdd(a.dW_direct + (long long)cc * a.kbits + k, sum);
+    }
+}
+
+cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
+    if (a.C % 4) return cudaErrorInvalidValue;
+    const long long rs = (long long)a.B * a.H * a.W * a.C;
+    if (rs == 0 || a.R == 0) return cudaSuccess;
+    if (a.xmask) {
+        if (256 % a.C || a.kbits > 32) return cudaErrorInvalidValue;
+        int sms = 148;
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        const long long npix = (long long)a.B * a.H * a.W;
+        const int spb = 256 / a.C;
+        long long blocks = (npix + spb - 1) / spb;
+        const long long cap = 4LL * sms;
+        if (blocks > cap) blocks = cap;
+        lif_bwd_direct_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a);
+    } else {
+        const long long P = rs / 4;
+        lif_bwd_kernel<8><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
+    }
+    return cudaGetLastError();
+}
+
+// ============================================================================ input staging / SAM
+SK_DEV void sam_add(unsigned *s_part, long long t, unsigned v) {
+    // warp-aggregate when the whole warp is in the same timestep
+    const unsigned mask = 0xffffffffu;
+    const long long t0 = __shfl_sync(mask, t, 0);
+    const bool same = __all_sync(mask, t == t0);
+    if (same) {
+        const unsigned tot = __reduce_add_sync(mask, v);
+        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(s_part + t0 * 32 + (blockIdx.x & 31), tot);
+    } else if (v) {
+        atomicAdd(s_part + t * 32 + (blockIdx.x & 31), v);
+    }
+}
+
+__global__ void stage_bits_kernel(const uint8_t *__restrict__ x, uint32_t *__restrict__ xmask, unsigned *s_part,
+                                  int T, int B, int H, int W, int C0) {
+    const long long total = (long long)T * B * H * W;
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool ok = i < total;
+    long long t = 0;
+    unsigned cnt = 0;
+    if (ok) {
+        const int xx = (int)(i % W);
+        const int yy = (int)((i / W) % H);
+        const long long tb = i / ((long long)H * W);  // t*B + b
+        t = tb / B;
+        uint32_t m = 0;
+        for (int dy = 0; dy < 3; ++dy) {
+            const int y = yy + dy - 1;
+            if (y < 0 || y >= H) continue;
+            for (int dx = 0; dx < 3; ++dx) {
+                const int xq = xx + dx - 1;
+                if (xq < 0 || xq >= W) continue;
+                const uint8_t *px = x + ((tb * H + y) * W + xq) * C0;
+                for (int ci = 0; ci < C0; ++ci)
+                    if (px[ci]) m |= 1u << ((dy * 3 + dx) * C0 + ci);
+            }
+        }
+        xmask[i] = m;
+        const uint8_t *pc = x + i * C0;
+        for (int ci = 0; ci < C0; ++ci) cnt += pc[ci] ? 1u : 0u;
+    } else {
+        t = (long long)T - 1;
+    }
+    sam_add(s_part, t, cnt);
+}
+
+cudaError_t launch_stage_bits(const uint8_t *x, uint32_t *xmask, unsigned *s_part, int T, int B, int H, int W,
+                              int C0, cudaStream_t s) {
+    const long long total = (long long)T * B * H * W;
+    stage_bits_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, xmask, s_part, T, B, H, W, C0);
+    return cudaGetLastError();
+}
+
+__global__ void stage_bf16_kernel(const uint8_t *__restrict__ x, uint16_t *__restrict__ xb, unsigned *s_part, int T,
+                                  int B, int D) {
+    const long long total = (long long)T * B * D;
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    long long t = (long long)T - 1;
+    unsigned v = 0;
+    if (i < total) {
+        v = x[i] ? 1u : 0u;
+        xb[i] = v ? (uint16_t)0x3F80 : (uint16_t)0;
+        t = i / ((long long)B * D);
+    }
+    sam_add(s_part, t, v);
+}
+
+cudaError_t launch_stage_bf16(const uint8_t *x, uint16_t *xb, unsigned *s_part, int T, int B, int D, cudaStream_t s) {
+    const long long total = (long long)T * B * D;
+    stage_bf16_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, xb, s_part, T, B, D);
+    return cudaGetLastError();
+}
+
+__global__ void gather_rows_kernel(const uint16_t *__restrict__ src, uint16_t *__restrict__ dst, const int *rows, int R,
+                                   long long row_elems) {
+    const long long total = (long long)R * row_elems;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+        const long long r = i / row_elems, e = i % row_elems;
+        dst[i] = src[(long long)rows[r] * row_elems + e];
+    }
+}
+
+cudaError_t launch_gather_rows(const uint16_t *src, uint16_t *dst, const int *rows, int R, size_t row_elems,
+                               cudaStream_t s) {
+    const long long total = (long long)R * (long long)row_elems;
+    if (total == 0) return cudaSuccess;
+    long long blocks = (total + 255) / 256;
+    if (blocks > 65535) blocks = 65535;
+    gather_rows_kernel<<<(unsigned)blocks, 256, 0, s>>>(src, dst, rows, R, (long long)row_elems);
+    return cudaGetLastError();
+}
+
+__global__ void sam_finalize_kernel(const unsigned *s_part, long long *s, int T) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    long long tot = 0;
+    for (int i = 0; i < 32; ++i) tot += s_part[t * 32 + i];
+    s[t] = tot;
+}
+
+cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st) {
+    sam_finalize_kernel<<<(T + 255) / 256, 256, 0, st>>>(s_part, s, T);
+    return cudaGetLastError();
+}
+
+// ============================================================================ readout + loss
+__global__ void readout_loss_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ cnt, const int *labels,
+                                    float *z, float *dz, float *loss, float *g_last, int D, int K, float invT,
+                                    float invBg) {
+    extern __shared__ float sh[];  // zs[K], dzs[K]
+    float *zs = sh, *dzs = sh + K;
+    const int b = blockIdx.x;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    const float *cb = cnt + (long long)b * D;
+    for (int k = warp; k < K; k += nw) {
+        float acc = 0.f;
+        for (int n = lane; n < D; n += 32) acc += bf_bits2f(WbL[(long long)k * D + n]) * cb[n];
+        for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+        if (lane == 0) {
+            zs[k] = acc * invT;
+            z[(long long)b * K + k] = acc * invT;
+        }
+    }
+    __syncthreads();
+    if (warp == 0) {
+        float mx = -INFINITY;
+        for (int k = lane; k < K; k += 32) mx = fmaxf(mx, zs[k]);
+        for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        float se = 0.f;
+        for (int k = lane; k < K; k += 32) se += expf(zs[k] - mx);
+        for (int o = 16; o; o >>= 1) se += __shfl_xor_sync(0xffffffffu, se, o);
+        const int y = labels[b];
+        for (int k = lane; k < K; k += 32) {
+            const float pr = expf(zs[k] - mx) / se;
+            const float v = (pr - (k == y ? 1.f : 0.f)) * invBg;
+            dzs[k] = v;
+            dz[(long long)b * K + k] = v;
+        }
+        if (lane == 0) atomicAdd(loss, (logf(se) + mx - zs[y]) * invBg);
+    }
+    __syncthreads();
+    for (int n = threadIdx.x; n < D; n += blockDim.x) {
+        float acc = 0.f;
+        for (int k = 0; k < K; ++k) acc += dzs[k] * bf_bits2f(WbL[(long long)k * D + n]);
+        g_last[(long long)b * D + n] = acc * invT;
+    }
+}
+
+cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int *labels, float *z, float *dz,
+                                float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
+                                cudaStream_t s) {
+    readout_loss_kernel<<<B, 256, 2 * K * sizeof(float), s>>>(WbL, cnt, labels, z, dz, loss, g_last, D, K, invT, invBg);
+    return cudaGetLastError();
+}
+
+__global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (long long)K * D) return;
+    const int k = (int)(i / D), n = (int)(i % D);
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b) acc += dz[(long long)b * K + k] * cnt_kept[(long long)b * D + n];
+    dWL[i] = acc * invT;
+}
+
+cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT,
+                                 cudaStream_t s) {
+    const long long n = (long long)K * D;
+    readout_wgrad_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(dz, cnt_kept, dWL, B, D, K, invT);
+    return cudaGetLastError();
+}
+
+// ============================================================================ Adam + shadows
+__global__ void adam_kernel(float *w, const float *g, float *m, float *v, uint16_t *wb, long long n, float lr, float b1,
+                            float b2, float eps, float bc1, float bc2_sqrt) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const float gi = g[i];
+    const float mi = b1 * m[i] + (1.f - b1) * gi;
+    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
+    m[i] = mi;
+    v[i] = vi;
+    const float wi = w[i] - (lr / bc1) * mi / (sqrtf(vi) / bc2_sqrt + eps);
+    w[i] = wi;
+    wb[i] = f2bf_bits(wi);
+}
+
+cudaError_t launch_adam(float *w, const float *g, float *m, float *v, uint16_t *wb, size_t n, float lr, float b1,
+                        float b2, float eps, float bc1, float bc2_sqrt, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    adam_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1, bc2_sqrt);
+    return cudaGetLastError();
+}
+
+__global__ void cast_bf16_kernel(const float *w, uint16_t *wb, long long n) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n) wb[i] = f2bf_bits(w[i]);
+}
+
+cudaError_t launch_cast_bf16(const float *w, uint16_t *wb, size_t n, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    cast_bf16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(w, wb, (long long)n);
+    return cudaGetLastError();
+}
+
+// dst[c][t][a] = src[a][t][c]
+__global__ void transpose_bf16_kernel(const uint16_t *src, uint16_t *dst, int A, int Tp, int Cc) {
+    __shared__ uint16_t tile[32][33];
+    const int t = blockIdx.z;
+    const int a0 = blockIdx.y * 32, c0 = blockIdx.x * 32;
+    for (int i = threadIdx.y; i < 32; i += blockDim.y) {
+        const int a = a0 + i, c = c0 + threadIdx.x;
+        if (a < A && c < Cc) tile[i][threadIdx.x] = src[((long long)a * Tp + t) * Cc + c];
+    }
+    __syncthreads();
+    for (int i = threadIdx.y; i < 32; i += blockDim.y) {
+        const int c = c0 + i, a = a0 + threadIdx.x;
+        if (a < A && c < Cc) dst[((long long)c * Tp + t) * A + a] = tile[threadIdx.x][i];
+    }
+}
+
+cudaError_t launch_transpose_bf16(const uint16_t *src, uint16_t *dst, int A, int Tp, int Cc, cudaStream_t s) {
+    dim3 grid((Cc + 31) / 32, (A + 31) / 32, Tp);
+    transpose_bf16_kernel<<<grid, dim3(32, 8), 0, s>>>(src, dst, A, Tp, Cc);
+    return cudaGetLastError();
+}
+
+}  // namespace sk

@@ -1,0 +1,371 @@
+"""Thin ctypes binding of include/skipper.h (argument marshalling only).
+
+Every step of the training path runs in libskipper.so (sm_100a kernels); this
+module only converts Python/torch objects into pointers and sizes.  PyTorch is
+used for device memory (the caching allocator, so torch's memory statistics
+count the library's buffers), streams and process groups.  There is no CPU or
+PyTorch fallback: if the library is missing this module raises on import.
+"""
+from __future__ import annotations
+
+import ctypes as ct
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libskipper.so")
+
+MODE = {"full": 0, "ckpt": 1, "skip": 2}
+PASS_FIRST, PASS_RECOMPUTE, PASS_RECORD = 0, 1, 2
+LAYER_KIND = {"fc": 0, "conv": 1, "readout": 2}
+SURROGATE = {"triangle": 0, "fast_sigmoid": 1}
+STATUS = {0: "ok", 1: "EINVAL", 2: "ENOMEM", 3: "ECUDA", 4: "ENCCL", 5: "EORDER", 6: "EFAILED", 7: "EUNSUPPORTED"}
+
+
+class SkipperError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Layer(ct.Structure):
+    _fields_ = [("kind", ct.c_int), ("cin", ct.c_int), ("cout", ct.c_int), ("h", ct.c_int), ("w", ct.c_int),
+                ("pool", ct.c_int), ("lam", ct.c_float), ("theta", ct.c_float)]
+
+
+class Config(ct.Structure):
+    _fields_ = [("T", ct.c_int), ("C", ct.c_int), ("p", ct.c_double), ("mode", ct.c_int), ("batch", ct.c_int),
+                ("global_batch", ct.c_int), ("surrogate", ct.c_int), ("surr_gamma", ct.c_float),
+                ("lr", ct.c_float), ("beta1", ct.c_float), ("beta2", ct.c_float), ("eps", ct.c_float),
+                ("debug_record", ct.c_int)]
+
+
+ALLOC_FN = ct.CFUNCTYPE(ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
+FREE_FN = ct.CFUNCTYPE(None, ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
+
+
+class Allocator(ct.Structure):
+    _fields_ = [("alloc", ALLOC_FN), ("free", FREE_FN), ("user", ct.c_void_p)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                          "(python -m paper_conf_micro_singhslsknnd22_b200.build)")
+    lib = ct.CDLL(LIB_PATH)
+    P, I, S = ct.c_void_p, ct.c_int, ct.c_size_t
+    sig = {
+        "skipper_create": (I, [ct.POINTER(Layer), I, ct.POINTER(Config), ct.POINTER(Allocator), P, ct.POINTER(P)]),
+        "skipper_destroy": (None, [P]),
+        "skipper_last_error": (ct.c_char_p, [P]),
+        "skipper_set_weights": (I, [P, I, P]),
+        "skipper_get_weights": (I, [P, I, P]),
+        "skipper_get_grads": (I, [P, I, P]),
+        "skipper_weight_count": (S, [P, I]),
+        "skipper_forward_segment": (I, [P, I, I, P, P]),
+        "skipper_backward_segment": (I, [P, I]),
+        "skipper_optimizer_step": (I, [P]),
+        "skipper_step": (I, [P, P, P, P]),
+        "skipper_step_host": (I, [P, P, P, P]),
+        "skipper_comm_unique_id": (I, [P]),
+        "skipper_comm_init": (I, [P, P, I, I]),
+        "skipper_get_loss": (I, [P, P]),
+        "skipper_get_spike_sums": (I, [P, P]),
+        "skipper_get_keep_mask": (I, [P, P]),
+        "skipper_get_sst": (I, [P, P]),
+        "skipper_mem_stats": (I, [P, P, P]),
+        "skipper_reset_peak": (I, [P]),
+        "skipper_debug_copy": (I, [P, I, I, P, S]),
+        "skipper_sst_host": (ct.c_double, [P, I, ct.c_double]),
+        "skipper_workspace_bytes": (S, [ct.POINTER(Layer), I, ct.POINTER(Config), I]),
+        "skipper_status_string": (ct.c_char_p, [I]),
+        "skipper_build_info": (ct.c_char_p, []),
+        "skipper_k_fc_fwd": (I, [P, P, P, I, I, I, P]),
+        "skipper_k_fc_wgrad": (I, [P, P, P, I, I, I, I, P]),
+        "skipper_k_conv_fwd": (I, [P, P, P, I, I, I, I, I, P]),
+        "skipper_k_conv_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
+        "skipper_k_conv_wgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
+        "skipper_k_num_sms": (I, []),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    return lib
+
+
+lib = _load()
+
+
+def _check(status, ctx=None):
+    if status != 0:
+        msg = lib.skipper_last_error(ctx)
+        raise SkipperError(status, msg.decode() if msg else "")
+
+
+def make_layers(net):
+    arr = (Layer * len(net["layers"]))()
+    for i, L in enumerate(net["layers"]):
+        arr[i] = Layer(LAYER_KIND[L["kind"]], L["cin"], L["cout"], L.get("h", 1), L.get("w", 1),
+                       L.get("pool", 0), float(L.get("lam", 1.0)), float(L.get("theta", 1.0)))
+    return arr
+
+
+def make_config(T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle", gamma=0.3,
+                lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False):
+    return Config(T, C, float(p), MODE[mode], batch, global_batch, SURROGATE[surrogate], gamma, lr, beta1, beta2,
+                  eps, 1 if debug_record else 0)
+
+
+def sst_host(values, p):
+    """Eq.5 for one segment as implemented in the library (host code)."""
+    a = np.ascontiguousarray(values, dtype=np.int64)
+    return lib.skipper_sst_host(a.ctypes.data, a.size, float(p))
+
+
+def workspace_bytes(net, cfg: Config, kept_max=-1):
+    layers = make_layers(net)
+    return lib.skipper_workspace_bytes(layers, len(net["layers"]), ct.byref(cfg), kept_max)
+
+
+def _torch():
+    import torch
+    return torch
+
+
+class TorchAllocator:
+    """Routes library allocations through torch's CUDA caching allocator."""
+
+    def __init__(self, device):
+        torch = _torch()
+        self.device = device
+
+        def _alloc(nbytes, stream, user):
+            try:
+                return torch.cuda.caching_allocator_alloc(int(nbytes), device=self.device, stream=stream or 0)
+            except Exception:  # noqa: BLE001 - reported to the library as NULL -> ENOMEM
+                return None
+
+        def _free(ptr, nbytes, stream, user):
+            torch.cuda.caching_allocator_delete(ptr)
+
+        self._a = ALLOC_FN(_alloc)
+        self._f = FREE_FN(_free)
+        self.struct = Allocator(self._a, self._f, None)
+
+
+class SkipperNet:
+    """One training context (one GPU / rank).  `net` is a synth.configs-style dict."""
+
+    def __init__(self, net, T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle",
+                 gamma=0.3, lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, stream=None,
+                 torch_allocator=True):
+        torch = _torch()
+        self.net = net
+        self.T, self.B = T, batch
+        self.mode = mode
+        self.C = 1 if mode == "full" else C
+        self.device = torch.cuda.current_device()
+        self.stream = stream if stream is not None else torch.cuda.current_stream()
+        self.cfg = make_config(T, C, p, mode, batch, global_batch, surrogate, gamma, lr, beta1, beta2, eps,
+                               debug_record)
+        self._layers = make_layers(net)
+        self._alloc = TorchAllocator(self.device) if torch_allocator else None
+        h = ct.c_void_p()
+        st = _check(lib.skipper_create(self._layers, len(net["layers"]), ct.byref(self.cfg),
+                                       ct.byref(self._alloc.struct) if self._alloc else None,
+                                       ct.c_void_p(self.stream.cuda_stream), ct.byref(h)))
+        del st
+        self.ctx = h
+        self.n_layers = len(net["layers"])
+        self.spiking = [L for L in net["layers"] if L["kind"] != "readout"]
+
+    # ------------------------------------------------------------------ lifecycle
+    def close(self):
+        if getattr(self, "ctx", None):
+            lib.skipper_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    def warning(self):
+        msg = lib.skipper_last_error(self.ctx)
+        return msg.decode() if msg else ""
+
+    def _c(self, status):
+        _check(status, self.ctx)
+
+    # ------------------------------------------------------------------ weights
+    def weight_count(self, layer):
+        return lib.skipper_weight_count(self.ctx, layer)
+
+    def set_weights(self, weights):
+        torch = _torch()
+        for i, w in enumerate(weights):
+            t = torch.as_tensor(np.asarray(w, np.float32) if isinstance(w, np.ndarray) else w)
+            t = t.to(device=self.device, dtype=torch.float32).contiguous()
+            if t.numel() != self.weight_count(i):
+                raise ValueError(f"layer {i}: {t.numel()} weights, expected {self.weight_count(i)}")
+            self._c(lib.skipper_set_weights(self.ctx, i, ct.c_void_p(t.data_ptr())))
+            self._keep = t
+        self.stream.synchronize()
+
+    def _per_layer(self, fn):
+        torch = _torch()
+        out = []
+        for i, L in enumerate(self.net["layers"]):
+            shape = (L["cout"], 3, 3, L["cin"]) if L["kind"] == "conv" else (L["cout"], L["cin"])
+            t = torch.empty(shape, dtype=torch.float32, device=self.device)
+            self._c(fn(self.ctx, i, ct.c_void_p(t.data_ptr())))
+            out.append(t)
+        self.stream.synchronize()
+        return out
+
+    def weights(self):
+        return self._per_layer(lib.skipper_get_weights)
+
+    def grads(self):
+        return self._per_layer(lib.skipper_get_grads)
+
+    # ------------------------------------------------------------------ training
+    def step(self, x, y, want_loss=True):
+        loss = ct.c_float(0.0)
+        self._c(lib.skipper_step(self.ctx, ct.c_void_p(x.data_ptr()), ct.c_void_p(y.data_ptr()),
+                                 ct.byref(loss) if want_loss else None))
+        return float(loss.value) if want_loss else None
+
+    def step_host(self, x_host: np.ndarray, y_host: np.ndarray):
+        loss = ct.c_float(0.0)
+        self._c(lib.skipper_step_host(self.ctx, ct.c_void_p(x_host.ctypes.data), ct.c_void_p(y_host.ctypes.data),
+                                      ct.byref(loss)))
+        return float(loss.value)
+
+    def forward_segment(self, seg, pass_, x, y=None):
+        self._c(lib.skipper_forward_segment(self.ctx, seg, pass_, ct.c_void_p(x.data_ptr()),
+                                            ct.c_void_p(y.data_ptr()) if y is not None else None))
+
+    def backward_segment(self, seg):
+        self._c(lib.skipper_backward_segment(self.ctx, seg))
+
+    def optimizer_step(self):
+        self._c(lib.skipper_optimizer_step(self.ctx))
+
+    # ------------------------------------------------------------------ data parallel
+    @staticmethod
+    def comm_unique_id() -> bytes:
+        buf = (ct.c_ubyte * 128)()
+        _check(lib.skipper_comm_unique_id(buf))
+        return bytes(buf)
+
+    def comm_init(self, uid: bytes, rank: int, world: int):
+        buf = (ct.c_ubyte * 128).from_buffer_copy(uid)
+        self._c(lib.skipper_comm_init(self.ctx, buf, rank, world))
+
+    # ------------------------------------------------------------------ introspection
+    def loss(self):
+        v = ct.c_float()
+        self._c(lib.skipper_get_loss(self.ctx, ct.byref(v)))
+        return float(v.value)
+
+    def spike_sums(self):
+        a = np.zeros(self.T, np.int64)
+        self._c(lib.skipper_get_spike_sums(self.ctx, a.ctypes.data))
+        return a
+
+    def keep_mask(self):
+        a = np.zeros(self.T, np.uint8)
+        self._c(lib.skipper_get_keep_mask(self.ctx, a.ctypes.data))
+        return a.astype(bool)
+
+    def sst(self):
+        a = np.zeros(self.C, np.float64)
+        self._c(lib.skipper_get_sst(self.ctx, a.ctypes.data))
+        return a
+
+    def mem_stats(self):
+        cur, peak = ct.c_size_t(), ct.c_size_t()
+        self._c(lib.skipper_mem_stats(self.ctx, ct.byref(cur), ct.byref(peak)))
+        return cur.value, peak.value
+
+    def reset_peak(self):
+        self._c(lib.skipper_reset_peak(self.ctx))
+
+    def debug(self, which, layer):
+        """which: 0 first-pass U, 1 first-pass o, 2 recomputed U, 3 recomputed o -> [T][B][neuron shape]."""
+        torch = _torch()
+        L = self.spiking[layer]
+        shape = (L["h"], L["w"], L["cout"]) if L["kind"] == "conv" else (L["cout"],)
+        dtype = torch.float32 if which in (0, 2) else torch.uint8
+        t = torch.empty((self.T, self.B) + shape, dtype=dtype, device=self.device)
+        self._c(lib.skipper_debug_copy(self.ctx, which, layer, ct.c_void_p(t.data_ptr()),
+                                       t.numel() * t.element_size()))
+        self.stream.synchronize()
+        return t
+
+
+# ---------------------------------------------------------------------- kernel-level entry points
+def _ptr(t):
+    return ct.c_void_p(t.data_ptr())
+
+
+def _stream_handle():
+    return ct.c_void_p(_torch().cuda.current_stream().cuda_stream)
+
+
+def k_fc_fwd(A, B):
+    """C[M][N] = A[M][K] . B[N][K]^T on the tcgen05 path (bf16 in, fp32 out)."""
+    torch = _torch()
+    M, K = A.shape
+    N = B.shape[0]
+    out = torch.empty((M, N), dtype=torch.float32, device=A.device)
+    _check(lib.skipper_k_fc_fwd(_ptr(A), _ptr(B), _ptr(out), M, N, K, _stream_handle()))
+    return out
+
+
+def k_fc_wgrad(D, X, out=None):
+    torch = _torch()
+    M, N = D.shape
+    K = X.shape[1]
+    acc = out is not None
+    if out is None:
+        out = torch.empty((N, K), dtype=torch.float32, device=D.device)
+    _check(lib.skipper_k_fc_wgrad(_ptr(D), _ptr(X), _ptr(out), M, N, K, 1 if acc else 0, _stream_handle()))
+    return out
+
+
+def k_conv_fwd(X, Wk):
+    """X [nb][h][w][cin] bf16, Wk [cout][3][3][cin] bf16 -> Y [nb][h][w][cout] fp32."""
+    torch = _torch()
+    nb, h, w, cin = X.shape
+    cout = Wk.shape[0]
+    out = torch.empty((nb, h, w, cout), dtype=torch.float32, device=X.device)
+    _check(lib.skipper_k_conv_fwd(_ptr(X), _ptr(Wk), _ptr(out), nb, h, w, cin, cout, _stream_handle()))
+    return out
+
+
+def k_conv_dgrad(D, Wt):
+    """D [nb][h][w][cout] bf16, Wt [cin][3][3][cout] bf16 -> G [nb][h][w][cin] fp32."""
+    torch = _torch()
+    nb, h, w, cout = D.shape
+    cin = Wt.shape[0]
+    out = torch.empty((nb, h, w, cin), dtype=torch.float32, device=D.device)
+    _check(lib.skipper_k_conv_dgrad(_ptr(D), _ptr(Wt), _ptr(out), nb, h, w, cin, cout, _stream_handle()))
+    return out
+
+
+def k_conv_wgrad(D, X, out=None):
+    """D [nb][h][w][cout], X [nb][h][w][cin] bf16 -> dW [cout][3][3][cin] fp32."""
+    torch = _torch()
+    nb, h, w, cout = D.shape
+    cin = X.shape[3]
+    acc = out is not None
+    if out is None:
+        out = torch.empty((cout, 3, 3, cin), dtype=torch.float32, device=D.device)
+    _check(lib.skipper_k_conv_wgrad(_ptr(D), _ptr(X), _ptr(out), nb, h, w, cin, cout, 1 if acc else 0,
+                                    _stream_handle()))
+    return out

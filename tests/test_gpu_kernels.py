@@ -1,0 +1,113 @@
+"""Per-kernel parity of the tcgen05/TMA synaptic contractions (K2) against a plain
+PyTorch float64 reference of the same op.  Inputs are exact in bf16; spike-like
+operands with grid weights make every fp32 sum exact, so those cases must match
+bit for bit; random-normal cases are checked to fp32-accumulation tolerance."""
+import pytest
+import torch
+import torch.nn.functional as F
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_micro_singhslsknnd22_b200 as pk  # noqa: F401  (fails loudly if the .so is missing)
+    torch.backends.cuda.matmul.allow_tf32 = False
+    torch.backends.cudnn.allow_tf32 = False
+
+
+def bf16_bits(t):
+    return t.to(torch.bfloat16).view(torch.int16).contiguous()
+
+
+def spikes(shape, rate=0.3, gen=None):
+    return (torch.rand(shape, generator=gen) < rate).float()
+
+
+def grid(shape, e=8, gen=None):
+    return torch.randint(-255, 256, shape, generator=gen).float() * 2.0 ** -e
+
+
+@pytest.mark.parametrize("M,N,K", [(640, 1024, 8192), (100, 128, 784), (37, 24, 40), (300, 264, 136),
+                                   (1, 8, 8), (257, 512, 1024), (129, 64, 64)])
+def test_fc_fwd_exact(M, N, K):
+    from paper_conf_micro_singhslsknnd22_b200 import k_fc_fwd
+    g = torch.Generator().manual_seed(M * 7 + N)
+    A = spikes((M, K), gen=g)
+    B = grid((N, K), gen=g)
+    ref = (A.double() @ B.double().T).float()
+    out = k_fc_fwd(bf16_bits(A).cuda(), bf16_bits(B).cuda()).cpu()
+    assert torch.equal(out, ref), (out - ref).abs().max()
+
+
+def test_fc_fwd_random_normal():
+    from paper_conf_micro_singhslsknnd22_b200 import k_fc_fwd
+    g = torch.Generator().manual_seed(0)
+    A = torch.randn(333, 704, generator=g).bfloat16()
+    B = torch.randn(200, 704, generator=g).bfloat16()
+    ref = A.double() @ B.double().T
+    out = k_fc_fwd(A.view(torch.int16).cuda(), B.view(torch.int16).cuda()).cpu().double()
+    assert (out - ref).norm() / ref.norm() < 1e-6
+
+
+@pytest.mark.parametrize("M,N,K", [(640, 1024, 1024), (80, 128, 784), (37, 24, 40), (1000, 136, 200),
+                                   (4096, 64, 128)])
+def test_fc_wgrad(M, N, K):
+    from paper_conf_micro_singhslsknnd22_b200 import k_fc_wgrad
+    g = torch.Generator().manual_seed(M + K)
+    D = grid((M, N), e=12, gen=g)
+    X = spikes((M, K), gen=g)
+    ref = D.double().T @ X.double()
+    out = k_fc_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda()).cpu().double()
+    assert (out - ref).abs().max() <= 1e-6 * ref.abs().max() + 1e-12
+    # accumulate mode adds into the existing buffer
+    acc = torch.full((N, K), 0.5, device="cuda")
+    k_fc_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda(), out=acc)
+    assert (acc.cpu().double() - 0.5 - ref).abs().max() <= 1e-6 * ref.abs().max() + 1e-6
+
+
+CONV_SHAPES = [(6, 16, 16, 64, 128), (3, 8, 8, 128, 256), (5, 4, 4, 64, 64), (33, 2, 2, 64, 128),
+               (2, 32, 32, 64, 64), (7, 16, 16, 128, 128), (3, 4, 4, 512, 512)]
+
+
+def conv_ref(X, W):  # X [nb][h][w][ci], W [co][3][3][ci]
+    return F.conv2d(X.permute(0, 3, 1, 2).double(), W.permute(0, 3, 1, 2).double(), padding=1).permute(0, 2, 3, 1)
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout", CONV_SHAPES)
+def test_conv_fwd_exact(nb, h, w, cin, cout):
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_fwd
+    g = torch.Generator().manual_seed(nb * h + cin)
+    X = spikes((nb, h, w, cin), gen=g) * 0.25 * torch.randint(0, 5, (nb, h, w, cin), generator=g)  # pooled values
+    W = grid((cout, 3, 3, cin), gen=g)
+    ref = conv_ref(X, W).float()
+    out = k_conv_fwd(bf16_bits(X).cuda(), bf16_bits(W).cuda()).cpu()
+    assert torch.equal(out, ref), (out - ref).abs().max()
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout", CONV_SHAPES)
+def test_conv_dgrad(nb, h, w, cin, cout):
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_dgrad
+    g = torch.Generator().manual_seed(nb * w + cout)
+    D = grid((nb, h, w, cout), e=10, gen=g)
+    W = grid((cout, 3, 3, cin), gen=g)
+    X = torch.zeros((nb, h, w, cin), dtype=torch.float64, requires_grad=True)
+    conv_ref(X, W).backward(D.double())
+    ref = X.grad
+    Wt = W.permute(3, 1, 2, 0).contiguous()  # [cin][3][3][cout]
+    out = k_conv_dgrad(bf16_bits(D).cuda(), bf16_bits(Wt).cuda()).cpu().double()
+    assert (out - ref).abs().max() <= 1e-6 * ref.abs().max() + 1e-12
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout", CONV_SHAPES)
+def test_conv_wgrad(nb, h, w, cin, cout):
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_wgrad
+    g = torch.Generator().manual_seed(nb + h + cout)
+    D = grid((nb, h, w, cout), e=12, gen=g)
+    X = spikes((nb, h, w, cin), gen=g)
+    Wv = torch.zeros((cout, 3, 3, cin), dtype=torch.float64, requires_grad=True)
+    conv_ref(X, Wv).backward(D.double())
+    ref = Wv.grad
+    out = k_conv_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda()).cpu().double()
+    assert (out - ref).abs().max() <= 1e-5 * ref.abs().max() + 1e-12

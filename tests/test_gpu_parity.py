@@ -1,0 +1,160 @@
+"""End-to-end parity of the CUDA training step (through the C ABI) with the CPU
+oracle on the same seeded inputs (SURVEY.md §8(c) tolerances):
+  spikes bit-exact (first pass and recompute), membranes within 1e-5 relative
+  (bit-exact expected under the arithmetic contract), s_t and keep masks exact,
+  weight gradients within 1e-3 (normwise and max-abs), loss within 1e-5,
+  post-Adam weights where the gradient is significant."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import StepConfig, adam_update, train_step
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+
+
+def run_gpu(net, W, x, y, T, C, p, mode, steps=1):
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    B = x.shape[1]
+    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True)
+    m.set_weights(W)
+    xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
+    yd = torch.from_numpy(np.ascontiguousarray(y)).cuda()
+    loss = m.step(xd, yd)
+    return m, loss
+
+
+def grad_ok(g, r, tol=1e-3):
+    g = np.asarray(g, np.float64)
+    r = np.asarray(r, np.float64)
+    nr = np.linalg.norm(r)
+    if nr == 0:
+        return np.abs(g).max() == 0, "zero ref"
+    rel = np.linalg.norm(g - r) / nr
+    mx = np.abs(g - r).max() / np.abs(r).max()
+    return rel <= tol and mx <= tol, f"normwise {rel:.2e} maxabs {mx:.2e}"
+
+
+def check_parity(name, T, B, C, p, mode, lam=None, seed=0):
+    net = synth.net_config(name, lam=lam)
+    W = synth.make_weights(net, seed=seed)
+    x, y = synth.make_inputs(net, T, B, seed=seed + 1)
+    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True))
+    m, loss = run_gpu(net, W, x, y, T, C, p, mode)
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    # SAM and mask (Eq.4, Eq.5)
+    np.testing.assert_array_equal(m.spike_sums(), ref.s)
+    np.testing.assert_array_equal(m.keep_mask(), ref.keep)
+    # first pass and recomputed states per layer
+    for l in range(len(spk)):
+        fo = m.debug(1, l).cpu().numpy()
+        assert np.array_equal(fo, ref.first_o[l]), f"layer {l}: {np.count_nonzero(fo != ref.first_o[l])} first-pass spikes differ"
+        fU = m.debug(0, l).cpu().numpy()
+        np.testing.assert_allclose(fU, ref.first_U[l], rtol=1e-5, atol=1e-6)
+        ro = m.debug(3, l).cpu().numpy()
+        assert np.array_equal(ro, ref.rec_o[l]), f"layer {l}: {np.count_nonzero(ro != ref.rec_o[l])} recomputed spikes differ"
+        rU = m.debug(2, l).cpu().numpy()
+        np.testing.assert_allclose(rU, ref.rec_U[l], rtol=1e-5, atol=1e-6)
+    assert loss == pytest.approx(ref.loss, rel=1e-5)
+    grads = m.grads()
+    for l, (g, r) in enumerate(zip(grads, ref.dW)):
+        ok, msg = grad_ok(g.cpu().numpy(), r)
+        assert ok, f"layer {l} dW: {msg}"
+    # one Adam step from the shared starting point
+    w_new = m.weights()
+    for l, (wn, w0, r) in enumerate(zip(w_new, W, ref.dW)):
+        wr, _, _ = adam_update(w0, r, np.zeros_like(r), np.zeros_like(r), 1)
+        sig = np.abs(r) > 1e-3 * np.abs(r).max()
+        np.testing.assert_allclose(wn.cpu().numpy()[sig], wr[sig], rtol=0, atol=2e-6)
+    return m, ref
+
+
+@pytest.mark.parametrize("mode", ["full", "ckpt", "skip"])
+def test_cfg1_fc784_full_size(mode):
+    """BASELINE.json configs[0]: 784-128-10, T=20, B=4, C=2, p=50."""
+    check_parity("fc784", T=20, B=4, C=2, p=50.0, mode=mode)
+
+
+@pytest.mark.parametrize("mode,lam", [("full", 1.0), ("ckpt", 0.99), ("skip", 0.5), ("skip", 0.99)])
+def test_tiny_fc(mode, lam):
+    check_parity("tiny_fc", T=12, B=3, C=2, p=40.0, mode=mode, lam=lam)
+
+
+@pytest.mark.parametrize("mode,lam", [("full", 0.99), ("ckpt", 1.0), ("skip", 0.99), ("skip", 0.75)])
+def test_tiny_conv(mode, lam):
+    check_parity("tiny_conv", T=12, B=3, C=2, p=50.0, mode=mode, lam=lam)
+
+
+@pytest.mark.parametrize("mode", ["full", "skip"])
+def test_vgg5_reduced(mode):
+    """cfg 2 topology (VGG-5) at reduced T and B: every kernel kind, several tiles, ragged tails."""
+    check_parity("vgg5", T=14, B=2, C=2, p=40.0, mode=mode)
+
+
+def test_skip_p0_equals_ckpt_on_gpu():
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, 12, 2)
+    m1, l1 = run_gpu(net, W, x, y, 12, 2, 0.0, "skip")
+    m2, l2 = run_gpu(net, W, x, y, 12, 2, 0.0, "ckpt")
+    assert l1 == l2 and m1.keep_mask().all()
+    # same schedule; only the order of the split-K fp32 atomic adds in wgrad may differ
+    for a, b in zip(m1.grads(), m2.grads()):
+        a, b = a.double(), b.double()
+        assert (a - b).norm() <= 1e-6 * b.norm() + 1e-12
+
+
+def test_ckpt_equals_full_on_gpu():
+    """Checkpointing reaches the BPTT gradient; same GEMM K-order -> bitwise or ~1e-6."""
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, 12, 2)
+    m1, l1 = run_gpu(net, W, x, y, 12, 2, 0.0, "full")
+    m2, l2 = run_gpu(net, W, x, y, 12, 2, 0.0, "ckpt")
+    assert l1 == l2
+    for a, b in zip(m1.grads(), m2.grads()):
+        a, b = a.double(), b.double()
+        assert (a - b).norm() <= 1e-5 * b.norm() + 1e-12
+
+
+def test_segment_api_order_errors():
+    from paper_conf_micro_singhslsknnd22_b200 import PASS_FIRST, PASS_RECOMPUTE, SkipperError, SkipperNet
+    net = synth.net_config("tiny_fc")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, 12, 2)
+    m = SkipperNet(net, 12, C=2, p=50.0, mode="skip", batch=2)
+    m.set_weights(W)
+    xd, yd = torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda()
+    with pytest.raises(SkipperError, match="EORDER"):
+        m.forward_segment(1, PASS_FIRST, xd)
+    with pytest.raises(SkipperError, match="EORDER"):
+        m.backward_segment(1)
+    m.forward_segment(0, PASS_FIRST, xd)
+    m.forward_segment(1, PASS_FIRST, xd, yd)
+    with pytest.raises(SkipperError, match="EORDER"):
+        m.forward_segment(0, PASS_RECOMPUTE, xd)
+    m.forward_segment(1, PASS_RECOMPUTE, xd)
+    m.backward_segment(1)
+    m.forward_segment(0, PASS_RECOMPUTE, xd)
+    m.backward_segment(0)
+    m.optimizer_step()
+
+
+def test_memory_ordering_full_ckpt_skip():
+    """Peak library memory: FULL > CKPT > SKIP on the same workload (Eq.3, Eq.6)."""
+    net = synth.net_config("vgg5")
+    W = synth.make_weights(net)
+    T, B = 60, 4
+    x, y = synth.make_inputs(net, T, B)
+    peaks = {}
+    for mode, C, p in [("full", 1, 0.0), ("ckpt", 6, 0.0), ("skip", 6, 40.0)]:
+        m, _ = run_gpu(net, W, x, y, T, C, p, mode)
+        peaks[mode] = m.mem_stats()[1]
+        m.close()
+    assert peaks["full"] > peaks["ckpt"] > peaks["skip"], peaks
