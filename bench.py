@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""Benchmark: SNN train samples/s and peak HBM (Skipper vs full BPTT), VGG-CIFAR.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload cfg2_vgg5] [--mode skip]
+    python bench.py --impl reference ...      (the CPU oracle arm)
+
+One step = one full training iteration through the C ABI (skipper_step): first
+forward pass with checkpoints + SAM, loss, SST/keep mask, per-segment recompute
+and backward, gradient allreduce (N>1), Adam.  Inputs resident in HBM; L2 is
+flushed (512 MB write) between timed steps; each step timed with CUDA events on
+the library's stream; max over ranks.  Rank 0 prints one JSON line.
+"""
+from __future__ import annotations
+
+import os
+
+_CORES = len(os.sched_getaffinity(0))
+for _v in ("OMP_NUM_THREADS", "OPENBLAS_NUM_THREADS", "MKL_NUM_THREADS"):
+    os.environ.setdefault(_v, str(_CORES))
+
+import argparse  # noqa: E402
+import json  # noqa: E402
+import statistics  # noqa: E402
+import subprocess  # noqa: E402
+import sys  # noqa: E402
+import tempfile  # noqa: E402
+import time  # noqa: E402
+
+import numpy as np  # noqa: E402
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "SNN train samples/s and peak HBM GB vs T (Skipper vs full BPTT), VGG-CIFAR"
+UNIT = "samples/s"
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d["bf16_tflops_sustained"], "source": "measured"}
+    except Exception:  # noqa: BLE001
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "source": "fallback"}
+
+
+def workload_config(args):
+    wl = synth.workload(args.workload)
+    net = synth.net_config(wl["net"])
+    if args.T:
+        wl["T"] = args.T
+    if args.batch:
+        wl["B"] = args.batch
+    if args.C:
+        wl["C"] = args.C
+    if args.p is not None:
+        wl["p"] = args.p
+    return wl, net
+
+
+def describe(net):
+    parts = []
+    for L in net["layers"]:
+        if L["kind"] == "conv":
+            parts.append(f"conv{L['cin']}-{L['cout']}@{L['h']}" + ("p" if L["pool"] else ""))
+        elif L["kind"] == "fc":
+            parts.append(f"fc{L['cin']}-{L['cout']}")
+        else:
+            parts.append(f"readout{L['cin']}-{L['cout']}")
+    return " ".join(parts)
+
+
+# ------------------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.f = None
+
+    def start(self):
+        try:
+            self.f = tempfile.TemporaryFile(mode="w+")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:  # noqa: BLE001
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:  # noqa: BLE001
+            self.proc.kill()
+        self.f.seek(0)
+        rows = [r.split(",") for r in self.f.read().strip().splitlines() if r.strip()]
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[0]))
+                mx = float(r[1])
+                for nm, v in zip(names, r[4:8]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except (ValueError, IndexError):
+                continue
+        loaded = [v for v in sm if mx and v > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------- oracle arms
+def oracle_samples_per_s(net, wl, mode, B_s, steps, warmup=0):
+    """Time the CPU oracle (as it stands) on a bounded sample: B_s samples, full T."""
+    from oracle import StepConfig, train_step
+    x, y = synth.make_inputs(net, wl["T"], B_s, seed=1)
+    W = synth.make_weights(net)
+    cfg = StepConfig(T=wl["T"], C=wl["C"], p=wl["p"], mode=mode, global_batch=B_s)
+    for _ in range(warmup):
+        train_step(net, W, x, y, cfg)
+    times = []
+    for _ in range(steps):
+        t0 = time.perf_counter()
+        train_step(net, W, x, y, cfg)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    return B_s * steps / tot, 1000.0 * tot / steps
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl, net = workload_config(args)
+    B_s = args.ref_batch
+    val, ms = oracle_samples_per_s(net, wl, args.mode, B_s, args.steps, args.warmup)
+    sample = f"B={B_s} of {wl['B']} per step, full T={wl['T']}, C={wl['C']}, p={wl['p']}, mode={args.mode}"
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32 forward / f64 backward", "data": "synthetic",
+        "config": config_block(args, wl, net),
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": _CORES, "kind": "oracle", "sample": sample},
+        "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def config_block(args, wl, net):
+    return {"workload": args.workload, "net": describe(net), "T": wl["T"], "per_gpu_batch": wl["B"],
+            "global_batch": wl["B"] * args.gpus, "C": wl["C"], "p": wl["p"], "mode": args.mode,
+            "parallelism": f"dp{args.gpus}", "l2": "flushed between timed steps (512 MB write)",
+            "inputs": "Poisson rate-coded CIFAR-shaped frames, seeded; grid-quantised random weights"}
+
+
+# ------------------------------------------------------------------------------------- GPU arm
+def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=False, e2e=False):
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    T, B, C, p = wl["T"], wl["B"], wl["C"], wl["p"]
+    x, y = synth.make_inputs(net, T, B, seed=1 + 1000 * rank)
+    W = synth.make_weights(net)
+    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, global_batch=B * world)
+    m.set_weights(W)
+    if world > 1:
+        obj = [m.comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        m.comm_init(obj[0], rank, world)
+    xd = torch.from_numpy(x).cuda()
+    yd = torch.from_numpy(y).cuda()
+    flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device="cuda")
+    for _ in range(args.warmup):
+        m.step(xd, yd, want_loss=False)
+    torch.cuda.synchronize()
+    m.reset_peak()
+    torch.cuda.reset_peak_memory_stats()
+    if profile:
+        m.profile(True)
+    clocks = ClockSampler(local_rank)
+    clocks.start() if profile else None
+    launches0 = m.launch_count()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    evs = []
+    for _ in range(args.steps):
+        flush.zero_()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        m.step(xd, yd, want_loss=False)
+        b.record(stream)
+        evs.append((a, b))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop() if profile else None
+    ms_list = [a.elapsed_time(b) for a, b in evs]
+    tot = torch.tensor([sum(ms_list)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    total_ms = float(tot.item())
+    launches = m.launch_count() - launches0
+    prof = m.profile_read() if profile else None
+    peak_lib = m.mem_stats()[1]
+    peak_torch = torch.cuda.max_memory_allocated()
+    loss = m.loss()
+    res = {"total_ms": total_ms, "ms_list": ms_list, "launches": launches, "prof": prof, "clocks": clk,
+           "peak_lib": peak_lib, "peak_torch": peak_torch, "loss": loss,
+           "kept_fraction": float(m.keep_mask().mean())}
+    if e2e:
+        xh = torch.from_numpy(x).pin_memory()
+        yh = torch.from_numpy(y).pin_memory()
+        xn, yn = xh.numpy(), yh.numpy()
+        for _ in range(2):
+            m.step_host(xn, yn)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        ts = []
+        for _ in range(args.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            m.step_host(xn, yn)       # H2D of x/labels, the step, D2H of s_t and the loss
+            b.record(stream)
+            ts.append((a, b))
+        torch.cuda.synchronize()
+        e2e_ms = torch.tensor([sum(a.elapsed_time(b) for a, b in ts)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(e2e_ms, op=dist.ReduceOp.MAX)
+        res["e2e_ms"] = float(e2e_ms.item())
+        res["h2d"] = int(x.nbytes + y.nbytes)
+        res["d2h"] = int(4 + 8 * T)
+    m.close()
+    del flush
+    torch.cuda.empty_cache()
+    return res
+
+
+def roofline(prof, peaks, steps):
+    """Dominant kernel class of the step and its achieved fraction of the B200 roofline."""
+    total = sum(v["ms"] for v in prof.values()) or 1.0
+    breakdown = {}
+    ridge = peaks["bf16_tflops_sustained"] * 1e12 / (peaks["hbm_gbs"] * 1e9)
+    for k, v in prof.items():
+        if v["launches"] == 0:
+            continue
+        per_ms = v["ms"] / v["launches"]
+        gbs = v["bytes"] / v["launches"] / (per_ms * 1e-3) / 1e9
+        tfs = v["flops"] / v["launches"] / (per_ms * 1e-3) / 1e12 if v["flops"] else 0.0
+        tensor = k.startswith("gemm") and v["flops"] / max(v["bytes"], 1) > ridge
+        breakdown[k] = {"ms_per_step": v["ms"] / steps, "share": v["ms"] / total, "launches_per_step": v["launches"] / steps,
+                        "GB/s": gbs, "TFLOP/s": tfs,
+                        "frac": (tfs / peaks["bf16_tflops_sustained"]) if tensor else (gbs / peaks["hbm_gbs"]),
+                        "bound": "tensor" if tensor else "hbm"}
+    dom = max(breakdown, key=lambda k: breakdown[k]["ms_per_step"])
+    d = breakdown[dom]
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tf):
+        try:
+            traffic = json.load(open(tf)).get(dom)
+        except Exception:  # noqa: BLE001
+            traffic = None
+    if d["bound"] == "tensor":
+        rf = {"bound": "tensor", "achieved": d["TFLOP/s"], "peak": peaks["bf16_tflops_sustained"], "unit": "TFLOP/s",
+              "frac": d["frac"], "traffic": traffic, "kernel": dom}
+    else:
+        rf = {"bound": "hbm", "achieved": d["GB/s"], "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": d["frac"],
+              "traffic": traffic, "kernel": dom}
+    rf["peak_source"] = peaks["source"] + (" (sustained bf16)" if d["bound"] == "tensor" else " (copy bandwidth)")
+    return rf, breakdown
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus != world and world > 1:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    import __graft_entry__
+    if rank == 0 and not os.path.exists(os.path.join(ROOT, "paper_conf_micro_singhslsknnd22_b200", "libskipper.so")):
+        __graft_entry__.build()
+    if world > 1:
+        dist.barrier()
+    wl, net = workload_config(args)
+    peaks = load_peaks()
+    main = run_mode(torch, dist, args, wl, net, args.mode, rank, world, local_rank, profile=True, e2e=True)
+    compare = {}
+    if not args.no_compare:
+        for mode in ("full", "ckpt"):
+            if mode == args.mode:
+                continue
+            try:
+                r = run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank)
+                compare[mode] = {"samples_per_s": wl["B"] * world * args.steps / (r["total_ms"] / 1e3),
+                                 "ms_per_step": r["total_ms"] / args.steps, "peak_hbm_gb": r["peak_lib"] / 1e9}
+            except Exception as e:  # noqa: BLE001
+                compare[mode] = {"error": str(e)[:200]}
+    if rank != 0:
+        if world > 1:
+            dist.barrier()
+            dist.destroy_process_group()
+        return
+    gb = wl["B"] * world
+    value = gb * args.steps / (main["total_ms"] / 1e3)
+    rf, breakdown = roofline(main["prof"], peaks, args.steps)
+    cfg = config_block(args, wl, net)
+    cfg["peak_hbm_gb"] = main["peak_lib"] / 1e9
+    cfg["peak_torch_allocated_gb"] = main["peak_torch"] / 1e9
+    cfg["kept_fraction"] = main["kept_fraction"]
+    cfg["compare"] = compare
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": main["total_ms"] / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic", "config": cfg,
+        "roofline": rf,
+        "e2e": {"value": gb * args.steps / (main["e2e_ms"] / 1e3), "unit": UNIT,
+                "h2d_bytes_per_step": main["h2d"] * world, "d2h_bytes_per_step": main["d2h"] * world},
+        "gpu_launches": main["launches"],
+        "clocks": main["clocks"],
+        "kernels": breakdown,
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        B_s = 2
+        val, ms = oracle_samples_per_s(net, wl, args.mode, B_s, 1)
+        line["cpu_baseline"] = {"value": val, "unit": UNIT, "cores": _CORES, "kind": "oracle",
+                                "sample": f"1 step, B={B_s} of {wl['B']}, full T={wl['T']}, C={wl['C']}, p={wl['p']}, "
+                                          f"mode={args.mode} ({ms / 1e3:.1f} s)"}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="cfg2_vgg5")
+    ap.add_argument("--mode", default="skip", choices=["skip", "ckpt", "full"])
+    ap.add_argument("--T", type=int, default=0)
+    ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--C", type=int, default=0)
+    ap.add_argument("--p", type=float, default=None)
+    ap.add_argument("--ref-batch", type=int, default=1)
+    ap.add_argument("--no-compare", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -164,6 +164,20 @@ skipper_status skipper_reset_peak(skipper_ctx *ctx);
  * N_l is the un-pooled neuron count of spiking layer `layer` (0-based). */
 skipper_status skipper_debug_copy(skipper_ctx *ctx, int which, int layer, void *dst_dev, size_t bytes);
 
+/* ---- profiling (bench / roofline) --------------------------------------------
+ * enable != 0: every kernel launch of the context is bracketed by CUDA events on
+ * the context stream and attributed to a kernel class, with its algorithmic HBM
+ * bytes and FLOPs.  Counters reset on every call.
+ * profile_read synchronises the stream (host sync) and returns the totals of one
+ * class since the last reset.  Classes are numbered 0..skipper_profile_num_classes()-1. */
+skipper_status skipper_profile(skipper_ctx *ctx, int enable);
+skipper_status skipper_profile_read(skipper_ctx *ctx, int cls, long long *launches, double *ms, double *bytes,
+                                    double *flops);
+const char *skipper_profile_class_name(int cls);
+int skipper_profile_num_classes(void);
+/* Kernel launches issued by this context since creation (always counted). */
+long long skipper_launch_count(const skipper_ctx *ctx);
+
 /* Pure host functions (no GPU needed). */
 /* Eq.5 for one segment: p-th percentile of n int64 values, numpy 'linear' method. */
 double skipper_sst_host(const long long *s, int n, double p);

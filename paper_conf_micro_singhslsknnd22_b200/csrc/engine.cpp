@@ -27,7 +27,7 @@ thread_local std::string g_last_error;
 
 struct Layer {
     skipper_layer d{};
-    bool fc = false, conv = false, pool = false, direct = false, readout = false;
+    bool fc = false, conv = false, pool = false, readout = false;
     int H = 1, W = 1, Cin = 0, Cout = 0, PH = 1, PW = 1;
     long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
     size_t wcount = 0;
@@ -37,6 +37,9 @@ struct Layer {
     uint8_t *o_run = nullptr, *cko = nullptr;
     uint16_t *Po = nullptr;    // arena rows
     float *Useg = nullptr;     // arena rows
+    int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
+    uint16_t *wbp = nullptr;   // layer 0 im2col: bf16 weights zero-padded to [cout][K0]
+    float *dwp = nullptr;      // layer 0 im2col: padded weight gradient
     float *dbg[2] = {nullptr, nullptr};     // first / recompute U
     uint8_t *dbgo[2] = {nullptr, nullptr};  // first / recompute o
 };
@@ -54,12 +57,12 @@ struct skipper_ctx {
     cudaStream_t st = nullptr;
     int T = 0, C = 1, S = 0, B = 0, Bg = 0;
     int num_sms = 148;
-    bool input_direct = false;  // first layer is the fused direct conv
+    int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
+    int K0 = 0;                 // im2col width (32 or 64)
     int in_h = 1, in_w = 1, in_c = 0;
-    long long in_elems = 0;     // per sample
+    long long in_elems = 0;     // input elements per sample (uint8 x)
+    long long in_row = 0;       // staged bf16 layer-0 operand elements per sample
     // persistent
-    uint32_t *xmask = nullptr;
-    uint16_t *xb = nullptr;
     unsigned *s_part = nullptr;
     long long *s_dev = nullptr;
     float *cnt = nullptr, *cnt_kept = nullptr, *z = nullptr, *dz = nullptr, *loss_dev = nullptr, *g_last = nullptr;
@@ -81,7 +84,7 @@ struct skipper_ctx {
     float *I_buf = nullptr;     // currents (fwd) and gradients wrt spikes (dgrad)
     uint16_t *d_buf = nullptr;  // delta (bf16)
     uint16_t *P2[2] = {nullptr, nullptr};
-    uint16_t *xg = nullptr;     // gathered fc-first input rows
+    uint16_t *xg = nullptr;     // staged layer-0 operand rows of the current pass
     // schedule state
     int phase = PH_IDLE;
     int next_seg = 0;
@@ -106,12 +109,11 @@ struct skipper_ctx {
 };
 
 enum KClass {
-    K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_DIRECT_FWD, K_READOUT, K_SCAN_BWD, K_DIRECT_BWD,
-    K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_GATHER, K_NCLASS
+    K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
+    K_NCLASS
 };
-static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "direct_conv_lif_fwd",
-                                               "readout_loss", "lif_bwd_scan", "direct_conv_bwd_wgrad",
-                                               "gemm_wgrad", "gemm_dgrad", "adam", "gather"};
+static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
+                                               "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -301,6 +303,16 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
         c->in_c = f.Cin;
     }
     c->in_elems = (long long)c->in_h * c->in_w * c->in_c;
+    c->in_row = c->in_elems;
+    if (f.conv) {
+        if (9 * f.Cin <= 64 && f.Cin % 64) {  // narrow input (RGB, DVS polarity): 3x3 im2col, K0 columns
+            c->in_kind = 1;
+            c->K0 = 9 * f.Cin <= 32 ? 32 : 64;
+            c->in_row = (long long)f.H * f.W * c->K0;
+        } else {
+            c->in_kind = 2;
+        }
+    }
     for (int i = 1; i < n; ++i) {
         const Layer &p = c->L[i - 1];
         const Layer &l = c->L[i];
@@ -315,10 +327,8 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
     // kernel support per layer
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
-        if (l.conv && i == 0 && 9 * l.Cin <= 32) {
-            l.direct = true;
-            if (256 % l.Cout) return fail(c, SKIPPER_EUNSUPPORTED, "layer 0: direct conv needs cout | 256");
-            c->input_direct = true;
+        if (l.conv && i == 0 && c->in_kind == 1) {
+            if (l.Cout % 8) return fail(c, SKIPPER_EUNSUPPORTED, "layer 0: cout %% 8 == 0");
             continue;
         }
         if (l.conv) {
@@ -358,10 +368,23 @@ static long long max_n(const skipper_ctx *c) {
 static long long max_gemm_io(const skipper_ctx *c) {  // fp32 I (fwd) and g (dgrad) per sample-row
     long long m = 0;
     for (int i = 0; i < c->Ls; ++i) {
-        if (!c->L[i].direct) m = std::max(m, c->L[i].N);
-        if (i > 0) m = std::max(m, c->L[i].Nin);
+        m = std::max(m, c->L[i].N * c->L[i].fsplit);
+        if (i > 0) m = std::max(m, c->L[i].Nin * c->L[i].dsplit);
     }
     return std::max(m, 4LL);
+}
+
+// Split-K for fc GEMMs whose output has too few 128 x BN tiles to fill the SMs (M = S*B rows is
+// small).  Fixed per layer from the first-pass shape so the recompute reduces in the same order.
+static int fc_splits(int M, int N, int K, int num_sms) {
+    const int bn = N <= 64 ? 64 : (N <= 128 ? 128 : 256);
+    const long long tiles = (long long)((M + 127) / 128) * ((N + bn - 1) / bn);
+    const int kb = (K + 63) / 64;
+    if (tiles >= num_sms || kb < 8) return 1;
+    int s = (int)((num_sms + tiles - 1) / tiles);
+    s = std::min(s, 8);
+    s = std::min(s, kb / 4);
+    return std::max(s, 1);
 }
 
 extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_layers, const skipper_config *cfg,
@@ -409,6 +432,13 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     c->S = c->T / c->C;
     c->num_sms = sk::device_num_sms();
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        if (!l.fc) continue;
+        const int rowsM = c->S * c->B;
+        l.fsplit = fc_splits(rowsM, l.Cout, l.Cin, c->num_sms);
+        if (i > 0) l.dsplit = fc_splits(rowsM, l.Cin, l.Cout, c->num_sms);
+    }
 
     // ---- persistent allocations
     c->dw_total = 0;
@@ -429,7 +459,11 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         l.dw = c->dw_all + off;
         off += l.wcount;
         if (!l.readout) {
-            if (i > 0 && !l.direct) AL(l.wt, l.wcount);
+            if (i > 0) AL(l.wt, l.wcount);
+            if (i == 0 && c->in_kind == 1) {
+                AL(l.wbp, (size_t)l.Cout * c->K0);
+                AL(l.dwp, (size_t)l.Cout * c->K0);
+            }
             const size_t bn = (size_t)c->B * l.N;
             AL(l.U_run, bn);
             AL(l.o_run, bn);
@@ -446,10 +480,6 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
             }
         }
     }
-    if (c->input_direct)
-        AL(c->xmask, (size_t)c->T * c->B * c->in_h * c->in_w);
-    else
-        AL(c->xb, (size_t)c->T * c->B * c->in_elems);
     AL(c->s_part, (size_t)c->T * 32);
     AL(c->s_dev, (size_t)c->T);
     const Layer &last = c->L[c->Ls - 1];
@@ -490,6 +520,8 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         dev_free(c, l.v, l.wcount * 4);
         dev_free(c, l.wb, l.wcount * 2);
         dev_free(c, l.wt, l.wcount * 2);
+        dev_free(c, l.wbp, (size_t)l.Cout * c->K0 * 2);
+        dev_free(c, l.dwp, (size_t)l.Cout * c->K0 * 4);
         if (!l.readout) {
             const size_t bn = (size_t)c->B * l.N;
             dev_free(c, l.U_run, bn * 4);
@@ -507,8 +539,6 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
     if (!c->L.empty() && c->Ls > 0) {
         const Layer &last = c->L[c->Ls - 1];
         const Layer &ro = c->L.back();
-        dev_free(c, c->xmask, (size_t)c->T * c->B * c->in_h * c->in_w * 4);
-        dev_free(c, c->xb, (size_t)c->T * c->B * c->in_elems * 2);
         dev_free(c, c->s_part, (size_t)c->T * 32 * 4);
         dev_free(c, c->s_dev, (size_t)c->T * 8);
         dev_free(c, c->cnt, (size_t)c->B * last.Nout * 4);
@@ -560,6 +590,7 @@ static skipper_status check_ctx(skipper_ctx *c) {
 static skipper_status refresh_shadows(skipper_ctx *c, int i) {
     Layer &l = c->L[i];
     CK(sk::launch_cast_bf16(l.w, l.wb, l.wcount, c->st));
+    if (l.wbp) CK(sk::launch_cast_pad_bf16(l.w, l.wbp, l.Cout, (int)(l.wcount / l.Cout), c->K0, c->st));
     if (l.wt) {
         if (l.conv)  // wt[ci][tap][co] = wb[co][tap][ci]
             CK(sk::launch_transpose_bf16(l.wb, l.wt, l.Cout, 9, l.Cin, c->st));
@@ -619,13 +650,15 @@ static skipper_status arena_first(skipper_ctx *c) {
     const size_t rowsB = (size_t)c->S * c->B;
     const size_t pbytes = al256(rowsB * max_nout(c) * 2);
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
-    c->arena_bytes = 2 * pbytes + ibytes;
+    const size_t xbytes = al256(rowsB * c->in_row * 2);
+    c->arena_bytes = 2 * pbytes + ibytes + xbytes;
     c->arena = dev_alloc(c, c->arena_bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "first-pass arena of %zu bytes", c->arena_bytes);
     char *p = static_cast<char *>(c->arena);
     c->P2[0] = reinterpret_cast<uint16_t *>(p);
     c->P2[1] = reinterpret_cast<uint16_t *>(p + pbytes);
     c->I_buf = reinterpret_cast<float *>(p + 2 * pbytes);
+    c->xg = reinterpret_cast<uint16_t *>(p + 2 * pbytes + ibytes);
     return SKIPPER_OK;
 }
 
@@ -636,7 +669,7 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     for (int i = 0; i < c->Ls; ++i) bytes += al256(rowsB * c->L[i].Nout * 2) + al256(rowsB * c->L[i].N * 4);
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t dbytes = al256(rowsB * max_n(c) * 2);
-    const size_t xbytes = c->input_direct ? 0 : al256(rowsB * c->in_elems * 2);
+    const size_t xbytes = al256(rowsB * c->in_row * 2);
     bytes += ibytes + dbytes + xbytes;
     c->arena_bytes = bytes;
     c->arena = dev_alloc(c, bytes);
@@ -653,7 +686,7 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     p += ibytes;
     c->d_buf = reinterpret_cast<uint16_t *>(p);
     p += dbytes;
-    if (xbytes) c->xg = reinterpret_cast<uint16_t *>(p);
+    c->xg = reinterpret_cast<uint16_t *>(p);
     return SKIPPER_OK;
 }
 
@@ -673,12 +706,15 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     sk::GemmLaunch g;
     const int nb = rows * c->B;
     bool ok;
-    if (l.conv)
+    if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
+        ok = sk::plan_fc(&g, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0);
+    else if (l.conv)
         ok = sk::plan_conv(&g, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
     else
-        ok = sk::plan_fc(&g, in, l.wb, I, nb, l.Cout, l.Cin);
+        ok = sk::plan_fc(&g, in, l.wb, I, nb, l.Cout, l.Cin, l.fsplit);
+    if (ok && g.d.splits != (l.fc ? l.fsplit : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
     const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
-    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4;
+    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4 * l.fsplit;
     return run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, bytes, 2.0 * M * l.Cout * K);
 }
 
@@ -702,16 +738,7 @@ static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
                 CKS(zero_dev(c, l.dbgo[k], bn * c->T));
             }
     }
-    {
-        const double xbytes = (double)c->T * c->B * c->in_elems;
-        if (c->input_direct) {
-            ProfScope ps(c, K_STAGE, xbytes + (double)c->T * c->B * c->in_h * c->in_w * 4, 0);
-            CK(sk::launch_stage_bits(x, c->xmask, c->s_part, c->T, c->B, c->in_h, c->in_w, c->in_c, c->st));
-        } else {
-            ProfScope ps(c, K_STAGE, xbytes * 3, 0);
-            CK(sk::launch_stage_bf16(x, c->xb, c->s_part, c->T, c->B, (int)c->in_elems, c->st));
-        }
-    }
+    if (c->L[0].dwp) CKS(zero_dev(c, c->L[0].dwp, (size_t)c->L[0].Cout * c->K0 * 4));
     c->x_cur = x;
     c->grads_ready = false;
     return SKIPPER_OK;
@@ -732,27 +759,39 @@ static double scan_bwd_bytes(const skipper_ctx *c, const Layer &l, const sk::Sca
     double b = rows * bn * 4;                                         // U
     b += a.g_broadcast ? bno * 4 : rows * bno * 4;                    // g (pooled resolution when pooled)
     if (a.delta) b += rows * bn * 2;                                  // delta (bf16)
-    if (a.xmask) b += rows * (double)c->B * l.H * l.W * 4 + (double)l.wcount * 4;
     b += bn * 8;                                                      // carry in/out
     return b;
 }
 
+// Layer-0 operand rows for R timesteps (t0 + r, or the device list `rows`) into c->xg.
+static skipper_status stage_input(skipper_ctx *c, const int *rows, int t0, int R, bool sam) {
+    const int kind = c->in_kind == 1 ? 1 : 0;
+    const double bytes = (double)R * c->B * (c->in_elems + c->in_row * 2);
+    ProfScope ps(c, K_STAGE, bytes, 0);
+    CK(sk::launch_stage_rows(c->x_cur, c->xg, rows, t0, R, c->B, c->in_h, c->in_w, c->in_c, kind, c->K0,
+                             c->in_elems, sam ? c->s_part : nullptr, c->st));
+    return SKIPPER_OK;
+}
+
 // Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
 static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
+    CKS(stage_input(c, nullptr, t0, R, true));
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in;
         uint16_t *out;
         if (record) {
-            in = i == 0 ? (c->xb ? c->xb : nullptr) : c->L[i - 1].Po;
+            in = i == 0 ? c->xg : c->L[i - 1].Po;
             out = l.Po;
         } else {
-            in = i == 0 ? (c->xb ? c->xb + (size_t)t0 * c->B * c->in_elems : nullptr) : c->P2[(i - 1) & 1];
+            in = i == 0 ? c->xg : c->P2[(i - 1) & 1];
             out = c->P2[i & 1];
         }
-        if (!l.direct) CKS(gemm_forward(c, i, in, c->I_buf, R));
+        CKS(gemm_forward(c, i, in, c->I_buf, R));
         sk::ScanFwdArgs a{};
-        a.I = l.direct ? nullptr : c->I_buf;
+        a.I = c->I_buf;
+        a.nsplit = l.fsplit;
+        a.split_stride = (long long)R * c->B * l.N;
         a.R = R;
         a.restore = 0;
         a.U_state = l.U_run;
@@ -774,13 +813,8 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         a.pool = l.pool ? 1 : 0;
         a.lam = l.d.lambda;
         a.theta = l.d.theta;
-        if (l.direct) {
-            a.xmask = c->xmask;
-            a.w_direct = l.wb;
-            a.kbits = 9 * l.Cin;
-        }
         {
-            ProfScope ps(c, l.direct ? K_DIRECT_FWD : K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
+            ProfScope ps(c, K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
             CK(sk::launch_lif_fwd(a, c->st));
         }
     }
@@ -834,18 +868,17 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
 static skipper_status recompute_segment(skipper_ctx *c, int seg) {
     const int R = (int)c->kept[seg].size();
     const int *row_t = c->kept_dev + (size_t)seg * c->S;
-    if (!c->input_direct) {
-        ProfScope ps(c, K_GATHER, 4.0 * R * c->B * c->in_elems, 0);
-        CK(sk::launch_gather_rows(c->xb, c->xg, row_t, R, (size_t)c->B * c->in_elems, c->st));
-    }
+    CKS(stage_input(c, row_t, 0, R, false));
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in = i == 0 ? c->xg : c->L[i - 1].Po;
-        const size_t in_row = (size_t)c->B * (i == 0 ? c->in_elems : c->L[i - 1].Nout);
-        if (!l.direct && R > 1)  // rows 1..R-1 (row 0 is the checkpoint)
+        const size_t in_row = (size_t)c->B * (i == 0 ? c->in_row : c->L[i - 1].Nout);
+        if (R > 1)  // rows 1..R-1 (row 0 is the checkpoint)
             CKS(gemm_forward(c, i, in + in_row, c->I_buf + (size_t)c->B * l.N, R - 1));
         sk::ScanFwdArgs a{};
-        a.I = l.direct ? nullptr : c->I_buf;
+        a.I = c->I_buf;
+        a.nsplit = l.fsplit;
+        a.split_stride = (long long)(R - 1) * c->B * l.N;  // the GEMM covered rows 1..R-1
         a.R = R;
         a.restore = 1;
         a.U_state = l.ckU + (size_t)seg * c->B * l.N;
@@ -864,13 +897,8 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
         a.pool = l.pool ? 1 : 0;
         a.lam = l.d.lambda;
         a.theta = l.d.theta;
-        if (l.direct) {
-            a.xmask = c->xmask;
-            a.w_direct = l.wb;
-            a.kbits = 9 * l.Cin;
-        }
         {
-            ProfScope ps(c, l.direct ? K_DIRECT_FWD : K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
+            ProfScope ps(c, K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
             CK(sk::launch_lif_fwd(a, c->st));
         }
     }
@@ -883,11 +911,13 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         Layer &l = c->L[i];
         sk::ScanBwdArgs a{};
         a.g = (i == c->Ls - 1) ? c->g_last : c->I_buf;
+        a.nsplit = (i == c->Ls - 1) ? 1 : c->L[i + 1].dsplit;  // dgrad of layer i+1 produced g
+        a.split_stride = (long long)R * c->B * l.Nout;
         a.g_broadcast = (i == c->Ls - 1) ? 1 : 0;
         a.g_pooled = l.pool ? 1 : 0;
         a.U = l.Useg;
         a.carry = l.carry;
-        a.delta = l.direct ? nullptr : c->d_buf;
+        a.delta = c->d_buf;
         a.R = R;
         a.B = c->B;
         a.H = l.H;
@@ -898,22 +928,17 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         a.theta = l.d.theta;
         a.surr = c->cfg.surrogate;
         a.gamma = c->cfg.surr_gamma;
-        if (l.direct) {
-            a.xmask = c->xmask;
-            a.row_t = row_t;
-            a.dW_direct = l.dw;
-            a.kbits = 9 * l.Cin;
-        }
         {
-            ProfScope ps(c, l.direct ? K_DIRECT_BWD : K_SCAN_BWD, scan_bwd_bytes(c, l, a), 0);
+            ProfScope ps(c, K_SCAN_BWD, scan_bwd_bytes(c, l, a), 0);
             CK(sk::launch_lif_bwd(a, c->st));
         }
-        if (l.direct) continue;
         const int nb = R * c->B;
-        const uint16_t *X = i == 0 ? (c->xg ? c->xg : c->xb) : c->L[i - 1].Po;
+        const uint16_t *X = i == 0 ? c->xg : c->L[i - 1].Po;
         sk::GemmLaunch g;
         bool ok;
-        if (l.conv)
+        if (i == 0 && c->in_kind == 1)
+            ok = sk::plan_fc_wgrad(&g, c->d_buf, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
+        else if (l.conv)
             ok = sk::plan_conv_wgrad(&g, c->d_buf, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
         else
             ok = sk::plan_fc_wgrad(&g, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
@@ -926,9 +951,9 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             if (l.conv)
                 ok = sk::plan_conv(&g, c->d_buf, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
             else
-                ok = sk::plan_fc(&g, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout);
+                ok = sk::plan_fc(&g, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, l.dsplit);
             const double M = (double)nb * l.H * l.W, K = (double)l.Cout * (l.conv ? 9 : 1);
-            const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4;
+            const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4 * l.dsplit;
             CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * (l.Nin / (l.H * l.W)) * K));
         }
     }
@@ -995,11 +1020,16 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
     const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
     const int R = full ? c->T : (int)c->kept[seg].size();
     const int *row_t = full ? nullptr : c->kept_dev + (size_t)seg * c->S;
-    if (full) c->xg = nullptr;  // layer-0 fc wgrad reads the staged input directly
     CKS(backward_rows(c, R, row_t));
     if (seg == 0) {
         const Layer &last = c->L[c->Ls - 1];
         const Layer &ro = c->L.back();
+        Layer &l0 = c->L[0];
+        if (l0.dwp) {  // padded im2col weight gradient -> [cout][9*cin]
+            const int cols = (int)(l0.wcount / l0.Cout);
+            ProfScope ps(c, K_UNPAD, (double)l0.Cout * (c->K0 + cols) * 4, 0);
+            CK(sk::launch_unpad_f32(l0.dwp, l0.dw, l0.Cout, cols, c->K0, c->st));
+        }
         ProfScope ps(c, K_READOUT, (double)c->B * (last.Nout + ro.Cout) * 4 + (double)ro.wcount * 4,
                      2.0 * c->B * last.Nout * ro.Cout);
         CK(sk::launch_readout_wgrad(c->dz, full ? c->cnt : c->cnt_kept, ro.dw, c->B, (int)last.Nout, ro.Cout,
@@ -1038,6 +1068,10 @@ extern "C" skipper_status skipper_optimizer_step(skipper_ctx *c) {
             ProfScope ps(c, K_ADAM, (double)l.wcount * 26, 0);
             CK(sk::launch_adam(l.w, l.dw, l.m, l.v, l.wb, l.wcount, c->cfg.lr, c->cfg.beta1, c->cfg.beta2, c->cfg.eps,
                                bc1, bc2s, c->st));
+        }
+        if (l.wbp) {
+            ProfScope ps(c, K_ADAM, (double)l.wcount * 6, 0);
+            CK(sk::launch_cast_pad_bf16(l.w, l.wbp, l.Cout, (int)(l.wcount / l.Cout), c->K0, c->st));
         }
         if (l.wt) {
             ProfScope ps(c, K_ADAM, (double)l.wcount * 4, 0);

@@ -17,7 +17,10 @@ enum OperandKind {
     OP_MNCONV = 3,  // MN-major shifted NHWC image (wgrad input operand), boxes {64, W, bh, bn}
 };
 
-enum StoreMode { STORE_OVERWRITE = 0, STORE_ATOMIC_ADD = 1 };
+// OVERWRITE: plain store; ATOMIC_ADD: TMA reduce-add (split-K wgrad, accumulation over segments);
+// SPLIT: split s stores its partial sum into slice s of [splits][M][N] (summed in fixed order by the
+// consuming scan - deterministic split-K for the forward / dgrad GEMMs).
+enum StoreMode { STORE_OVERWRITE = 0, STORE_ATOMIC_ADD = 1, STORE_SPLIT = 2 };
 
 // Passed by value to the kernel.
 struct GemmDev {
@@ -36,7 +39,7 @@ struct GemmDev {
 
 struct GemmLaunch {
     GemmDev d;
-    CUtensorMap ta, tb;
+    CUtensorMap ta, tb, tc;  // operands A, B and the fp32 output
     int bn;             // 64, 128 or 256
     int mn_major;       // 0: both operands K-major; 1: both MN-major (wgrad)
 };
@@ -49,7 +52,7 @@ bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint
 
 // Plans (return false on unsupported geometry).  All pointers are device pointers.
 // C[M][N] = A[M][K] . B[N][K]^T
-bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K);
+bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K, int splits = 1);
 // dW[N][K] (+)= D[M][N]^T . X[M][K]   (reduction over the M rows)
 bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms);
 // conv forward / dgrad: Y[nb,h,w,cout] from X[nb,h,w,cin] and Wk[cout][9][cin];

@@ -5,7 +5,8 @@
 //   warp 1      MMA issuer    (one thread: tcgen05.mma.cta_group::1.kind::f16, M=128, N=BN, K=16,
 //                              accumulators in TMEM, tcgen05.commit frees smem stages)
 //               + TMEM allocator (2 accumulator buffers so the epilogue of tile i overlaps tile i+1)
-//   warps 2-5   epilogue      (tcgen05.ld 32x32b -> registers -> fp32 store or red.add into global)
+//   warps 2-5   epilogue      (tcgen05.ld 32x32b -> registers -> 128B-swizzled smem -> TMA store, or
+//                              TMA reduce-add for split-K weight gradients)
 // Operands are bf16 (exact for spikes and grid weights), accumulation fp32.
 // Convolutions are implicit GEMMs: each K block is one 3x3 tap x 64 channels, loaded by a 4D TMA
 // box shifted by the tap offset; the zero padding is TMA's out-of-bounds fill.
@@ -28,7 +29,8 @@ struct GemmCfg {
     static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
     static constexpr int STAGES = (BN == 64) ? 8 : (BN == 128 ? 6 : 4);
     static constexpr uint32_t TMEM_COLS = (2 * BN <= 128) ? 128 : (2 * BN <= 256 ? 256 : 512);
-    static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+    static constexpr uint32_t EPI_BYTES = 4 * 2 * 4096;  // 4 epilogue warps x 2 buffers x (32 x 32 fp32)
+    static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + EPI_BYTES + 1024 /*align*/ + 256 /*barriers*/;
 };
 
 struct TileCoord {
@@ -50,13 +52,15 @@ SK_DEV TileCoord decode_tile(const GemmDev &g, int tile) {
 
 template <int BN, int MN>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const GemmDev g) {
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
+                   const __grid_constant__ CUtensorMap tcm, const GemmDev g) {
     using Cfg = GemmCfg<BN>;
     constexpr int STAGES = Cfg::STAGES;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023u) & ~1023u;
-    const uint32_t bars = base + STAGES * Cfg::STAGE_BYTES;
+    const uint32_t epi = base + STAGES * Cfg::STAGE_BYTES;  // 1024-aligned (stage bytes are multiples of 1 KB)
+    const uint32_t bars = epi + Cfg::EPI_BYTES;
     auto full_bar = [&](int s) { return bars + 8u * s; };
     auto empty_bar = [&](int s) { return bars + 8u * (STAGES + s); };
     auto tfull_bar = [&](int a) { return bars + 8u * (2 * STAGES + a); };
@@ -70,6 +74,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     if (warp == 0 && lane == 0) {
         tma_prefetch(&ta);
         tma_prefetch(&tb);
+        tma_prefetch(&tcm);
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(full_bar(s), 1);
             mbar_init(empty_bar(s), 1);
@@ -181,38 +186,44 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         }
     } else {
         // ---------------------------------------------------------------- epilogue
+        // Each warp owns TMEM lanes [32q, 32q+32) = 32 output rows.  Per 32-column chunk: TMEM ->
+        // registers -> a 4 KB smem box in the 128B-swizzle pattern (16-byte chunk j of row r at
+        // position j ^ (r & 7): conflict-free) -> one TMA store (or reduce-add) per box; two boxes
+        // per warp in flight.  TMA clips rows >= M and columns >= N.
         const int q = warp & 3;  // TMEM lane quadrant this warp may access
-        const int row = q * 32 + lane;
+        const uint32_t ebuf0 = epi + (uint32_t)q * 8192u;
         int acc = 0;
         uint32_t acc_phase = 0;
+        uint32_t nbox = 0;
         for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
             const TileCoord tc = decode_tile(g, tile);
             mbar_wait(tfull_bar(acc), acc_phase);
             tc_fence_after();
-            const int grow = tc.m_t * BM + row;
-            const bool row_ok = grow < g.M;
-            float *crow = g.C + (long long)grow * g.ldc + (long long)tc.tap * g.cols_per_tap;
+            const int row0 = tc.m_t * BM + q * 32;
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 uint32_t r[32];
                 tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c * 32, r);
                 tmem_ld_wait();
-                const int col0 = tc.n_t * BN + c * 32;
-                if (row_ok) {
+                const uint32_t buf = ebuf0 + (nbox & 1u) * 4096u;
+                if (lane == 0) bulk_wait_read<1>();  // the box that used `buf` two stores ago has been read
+                __syncwarp();
+                uint8_t *rowp = smem_raw + (buf - raw) + lane * 128;
 #pragma unroll
-                    for (int j = 0; j < 8; ++j) {
-                        const int col = col0 + 4 * j;
-                        if (col < g.N) {
-                            float *p = crow + col;
-                            const float a = __uint_as_float(r[4 * j]), b = __uint_as_float(r[4 * j + 1]);
-                            const float cc = __uint_as_float(r[4 * j + 2]), d = __uint_as_float(r[4 * j + 3]);
-                            if (g.store_mode == STORE_ATOMIC_ADD)
-                                red_add_v4(p, a, b, cc, d);
-                            else
-                                *reinterpret_cast<float4 *>(p) = make_float4(a, b, cc, d);
-                        }
-                    }
+                for (int j = 0; j < 8; ++j)
+                    *reinterpret_cast<uint4 *>(rowp + ((j ^ (lane & 7)) << 4)) =
+                        make_uint4(r[4 * j], r[4 * j + 1], r[4 * j + 2], r[4 * j + 3]);
+                fence_async_shared();
+                __syncwarp();
+                if (lane == 0) {
+                    const int col0 = tc.n_t * BN + c * 32;
+                    if (g.store_mode == STORE_ATOMIC_ADD)
+                        tma_reduce_add_3d(&tcm, buf, col0, tc.tap, row0);
+                    else
+                        tma_store_3d(&tcm, buf, col0, g.store_mode == STORE_SPLIT ? tc.split : tc.tap, row0);
+                    bulk_commit();
                 }
+                ++nbox;
             }
             tc_fence_before();
             __syncwarp();
@@ -220,6 +231,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             acc ^= 1;
             if (acc == 0) acc_phase ^= 1u;
         }
+        if (lane == 0) bulk_wait<0>();
     }
     tc_fence_before();
     __syncthreads();
@@ -260,6 +272,21 @@ bool make_map_2d(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// fp32 output viewed as [rows][taps][cols] (row pitch ldc, tap pitch tap_pitch floats), box 32 x 1 x 32.
+static bool make_map_out(CUtensorMap *m, float *ptr, uint64_t cols, uint64_t taps, uint64_t rows, uint64_t tap_pitch,
+                         uint64_t ldc) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    if ((ldc * 4) % 16 || (tap_pitch * 4) % 16 || (reinterpret_cast<uintptr_t>(ptr) & 15)) return false;
+    cuuint64_t dims[3] = {cols, taps, rows};
+    cuuint64_t strides[2] = {tap_pitch * 4, ldc * 4};
+    cuuint32_t box[3] = {32, 1, 32};
+    cuuint32_t es[3] = {1, 1, 1};
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, ptr, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+              CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint64_t H, uint64_t NB,
                    uint32_t box_w, uint32_t box_h, uint32_t box_n) {
     auto fn = encode_fn();
@@ -291,7 +318,7 @@ static bool conv_box(int h, int w, int rows, uint32_t *bw, uint32_t *bh, uint32_
     return *bn <= 256;
 }
 
-bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K) {
+bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K, int splits) {
     if (M <= 0 || N <= 0 || K <= 0 || N % 4 || K % 8) return false;
     GemmDev &d = g->d;
     d = GemmDev{};
@@ -302,16 +329,21 @@ bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N
     d.taps = 1;
     d.splits = 1;
     d.num_kb = cdiv(K, BK);
-    d.kb_per_split = d.num_kb;
+    if (splits < 1) splits = 1;
+    if (splits > d.num_kb) splits = d.num_kb;
+    d.kb_per_split = cdiv(d.num_kb, splits);
+    d.splits = cdiv(d.num_kb, d.kb_per_split);
     d.a_kind = OP_K2D;
     d.b_kind = OP_K2D;
     d.C = C;
     d.ldc = N;
     d.M = M;
     d.N = N;
-    d.store_mode = STORE_OVERWRITE;
+    d.store_mode = d.splits > 1 ? STORE_SPLIT : STORE_OVERWRITE;
     d.cols_per_tap = 0;
-    return make_map_2d(&g->ta, A, K, M, BK, BM) && make_map_2d(&g->tb, B, K, N, BK, g->bn);
+    // output viewed as [M][splits][N]: slice s at C + s*M*N
+    return make_map_2d(&g->ta, A, K, M, BK, BM) && make_map_2d(&g->tb, B, K, N, BK, g->bn) &&
+           make_map_out(&g->tc, C, N, d.splits, M, (uint64_t)M * N, N);
 }
 
 static void choose_splits(GemmDev &d, int base_tiles, int num_sms) {
@@ -342,7 +374,8 @@ bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M
     d.M = N;
     d.N = K;
     d.store_mode = STORE_ATOMIC_ADD;
-    return make_map_2d(&g->ta, D, N, M, 64, BK) && make_map_2d(&g->tb, X, K, M, 64, BK);
+    return make_map_2d(&g->ta, D, N, M, 64, BK) && make_map_2d(&g->tb, X, K, M, 64, BK) &&
+           make_map_out(&g->tc, dW, K, 1, N, K, K);
 }
 
 bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
@@ -374,7 +407,8 @@ bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, i
     d.M = (int)M;
     d.N = cout;
     d.store_mode = STORE_OVERWRITE;
-    return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn);
+    return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn) &&
+           make_map_out(&g->tc, Y, cout, 1, M, cout, cout);
 }
 
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
@@ -403,7 +437,8 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     d.M = cout;
     d.N = cin;
     d.store_mode = STORE_ATOMIC_ADD;
-    return make_map_2d(&g->ta, D, cout, M, 64, BK) && make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn);
+    return make_map_2d(&g->ta, D, cout, M, 64, BK) && make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn) &&
+           make_map_out(&g->tc, dW, cin, 9, cout, cin, 9ull * cin);
 }
 
 template <int BN, int MN>
@@ -418,7 +453,7 @@ static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sm
     }
     const int total = g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
     const int grid = total < num_sms ? total : num_sms;
-    gemm_tc_kernel<BN, MN><<<grid, NUM_THREADS, Cfg::SMEM_BYTES, stream>>>(g.ta, g.tb, g.d);
+    gemm_tc_kernel<BN, MN><<<grid, NUM_THREADS, Cfg::SMEM_BYTES, stream>>>(g.ta, g.tb, g.tc, g.d);
     return cudaGetLastError();
 }
 

@@ -11,7 +11,9 @@ enum { SURR_TRIANGLE = 0, SURR_FAST_SIGMOID = 1 };
 // K1: forward LIF temporal scan over the rows (timesteps) of one segment, Eq.1.
 // Neuron layout NHWC per row: row r holds B*H*W*C neurons (fc: H = W = 1).
 struct ScanFwdArgs {
-    const float *I;        // currents [R][B*N] (null for the direct conv kernel)
+    const float *I;        // currents [R][B*N]
+    int nsplit;            // I is the fixed-order sum of nsplit partial slices (deterministic split-K)
+    long long split_stride;  // floats between partial slices
     int R;                 // rows in the segment buffer
     int restore;           // RECOMPUTE: row 0 is the checkpoint (U_state/o_state), rows 1.. recomputed
     float *U_state;        // FIRST/RECORD: running U [B*N] (in/out); RECOMPUTE: checkpoint U (in)
@@ -28,16 +30,14 @@ struct ScanFwdArgs {
     uint8_t *dbg_o;
     int B, H, W, C, pool;
     float lam, theta;
-    // direct conv (first layer, Cin*9 <= 32): input bit masks [T][B*H*W], weights bf16 [C][9*Cin]
-    const uint32_t *xmask;
-    const uint16_t *w_direct;
-    int kbits;             // 9*Cin
 };
 cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s);
 
 // K4: reverse surrogate-gradient scan, Eq.2: delta_t = sigma'(U_t) g_t + lam delta_{next}.
 struct ScanBwdArgs {
     const float *g;        // gradient wrt the layer's output spikes
+    int nsplit;            // g = sum of nsplit partial slices, split_stride floats apart
+    long long split_stride;
     int g_pooled;          // g is at pooled resolution (x 0.25 spread, pool2^T)
     int g_broadcast;       // g is [B*Nout] for every row (readout gradient, same at each t)
     const float *U;        // [R][B*N]
@@ -48,21 +48,17 @@ struct ScanBwdArgs {
     float lam, theta;
     int surr;
     float gamma;
-    // direct conv: fused weight gradient dW[C][kbits] += sum delta_bf16 * input bit
-    const uint32_t *xmask;
-    const int *row_t;
-    float *dW_direct;
-    int kbits;
 };
 cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s);
 
-// Input staging (once per step): SAM term l = 0 (Eq.4) and the first layer's operand.
-cudaError_t launch_stage_bits(const uint8_t *x, uint32_t *xmask, unsigned *s_part, int T, int B, int H, int W,
-                              int C0, cudaStream_t s);
-cudaError_t launch_stage_bf16(const uint8_t *x, uint16_t *xb, unsigned *s_part, int T, int B, int D,
-                              cudaStream_t s);
-cudaError_t launch_gather_rows(const uint16_t *src, uint16_t *dst, const int *rows, int R, size_t row_elems,
-                               cudaStream_t s);
+// Layer-0 operand rows of one segment straight from the uint8 input x [T][B][...]:
+// kind 0: bf16 copy of x[t] (D = elements per sample); kind 1: 3x3/pad-1 im2col of an
+// H x W x C0 image zero-padded to K0 columns.  rows: device list of t (or null -> t0 + r).
+// s_part != null adds the SAM term l = 0 (Eq.4).
+cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, int t0, int R, int B, int H, int W,
+                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s);
+cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s);
+cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);
 
 // Readout integrator + softmax cross-entropy (reading 5) and its gradients.

@@ -1,5 +1,5 @@
-// lif_kernels.cu - K1 (forward LIF scan), K4 (reverse surrogate scan), the fused direct first-layer
-// conv kernels, input staging / SAM, readout + loss, Adam.  sm_100a CUDA cores; HBM-bound streams.
+// lif_kernels.cu - K1 (forward LIF scan), K4 (reverse surrogate scan), layer-0 input staging / SAM,
+// readout + loss, Adam.  sm_100a CUDA cores; HBM-bound streams.
 //
 // Eq.1:  U_t = lam*U_{t-1} + W o^{l-1}_t - theta*o^l_{t-1};  o_t = [U_t > theta]
 //   evaluated without FMA in the order ((lam*U) + I) - theta*o so that spikes are bit-identical to
@@ -33,12 +33,27 @@ SK_DEV uint2 pack_bf16x4(float a, float b, float c, float d) {
 
 SK_DEV float4 ldg4(const float *p) { return __ldg(reinterpret_cast<const float4 *>(p)); }
 
+// Sum of the split-K partial slices in fixed order s = 0, 1, ... (deterministic, identical in the
+// first pass and the recompute because the split count is a per-layer constant).
+SK_DEV float4 ldg4_split(const float *p, int nsplit, long long stride) {
+    float4 v = ldg4(p);
+    for (int s = 1; s < nsplit; ++s) {
+        const float4 w = ldg4(p + s * stride);
+        v.x = __fadd_rn(v.x, w.x);
+        v.y = __fadd_rn(v.y, w.y);
+        v.z = __fadd_rn(v.z, w.z);
+        v.w = __fadd_rn(v.w, w.w);
+    }
+    return v;
+}
+
 // ============================================================================ K1 forward scan
-// One thread owns 4 consecutive channels of NP pixels (NP = 4 for a 2x2 pooled window).
-template <int POOL, int DIRECT, int CH>
+// One thread owns 4 consecutive channels of NP pixels (NP = 4 for a 2x2 pooled window).  The
+// currents of CH rows are loaded before the recurrence runs over them (loads do not depend on
+// the recurrence), which keeps CH x NP 16-byte loads in flight per thread.
+template <int POOL, int CH>
 __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
     constexpr int NP = POOL ? 4 : 1;
-    extern __shared__ float ws[];  // DIRECT: fp32 copy of bf16 weights, [kbits][C]
     __shared__ unsigned red[8][CH];
     const int C = a.C;
     const int C4 = C >> 2;
@@ -48,12 +63,10 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
     const bool active = p < P;
     const long long rs = (long long)a.B * HW * C;  // neurons per row
     const long long ors = POOL ? rs / 4 : rs;       // outputs per row
-    const long long npix_row = (long long)a.B * HW;
 
-    long long nidx[NP], pix[NP], oidx = 0;
-    int c4 = 0;
+    long long nidx[NP], oidx = 0;
     if (active) {
-        c4 = (int)(p % C4);
+        const int c4 = (int)(p % C4);
         long long rest = p / C4;
         if (POOL) {
             const int PW = a.W / 2, PH = a.H / 2;
@@ -64,25 +77,16 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
 #pragma unroll
             for (int k = 0; k < NP; ++k) {
                 const int y = 2 * py + (k >> 1), x = 2 * px + (k & 1);
-                pix[k] = (b * a.H + y) * a.W + x;
-                nidx[k] = pix[k] * C + 4 * c4;
+                nidx[k] = ((b * a.H + y) * a.W + x) * C + 4 * c4;
             }
             oidx = ((b * PH + py) * PW + px) * C + 4 * c4;
         } else {
-            pix[0] = rest;
             nidx[0] = rest * C + 4 * c4;
             oidx = nidx[0];
         }
     } else {
 #pragma unroll
-        for (int k = 0; k < NP; ++k) nidx[k] = pix[k] = 0;
-    }
-    if (DIRECT) {
-        for (int i = threadIdx.x; i < a.kbits * C; i += blockDim.x) {
-            const int k = i / C, c = i % C;
-            ws[k * C + c] = bf_bits2f(a.w_direct[c * a.kbits + k]);
-        }
-        __syncthreads();
+        for (int k = 0; k < NP; ++k) nidx[k] = 0;
     }
 
     float U[NP][4], O[NP][4];
@@ -137,24 +141,13 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
     const int nwarps = blockDim.x >> 5;
     for (int rb = r0; rb < a.R; rb += CH) {
         float4 Iv[CH][NP];
-        uint32_t mk[CH][NP];
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb + j;
 #pragma unroll
-            for (int k = 0; k < NP; ++k) {
-                if (active && r < a.R) {
-                    if (DIRECT) {
-                        const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
-                        mk[j][k] = __ldg(a.xmask + t * npix_row + pix[k]);
-                    } else {
-                        Iv[j][k] = ldg4(a.I + (long long)r * rs + nidx[k]);
-                    }
-                } else {
-                    mk[j][k] = 0;
-                    Iv[j][k] = make_float4(0.f, 0.f, 0.f, 0.f);
-                }
-            }
+            for (int k = 0; k < NP; ++k)
+                Iv[j][k] = (active && r < a.R) ? ldg4_split(a.I + (long long)r * rs + nidx[k], a.nsplit, a.split_stride)
+                                               : make_float4(0.f, 0.f, 0.f, 0.f);
         }
         unsigned nspk[CH];
 #pragma unroll
@@ -164,20 +157,7 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
             if (active && r < a.R) {
 #pragma unroll
                 for (int k = 0; k < NP; ++k) {
-                    float4 Ik;
-                    if (DIRECT) {
-                        Ik = make_float4(0.f, 0.f, 0.f, 0.f);
-                        const uint32_t m = mk[j][k];
-                        for (int kb = 0; kb < a.kbits; ++kb) {
-                            if ((m >> kb) & 1u) {
-                                const float4 w = *reinterpret_cast<const float4 *>(&ws[kb * C + 4 * c4]);
-                                Ik.x += w.x; Ik.y += w.y; Ik.z += w.z; Ik.w += w.w;
-                            }
-                        }
-                    } else {
-                        Ik = Iv[j][k];
-                    }
-                    const float Ii[4] = {Ik.x, Ik.y, Ik.z, Ik.w};
+                    const float Ii[4] = {Iv[j][k].x, Iv[j][k].y, Iv[j][k].z, Iv[j][k].w};
 #pragma unroll
                     for (int i = 0; i < 4; ++i) {
                         U[k][i] = lif_update(U[k][i], Ii[i], O[k][i], a.lam, a.theta);
@@ -238,15 +218,10 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     const int threads = 256;
     const long long blocks = (P + threads - 1) / threads;
     if (blocks == 0) return cudaSuccess;
-    const bool direct = a.xmask != nullptr;
-    const size_t smem = direct ? (size_t)a.kbits * a.C * sizeof(float) : 0;
-    if (a.pool) {
-        if (direct) lif_fwd_kernel<1, 1, 4><<<(unsigned)blocks, threads, smem, s>>>(a);
-        else lif_fwd_kernel<1, 0, 4><<<(unsigned)blocks, threads, smem, s>>>(a);
-    } else {
-        if (direct) lif_fwd_kernel<0, 1, 8><<<(unsigned)blocks, threads, smem, s>>>(a);
-        else lif_fwd_kernel<0, 0, 8><<<(unsigned)blocks, threads, smem, s>>>(a);
-    }
+    if (a.pool)
+        lif_fwd_kernel<1, 4><<<(unsigned)blocks, threads, 0, s>>>(a);
+    else
+        lif_fwd_kernel<0, 8><<<(unsigned)blocks, threads, 0, s>>>(a);
     return cudaGetLastError();
 }
 
@@ -279,7 +254,7 @@ __global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
             if (r >= 0) {
-                gv[j] = ldg4(a.g + (long long)r * grs + gi);
+                gv[j] = ldg4_split(a.g + (long long)r * grs + gi, a.nsplit, a.split_stride);
                 uv[j] = ldg4(a.U + (long long)r * rs + n0);
             }
         }
@@ -299,191 +274,117 @@ __global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
     *reinterpret_cast<float4 *>(a.carry + n0) = d;
 }
 
-// Direct first layer: reverse scan fused with its weight gradient (the input is a 27-bit mask per
-// pixel, so dW[c][k] += bf16(delta) wherever input bit k is set).  One thread per (pixel, channel);
-// the mask is warp-uniform for C >= 32, so the per-bit branches do not diverge.
-template <int CH>
-__global__ void __launch_bounds__(256) lif_bwd_direct_kernel(const ScanBwdArgs a) {
-    __shared__ float red[256 * 32];
-    const int C = a.C;
-    const int c = threadIdx.x % C;
-    const int slot = threadIdx.x / C;
-    const int spb = blockDim.x / C;
-    const long long HW = (long long)a.H * a.W;
-    const long long npix = (long long)a.B * HW;
-    const long long rs = npix * C;
-    const float gs = a.g_pooled ? 0.25f : 1.0f;
-    float acc[32];
-#pragma unroll
-    for (int k = 0; k < 32; ++k) acc[k] = 0.f;
-    for (long long pixel = (long long)blockIdx.x * spb + slot; pixel < npix; pixel += (long long)gridDim.x * spb) {
-        const long long n = pixel * C + c;
-        long long gi = n, grs = rs;
-        if (a.g_pooled) {
-            const int x = (int)(pixel % a.W);
-            const int y = (int)((pixel / a.W) % a.H);
-            const long long b = pixel / HW;
-            gi = ((b * (a.H / 2) + y / 2) * (a.W / 2) + x / 2) * C + c;
-            grs = rs / 4;
-        }
-        if (a.g_broadcast) grs = 0;
-        float d = a.carry[n];
-        for (int rb = a.R - 1; rb >= 0; rb -= CH) {
-            float gv[CH], uv[CH];
-            uint32_t mk[CH];
-#pragma unroll
-            for (int j = 0; j < CH; ++j) {
-                const int r = rb - j;
-                if (r >= 0) {
-                    gv[j] = __ldg(a.g + (long long)r * grs + gi);
-                    uv[j] = __ldg(a.U + (long long)r * rs + n);
-                    const long long t = a.row_t ? a.row_t[r] : r;
-                    mk[j] = __ldg(a.xmask + t * npix + pixel);
-                } else {
-                    gv[j] = uv[j] = 0.f;
-                    mk[j] = 0;
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < CH; ++j) {
-                const int r = rb - j;
-                if (r >= 0) {
-                    d = surrogate(uv[j], a.theta, a.surr, a.gamma) * (gs * gv[j]) + a.lam * d;
-                    const float db = bf_bits2f(f2bf_bits(d));
-                    if (a.delta) a.delta[(long long)r * rs + n] = f2bf_bits(d);
-                    const uint32_t m = mk[j];
-#pragma unroll
-                    for (int k = 0; k < 32; ++k)
-                        if ((m >> k) & 1u) acc[k] += db;
-                }
-            }
-        }
-        a.carry[n] = d;
-    }
-#pragma unroll
-    for (int k = 0; k < 32; ++k) red[threadIdx.x * 32 + k] = acc[k];
-    __syncthreads();
-    for (int i = threadIdx.x; i < C * a.kbits; i += blockDim.x) {
-        const int cc = i / a.kbits, k = i % a.kbits;
-        float sum = 0.f;
-        for (int sl = 0; sl < spb; ++sl) sum += red[(sl * C + cc) * 32 + k];
-        if (sum != 0.f) atomicAdd(a.dW_direct + (long long)cc * a.kbits + k, sum);
-    }
-}
-
 cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     if (rs == 0 || a.R == 0) return cudaSuccess;
-    if (a.xmask) {
-        if (256 % a.C || a.kbits > 32) return cudaErrorInvalidValue;
-        int sms = 148;
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const long long npix = (long long)a.B * a.H * a.W;
-        const int spb = 256 / a.C;
-        long long blocks = (npix + spb - 1) / spb;
-        const long long cap = 4LL * sms;
-        if (blocks > cap) blocks = cap;
-        lif_bwd_direct_kernel<4><<<(unsigned)blocks, 256, 0, s>>>(a);
-    } else {
-        const long long P = rs / 4;
-        lif_bwd_kernel<8><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
-    }
+    const long long P = rs / 4;
+    lif_bwd_kernel<8><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 
 // ============================================================================ input staging / SAM
-SK_DEV void sam_add(unsigned *s_part, long long t, unsigned v) {
-    // warp-aggregate when the whole warp is in the same timestep
-    const unsigned mask = 0xffffffffu;
-    const long long t0 = __shfl_sync(mask, t, 0);
-    const bool same = __all_sync(mask, t == t0);
-    if (same) {
-        const unsigned tot = __reduce_add_sync(mask, v);
-        if ((threadIdx.x & 31) == 0 && tot) atomicAdd(s_part + t0 * 32 + (blockIdx.x & 31), tot);
-    } else if (v) {
-        atomicAdd(s_part + t * 32 + (blockIdx.x & 31), v);
-    }
-}
-
-__global__ void stage_bits_kernel(const uint8_t *__restrict__ x, uint32_t *__restrict__ xmask, unsigned *s_part,
-                                  int T, int B, int H, int W, int C0) {
-    const long long total = (long long)T * B * H * W;
+// Layer-0 operand rows for the timesteps of one segment (FIRST: t0 + r; RECOMPUTE: the kept list),
+// straight from the uint8 input.  kind 0: bf16 copy of x[t] (fc or conv-with-wide-Cin input);
+// kind 1: im2col of a 3x3 / pad-1 window, k = (dy*3+dx)*C0 + ci, zero-padded to K0 columns.
+// SAM term l = 0 (Eq.4) is counted when s_part is given (FIRST pass only).
+__global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__restrict__ dst, const int *rows, int t0,
+                                  int R, int B, int H, int W, int C0, int kind, int K0, long long D,
+                                  unsigned *s_part) {
+    const long long per_row = kind == 1 ? (long long)B * H * W : (long long)B * D;
+    const long long total = (long long)R * per_row;
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    const bool ok = i < total;
-    long long t = 0;
+    long long t = -1;
     unsigned cnt = 0;
-    if (ok) {
-        const int xx = (int)(i % W);
-        const int yy = (int)((i / W) % H);
-        const long long tb = i / ((long long)H * W);  // t*B + b
-        t = tb / B;
-        uint32_t m = 0;
-        for (int dy = 0; dy < 3; ++dy) {
-            const int y = yy + dy - 1;
-            if (y < 0 || y >= H) continue;
-            for (int dx = 0; dx < 3; ++dx) {
-                const int xq = xx + dx - 1;
-                if (xq < 0 || xq >= W) continue;
-                const uint8_t *px = x + ((tb * H + y) * W + xq) * C0;
-                for (int ci = 0; ci < C0; ++ci)
-                    if (px[ci]) m |= 1u << ((dy * 3 + dx) * C0 + ci);
-            }
-        }
-        xmask[i] = m;
-        const uint8_t *pc = x + i * C0;
-        for (int ci = 0; ci < C0; ++ci) cnt += pc[ci] ? 1u : 0u;
-    } else {
-        t = (long long)T - 1;
-    }
-    sam_add(s_part, t, cnt);
-}
-
-cudaError_t launch_stage_bits(const uint8_t *x, uint32_t *xmask, unsigned *s_part, int T, int B, int H, int W,
-                              int C0, cudaStream_t s) {
-    const long long total = (long long)T * B * H * W;
-    stage_bits_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, xmask, s_part, T, B, H, W, C0);
-    return cudaGetLastError();
-}
-
-__global__ void stage_bf16_kernel(const uint8_t *__restrict__ x, uint16_t *__restrict__ xb, unsigned *s_part, int T,
-                                  int B, int D) {
-    const long long total = (long long)T * B * D;
-    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    long long t = (long long)T - 1;
-    unsigned v = 0;
     if (i < total) {
-        v = x[i] ? 1u : 0u;
-        xb[i] = v ? (uint16_t)0x3F80 : (uint16_t)0;
-        t = i / ((long long)B * D);
+        const int r = (int)(i / per_row);
+        const long long e = i % per_row;
+        t = rows ? rows[r] : t0 + r;
+        if (kind == 1) {
+            const int xx = (int)(e % W);
+            const int yy = (int)((e / W) % H);
+            const long long b = e / ((long long)H * W);
+            const uint8_t *xt = x + (t * B + b) * (long long)H * W * C0;
+            uint16_t col[64];
+#pragma unroll
+            for (int k = 0; k < 64; ++k) col[k] = 0;
+            for (int dy = 0; dy < 3; ++dy) {
+                const int y = yy + dy - 1;
+                if (y < 0 || y >= H) continue;
+                for (int dx = 0; dx < 3; ++dx) {
+                    const int xq = xx + dx - 1;
+                    if (xq < 0 || xq >= W) continue;
+                    const uint8_t *px = xt + ((long long)y * W + xq) * C0;
+                    for (int ci = 0; ci < C0; ++ci)
+                        if (px[ci]) col[(dy * 3 + dx) * C0 + ci] = 0x3F80;
+                }
+            }
+            const uint8_t *pc = xt + ((long long)yy * W + xx) * C0;
+            for (int ci = 0; ci < C0; ++ci) cnt += pc[ci] ? 1u : 0u;
+            uint4 *o = reinterpret_cast<uint4 *>(dst + i * K0);
+            for (int q = 0; q < K0 / 8; ++q) {
+                uint4 v;
+                v.x = col[8 * q] | ((uint32_t)col[8 * q + 1] << 16);
+                v.y = col[8 * q + 2] | ((uint32_t)col[8 * q + 3] << 16);
+                v.z = col[8 * q + 4] | ((uint32_t)col[8 * q + 5] << 16);
+                v.w = col[8 * q + 6] | ((uint32_t)col[8 * q + 7] << 16);
+                o[q] = v;
+            }
+        } else {
+            const uint8_t v = x[t * (long long)B * D + e];
+            dst[i] = v ? (uint16_t)0x3F80 : (uint16_t)0;
+            cnt = v ? 1u : 0u;
+        }
     }
-    sam_add(s_part, t, v);
+    if (s_part) {
+        const unsigned mask = 0xffffffffu;
+        const long long tl = __shfl_sync(mask, t, 0);
+        const bool same = __all_sync(mask, t == tl || t < 0);
+        if (same) {
+            const unsigned tot = __reduce_add_sync(mask, cnt);
+            if ((threadIdx.x & 31) == 0 && tot && tl >= 0) atomicAdd(s_part + tl * 32 + (blockIdx.x & 31), tot);
+        } else if (cnt) {
+            atomicAdd(s_part + t * 32 + (blockIdx.x & 31), cnt);
+        }
+    }
 }
 
-cudaError_t launch_stage_bf16(const uint8_t *x, uint16_t *xb, unsigned *s_part, int T, int B, int D, cudaStream_t s) {
-    const long long total = (long long)T * B * D;
-    stage_bf16_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, xb, s_part, T, B, D);
+cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, int t0, int R, int B, int H, int W,
+                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s) {
+    const long long per_row = kind == 1 ? (long long)B * H * W : (long long)B * D;
+    const long long total = (long long)R * per_row;
+    if (total == 0) return cudaSuccess;
+    if (kind == 1 && (K0 % 8 || K0 > 64 || 9 * C0 > K0)) return cudaErrorInvalidValue;
+    stage_rows_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, dst, rows, t0, R, B, H, W, C0, kind, K0, D,
+                                                                     s_part);
     return cudaGetLastError();
 }
 
-__global__ void gather_rows_kernel(const uint16_t *__restrict__ src, uint16_t *__restrict__ dst, const int *rows, int R,
-                                   long long row_elems) {
-    const long long total = (long long)R * row_elems;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-        const long long r = i / row_elems, e = i % row_elems;
-        dst[i] = src[(long long)rows[r] * row_elems + e];
-    }
+// dst[r][c] = bf16(src[r][c]) for c < cols, 0 for cols <= c < ld   (layer-0 weights padded to K0)
+__global__ void cast_pad_bf16_kernel(const float *src, uint16_t *dst, int rows, int cols, int ld) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (long long)rows * ld) return;
+    const int r = (int)(i / ld), c = (int)(i % ld);
+    dst[i] = c < cols ? f2bf_bits(src[(long long)r * cols + c]) : (uint16_t)0;
 }
 
-cudaError_t launch_gather_rows(const uint16_t *src, uint16_t *dst, const int *rows, int R, size_t row_elems,
-                               cudaStream_t s) {
-    const long long total = (long long)R * (long long)row_elems;
-    if (total == 0) return cudaSuccess;
-    long long blocks = (total + 255) / 256;
-    if (blocks > 65535) blocks = 65535;
-    gather_rows_kernel<<<(unsigned)blocks, 256, 0, s>>>(src, dst, rows, R, (long long)row_elems);
+cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s) {
+    const long long n = (long long)rows * ld;
+    cast_pad_bf16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(src, dst, rows, cols, ld);
+    return cudaGetLastError();
+}
+
+// dst[r][c] = src[r][c] for c < cols  (padded weight gradient back to [rows][cols])
+__global__ void unpad_f32_kernel(const float *src, float *dst, int rows, int cols, int ld) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (long long)rows * cols) return;
+    const int r = (int)(i / cols), c = (int)(i % cols);
+    dst[i] = src[(long long)r * ld + c];
+}
+
+cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s) {
+    const long long n = (long long)rows * cols;
+    unpad_f32_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(src, dst, rows, cols, ld);
     return cudaGetLastError();
 }
 

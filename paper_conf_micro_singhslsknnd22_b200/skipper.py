@@ -50,6 +50,9 @@ class Allocator(ct.Structure):
 
 
 def _load():
+    # Load torch first so that libskipper.so binds to the same libcudart.so.12 instance as torch
+    # (one CUDA runtime per process: shared default-stream semantics, one error state).
+    import torch  # noqa: F401
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
                           "(python -m paper_conf_micro_singhslsknnd22_b200.build)")
@@ -87,6 +90,11 @@ def _load():
         "skipper_k_conv_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_wgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
         "skipper_k_num_sms": (I, []),
+        "skipper_profile": (I, [P, I]),
+        "skipper_profile_read": (I, [P, I, P, P, P, P]),
+        "skipper_profile_class_name": (ct.c_char_p, [I]),
+        "skipper_profile_num_classes": (I, []),
+        "skipper_launch_count": (ct.c_longlong, [P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -233,7 +241,16 @@ class SkipperNet:
         return self._per_layer(lib.skipper_get_grads)
 
     # ------------------------------------------------------------------ training
+    def _check_inputs(self, x, y=None):
+        torch = _torch()
+        if x.dtype != torch.uint8 or not x.is_cuda or not x.is_contiguous() or x.shape[0] != self.T \
+                or x.shape[1] != self.B:
+            raise ValueError(f"x must be a contiguous CUDA uint8 tensor [T={self.T}][B={self.B}][...]")
+        if y is not None and (y.dtype != torch.int32 or not y.is_cuda or y.numel() != self.B):
+            raise ValueError(f"labels must be a CUDA int32 tensor of {self.B} elements")
+
     def step(self, x, y, want_loss=True):
+        self._check_inputs(x, y)
         loss = ct.c_float(0.0)
         self._c(lib.skipper_step(self.ctx, ct.c_void_p(x.data_ptr()), ct.c_void_p(y.data_ptr()),
                                  ct.byref(loss) if want_loss else None))
@@ -295,6 +312,22 @@ class SkipperNet:
     def reset_peak(self):
         self._c(lib.skipper_reset_peak(self.ctx))
 
+    def profile(self, enable=True):
+        self._c(lib.skipper_profile(self.ctx, 1 if enable else 0))
+
+    def profile_read(self):
+        """{class name: dict(launches, ms, bytes, flops)} since the last profile() call (host sync)."""
+        out = {}
+        for k in range(lib.skipper_profile_num_classes()):
+            n, ms, b, f = ct.c_longlong(), ct.c_double(), ct.c_double(), ct.c_double()
+            self._c(lib.skipper_profile_read(self.ctx, k, ct.byref(n), ct.byref(ms), ct.byref(b), ct.byref(f)))
+            out[lib.skipper_profile_class_name(k).decode()] = {
+                "launches": n.value, "ms": ms.value, "bytes": b.value, "flops": f.value}
+        return out
+
+    def launch_count(self):
+        return lib.skipper_launch_count(self.ctx)
+
     def debug(self, which, layer):
         """which: 0 first-pass U, 1 first-pass o, 2 recomputed U, 3 recomputed o -> [T][B][neuron shape]."""
         torch = _torch()
@@ -309,7 +342,14 @@ class SkipperNet:
 
 
 # ---------------------------------------------------------------------- kernel-level entry points
-def _ptr(t):
+def _ptr(t, dtype=None):
+    torch = _torch()
+    if not t.is_cuda or not t.is_contiguous():
+        raise ValueError("kernel operands must be contiguous CUDA tensors")
+    if dtype == "bf16" and t.dtype not in (torch.int16, torch.bfloat16, torch.uint16):
+        raise ValueError(f"bf16 operand expected (bf16 or its int16 bit pattern), got {t.dtype}")
+    if dtype == "f32" and t.dtype != torch.float32:
+        raise ValueError(f"float32 output expected, got {t.dtype}")
     return ct.c_void_p(t.data_ptr())
 
 
@@ -323,7 +363,7 @@ def k_fc_fwd(A, B):
     M, K = A.shape
     N = B.shape[0]
     out = torch.empty((M, N), dtype=torch.float32, device=A.device)
-    _check(lib.skipper_k_fc_fwd(_ptr(A), _ptr(B), _ptr(out), M, N, K, _stream_handle()))
+    _check(lib.skipper_k_fc_fwd(_ptr(A, "bf16"), _ptr(B, "bf16"), _ptr(out, "f32"), M, N, K, _stream_handle()))
     return out
 
 
@@ -334,7 +374,7 @@ def k_fc_wgrad(D, X, out=None):
     acc = out is not None
     if out is None:
         out = torch.empty((N, K), dtype=torch.float32, device=D.device)
-    _check(lib.skipper_k_fc_wgrad(_ptr(D), _ptr(X), _ptr(out), M, N, K, 1 if acc else 0, _stream_handle()))
+    _check(lib.skipper_k_fc_wgrad(_ptr(D, "bf16"), _ptr(X, "bf16"), _ptr(out, "f32"), M, N, K, 1 if acc else 0, _stream_handle()))
     return out
 
 
@@ -344,7 +384,7 @@ def k_conv_fwd(X, Wk):
     nb, h, w, cin = X.shape
     cout = Wk.shape[0]
     out = torch.empty((nb, h, w, cout), dtype=torch.float32, device=X.device)
-    _check(lib.skipper_k_conv_fwd(_ptr(X), _ptr(Wk), _ptr(out), nb, h, w, cin, cout, _stream_handle()))
+    _check(lib.skipper_k_conv_fwd(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, _stream_handle()))
     return out
 
 
@@ -354,7 +394,7 @@ def k_conv_dgrad(D, Wt):
     nb, h, w, cout = D.shape
     cin = Wt.shape[0]
     out = torch.empty((nb, h, w, cin), dtype=torch.float32, device=D.device)
-    _check(lib.skipper_k_conv_dgrad(_ptr(D), _ptr(Wt), _ptr(out), nb, h, w, cin, cout, _stream_handle()))
+    _check(lib.skipper_k_conv_dgrad(_ptr(D, "bf16"), _ptr(Wt, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, _stream_handle()))
     return out
 
 
@@ -366,6 +406,6 @@ def k_conv_wgrad(D, X, out=None):
     acc = out is not None
     if out is None:
         out = torch.empty((cout, 3, 3, cin), dtype=torch.float32, device=D.device)
-    _check(lib.skipper_k_conv_wgrad(_ptr(D), _ptr(X), _ptr(out), nb, h, w, cin, cout, 1 if acc else 0,
+    _check(lib.skipper_k_conv_wgrad(_ptr(D, "bf16"), _ptr(X, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, 1 if acc else 0,
                                     _stream_handle()))
     return out

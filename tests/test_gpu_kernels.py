@@ -62,7 +62,7 @@ def test_fc_wgrad(M, N, K):
     out = k_fc_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda()).cpu().double()
     assert (out - ref).abs().max() <= 1e-6 * ref.abs().max() + 1e-12
     # accumulate mode adds into the existing buffer
-    acc = torch.full((N, K), 0.5, device="cuda")
+    acc = torch.full((N, K), 0.5, dtype=torch.float32, device="cuda")
     k_fc_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda(), out=acc)
     assert (acc.cpu().double() - 0.5 - ref).abs().max() <= 1e-6 * ref.abs().max() + 1e-6
 
@@ -111,3 +111,21 @@ def test_conv_wgrad(nb, h, w, cin, cout):
     ref = Wv.grad
     out = k_conv_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda()).cpu().double()
     assert (out - ref).abs().max() <= 1e-5 * ref.abs().max() + 1e-12
+
+
+def test_stream_ordering_with_torch():
+    """The library's kernels are ordered with torch's work on the same stream: a long GEMM
+    followed immediately by a torch copy of its output must see the finished result."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_fc_fwd
+    M, N, K = 1 << 16, 1024, 4096
+    A = torch.ones((M, K), dtype=torch.bfloat16, device="cuda")
+    B = torch.full((N, K), 0.5, dtype=torch.bfloat16, device="cuda")
+    for _ in range(3):
+        out = k_fc_fwd(A.view(torch.int16), B.view(torch.int16))
+        host = out.cpu()                      # no explicit synchronize
+        assert torch.all(host == K * 0.5)
+        side = torch.cuda.Stream()
+        with torch.cuda.stream(side):
+            out2 = k_fc_fwd(A.view(torch.int16), B.view(torch.int16))
+            h2 = out2.cpu()
+        assert torch.all(h2 == K * 0.5)

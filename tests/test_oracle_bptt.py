@@ -16,7 +16,6 @@ import synth
 from oracle import StepConfig, train_step
 from oracle.bptt import readout
 
-torch.set_default_dtype(torch.float64)
 
 
 class Spike(torch.autograd.Function):
@@ -47,7 +46,7 @@ def t_out(layer, o):
 
 def torch_full_bptt(net, W, x, y, gamma=0.3):
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
-    Wt = [torch.tensor(w.astype(np.float64), requires_grad=True) for w in W]
+    Wt = [torch.tensor(w.astype(np.float64), dtype=torch.float64, requires_grad=True) for w in W]
     T, B = x.shape[:2]
     U = [None] * len(spk)
     o = [None] * len(spk)
@@ -75,7 +74,7 @@ def torch_skip_bptt(net, W, x, kept, dz, T, gamma=0.3):
     value (from a no-grad first pass) with straight-through gradient paths to its
     own current I_{cS} and (times lam) to the previous segment's last kept U."""
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
-    Wt = [torch.tensor(w.astype(np.float64), requires_grad=True) for w in W]
+    Wt = [torch.tensor(w.astype(np.float64), dtype=torch.float64, requires_grad=True) for w in W]
     B = x.shape[1]
     # first pass, no grad: checkpoint states at each segment start
     ck = {}
@@ -113,7 +112,7 @@ def torch_skip_bptt(net, W, x, kept, dz, T, gamma=0.3):
             cnt = cnt + a
         prev_last = list(U)
     z = cnt.reshape(B, -1) @ Wt[-1].T / T
-    surrogate_loss = (torch.tensor(dz) * z).sum()
+    surrogate_loss = (torch.tensor(dz, dtype=torch.float64) * z).sum()
     surrogate_loss.backward()
     return [w.grad.numpy() for w in Wt]
 
