@@ -185,8 +185,6 @@ def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=
     torch.cuda.synchronize()
     m.reset_peak()
     torch.cuda.reset_peak_memory_stats()
-    if profile:
-        m.profile(True)
     clocks = ClockSampler(local_rank)
     clocks.start() if profile else None
     launches0 = m.launch_count()
@@ -213,7 +211,17 @@ def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
     total_ms = float(tot.item())
     launches = m.launch_count() - launches0
-    prof = m.profile_read() if profile else None
+    prof = None
+    if profile:
+        # kernel-class attribution: the same K steps again with every launch bracketed by CUDA
+        # events on the library stream (kept out of the headline timing: the event records add
+        # host work per launch)
+        m.profile(True)
+        for _ in range(args.steps):
+            flush.zero_()
+            m.step(xd, yd, want_loss=False)
+        prof = m.profile_read()
+        m.profile(False)
     peak_lib = m.mem_stats()[1]
     peak_torch = torch.cuda.max_memory_allocated()
     loss = m.loss()

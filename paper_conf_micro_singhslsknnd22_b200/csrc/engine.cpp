@@ -16,7 +16,9 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include "comm.h"
@@ -45,6 +47,33 @@ struct Layer {
 };
 
 enum Phase { PH_IDLE = 0, PH_FIRST, PH_READY_BWD, PH_RECOMPUTED, PH_BWD_DONE };
+
+// GEMM plans (three encoded TMA descriptors each) are cached by operand pointers and shape: the
+// segment arenas come back at the same addresses step after step, so steady-state steps encode no
+// tensor maps on the host.
+struct PlanKey {
+    int op;
+    const void *a, *b;
+    const void *c;
+    long long M;
+    int N, K, h, w, x;
+    bool operator==(const PlanKey &o) const {
+        return op == o.op && a == o.a && b == o.b && c == o.c && M == o.M && N == o.N && K == o.K && h == o.h &&
+               w == o.w && x == o.x;
+    }
+};
+struct PlanKeyHash {
+    size_t operator()(const PlanKey &k) const {
+        size_t h = std::hash<const void *>()(k.a);
+        auto mix = [&h](size_t v) { h ^= v + 0x9e3779b97f4a7c15ULL + (h << 6) + (h >> 2); };
+        mix(std::hash<const void *>()(k.b));
+        mix(std::hash<const void *>()(k.c));
+        mix((size_t)k.M);
+        mix((size_t)k.op * 131 + k.N);
+        mix((size_t)k.K * 31 + k.h * 7 + k.w * 3 + k.x);
+        return h;
+    }
+};
 
 }  // namespace
 
@@ -97,6 +126,7 @@ struct skipper_ctx {
     bool poisoned = false;
     // comm
     sk::Comm comm;
+    std::unordered_map<PlanKey, sk::GemmLaunch, PlanKeyHash> plans;
     // profiling (per kernel class: launches, device ms, algorithmic bytes and flops)
     bool prof_on = false;
     std::vector<cudaEvent_t> ev_pool;
@@ -691,6 +721,19 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
 }
 
 // ------------------------------------------------------------------------------------ GEMM dispatch
+// Cached GEMM plan: builds (and encodes the tensor maps) on first use of a (pointers, shape) key.
+static bool get_plan(skipper_ctx *c, const PlanKey &k, sk::GemmLaunch &g, const std::function<bool(sk::GemmLaunch *)> &make) {
+    auto it = c->plans.find(k);
+    if (it != c->plans.end()) {
+        g = it->second;
+        return true;
+    }
+    if (!make(&g)) return false;
+    if (c->plans.size() > 4096) c->plans.clear();
+    c->plans.emplace(k, g);
+    return true;
+}
+
 static skipper_status run_gemm(skipper_ctx *c, const sk::GemmLaunch &g, bool ok, const char *what, int layer,
                                int cls, double bytes, double flops) {
     if (!ok) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: cannot plan %s GEMM (tensor map)", layer, what);
@@ -707,11 +750,16 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     const int nb = rows * c->B;
     bool ok;
     if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
-        ok = sk::plan_fc(&g, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0);
+        ok = get_plan(c, {0, in, l.wbp, I, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 1}, g,
+                      [&](sk::GemmLaunch *p) { return sk::plan_fc(p, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0); });
     else if (l.conv)
-        ok = sk::plan_conv(&g, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
+        ok = get_plan(c, {1, in, l.wb, I, nb, l.Cin, l.Cout, l.H, l.W, 1}, g, [&](sk::GemmLaunch *p) {
+            return sk::plan_conv(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
+        });
     else
-        ok = sk::plan_fc(&g, in, l.wb, I, nb, l.Cout, l.Cin, l.fsplit);
+        ok = get_plan(c, {0, in, l.wb, I, nb, l.Cout, l.Cin, 0, 0, l.fsplit}, g, [&](sk::GemmLaunch *p) {
+            return sk::plan_fc(p, in, l.wb, I, nb, l.Cout, l.Cin, l.fsplit);
+        });
     if (ok && g.d.splits != (l.fc ? l.fsplit : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
     const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
     const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4 * l.fsplit;
@@ -937,11 +985,18 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         sk::GemmLaunch g;
         bool ok;
         if (i == 0 && c->in_kind == 1)
-            ok = sk::plan_fc_wgrad(&g, c->d_buf, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
+            ok = get_plan(c, {2, c->d_buf, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
+                          [&](sk::GemmLaunch *p) {
+                              return sk::plan_fc_wgrad(p, c->d_buf, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
+                          });
         else if (l.conv)
-            ok = sk::plan_conv_wgrad(&g, c->d_buf, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
+            ok = get_plan(c, {3, c->d_buf, X, l.dw, nb, l.Cin, l.Cout, l.H, l.W, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_conv_wgrad(p, c->d_buf, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
+            });
         else
-            ok = sk::plan_fc_wgrad(&g, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
+            ok = get_plan(c, {2, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_fc_wgrad(p, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
+            });
         {
             const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
             const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
@@ -949,9 +1004,15 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         }
         if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
             if (l.conv)
-                ok = sk::plan_conv(&g, c->d_buf, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
+                ok = get_plan(c, {1, c->d_buf, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g,
+                              [&](sk::GemmLaunch *p) {
+                                  return sk::plan_conv(p, c->d_buf, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
+                              });
             else
-                ok = sk::plan_fc(&g, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, l.dsplit);
+                ok = get_plan(c, {0, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, 0, 0, l.dsplit}, g,
+                              [&](sk::GemmLaunch *p) {
+                                  return sk::plan_fc(p, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, l.dsplit);
+                              });
             const double M = (double)nb * l.H * l.W, K = (double)l.Cout * (l.conv ? 9 : 1);
             const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4 * l.dsplit;
             CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * (l.Nin / (l.H * l.W)) * K));

@@ -48,13 +48,16 @@ SK_DEV float4 ldg4_split(const float *p, int nsplit, long long stride) {
 }
 
 // ============================================================================ K1 forward scan
-// One thread owns 4 consecutive channels of NP pixels (NP = 4 for a 2x2 pooled window).  The
-// currents of CH rows are loaded before the recurrence runs over them (loads do not depend on
-// the recurrence), which keeps CH x NP 16-byte loads in flight per thread.
-template <int POOL, int CH>
-__global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
+// One thread owns 4 consecutive channels of NP pixels (NP = 4: the 2x2 window of one pooled output).
+// The currents of CH rows are loaded before the recurrence consumes them (the loads do not depend
+// on the recurrence); __launch_bounds__(256, 4) keeps the register file at <= 64 per thread so
+// 32 warps per SM keep enough 16-byte loads in flight for HBM.  Spike counts per row (SAM, Eq.4)
+// go through shared-memory atomics and one global atomic per row per block at the end.
+template <int POOL, int SPLIT>
+__global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFwdArgs a) {
     constexpr int NP = POOL ? 4 : 1;
-    __shared__ unsigned red[8][CH];
+    constexpr int CH = POOL ? 2 : (SPLIT ? 4 : 8);
+    extern __shared__ unsigned s_cnt[];  // [R] block spike count per row (when a.s_part)
     const int C = a.C;
     const int C4 = C >> 2;
     const long long HW = (long long)a.H * a.W;
@@ -63,11 +66,17 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
     const bool active = p < P;
     const long long rs = (long long)a.B * HW * C;  // neurons per row
     const long long ors = POOL ? rs / 4 : rs;       // outputs per row
+    const int nspl = SPLIT ? a.nsplit : 1;
 
-    long long nidx[NP], oidx = 0;
-    if (active) {
-        const int c4 = (int)(p % C4);
-        long long rest = p / C4;
+    if (a.s_part) {
+        for (int r = threadIdx.x; r < a.R; r += blockDim.x) s_cnt[r] = 0;
+        __syncthreads();
+    }
+    int nidx[NP], oidx = 0;  // offsets within one row (a row holds < 2^31 neurons)
+    {
+        const long long pp = active ? p : 0;
+        const int c4 = (int)(pp % C4);
+        long long rest = pp / C4;
         if (POOL) {
             const int PW = a.W / 2, PH = a.H / 2;
             const int px = (int)(rest % PW);
@@ -75,42 +84,40 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
             const int py = (int)(rest % PH);
             const long long b = rest / PH;
 #pragma unroll
-            for (int k = 0; k < NP; ++k) {
-                const int y = 2 * py + (k >> 1), x = 2 * px + (k & 1);
-                nidx[k] = ((b * a.H + y) * a.W + x) * C + 4 * c4;
-            }
-            oidx = ((b * PH + py) * PW + px) * C + 4 * c4;
+            for (int k = 0; k < NP; ++k)
+                nidx[k] = (int)(((b * a.H + 2 * py + (k >> 1)) * a.W + 2 * px + (k & 1)) * C + 4 * c4);
+            oidx = (int)(((b * PH + py) * PW + px) * C + 4 * c4);
         } else {
-            nidx[0] = rest * C + 4 * c4;
+            nidx[0] = (int)(rest * C + 4 * c4);
             oidx = nidx[0];
+        }
+    }
+
+    float U[NP][4];
+    uint32_t ob = 0;  // spike bits, bit 4k+i
+    if (active) {
+#pragma unroll
+        for (int k = 0; k < NP; ++k) {
+            const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nidx[k]);
+            const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nidx[k]);
+            U[k][0] = u.x; U[k][1] = u.y; U[k][2] = u.z; U[k][3] = u.w;
+            ob |= (o4.x ? 1u : 0u) << (4 * k) | (o4.y ? 1u : 0u) << (4 * k + 1) |
+                  (o4.z ? 1u : 0u) << (4 * k + 2) | (o4.w ? 1u : 0u) << (4 * k + 3);
         }
     } else {
 #pragma unroll
-        for (int k = 0; k < NP; ++k) nidx[k] = 0;
-    }
-
-    float U[NP][4], O[NP][4];
-#pragma unroll
-    for (int k = 0; k < NP; ++k) {
-        if (active) {
-            const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nidx[k]);
-            const uchar4 ob = *reinterpret_cast<const uchar4 *>(a.o_state + nidx[k]);
-            U[k][0] = u.x; U[k][1] = u.y; U[k][2] = u.z; U[k][3] = u.w;
-            O[k][0] = ob.x; O[k][1] = ob.y; O[k][2] = ob.z; O[k][3] = ob.w;
-        } else {
-#pragma unroll
-            for (int i = 0; i < 4; ++i) U[k][i] = O[k][i] = 0.f;
-        }
+        for (int k = 0; k < NP; ++k) U[k][0] = U[k][1] = U[k][2] = U[k][3] = 0.f;
     }
     float cacc[4] = {0.f, 0.f, 0.f, 0.f};
+    auto bit = [&](int k, int i) { return (float)((ob >> (4 * k + i)) & 1u); };
 
-    auto emit_row = [&](int r) {  // write outputs of row r from the current (U, O)
+    auto emit_row = [&](int r) {  // outputs of row r from the current (U, spikes)
         float out[4];
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
             float sum = 0.f;
 #pragma unroll
-            for (int k = 0; k < NP; ++k) sum += O[k][i];
+            for (int k = 0; k < NP; ++k) sum += bit(k, i);
             out[i] = POOL ? sum * 0.25f : sum;
             cacc[i] += out[i];
         }
@@ -127,7 +134,8 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
             for (int k = 0; k < NP; ++k) {
                 *reinterpret_cast<float4 *>(a.dbg_U + t * rs + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
                 *reinterpret_cast<uchar4 *>(a.dbg_o + t * rs + nidx[k]) =
-                    make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+                    make_uchar4((unsigned char)bit(k, 0), (unsigned char)bit(k, 1), (unsigned char)bit(k, 2),
+                                (unsigned char)bit(k, 3));
             }
         }
     };
@@ -137,60 +145,55 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
         if (active) emit_row(0);
         r0 = 1;
     }
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int nwarps = blockDim.x >> 5;
+    const int lane = threadIdx.x & 31;
     for (int rb = r0; rb < a.R; rb += CH) {
         float4 Iv[CH][NP];
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb + j;
 #pragma unroll
-            for (int k = 0; k < NP; ++k)
-                Iv[j][k] = (active && r < a.R) ? ldg4_split(a.I + (long long)r * rs + nidx[k], a.nsplit, a.split_stride)
-                                               : make_float4(0.f, 0.f, 0.f, 0.f);
+            for (int k = 0; k < NP; ++k) {
+                if (active && r < a.R) {
+                    const float *src = a.I + (long long)r * rs + nidx[k];
+                    Iv[j][k] = SPLIT ? ldg4_split(src, nspl, a.split_stride) : ldg4(src);
+                } else {
+                    Iv[j][k] = make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+            }
         }
-        unsigned nspk[CH];
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb + j;
-            nspk[j] = 0;
-            if (active && r < a.R) {
+            if (r >= a.R) break;  // block-uniform
+            unsigned nspk = 0;
+            if (active) {
+                uint32_t nb = 0;
 #pragma unroll
                 for (int k = 0; k < NP; ++k) {
                     const float Ii[4] = {Iv[j][k].x, Iv[j][k].y, Iv[j][k].z, Iv[j][k].w};
 #pragma unroll
                     for (int i = 0; i < 4; ++i) {
-                        U[k][i] = lif_update(U[k][i], Ii[i], O[k][i], a.lam, a.theta);
-                        O[k][i] = U[k][i] > a.theta ? 1.f : 0.f;
-                        nspk[j] += (unsigned)O[k][i];
+                        U[k][i] = lif_update(U[k][i], Ii[i], bit(k, i), a.lam, a.theta);
+                        nb |= (U[k][i] > a.theta ? 1u : 0u) << (4 * k + i);
                     }
                 }
+                ob = nb;
+                nspk = __popc(ob);
                 emit_row(r);
                 if (a.ckU && r == 0) {
 #pragma unroll
                     for (int k = 0; k < NP; ++k) {
                         *reinterpret_cast<float4 *>(a.ckU + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
                         *reinterpret_cast<uchar4 *>(a.cko + nidx[k]) =
-                            make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+                            make_uchar4((unsigned char)bit(k, 0), (unsigned char)bit(k, 1), (unsigned char)bit(k, 2),
+                                        (unsigned char)bit(k, 3));
                     }
                 }
             }
-        }
-        if (a.s_part) {  // block-uniform
-#pragma unroll
-            for (int j = 0; j < CH; ++j) {
-                const unsigned v = __reduce_add_sync(0xffffffffu, nspk[j]);
-                if (lane == 0) red[warp][j] = v;
+            if (a.s_part) {
+                const unsigned v = __reduce_add_sync(0xffffffffu, nspk);
+                if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
             }
-            __syncthreads();
-            if (threadIdx.x < CH && rb + (int)threadIdx.x < a.R) {
-                unsigned tot = 0;
-                for (int w = 0; w < nwarps; ++w) tot += red[w][threadIdx.x];
-                const int r = rb + threadIdx.x;
-                const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
-                if (tot) atomicAdd(a.s_part + t * 32 + (blockIdx.x & 31), tot);
-            }
-            __syncthreads();
         }
     }
     if (active) {
@@ -199,7 +202,8 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
             for (int k = 0; k < NP; ++k) {
                 *reinterpret_cast<float4 *>(a.U_state + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
                 *reinterpret_cast<uchar4 *>(a.o_state + nidx[k]) =
-                    make_uchar4((unsigned char)O[k][0], (unsigned char)O[k][1], (unsigned char)O[k][2], (unsigned char)O[k][3]);
+                    make_uchar4((unsigned char)bit(k, 0), (unsigned char)bit(k, 1), (unsigned char)bit(k, 2),
+                                (unsigned char)bit(k, 3));
             }
         }
         if (a.cnt) {
@@ -207,6 +211,14 @@ __global__ void __launch_bounds__(256) lif_fwd_kernel(const ScanFwdArgs a) {
             float4 cv = *cp;
             cv.x += cacc[0]; cv.y += cacc[1]; cv.z += cacc[2]; cv.w += cacc[3];
             *cp = cv;
+        }
+    }
+    if (a.s_part) {
+        __syncthreads();
+        for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
+            const unsigned v = s_cnt[r];
+            const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+            if (v) atomicAdd(a.s_part + t * 32 + (blockIdx.x & 31), v);
         }
     }
 }
@@ -218,16 +230,24 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     const int threads = 256;
     const long long blocks = (P + threads - 1) / threads;
     if (blocks == 0) return cudaSuccess;
-    if (a.pool)
-        lif_fwd_kernel<1, 4><<<(unsigned)blocks, threads, 0, s>>>(a);
-    else
-        lif_fwd_kernel<0, 8><<<(unsigned)blocks, threads, 0, s>>>(a);
+    const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
+    if (smem > 48 * 1024) return cudaErrorInvalidValue;
+    const bool split = a.nsplit > 1;
+    if (a.pool) {
+        if (split) lif_fwd_kernel<1, 1><<<(unsigned)blocks, threads, smem, s>>>(a);
+        else lif_fwd_kernel<1, 0><<<(unsigned)blocks, threads, smem, s>>>(a);
+    } else {
+        if (split) lif_fwd_kernel<0, 1><<<(unsigned)blocks, threads, smem, s>>>(a);
+        else lif_fwd_kernel<0, 0><<<(unsigned)blocks, threads, smem, s>>>(a);
+    }
     return cudaGetLastError();
 }
 
 // ============================================================================ K4 reverse scan
-template <int CH>
-__global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
+// One thread owns 4 neurons; CH rows of (g, U) are loaded ahead of the reverse recurrence.
+template <int SPLIT>
+__global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
+    constexpr int CH = 4;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
     const long long rs = (long long)a.B * HW * C;
@@ -247,6 +267,7 @@ __global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
     }
     if (a.g_broadcast) grs = 0;
     const float gs = a.g_pooled ? 0.25f : 1.0f;
+    const int nspl = SPLIT ? a.nsplit : 1;
     float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
     for (int rb = a.R - 1; rb >= 0; rb -= CH) {
         float4 gv[CH], uv[CH];
@@ -254,7 +275,8 @@ __global__ void __launch_bounds__(256) lif_bwd_kernel(const ScanBwdArgs a) {
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
             if (r >= 0) {
-                gv[j] = ldg4_split(a.g + (long long)r * grs + gi, a.nsplit, a.split_stride);
+                const float *src = a.g + (long long)r * grs + gi;
+                gv[j] = SPLIT ? ldg4_split(src, nspl, a.split_stride) : ldg4(src);
                 uv[j] = ldg4(a.U + (long long)r * rs + n0);
             }
         }
@@ -279,11 +301,13 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     if (rs == 0 || a.R == 0) return cudaSuccess;
     const long long P = rs / 4;
-    lif_bwd_kernel<8><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
+    if (a.nsplit > 1)
+        lif_bwd_kernel<1><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
+    else
+        lif_bwd_kernel<0><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
     return cudaGetLastError();
 }
 
-// ============================================================================ input staging / SAM
 // Layer-0 operand rows for the timesteps of one segment (FIRST: t0 + r; RECOMPUTE: the kept list),
 // straight from the uint8 input.  kind 0: bf16 copy of x[t] (fc or conv-with-wide-Cin input);
 // kind 1: im2col of a 3x3 / pad-1 window, k = (dy*3+dx)*C0 + ci, zero-padded to K0 columns.
@@ -305,9 +329,7 @@ __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__res
             const int yy = (int)((e / W) % H);
             const long long b = e / ((long long)H * W);
             const uint8_t *xt = x + (t * B + b) * (long long)H * W * C0;
-            uint16_t col[64];
-#pragma unroll
-            for (int k = 0; k < 64; ++k) col[k] = 0;
+            uint64_t m = 0;  // bit k = im2col column k (registers only: no dynamically indexed arrays)
             for (int dy = 0; dy < 3; ++dy) {
                 const int y = yy + dy - 1;
                 if (y < 0 || y >= H) continue;
@@ -316,19 +338,23 @@ __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__res
                     if (xq < 0 || xq >= W) continue;
                     const uint8_t *px = xt + ((long long)y * W + xq) * C0;
                     for (int ci = 0; ci < C0; ++ci)
-                        if (px[ci]) col[(dy * 3 + dx) * C0 + ci] = 0x3F80;
+                        if (__ldg(px + ci)) m |= 1ull << ((dy * 3 + dx) * C0 + ci);
                 }
             }
             const uint8_t *pc = xt + ((long long)yy * W + xx) * C0;
-            for (int ci = 0; ci < C0; ++ci) cnt += pc[ci] ? 1u : 0u;
+            for (int ci = 0; ci < C0; ++ci) cnt += __ldg(pc + ci) ? 1u : 0u;
             uint4 *o = reinterpret_cast<uint4 *>(dst + i * K0);
-            for (int q = 0; q < K0 / 8; ++q) {
-                uint4 v;
-                v.x = col[8 * q] | ((uint32_t)col[8 * q + 1] << 16);
-                v.y = col[8 * q + 2] | ((uint32_t)col[8 * q + 3] << 16);
-                v.z = col[8 * q + 4] | ((uint32_t)col[8 * q + 5] << 16);
-                v.w = col[8 * q + 6] | ((uint32_t)col[8 * q + 7] << 16);
-                o[q] = v;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                if (q < K0 / 8) {
+                    uint32_t w[4];
+#pragma unroll
+                    for (int h = 0; h < 4; ++h) {
+                        const int k = 8 * q + 2 * h;
+                        w[h] = (((m >> k) & 1ull) ? 0x3F80u : 0u) | (((m >> (k + 1)) & 1ull) ? 0x3F800000u : 0u);
+                    }
+                    o[q] = make_uint4(w[0], w[1], w[2], w[3]);
+                }
             }
         } else {
             const uint8_t v = x[t * (long long)B * D + e];
