@@ -163,3 +163,30 @@ SK_DEV uint16_t f2bf_bits(float x) {  // round-to-nearest-even
 SK_DEV float bf_bits2f(uint16_t b) { return __uint_as_float(static_cast<uint32_t>(b) << 16); }
 
 }  // namespace sk
+
+namespace sk {
+// ---------------------------------------------------------------- clusters / multicast
+SK_DEV uint32_t cluster_ctarank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+SK_DEV void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// TMA 2D load multicast to every CTA in `mask` (same smem offset and mbarrier offset in each)
+SK_DEV void tma_load_2d_mc(uint32_t dst, const void *tmap, uint32_t bar, int c0, int c1, uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+        " [%0], [%1, {%4, %5}], [%2], %3;" ::"r"(dst),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar), "h"(mask), "r"(c0), "r"(c1)
+        : "memory");
+}
+// tcgen05.commit arriving on the same-offset mbarrier of every CTA in `mask`
+SK_DEV void tc_commit_mc(uint32_t bar, uint16_t mask) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                     bar),
+                 "h"(mask)
+                 : "memory");
+}
+}  // namespace sk

@@ -15,6 +15,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <string>
@@ -88,6 +89,7 @@ struct skipper_ctx {
     int num_sms = 148;
     int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
     int K0 = 0;                 // im2col width (32 or 64)
+    bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
     int in_h = 1, in_w = 1, in_c = 0;
     long long in_elems = 0;     // input elements per sample (uint8 x)
     long long in_row = 0;       // staged bf16 layer-0 operand elements per sample
@@ -140,10 +142,11 @@ struct skipper_ctx {
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
-    K_NCLASS
+    K_L0_FWD, K_NCLASS
 };
 static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
-                                               "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad"};
+                                               "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad",
+                                               "layer0_fused_fwd"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -462,6 +465,12 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     c->S = c->T / c->C;
     c->num_sms = sk::device_num_sms();
+    {
+        const Layer &f = c->L[0];
+        const char *e = getenv("SKIPPER_NO_L0_FUSION");
+        c->l0_fused = c->in_kind == 1 && c->K0 == 32 && c->Ls >= 2 && !(e && atoi(e)) &&
+                      sk::layer0_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
+    }
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         if (!l.fc) continue;
@@ -821,9 +830,48 @@ static skipper_status stage_input(skipper_ctx *c, const int *rows, int t0, int R
     return SKIPPER_OK;
 }
 
+// Layer 0 as one fused kernel: im2col in smem, tcgen05, LIF, pooling, SAM, checkpoint (layer0.cu).
+static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const int *row_t, bool restore,
+                                   bool record, uint16_t *out) {
+    Layer &l = c->L[0];
+    const size_t bn = (size_t)c->B * l.N;
+    sk::L0FwdArgs a{};
+    a.x = c->x_cur;
+    a.T = c->T;
+    a.B = c->B;
+    a.H = l.H;
+    a.W = l.W;
+    a.C0 = l.Cin;
+    a.row_t = row_t;
+    a.t0 = t0;
+    a.R = R;
+    a.restore = restore ? 1 : 0;
+    a.wbp = l.wbp;
+    a.N = l.Cout;
+    a.pool = l.pool ? 1 : 0;
+    a.lam = l.d.lambda;
+    a.theta = l.d.theta;
+    a.U_state = restore ? l.ckU + (size_t)seg * bn : l.U_run;
+    a.o_state = restore ? l.cko + (size_t)seg * bn : l.o_run;
+    a.U_out = (restore || record) ? l.Useg : nullptr;
+    a.Po_out = out;
+    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
+    a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.s_part = restore ? nullptr : c->s_part;
+    a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
+    a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
+    const double bytes = (double)R * c->B * (c->in_elems + l.Nout * 2 + (a.U_out ? l.N * 4 : 0)) + bn * 10;
+    const double flops = 2.0 * R * c->B * l.H * l.W * l.Cout * 9 * l.Cin;
+    ProfScope ps(c, K_L0_FWD, bytes, flops);
+    CK(sk::launch_layer0_fwd(a, c->st, c->num_sms));
+    return SKIPPER_OK;
+}
+
 // Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
 static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
-    CKS(stage_input(c, nullptr, t0, R, true));
+    // the staged layer-0 operand is needed by the first pass unless layer 0 is fused, and by the
+    // layer-0 weight gradient of FULL mode
+    if (!c->l0_fused || record) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in;
@@ -834,6 +882,10 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         } else {
             in = i == 0 ? c->xg : c->P2[(i - 1) & 1];
             out = c->P2[i & 1];
+        }
+        if (i == 0 && c->l0_fused) {
+            CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));
+            continue;
         }
         CKS(gemm_forward(c, i, in, c->I_buf, R));
         sk::ScanFwdArgs a{};
@@ -919,6 +971,10 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
     CKS(stage_input(c, row_t, 0, R, false));
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
+        if (i == 0 && c->l0_fused) {
+            CKS(layer0_fused(c, seg, R, 0, row_t, true, false, l.Po));
+            continue;
+        }
         const uint16_t *in = i == 0 ? c->xg : c->L[i - 1].Po;
         const size_t in_row = (size_t)c->B * (i == 0 ? c->in_row : c->L[i - 1].Nout);
         if (R > 1)  // rows 1..R-1 (row 0 is the checkpoint)

@@ -30,7 +30,9 @@ struct GemmDev {
     int conv_cb;        // channel blocks of 64 per tap (A = OP_KCONV)
     int conv_hw, conv_w;  // image H*W and W (row -> (image, y) decode)
     int conv_sign;      // +1 forward / wgrad, -1 dgrad (flipped taps)
-    int cols_per_tap;   // wgrad conv: output column offset per tap (= Cin)
+    int cols_per_tap;   // output column offset per tap (unused when 0)
+    int wg_cin;         // wgrad conv with N = (tap, cin): channels per tap (0 = N is one tap's channels)
+    int transpose_out;  // the tile is D^T: TMEM lanes are output columns, TMEM columns output rows
     float *C;
     long long ldc;
     int M, N;           // valid output extent (rows, columns of one tap block)
@@ -42,6 +44,7 @@ struct GemmLaunch {
     CUtensorMap ta, tb, tc;  // operands A, B and the fp32 output
     int bn;             // 64, 128 or 256
     int mn_major;       // 0: both operands K-major; 1: both MN-major (wgrad)
+    int cs = 1;         // cluster size: B tile multicast across cs CTAs working on consecutive M tiles
 };
 
 // Tensor-map builders (bf16, 128-byte swizzle, OOB -> zero).

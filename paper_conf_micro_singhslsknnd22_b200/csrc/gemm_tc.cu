@@ -14,6 +14,7 @@
 #include "gemm.h"
 
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 
 namespace sk {
@@ -37,6 +38,30 @@ struct TileCoord {
     int m_t, n_t, tap, split, kb0, kb1;
 };
 
+// CS > 1: a cluster of CS CTAs walks groups of CS consecutive M tiles sharing one N tile; each CTA
+// loads its own A tile and 1/CS of the B tile, multicast to the whole cluster.
+template <int CS>
+SK_DEV int iter_count(const GemmDev &g) {
+    if (CS == 1) return g.m_tiles * g.n_tiles * g.taps * g.splits;
+    return ((g.m_tiles + CS - 1) / CS) * g.n_tiles;
+}
+
+SK_DEV TileCoord decode_tile(const GemmDev &g, int tile);
+
+template <int CS>
+SK_DEV TileCoord tile_at(const GemmDev &g, int it, int rank) {
+    if (CS == 1) return decode_tile(g, it);
+    const int mg = (g.m_tiles + CS - 1) / CS;
+    TileCoord c;
+    c.m_t = (it % mg) * CS + rank;
+    c.n_t = it / mg;
+    c.tap = 0;
+    c.split = 0;
+    c.kb0 = 0;
+    c.kb1 = g.num_kb;
+    return c;
+}
+
 SK_DEV TileCoord decode_tile(const GemmDev &g, int tile) {
     TileCoord c;
     c.m_t = tile % g.m_tiles;
@@ -50,7 +75,7 @@ SK_DEV TileCoord decode_tile(const GemmDev &g, int tile) {
     return c;
 }
 
-template <int BN, int MN>
+template <int BN, int MN, int CS>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
                    const __grid_constant__ CUtensorMap tcm, const GemmDev g) {
@@ -77,7 +102,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         tma_prefetch(&tcm);
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(full_bar(s), 1);
-            mbar_init(empty_bar(s), 1);
+            mbar_init(empty_bar(s), CS);  // every CTA of the cluster frees the stage (multicast B)
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(tfull_bar(a), 1);
@@ -87,19 +112,26 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
     tc_fence_before();
-    __syncthreads();
+    if (CS > 1)
+        cluster_sync_all();
+    else
+        __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(tmem_slot_ptr);
 
-    const int total = g.m_tiles * g.n_tiles * g.taps * g.splits;
+    const int total = iter_count<CS>(g);
+    const int rank = CS > 1 ? (int)cluster_ctarank() : 0;
+    const int it0 = CS > 1 ? (int)blockIdx.x / CS : (int)blockIdx.x;
+    const int itstep = CS > 1 ? (int)gridDim.x / CS : (int)gridDim.x;
+    constexpr uint16_t mc_mask = (uint16_t)((1u << CS) - 1u);
 
     if (warp == 0) {
         if (lane == 0) {
             // ------------------------------------------------------------ TMA producer
             int stage = 0;
             uint32_t phase = 0;
-            for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
-                const TileCoord tc = decode_tile(g, tile);
+            for (int tile = it0; tile < total; tile += itstep) {
+                const TileCoord tc = tile_at<CS>(g, tile, rank);
                 const int tdy = tc.tap / 3 - 1, tdx = tc.tap % 3 - 1;
                 for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
                     mbar_wait(empty_bar(stage), phase ^ 1u);
@@ -122,19 +154,38 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         tma_load_2d(sa + 8192u, &ta, fb, tc.m_t * BM + 64, kb * BK);
                     }
                     // ---- B
-                    if (g.b_kind == OP_K2D) {
+                    if (CS > 1) {  // K-major B slice multicast to the cluster
+                        constexpr uint32_t SL = BN / CS;
+                        tma_load_2d_mc(sb + (uint32_t)rank * SL * 128u, &tb, fb, kb * BK, tc.n_t * BN + rank * (int)SL,
+                                       mc_mask);
+                    } else if (g.b_kind == OP_K2D) {
                         tma_load_2d(sb, &tb, fb, kb * BK, tc.n_t * BN);
                     } else if (g.b_kind == OP_MN2D) {
 #pragma unroll
                         for (int i = 0; i < BN / 64; ++i)
                             tma_load_2d(sb + 8192u * i, &tb, fb, tc.n_t * BN + 64 * i, kb * BK);
-                    } else {  // OP_MNCONV: K rows kb*64.. of the image, shifted by the tile's tap
+                    } else if (g.b_kind == OP_KCONV) {  // activations as the N operand (transposed conv)
+                        const int tap = kb / g.conv_cb, cblk = kb % g.conv_cb;
+                        const int dy = tap / 3 - 1, dx = tap % 3 - 1;
+                        const int m0 = tc.n_t * BN;
+                        const int n0 = m0 / g.conv_hw;
+                        const int y0 = (m0 % g.conv_hw) / g.conv_w;
+                        tma_load_4d(sb, &tb, fb, cblk * BK, g.conv_sign * dx, y0 + g.conv_sign * dy, n0);
+                    } else {  // OP_MNCONV: K rows kb*64.. of the image, shifted by the tap of each 64-chunk
                         const int m0 = kb * BK;
                         const int n0 = m0 / g.conv_hw;
                         const int y0 = (m0 % g.conv_hw) / g.conv_w;
 #pragma unroll
-                        for (int i = 0; i < BN / 64; ++i)
-                            tma_load_4d(sb + 8192u * i, &tb, fb, tc.n_t * BN + 64 * i, tdx, y0 + tdy, n0);
+                        for (int i = 0; i < BN / 64; ++i) {
+                            int ci0 = tc.n_t * BN + 64 * i, ddy = tdy, ddx = tdx;
+                            if (g.wg_cin) {  // N = (tap, cin): this chunk's tap
+                                const int tp = ci0 / g.wg_cin;
+                                ci0 -= tp * g.wg_cin;
+                                ddy = tp / 3 - 1;
+                                ddx = tp % 3 - 1;
+                            }
+                            tma_load_4d(sb + 8192u * i, &tb, fb, ci0, ddx, y0 + ddy, n0);
+                        }
                     }
                     if (++stage == STAGES) {
                         stage = 0;
@@ -151,8 +202,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
-            for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
-                const TileCoord tc = decode_tile(g, tile);
+            for (int tile = it0; tile < total; tile += itstep) {
+                const TileCoord tc = tile_at<CS>(g, tile, rank);
                 mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + acc * BN;
@@ -173,7 +224,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         }
                         tc_mma_f16(d_tmem, ad, bd, idesc, (kb > tc.kb0 || k > 0) ? 1u : 0u);
                     }
-                    tc_commit(empty_bar(stage));
+                    if (CS > 1)
+                        tc_commit_mc(empty_bar(stage), mc_mask);
+                    else
+                        tc_commit(empty_bar(stage));
                     if (++stage == STAGES) {
                         stage = 0;
                         phase ^= 1u;
@@ -195,8 +249,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         int acc = 0;
         uint32_t acc_phase = 0;
         uint32_t nbox = 0;
-        for (int tile = blockIdx.x; tile < total; tile += gridDim.x) {
-            const TileCoord tc = decode_tile(g, tile);
+        for (int tile = it0; tile < total; tile += itstep) {
+            const TileCoord tc = tile_at<CS>(g, tile, rank);
             mbar_wait(tfull_bar(acc), acc_phase);
             tc_fence_after();
             const int row0 = tc.m_t * BM + q * 32;
@@ -208,14 +262,26 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const uint32_t buf = ebuf0 + (nbox & 1u) * 4096u;
                 if (lane == 0) bulk_wait_read<1>();  // the box that used `buf` two stores ago has been read
                 __syncwarp();
-                uint8_t *rowp = smem_raw + (buf - raw) + lane * 128;
+                if (g.transpose_out) {
+                    // D^T tile: lane = output column (TMEM lane), register p = output row (pixel);
+                    // box row p, column lane, 128B-swizzled: conflict-free 4-byte stores
+                    uint8_t *bp = smem_raw + (buf - raw) + ((lane & 3) << 2);
 #pragma unroll
-                for (int j = 0; j < 8; ++j)
-                    *reinterpret_cast<uint4 *>(rowp + ((j ^ (lane & 7)) << 4)) =
-                        make_uint4(r[4 * j], r[4 * j + 1], r[4 * j + 2], r[4 * j + 3]);
+                    for (int pr = 0; pr < 32; ++pr)
+                        *reinterpret_cast<uint32_t *>(bp + pr * 128 + ((((lane >> 2) ^ (pr & 7))) << 4)) = r[pr];
+                } else {
+                    uint8_t *rowp = smem_raw + (buf - raw) + lane * 128;
+#pragma unroll
+                    for (int j = 0; j < 8; ++j)
+                        *reinterpret_cast<uint4 *>(rowp + ((j ^ (lane & 7)) << 4)) =
+                            make_uint4(r[4 * j], r[4 * j + 1], r[4 * j + 2], r[4 * j + 3]);
+                }
                 fence_async_shared();
                 __syncwarp();
-                if (lane == 0) {
+                if (lane == 0 && g.transpose_out) {
+                    tma_store_3d(&tcm, buf, row0, 0, tc.n_t * BN + c * 32);
+                    bulk_commit();
+                } else if (lane == 0) {
                     const int col0 = tc.n_t * BN + c * 32;
                     if (g.store_mode == STORE_ATOMIC_ADD)
                         tma_reduce_add_3d(&tcm, buf, col0, tc.tap, row0);
@@ -235,6 +301,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     }
     tc_fence_before();
     __syncthreads();
+    if (CS > 1) cluster_sync_all();  // no CTA leaves while peers may still signal its barriers
     tc_fence_after();
     if (warp == 1) tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
 }
@@ -302,6 +369,19 @@ bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint
 }
 
 static int pick_bn(int N) { return N <= 64 ? 64 : (N <= 128 ? 128 : 256); }
+
+// Cluster size for B multicast (K-major, unsplit GEMMs with enough M tiles).  SKIPPER_GEMM_CS
+// overrides the default (1, 2 or 4).
+static int pick_cs(const GemmDev &d) {
+    static int def = -1;
+    if (def < 0) {
+        const char *e = getenv("SKIPPER_GEMM_CS");
+        def = e ? atoi(e) : 2;
+        if (def != 1 && def != 2 && def != 4) def = 2;
+    }
+    if (d.splits != 1 || d.taps != 1 || d.m_tiles < 2 * def) return 1;
+    return def;
+}
 static int cdiv(long long a, long long b) { return (int)((a + b - 1) / b); }
 
 // box geometry covering `rows` consecutive flat rows of an [nb][h][w] image stack
@@ -341,8 +421,9 @@ bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N
     d.N = N;
     d.store_mode = d.splits > 1 ? STORE_SPLIT : STORE_OVERWRITE;
     d.cols_per_tap = 0;
+    g->cs = pick_cs(d);
     // output viewed as [M][splits][N]: slice s at C + s*M*N
-    return make_map_2d(&g->ta, A, K, M, BK, BM) && make_map_2d(&g->tb, B, K, N, BK, g->bn) &&
+    return make_map_2d(&g->ta, A, K, M, BK, BM) && make_map_2d(&g->tb, B, K, N, BK, g->bn / g->cs) &&
            make_map_out(&g->tc, C, N, d.splits, M, (uint64_t)M * N, N);
 }
 
@@ -362,6 +443,7 @@ bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M
     d = GemmDev{};
     g->bn = pick_bn(K);
     g->mn_major = 1;
+    g->cs = 1;
     d.m_tiles = cdiv(N, BM);
     d.n_tiles = cdiv(K, g->bn);
     d.taps = 1;
@@ -383,6 +465,37 @@ bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, i
     // forward: A = X (cin channels), B = Wk [cout][9*cin], out channels cout.
     // dgrad (sign = -1): caller passes X = D (cout channels of the layer) as "cin" and Wt as Wk.
     if (cin % 64 || cout % 8) return false;
+    uint32_t tw, th, tn;
+    if (cout <= 128 && conv_box(h, w, 256, &tw, &th, &tn)) {
+        // Narrow output: compute Y^T = Wk . X^T so the pixels are the 256-wide N side of the tile
+        // (128 x 256 tiles run the tensor cores far better than 128 x 128 / 128 x 64 ones).
+        const long long M = (long long)nb * h * w;
+        GemmDev &d = g->d;
+        d = GemmDev{};
+        g->bn = 256;
+        g->mn_major = 0;
+        g->cs = 1;
+        d.m_tiles = 1;
+        d.n_tiles = cdiv(M, 256);
+        d.taps = 1;
+        d.splits = 1;
+        d.conv_cb = cin / 64;
+        d.num_kb = 9 * d.conv_cb;
+        d.kb_per_split = d.num_kb;
+        d.a_kind = OP_K2D;
+        d.b_kind = OP_KCONV;
+        d.conv_hw = h * w;
+        d.conv_w = w;
+        d.conv_sign = sign;
+        d.transpose_out = 1;
+        d.C = Y;
+        d.ldc = cout;
+        d.M = cout;
+        d.N = (int)M;
+        d.store_mode = STORE_OVERWRITE;
+        return make_map_2d(&g->ta, Wk, 9ull * cin, cout, BK, BM) && make_map_conv(&g->tb, X, cin, w, h, nb, tw, th, tn) &&
+               make_map_out(&g->tc, Y, cout, 1, M, cout, cout);
+    }
     uint32_t bw, bh, bnn;
     if (!conv_box(h, w, BM, &bw, &bh, &bnn)) return false;
     const long long M = (long long)nb * h * w;
@@ -407,7 +520,8 @@ bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, i
     d.M = (int)M;
     d.N = cout;
     d.store_mode = STORE_OVERWRITE;
-    return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn) &&
+    g->cs = pick_cs(d);
+    return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn / g->cs) &&
            make_map_out(&g->tc, Y, cout, 1, M, cout, cout);
 }
 
@@ -419,55 +533,95 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     const long long M = (long long)nb * h * w;
     GemmDev &d = g->d;
     d = GemmDev{};
-    g->bn = pick_bn(cin);
+    // N = (tap, cin) = 9*cin columns in 256-wide tiles; each 64-column chunk is one tap's shifted box
+    g->bn = 256;
     g->mn_major = 1;
+    g->cs = 1;
     d.m_tiles = cdiv(cout, BM);
-    d.n_tiles = cdiv(cin, g->bn);
-    d.taps = 9;
+    d.n_tiles = cdiv(9LL * cin, g->bn);
+    d.taps = 1;
+    d.wg_cin = cin;
     d.num_kb = cdiv(M, BK);
-    choose_splits(d, d.m_tiles * d.n_tiles * 9, num_sms);
+    choose_splits(d, d.m_tiles * d.n_tiles, num_sms);
     d.a_kind = OP_MN2D;
     d.b_kind = OP_MNCONV;
     d.conv_hw = h * w;
     d.conv_w = w;
     d.conv_sign = 1;
-    d.cols_per_tap = cin;
+    d.cols_per_tap = 0;
     d.C = dW;
     d.ldc = 9ll * cin;
     d.M = cout;
-    d.N = cin;
+    d.N = 9 * cin;
     d.store_mode = STORE_ATOMIC_ADD;
     return make_map_2d(&g->ta, D, cout, M, 64, BK) && make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn) &&
-           make_map_out(&g->tc, dW, cin, 9, cout, cin, 9ull * cin);
+           make_map_out(&g->tc, dW, 9ull * cin, 1, cout, 9ull * cin, 9ull * cin);
 }
 
-template <int BN, int MN>
+template <int BN, int MN, int CS>
 static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
     using Cfg = GemmCfg<BN>;
-    static bool attr_done = false;
-    if (!attr_done) {
-        cudaError_t e = cudaFuncSetAttribute(gemm_tc_kernel<BN, MN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)Cfg::SMEM_BYTES);
+    auto kern = gemm_tc_kernel<BN, MN, CS>;
+    static int max_clusters = -1;
+    if (max_clusters < 0) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM_BYTES);
         if (e != cudaSuccess) return e;
-        attr_done = true;
+        max_clusters = num_sms / CS;
+        if (CS > 1) {
+            cudaLaunchConfig_t qc{};
+            qc.gridDim = dim3(CS * max_clusters);
+            qc.blockDim = dim3(NUM_THREADS);
+            qc.dynamicSmemBytes = Cfg::SMEM_BYTES;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = CS;
+            at[0].val.clusterDim.y = 1;
+            at[0].val.clusterDim.z = 1;
+            qc.attrs = at;
+            qc.numAttrs = 1;
+            int n = 0;
+            if (cudaOccupancyMaxActiveClusters(&n, kern, &qc) == cudaSuccess && n > 0) max_clusters = n;
+            cudaGetLastError();
+        }
     }
-    const int total = g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
-    const int grid = total < num_sms ? total : num_sms;
-    gemm_tc_kernel<BN, MN><<<grid, NUM_THREADS, Cfg::SMEM_BYTES, stream>>>(g.ta, g.tb, g.tc, g.d);
-    return cudaGetLastError();
+    const int total = CS > 1 ? ((g.d.m_tiles + CS - 1) / CS) * g.d.n_tiles : g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
+    const int units = total < max_clusters ? total : max_clusters;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(units * CS);
+    cfg.blockDim = dim3(NUM_THREADS);
+    cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
+    cfg.stream = stream;
+    cudaLaunchAttribute attrs[1];
+    attrs[0].id = cudaLaunchAttributeClusterDimension;
+    attrs[0].val.clusterDim.x = CS;
+    attrs[0].val.clusterDim.y = 1;
+    attrs[0].val.clusterDim.z = 1;
+    cfg.attrs = attrs;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, g.ta, g.tb, g.tc, g.d);
 }
 
 cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
     const int total = g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits;
     if (total <= 0) return cudaSuccess;
     if (g.mn_major) {
-        if (g.bn == 64) return launch_t<64, 1>(g, stream, num_sms);
-        if (g.bn == 128) return launch_t<128, 1>(g, stream, num_sms);
-        return launch_t<256, 1>(g, stream, num_sms);
+        if (g.bn == 64) return launch_t<64, 1, 1>(g, stream, num_sms);
+        if (g.bn == 128) return launch_t<128, 1, 1>(g, stream, num_sms);
+        return launch_t<256, 1, 1>(g, stream, num_sms);
     }
-    if (g.bn == 64) return launch_t<64, 0>(g, stream, num_sms);
-    if (g.bn == 128) return launch_t<128, 0>(g, stream, num_sms);
-    return launch_t<256, 0>(g, stream, num_sms);
+    if (g.cs == 4) {
+        if (g.bn == 64) return launch_t<64, 0, 4>(g, stream, num_sms);
+        if (g.bn == 128) return launch_t<128, 0, 4>(g, stream, num_sms);
+        return launch_t<256, 0, 4>(g, stream, num_sms);
+    }
+    if (g.cs == 2) {
+        if (g.bn == 64) return launch_t<64, 0, 2>(g, stream, num_sms);
+        if (g.bn == 128) return launch_t<128, 0, 2>(g, stream, num_sms);
+        return launch_t<256, 0, 2>(g, stream, num_sms);
+    }
+    if (g.bn == 64) return launch_t<64, 0, 1>(g, stream, num_sms);
+    if (g.bn == 128) return launch_t<128, 0, 1>(g, stream, num_sms);
+    return launch_t<256, 0, 1>(g, stream, num_sms);
 }
 
 int device_num_sms() {

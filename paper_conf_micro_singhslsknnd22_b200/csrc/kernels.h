@@ -61,6 +61,28 @@ cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int 
 cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);
 
+// Fused first layer for narrow inputs (layer0.cu): im2col in smem + tcgen05 + LIF + pool + SAM.
+struct L0FwdArgs {
+    const uint8_t *x;      // input spikes [T][B][H][W][C0]
+    int T, B, H, W, C0;
+    const int *row_t;      // absolute t per row (device) or null -> t0 + r
+    int t0, R, restore;    // restore: row 0 is the checkpoint (U_state/o_state), no MMA for it
+    const uint16_t *wbp;   // bf16 weights [N][32] (k = (dy*3+dx)*C0 + ci, zero padded)
+    int N, pool;
+    float lam, theta;
+    float *U_state;        // FIRST/RECORD: running state (in/out); RECOMPUTE: checkpoint (in)
+    uint8_t *o_state;
+    float *U_out;          // [R][B*H*W*N] or null
+    uint16_t *Po_out;      // [R][B*PH*PW*N] bf16
+    float *ckU;            // FIRST: checkpoint slot (after row 0) or null
+    uint8_t *cko;
+    unsigned *s_part;      // SAM partials (input + this layer) or null
+    float *dbg_U;
+    uint8_t *dbg_o;
+};
+bool layer0_supported(int B, int H, int W, int C0, int N, int pool);
+cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms);
+
 // Readout integrator + softmax cross-entropy (reading 5) and its gradients.
 cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int *labels, float *z, float *dz,
                                 float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
