@@ -41,6 +41,7 @@ struct Layer {
     uint16_t *Po = nullptr;    // arena rows
     float *Useg = nullptr;     // arena rows
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
+    int fsplitT = 1;             // forward split-K of the whole-sequence first pass (fc tail layers)
     uint16_t *wbp = nullptr;   // layer 0 im2col: bf16 weights zero-padded to [cout][K0]
     float *dwp = nullptr;      // layer 0 im2col: padded weight gradient
     float *dbg[2] = {nullptr, nullptr};     // first / recompute U
@@ -85,11 +86,19 @@ struct skipper_ctx {
     skipper_allocator alloc{};
     bool own_alloc = true;
     cudaStream_t st = nullptr;
+    // side stream: the weight-gradient GEMM of layer l runs there, overlapping the dgrad of layer l
+    // and the reverse scan of layer l-1 on the main stream (delta is double-buffered)
+    cudaStream_t st2 = nullptr;
+    cudaEvent_t ev_ready[2] = {nullptr, nullptr}, ev_done[2] = {nullptr, nullptr};
+    bool w_pending[2] = {false, false};
     int T = 0, C = 1, S = 0, B = 0, Bg = 0;
     int num_sms = 148;
     int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
     int K0 = 0;                 // im2col width (32 or 64)
     bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
+    int tail0 = 0;              // first layer of the fc tail: the first pass runs it over all T at once
+    uint16_t *tail_in = nullptr, *tailP[2] = {nullptr, nullptr};
+    float *tail_I = nullptr;
     int in_h = 1, in_w = 1, in_c = 0;
     long long in_elems = 0;     // input elements per sample (uint8 x)
     long long in_row = 0;       // staged bf16 layer-0 operand elements per sample
@@ -114,6 +123,7 @@ struct skipper_ctx {
     size_t arena_bytes = 0;
     float *I_buf = nullptr;     // currents (fwd) and gradients wrt spikes (dgrad)
     uint16_t *d_buf = nullptr;  // delta (bf16)
+    uint16_t *d_buf2[2] = {nullptr, nullptr};
     uint16_t *P2[2] = {nullptr, nullptr};
     uint16_t *xg = nullptr;     // staged layer-0 operand rows of the current pass
     // schedule state
@@ -161,23 +171,25 @@ static cudaEvent_t ev_get(skipper_ctx *c) {
 // context stream together with its algorithmic bytes / flops.
 struct ProfScope {
     skipper_ctx *c;
+    cudaStream_t s;
     int rec = -1;
-    ProfScope(skipper_ctx *c_, int cls, double bytes, double flops) : c(c_) {
+    ProfScope(skipper_ctx *c_, int cls, double bytes, double flops, cudaStream_t s_ = nullptr) : c(c_), s(s_) {
+        if (!s) s = c->st;
         c->launches++;
         if (!c->prof_on) return;
         cudaEvent_t a = ev_get(c), b = ev_get(c);
-        cudaEventRecord(a, c->st);
+        cudaEventRecord(a, s);
         c->prof_recs.push_back({cls, a, b, bytes, flops});
         rec = (int)c->prof_recs.size() - 1;
     }
     ~ProfScope() {
-        if (rec >= 0) cudaEventRecord(c->prof_recs[rec].b, c->st);
+        if (rec >= 0) cudaEventRecord(c->prof_recs[rec].b, s);
     }
 };
 
 static void prof_resolve(skipper_ctx *c) {
     if (c->prof_recs.empty()) return;
-    cudaEventSynchronize(c->prof_recs.back().b);
+    for (auto &r : c->prof_recs) cudaEventSynchronize(r.b);
     for (auto &r : c->prof_recs) {
         float ms = 0.f;
         if (cudaEventElapsedTime(&ms, r.a, r.b) == cudaSuccess) {
@@ -465,6 +477,12 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     c->S = c->T / c->C;
     c->num_sms = sk::device_num_sms();
+    if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess)
+        return bail(fail(c, SKIPPER_ECUDA, "side stream creation failed"));
+    for (int k = 0; k < 2; ++k)
+        if (cudaEventCreateWithFlags(&c->ev_ready[k], cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_done[k], cudaEventDisableTiming) != cudaSuccess)
+            return bail(fail(c, SKIPPER_ECUDA, "event creation failed"));
     {
         const Layer &f = c->L[0];
         const char *e = getenv("SKIPPER_NO_L0_FUSION");
@@ -476,8 +494,15 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         if (!l.fc) continue;
         const int rowsM = c->S * c->B;
         l.fsplit = fc_splits(rowsM, l.Cout, l.Cin, c->num_sms);
+        l.fsplitT = fc_splits(c->T * c->B, l.Cout, l.Cin, c->num_sms);
         if (i > 0) l.dsplit = fc_splits(rowsM, l.Cin, l.Cout, c->num_sms);
     }
+    // The fc tail (a few thousand neurons per sample) would run as tiny latency-bound launches per
+    // segment; in the first pass it is evaluated layer-major over the whole sequence instead (its
+    // recurrences still run in time order; checkpoints are written every S rows).
+    c->tail0 = c->Ls;
+    while (c->tail0 > 0 && c->L[c->tail0 - 1].fc) --c->tail0;
+    if (cfg->mode == SKIPPER_MODE_FULL) c->tail0 = c->Ls;
 
     // ---- persistent allocations
     c->dw_total = 0;
@@ -592,6 +617,14 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
     }
     if (c->st) cudaStreamSynchronize(c->st);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
+    if (c->st2) {
+        cudaStreamSynchronize(c->st2);
+        cudaStreamDestroy(c->st2);
+    }
+    for (int k = 0; k < 2; ++k) {
+        if (c->ev_ready[k]) cudaEventDestroy(c->ev_ready[k]);
+        if (c->ev_done[k]) cudaEventDestroy(c->ev_done[k]);
+    }
     c->comm.destroy();
     delete c;
 }
@@ -679,8 +712,11 @@ static skipper_status arena_free(skipper_ctx *c) {
     }
     c->I_buf = nullptr;
     c->d_buf = nullptr;
+    c->d_buf2[0] = c->d_buf2[1] = nullptr;
     c->P2[0] = c->P2[1] = nullptr;
     c->xg = nullptr;
+    c->tail_in = c->tailP[0] = c->tailP[1] = nullptr;
+    c->tail_I = nullptr;
     return SKIPPER_OK;
 }
 
@@ -690,7 +726,20 @@ static skipper_status arena_first(skipper_ctx *c) {
     const size_t pbytes = al256(rowsB * max_nout(c) * 2);
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
-    c->arena_bytes = 2 * pbytes + ibytes + xbytes;
+    // fc tail over all T rows: its input rows, ping-pong outputs, currents (with split partials)
+    size_t tin = 0, tp = 0, ti = 0;
+    if (c->tail0 < c->Ls) {
+        const size_t rowsT = (size_t)c->T * c->B;
+        tin = al256(rowsT * (c->tail0 == 0 ? c->in_row : c->L[c->tail0 - 1].Nout) * 2);
+        long long mo = 0, mi = 0;
+        for (int i = c->tail0; i < c->Ls; ++i) {
+            mo = std::max(mo, c->L[i].Nout);
+            mi = std::max(mi, c->L[i].N * c->L[i].fsplitT);
+        }
+        tp = al256(rowsT * mo * 2);
+        ti = al256(rowsT * mi * 4);
+    }
+    c->arena_bytes = 2 * pbytes + ibytes + xbytes + tin + 2 * tp + ti;
     c->arena = dev_alloc(c, c->arena_bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "first-pass arena of %zu bytes", c->arena_bytes);
     char *p = static_cast<char *>(c->arena);
@@ -698,6 +747,11 @@ static skipper_status arena_first(skipper_ctx *c) {
     c->P2[1] = reinterpret_cast<uint16_t *>(p + pbytes);
     c->I_buf = reinterpret_cast<float *>(p + 2 * pbytes);
     c->xg = reinterpret_cast<uint16_t *>(p + 2 * pbytes + ibytes);
+    char *q = p + 2 * pbytes + ibytes + xbytes;
+    c->tail_in = tin ? reinterpret_cast<uint16_t *>(q) : nullptr;
+    c->tailP[0] = tp ? reinterpret_cast<uint16_t *>(q + tin) : nullptr;
+    c->tailP[1] = tp ? reinterpret_cast<uint16_t *>(q + tin + tp) : nullptr;
+    c->tail_I = ti ? reinterpret_cast<float *>(q + tin + 2 * tp) : nullptr;
     return SKIPPER_OK;
 }
 
@@ -709,7 +763,7 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t dbytes = al256(rowsB * max_n(c) * 2);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
-    bytes += ibytes + dbytes + xbytes;
+    bytes += ibytes + 2 * dbytes + xbytes;
     c->arena_bytes = bytes;
     c->arena = dev_alloc(c, bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "segment arena of %zu bytes (%d rows)", bytes, R);
@@ -724,7 +778,9 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     c->I_buf = reinterpret_cast<float *>(p);
     p += ibytes;
     c->d_buf = reinterpret_cast<uint16_t *>(p);
-    p += dbytes;
+    c->d_buf2[0] = c->d_buf;
+    c->d_buf2[1] = reinterpret_cast<uint16_t *>(p + dbytes);
+    p += 2 * dbytes;
     c->xg = reinterpret_cast<uint16_t *>(p);
     return SKIPPER_OK;
 }
@@ -744,16 +800,18 @@ static bool get_plan(skipper_ctx *c, const PlanKey &k, sk::GemmLaunch &g, const 
 }
 
 static skipper_status run_gemm(skipper_ctx *c, const sk::GemmLaunch &g, bool ok, const char *what, int layer,
-                               int cls, double bytes, double flops) {
+                               int cls, double bytes, double flops, cudaStream_t s = nullptr) {
     if (!ok) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: cannot plan %s GEMM (tensor map)", layer, what);
-    ProfScope ps(c, cls, bytes, flops);
-    CK(sk::gemm_run(g, c->st, c->num_sms));
+    if (!s) s = c->st;
+    ProfScope ps(c, cls, bytes, flops, s);
+    CK(sk::gemm_run(g, s, c->num_sms));
     return SKIPPER_OK;
 }
 
 // I rows = input rows x W^T for spiking layer i over `rows` timestep rows.
-static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, float *I, int rows) {
+static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, float *I, int rows, int splits = -1) {
     Layer &l = c->L[i];
+    const int fsp = splits > 0 ? splits : l.fsplit;
     if (rows <= 0) return SKIPPER_OK;
     sk::GemmLaunch g;
     const int nb = rows * c->B;
@@ -766,12 +824,12 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
             return sk::plan_conv(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
         });
     else
-        ok = get_plan(c, {0, in, l.wb, I, nb, l.Cout, l.Cin, 0, 0, l.fsplit}, g, [&](sk::GemmLaunch *p) {
-            return sk::plan_fc(p, in, l.wb, I, nb, l.Cout, l.Cin, l.fsplit);
+        ok = get_plan(c, {0, in, l.wb, I, nb, l.Cout, l.Cin, 0, 0, fsp}, g, [&](sk::GemmLaunch *p) {
+            return sk::plan_fc(p, in, l.wb, I, nb, l.Cout, l.Cin, fsp);
         });
-    if (ok && g.d.splits != (l.fc ? l.fsplit : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
+    if (ok && g.d.splits != (l.fc ? fsp : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
     const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
-    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4 * l.fsplit;
+    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4 * (l.fc ? fsp : 1);
     return run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, bytes, 2.0 * M * l.Cout * K);
 }
 
@@ -830,6 +888,51 @@ static skipper_status stage_input(skipper_ctx *c, const int *rows, int t0, int R
     return SKIPPER_OK;
 }
 
+// First pass of the fc tail over all T rows (layer-major): GEMM with M = T*B, one scan per layer.
+static skipper_status forward_tail_first(skipper_ctx *c) {
+    if (c->tail0 >= c->Ls) return SKIPPER_OK;
+    const int T = c->T;
+    if (c->tail0 == 0) {
+        uint16_t *save = c->xg;
+        c->xg = c->tail_in;
+        skipper_status st = stage_input(c, nullptr, 0, T, true);
+        c->xg = save;
+        CKS(st);
+    }
+    for (int i = c->tail0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        const uint16_t *in = i == c->tail0 ? c->tail_in : c->tailP[(i - c->tail0 - 1) & 1];
+        uint16_t *out = c->tailP[(i - c->tail0) & 1];
+        CKS(gemm_forward(c, i, in, c->tail_I, T, l.fsplitT));
+        sk::ScanFwdArgs a{};
+        a.I = c->tail_I;
+        a.nsplit = l.fsplitT;
+        a.split_stride = (long long)T * c->B * l.N;
+        a.R = T;
+        a.U_state = l.U_run;
+        a.o_state = l.o_run;
+        a.Po_out = out;
+        a.ckU = l.ckU;
+        a.cko = l.cko;
+        a.ck_every = c->S;
+        a.s_part = c->s_part;
+        a.t0 = 0;
+        a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
+        a.dbg_U = c->cfg.debug_record ? l.dbg[0] : nullptr;
+        a.dbg_o = c->cfg.debug_record ? l.dbgo[0] : nullptr;
+        a.B = c->B;
+        a.H = l.H;
+        a.W = l.W;
+        a.C = l.Cout;
+        a.pool = l.pool ? 1 : 0;
+        a.lam = l.d.lambda;
+        a.theta = l.d.theta;
+        ProfScope ps(c, K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
+        CK(sk::launch_lif_fwd(a, c->st));
+    }
+    return SKIPPER_OK;
+}
+
 // Layer 0 as one fused kernel: im2col in smem, tcgen05, LIF, pooling, SAM, checkpoint (layer0.cu).
 static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const int *row_t, bool restore,
                                    bool record, uint16_t *out) {
@@ -869,10 +972,11 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
 
 // Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
 static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
-    // the staged layer-0 operand is needed by the first pass unless layer 0 is fused, and by the
-    // layer-0 weight gradient of FULL mode
-    if (!c->l0_fused || record) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
-    for (int i = 0; i < c->Ls; ++i) {
+    // the staged layer-0 operand is needed by the first pass unless layer 0 is fused (or part of the
+    // whole-sequence fc tail), and by the layer-0 weight gradient of FULL mode
+    const int iend = record ? c->Ls : c->tail0;
+    if (record || (iend > 0 && !c->l0_fused)) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
+    for (int i = 0; i < iend; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in;
         uint16_t *out;
@@ -881,7 +985,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
             out = l.Po;
         } else {
             in = i == 0 ? c->xg : c->P2[(i - 1) & 1];
-            out = c->P2[i & 1];
+            out = (i == c->tail0 - 1) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i & 1];
         }
         if (i == 0 && c->l0_fused) {
             CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));
@@ -1010,9 +1114,24 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
 }
 
 // Eq.2 backward over the R stored rows of a segment (layer-major, reverse t inside the scan).
+static skipper_status join_wgrads(skipper_ctx *c) {
+    for (int k = 0; k < 2; ++k)
+        if (c->w_pending[k]) {
+            CK(cudaStreamWaitEvent(c->st, c->ev_done[k], 0));
+            c->w_pending[k] = false;
+        }
+    return SKIPPER_OK;
+}
+
 static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
     for (int i = c->Ls - 1; i >= 0; --i) {
         Layer &l = c->L[i];
+        const int par = i & 1;
+        uint16_t *dcur = c->d_buf2[par];
+        if (c->w_pending[par]) {  // the wgrad of layer i+2 still reads this delta buffer
+            CK(cudaStreamWaitEvent(c->st, c->ev_done[par], 0));
+            c->w_pending[par] = false;
+        }
         sk::ScanBwdArgs a{};
         a.g = (i == c->Ls - 1) ? c->g_last : c->I_buf;
         a.nsplit = (i == c->Ls - 1) ? 1 : c->L[i + 1].dsplit;  // dgrad of layer i+1 produced g
@@ -1021,7 +1140,7 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         a.g_pooled = l.pool ? 1 : 0;
         a.U = l.Useg;
         a.carry = l.carry;
-        a.delta = c->d_buf;
+        a.delta = dcur;
         a.R = R;
         a.B = c->B;
         a.H = l.H;
@@ -1041,40 +1160,45 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         sk::GemmLaunch g;
         bool ok;
         if (i == 0 && c->in_kind == 1)
-            ok = get_plan(c, {2, c->d_buf, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
+            ok = get_plan(c, {2, dcur, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
                           [&](sk::GemmLaunch *p) {
-                              return sk::plan_fc_wgrad(p, c->d_buf, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
+                              return sk::plan_fc_wgrad(p, dcur, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
                           });
         else if (l.conv)
-            ok = get_plan(c, {3, c->d_buf, X, l.dw, nb, l.Cin, l.Cout, l.H, l.W, 0}, g, [&](sk::GemmLaunch *p) {
-                return sk::plan_conv_wgrad(p, c->d_buf, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
+            ok = get_plan(c, {3, dcur, X, l.dw, nb, l.Cin, l.Cout, l.H, l.W, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_conv_wgrad(p, dcur, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
             });
         else
-            ok = get_plan(c, {2, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
-                return sk::plan_fc_wgrad(p, c->d_buf, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
+            ok = get_plan(c, {2, dcur, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_fc_wgrad(p, dcur, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
             });
-        {
+        {   // weight gradient on the side stream, after this layer's delta is written
+            CK(cudaEventRecord(c->ev_ready[par], c->st));
+            CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
             const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
             const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
-            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K));
+            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K, c->st2));
+            CK(cudaEventRecord(c->ev_done[par], c->st2));
+            c->w_pending[par] = true;
         }
         if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
             if (l.conv)
-                ok = get_plan(c, {1, c->d_buf, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g,
+                ok = get_plan(c, {1, dcur, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g,
                               [&](sk::GemmLaunch *p) {
-                                  return sk::plan_conv(p, c->d_buf, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
+                                  return sk::plan_conv(p, dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1);
                               });
             else
-                ok = get_plan(c, {0, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, 0, 0, l.dsplit}, g,
+                ok = get_plan(c, {0, dcur, l.wt, c->I_buf, nb, l.Cin, l.Cout, 0, 0, l.dsplit}, g,
                               [&](sk::GemmLaunch *p) {
-                                  return sk::plan_fc(p, c->d_buf, l.wt, c->I_buf, nb, l.Cin, l.Cout, l.dsplit);
+                                  return sk::plan_fc(p, dcur, l.wt, c->I_buf, nb, l.Cin, l.Cout, l.dsplit);
                               });
             const double M = (double)nb * l.H * l.W, K = (double)l.Cout * (l.conv ? 9 : 1);
             const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4 * l.dsplit;
             CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * (l.Nin / (l.H * l.W)) * K));
         }
     }
-    return SKIPPER_OK;
+    // the next segment reuses the arena (X operands, delta buffers): wait for the weight gradients
+    return join_wgrads(c);
 }
 
 // ------------------------------------------------------------------------------------ public schedule
@@ -1111,6 +1235,7 @@ extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int p
         c->next_seg = seg + 1;
         if (seg == c->C - 1) {
             if (!labels_dev) return fail(c, SKIPPER_EINVAL, "the last FIRST segment needs labels");
+            CKS(forward_tail_first(c));
             CKS(finish_first(c, labels_dev));
             CKS(arena_rows(c, c->Kmax));
             c->phase = PH_READY_BWD;
@@ -1334,12 +1459,29 @@ extern "C" skipper_status skipper_comm_init(skipper_ctx *c, const unsigned char 
 
 // ------------------------------------------------------------------------------------ kernel-level API
 // (include/skipper_kernels.h) - the same launchers skipper_step uses, for per-kernel parity tests.
-static int kapi_run(const sk::GemmLaunch &g, bool ok, void *stream, const char *what) {
+static int kapi_run(const sk::GemmLaunch &g0, bool ok, void *stream, const char *what) {
     if (!ok) {
         g_last_error = std::string(what) + ": unsupported shape or tensor-map failure";
         return SKIPPER_EUNSUPPORTED;
     }
+    sk::GemmLaunch g = g0;
+    static unsigned long long *stats = nullptr;
+    const char *se = getenv("SKIPPER_GEMM_STATS");
+    if (se && atoi(se)) {  // diagnostics: per-role barrier wait cycles of this launch
+        if (!stats) cudaMalloc(&stats, 8 * sizeof(unsigned long long));
+        cudaMemsetAsync(stats, 0, 8 * sizeof(unsigned long long), static_cast<cudaStream_t>(stream));
+        g.d.stats = stats;
+    }
     cudaError_t e = sk::gemm_run(g, static_cast<cudaStream_t>(stream), sk::device_num_sms());
+    if (g.d.stats && e == cudaSuccess) {
+        unsigned long long h[8];
+        cudaMemcpyAsync(h, stats, sizeof h, cudaMemcpyDeviceToHost, static_cast<cudaStream_t>(stream));
+        cudaStreamSynchronize(static_cast<cudaStream_t>(stream));
+        const double cta = (double)h[3];
+        fprintf(stderr, "[gemm-stats %s] bn=%d mn=%d cs=%d tiles=%d kb=%d: producer<-empty %.2f  mma<-tmem %.2f  mma<-data %.2f  epi<-acc %.2f (fractions of CTA cycles)\n",
+                what, g.bn, g.mn_major, g.cs, g.d.m_tiles * g.d.n_tiles * g.d.taps * g.d.splits, g.d.kb_per_split,
+                h[0] / cta, h[1] / cta, h[4] / cta, h[2] / (4 * cta));
+    }
     if (e != cudaSuccess) {
         g_last_error = std::string(what) + ": " + cudaGetErrorString(e);
         return SKIPPER_ECUDA;

@@ -37,6 +37,7 @@ struct GemmDev {
     long long ldc;
     int M, N;           // valid output extent (rows, columns of one tap block)
     int store_mode;
+    unsigned long long *stats;  // optional pipeline wait statistics (null in production)
 };
 
 struct GemmLaunch {

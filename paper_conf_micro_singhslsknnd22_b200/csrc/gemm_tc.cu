@@ -75,6 +75,17 @@ SK_DEV TileCoord decode_tile(const GemmDev &g, int tile) {
     return c;
 }
 
+// Optional pipeline statistics (g.stats != null): cycles each role spends blocked on its barrier.
+SK_DEV void mbar_wait_t(uint32_t bar, uint32_t parity, unsigned long long *acc) {
+    if (acc) {
+        const long long t0 = clock64();
+        mbar_wait(bar, parity);
+        *acc += (unsigned long long)(clock64() - t0);
+    } else {
+        mbar_wait(bar, parity);
+    }
+}
+
 template <int BN, int MN, int CS>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
@@ -95,6 +106,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
+    unsigned long long w_stat = 0, *wst = g.stats ? &w_stat : nullptr;
+    const long long t_start = clock64();
 
     if (warp == 0 && lane == 0) {
         tma_prefetch(&ta);
@@ -134,7 +147,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const TileCoord tc = tile_at<CS>(g, tile, rank);
                 const int tdy = tc.tap / 3 - 1, tdx = tc.tap % 3 - 1;
                 for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
-                    mbar_wait(empty_bar(stage), phase ^ 1u);
+                    mbar_wait_t(empty_bar(stage), phase ^ 1u, wst);
                     const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                     const uint32_t sb = sa + Cfg::A_BYTES;
                     const uint32_t fb = full_bar(stage);
@@ -204,11 +217,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             uint32_t acc_phase = 0;
             for (int tile = it0; tile < total; tile += itstep) {
                 const TileCoord tc = tile_at<CS>(g, tile, rank);
-                mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
+                mbar_wait_t(tempty_bar(acc), acc_phase ^ 1u, wst);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + acc * BN;
                 for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
-                    mbar_wait(full_bar(stage), phase);
+                    if (wst) {  // MMA waiting on TMA data is accounted separately (slot 4)
+                        unsigned long long f = 0;
+                        mbar_wait_t(full_bar(stage), phase, &f);
+                        atomicAdd(g.stats + 4, f);
+                    } else {
+                        mbar_wait(full_bar(stage), phase);
+                    }
                     tc_fence_after();
                     const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                     const uint32_t sb = sa + Cfg::A_BYTES;
@@ -251,7 +270,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         uint32_t nbox = 0;
         for (int tile = it0; tile < total; tile += itstep) {
             const TileCoord tc = tile_at<CS>(g, tile, rank);
-            mbar_wait(tfull_bar(acc), acc_phase);
+            mbar_wait_t(tfull_bar(acc), acc_phase, lane == 0 ? wst : nullptr);
             tc_fence_after();
             const int row0 = tc.m_t * BM + q * 32;
 #pragma unroll 1
@@ -298,6 +317,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             if (acc == 0) acc_phase ^= 1u;
         }
         if (lane == 0) bulk_wait<0>();
+    }
+    if (g.stats && lane == 0) {
+        // slots: 0 producer<-empty, 1 MMA<-tempty, 2 epilogue<-tfull (sum of 4 warps), 3 CTA cycles,
+        // 4 MMA<-full (TMA data)
+        const int slot = warp == 0 ? 0 : (warp == 1 ? 1 : 2);
+        atomicAdd(g.stats + slot, w_stat);
+        if (warp == 0) atomicAdd(g.stats + 3, (unsigned long long)(clock64() - t_start));
     }
     tc_fence_before();
     __syncthreads();

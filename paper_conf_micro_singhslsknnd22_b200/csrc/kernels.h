@@ -22,6 +22,7 @@ struct ScanFwdArgs {
     uint16_t *Po_out;      // [R][B*Nout] bf16 layer output (pooled if pool) - next GEMM operand
     float *ckU;            // FIRST: checkpoint slot written after row 0, else null
     uint8_t *cko;
+    int ck_every;          // >0: rows r % ck_every == 0 write checkpoint slot r / ck_every (whole-T scans)
     unsigned *s_part;      // SAM partials [T][32] or null (FIRST/RECORD only)
     const int *row_t;      // absolute t of each row (device) or null -> t0 + r
     int t0;

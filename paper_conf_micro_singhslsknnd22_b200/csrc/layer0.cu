@@ -184,11 +184,12 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                     const uint32_t v1 = __funnelshift_r(cw[dy][1], cw[dy][2], 8 * cshift);
                     const uint32_t v2 = __funnelshift_r(cw[dy][2], cw[dy][3], 8 * cshift);
                     const uint32_t v[3] = {v0, v1, v2};
-                    for (int j = 0; j < 3 * a.C0; ++j) {
-                        const uint32_t byte = (v[j >> 2] >> (8 * (j & 3))) & 0xFFu;
-                        if (byte) {
-                            m |= 1u << (dy * 3 * a.C0 + j);
-                            if (dy == 1 && j >= a.C0 && j < 2 * a.C0) ++cnt;
+#pragma unroll
+                    for (int j = 0; j < 9; ++j) {  // 3*C0 <= 9 window bytes of this input row
+                        if (j < 3 * a.C0) {
+                            const uint32_t nz = ((v[j >> 2] >> (8 * (j & 3))) & 0xFFu) ? 1u : 0u;
+                            m |= nz << (dy * 3 * a.C0 + j);
+                            if (dy == 1) cnt += (j >= a.C0 && j < 2 * a.C0) ? nz : 0u;
                         }
                     }
                 }
@@ -302,15 +303,17 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                     const uint32_t twos = cc0 ^ cc1 ^ k01, fours = cc0 & cc1;
                     const int sub = lane & 3;
                     uint32_t pk[4];
+                    const uint32_t o8 = (ones >> (sub * 8)) & 0xFFu, t8 = (twos >> (sub * 8)) & 0xFFu;
+                    const uint32_t f8 = (fours >> (sub * 8)) & 0xFFu;
 #pragma unroll
                     for (int e = 0; e < 4; ++e) {
                         uint32_t v2 = 0;
 #pragma unroll
                         for (int hh = 0; hh < 2; ++hh) {
-                            const int ch = sub * 8 + 2 * e + hh;
-                            const int n = ((ones >> ch) & 1u) + 2 * ((twos >> ch) & 1u) + 4 * ((fours >> ch) & 1u);
-                            const uint32_t bits = n == 0 ? 0u : (n == 1 ? 0x3E80u : (n == 2 ? 0x3F00u : (n == 3 ? 0x3F40u : 0x3F80u)));
-                            v2 |= bits << (16 * hh);
+                            const int ch = 2 * e + hh;
+                            const uint32_t n = ((o8 >> ch) & 1u) + 2u * ((t8 >> ch) & 1u) + 4u * ((f8 >> ch) & 1u);
+                            // n/4 is exact in bf16: its bits are the top half of the fp32 bits
+                            v2 |= (__float_as_uint(__uint2float_rn(n) * 0.25f) >> 16) << (16 * hh);
                         }
                         pk[e] = v2;
                     }

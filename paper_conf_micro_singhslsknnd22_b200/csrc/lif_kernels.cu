@@ -33,17 +33,36 @@ SK_DEV uint2 pack_bf16x4(float a, float b, float c, float d) {
 
 SK_DEV float4 ldg4(const float *p) { return __ldg(reinterpret_cast<const float4 *>(p)); }
 
+static constexpr int MAX_SPLIT = 8;
+
 // Sum of the split-K partial slices in fixed order s = 0, 1, ... (deterministic, identical in the
-// first pass and the recompute because the split count is a per-layer constant).
+// first pass and the recompute because the split count is a per-layer constant).  All partial
+// loads are issued before the (ordered) additions.
 SK_DEV float4 ldg4_split(const float *p, int nsplit, long long stride) {
-    float4 v = ldg4(p);
-    for (int s = 1; s < nsplit; ++s) {
-        const float4 w = ldg4(p + s * stride);
-        v.x = __fadd_rn(v.x, w.x);
-        v.y = __fadd_rn(v.y, w.y);
-        v.z = __fadd_rn(v.z, w.z);
-        v.w = __fadd_rn(v.w, w.w);
+    float4 w[MAX_SPLIT];
+#pragma unroll
+    for (int s = 0; s < MAX_SPLIT; ++s)
+        w[s] = s < nsplit ? ldg4(p + s * stride) : make_float4(0.f, 0.f, 0.f, 0.f);
+    float4 v = w[0];
+#pragma unroll
+    for (int s = 1; s < MAX_SPLIT; ++s) {
+        if (s < nsplit) {
+            v.x = __fadd_rn(v.x, w[s].x);
+            v.y = __fadd_rn(v.y, w[s].y);
+            v.z = __fadd_rn(v.z, w[s].z);
+            v.w = __fadd_rn(v.w, w[s].w);
+        }
     }
+    return v;
+}
+SK_DEV float ldg_split(const float *p, int nsplit, long long stride) {
+    float w[MAX_SPLIT];
+#pragma unroll
+    for (int s = 0; s < MAX_SPLIT; ++s) w[s] = s < nsplit ? __ldg(p + s * stride) : 0.f;
+    float v = w[0];
+#pragma unroll
+    for (int s = 1; s < MAX_SPLIT; ++s)
+        if (s < nsplit) v = __fadd_rn(v, w[s]);
     return v;
 }
 
@@ -180,11 +199,12 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
                 ob = nb;
                 nspk = __popc(ob);
                 emit_row(r);
-                if (a.ckU && r == 0) {
+                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0)) {
+                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * rs : 0;
 #pragma unroll
                     for (int k = 0; k < NP; ++k) {
-                        *reinterpret_cast<float4 *>(a.ckU + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
-                        *reinterpret_cast<uchar4 *>(a.cko + nidx[k]) =
+                        *reinterpret_cast<float4 *>(a.ckU + slot + nidx[k]) = make_float4(U[k][0], U[k][1], U[k][2], U[k][3]);
+                        *reinterpret_cast<uchar4 *>(a.cko + slot + nidx[k]) =
                             make_uchar4((unsigned char)bit(k, 0), (unsigned char)bit(k, 1), (unsigned char)bit(k, 2),
                                         (unsigned char)bit(k, 3));
                     }
@@ -223,8 +243,96 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
     }
 }
 
+// Small unpooled layers (fc): one thread per neuron so that a 64k-neuron row still fills the GPU;
+// the split-K partial currents of CH rows are all in flight before the recurrence consumes them.
+template <int CH, int SPLIT>
+__global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a) {
+    extern __shared__ unsigned s_cnt[];
+    const long long rs = (long long)a.B * a.H * a.W * a.C;
+    const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool active = n < rs;
+    if (a.s_part) {
+        for (int r = threadIdx.x; r < a.R; r += blockDim.x) s_cnt[r] = 0;
+        __syncthreads();
+    }
+    float U = active ? a.U_state[n] : 0.f;
+    float o = (active && a.o_state[n]) ? 1.f : 0.f;
+    float cacc = 0.f;
+    auto emit = [&](int r) {
+        a.Po_out[(long long)r * rs + n] = o != 0.f ? (uint16_t)0x3F80 : (uint16_t)0;
+        cacc += o;
+        if (a.U_out) a.U_out[(long long)r * rs + n] = U;
+        if (a.dbg_U) {
+            const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+            a.dbg_U[t * rs + n] = U;
+            a.dbg_o[t * rs + n] = o != 0.f ? 1 : 0;
+        }
+    };
+    int r0 = 0;
+    if (a.restore) {
+        if (active) emit(0);
+        r0 = 1;
+    }
+    const int lane = threadIdx.x & 31;
+    for (int rb = r0; rb < a.R; rb += CH) {
+        float Iv[CH];
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb + j;
+            const float *src = a.I + (long long)r * rs + n;
+            Iv[j] = (active && r < a.R) ? (SPLIT ? ldg_split(src, a.nsplit, a.split_stride) : __ldg(src)) : 0.f;
+        }
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb + j;
+            if (r >= a.R) break;
+            unsigned spk = 0;
+            if (active) {
+                U = lif_update(U, Iv[j], o, a.lam, a.theta);
+                o = U > a.theta ? 1.f : 0.f;
+                spk = o != 0.f ? 1u : 0u;
+                emit(r);
+                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0)) {
+                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * rs : 0;
+                    a.ckU[slot + n] = U;
+                    a.cko[slot + n] = (uint8_t)spk;
+                }
+            }
+            if (a.s_part) {
+                const unsigned v = __reduce_add_sync(0xffffffffu, spk);
+                if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
+            }
+        }
+    }
+    if (active) {
+        if (!a.restore) {
+            a.U_state[n] = U;
+            a.o_state[n] = o != 0.f ? 1 : 0;
+        }
+        if (a.cnt) a.cnt[n] += cacc;
+    }
+    if (a.s_part) {
+        __syncthreads();
+        for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
+            const unsigned v = s_cnt[r];
+            const long long t = a.row_t ? a.row_t[r] : a.t0 + r;
+            if (v) atomicAdd(a.s_part + t * 32 + (blockIdx.x & 31), v);
+        }
+    }
+}
+
 cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
+    if (!a.pool && a.H * a.W == 1 && (long long)a.B * a.C <= (1LL << 20)) {  // fc layers
+        const long long rs = (long long)a.B * a.C;
+        const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
+        if (smem > 48 * 1024) return cudaErrorInvalidValue;
+        if (a.nsplit > 1)
+            lif_fwd_small_kernel<4, 1><<<(unsigned)((rs + 255) / 256), 256, smem, s>>>(a);
+        else
+            lif_fwd_small_kernel<16, 0><<<(unsigned)((rs + 255) / 256), 256, smem, s>>>(a);
+        return cudaGetLastError();
+    }
     const long long HW = (long long)a.H * a.W;
     const long long P = a.pool ? (long long)a.B * (a.H / 2) * (a.W / 2) * (a.C / 4) : (long long)a.B * HW * (a.C / 4);
     const int threads = 256;
@@ -296,10 +404,49 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
     *reinterpret_cast<float4 *>(a.carry + n0) = d;
 }
 
+// Small unpooled layers (fc): one thread per neuron (see lif_fwd_small_kernel).
+template <int CH, int SPLIT>
+__global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a) {
+    const long long rs = (long long)a.B * a.C;
+    const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (n >= rs) return;
+    const long long grs = a.g_broadcast ? 0 : rs;
+    float d = a.carry[n];
+    for (int rb = a.R - 1; rb >= 0; rb -= CH) {
+        float gv[CH], uv[CH];
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb - j;
+            gv[j] = uv[j] = 0.f;
+            if (r >= 0) {
+                const float *src = a.g + (long long)r * grs + n;
+                gv[j] = SPLIT ? ldg_split(src, a.nsplit, a.split_stride) : __ldg(src);
+                uv[j] = __ldg(a.U + (long long)r * rs + n);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < CH; ++j) {
+            const int r = rb - j;
+            if (r >= 0) {
+                d = surrogate(uv[j], a.theta, a.surr, a.gamma) * gv[j] + a.lam * d;
+                if (a.delta) a.delta[(long long)r * rs + n] = f2bf_bits(d);
+            }
+        }
+    }
+    a.carry[n] = d;
+}
+
 cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     if (rs == 0 || a.R == 0) return cudaSuccess;
+    if (!a.g_pooled && a.H * a.W == 1 && rs <= (1LL << 20)) {  // fc layers
+        if (a.nsplit > 1)
+            lif_bwd_small_kernel<4, 1><<<(unsigned)((rs + 255) / 256), 256, 0, s>>>(a);
+        else
+            lif_bwd_small_kernel<16, 0><<<(unsigned)((rs + 255) / 256), 256, 0, s>>>(a);
+        return cudaGetLastError();
+    }
     const long long P = rs / 4;
     if (a.nsplit > 1)
         lif_bwd_kernel<1><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
