@@ -166,7 +166,10 @@ def config_block(args, wl, net):
 
 
 # ------------------------------------------------------------------------------------- GPU arm
-def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=False, e2e=False):
+def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=False, e2e=False, steps=None,
+             warmup=None):
+    steps = steps or args.steps
+    warmup = warmup or args.warmup
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
     T, B, C, p = wl["T"], wl["B"], wl["C"], wl["p"]
     x, y = synth.make_inputs(net, T, B, seed=1 + 1000 * rank)
@@ -180,7 +183,7 @@ def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=
     xd = torch.from_numpy(x).cuda()
     yd = torch.from_numpy(y).cuda()
     flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device="cuda")
-    for _ in range(args.warmup):
+    for _ in range(warmup):
         m.step(xd, yd, want_loss=False)
     torch.cuda.synchronize()
     m.reset_peak()
@@ -193,7 +196,7 @@ def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
     evs = []
-    for _ in range(args.steps):
+    for _ in range(steps):
         flush.zero_()
         a = torch.cuda.Event(enable_timing=True)
         b = torch.cuda.Event(enable_timing=True)
@@ -325,6 +328,23 @@ def run_ours(args):
                                  "ms_per_step": r["total_ms"] / args.steps, "peak_hbm_gb": r["peak_lib"] / 1e9}
             except Exception as e:  # noqa: BLE001
                 compare[mode] = {"error": str(e)[:200]}
+    # peak HBM and throughput vs T (the metric's "vs T"): Skipper vs full BPTT, segment length S fixed
+    t_sweep = {}
+    if not args.no_compare and args.t_sweep:
+        S = wl["T"] // wl["C"]
+        for T in [int(v) for v in args.t_sweep.split(",") if v]:
+            if T % S:
+                continue
+            w2 = dict(wl, T=T, C=T // S)
+            row = {}
+            for mode in ("skip", "full"):
+                try:
+                    r = run_mode(torch, dist, args, w2, net, mode, rank, world, local_rank, steps=3, warmup=3)
+                    row[mode] = {"samples_per_s": w2["B"] * world * 3 / (r["total_ms"] / 1e3),
+                                 "peak_hbm_gb": r["peak_lib"] / 1e9}
+                except Exception as e:  # noqa: BLE001
+                    row[mode] = {"error": str(e)[:160]}
+            t_sweep[str(T)] = row
     if rank != 0:
         if world > 1:
             dist.barrier()
@@ -338,6 +358,8 @@ def run_ours(args):
     cfg["peak_torch_allocated_gb"] = main["peak_torch"] / 1e9
     cfg["kept_fraction"] = main["kept_fraction"]
     cfg["compare"] = compare
+    if t_sweep:
+        cfg["t_sweep"] = t_sweep
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": main["total_ms"] / args.steps, "higher_is_better": True,
@@ -376,6 +398,7 @@ def main():
     ap.add_argument("--ref-batch", type=int, default=1)
     ap.add_argument("--no-compare", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--t-sweep", default="50,200,400", help="extra T values for peak-HBM / throughput vs T")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

@@ -70,7 +70,9 @@ def check_parity(name, T, B, C, p, mode, lam=None, seed=0):
     w_new = m.weights()
     for l, (wn, w0, r) in enumerate(zip(w_new, W, ref.dW)):
         wr, _, _ = adam_update(w0, r, np.zeros_like(r), np.zeros_like(r), 1)
-        sig = np.abs(r) > 1e-3 * np.abs(r).max()
+        # where the first Adam step is well conditioned: |g| well above eps (the update is
+        # g / (|g| + eps), ill-conditioned for |g| ~ eps = 1e-8) and not in the cancelling tail
+        sig = np.abs(r) > max(1e-3 * np.abs(r).max(), 1e-6)
         np.testing.assert_allclose(wn.cpu().numpy()[sig], wr[sig], rtol=0, atol=2e-6)
     return m, ref
 
@@ -158,3 +160,9 @@ def test_memory_ordering_full_ckpt_skip():
         peaks[mode] = m.mem_stats()[1]
         m.close()
     assert peaks["full"] > peaks["ckpt"] > peaks["skip"], peaks
+
+
+@pytest.mark.parametrize("mode", ["skip", "full"])
+def test_vgg11_reduced(mode):
+    """cfg 3 topology (VGG-11: 8 conv incl. 256/512-channel layers down to 2x2, fc 512-4096-4096)."""
+    check_parity("vgg11", T=24, B=2, C=2, p=50.0, mode=mode)
