@@ -96,6 +96,7 @@ struct skipper_ctx {
     int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
     int K0 = 0;                 // im2col width (32 or 64)
     bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
+    bool l0_bwd_fused = false;  // layer 0 backward: fused reverse scan + tcgen05 weight gradient
     int tail0 = 0;              // first layer of the fc tail: the first pass runs it over all T at once
     uint16_t *tail_in = nullptr, *tailP[2] = {nullptr, nullptr};
     float *tail_I = nullptr;
@@ -152,11 +153,11 @@ struct skipper_ctx {
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
-    K_L0_FWD, K_NCLASS
+    K_L0_FWD, K_L0_BWD, K_NCLASS
 };
 static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
                                                "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad",
-                                               "layer0_fused_fwd"};
+                                               "layer0_fused_fwd", "layer0_fused_bwd"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -488,6 +489,9 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         const char *e = getenv("SKIPPER_NO_L0_FUSION");
         c->l0_fused = c->in_kind == 1 && c->K0 == 32 && c->Ls >= 2 && !(e && atoi(e)) &&
                       sk::layer0_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
+        const char *e2 = getenv("SKIPPER_NO_L0_BWD_FUSION");
+        c->l0_bwd_fused = c->l0_fused && !(e2 && atoi(e2)) &&
+                          sk::layer0_bwd_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
     }
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
@@ -975,7 +979,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
     // the staged layer-0 operand is needed by the first pass unless layer 0 is fused (or part of the
     // whole-sequence fc tail), and by the layer-0 weight gradient of FULL mode
     const int iend = record ? c->Ls : c->tail0;
-    if (record || (iend > 0 && !c->l0_fused)) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
+    if ((record && !c->l0_bwd_fused) || (iend > 0 && !c->l0_fused)) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
     for (int i = 0; i < iend; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in;
@@ -1040,6 +1044,7 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     ProfScope ps0(c, K_READOUT, (double)c->T * 32 * 4, 0);
     CK(sk::launch_sam_finalize(c->s_part, c->s_dev, c->T, c->st));
     ProfScope ps1(c, K_READOUT, (double)c->B * last.Nout * 8 + (double)ro.wcount * 2, 4.0 * c->B * last.Nout * ro.Cout);
+    c->launches += 2;  // z, cross-entropy and dL/da^{L-1} kernels
     CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
                                ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
     CKS(comm_allreduce_s(c));
@@ -1072,7 +1077,7 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
 static skipper_status recompute_segment(skipper_ctx *c, int seg) {
     const int R = (int)c->kept[seg].size();
     const int *row_t = c->kept_dev + (size_t)seg * c->S;
-    CKS(stage_input(c, row_t, 0, R, false));
+    if (!c->l0_bwd_fused) CKS(stage_input(c, row_t, 0, R, false));  // layer-0 weight-gradient operand
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         if (i == 0 && c->l0_fused) {
@@ -1126,6 +1131,32 @@ static skipper_status join_wgrads(skipper_ctx *c) {
 static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
     for (int i = c->Ls - 1; i >= 0; --i) {
         Layer &l = c->L[i];
+        if (i == 0 && c->l0_bwd_fused) {  // reverse scan + weight gradient in one kernel, no delta in HBM
+            sk::L0BwdArgs b{};
+            b.x = c->x_cur;
+            b.T = c->T;
+            b.B = c->B;
+            b.H = l.H;
+            b.W = l.W;
+            b.C0 = l.Cin;
+            b.row_t = row_t;
+            b.R = R;
+            b.U = l.Useg;
+            b.g = (c->Ls == 1) ? c->g_last : c->I_buf;
+            b.carry = l.carry;
+            b.dW = l.dwp;
+            b.N = l.Cout;
+            b.pool = l.pool ? 1 : 0;
+            b.lam = l.d.lambda;
+            b.theta = l.d.theta;
+            b.surr = c->cfg.surrogate;
+            b.gamma = c->cfg.surr_gamma;
+            const double rows = (double)R * c->B;
+            const double bytes = rows * (l.N * 4 + l.Nout * 4 + c->in_elems) + (double)c->B * l.N * 8;
+            ProfScope ps(c, K_L0_BWD, bytes, 2.0 * rows * l.H * l.W * l.Cout * 9 * l.Cin);
+            CK(sk::launch_layer0_bwd(b, c->st, c->num_sms));
+            continue;
+        }
         const int par = i & 1;
         uint16_t *dcur = c->d_buf2[par];
         if (c->w_pending[par]) {  // the wgrad of layer i+2 still reads this delta buffer
@@ -1172,7 +1203,11 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             ok = get_plan(c, {2, dcur, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
                 return sk::plan_fc_wgrad(p, dcur, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
             });
-        {   // weight gradient on the side stream, after this layer's delta is written
+        if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
+            const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
+            const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
+            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K));
+        } else {   // weight gradient on the side stream, after this layer's delta is written
             CK(cudaEventRecord(c->ev_ready[par], c->st));
             CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
             const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);

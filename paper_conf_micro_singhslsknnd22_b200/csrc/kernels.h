@@ -82,6 +82,24 @@ struct L0FwdArgs {
     uint8_t *dbg_o;
 };
 bool layer0_supported(int B, int H, int W, int C0, int N, int pool);
+
+// Fused layer-0 backward (layer0.cu): Eq.2 reverse scan + weight gradient on the tensor cores.
+struct L0BwdArgs {
+    const uint8_t *x;
+    int T, B, H, W, C0;
+    const int *row_t;      // absolute t per row (device) or null -> r
+    int R;
+    const float *U;        // [R][B*H*W*N] stored membranes
+    const float *g;        // [R][B*PH*PW*N] gradient wrt the (pooled) output
+    float *carry;          // [B*H*W*N] in/out
+    float *dW;             // [N][32] fp32, accumulated (k = (dy*3+dx)*C0 + ci)
+    int N, pool;
+    float lam, theta;
+    int surr;
+    float gamma;
+};
+bool layer0_bwd_supported(int B, int H, int W, int C0, int N, int pool);
+cudaError_t launch_layer0_bwd(const L0BwdArgs &a, cudaStream_t s, int num_sms);
 cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms);
 
 // Readout integrator + softmax cross-entropy (reading 5) and its gradients.

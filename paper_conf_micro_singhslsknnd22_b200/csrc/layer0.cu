@@ -443,3 +443,266 @@ cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
 }
 
 }  // namespace sk
+
+namespace sk {
+
+// ============================================================================ fused layer-0 backward
+// Eq.2 reverse scan of the first layer fused with its weight gradient:
+//   delta_t = sigma'(U_t) * pool2^T(g_t) + lam * delta_{t+1}   (8 warps, 32 channels each, carry in
+//   registers across the kept rows of a tile), bf16(delta) written straight into shared memory as the
+//   MN-major A operand of  dW[co][k] += sum_pixels delta[px][co] * im2col(x_t)[px][k]  (tcgen05,
+//   M = 128 (Cout 64 used), N = 64 (27 used), K = 128 pixels per row), accumulated in TMEM over all
+//   rows of all tiles of the CTA; the im2col operand is built from the uint8 input by 4 producer warps.
+// Neither delta nor the im2col rows touch HBM.
+static constexpr int LB_STAGES = 4;
+static constexpr uint32_t LB_OP_BYTES = 128 * 128;  // 128 pixel lines x 128 B
+
+SK_DEV float surr_grad(float U, float th, int kind, float gamma) {
+    if (kind == 0) {
+        const float v = 1.0f - fabsf(U - th) / th;
+        return v > 0.0f ? gamma * v : 0.0f;
+    }
+    const float d = 1.0f + gamma * fabsf(U - th);
+    return 1.0f / (d * d);
+}
+
+__global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs a, const L0Tile tg) {
+    constexpr int N = 64;
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023u) & ~1023u;
+    const uint32_t sA = base;                               // delta^T operands
+    const uint32_t sB = sA + LB_STAGES * LB_OP_BYTES;       // im2col^T operands
+    const uint32_t bars = sB + LB_STAGES * LB_OP_BYTES;
+    auto full_bar = [&](int s) { return bars + 8u * s; };
+    auto empty_bar = [&](int s) { return bars + 8u * (LB_STAGES + s); };
+    const uint32_t done_bar = bars + 8u * (2 * LB_STAGES);
+    const uint32_t tmem_slot = done_bar + 8;
+    uint8_t *sA_ptr = smem_raw + (sA - raw);
+    uint8_t *sB_ptr = smem_raw + (sB - raw);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int HW = a.H * a.W;
+    const int tiles = tg.tiles_b * tg.tiles_y * tg.tiles_x;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < LB_STAGES; ++s) {
+            mbar_init(full_bar(s), 4 + 8);  // 4 producer warps + 8 delta warps
+            mbar_init(empty_bar(s), 1);
+        }
+        mbar_init(done_bar, 1);
+        fence_mbar_init();
+    }
+    if (warp == L0_MMA_WARP) tmem_alloc<64>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+
+    auto tile_origin = [&](int tile, int &b0, int &y0, int &x0) {
+        const int tx = tile % tg.tiles_x;
+        const int ty = (tile / tg.tiles_x) % tg.tiles_y;
+        const int tb = tile / (tg.tiles_x * tg.tiles_y);
+        b0 = tb * tg.TB;
+        y0 = ty * tg.TH;
+        x0 = tx * tg.TW;
+    };
+    auto row_time = [&](int r) -> long long { return a.row_t ? a.row_t[r] : (long long)r; };
+    // 128B-swizzled position of 16-byte chunk j of pixel line r inside a 128-line operand
+    auto line_off = [](int r, int j) -> uint32_t {
+        return (uint32_t)((r >> 3) * 1024 + (r & 7) * 128 + ((j ^ (r & 7)) << 4));
+    };
+
+    if (warp < 4) {
+        // ------------------------------------------------------------ producers: im2col^T lines
+        const int r = threadIdx.x;
+        const int rowbytes = a.W * a.C0, rowwords = rowbytes >> 2;
+        int stage = 0;
+        uint32_t phase = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            int b0, y0, x0, bl, yl, xl;
+            tile_origin(tile, b0, y0, x0);
+            l0_row_pos(tg, a.pool, r, bl, yl, xl);
+            const int b = b0 + bl, yy = y0 + yl, xx = x0 + xl;
+            const bool ok = b < a.B;
+            const int bstart = a.C0 * (xx - 1);
+            const int w0 = bstart >= 0 ? (bstart >> 2) : -1;
+            const int shift = bstart - 4 * w0;
+            for (int ri = a.R - 1; ri >= 0; --ri) {
+                const long long t = row_time(ri);
+                uint32_t m = 0;
+#pragma unroll
+                for (int dy = 0; dy < 3; ++dy) {
+                    const int y = yy + dy - 1;
+                    const bool rok = ok && y >= 0 && y < a.H;
+                    const uint32_t *rowp = reinterpret_cast<const uint32_t *>(
+                        a.x + ((t * a.B + (rok ? b : 0)) * a.H + (rok ? y : 0)) * (long long)rowbytes);
+                    uint32_t wv[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const int wi = w0 + j;
+                        wv[j] = (rok && wi >= 0 && wi < rowwords) ? __ldg(rowp + wi) : 0u;
+                    }
+                    const uint32_t v[3] = {__funnelshift_r(wv[0], wv[1], 8 * shift), __funnelshift_r(wv[1], wv[2], 8 * shift),
+                                           __funnelshift_r(wv[2], wv[3], 8 * shift)};
+#pragma unroll
+                    for (int j = 0; j < 9; ++j)
+                        if (j < 3 * a.C0 && ((v[j >> 2] >> (8 * (j & 3))) & 0xFFu)) m |= 1u << (dy * 3 * a.C0 + j);
+                }
+                mbar_wait(empty_bar(stage), phase ^ 1u);
+                uint8_t *dst = sB_ptr + stage * LB_OP_BYTES;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    uint32_t w[4] = {0u, 0u, 0u, 0u};
+                    if (j < 4) {
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            const int k = 8 * j + 2 * e;
+                            w[e] = (((m >> k) & 1u) ? 0x3F80u : 0u) | (((m >> (k + 1)) & 1u) ? 0x3F800000u : 0u);
+                        }
+                    }
+                    *reinterpret_cast<uint4 *>(dst + line_off(r, j)) = make_uint4(w[0], w[1], w[2], w[3]);
+                }
+                fence_async_shared();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(full_bar(stage));
+                if (++stage == LB_STAGES) {
+                    stage = 0;
+                    phase ^= 1u;
+                }
+            }
+        }
+    } else if (warp == L0_MMA_WARP) {
+        // ------------------------------------------------------------ MMA: dW^T tile in TMEM
+        if (lane == 0) {
+            constexpr uint32_t idesc = umma_idesc_bf16(128, N, 1, 1);
+            int stage = 0;
+            uint32_t phase = 0;
+            bool first = true;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                for (int ri = a.R - 1; ri >= 0; --ri) {
+                    mbar_wait(full_bar(stage), phase);
+                    tc_fence_after();
+                    const uint32_t a0 = sA + stage * LB_OP_BYTES, b0 = sB + stage * LB_OP_BYTES;
+#pragma unroll
+                    for (int k = 0; k < 8; ++k) {  // 16 pixels per MMA
+                        tc_mma_f16(tmem_base, umma_desc_sw128(a0 + k * 2048u, 0u, 1024u),
+                                   umma_desc_sw128(b0 + k * 2048u, 8192u, 1024u), idesc, (first && k == 0) ? 0u : 1u);
+                    }
+                    first = false;
+                    tc_commit(empty_bar(stage));
+                    if (++stage == LB_STAGES) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                }
+            }
+            tc_commit(done_bar);
+        }
+    } else {
+        // ------------------------------------------------------------ delta warps
+        const int q = warp & 3;
+        const int h = (warp - L0_EPI_WARP0) >> 2;
+        const int r = q * 32 + lane;
+        const int c0 = h * 32;
+        const int PH = a.pool ? a.H / 2 : a.H, PW = a.pool ? a.W / 2 : a.W;
+        const long long rs = (long long)a.B * HW * N, grs = (long long)a.B * PH * PW * N;
+        const float gs = a.pool ? 0.25f : 1.0f;
+        int stage = 0;
+        uint32_t phase = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            int b0, y0, x0, bl, yl, xl;
+            tile_origin(tile, b0, y0, x0);
+            l0_row_pos(tg, a.pool, r, bl, yl, xl);
+            const int b = b0 + bl, yy = y0 + yl, xx = x0 + xl;
+            const bool ok = b < a.B;
+            const long long pix = ((long long)(ok ? b : 0) * a.H + yy) * a.W + xx;
+            const long long opix = a.pool ? ((long long)(ok ? b : 0) * PH + (yy >> 1)) * PW + (xx >> 1) : pix;
+            float d[32];
+#pragma unroll
+            for (int c = 0; c < 32; c += 4) {
+                const float4 v = ok ? *reinterpret_cast<const float4 *>(a.carry + pix * N + c0 + c) : make_float4(0.f, 0.f, 0.f, 0.f);
+                d[c] = v.x; d[c + 1] = v.y; d[c + 2] = v.z; d[c + 3] = v.w;
+            }
+            for (int ri = a.R - 1; ri >= 0; --ri) {
+                float4 uv[8], gv[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    uv[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.U + ri * rs + pix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    gv[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.g + ri * grs + opix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                }
+                uint32_t pk[16];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const float u[4] = {uv[j].x, uv[j].y, uv[j].z, uv[j].w};
+                    const float gg[4] = {gv[j].x, gv[j].y, gv[j].z, gv[j].w};
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) {
+                        const int c = 4 * j + e;
+                        d[c] = surr_grad(u[e], a.theta, a.surr, a.gamma) * (gs * gg[e]) + a.lam * d[c];
+                    }
+                    pk[2 * j] = (uint32_t)f2bf_bits(d[4 * j]) | ((uint32_t)f2bf_bits(d[4 * j + 1]) << 16);
+                    pk[2 * j + 1] = (uint32_t)f2bf_bits(d[4 * j + 2]) | ((uint32_t)f2bf_bits(d[4 * j + 3]) << 16);
+                }
+                mbar_wait(empty_bar(stage), phase ^ 1u);
+                uint8_t *dst = sA_ptr + stage * LB_OP_BYTES;
+#pragma unroll
+                for (int j = 0; j < 4; ++j)  // this warp's 32 channels = 16-byte chunks h*4 .. h*4+3
+                    *reinterpret_cast<uint4 *>(dst + line_off(r, h * 4 + j)) =
+                        ok ? make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]) : make_uint4(0u, 0u, 0u, 0u);
+                fence_async_shared();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(full_bar(stage));
+                if (++stage == LB_STAGES) {
+                    stage = 0;
+                    phase ^= 1u;
+                }
+            }
+            if (ok) {
+#pragma unroll
+                for (int c = 0; c < 32; c += 4)
+                    *reinterpret_cast<float4 *>(a.carry + pix * N + c0 + c) = make_float4(d[c], d[c + 1], d[c + 2], d[c + 3]);
+            }
+        }
+        // drain dW^T rows 0..63 (Cout) x columns 0..31 (k) into the fp32 weight gradient
+        if (q < 2 && h == 0 && tiles > (int)blockIdx.x) {
+            mbar_wait(done_bar, 0);
+            tc_fence_after();
+            uint32_t v[32];
+            tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16), v);
+            tmem_ld_wait();
+            float *dst = a.dW + (long long)(q * 32 + lane) * 32;
+#pragma unroll
+            for (int k = 0; k < 32; k += 4)
+                red_add_v4(dst + k, __uint_as_float(v[k]), __uint_as_float(v[k + 1]), __uint_as_float(v[k + 2]),
+                           __uint_as_float(v[k + 3]));
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    if (warp == L0_MMA_WARP) tmem_dealloc<64>(tmem_base);
+}
+
+bool layer0_bwd_supported(int B, int H, int W, int C0, int N, int pool) {
+    L0Tile g;
+    return N == 64 && 9 * C0 <= 32 && (W * C0) % 4 == 0 && l0_tiling(B, H, W, pool, &g);
+}
+
+cudaError_t launch_layer0_bwd(const L0BwdArgs &a, cudaStream_t s, int num_sms) {
+    L0Tile g;
+    if (a.N != 64 || 9 * a.C0 > 32 || !l0_tiling(a.B, a.H, a.W, a.pool, &g)) return cudaErrorInvalidValue;
+    const int tiles = g.tiles_b * g.tiles_y * g.tiles_x;
+    if (tiles == 0 || a.R == 0) return cudaSuccess;
+    const uint32_t smem = 1024 + 2 * LB_STAGES * LB_OP_BYTES + 8 * (2 * LB_STAGES + 1) + 16;
+    static bool set = false;
+    if (!set) {
+        cudaFuncSetAttribute(layer0_bwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        set = true;
+    }
+    const int grid = tiles < num_sms ? tiles : num_sms;
+    layer0_bwd_kernel<<<grid, 32 * 13, smem, s>>>(a, g);
+    return cudaGetLastError();
+}
+
+}  // namespace sk

@@ -575,52 +575,61 @@ cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cud
 }
 
 // ============================================================================ readout + loss
-__global__ void readout_loss_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ cnt, const int *labels,
-                                    float *z, float *dz, float *loss, float *g_last, int D, int K, float invT,
-                                    float invBg) {
-    extern __shared__ float sh[];  // zs[K], dzs[K]
-    float *zs = sh, *dzs = sh + K;
-    const int b = blockIdx.x;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+// z[b][k] = (1/T) sum_n W^L[k][n] cnt[b][n]: one warp per (b, k)
+__global__ void readout_z_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ cnt, float *z, int B, int D,
+                                 int K, float invT) {
+    const long long w = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (w >= (long long)B * K) return;
+    const int b = (int)(w / K), k = (int)(w % K);
+    const uint16_t *wr = WbL + (long long)k * D;
     const float *cb = cnt + (long long)b * D;
-    for (int k = warp; k < K; k += nw) {
-        float acc = 0.f;
-        for (int n = lane; n < D; n += 32) acc += bf_bits2f(WbL[(long long)k * D + n]) * cb[n];
-        for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-        if (lane == 0) {
-            zs[k] = acc * invT;
-            z[(long long)b * K + k] = acc * invT;
-        }
+    float acc = 0.f;
+    for (int n = lane; n < D; n += 32) acc += bf_bits2f(wr[n]) * cb[n];
+    for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) z[w] = acc * invT;
+}
+
+// softmax cross-entropy per sample (one warp per sample): loss += CE / B_global, dz
+__global__ void readout_ce_kernel(const float *z, const int *labels, float *dz, float *loss, int B, int K, float invBg) {
+    const int b = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
+    if (b >= B) return;
+    const float *zb = z + (long long)b * K;
+    float mx = -INFINITY;
+    for (int k = lane; k < K; k += 32) mx = fmaxf(mx, zb[k]);
+    for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    float se = 0.f;
+    for (int k = lane; k < K; k += 32) se += expf(zb[k] - mx);
+    for (int o = 16; o; o >>= 1) se += __shfl_xor_sync(0xffffffffu, se, o);
+    const int y = labels[b];
+    for (int k = lane; k < K; k += 32) {
+        const float pr = expf(zb[k] - mx) / se;
+        dz[(long long)b * K + k] = (pr - (k == y ? 1.f : 0.f)) * invBg;
     }
-    __syncthreads();
-    if (warp == 0) {
-        float mx = -INFINITY;
-        for (int k = lane; k < K; k += 32) mx = fmaxf(mx, zs[k]);
-        for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-        float se = 0.f;
-        for (int k = lane; k < K; k += 32) se += expf(zs[k] - mx);
-        for (int o = 16; o; o >>= 1) se += __shfl_xor_sync(0xffffffffu, se, o);
-        const int y = labels[b];
-        for (int k = lane; k < K; k += 32) {
-            const float pr = expf(zs[k] - mx) / se;
-            const float v = (pr - (k == y ? 1.f : 0.f)) * invBg;
-            dzs[k] = v;
-            dz[(long long)b * K + k] = v;
-        }
-        if (lane == 0) atomicAdd(loss, (logf(se) + mx - zs[y]) * invBg);
-    }
-    __syncthreads();
-    for (int n = threadIdx.x; n < D; n += blockDim.x) {
-        float acc = 0.f;
-        for (int k = 0; k < K; ++k) acc += dzs[k] * bf_bits2f(WbL[(long long)k * D + n]);
-        g_last[(long long)b * D + n] = acc * invT;
-    }
+    if (lane == 0) atomicAdd(loss, (logf(se) + mx - zb[y]) * invBg);
+}
+
+// g_last[b][n] = (1/T) sum_k dz[b][k] W^L[k][n]: the gradient wrt the readout input, same at every t
+__global__ void readout_g_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ dz, float *g_last, int B,
+                                 int D, int K, float invT) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (long long)B * D) return;
+    const int b = (int)(i / D), n = (int)(i % D);
+    const float *db = dz + (long long)b * K;
+    float acc = 0.f;
+    for (int k = 0; k < K; ++k) acc += __ldg(db + k) * bf_bits2f(WbL[(long long)k * D + n]);
+    g_last[i] = acc * invT;
 }
 
 cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int *labels, float *z, float *dz,
                                 float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
                                 cudaStream_t s) {
-    readout_loss_kernel<<<B, 256, 2 * K * sizeof(float), s>>>(WbL, cnt, labels, z, dz, loss, g_last, D, K, invT, invBg);
+    const long long warps = (long long)B * K;
+    readout_z_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, s>>>(WbL, cnt, z, B, D, K, invT);
+    readout_ce_kernel<<<(B + 7) / 8, 256, 0, s>>>(z, labels, dz, loss, B, K, invBg);
+    const long long n = (long long)B * D;
+    readout_g_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(WbL, dz, g_last, B, D, K, invT);
     return cudaGetLastError();
 }
 
