@@ -489,8 +489,9 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         const char *e = getenv("SKIPPER_NO_L0_FUSION");
         c->l0_fused = c->in_kind == 1 && c->K0 == 32 && c->Ls >= 2 && !(e && atoi(e)) &&
                       sk::layer0_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
-        const char *e2 = getenv("SKIPPER_NO_L0_BWD_FUSION");
-        c->l0_bwd_fused = c->l0_fused && !(e2 && atoi(e2)) &&
+        // opt-in: measured slower than reverse scan + im2col wgrad GEMM on VGG-5
+        const char *e2 = getenv("SKIPPER_L0_BWD_FUSION");
+        c->l0_bwd_fused = c->l0_fused && (e2 && atoi(e2)) &&
                           sk::layer0_bwd_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
     }
     for (int i = 0; i < c->Ls; ++i) {

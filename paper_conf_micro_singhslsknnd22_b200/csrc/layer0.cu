@@ -11,8 +11,32 @@
 //   the input and this layer, checkpoint write at the segment start, stored U (recompute/full).
 // The currents never touch HBM: per neuron-step only the layer output (0.5 B pooled) and, when
 // stored, U (4 B) are written.
+#include <cstdio>
+#include <cstdlib>
+
 #include "common.cuh"
 #include "kernels.h"
+
+
+#ifdef SK_L0_STATS
+// diagnostic build (-DSK_L0_STATS): lane 0 of each role's first warp in CTA 0 accumulates the cycles
+// spent in each wait / section and prints them when the CTA ends
+#define L0_STAT_DECL                      \
+    long long l0s_[8] = {0, 0, 0, 0, 0, 0, 0, 0}; \
+    long long l0t_ = 0;                   \
+    const long long l0k_ = clock64()
+#define L0_T0 l0t_ = clock64()
+#define L0_T1(i) l0s_[i] += clock64() - l0t_
+#define L0_STAT_DUMP                                                                                        \
+    if (blockIdx.x == 0 && lane == 0 && (warp == 0 || warp == 8 || warp == 9))        \
+        printf("l0stats warp %d total %lld s1 %lld s2 %lld s3 %lld s4 %lld s5 %lld s6 %lld " \
+               "lif %lld\n", warp, clock64() - l0k_, l0s_[1], l0s_[2], l0s_[3], l0s_[4], l0s_[5], l0s_[6], l0s_[7])
+#else
+#define L0_STAT_DECL
+#define L0_T0
+#define L0_T1(i)
+#define L0_STAT_DUMP
+#endif
 
 namespace sk {
 
@@ -21,9 +45,20 @@ namespace sk {
 static constexpr int L0_PROD_WARPS = 4;
 static constexpr int L0_MMA_WARP = 4;
 static constexpr int L0_EPI_WARP0 = 5;
-static constexpr int L0_STAGES = 4;
+static constexpr int L0_STAGES = 6;
+static constexpr int L0_NACC = 4;  // TMEM accumulator ring (rows in flight between MMA and epilogue)
 static constexpr uint32_t L0_A_BYTES = 128 * 32 * 2;  // 128 rows x K=32 bf16
 static constexpr uint32_t L0_PLANE_A = 128 * 16;      // one 8-column K chunk of all 128 rows
+// forward kernel: warps 0-7 producers (two groups alternating rows), warp 8 MMA, warps 9..: epilogue
+static constexpr int L0_PGROUPS = 2;
+static constexpr int F0_PROD_WARPS = 4 * L0_PGROUPS;
+static constexpr int F0_MMA_WARP = F0_PROD_WARPS;
+static constexpr int F0_EPI_WARP0 = F0_PROD_WARPS + 1;
+static constexpr int L0_PD = 4;                                  // producer fetch depth (rows)
+static constexpr uint32_t L0_RING_BYTES = L0_PD * 6 * 128 * 8;  // 6 window chunks per row and thread
+
+// bit 0 of each byte of w -> 4-bit mask (byte i -> bit i); exact for bytes in {0,1}
+SK_DEV uint32_t byte_bits4(uint32_t w) { return ((w & 0x01010101u) * 0x10204080u) >> 28; }
 
 SK_DEV float lif_step0(float U, float I, float o, float lam, float th) {
     return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
@@ -61,23 +96,29 @@ SK_DEV void l0_row_pos(const L0Tile &g, int pool, int r, int &bl, int &yl, int &
     }
 }
 
-template <int NCH>  // Cout = 32 * NCH
-__global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_kernel(const L0FwdArgs a, const L0Tile tg) {
+// Cout = 32 * NCH; each epilogue warp owns CW channels of 32 pixels (4 * N / CW epilogue warps)
+template <int NCH, int CW>
+__global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
+    layer0_fwd_kernel(const L0FwdArgs a, const L0Tile tg) {
     constexpr int N = 32 * NCH;
+    constexpr int NEPI = 4 * N / CW;
     constexpr uint32_t PLANE_B = N * 16;
-    constexpr uint32_t TMEM_COLS = (2 * N <= 64) ? 64 : (2 * N <= 128 ? 128 : 256);
+    constexpr uint32_t TMEM_COLS = (L0_NACC * N <= 64) ? 64 : (L0_NACC * N <= 128 ? 128 : (L0_NACC * N <= 256 ? 256 : 512));
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023u) & ~1023u;
     const uint32_t sA = base;                                 // L0_STAGES x 8 KB
     const uint32_t sB = sA + L0_STAGES * L0_A_BYTES;          // N x 32 bf16
-    const uint32_t bars = sB + 4 * PLANE_B;
+    const uint32_t sRing = sB + 4 * PLANE_B;                   // producer fetch ring
+    const uint32_t bars = sRing + L0_PGROUPS * L0_RING_BYTES;
     auto full_bar = [&](int s) { return bars + 8u * s; };
     auto empty_bar = [&](int s) { return bars + 8u * (L0_STAGES + s); };
     auto tfull_bar = [&](int i) { return bars + 8u * (2 * L0_STAGES + i); };
-    auto tempty_bar = [&](int i) { return bars + 8u * (2 * L0_STAGES + 2 + i); };
-    const uint32_t tmem_slot = bars + 8u * (2 * L0_STAGES + 4);
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * L0_STAGES + L0_NACC + i); };
+    const uint32_t tmem_slot = bars + 8u * (2 * L0_STAGES + 2 * L0_NACC);
     unsigned *row_cnt = reinterpret_cast<unsigned *>(smem_raw + (tmem_slot + 16 - raw));
+    long long *s_rowt = reinterpret_cast<long long *>(smem_raw + ((tmem_slot + 16 + 4 * a.R + 7) & ~7u) - raw);
+    uint2 *s_lut = reinterpret_cast<uint2 *>(s_rowt + a.R);  // 4 bits -> 4 bf16 {0, 1}
     uint8_t *sB_ptr = smem_raw + (sB - raw);
     uint8_t *sA_ptr = smem_raw + (sA - raw);
 
@@ -91,23 +132,32 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
         const int n = i >> 5, k = i & 31;
         *reinterpret_cast<uint16_t *>(sB_ptr + (k >> 3) * PLANE_B + n * 16 + (k & 7) * 2) = a.wbp[n * 32 + k];
     }
-    for (int r = threadIdx.x; r < a.R; r += blockDim.x) row_cnt[r] = 0;
+    for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
+        row_cnt[r] = 0;
+        s_rowt[r] = a.row_t ? a.row_t[r] : (long long)a.t0 + r;
+    }
+    if (threadIdx.x < 16) {
+        const uint32_t i = threadIdx.x;
+        s_lut[i] = make_uint2(((i & 1u) ? 0x3F80u : 0u) | ((i & 2u) ? 0x3F800000u : 0u),
+                              ((i & 4u) ? 0x3F80u : 0u) | ((i & 8u) ? 0x3F800000u : 0u));
+    }
     fence_async_shared();
     if (threadIdx.x == 0) {
         for (int s = 0; s < L0_STAGES; ++s) {
-            mbar_init(full_bar(s), L0_PROD_WARPS);
+            mbar_init(full_bar(s), 4);  // the 4 warps of the group that owns the stage
             mbar_init(empty_bar(s), 1);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < L0_NACC; ++i) {
             mbar_init(tfull_bar(i), 1);
-            mbar_init(tempty_bar(i), 4 * NCH);
+            mbar_init(tempty_bar(i), NEPI);
         }
         fence_mbar_init();
     }
-    if (warp == L0_MMA_WARP) tmem_alloc<TMEM_COLS>(tmem_slot);
+    if (warp == F0_MMA_WARP) tmem_alloc<TMEM_COLS>(tmem_slot);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
+    L0_STAT_DECL;
     const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
 
     auto tile_origin = [&](int tile, int &b0, int &y0, int &x0) {
@@ -118,107 +168,141 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
         y0 = ty * tg.TH;
         x0 = tx * tg.TW;
     };
-    auto row_time = [&](int r) -> long long { return a.row_t ? a.row_t[r] : (long long)a.t0 + r; };
+    auto row_time = [&](int r) -> long long { return s_rowt[r]; };
 
-    if (warp < L0_PROD_WARPS) {
+    if (warp < F0_PROD_WARPS) {
         // ------------------------------------------------------------ producers: im2col -> smem
-        // thread r builds tile row r from three 16-byte windows of the uint8 input rows y-1, y, y+1
-        // (loads issued one row ahead of the build so their latency overlaps the barrier waits)
-        const int r = threadIdx.x;  // 0..127
+        // thread r builds tile row r from three 16-byte windows of the uint8 input rows y-1, y, y+1.
+        // The 12 window words of each row are fetched with cp.async into a private shared-memory ring
+        // L0_PD rows ahead of the build, so the global-load latency is off the producer's critical path.
+        const int grp = warp / 4;          // producer group: rows it = grp (mod L0_PGROUPS)
+        const int r = threadIdx.x & 127;  // tile row built by this thread
         const int rowbytes = a.W * a.C0;
-        const int rowwords = rowbytes >> 2;
-        int stage = 0;
+        int stage = grp;
         uint32_t phase = 0;
         const int nit_tile = a.R - r_mma0;
-        auto fetch = [&](int tile, int ri, uint32_t (&wv)[3][4], int &shift, bool &ok, bool &ctr) {
-            int b0, y0, x0, bl, yl, xl;
+        // ring slot layout [slot][chunk][thread] of 8-byte chunks (conflict-free 64-bit accesses)
+        const uint32_t ring = sRing + grp * L0_RING_BYTES;
+        auto slot_chunk = [&](int slot, int w) { return ring + ((uint32_t)(slot * 6 + w) * 128u + r) * 8u; };
+        const int rowchunks = rowbytes >> 3;
+        int bl, yl, xl;  // this thread's pixel within every tile
+        l0_row_pos(tg, a.pool, r, bl, yl, xl);
+        int pb = 0, pyy = 0, pxx = 0;  // fetch cursor's pixel, updated per tile
+        auto fetch_pixel = [&](int tile) {
+            int b0, y0, x0;
             tile_origin(tile, b0, y0, x0);
-            l0_row_pos(tg, a.pool, r, bl, yl, xl);
-            const int b = b0 + bl, yy = y0 + yl, xx = x0 + xl;
-            ok = b < a.B;
-            ctr = ok;
-            const long long t = row_time(ri);
-            const int bstart = a.C0 * (xx - 1);
-            const int w0 = bstart >= 0 ? (bstart >> 2) : -1;
-            shift = bstart - 4 * w0;
+            pb = b0 + bl;
+            pyy = y0 + yl;
+            pxx = x0 + xl;
+        };
+        auto issue = [&](int tile, int ri, int slot) {
+            if (tile < tiles) {
+                const int b = pb, yy = pyy, xx = pxx;
+                const bool ok = b < a.B;
+                const long long t = s_rowt[ri];
+                // the 3*C0 <= 9 window bytes [bstart, bstart + 3*C0) lie in two aligned 8-byte chunks
+                const int bstart = a.C0 * (xx - 1);
+                const int w0 = bstart >> 3;  // floor (bstart >= -C0)
 #pragma unroll
-            for (int dy = 0; dy < 3; ++dy) {
-                const int y = yy + dy - 1;
-                const bool rok = ok && y >= 0 && y < a.H;
-                const uint32_t *rowp =
-                    reinterpret_cast<const uint32_t *>(a.x + ((t * a.B + (rok ? b : 0)) * a.H + (rok ? y : 0)) * (long long)rowbytes);
+                for (int dy = 0; dy < 3; ++dy) {
+                    const int y = yy + dy - 1;
+                    const bool rok = ok && y >= 0 && y < a.H;
+                    const uint2 *rowp = reinterpret_cast<const uint2 *>(
+                        a.x + ((t * a.B + (rok ? b : 0)) * a.H + (rok ? y : 0)) * (long long)rowbytes);
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    const int wi = w0 + j;
-                    wv[dy][j] = (rok && wi >= 0 && wi < rowwords) ? __ldg(rowp + wi) : 0u;
+                    for (int j = 0; j < 2; ++j) {
+                        const int wi = w0 + j;
+                        const bool in = rok && wi >= 0 && wi < rowchunks;
+                        cp_async8(slot_chunk(slot, dy * 2 + j), in ? (const void *)(rowp + wi) : (const void *)a.x,
+                                  in ? 8u : 0u);
+                    }
                 }
             }
+            cp_async_commit();  // one group per row (possibly empty) keeps the wait count uniform
         };
-        uint32_t nx[3][4];
-        int nshift = 0;
-        bool nok = false, nctr = false;
-        int tile = blockIdx.x, ri = r_mma0;
-        if (tile < tiles && nit_tile > 0) fetch(tile, ri, nx, nshift, nok, nctr);
-        while (tile < tiles && nit_tile > 0) {
-            uint32_t cw[3][4];
+        auto advance = [&](int &tl, int &rr) -> bool {  // next row of this group (L0_PGROUPS rows on)
+            bool nt = false;
 #pragma unroll
-            for (int dy = 0; dy < 3; ++dy)
-#pragma unroll
-                for (int j = 0; j < 4; ++j) cw[dy][j] = nx[dy][j];
-            const int cshift = nshift;
-            const bool cok = nok;
-            const int cri = ri;
-            // advance and prefetch the next row
+            for (int k = 0; k < L0_PGROUPS; ++k)
+                if (++rr == a.R) {
+                    rr = r_mma0;
+                    tl += gridDim.x;
+                    nt = true;
+                }
+            return nt;
+        };
+        int tile = blockIdx.x, ri = r_mma0;  // build cursor
+        for (int k = 0; k < grp && nit_tile > 0; ++k)
             if (++ri == a.R) {
                 ri = r_mma0;
                 tile += gridDim.x;
             }
-            if (tile < tiles) fetch(tile, ri, nx, nshift, nok, nctr);
+        int ptile = tile, pri = ri;  // fetch cursor, L0_PD rows (of this group) ahead
+        int cb = 0, cxx = 0;  // build cursor's pixel
+        auto build_pixel = [&](int tile) {
+            int b0, y0, x0;
+            tile_origin(tile, b0, y0, x0);
+            cb = b0 + bl;
+            cxx = x0 + xl;
+        };
+        if (nit_tile > 0) {
+            if (ptile < tiles) fetch_pixel(ptile);
+            build_pixel(tile);
+#pragma unroll
+            for (int d = 0; d < L0_PD; ++d) {
+                issue(ptile, pri, d);
+                if (advance(ptile, pri) && ptile < tiles) fetch_pixel(ptile);
+            }
+        }
+        int slot = 0;
+        while (tile < tiles && nit_tile > 0) {
+            L0_T0; cp_async_wait<L0_PD - 1>(); L0_T1(1); L0_T0;  // this row's group has landed
+            const bool cok = cb < a.B;
+            const int cshift = (a.C0 * (cxx - 1)) & 7;  // window offset in its first chunk
+            const int cri = ri;
             // build the im2col row: bit (dy*3+dx)*C0+ci <- window byte dx*C0+ci of row dy
             uint32_t m = 0;
             unsigned cnt = 0;
             if (cok) {
+                const uint2 *wv = reinterpret_cast<const uint2 *>(smem_raw + (slot_chunk(slot, 0) - raw));
+                const uint32_t wmask = (1u << (3 * a.C0)) - 1u;
 #pragma unroll
                 for (int dy = 0; dy < 3; ++dy) {
-                    const uint32_t v0 = __funnelshift_r(cw[dy][0], cw[dy][1], 8 * cshift);
-                    const uint32_t v1 = __funnelshift_r(cw[dy][1], cw[dy][2], 8 * cshift);
-                    const uint32_t v2 = __funnelshift_r(cw[dy][2], cw[dy][3], 8 * cshift);
-                    const uint32_t v[3] = {v0, v1, v2};
-#pragma unroll
-                    for (int j = 0; j < 9; ++j) {  // 3*C0 <= 9 window bytes of this input row
-                        if (j < 3 * a.C0) {
-                            const uint32_t nz = ((v[j >> 2] >> (8 * (j & 3))) & 0xFFu) ? 1u : 0u;
-                            m |= nz << (dy * 3 * a.C0 + j);
-                            if (dy == 1) cnt += (j >= a.C0 && j < 2 * a.C0) ? nz : 0u;
-                        }
-                    }
+                    const uint2 c0 = wv[(dy * 2 + 0) * 128], c1 = wv[(dy * 2 + 1) * 128];
+                    // spike bytes are {0,1} (ABI): gather bit 0 of each byte into a 16-bit mask
+                    const uint32_t nib = byte_bits4(c0.x) | byte_bits4(c0.y) << 4 | byte_bits4(c1.x) << 8 |
+                                         byte_bits4(c1.y) << 12;
+                    m |= ((nib >> cshift) & wmask) << (dy * 3 * a.C0);
                 }
+                cnt = __popc((m >> (4 * a.C0)) & ((1u << a.C0) - 1u));  // centre tap of the centre row
             }
-            mbar_wait(empty_bar(stage), phase ^ 1u);
+            L0_T1(3); L0_T0;  // refill this slot (own words only, already consumed above) with the row L0_PD ahead
+            issue(ptile, pri, slot);
+            if (advance(ptile, pri) && ptile < tiles) fetch_pixel(ptile);
+            if (++slot == L0_PD) slot = 0;
+            if (advance(tile, ri) && tile < tiles) build_pixel(tile);
+            L0_T1(4); L0_T0; mbar_wait(empty_bar(stage), phase ^ 1u); L0_T1(2); L0_T0;
             uint8_t *dst = sA_ptr + stage * L0_A_BYTES + r * 16;
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                uint32_t w[4];
-#pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                    const int k = 8 * j + 2 * e;
-                    w[e] = (((m >> k) & 1u) ? 0x3F80u : 0u) | (((m >> (k + 1)) & 1u) ? 0x3F800000u : 0u);
-                }
-                *reinterpret_cast<uint4 *>(dst + j * L0_PLANE_A) = make_uint4(w[0], w[1], w[2], w[3]);
+            for (int j = 0; j < 4; ++j) {  // 8 K columns per 16-byte core-matrix row, via the nibble table
+                const uint2 lo = s_lut[(m >> (8 * j)) & 15u], hi = s_lut[(m >> (8 * j + 4)) & 15u];
+                *reinterpret_cast<uint4 *>(dst + j * L0_PLANE_A) = make_uint4(lo.x, lo.y, hi.x, hi.y);
             }
             if (a.s_part) {
                 const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
                 if (lane == 0 && v) atomicAdd(&row_cnt[cri], v);
             }
-            fence_async_shared();
+            L0_T1(5); L0_T0; fence_async_shared(); L0_T1(6);
             __syncwarp();
             if (lane == 0) mbar_arrive(full_bar(stage));
-            if (++stage == L0_STAGES) {
-                stage = 0;
+            stage += L0_PGROUPS;
+            if (stage >= L0_STAGES) {
+                stage -= L0_STAGES;
                 phase ^= 1u;
             }
         }
-    } else if (warp == L0_MMA_WARP) {
+        cp_async_wait<0>();
+    } else if (warp == F0_MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
         if (lane == 0) {
             constexpr uint32_t idesc = umma_idesc_bf16(128, N, 0, 0);
@@ -228,8 +312,8 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
             uint32_t acc_phase = 0;
             for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
                 for (int ri = r_mma0; ri < a.R; ++ri) {
-                    mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
-                    mbar_wait(full_bar(stage), phase);
+                    L0_T0; mbar_wait(tempty_bar(acc), acc_phase ^ 1u); L0_T1(3);
+                    L0_T0; mbar_wait(full_bar(stage), phase); L0_T1(4);
                     tc_fence_after();
                     const uint32_t a0 = sA + stage * L0_A_BYTES;
 #pragma unroll
@@ -242,8 +326,10 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                         stage = 0;
                         phase ^= 1u;
                     }
-                    acc ^= 1;
-                    if (acc == 0) acc_phase ^= 1u;
+                    if (++acc == L0_NACC) {
+                        acc = 0;
+                        acc_phase ^= 1u;
+                    }
                 }
             }
         }
@@ -251,15 +337,16 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
         // ------------------------------------------------------------ epilogue: LIF over rows
         // warp (q, h): TMEM lane quadrant q = warp % 4 (32 tile rows = pixels), channel chunk h
         const int q = warp & 3;
-        const int h = (warp - L0_EPI_WARP0) >> 2;
+        const int h = (warp - F0_EPI_WARP0) >> 2;
         const int row = q * 32 + lane;
         const long long rs = (long long)a.B * HW * N;
         const int PH = a.pool ? a.H / 2 : a.H, PW = a.pool ? a.W / 2 : a.W;
         const long long ors = (long long)a.B * PH * PW * N;
-        const int c0 = h * 32;
+        const int c0 = h * CW;
         int acc = 0;
         uint32_t acc_phase = 0;
         for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            L0_T0;
             int b0, y0, x0, bl, yl, xl;
             tile_origin(tile, b0, y0, x0);
             l0_row_pos(tg, a.pool, row, bl, yl, xl);
@@ -268,11 +355,11 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
             const long long pix = ((long long)(valid ? b : 0) * a.H + yy) * a.W + xx;
             const long long opix = a.pool ? ((long long)(valid ? b : 0) * PH + (yy >> 1)) * PW + (xx >> 1) : pix;
             const long long nbase = pix * N + c0;
-            float U[32];
+            float U[CW];
             uint32_t ob = 0;
             if (valid) {
 #pragma unroll
-                for (int c = 0; c < 32; c += 4) {
+                for (int c = 0; c < CW; c += 4) {
                     const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nbase + c);
                     U[c] = u.x; U[c + 1] = u.y; U[c + 2] = u.z; U[c + 3] = u.w;
                     const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nbase + c);
@@ -281,11 +368,11 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                 }
             } else {
 #pragma unroll
-                for (int c = 0; c < 32; ++c) U[c] = 0.f;
+                for (int c = 0; c < CW; ++c) U[c] = 0.f;
             }
             auto store_state = [&](float *Ud, uint8_t *od) {
 #pragma unroll
-                for (int c = 0; c < 32; c += 4) {
+                for (int c = 0; c < CW; c += 4) {
                     *reinterpret_cast<float4 *>(Ud + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
                     *reinterpret_cast<uchar4 *>(od + c) =
                         make_uchar4((ob >> c) & 1u, (ob >> (c + 1)) & 1u, (ob >> (c + 2)) & 1u, (ob >> (c + 3)) & 1u);
@@ -301,12 +388,14 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                     const uint32_t s0 = w0 ^ w1, cc0 = w0 & w1, s1 = w2 ^ w3, cc1 = w2 & w3;
                     const uint32_t ones = s0 ^ s1, k01 = s0 & s1;
                     const uint32_t twos = cc0 ^ cc1 ^ k01, fours = cc0 & cc1;
+                    constexpr int PL = CW / 4;  // channels this lane writes
                     const int sub = lane & 3;
-                    uint32_t pk[4];
-                    const uint32_t o8 = (ones >> (sub * 8)) & 0xFFu, t8 = (twos >> (sub * 8)) & 0xFFu;
-                    const uint32_t f8 = (fours >> (sub * 8)) & 0xFFu;
+                    uint32_t pk[PL / 2];
+                    const uint32_t msk = (1u << PL) - 1u;
+                    const uint32_t o8 = (ones >> (sub * PL)) & msk, t8 = (twos >> (sub * PL)) & msk;
+                    const uint32_t f8 = (fours >> (sub * PL)) & msk;
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) {
+                    for (int e = 0; e < PL / 2; ++e) {
                         uint32_t v2 = 0;
 #pragma unroll
                         for (int hh = 0; hh < 2; ++hh) {
@@ -317,12 +406,16 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                         }
                         pk[e] = v2;
                     }
-                    if (valid)
-                        *reinterpret_cast<uint4 *>(a.Po_out + (long long)ri * ors + opix * N + c0 + sub * 8) =
-                            make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                    if (valid) {
+                        uint16_t *po = a.Po_out + (long long)ri * ors + opix * N + c0 + sub * PL;
+                        if (PL == 8)
+                            *reinterpret_cast<uint4 *>(po) = make_uint4(pk[0], pk[1 % (PL / 2)], pk[2 % (PL / 2)], pk[3 % (PL / 2)]);
+                        else
+                            *reinterpret_cast<uint2 *>(po) = make_uint2(pk[0], pk[1 % (PL / 2)]);
+                    }
                 } else if (valid) {
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) {
+                    for (int j = 0; j < CW / 8; ++j) {
                         uint32_t pk[4];
 #pragma unroll
                         for (int e = 0; e < 4; ++e) {
@@ -336,7 +429,7 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
                 if (valid) {
                     if (a.U_out) {
 #pragma unroll
-                        for (int c = 0; c < 32; c += 4)
+                        for (int c = 0; c < CW; c += 4)
                             *reinterpret_cast<float4 *>(a.U_out + (long long)ri * rs + nbase + c) =
                                 make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
                     }
@@ -349,35 +442,45 @@ __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + 4 * NCH), 1) layer0_fwd_k
             };
 
             if (a.restore) emit(0);
+            L0_T1(1);
             for (int ri = r_mma0; ri < a.R; ++ri) {
-                mbar_wait(tfull_bar(acc), acc_phase);
+                L0_T0; mbar_wait(tfull_bar(acc), acc_phase); L0_T1(5); L0_T0;
                 tc_fence_after();
-                uint32_t r[32];
-                tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
-                tmem_ld_wait();
+                uint32_t r[CW];
+                if constexpr (CW == 32)
+                    tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+                else
+                    tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+                tmem_ld_wait(); L0_T1(6); L0_T0;
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty_bar(acc));
-                acc ^= 1;
-                if (acc == 0) acc_phase ^= 1u;
+                if (++acc == L0_NACC) {
+                    acc = 0;
+                    acc_phase ^= 1u;
+                }
                 uint32_t nb = 0;
 #pragma unroll
-                for (int c = 0; c < 32; ++c) {
+                for (int c = 0; c < CW; ++c) {
                     const float u = lif_step0(U[c], __uint_as_float(r[c]), (float)((ob >> c) & 1u), a.lam, a.theta);
                     U[c] = u;
                     nb |= (u > a.theta ? 1u : 0u) << c;
                 }
-                ob = nb;
-                emit(ri);
+                ob = nb; L0_T1(7); L0_T0;
+                emit(ri); L0_T1(3); L0_T0;
                 if (a.ckU && ri == 0 && valid) store_state(a.ckU + nbase, a.cko + nbase);
+                L0_T1(2);
             }
+            L0_T0;
             if (!a.restore && valid) store_state(a.U_state + nbase, a.o_state + nbase);
+            L0_T1(4);
         }
     }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
-    if (warp == L0_MMA_WARP) tmem_dealloc<TMEM_COLS>(tmem_base);
+    if (warp == F0_MMA_WARP) tmem_dealloc<TMEM_COLS>(tmem_base);
+    L0_STAT_DUMP;
     if (a.s_part) {
         for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
             const unsigned v = row_cnt[r];
@@ -411,7 +514,7 @@ static bool l0_tiling(int B, int H, int W, int pool, L0Tile *g) {
 
 bool layer0_supported(int B, int H, int W, int C0, int N, int pool) {
     L0Tile g;
-    return 9 * C0 <= 32 && (N == 32 || N == 64) && (W * C0) % 4 == 0 && l0_tiling(B, H, W, pool, &g);
+    return 9 * C0 <= 32 && (N == 32 || N == 64) && (W * C0) % 8 == 0 && l0_tiling(B, H, W, pool, &g);
 }
 
 cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
@@ -419,23 +522,34 @@ cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
     if (9 * a.C0 > 32 || !l0_tiling(a.B, a.H, a.W, a.pool, &g)) return cudaErrorInvalidValue;
     const int tiles = g.tiles_b * g.tiles_y * g.tiles_x;
     if (tiles == 0 || a.R == 0) return cudaSuccess;
-    const uint32_t smem = 1024 + L0_STAGES * L0_A_BYTES + 4 * a.N * 16 + 8 * (2 * L0_STAGES + 4) + 16 + 4 * a.R;
+    const uint32_t smem =
+        1024 + L0_STAGES * L0_A_BYTES + 4 * a.N * 16 + L0_PGROUPS * L0_RING_BYTES + 8 * (2 * L0_STAGES + 2 * L0_NACC) + 16 + 4 * a.R + 8 + 8 * a.R + 128;
+    if (smem > 200 * 1024) return cudaErrorInvalidValue;
     const int grid = tiles < num_sms ? tiles : num_sms;
-    if (a.W * a.C0 % 4) return cudaErrorInvalidValue;
-    if (a.N == 64) {
+    if (a.W * a.C0 % 8) return cudaErrorInvalidValue;
+    // epilogue warps own 32 channels each (fewer, longer warps measured faster than 16-channel ones)
+    static const bool cw32 = !(getenv("SKIPPER_L0_CW16") && atoi(getenv("SKIPPER_L0_CW16")));
+    if (a.N == 64 && cw32) {
         static bool set = false;
         if (!set) {
-            cudaFuncSetAttribute(layer0_fwd_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+            cudaFuncSetAttribute(layer0_fwd_kernel<2, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
             set = true;
         }
-        layer0_fwd_kernel<2><<<grid, 32 * (L0_EPI_WARP0 + 8), smem, s>>>(a, g);
+        layer0_fwd_kernel<2, 32><<<grid, 32 * (F0_EPI_WARP0 + 8), smem, s>>>(a, g);
+    } else if (a.N == 64) {
+        static bool set = false;
+        if (!set) {
+            cudaFuncSetAttribute(layer0_fwd_kernel<2, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+            set = true;
+        }
+        layer0_fwd_kernel<2, 16><<<grid, 32 * (F0_EPI_WARP0 + 16), smem, s>>>(a, g);
     } else if (a.N == 32) {
         static bool set = false;
         if (!set) {
-            cudaFuncSetAttribute(layer0_fwd_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+            cudaFuncSetAttribute(layer0_fwd_kernel<1, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
             set = true;
         }
-        layer0_fwd_kernel<1><<<grid, 32 * (L0_EPI_WARP0 + 4), smem, s>>>(a, g);
+        layer0_fwd_kernel<1, 16><<<grid, 32 * (F0_EPI_WARP0 + 8), smem, s>>>(a, g);
     } else {
         return cudaErrorInvalidValue;
     }
@@ -466,7 +580,9 @@ SK_DEV float surr_grad(float U, float th, int kind, float gamma) {
     return 1.0f / (d * d);
 }
 
-__global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs a, const L0Tile tg) {
+static constexpr int LB_DWARPS = 16;  // delta warps: 4 lane quadrants x 4 chunks of 16 channels
+
+__global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + LB_DWARPS), 1) layer0_bwd_kernel(const L0BwdArgs a, const L0Tile tg) {
     constexpr int N = 64;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
@@ -487,7 +603,7 @@ __global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs 
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < LB_STAGES; ++s) {
-            mbar_init(full_bar(s), 4 + 8);  // 4 producer warps + 8 delta warps
+            mbar_init(full_bar(s), 4 + LB_DWARPS);  // producer warps + delta warps
             mbar_init(empty_bar(s), 1);
         }
         mbar_init(done_bar, 1);
@@ -601,10 +717,12 @@ __global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs 
         }
     } else {
         // ------------------------------------------------------------ delta warps
+        // warp (q, h): pixels 32q..32q+31 (TMEM/operand line = pixel), channels 16h..16h+15; the next
+        // row's U and g are loaded before the current row is processed (rows walk backwards in t)
         const int q = warp & 3;
         const int h = (warp - L0_EPI_WARP0) >> 2;
         const int r = q * 32 + lane;
-        const int c0 = h * 32;
+        const int c0 = h * 16;
         const int PH = a.pool ? a.H / 2 : a.H, PW = a.pool ? a.W / 2 : a.W;
         const long long rs = (long long)a.B * HW * N, grs = (long long)a.B * PH * PW * N;
         const float gs = a.pool ? 0.25f : 1.0f;
@@ -618,22 +736,26 @@ __global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs 
             const bool ok = b < a.B;
             const long long pix = ((long long)(ok ? b : 0) * a.H + yy) * a.W + xx;
             const long long opix = a.pool ? ((long long)(ok ? b : 0) * PH + (yy >> 1)) * PW + (xx >> 1) : pix;
-            float d[32];
+            float d[16];
 #pragma unroll
-            for (int c = 0; c < 32; c += 4) {
+            for (int c = 0; c < 16; c += 4) {
                 const float4 v = ok ? *reinterpret_cast<const float4 *>(a.carry + pix * N + c0 + c) : make_float4(0.f, 0.f, 0.f, 0.f);
                 d[c] = v.x; d[c + 1] = v.y; d[c + 2] = v.z; d[c + 3] = v.w;
             }
-            for (int ri = a.R - 1; ri >= 0; --ri) {
-                float4 uv[8], gv[8];
+            float4 uv[4], gv[4], un[4], gn[4];
+            auto load_row = [&](int ri, float4 (&u)[4], float4 (&gg)[4]) {
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
-                    uv[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.U + ri * rs + pix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
-                    gv[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.g + ri * grs + opix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int j = 0; j < 4; ++j) {
+                    u[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.U + ri * rs + pix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
+                    gg[j] = ok ? __ldg(reinterpret_cast<const float4 *>(a.g + ri * grs + opix * N + c0 + 4 * j)) : make_float4(0.f, 0.f, 0.f, 0.f);
                 }
-                uint32_t pk[16];
+            };
+            load_row(a.R - 1, uv, gv);
+            for (int ri = a.R - 1; ri >= 0; --ri) {
+                if (ri > 0) load_row(ri - 1, un, gn);
+                uint32_t pk[8];
 #pragma unroll
-                for (int j = 0; j < 8; ++j) {
+                for (int j = 0; j < 4; ++j) {
                     const float u[4] = {uv[j].x, uv[j].y, uv[j].z, uv[j].w};
                     const float gg[4] = {gv[j].x, gv[j].y, gv[j].z, gv[j].w};
 #pragma unroll
@@ -647,8 +769,8 @@ __global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs 
                 mbar_wait(empty_bar(stage), phase ^ 1u);
                 uint8_t *dst = sA_ptr + stage * LB_OP_BYTES;
 #pragma unroll
-                for (int j = 0; j < 4; ++j)  // this warp's 32 channels = 16-byte chunks h*4 .. h*4+3
-                    *reinterpret_cast<uint4 *>(dst + line_off(r, h * 4 + j)) =
+                for (int j = 0; j < 2; ++j)  // this warp's 16 channels = 16-byte chunks 2h, 2h+1
+                    *reinterpret_cast<uint4 *>(dst + line_off(r, h * 2 + j)) =
                         ok ? make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]) : make_uint4(0u, 0u, 0u, 0u);
                 fence_async_shared();
                 __syncwarp();
@@ -657,10 +779,15 @@ __global__ void __launch_bounds__(32 * 13, 1) layer0_bwd_kernel(const L0BwdArgs 
                     stage = 0;
                     phase ^= 1u;
                 }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    uv[j] = un[j];
+                    gv[j] = gn[j];
+                }
             }
             if (ok) {
 #pragma unroll
-                for (int c = 0; c < 32; c += 4)
+                for (int c = 0; c < 16; c += 4)
                     *reinterpret_cast<float4 *>(a.carry + pix * N + c0 + c) = make_float4(d[c], d[c + 1], d[c + 2], d[c + 3]);
             }
         }
@@ -701,7 +828,7 @@ cudaError_t launch_layer0_bwd(const L0BwdArgs &a, cudaStream_t s, int num_sms) {
         set = true;
     }
     const int grid = tiles < num_sms ? tiles : num_sms;
-    layer0_bwd_kernel<<<grid, 32 * 13, smem, s>>>(a, g);
+    layer0_bwd_kernel<<<grid, 32 * (L0_EPI_WARP0 + LB_DWARPS), smem, s>>>(a, g);
     return cudaGetLastError();
 }
 
