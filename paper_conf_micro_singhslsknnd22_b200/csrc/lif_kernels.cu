@@ -355,7 +355,7 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
 // One thread owns 4 neurons; CH rows of (g, U) are loaded ahead of the reverse recurrence.
 template <int SPLIT>
 __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
-    constexpr int CH = 4;
+    constexpr int CH = SPLIT ? 1 : 2;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
     const long long rs = (long long)a.B * HW * C;
@@ -377,8 +377,8 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
     const float gs = a.g_pooled ? 0.25f : 1.0f;
     const int nspl = SPLIT ? a.nsplit : 1;
     float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
-    for (int rb = a.R - 1; rb >= 0; rb -= CH) {
-        float4 gv[CH], uv[CH];
+    // two chunks of CH rows in flight: loads of the next (earlier) chunk overlap the recurrence
+    auto load = [&](float4 (&gv)[CH], float4 (&uv)[CH], int rb) {
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
@@ -388,6 +388,8 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
                 uv[j] = ldg4(a.U + (long long)r * rs + n0);
             }
         }
+    };
+    auto consume = [&](const float4 (&gv)[CH], const float4 (&uv)[CH], int rb) {
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
@@ -399,6 +401,17 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
                 if (a.delta)
                     *reinterpret_cast<uint2 *>(a.delta + (long long)r * rs + n0) = pack_bf16x4(d.x, d.y, d.z, d.w);
             }
+        }
+    };
+    {
+        float4 gA[CH], uA[CH], gB[CH], uB[CH];
+        load(gA, uA, a.R - 1);
+        for (int rb = a.R - 1; rb >= 0; rb -= 2 * CH) {
+            if (rb - CH >= 0) load(gB, uB, rb - CH);
+            consume(gA, uA, rb);
+            if (rb - CH < 0) break;
+            if (rb - 2 * CH >= 0) load(gA, uA, rb - 2 * CH);
+            consume(gB, uB, rb - CH);
         }
     }
     *reinterpret_cast<float4 *>(a.carry + n0) = d;
