@@ -1,0 +1,371 @@
+// conv_lif.cu - K2+K1 fused for 3x3 convolution layers: synaptic current on the tcgen05 tensor cores
+// and the LIF recurrence (Eq.1) in the epilogue, so the fp32 currents never reach HBM.
+//
+// Work unit = (tile of 128 output pixels of one timestep, tile of BN output channels).  A CTA walks the
+// rows (timesteps) of its unit in order: for every row the implicit-GEMM K loop (one 3x3 tap x 64
+// input channels per K block, 4D TMA box shifted by the tap, zero padding = TMA out-of-bounds fill)
+// accumulates I_t into one of two TMEM accumulators; the epilogue warps hold the membrane potentials
+// of the unit in registers across rows (thread = pixel, BN/2 channels), apply
+//     U_t = ((lam * U_{t-1}) + I_t) - theta * o_{t-1},   o_t = [U_t > theta]      (no FMA, as the oracle)
+// and write the layer output (bf16 spikes, or their 2x2 average through a shared-memory exchange),
+// the stored membranes (RECORD / RECOMPUTE), the segment checkpoint, the SAM counts (Eq.4)
+// and the debug record.  The MMA of row t+1 overlaps the epilogue of row t.
+//
+//   warp 0      TMA producer            warp 1      MMA issuer + TMEM owner
+//   warps 2-9   epilogue: warp w reads TMEM lane quadrant w % 4 (32 pixels), channel half (w - 2) / 4
+#include "common.cuh"
+#include "gemm.h"
+
+namespace sk {
+
+static constexpr int CL_BM = 128;
+static constexpr int CL_BK = 64;
+static constexpr int CL_EPI_WARPS = 8;
+static constexpr int CL_THREADS = 32 * (2 + CL_EPI_WARPS);
+
+template <int BN>
+struct ClCfg {
+    static constexpr uint32_t A_BYTES = CL_BM * CL_BK * 2;
+    static constexpr uint32_t B_BYTES = BN * CL_BK * 2;
+    static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int STAGES = BN == 128 ? 6 : 8;
+    static constexpr uint32_t TMEM_COLS = 2 * BN <= 128 ? 128 : 256;
+    static constexpr int CW = BN / 2;                        // channels per epilogue thread
+    static constexpr uint32_t SPK_BYTES = 2u * CL_BM * (BN / 32) * 4u;  // 2 buffers of spike words
+    static constexpr uint32_t FIXED_BYTES = 1024 + STAGES * STAGE_BYTES + SPK_BYTES + 8 * (2 * STAGES + 4) + 16;
+};
+
+SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+}
+
+template <int BN, int POOL>
+__global__ void __launch_bounds__(CL_THREADS, 1)
+    conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
+    using Cfg = ClCfg<BN>;
+    constexpr int STAGES = Cfg::STAGES;
+    constexpr int CW = Cfg::CW;
+    constexpr int NW = BN / 32;  // spike words per pixel
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023u) & ~1023u;
+    const uint32_t spk = base + STAGES * Cfg::STAGE_BYTES;
+    const uint32_t bars = spk + Cfg::SPK_BYTES;
+    auto full_bar = [&](int s) { return bars + 8u * s; };
+    auto empty_bar = [&](int s) { return bars + 8u * (STAGES + s); };
+    auto tfull_bar = [&](int i) { return bars + 8u * (2 * STAGES + i); };
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * STAGES + 2 + i); };
+    const uint32_t tmem_slot = bars + 8u * (2 * STAGES + 4);
+    unsigned *s_cnt = reinterpret_cast<unsigned *>(smem_raw + (tmem_slot + 16 - raw));
+    uint32_t *s_spk = reinterpret_cast<uint32_t *>(smem_raw + (spk - raw));
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int units = a.m_tiles * a.n_tiles;
+    const int r_mma0 = a.restore ? 1 : 0;
+    const int HW = a.H * a.W;
+    const int BHW = a.B * HW;
+
+    for (int r = threadIdx.x; r < a.R; r += blockDim.x) s_cnt[r] = 0;
+    if (threadIdx.x == 0) {
+        tma_prefetch(&ta);
+        tma_prefetch(&tb);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(full_bar(s), 1);
+            mbar_init(empty_bar(s), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(tfull_bar(i), 1);
+            mbar_init(tempty_bar(i), CL_EPI_WARPS);
+        }
+        fence_mbar_init();
+    }
+    if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+    auto row_time = [&](int r) -> long long { return a.row_t ? (long long)a.row_t[r] : (long long)a.t0 + r; };
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ TMA producer
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int u = blockIdx.x; u < units; u += gridDim.x) {
+                const int mt = u % a.m_tiles, nt = u / a.m_tiles;
+                for (int r = r_mma0; r < a.R; ++r) {
+                    const long long m0 = (long long)r * BHW + (long long)mt * CL_BM;  // flat input pixel
+                    const int n0 = (int)(m0 / HW);
+                    const int y0 = (int)((m0 % HW) / a.W);
+                    for (int kb = 0; kb < a.num_kb; ++kb) {
+                        const int tap = kb / a.conv_cb, cblk = kb % a.conv_cb;
+                        mbar_wait(empty_bar(stage), phase ^ 1u);
+                        const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
+                        const uint32_t fb = full_bar(stage);
+                        mbar_expect_tx(fb, Cfg::STAGE_BYTES);
+                        tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
+                        tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
+                        if (++stage == STAGES) {
+                            stage = 0;
+                            phase ^= 1u;
+                        }
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ MMA issuer
+            constexpr uint32_t idesc = umma_idesc_bf16(CL_BM, BN, 0, 0);
+            int stage = 0;
+            uint32_t phase = 0;
+            int acc = 0;
+            uint32_t acc_phase = 0;
+            for (int u = blockIdx.x; u < units; u += gridDim.x) {
+                for (int r = r_mma0; r < a.R; ++r) {
+                    mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
+                    tc_fence_after();
+                    const uint32_t d_tmem = tmem_base + acc * BN;
+                    for (int kb = 0; kb < a.num_kb; ++kb) {
+                        mbar_wait(full_bar(stage), phase);
+                        tc_fence_after();
+                        const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
+                        const uint32_t sb = sa + Cfg::A_BYTES;
+#pragma unroll
+                        for (int k = 0; k < CL_BK / 16; ++k)
+                            tc_mma_f16(d_tmem, umma_desc_sw128(sa + k * 32u, 16u, 1024u),
+                                       umma_desc_sw128(sb + k * 32u, 16u, 1024u), idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                        tc_commit(empty_bar(stage));
+                        if (++stage == STAGES) {
+                            stage = 0;
+                            phase ^= 1u;
+                        }
+                    }
+                    tc_commit(tfull_bar(acc));
+                    acc ^= 1;
+                    if (acc == 0) acc_phase ^= 1u;
+                }
+            }
+        }
+    } else {
+        // ---------------------------------------------------------------- epilogue: LIF over rows
+        const int q = warp & 3;
+        const int h = (warp - 2) >> 2;
+        const int p = q * 32 + lane;  // tile row = output pixel
+        const int etid = threadIdx.x - 64;  // 0..255
+        const long long rs = (long long)BHW * a.Cout;  // neurons per row
+        const int PH = a.H / 2, PW = a.W / 2;
+        const long long prs = POOL ? rs / 4 : rs;  // outputs per row
+        // tile geometry: rows of W pixels, bh image rows per image, 128 / (bh * W) images
+        const int bh = HW >= CL_BM ? CL_BM / a.W : a.H;
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        uint32_t ebuf = 0;  // spike exchange buffer parity, flips every emitted row (across units too)
+        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            const int mt = u % a.m_tiles, nt = u / a.m_tiles;
+            const int pg = mt * CL_BM + p;  // pixel within a row
+            const bool valid = pg < BHW;
+            const int ch0 = nt * BN + h * CW;
+            const long long nidx = (long long)(valid ? pg : 0) * a.Cout + ch0;
+            float U[CW];
+            uint32_t ob[CW / 32];
+            if (valid) {
+#pragma unroll
+                for (int c = 0; c < CW; c += 4) {
+                    const float4 v = *reinterpret_cast<const float4 *>(a.U_state + nidx + c);
+                    U[c] = v.x; U[c + 1] = v.y; U[c + 2] = v.z; U[c + 3] = v.w;
+                }
+#pragma unroll
+                for (int j = 0; j < CW / 32; ++j) {
+                    uint32_t w = 0;
+#pragma unroll
+                    for (int c = 0; c < 32; c += 4) {
+                        const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nidx + 32 * j + c);
+                        w |= (o4.x ? 1u : 0u) << c | (o4.y ? 1u : 0u) << (c + 1) | (o4.z ? 1u : 0u) << (c + 2) |
+                             (o4.w ? 1u : 0u) << (c + 3);
+                    }
+                    ob[j] = w;
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < CW; ++c) U[c] = 0.f;
+#pragma unroll
+                for (int j = 0; j < CW / 32; ++j) ob[j] = 0u;
+            }
+            auto store_state = [&](float *Ud, uint8_t *od) {
+#pragma unroll
+                for (int c = 0; c < CW; c += 4) {
+                    *reinterpret_cast<float4 *>(Ud + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    const uint32_t w = ob[c >> 5] >> (c & 31);
+                    *reinterpret_cast<uchar4 *>(od + c) = make_uchar4(w & 1u, (w >> 1) & 1u, (w >> 2) & 1u, (w >> 3) & 1u);
+                }
+            };
+            auto emit = [&](int r) {
+                const long long t = row_time(r);
+                unsigned cnt = 0;
+                if (valid) {
+#pragma unroll
+                    for (int j = 0; j < CW / 32; ++j) cnt += __popc(ob[j]);
+                    if (a.U_out) {
+                        float *dst = a.U_out + (long long)r * rs + nidx;
+#pragma unroll
+                        for (int c = 0; c < CW; c += 4)
+                            *reinterpret_cast<float4 *>(dst + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    }
+                    if (a.dbg_U) store_state(a.dbg_U + t * rs + nidx, a.dbg_o + t * rs + nidx);
+                    if (!POOL) {
+                        uint16_t *dst = a.Po_out + (long long)r * rs + nidx;
+#pragma unroll
+                        for (int c = 0; c < CW; c += 8) {
+                            const uint32_t w = ob[c >> 5] >> (c & 31);
+                            uint32_t pk[4];
+#pragma unroll
+                            for (int e = 0; e < 4; ++e)
+                                pk[e] = (((w >> (2 * e)) & 1u) ? 0x3F80u : 0u) | (((w >> (2 * e + 1)) & 1u) ? 0x3F800000u : 0u);
+                            *reinterpret_cast<uint4 *>(dst + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                        }
+                    }
+                }
+                if (POOL) {
+                    // spike words -> smem [pixel][word] (buffer r & 1), then 2x2 window sums by all
+                    // epilogue threads: item = (pooled pixel of the tile, 8-channel group)
+                    uint32_t *sw = s_spk + (ebuf & 1u) * (CL_BM * NW);
+                    ++ebuf;
+#pragma unroll
+                    for (int j = 0; j < CW / 32; ++j) sw[p * NW + h * (CW / 32) + j] = valid ? ob[j] : 0u;
+                    asm volatile("bar.sync 1, %0;" ::"n"(32 * CL_EPI_WARPS) : "memory");
+                    const int PWt = a.W / 2, PHt = bh / 2;
+                    constexpr int GROUPS = BN / 8;
+                    for (int it = etid; it < (CL_BM / 4) * GROUPS; it += 32 * CL_EPI_WARPS) {
+                        const int qp = it / GROUPS, gsel = it % GROUPS;
+                        const int img = qp / (PHt * PWt), py = (qp / PWt) % PHt, px = qp % PWt;
+                        const int p00 = (img * bh + 2 * py) * a.W + 2 * px;
+                        const int pg00 = mt * CL_BM + p00;
+                        if (pg00 >= BHW) continue;
+                        const int wsel = gsel >> 2, sh = (gsel & 3) * 8;
+                        const uint32_t w0 = sw[p00 * NW + wsel] >> sh, w1 = sw[(p00 + 1) * NW + wsel] >> sh;
+                        const uint32_t w2 = sw[(p00 + a.W) * NW + wsel] >> sh, w3 = sw[(p00 + a.W + 1) * NW + wsel] >> sh;
+                        uint32_t pk[4];
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            uint32_t v2 = 0;
+#pragma unroll
+                            for (int hh = 0; hh < 2; ++hh) {
+                                const int ch = 2 * e + hh;
+                                const uint32_t n = ((w0 >> ch) & 1u) + ((w1 >> ch) & 1u) + ((w2 >> ch) & 1u) + ((w3 >> ch) & 1u);
+                                v2 |= (__float_as_uint(__uint2float_rn(n) * 0.25f) >> 16) << (16 * hh);
+                            }
+                            pk[e] = v2;
+                        }
+                        const int b = pg00 / HW, yy = (pg00 % HW) / a.W, xx = pg00 % a.W;
+                        const long long oidx = (((long long)b * PH + (yy >> 1)) * PW + (xx >> 1)) * a.Cout + nt * BN + gsel * 8;
+                        *reinterpret_cast<uint4 *>(a.Po_out + (long long)r * prs + oidx) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                    }
+                }
+                if (a.s_part) {
+                    const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
+                    if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
+                }
+            };
+
+            if (a.restore) emit(0);
+            for (int r = r_mma0; r < a.R; ++r) {
+                mbar_wait(tfull_bar(acc), acc_phase);
+                tc_fence_after();
+#pragma unroll
+                for (int j = 0; j < CW / 32; ++j) {
+                    uint32_t v[32];
+                    tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + h * CW + j * 32, v);
+                    tmem_ld_wait();
+                    uint32_t nb = 0;
+#pragma unroll
+                    for (int c = 0; c < 32; ++c) {
+                        const float uu = cl_lif(U[32 * j + c], __uint_as_float(v[c]), (float)((ob[j] >> c) & 1u), a.lam, a.theta);
+                        U[32 * j + c] = uu;
+                        nb |= (uu > a.theta ? 1u : 0u) << c;
+                    }
+                    ob[j] = nb;
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(tempty_bar(acc));
+                acc ^= 1;
+                if (acc == 0) acc_phase ^= 1u;
+                emit(r);
+                if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
+            }
+            if (!a.restore && valid) store_state(a.U_state + nidx, a.o_state + nidx);
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    if (warp == 1) tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+    if (a.s_part) {
+        for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
+            const unsigned v = s_cnt[r];
+            if (v) atomicAdd(a.s_part + row_time(r) * 32 + (blockIdx.x & 31), v);
+        }
+    }
+}
+
+bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {
+    if (cin % 64 || (cout != 64 && cout % 128)) return false;
+    if (W > CL_BM || CL_BM % W) return false;
+    const int HW = H * W;
+    if (HW >= CL_BM) {
+        const int bh = CL_BM / W;
+        if (H % bh) return false;
+        if (pool && bh % 2) return false;
+    } else if (CL_BM % HW) {
+        return false;
+    }
+    if (pool && (H % 2 || W % 2)) return false;
+    (void)B;
+    return true;
+}
+
+template <int BN, int POOL>
+static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const ConvLifArgs &a, cudaStream_t s,
+                             int num_sms) {
+    using Cfg = ClCfg<BN>;
+    auto kern = conv_lif_kernel<BN, POOL>;
+    const uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
+    if (smem > 227u * 1024u) return cudaErrorInvalidValue;
+    static uint32_t set = 0;
+    if (smem > set) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        set = smem;
+    }
+    const int units = a.m_tiles * a.n_tiles;
+    const int grid = units < num_sms ? units : num_sms;
+    kern<<<grid, CL_THREADS, smem, s>>>(ta, tb, a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms) {
+    if (!conv_lif_supported(a.B, a.H, a.W, a.Cin, a.Cout, a.pool)) return cudaErrorInvalidValue;
+    if (a.R <= 0) return cudaSuccess;
+    const int bn = a.Cout == 64 ? 64 : 128;
+    const int HW = a.H * a.W;
+    uint32_t bw = a.W, bhh, bnn;
+    if (HW >= CL_BM) {
+        bhh = CL_BM / a.W;
+        bnn = 1;
+    } else {
+        bhh = a.H;
+        bnn = CL_BM / HW;
+    }
+    CUtensorMap ta, tb;
+    if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, bhh, bnn)) return cudaErrorInvalidValue;
+    if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, bn)) return cudaErrorInvalidValue;
+    a.conv_cb = a.Cin / 64;
+    a.num_kb = 9 * a.conv_cb;
+    a.m_tiles = (a.B * HW + CL_BM - 1) / CL_BM;
+    a.n_tiles = a.Cout / bn;
+    if (bn == 64) return a.pool ? launch_cl<64, 1>(ta, tb, a, s, num_sms) : launch_cl<64, 0>(ta, tb, a, s, num_sms);
+    return a.pool ? launch_cl<128, 1>(ta, tb, a, s, num_sms) : launch_cl<128, 0>(ta, tb, a, s, num_sms);
+}
+
+}  // namespace sk

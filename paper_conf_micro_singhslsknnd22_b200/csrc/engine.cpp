@@ -42,6 +42,7 @@ struct Layer {
     float *Useg = nullptr;     // arena rows
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
     int fsplitT = 1;             // forward split-K of the whole-sequence first pass (fc tail layers)
+    bool cfused = false;         // conv layer: GEMM + LIF scan as one kernel (conv_lif.cu)
     uint16_t *wbp = nullptr;   // layer 0 im2col: bf16 weights zero-padded to [cout][K0]
     float *dwp = nullptr;      // layer 0 im2col: padded weight gradient
     float *dbg[2] = {nullptr, nullptr};     // first / recompute U
@@ -153,11 +154,11 @@ struct skipper_ctx {
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
-    K_L0_FWD, K_L0_BWD, K_NCLASS
+    K_L0_FWD, K_L0_BWD, K_CONV_LIF, K_NCLASS
 };
 static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
                                                "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad",
-                                               "layer0_fused_fwd", "layer0_fused_bwd"};
+                                               "layer0_fused_fwd", "layer0_fused_bwd", "gemm_lif_fwd"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -493,6 +494,14 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         const char *e2 = getenv("SKIPPER_L0_BWD_FUSION");
         c->l0_bwd_fused = c->l0_fused && (e2 && atoi(e2)) &&
                           sk::layer0_bwd_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
+        // conv layers after the first: tensor-core GEMM + LIF scan fused (not the last spiking layer,
+        // whose scan also accumulates the readout counts)
+        const char *e3 = getenv("SKIPPER_NO_CONV_FUSION");
+        for (int i = 1; i < c->Ls - 1; ++i) {
+            Layer &l = c->L[i];
+            l.cfused = l.conv && !(e3 && atoi(e3)) &&
+                       sk::conv_lif_supported(c->B, l.H, l.W, l.Cin, l.Cout, l.pool ? 1 : 0);
+        }
     }
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
@@ -975,6 +984,43 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     return SKIPPER_OK;
 }
 
+// Conv layer i >= 1 as one kernel: tcgen05 implicit GEMM + LIF epilogue (conv_lif.cu).
+static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16_t *in, int R, int t0,
+                                    const int *row_t, bool restore, bool record, uint16_t *out) {
+    Layer &l = c->L[i];
+    const size_t bn = (size_t)c->B * l.N;
+    sk::ConvLifArgs a{};
+    a.B = c->B;
+    a.H = l.H;
+    a.W = l.W;
+    a.Cin = l.Cin;
+    a.Cout = l.Cout;
+    a.pool = l.pool ? 1 : 0;
+    a.R = R;
+    a.restore = restore ? 1 : 0;
+    a.t0 = t0;
+    a.row_t = row_t;
+    a.U_state = restore ? l.ckU + (size_t)seg * bn : l.U_run;
+    a.o_state = restore ? l.cko + (size_t)seg * bn : l.o_run;
+    a.U_out = (restore || record) ? l.Useg : nullptr;
+    a.Po_out = out;
+    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
+    a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.s_part = restore ? nullptr : c->s_part;
+    a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
+    a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
+    a.lam = l.d.lambda;
+    a.theta = l.d.theta;
+    const double comp = R - (restore ? 1 : 0);
+    double bytes = comp * c->B * l.Nin * 2 + (double)l.wcount * 2 + (double)R * c->B * l.Nout * 2 + bn * 10;
+    if (a.U_out) bytes += (double)R * bn * 4;
+    if (a.ckU) bytes += bn * 5;
+    const double flops = 2.0 * comp * c->B * l.H * l.W * l.Cout * 9.0 * l.Cin;
+    ProfScope ps(c, K_CONV_LIF, bytes, flops);
+    CK(sk::launch_conv_lif(in, R, l.wb, a, c->st, c->num_sms));
+    return SKIPPER_OK;
+}
+
 // Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
 static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
     // the staged layer-0 operand is needed by the first pass unless layer 0 is fused (or part of the
@@ -994,6 +1040,10 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         }
         if (i == 0 && c->l0_fused) {
             CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));
+            continue;
+        }
+        if (l.cfused) {
+            CKS(conv_lif_rows(c, i, seg, in, R, t0, nullptr, false, record, out));
             continue;
         }
         CKS(gemm_forward(c, i, in, c->I_buf, R));
@@ -1086,6 +1136,10 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
             continue;
         }
         const uint16_t *in = i == 0 ? c->xg : c->L[i - 1].Po;
+        if (l.cfused) {
+            CKS(conv_lif_rows(c, i, seg, in, R, 0, row_t, true, false, l.Po));
+            continue;
+        }
         const size_t in_row = (size_t)c->B * (i == 0 ? c->in_row : c->L[i - 1].Nout);
         if (R > 1)  // rows 1..R-1 (row 0 is the checkpoint)
             CKS(gemm_forward(c, i, in + in_row, c->I_buf + (size_t)c->B * l.N, R - 1));

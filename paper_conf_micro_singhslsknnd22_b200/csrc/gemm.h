@@ -69,6 +69,29 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
 
 cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms);
 
+// Fused 3x3 convolution + LIF scan over the R rows of a segment (conv_lif.cu).  The input X is the
+// previous layer's output [rows_in][B][H][W][Cin] bf16 (row r of the segment reads input row r), Wk is
+// [Cout][9][Cin] bf16.  State / output pointers follow ScanFwdArgs (kernels.h); cnt is not supported.
+struct ConvLifArgs {
+    int B, H, W, Cin, Cout, pool;
+    int R, restore, t0;
+    const int *row_t;
+    float *U_state;
+    uint8_t *o_state;
+    float *U_out;
+    uint16_t *Po_out;
+    float *ckU;
+    uint8_t *cko;
+    unsigned *s_part;
+    float *dbg_U;
+    uint8_t *dbg_o;
+    float lam, theta;
+    // filled by launch_conv_lif
+    int m_tiles, n_tiles, num_kb, conv_cb;
+};
+bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool);
+cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms);
+
 int device_num_sms();
 
 }  // namespace sk
