@@ -16,6 +16,28 @@
 #include "common.cuh"
 #include "gemm.h"
 
+#include <cstdio>
+#include <cstdlib>
+
+#ifdef SK_L0_STATS
+// diagnostic build (-DSK_L0_STATS): lane 0 of warps 0, 1, 2 of CTA 0 accumulates cycles per section
+#define CL_STAT_DECL                               \
+    long long cls_[8] = {0, 0, 0, 0, 0, 0, 0, 0}; \
+    long long clt_ = 0;                            \
+    const long long clk_ = clock64()
+#define CL_T0 clt_ = clock64()
+#define CL_T1(i) cls_[i] += clock64() - clt_
+#define CL_STAT_DUMP                                                                                             \
+    if (blockIdx.x == 0 && lane == 0 && warp <= 2)                                                               \
+        printf("clstats warp %d total %lld s1 %lld s2 %lld s3 %lld s4 %lld s5 %lld\n", warp, clock64() - clk_, \
+               cls_[1], cls_[2], cls_[3], cls_[4], cls_[5])
+#else
+#define CL_STAT_DECL
+#define CL_T0
+#define CL_T1(i)
+#define CL_STAT_DUMP
+#endif
+
 namespace sk {
 
 static constexpr int CL_BM = 128;
@@ -39,7 +61,11 @@ SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
     return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
 }
 
-template <int BN, int POOL>
+// CS > 1: a cluster of CS CTAs works on CS consecutive pixel tiles of the same channel tile; each CTA
+// loads its own A tile and 1/CS of the weight tile, multicast to the cluster (L2 -> SM traffic of the
+// weights / CS).  Every CTA runs the same number of unit iterations (phantom units past the end
+// load and multiply but write nothing) so the multicast partners stay in step.
+template <int BN, int POOL, int CS>
 __global__ void __launch_bounds__(CL_THREADS, 1)
     conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
     using Cfg = ClCfg<BN>;
@@ -71,7 +97,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
         tma_prefetch(&tb);
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(full_bar(s), 1);
-            mbar_init(empty_bar(s), 1);
+            mbar_init(empty_bar(s), CS);  // every CTA of the cluster frees the stage (multicast B)
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(tfull_bar(i), 1);
@@ -81,9 +107,16 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     }
     if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
     tc_fence_before();
-    __syncthreads();
+    if (CS > 1)
+        cluster_sync_all();
+    else
+        __syncthreads();
     tc_fence_after();
+    const int niter = (units + gridDim.x - 1) / gridDim.x;  // uniform across the grid
+    const int rank = CS > 1 ? (int)cluster_ctarank() : 0;
+    constexpr uint16_t mc_mask = (uint16_t)((1u << CS) - 1u);
     const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+    CL_STAT_DECL;
     auto row_time = [&](int r) -> long long { return a.row_t ? (long long)a.row_t[r] : (long long)a.t0 + r; };
 
     if (warp == 0) {
@@ -91,7 +124,8 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             // ------------------------------------------------------------ TMA producer
             int stage = 0;
             uint32_t phase = 0;
-            for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            for (int it = 0; it < niter; ++it) {
+                const int u = blockIdx.x + it * gridDim.x;
                 const int mt = u % a.m_tiles, nt = u / a.m_tiles;
                 for (int r = r_mma0; r < a.R; ++r) {
                     const long long m0 = (long long)r * BHW + (long long)mt * CL_BM;  // flat input pixel
@@ -99,12 +133,20 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     const int y0 = (int)((m0 % HW) / a.W);
                     for (int kb = 0; kb < a.num_kb; ++kb) {
                         const int tap = kb / a.conv_cb, cblk = kb % a.conv_cb;
+                        CL_T0;
                         mbar_wait(empty_bar(stage), phase ^ 1u);
+                        CL_T1(1);
                         const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                         const uint32_t fb = full_bar(stage);
                         mbar_expect_tx(fb, Cfg::STAGE_BYTES);
                         tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
-                        tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
+                        if (CS > 1) {
+                            constexpr uint32_t SL = BN / CS;
+                            tma_load_2d_mc(sa + Cfg::A_BYTES + (uint32_t)rank * SL * 128u, &tb, fb, kb * CL_BK,
+                                           nt * BN + rank * (int)SL, mc_mask);
+                        } else {
+                            tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
+                        }
                         if (++stage == STAGES) {
                             stage = 0;
                             phase ^= 1u;
@@ -121,13 +163,17 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
-            for (int u = blockIdx.x; u < units; u += gridDim.x) {
+            for (int it = 0; it < niter; ++it) {
                 for (int r = r_mma0; r < a.R; ++r) {
+                    CL_T0;
                     mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
+                    CL_T1(1);
                     tc_fence_after();
                     const uint32_t d_tmem = tmem_base + acc * BN;
                     for (int kb = 0; kb < a.num_kb; ++kb) {
+                        CL_T0;
                         mbar_wait(full_bar(stage), phase);
+                        CL_T1(2);
                         tc_fence_after();
                         const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                         const uint32_t sb = sa + Cfg::A_BYTES;
@@ -135,7 +181,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         for (int k = 0; k < CL_BK / 16; ++k)
                             tc_mma_f16(d_tmem, umma_desc_sw128(sa + k * 32u, 16u, 1024u),
                                        umma_desc_sw128(sb + k * 32u, 16u, 1024u), idesc, (kb > 0 || k > 0) ? 1u : 0u);
-                        tc_commit(empty_bar(stage));
+                        if (CS > 1)
+                            tc_commit_mc(empty_bar(stage), mc_mask);
+                        else
+                            tc_commit(empty_bar(stage));
                         if (++stage == STAGES) {
                             stage = 0;
                             phase ^= 1u;
@@ -161,10 +210,12 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
         int acc = 0;
         uint32_t acc_phase = 0;
         uint32_t ebuf = 0;  // spike exchange buffer parity, flips every emitted row (across units too)
-        for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        for (int it = 0; it < niter; ++it) {
+            const int u = blockIdx.x + it * gridDim.x;
+            const bool uvalid = u < units;
             const int mt = u % a.m_tiles, nt = u / a.m_tiles;
             const int pg = mt * CL_BM + p;  // pixel within a row
-            const bool valid = pg < BHW;
+            const bool valid = uvalid && pg < BHW;
             const int ch0 = nt * BN + h * CW;
             const long long nidx = (long long)(valid ? pg : 0) * a.Cout + ch0;
             float U[CW];
@@ -241,7 +292,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         const int img = qp / (PHt * PWt), py = (qp / PWt) % PHt, px = qp % PWt;
                         const int p00 = (img * bh + 2 * py) * a.W + 2 * px;
                         const int pg00 = mt * CL_BM + p00;
-                        if (pg00 >= BHW) continue;
+                        if (!uvalid || pg00 >= BHW) continue;
                         const int wsel = gsel >> 2, sh = (gsel & 3) * 8;
                         const uint32_t w0 = sw[p00 * NW + wsel] >> sh, w1 = sw[(p00 + 1) * NW + wsel] >> sh;
                         const uint32_t w2 = sw[(p00 + a.W) * NW + wsel] >> sh, w3 = sw[(p00 + a.W + 1) * NW + wsel] >> sh;
@@ -270,7 +321,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
 
             if (a.restore) emit(0);
             for (int r = r_mma0; r < a.R; ++r) {
+                CL_T0;
                 mbar_wait(tfull_bar(acc), acc_phase);
+                CL_T1(1);
+                CL_T0;
                 tc_fence_after();
 #pragma unroll
                 for (int j = 0; j < CW / 32; ++j) {
@@ -291,7 +345,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 if (lane == 0) mbar_arrive(tempty_bar(acc));
                 acc ^= 1;
                 if (acc == 0) acc_phase ^= 1u;
+                CL_T1(2);
+                CL_T0;
                 emit(r);
+                CL_T1(3);
                 if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
             }
             if (!a.restore && valid) store_state(a.U_state + nidx, a.o_state + nidx);
@@ -299,8 +356,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     }
     tc_fence_before();
     __syncthreads();
+    if (CS > 1) cluster_sync_all();  // no CTA leaves while peers may still signal its barriers
     tc_fence_after();
     if (warp == 1) tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+    CL_STAT_DUMP;
     if (a.s_part) {
         for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
             const unsigned v = s_cnt[r];
@@ -325,11 +384,11 @@ bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {
     return true;
 }
 
-template <int BN, int POOL>
+template <int BN, int POOL, int CS>
 static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const ConvLifArgs &a, cudaStream_t s,
                              int num_sms) {
     using Cfg = ClCfg<BN>;
-    auto kern = conv_lif_kernel<BN, POOL>;
+    auto kern = conv_lif_kernel<BN, POOL, CS>;
     const uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
     if (smem > 227u * 1024u) return cudaErrorInvalidValue;
     static uint32_t set = 0;
@@ -339,9 +398,36 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const
         set = smem;
     }
     const int units = a.m_tiles * a.n_tiles;
-    const int grid = units < num_sms ? units : num_sms;
-    kern<<<grid, CL_THREADS, smem, s>>>(ta, tb, a);
-    return cudaGetLastError();
+    int grid = units < num_sms ? units : num_sms;
+    grid -= grid % CS;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(CL_THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attrs[1];
+    attrs[0].id = cudaLaunchAttributeClusterDimension;
+    attrs[0].val.clusterDim.x = CS;
+    attrs[0].val.clusterDim.y = 1;
+    attrs[0].val.clusterDim.z = 1;
+    cfg.attrs = attrs;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kern, ta, tb, a);
+}
+
+// cluster size for the weight multicast: SKIPPER_CL_CS (1, 2, 4), default 1 (measured no gain: the
+// kernel is bound by shared-memory bandwidth, MMA operand reads + TMA writes); 1 when the pixel tiles
+// of one channel tile do not split into whole clusters
+static int cl_pick_cs(int m_tiles, int units) {
+    static int def = -1;
+    if (def < 0) {
+        const char *e = getenv("SKIPPER_CL_CS");
+        def = e ? atoi(e) : 1;
+        if (def != 1 && def != 2 && def != 4) def = 1;
+    }
+    int cs = def;
+    while (cs > 1 && (m_tiles % cs || units < 2 * cs)) cs >>= 1;
+    return cs;
 }
 
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms) {
@@ -357,15 +443,25 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
         bhh = a.H;
         bnn = CL_BM / HW;
     }
-    CUtensorMap ta, tb;
-    if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, bhh, bnn)) return cudaErrorInvalidValue;
-    if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, bn)) return cudaErrorInvalidValue;
     a.conv_cb = a.Cin / 64;
     a.num_kb = 9 * a.conv_cb;
     a.m_tiles = (a.B * HW + CL_BM - 1) / CL_BM;
     a.n_tiles = a.Cout / bn;
-    if (bn == 64) return a.pool ? launch_cl<64, 1>(ta, tb, a, s, num_sms) : launch_cl<64, 0>(ta, tb, a, s, num_sms);
-    return a.pool ? launch_cl<128, 1>(ta, tb, a, s, num_sms) : launch_cl<128, 0>(ta, tb, a, s, num_sms);
+    const int cs = cl_pick_cs(a.m_tiles, a.m_tiles * a.n_tiles);
+    CUtensorMap ta, tb;
+    if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, bhh, bnn)) return cudaErrorInvalidValue;
+    if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, bn / cs)) return cudaErrorInvalidValue;
+#define CL_LAUNCH(BN_, CS_)                                                                                  \
+    return a.pool ? launch_cl<BN_, 1, CS_>(ta, tb, a, s, num_sms) : launch_cl<BN_, 0, CS_>(ta, tb, a, s, num_sms)
+    if (bn == 64) {
+        if (cs == 4) CL_LAUNCH(64, 4);
+        if (cs == 2) CL_LAUNCH(64, 2);
+        CL_LAUNCH(64, 1);
+    }
+    if (cs == 4) CL_LAUNCH(128, 4);
+    if (cs == 2) CL_LAUNCH(128, 2);
+    CL_LAUNCH(128, 1);
+#undef CL_LAUNCH
 }
 
 }  // namespace sk
