@@ -33,6 +33,18 @@ int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, floa
 int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float *dW,
                          int nb, int h, int w, int cin, int cout, int accumulate, void *stream);
 
+/* Fused 3x3 convolution + LIF over R timestep rows (Eq.1): for r = 0..R-1
+ *   I_r = conv_fwd(X_r, Wk)  (bf16 x bf16 -> fp32, tensor cores, never written to memory)
+ *   U_r = ((lam * U_{r-1}) + I_r) - theta * o_{r-1},   o_r = [U_r > theta]
+ * X [R][nb][h][w][cin] bf16 (nb = batch), Wk [cout][9][cin] bf16.  U_state [nb*h*w*cout] fp32 and
+ * o_state (uint8) hold (U_{-1}, o_{-1}) on entry and (U_{R-1}, o_{R-1}) on return.  Outputs:
+ * P [R][nb][h'][w'][cout] bf16 spikes (pool = 1: 2x2 average, h' = h/2), U_out [R][nb*h*w*cout] fp32
+ * (may be NULL).  Limits: cin % 64 == 0, cout 64 or a multiple of 128, 128 % w == 0 and the 128-pixel
+ * tile covering whole image rows.  EUNSUPPORTED otherwise. */
+int skipper_k_conv_lif(const unsigned short *X, const unsigned short *Wk, float *U_state, unsigned char *o_state,
+                       unsigned short *P, float *U_out, int R, int nb, int h, int w, int cin, int cout, int pool,
+                       float lam, float theta, void *stream);
+
 /* Number of SMs the persistent kernels size their grids for (148 on B200). */
 int skipper_k_num_sms(void);
 

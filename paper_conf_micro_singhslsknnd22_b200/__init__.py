@@ -6,6 +6,6 @@ not been built (no CPU fallback).
 """
 from .skipper import (  # noqa: F401
     SkipperNet, SkipperError, lib, sst_host, workspace_bytes, make_config, make_layers,
-    k_fc_fwd, k_fc_wgrad, k_conv_fwd, k_conv_dgrad, k_conv_wgrad,
+    k_fc_fwd, k_fc_wgrad, k_conv_fwd, k_conv_dgrad, k_conv_wgrad, k_conv_lif,
     PASS_FIRST, PASS_RECOMPUTE, PASS_RECORD,
 )

@@ -44,52 +44,76 @@ static constexpr int CL_BM = 128;
 static constexpr int CL_BK = 64;
 static constexpr int CL_EPI_WARPS = 8;
 static constexpr int CL_THREADS = 32 * (2 + CL_EPI_WARPS);
+static constexpr int CL_MAXST = 8;  // max smem ring stages
 
-template <int BN>
+template <int BN, int PAIR>
 struct ClCfg {
     static constexpr uint32_t A_BYTES = CL_BM * CL_BK * 2;
-    static constexpr uint32_t B_BYTES = BN * CL_BK * 2;
+    static constexpr uint32_t B_BYTES = (PAIR ? BN / 2 : BN) * CL_BK * 2;  // this CTA's slice of the weights
     static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
-    static constexpr int STAGES = BN == 128 ? 6 : 8;
+    static constexpr int STAGES = STAGE_BYTES <= 24576 ? 8 : 6;  // streamed-weight ring depth
     static constexpr uint32_t TMEM_COLS = 2 * BN <= 128 ? 128 : 256;
     static constexpr int CW = BN / 2;                        // channels per epilogue thread
     static constexpr uint32_t SPK_BYTES = 2u * CL_BM * (BN / 32) * 4u;  // 2 buffers of spike words
-    static constexpr uint32_t FIXED_BYTES = 1024 + STAGES * STAGE_BYTES + SPK_BYTES + 8 * (2 * STAGES + 4) + 16;
+    static constexpr uint32_t BAR_BYTES = 8 * (2 * CL_MAXST + 6) + 16;
+    static constexpr uint32_t FIXED_BYTES = 1024 + SPK_BYTES + BAR_BYTES;  // + stages (+ resident weights)
 };
 
 SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
     return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
 }
 
-// CS > 1: a cluster of CS CTAs works on CS consecutive pixel tiles of the same channel tile; each CTA
-// loads its own A tile and 1/CS of the weight tile, multicast to the cluster (L2 -> SM traffic of the
-// weights / CS).  Every CTA runs the same number of unit iterations (phantom units past the end
-// load and multiply but write nothing) so the multicast partners stay in step.
-template <int BN, int POOL, int CS>
+// PAIR = 1: a cluster of two CTAs on the two SMs of a TPC runs M = 256 MMAs (tcgen05 cta_group::2):
+// each CTA loads its own 128-pixel A tile and half of the weight tile (BN/2 channels) into its own
+// shared memory, the leader's MMA reads both halves and writes each CTA's 128 accumulator rows into
+// that CTA's TMEM.  Per SM that halves the weight bytes both read by the MMA and written by TMA —
+// the kernel is shared-memory-bandwidth bound.  Every CTA runs the same number of unit
+// iterations (phantom units past the end load and multiply but write nothing).
+// RESB = 1 (pairs only): each CTA keeps its half of the unit's weights resident in shared memory for
+// all rows of the unit (loaded once), so the ring streams only activations: per SM the TMA ingress
+// per MMA drops from 24 KB to 16 KB per K block (the kernel is bound by per-SM TMA ingress).
+template <int BN, int POOL, int PAIR, int RESB>
 __global__ void __launch_bounds__(CL_THREADS, 1)
     conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
-    using Cfg = ClCfg<BN>;
-    constexpr int STAGES = Cfg::STAGES;
+    using Cfg = ClCfg<BN, PAIR>;
     constexpr int CW = Cfg::CW;
     constexpr int NW = BN / 32;  // spike words per pixel
+    const int STAGES = RESB ? a.stages : Cfg::STAGES;
+    constexpr uint32_t SBYTES = RESB ? Cfg::A_BYTES : Cfg::STAGE_BYTES;  // bytes per ring stage
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023u) & ~1023u;
-    const uint32_t spk = base + STAGES * Cfg::STAGE_BYTES;
+    const uint32_t bres = base;  // resident weights [num_kb][BN/2 rows][128 B] (RESB)
+    const uint32_t sring = base + (RESB ? (uint32_t)a.num_kb * Cfg::B_BYTES : 0u);
+    const uint32_t spk = sring + STAGES * SBYTES;
     const uint32_t bars = spk + Cfg::SPK_BYTES;
     auto full_bar = [&](int s) { return bars + 8u * s; };
-    auto empty_bar = [&](int s) { return bars + 8u * (STAGES + s); };
-    auto tfull_bar = [&](int i) { return bars + 8u * (2 * STAGES + i); };
-    auto tempty_bar = [&](int i) { return bars + 8u * (2 * STAGES + 2 + i); };
-    const uint32_t tmem_slot = bars + 8u * (2 * STAGES + 4);
+    auto empty_bar = [&](int s) { return bars + 8u * (CL_MAXST + s); };
+    auto tfull_bar = [&](int i) { return bars + 8u * (2 * CL_MAXST + i); };
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CL_MAXST + 2 + i); };
+    const uint32_t bfull_bar = bars + 8u * (2 * CL_MAXST + 4);
+    const uint32_t bempty_bar = bars + 8u * (2 * CL_MAXST + 5);
+    const uint32_t tmem_slot = bars + 8u * (2 * CL_MAXST + 6);
     unsigned *s_cnt = reinterpret_cast<unsigned *>(smem_raw + (tmem_slot + 16 - raw));
     uint32_t *s_spk = reinterpret_cast<uint32_t *>(smem_raw + (spk - raw));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int units = a.m_tiles * a.n_tiles;
     const int r_mma0 = a.restore ? 1 : 0;
     const int HW = a.H * a.W;
     const int BHW = a.B * HW;
+    // work decomposition: PAIR -> pair index / rank; unit = (pixel-tile group, channel tile)
+    const int rank = PAIR ? (int)cluster_ctarank() : 0;
+    const int grp_tiles = PAIR ? a.m_tiles / 2 : a.m_tiles;  // pixel-tile groups per channel tile
+    const int units = grp_tiles * a.n_tiles;
+    const int wid = PAIR ? (int)blockIdx.x / 2 : (int)blockIdx.x;
+    const int nworkers = PAIR ? (int)gridDim.x / 2 : (int)gridDim.x;
+    const int niter = (units + nworkers - 1) / nworkers;  // uniform across the grid
+    auto unit_tile = [&](int it, int &mt, int &nt) -> bool {
+        const int u = wid + it * nworkers;
+        mt = (u % grp_tiles) * (PAIR ? 2 : 1) + rank;
+        nt = u / grp_tiles;
+        return u < units;
+    };
 
     for (int r = threadIdx.x; r < a.R; r += blockDim.x) s_cnt[r] = 0;
     if (threadIdx.x == 0) {
@@ -97,36 +121,46 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
         tma_prefetch(&tb);
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(full_bar(s), 1);
-            mbar_init(empty_bar(s), CS);  // every CTA of the cluster frees the stage (multicast B)
+            mbar_init(empty_bar(s), 1);
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(tfull_bar(i), 1);
-            mbar_init(tempty_bar(i), CL_EPI_WARPS);
+            mbar_init(tempty_bar(i), CL_EPI_WARPS * (PAIR ? 2 : 1));  // epilogue warps of both CTAs
         }
+        mbar_init(bfull_bar, 1);
+        mbar_init(bempty_bar, 1);
         fence_mbar_init();
     }
-    if (warp == 1) tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    if (warp == 1) {
+        if (PAIR)
+            tmem_alloc_2sm<Cfg::TMEM_COLS>(tmem_slot);
+        else
+            tmem_alloc<Cfg::TMEM_COLS>(tmem_slot);
+    }
     tc_fence_before();
-    if (CS > 1)
+    if (PAIR)
         cluster_sync_all();
     else
         __syncthreads();
     tc_fence_after();
-    const int niter = (units + gridDim.x - 1) / gridDim.x;  // uniform across the grid
-    const int rank = CS > 1 ? (int)cluster_ctarank() : 0;
-    constexpr uint16_t mc_mask = (uint16_t)((1u << CS) - 1u);
     const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
     CL_STAT_DECL;
     auto row_time = [&](int r) -> long long { return a.row_t ? (long long)a.row_t[r] : (long long)a.t0 + r; };
 
     if (warp == 0) {
         if (lane == 0) {
-            // ------------------------------------------------------------ TMA producer
+            // ------------------------------------------------------------ TMA producer (both CTAs)
             int stage = 0;
             uint32_t phase = 0;
             for (int it = 0; it < niter; ++it) {
-                const int u = blockIdx.x + it * gridDim.x;
-                const int mt = u % a.m_tiles, nt = u / a.m_tiles;
+                int mt, nt;
+                unit_tile(it, mt, nt);
+                if (RESB) {  // this unit's weight half, once
+                    if (it > 0) mbar_wait(bempty_bar, (uint32_t)(it - 1) & 1u);
+                    if (rank == 0) mbar_expect_tx(bfull_bar, 2u * a.num_kb * Cfg::B_BYTES);
+                    for (int kb = 0; kb < a.num_kb; ++kb)
+                        tma_load_2d_2sm(bres + kb * Cfg::B_BYTES, &tb, bfull_bar, kb * CL_BK, nt * BN + rank * (BN / 2));
+                }
                 for (int r = r_mma0; r < a.R; ++r) {
                     const long long m0 = (long long)r * BHW + (long long)mt * CL_BM;  // flat input pixel
                     const int n0 = (int)(m0 / HW);
@@ -136,15 +170,17 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         CL_T0;
                         mbar_wait(empty_bar(stage), phase ^ 1u);
                         CL_T1(1);
-                        const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
+                        const uint32_t sa = sring + stage * SBYTES;
                         const uint32_t fb = full_bar(stage);
-                        mbar_expect_tx(fb, Cfg::STAGE_BYTES);
-                        tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
-                        if (CS > 1) {
-                            constexpr uint32_t SL = BN / CS;
-                            tma_load_2d_mc(sa + Cfg::A_BYTES + (uint32_t)rank * SL * 128u, &tb, fb, kb * CL_BK,
-                                           nt * BN + rank * (int)SL, mc_mask);
+                        if (PAIR) {
+                            // both CTAs' bytes land on the leader's full barrier
+                            if (rank == 0) mbar_expect_tx(fb, 2 * SBYTES);
+                            tma_load_4d_2sm(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
+                            if (!RESB)
+                                tma_load_2d_2sm(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN + rank * (BN / 2));
                         } else {
+                            mbar_expect_tx(fb, Cfg::STAGE_BYTES);
+                            tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
                             tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
                         }
                         if (++stage == STAGES) {
@@ -156,14 +192,18 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            // ------------------------------------------------------------ MMA issuer
-            constexpr uint32_t idesc = umma_idesc_bf16(CL_BM, BN, 0, 0);
+        if (lane == 0 && rank == 0) {
+            // ------------------------------------------------------------ MMA issuer (leader)
+            constexpr uint32_t idesc = umma_idesc_bf16(PAIR ? 2 * CL_BM : CL_BM, BN, 0, 0);
             int stage = 0;
             uint32_t phase = 0;
             int acc = 0;
             uint32_t acc_phase = 0;
             for (int it = 0; it < niter; ++it) {
+                if (RESB) {
+                    mbar_wait(bfull_bar, (uint32_t)it & 1u);
+                    tc_fence_after();
+                }
                 for (int r = r_mma0; r < a.R; ++r) {
                     CL_T0;
                     mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
@@ -175,14 +215,20 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         mbar_wait(full_bar(stage), phase);
                         CL_T1(2);
                         tc_fence_after();
-                        const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
-                        const uint32_t sb = sa + Cfg::A_BYTES;
+                        const uint32_t sa = sring + stage * SBYTES;
+                        const uint32_t sb = RESB ? bres + kb * Cfg::B_BYTES : sa + Cfg::A_BYTES;
 #pragma unroll
-                        for (int k = 0; k < CL_BK / 16; ++k)
-                            tc_mma_f16(d_tmem, umma_desc_sw128(sa + k * 32u, 16u, 1024u),
-                                       umma_desc_sw128(sb + k * 32u, 16u, 1024u), idesc, (kb > 0 || k > 0) ? 1u : 0u);
-                        if (CS > 1)
-                            tc_commit_mc(empty_bar(stage), mc_mask);
+                        for (int k = 0; k < CL_BK / 16; ++k) {
+                            if (a.diag & 2) break;  // diagnostic: no MMA
+                            const uint64_t ad = umma_desc_sw128(sa + k * 32u, 16u, 1024u);
+                            const uint64_t bd = umma_desc_sw128(sb + k * 32u, 16u, 1024u);
+                            if (PAIR)
+                                tc_mma_f16_2sm(d_tmem, ad, bd, idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                            else
+                                tc_mma_f16(d_tmem, ad, bd, idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                        }
+                        if (PAIR)
+                            tc_commit_2sm_mc(empty_bar(stage), 3);
                         else
                             tc_commit(empty_bar(stage));
                         if (++stage == STAGES) {
@@ -190,10 +236,14 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                             phase ^= 1u;
                         }
                     }
-                    tc_commit(tfull_bar(acc));
+                    if (PAIR)
+                        tc_commit_2sm_mc(tfull_bar(acc), 3);
+                    else
+                        tc_commit(tfull_bar(acc));
                     acc ^= 1;
                     if (acc == 0) acc_phase ^= 1u;
                 }
+                if (RESB) tc_commit_2sm_mc(bempty_bar, 3);  // this unit's weights may be replaced
             }
         }
     } else {
@@ -211,9 +261,8 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
         uint32_t acc_phase = 0;
         uint32_t ebuf = 0;  // spike exchange buffer parity, flips every emitted row (across units too)
         for (int it = 0; it < niter; ++it) {
-            const int u = blockIdx.x + it * gridDim.x;
-            const bool uvalid = u < units;
-            const int mt = u % a.m_tiles, nt = u / a.m_tiles;
+            int mt, nt;
+            const bool uvalid = unit_tile(it, mt, nt);
             const int pg = mt * CL_BM + p;  // pixel within a row
             const bool valid = uvalid && pg < BHW;
             const int ch0 = nt * BN + h * CW;
@@ -319,7 +368,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 }
             };
 
-            if (a.restore) emit(0);
+            if (a.restore && !(a.diag & 1)) emit(0);
             for (int r = r_mma0; r < a.R; ++r) {
                 CL_T0;
                 mbar_wait(tfull_bar(acc), acc_phase);
@@ -328,6 +377,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 tc_fence_after();
 #pragma unroll
                 for (int j = 0; j < CW / 32; ++j) {
+                    if (a.diag & 1) break;  // diagnostic: epilogue does no LIF / output work
                     uint32_t v[32];
                     tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + h * CW + j * 32, v);
                     tmem_ld_wait();
@@ -342,12 +392,17 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 }
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(tempty_bar(acc));
+                if (lane == 0) {
+                    if (PAIR)
+                        mbar_arrive_leader(tempty_bar(acc));
+                    else
+                        mbar_arrive(tempty_bar(acc));
+                }
                 acc ^= 1;
                 if (acc == 0) acc_phase ^= 1u;
                 CL_T1(2);
                 CL_T0;
-                emit(r);
+                if (!(a.diag & 1)) emit(r);
                 CL_T1(3);
                 if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
             }
@@ -356,9 +411,14 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     }
     tc_fence_before();
     __syncthreads();
-    if (CS > 1) cluster_sync_all();  // no CTA leaves while peers may still signal its barriers
+    if (PAIR) cluster_sync_all();  // no CTA leaves while its peer may still signal its barriers
     tc_fence_after();
-    if (warp == 1) tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+    if (warp == 1) {
+        if (PAIR)
+            tmem_dealloc_2sm<Cfg::TMEM_COLS>(tmem_base);
+        else
+            tmem_dealloc<Cfg::TMEM_COLS>(tmem_base);
+    }
     CL_STAT_DUMP;
     if (a.s_part) {
         for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
@@ -384,12 +444,22 @@ bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {
     return true;
 }
 
-template <int BN, int POOL, int CS>
-static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const ConvLifArgs &a, cudaStream_t s,
+template <int BN, int POOL, int PAIR, int RESB>
+static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvLifArgs a, cudaStream_t s,
                              int num_sms) {
-    using Cfg = ClCfg<BN>;
-    auto kern = conv_lif_kernel<BN, POOL, CS>;
-    const uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
+    using Cfg = ClCfg<BN, PAIR>;
+    auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB>;
+    uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
+    if (RESB) {
+        const uint32_t resb = (uint32_t)a.num_kb * Cfg::B_BYTES;
+        const int room = (int)((227u * 1024u - smem - resb) / Cfg::A_BYTES);
+        a.stages = room < CL_MAXST ? room : CL_MAXST;
+        if (a.stages < 3) return cudaErrorInvalidValue;
+        smem += resb + a.stages * Cfg::A_BYTES;
+    } else {
+        a.stages = Cfg::STAGES;
+        smem += Cfg::STAGES * Cfg::STAGE_BYTES;
+    }
     if (smem > 227u * 1024u) return cudaErrorInvalidValue;
     static uint32_t set = 0;
     if (smem > set) {
@@ -397,9 +467,9 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const
         if (e != cudaSuccess) return e;
         set = smem;
     }
-    const int units = a.m_tiles * a.n_tiles;
-    int grid = units < num_sms ? units : num_sms;
-    grid -= grid % CS;
+    const int workers = PAIR ? (a.m_tiles / 2) * a.n_tiles : a.m_tiles * a.n_tiles;
+    const int max_workers = PAIR ? num_sms / 2 : num_sms;
+    const int grid = (workers < max_workers ? workers : max_workers) * (PAIR ? 2 : 1);
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(CL_THREADS);
@@ -407,7 +477,7 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const
     cfg.stream = s;
     cudaLaunchAttribute attrs[1];
     attrs[0].id = cudaLaunchAttributeClusterDimension;
-    attrs[0].val.clusterDim.x = CS;
+    attrs[0].val.clusterDim.x = PAIR ? 2 : 1;
     attrs[0].val.clusterDim.y = 1;
     attrs[0].val.clusterDim.z = 1;
     cfg.attrs = attrs;
@@ -415,19 +485,12 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, const
     return cudaLaunchKernelEx(&cfg, kern, ta, tb, a);
 }
 
-// cluster size for the weight multicast: SKIPPER_CL_CS (1, 2, 4), default 1 (measured no gain: the
-// kernel is bound by shared-memory bandwidth, MMA operand reads + TMA writes); 1 when the pixel tiles
-// of one channel tile do not split into whole clusters
-static int cl_pick_cs(int m_tiles, int units) {
-    static int def = -1;
-    if (def < 0) {
-        const char *e = getenv("SKIPPER_CL_CS");
-        def = e ? atoi(e) : 1;
-        if (def != 1 && def != 2 && def != 4) def = 1;
-    }
-    int cs = def;
-    while (cs > 1 && (m_tiles % cs || units < 2 * cs)) cs >>= 1;
-    return cs;
+// CTA pairs (SKIPPER_CL_PAIR=1 enables) when the pixel tiles of a channel tile pair up
+static bool cl_use_pair(int m_tiles) {
+    const char *e = getenv("SKIPPER_CL_PAIR");  // read per launch so tests can cover both variants
+    // default off: pairs measured ~2 % slower (the kernel is bound by per-SM TMA processing of the
+    // 4D activation boxes, not by shared-memory bandwidth or the MMA)
+    return e && atoi(e) != 0 && m_tiles % 2 == 0;
 }
 
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms) {
@@ -447,20 +510,29 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
     a.num_kb = 9 * a.conv_cb;
     a.m_tiles = (a.B * HW + CL_BM - 1) / CL_BM;
     a.n_tiles = a.Cout / bn;
-    const int cs = cl_pick_cs(a.m_tiles, a.m_tiles * a.n_tiles);
+    const bool pair = cl_use_pair(a.m_tiles);
+    {
+        static const int diag = getenv("SKIPPER_CL_DIAG") ? atoi(getenv("SKIPPER_CL_DIAG")) : 0;
+        a.diag = diag;  // timing experiments only (results are wrong when set)
+    }
     CUtensorMap ta, tb;
     if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, bhh, bnn)) return cudaErrorInvalidValue;
-    if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, bn / cs)) return cudaErrorInvalidValue;
-#define CL_LAUNCH(BN_, CS_)                                                                                  \
-    return a.pool ? launch_cl<BN_, 1, CS_>(ta, tb, a, s, num_sms) : launch_cl<BN_, 0, CS_>(ta, tb, a, s, num_sms)
+    if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, pair ? bn / 2 : bn)) return cudaErrorInvalidValue;
+    // resident weights when this CTA's half fits next to >= 4 activation stages
+    const int resb_env = getenv("SKIPPER_CL_RESB") ? atoi(getenv("SKIPPER_CL_RESB")) : 1;
+    const uint32_t half_bytes = (uint32_t)a.num_kb * (uint32_t)(bn / 2) * CL_BK * 2;
+    const bool resb = pair && resb_env && half_bytes + 4u * CL_BM * CL_BK * 2 + 8192u + 4u * a.R <= 220u * 1024u;
+#define CL_LAUNCH(BN_, PAIR_, RESB_)                                                                           \
+    return a.pool ? launch_cl<BN_, 1, PAIR_, RESB_>(ta, tb, a, s, num_sms)                                      \
+                  : launch_cl<BN_, 0, PAIR_, RESB_>(ta, tb, a, s, num_sms)
     if (bn == 64) {
-        if (cs == 4) CL_LAUNCH(64, 4);
-        if (cs == 2) CL_LAUNCH(64, 2);
-        CL_LAUNCH(64, 1);
+        if (resb) CL_LAUNCH(64, 1, 1);
+        if (pair) CL_LAUNCH(64, 1, 0);
+        CL_LAUNCH(64, 0, 0);
     }
-    if (cs == 4) CL_LAUNCH(128, 4);
-    if (cs == 2) CL_LAUNCH(128, 2);
-    CL_LAUNCH(128, 1);
+    if (resb) CL_LAUNCH(128, 1, 1);
+    if (pair) CL_LAUNCH(128, 1, 0);
+    CL_LAUNCH(128, 0, 0);
 #undef CL_LAUNCH
 }
 

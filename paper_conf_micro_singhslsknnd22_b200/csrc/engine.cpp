@@ -1602,6 +1602,35 @@ extern "C" int skipper_k_conv_fwd(const unsigned short *X, const unsigned short 
     return kapi_run(g, ok, stream, "conv_fwd");
 }
 
+extern "C" int skipper_k_conv_lif(const unsigned short *X, const unsigned short *Wk, float *U_state,
+                                  unsigned char *o_state, unsigned short *P, float *U_out, int R, int nb, int h, int w,
+                                  int cin, int cout, int pool, float lam, float theta, void *stream) {
+    if (!sk::conv_lif_supported(nb, h, w, cin, cout, pool)) {
+        g_last_error = "conv_lif: unsupported shape";
+        return SKIPPER_EUNSUPPORTED;
+    }
+    sk::ConvLifArgs a{};
+    a.B = nb;
+    a.H = h;
+    a.W = w;
+    a.Cin = cin;
+    a.Cout = cout;
+    a.pool = pool;
+    a.R = R;
+    a.U_state = U_state;
+    a.o_state = o_state;
+    a.U_out = U_out;
+    a.Po_out = P;
+    a.lam = lam;
+    a.theta = theta;
+    cudaError_t e = sk::launch_conv_lif(X, R, Wk, a, static_cast<cudaStream_t>(stream), sk::device_num_sms());
+    if (e != cudaSuccess) {
+        g_last_error = std::string("conv_lif: ") + cudaGetErrorString(e);
+        return SKIPPER_ECUDA;
+    }
+    return SKIPPER_OK;
+}
+
 extern "C" int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, float *G, int nb, int h, int w,
                                     int cin, int cout, void *stream) {
     sk::GemmLaunch g;

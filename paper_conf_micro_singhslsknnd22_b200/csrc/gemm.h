@@ -88,6 +88,8 @@ struct ConvLifArgs {
     float lam, theta;
     // filled by launch_conv_lif
     int m_tiles, n_tiles, num_kb, conv_cb;
+    int stages;  // activation ring depth (resident-weight variant)
+    int diag;  // SKIPPER_CL_DIAG timing experiments: 1 = no epilogue work, 2 = no MMA
 };
 bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool);
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms);

@@ -89,6 +89,7 @@ def _load():
         "skipper_k_conv_fwd": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_wgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
+        "skipper_k_conv_lif": (I, [P, P, P, P, P, P, I, I, I, I, I, I, I, ct.c_float, ct.c_float, P]),
         "skipper_k_num_sms": (I, []),
         "skipper_profile": (I, [P, I]),
         "skipper_profile_read": (I, [P, I, P, P, P, P]),
@@ -386,6 +387,24 @@ def k_conv_fwd(X, Wk):
     out = torch.empty((nb, h, w, cout), dtype=torch.float32, device=X.device)
     _check(lib.skipper_k_conv_fwd(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, _stream_handle()))
     return out
+
+
+def k_conv_lif(X, Wk, U_state, o_state, pool, lam, theta, store_u=True):
+    """Fused conv + LIF over R rows.  X [R][nb][h][w][cin] bf16, Wk [cout][3][3][cin] bf16,
+    U_state [nb][h][w][cout] fp32 and o_state (uint8) in/out.  Returns (P, U_out): P [R][nb][h'][w'][cout]
+    bf16 spikes (2x2 averaged when pool), U_out [R][nb][h][w][cout] fp32 (None unless store_u)."""
+    torch = _torch()
+    R, nb, h, w, cin = X.shape
+    cout = Wk.shape[0]
+    if U_state.dtype != torch.float32 or o_state.dtype != torch.uint8:
+        raise ValueError("U_state must be float32 and o_state uint8")
+    ph, pw = (h // 2, w // 2) if pool else (h, w)
+    P = torch.empty((R, nb, ph, pw, cout), dtype=torch.bfloat16, device=X.device)
+    U = torch.empty((R, nb, h, w, cout), dtype=torch.float32, device=X.device) if store_u else None
+    _check(lib.skipper_k_conv_lif(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(U_state, "f32"), _ptr(o_state),
+                                  _ptr(P, "bf16"), _ptr(U, "f32") if U is not None else None, R, nb, h, w, cin, cout,
+                                  1 if pool else 0, float(lam), float(theta), _stream_handle()))
+    return P, U
 
 
 def k_conv_dgrad(D, Wt):

@@ -129,3 +129,39 @@ def test_stream_ordering_with_torch():
             out2 = k_fc_fwd(A.view(torch.int16), B.view(torch.int16))
             h2 = out2.cpu()
         assert torch.all(h2 == K * 0.5)
+
+
+CONV_LIF_SHAPES = [(5, 6, 16, 16, 64, 128, 1), (4, 3, 8, 8, 128, 256, 0), (3, 5, 4, 4, 64, 64, 1),
+                   (6, 2, 32, 32, 64, 64, 1), (3, 7, 16, 16, 128, 128, 0), (1, 2, 16, 16, 64, 128, 1)]
+
+
+@pytest.mark.parametrize("variant", ["single", "pair", "pair_streamed_w"])
+@pytest.mark.parametrize("R,nb,h,w,cin,cout,pool", CONV_LIF_SHAPES)
+def test_conv_lif_exact(R, nb, h, w, cin, cout, pool, variant, monkeypatch):
+    """Fused conv + LIF (Eq.1) against conv2d in float64 (exact on the grid, rounded once to fp32) and
+    the LIF update in fp32 without FMA; spikes, pooled outputs and final state bit-exact."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_lif
+    monkeypatch.setenv("SKIPPER_CL_PAIR", "0" if variant == "single" else "1")  # CTA pair (cta_group::2)
+    monkeypatch.setenv("SKIPPER_CL_RESB", "0" if variant == "pair_streamed_w" else "1")  # resident weights
+    g = torch.Generator().manual_seed(R * 131 + nb * h + cin + pool)
+    X = spikes((R, nb, h, w, cin), gen=g) * 0.25 * torch.randint(1, 5, (R, nb, h, w, cin), generator=g)
+    W = grid((cout, 3, 3, cin), e=9, gen=g)
+    U0 = grid((nb, h, w, cout), e=9, gen=g) * 0.5
+    o0 = (torch.rand((nb, h, w, cout), generator=g) < 0.2).to(torch.uint8)
+    lam, theta = 0.75, 1.0
+    U, o = U0.clone(), o0.float()
+    refP, refU = [], []
+    for r in range(R):
+        I = conv_ref(X[r], W).float()
+        U = (lam * U + I) - theta * o
+        o = (U > theta).float()
+        refU.append(U.clone())
+        refP.append(F.avg_pool2d(o.permute(0, 3, 1, 2), 2).permute(0, 2, 3, 1) if pool else o.clone())
+    Us, os_ = U0.clone().cuda(), o0.clone().cuda()
+    P, Uo = k_conv_lif(bf16_bits(X).cuda(), bf16_bits(W).cuda(), Us, os_, pool, lam, theta)
+    P = P.cpu().float()
+    for r in range(R):
+        assert torch.equal(P[r], refP[r]), f"row {r}: {int((P[r] != refP[r]).sum())} outputs differ"
+        assert torch.equal(Uo[r].cpu(), refU[r]), f"row {r}: U max diff {(Uo[r].cpu() - refU[r]).abs().max()}"
+    assert torch.equal(Us.cpu(), refU[-1])
+    assert torch.equal(os_.cpu(), (refU[-1] > theta).to(torch.uint8))
