@@ -45,6 +45,7 @@ static constexpr int CL_BK = 64;
 static constexpr int CL_EPI_WARPS = 8;
 static constexpr int CL_THREADS = 32 * (2 + CL_EPI_WARPS);
 static constexpr int CL_MAXST = 8;  // max smem ring stages
+static constexpr uint32_t CL_AH_MAX = 24576;  // halo activation box: (128 / W + 2) * W * 128 B, W <= 32
 
 template <int BN, int PAIR>
 struct ClCfg {
@@ -52,10 +53,11 @@ struct ClCfg {
     static constexpr uint32_t B_BYTES = (PAIR ? BN / 2 : BN) * CL_BK * 2;  // this CTA's slice of the weights
     static constexpr uint32_t STAGE_BYTES = A_BYTES + B_BYTES;
     static constexpr int STAGES = STAGE_BYTES <= 24576 ? 8 : 6;  // streamed-weight ring depth
-    static constexpr uint32_t TMEM_COLS = 2 * BN <= 128 ? 128 : 256;
+    static constexpr int NACC = 512 / BN < 4 ? 512 / BN : 4;  // TMEM accumulator ring (rows in flight)
+    static constexpr uint32_t TMEM_COLS = NACC * BN <= 128 ? 128 : (NACC * BN <= 256 ? 256 : 512);
     static constexpr int CW = BN / 2;                        // channels per epilogue thread
     static constexpr uint32_t SPK_BYTES = 2u * CL_BM * (BN / 32) * 4u;  // 2 buffers of spike words
-    static constexpr uint32_t BAR_BYTES = 8 * (2 * CL_MAXST + 6) + 16;
+    static constexpr uint32_t BAR_BYTES = 8 * (2 * CL_MAXST + 10) + 16;
     static constexpr uint32_t FIXED_BYTES = 1024 + SPK_BYTES + BAR_BYTES;  // + stages (+ resident weights)
 };
 
@@ -72,14 +74,21 @@ SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
 // RESB = 1 (pairs only): each CTA keeps its half of the unit's weights resident in shared memory for
 // all rows of the unit (loaded once), so the ring streams only activations: per SM the TMA ingress
 // per MMA drops from 24 KB to 16 KB per K block (the kernel is bound by per-SM TMA ingress).
-template <int BN, int POOL, int PAIR, int RESB>
+// HALO = 1 (single CTA, tiles of whole image rows, W >= 8): per (row, 64-channel block, dx) ONE
+// activation box of bh + 2 image rows (the tile plus its vertical halo, zero-filled out of bounds) is
+// loaded together with the weights of the three vertical taps; the three dy taps read the same box at
+// descriptor offsets of dy * W rows (multiples of the 1024-byte swizzle atom).  Activation boxes per
+// row: 3 * Cin/64 instead of 9 * Cin/64 (the kernel is bound by per-SM TMA box processing).
+template <int BN, int POOL, int PAIR, int RESB, int HALO>
 __global__ void __launch_bounds__(CL_THREADS, 1)
     conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
     using Cfg = ClCfg<BN, PAIR>;
     constexpr int CW = Cfg::CW;
     constexpr int NW = BN / 32;  // spike words per pixel
-    const int STAGES = RESB ? a.stages : Cfg::STAGES;
-    constexpr uint32_t SBYTES = RESB ? Cfg::A_BYTES : Cfg::STAGE_BYTES;  // bytes per ring stage
+    const int STAGES = a.stages;
+    constexpr uint32_t SBYTES =
+        RESB ? Cfg::A_BYTES : (HALO ? CL_AH_MAX + 3 * Cfg::B_BYTES : Cfg::STAGE_BYTES);  // bytes per ring stage
+    const int steps = HALO ? 3 * a.conv_cb : a.num_kb;  // ring stages per row
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023u) & ~1023u;
@@ -89,11 +98,12 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     const uint32_t bars = spk + Cfg::SPK_BYTES;
     auto full_bar = [&](int s) { return bars + 8u * s; };
     auto empty_bar = [&](int s) { return bars + 8u * (CL_MAXST + s); };
+    constexpr int NACC = Cfg::NACC;
     auto tfull_bar = [&](int i) { return bars + 8u * (2 * CL_MAXST + i); };
-    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CL_MAXST + 2 + i); };
-    const uint32_t bfull_bar = bars + 8u * (2 * CL_MAXST + 4);
-    const uint32_t bempty_bar = bars + 8u * (2 * CL_MAXST + 5);
-    const uint32_t tmem_slot = bars + 8u * (2 * CL_MAXST + 6);
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CL_MAXST + 4 + i); };
+    const uint32_t bfull_bar = bars + 8u * (2 * CL_MAXST + 8);
+    const uint32_t bempty_bar = bars + 8u * (2 * CL_MAXST + 9);
+    const uint32_t tmem_slot = bars + 8u * (2 * CL_MAXST + 10);
     unsigned *s_cnt = reinterpret_cast<unsigned *>(smem_raw + (tmem_slot + 16 - raw));
     uint32_t *s_spk = reinterpret_cast<uint32_t *>(smem_raw + (spk - raw));
 
@@ -123,7 +133,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             mbar_init(full_bar(s), 1);
             mbar_init(empty_bar(s), 1);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < NACC; ++i) {
             mbar_init(tfull_bar(i), 1);
             mbar_init(tempty_bar(i), CL_EPI_WARPS * (PAIR ? 2 : 1));  // epilogue warps of both CTAs
         }
@@ -165,14 +175,22 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     const long long m0 = (long long)r * BHW + (long long)mt * CL_BM;  // flat input pixel
                     const int n0 = (int)(m0 / HW);
                     const int y0 = (int)((m0 % HW) / a.W);
-                    for (int kb = 0; kb < a.num_kb; ++kb) {
+                    for (int kb = 0; kb < steps; ++kb) {
                         const int tap = kb / a.conv_cb, cblk = kb % a.conv_cb;
                         CL_T0;
                         mbar_wait(empty_bar(stage), phase ^ 1u);
                         CL_T1(1);
                         const uint32_t sa = sring + stage * SBYTES;
                         const uint32_t fb = full_bar(stage);
-                        if (PAIR) {
+                        if (HALO) {  // step = (cblk, dx): halo box + weights of taps (dy, dx), dy = -1..1
+                            const int hc = kb / 3, dxi = kb % 3;
+                            mbar_expect_tx(fb, a.halo_bytes + 3 * Cfg::B_BYTES);
+                            tma_load_4d(sa, &ta, fb, hc * CL_BK, dxi - 1, y0 - 1, n0);
+#pragma unroll
+                            for (int dyi = 0; dyi < 3; ++dyi)
+                                tma_load_2d(sa + CL_AH_MAX + dyi * Cfg::B_BYTES, &tb, fb,
+                                            ((dyi * 3 + dxi) * a.conv_cb + hc) * CL_BK, nt * BN);
+                        } else if (PAIR) {
                             // both CTAs' bytes land on the leader's full barrier
                             if (rank == 0) mbar_expect_tx(fb, 2 * SBYTES);
                             tma_load_4d_2sm(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
@@ -180,7 +198,12 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                                 tma_load_2d_2sm(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN + rank * (BN / 2));
                         } else {
                             mbar_expect_tx(fb, Cfg::STAGE_BYTES);
-                            tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
+                            if (a.diag & 8)  // diagnostic: A as a 2D box of the flat [pixels][cin] view
+                                tma_load_2d(sa, &ta, fb, cblk * CL_BK, (int)m0);
+                            else if (a.diag & 4)  // diagnostic: centre tap only (no out-of-bounds lines)
+                                tma_load_4d(sa, &ta, fb, cblk * CL_BK, 0, y0, n0);
+                            else
+                                tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
                             tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
                         }
                         if (++stage == STAGES) {
@@ -210,22 +233,28 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     CL_T1(1);
                     tc_fence_after();
                     const uint32_t d_tmem = tmem_base + acc * BN;
-                    for (int kb = 0; kb < a.num_kb; ++kb) {
+                    for (int kb = 0; kb < steps; ++kb) {
                         CL_T0;
                         mbar_wait(full_bar(stage), phase);
                         CL_T1(2);
                         tc_fence_after();
                         const uint32_t sa = sring + stage * SBYTES;
-                        const uint32_t sb = RESB ? bres + kb * Cfg::B_BYTES : sa + Cfg::A_BYTES;
+                        const uint32_t sb = RESB ? bres + kb * Cfg::B_BYTES : sa + (HALO ? CL_AH_MAX : Cfg::A_BYTES);
 #pragma unroll
-                        for (int k = 0; k < CL_BK / 16; ++k) {
-                            if (a.diag & 2) break;  // diagnostic: no MMA
-                            const uint64_t ad = umma_desc_sw128(sa + k * 32u, 16u, 1024u);
-                            const uint64_t bd = umma_desc_sw128(sb + k * 32u, 16u, 1024u);
-                            if (PAIR)
-                                tc_mma_f16_2sm(d_tmem, ad, bd, idesc, (kb > 0 || k > 0) ? 1u : 0u);
-                            else
-                                tc_mma_f16(d_tmem, ad, bd, idesc, (kb > 0 || k > 0) ? 1u : 0u);
+                        for (int dyi = 0; dyi < (HALO ? 3 : 1); ++dyi) {
+                            const uint32_t sad = sa + (uint32_t)dyi * (uint32_t)a.W * 128u;  // dy shift: W rows
+                            const uint32_t sbd = sb + (uint32_t)dyi * Cfg::B_BYTES;
+#pragma unroll
+                            for (int k = 0; k < CL_BK / 16; ++k) {
+                                if (a.diag & 2) break;  // diagnostic: no MMA
+                                const uint64_t ad = umma_desc_sw128(sad + k * 32u, 16u, 1024u);
+                                const uint64_t bd = umma_desc_sw128(sbd + k * 32u, 16u, 1024u);
+                                const uint32_t accum = (kb > 0 || dyi > 0 || k > 0) ? 1u : 0u;
+                                if (PAIR)
+                                    tc_mma_f16_2sm(d_tmem, ad, bd, idesc, accum);
+                                else
+                                    tc_mma_f16(d_tmem, ad, bd, idesc, accum);
+                            }
                         }
                         if (PAIR)
                             tc_commit_2sm_mc(empty_bar(stage), 3);
@@ -240,8 +269,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         tc_commit_2sm_mc(tfull_bar(acc), 3);
                     else
                         tc_commit(tfull_bar(acc));
-                    acc ^= 1;
-                    if (acc == 0) acc_phase ^= 1u;
+                    if (++acc == NACC) {
+                        acc = 0;
+                        acc_phase ^= 1u;
+                    }
                 }
                 if (RESB) tc_commit_2sm_mc(bempty_bar, 3);  // this unit's weights may be replaced
             }
@@ -398,8 +429,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     else
                         mbar_arrive(tempty_bar(acc));
                 }
-                acc ^= 1;
-                if (acc == 0) acc_phase ^= 1u;
+                if (++acc == NACC) {
+                    acc = 0;
+                    acc_phase ^= 1u;
+                }
                 CL_T1(2);
                 CL_T0;
                 if (!(a.diag & 1)) emit(r);
@@ -444,22 +477,18 @@ bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {
     return true;
 }
 
-template <int BN, int POOL, int PAIR, int RESB>
+template <int BN, int POOL, int PAIR, int RESB, int HALO>
 static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvLifArgs a, cudaStream_t s,
                              int num_sms) {
     using Cfg = ClCfg<BN, PAIR>;
-    auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB>;
+    auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB, HALO>;
     uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
-    if (RESB) {
-        const uint32_t resb = (uint32_t)a.num_kb * Cfg::B_BYTES;
-        const int room = (int)((227u * 1024u - smem - resb) / Cfg::A_BYTES);
-        a.stages = room < CL_MAXST ? room : CL_MAXST;
-        if (a.stages < 3) return cudaErrorInvalidValue;
-        smem += resb + a.stages * Cfg::A_BYTES;
-    } else {
-        a.stages = Cfg::STAGES;
-        smem += Cfg::STAGES * Cfg::STAGE_BYTES;
-    }
+    const uint32_t resb = RESB ? (uint32_t)a.num_kb * Cfg::B_BYTES : 0u;
+    const uint32_t sbytes = RESB ? Cfg::A_BYTES : (HALO ? CL_AH_MAX + 3 * Cfg::B_BYTES : Cfg::STAGE_BYTES);
+    const int room = (int)((227u * 1024u - smem - resb) / sbytes);
+    a.stages = room < CL_MAXST ? room : CL_MAXST;
+    if (a.stages < 2) return cudaErrorInvalidValue;
+    smem += resb + a.stages * sbytes;
     if (smem > 227u * 1024u) return cudaErrorInvalidValue;
     static uint32_t set = 0;
     if (smem > set) {
@@ -515,24 +544,36 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
         static const int diag = getenv("SKIPPER_CL_DIAG") ? atoi(getenv("SKIPPER_CL_DIAG")) : 0;
         a.diag = diag;  // timing experiments only (results are wrong when set)
     }
+
     CUtensorMap ta, tb;
-    if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, bhh, bnn)) return cudaErrorInvalidValue;
+    // halo boxes: single CTA, tiles of whole image rows of one image, W >= 8 (dy offsets of W rows
+    // stay on 1024-byte swizzle atoms), box within CL_AH_MAX
+    const char *he = getenv("SKIPPER_CL_HALO");
+    const bool halo = !pair && !(he && atoi(he) == 0) && HW >= CL_BM && a.W >= 8 && a.W <= 32 && !(a.diag & 12);
+    a.halo_bytes = halo ? (int)((bhh + 2) * bw * 128u) : 0;
+    if (a.diag & 8) {
+        if (!make_map_2d(&ta, X, a.Cin, (uint64_t)rows_in * a.B * HW, CL_BK, CL_BM)) return cudaErrorInvalidValue;
+    } else if (!make_map_conv(&ta, X, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, bw, halo ? bhh + 2 : bhh, bnn)) {
+        return cudaErrorInvalidValue;
+    }
     if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, pair ? bn / 2 : bn)) return cudaErrorInvalidValue;
     // resident weights when this CTA's half fits next to >= 4 activation stages
     const int resb_env = getenv("SKIPPER_CL_RESB") ? atoi(getenv("SKIPPER_CL_RESB")) : 1;
     const uint32_t half_bytes = (uint32_t)a.num_kb * (uint32_t)(bn / 2) * CL_BK * 2;
     const bool resb = pair && resb_env && half_bytes + 4u * CL_BM * CL_BK * 2 + 8192u + 4u * a.R <= 220u * 1024u;
-#define CL_LAUNCH(BN_, PAIR_, RESB_)                                                                           \
-    return a.pool ? launch_cl<BN_, 1, PAIR_, RESB_>(ta, tb, a, s, num_sms)                                      \
-                  : launch_cl<BN_, 0, PAIR_, RESB_>(ta, tb, a, s, num_sms)
+#define CL_LAUNCH(BN_, PAIR_, RESB_, HALO_)                                                                    \
+    return a.pool ? launch_cl<BN_, 1, PAIR_, RESB_, HALO_>(ta, tb, a, s, num_sms)                               \
+                  : launch_cl<BN_, 0, PAIR_, RESB_, HALO_>(ta, tb, a, s, num_sms)
     if (bn == 64) {
-        if (resb) CL_LAUNCH(64, 1, 1);
-        if (pair) CL_LAUNCH(64, 1, 0);
-        CL_LAUNCH(64, 0, 0);
+        if (resb) CL_LAUNCH(64, 1, 1, 0);
+        if (pair) CL_LAUNCH(64, 1, 0, 0);
+        if (halo) CL_LAUNCH(64, 0, 0, 1);
+        CL_LAUNCH(64, 0, 0, 0);
     }
-    if (resb) CL_LAUNCH(128, 1, 1);
-    if (pair) CL_LAUNCH(128, 1, 0);
-    CL_LAUNCH(128, 0, 0);
+    if (resb) CL_LAUNCH(128, 1, 1, 0);
+    if (pair) CL_LAUNCH(128, 1, 0, 0);
+    if (halo) CL_LAUNCH(128, 0, 0, 1);
+    CL_LAUNCH(128, 0, 0, 0);
 #undef CL_LAUNCH
 }
 

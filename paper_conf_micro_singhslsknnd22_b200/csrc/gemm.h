@@ -88,7 +88,8 @@ struct ConvLifArgs {
     float lam, theta;
     // filled by launch_conv_lif
     int m_tiles, n_tiles, num_kb, conv_cb;
-    int stages;  // activation ring depth (resident-weight variant)
+    int stages;      // smem ring depth
+    int halo_bytes;  // bytes of one halo activation box (HALO variant)
     int diag;  // SKIPPER_CL_DIAG timing experiments: 1 = no epilogue work, 2 = no MMA
 };
 bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool);

@@ -135,7 +135,7 @@ CONV_LIF_SHAPES = [(5, 6, 16, 16, 64, 128, 1), (4, 3, 8, 8, 128, 256, 0), (3, 5,
                    (6, 2, 32, 32, 64, 64, 1), (3, 7, 16, 16, 128, 128, 0), (1, 2, 16, 16, 64, 128, 1)]
 
 
-@pytest.mark.parametrize("variant", ["single", "pair", "pair_streamed_w"])
+@pytest.mark.parametrize("variant", ["single", "single_tap_boxes", "pair", "pair_streamed_w"])
 @pytest.mark.parametrize("R,nb,h,w,cin,cout,pool", CONV_LIF_SHAPES)
 def test_conv_lif_exact(R, nb, h, w, cin, cout, pool, variant, monkeypatch):
     """Fused conv + LIF (Eq.1) against conv2d in float64 (exact on the grid, rounded once to fp32) and
@@ -143,6 +143,7 @@ def test_conv_lif_exact(R, nb, h, w, cin, cout, pool, variant, monkeypatch):
     from paper_conf_micro_singhslsknnd22_b200 import k_conv_lif
     monkeypatch.setenv("SKIPPER_CL_PAIR", "0" if variant == "single" else "1")  # CTA pair (cta_group::2)
     monkeypatch.setenv("SKIPPER_CL_RESB", "0" if variant == "pair_streamed_w" else "1")  # resident weights
+    monkeypatch.setenv("SKIPPER_CL_HALO", "0" if variant == "single_tap_boxes" else "1")  # halo activation boxes
     g = torch.Generator().manual_seed(R * 131 + nb * h + cin + pool)
     X = spikes((R, nb, h, w, cin), gen=g) * 0.25 * torch.randint(1, 5, (R, nb, h, w, cin), generator=g)
     W = grid((cout, 3, 3, cin), e=9, gen=g)
