@@ -86,8 +86,8 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     constexpr int CW = Cfg::CW;
     constexpr int NW = BN / 32;  // spike words per pixel
     const int STAGES = a.stages;
-    constexpr uint32_t SBYTES =
-        RESB ? Cfg::A_BYTES : (HALO ? CL_AH_MAX + 3 * Cfg::B_BYTES : Cfg::STAGE_BYTES);  // bytes per ring stage
+    constexpr uint32_t A_STAGE = HALO ? CL_AH_MAX : Cfg::A_BYTES;                  // activation part of a stage
+    constexpr uint32_t SBYTES = A_STAGE + (RESB ? 0u : (HALO ? 3u : 1u) * Cfg::B_BYTES);  // bytes per ring stage
     const int steps = HALO ? 3 * a.conv_cb : a.num_kb;  // ring stages per row
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
@@ -182,14 +182,29 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         CL_T1(1);
                         const uint32_t sa = sring + stage * SBYTES;
                         const uint32_t fb = full_bar(stage);
-                        if (HALO) {  // step = (cblk, dx): halo box + weights of taps (dy, dx), dy = -1..1
+                        if (a.diag & 16) {  // diagnostic: no loads (MMA on stale smem)
+                            if (!PAIR || rank == 0) mbar_arrive(fb);
+                        } else if (HALO) {  // step = (cblk, dx): halo box + weights of taps (dy, dx), dy = -1..1
                             const int hc = kb / 3, dxi = kb % 3;
-                            mbar_expect_tx(fb, a.halo_bytes + 3 * Cfg::B_BYTES);
-                            tma_load_4d(sa, &ta, fb, hc * CL_BK, dxi - 1, y0 - 1, n0);
+                            const uint32_t bytes = a.halo_bytes + (RESB ? 0u : 3u * Cfg::B_BYTES);
+                            if (PAIR) {
+                                if (rank == 0) mbar_expect_tx(fb, 2 * bytes);
+                                tma_load_4d_2sm(sa, &ta, fb, hc * CL_BK, dxi - 1, y0 - 1, n0);
+                            } else {
+                                mbar_expect_tx(fb, bytes);
+                                tma_load_4d(sa, &ta, fb, hc * CL_BK, dxi - 1, y0 - 1, n0);
+                            }
+                            if (!RESB) {
 #pragma unroll
-                            for (int dyi = 0; dyi < 3; ++dyi)
-                                tma_load_2d(sa + CL_AH_MAX + dyi * Cfg::B_BYTES, &tb, fb,
-                                            ((dyi * 3 + dxi) * a.conv_cb + hc) * CL_BK, nt * BN);
+                                for (int dyi = 0; dyi < 3; ++dyi) {
+                                    const int kc = ((dyi * 3 + dxi) * a.conv_cb + hc) * CL_BK;
+                                    if (PAIR)
+                                        tma_load_2d_2sm(sa + CL_AH_MAX + dyi * Cfg::B_BYTES, &tb, fb, kc,
+                                                        nt * BN + rank * (BN / 2));
+                                    else
+                                        tma_load_2d(sa + CL_AH_MAX + dyi * Cfg::B_BYTES, &tb, fb, kc, nt * BN);
+                                }
+                            }
                         } else if (PAIR) {
                             // both CTAs' bytes land on the leader's full barrier
                             if (rank == 0) mbar_expect_tx(fb, 2 * SBYTES);
@@ -239,11 +254,13 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         CL_T1(2);
                         tc_fence_after();
                         const uint32_t sa = sring + stage * SBYTES;
-                        const uint32_t sb = RESB ? bres + kb * Cfg::B_BYTES : sa + (HALO ? CL_AH_MAX : Cfg::A_BYTES);
+                        const uint32_t sb = RESB ? bres + kb * Cfg::B_BYTES : sa + A_STAGE;
 #pragma unroll
                         for (int dyi = 0; dyi < (HALO ? 3 : 1); ++dyi) {
                             const uint32_t sad = sa + (uint32_t)dyi * (uint32_t)a.W * 128u;  // dy shift: W rows
-                            const uint32_t sbd = sb + (uint32_t)dyi * Cfg::B_BYTES;
+                            uint32_t sbd = sb + (uint32_t)dyi * Cfg::B_BYTES;
+                            if (HALO && RESB)  // resident weights of tap (dy, dx) for this channel block
+                                sbd = bres + (uint32_t)(((dyi * 3 + kb % 3) * a.conv_cb + kb / 3) * Cfg::B_BYTES);
 #pragma unroll
                             for (int k = 0; k < CL_BK / 16; ++k) {
                                 if (a.diag & 2) break;  // diagnostic: no MMA
@@ -484,7 +501,7 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvL
     auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB, HALO>;
     uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
     const uint32_t resb = RESB ? (uint32_t)a.num_kb * Cfg::B_BYTES : 0u;
-    const uint32_t sbytes = RESB ? Cfg::A_BYTES : (HALO ? CL_AH_MAX + 3 * Cfg::B_BYTES : Cfg::STAGE_BYTES);
+    const uint32_t sbytes = (HALO ? CL_AH_MAX : Cfg::A_BYTES) + (RESB ? 0u : (HALO ? 3u : 1u) * Cfg::B_BYTES);
     const int room = (int)((227u * 1024u - smem - resb) / sbytes);
     a.stages = room < CL_MAXST ? room : CL_MAXST;
     if (a.stages < 2) return cudaErrorInvalidValue;
@@ -549,7 +566,7 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
     // halo boxes: single CTA, tiles of whole image rows of one image, W >= 8 (dy offsets of W rows
     // stay on 1024-byte swizzle atoms), box within CL_AH_MAX
     const char *he = getenv("SKIPPER_CL_HALO");
-    const bool halo = !pair && !(he && atoi(he) == 0) && HW >= CL_BM && a.W >= 8 && a.W <= 32 && !(a.diag & 12);
+    const bool halo = !(he && atoi(he) == 0) && HW >= CL_BM && a.W >= 8 && a.W <= 32 && !(a.diag & 12);
     a.halo_bytes = halo ? (int)((bhh + 2) * bw * 128u) : 0;
     if (a.diag & 8) {
         if (!make_map_2d(&ta, X, a.Cin, (uint64_t)rows_in * a.B * HW, CL_BK, CL_BM)) return cudaErrorInvalidValue;
@@ -560,17 +577,21 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
     // resident weights when this CTA's half fits next to >= 4 activation stages
     const int resb_env = getenv("SKIPPER_CL_RESB") ? atoi(getenv("SKIPPER_CL_RESB")) : 1;
     const uint32_t half_bytes = (uint32_t)a.num_kb * (uint32_t)(bn / 2) * CL_BK * 2;
-    const bool resb = pair && resb_env && half_bytes + 4u * CL_BM * CL_BK * 2 + 8192u + 4u * a.R <= 220u * 1024u;
+    const bool resb = pair && resb_env && half_bytes + 3u * CL_AH_MAX + 8192u + 4u * a.R <= 226u * 1024u;
 #define CL_LAUNCH(BN_, PAIR_, RESB_, HALO_)                                                                    \
     return a.pool ? launch_cl<BN_, 1, PAIR_, RESB_, HALO_>(ta, tb, a, s, num_sms)                               \
                   : launch_cl<BN_, 0, PAIR_, RESB_, HALO_>(ta, tb, a, s, num_sms)
     if (bn == 64) {
+        if (resb && halo) CL_LAUNCH(64, 1, 1, 1);
         if (resb) CL_LAUNCH(64, 1, 1, 0);
+        if (pair && halo) CL_LAUNCH(64, 1, 0, 1);
         if (pair) CL_LAUNCH(64, 1, 0, 0);
         if (halo) CL_LAUNCH(64, 0, 0, 1);
         CL_LAUNCH(64, 0, 0, 0);
     }
+    if (resb && halo) CL_LAUNCH(128, 1, 1, 1);
     if (resb) CL_LAUNCH(128, 1, 1, 0);
+    if (pair && halo) CL_LAUNCH(128, 1, 0, 1);
     if (pair) CL_LAUNCH(128, 1, 0, 0);
     if (halo) CL_LAUNCH(128, 0, 0, 1);
     CL_LAUNCH(128, 0, 0, 0);
