@@ -36,7 +36,7 @@ import numpy as np
 from .layers import conv3x3, conv3x3_input_grad, conv3x3_weight_grad, pool2, pool2_T
 from .lif import lif_step, surrogate_grad
 from .numerics import bf16_round
-from .skipper import keep_mask, kept_lists, spike_sum_threshold
+from .skipper import keep_mask, kept_lists, sam_weighted, spike_sum_threshold
 
 
 @dataclass
@@ -53,6 +53,8 @@ class StepConfig:
     dz: np.ndarray | None = None         # test hook: impose the readout gradient
     T_norm: int | None = None            # readout normalisation (default T)
     s_global: np.ndarray | None = None   # data-parallel: allreduced s (reading 19)
+    sam: str = "spikes"                  # SAM metric: "spikes" (Eq.4) | "weighted" (NEXT-2, reading 22)
+    counts_global: np.ndarray | None = None  # data-parallel: allreduced per-layer counts (weighted SAM)
     record: bool = False
     trace: bool = False
 
@@ -63,6 +65,8 @@ class StepResult:
     z: np.ndarray
     dz: np.ndarray
     s: np.ndarray                 # int64 [T], local batch
+    counts: np.ndarray            # int64 [L_n + 1][T] per-layer spike counts (row 0 = input), local batch
+    sam: np.ndarray               # the policy metric the mask is computed from (int64 or float64 [T])
     sst: np.ndarray | None        # float64 [C] (skip mode)
     keep: np.ndarray              # bool [T]
     kept: list                    # per segment, ascending kept t
@@ -173,6 +177,7 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
     U = [np.zeros((B,) + neuron_shape(L), np.float32) for L in spk]
     o = [np.zeros((B,) + neuron_shape(L), np.uint8) for L in spk]
     s = np.zeros(T, np.int64)
+    counts = np.zeros((len(spk) + 1, T), np.int64)
     cnt = np.zeros((B,) + out_shape(spk[-1]), np.float64)
     ckpt = {}
     stored = []          # FULL: list over t of (U list, o list, a list)
@@ -181,6 +186,9 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
     for t in range(T):
         U, o, a = forward_step(net, Wb, x[t], U, o)
         s[t] = spike_sum(x[t], o)
+        counts[0, t] = int(np.asarray(x[t], np.int64).sum())
+        for l in range(len(spk)):
+            counts[l + 1, t] = int(np.asarray(o[l], np.int64).sum())
         cnt += a[-1]
         if record:
             for l in range(len(spk)):
@@ -196,7 +204,7 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
                 trace.append(("ckpt", t))
         if trace is not None:
             trace.append(("first", t))
-    return {"s": s, "cnt": cnt, "ckpt": ckpt, "stored": stored,
+    return {"s": s, "counts": counts, "cnt": cnt, "ckpt": ckpt, "stored": stored,
             "first_U": first_U, "first_o": first_o}
 
 
@@ -299,7 +307,14 @@ def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
     if cfg.dz is not None:
         dz = np.asarray(cfg.dz, np.float64)
 
-    s_pol = s if cfg.s_global is None else np.asarray(cfg.s_global, np.int64)
+    if cfg.sam == "weighted":
+        counts = first["counts"] if cfg.counts_global is None else np.asarray(cfg.counts_global, np.int64)
+        neurons = [int(np.prod(x.shape[2:]))] + [int(np.prod(neuron_shape(L))) for L in spk]
+        s_pol = sam_weighted(counts, neurons)
+    elif cfg.sam == "spikes":
+        s_pol = s if cfg.s_global is None else np.asarray(cfg.s_global, np.int64)
+    else:
+        raise ValueError(f"unknown SAM metric {cfg.sam!r}")
     sst = None
     if mode == "skip":
         if cfg.keep is not None:
@@ -344,7 +359,7 @@ def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
                 trace.append(("release", c))
     # readout weight gradient once, over the kept rows of every segment
     dW[Ls] += dz.T @ cnt_kept.reshape(B, -1) / T_norm
-    return StepResult(loss=loss, z=z, dz=dz, s=s, sst=sst, keep=keep, kept=kept, dW=dW,
+    return StepResult(loss=loss, z=z, dz=dz, s=s, counts=first["counts"], sam=s_pol, sst=sst, keep=keep, kept=kept, dW=dW,
                       cnt=first["cnt"], cnt_kept=cnt_kept, ledger_peak=ledger.peak,
                       first_U=first["first_U"], first_o=first["first_o"],
                       rec_U=rec_U, rec_o=rec_o, trace=trace or [])

@@ -10,6 +10,10 @@ Keep rule: recompute t iff s_t > SST_c, otherwise skip.
   reading 9: t = cS is the checkpoint and is never skipped (Fig. 6 skips only
   within t in {1..9} and {11..19}, P:899-901);
   reading 13: strict '>', and p == 0 keeps every step (SKIP(p=0) == CKPT).
+SAM variants (NEXT-2, "the sum of spike counts weighted by the neuron count in each
+layer"): reading 22 - 'weighted' divides each layer's count by its neurons per sample (l = 0 is the
+input), s_t = sum_l count_l,t / N_l in float64, summed in layer order l = 0..L_n (per-layer firing
+rates, so small layers weigh as much as large ones).  The default 'spikes' is Eq.4.
 Memory, Eq.3 (P:816-838) ActCost = O(T/C) + O(C); Eq.6 (P:1063-1076)
   ActCost_skipper = O((1-p/100) T/C) + O(C); Eq.7 (P:1077-1102) p/100 <= 1 - C*L_n/T.
 """
@@ -18,10 +22,26 @@ from __future__ import annotations
 import numpy as np
 
 
+def _metric(s):
+    """SAM values as given: integer spike sums stay int64, fractional metrics float64."""
+    s = np.asarray(s)
+    return s.astype(np.int64) if np.issubdtype(s.dtype, np.integer) else s.astype(np.float64)
+
+
+def sam_weighted(counts: np.ndarray, neurons) -> np.ndarray:
+    """NEXT-2 metric (reading 22): counts int64 [L_n + 1][T] (row 0 = input spikes), neurons per
+    sample of each row -> s_t = sum_l counts[l][t] / neurons[l], float64, accumulated in l order."""
+    counts = np.asarray(counts, np.int64)
+    s = np.zeros(counts.shape[1], np.float64)
+    for l in range(counts.shape[0]):
+        s = s + counts[l].astype(np.float64) / float(neurons[l])
+    return s
+
+
 def spike_sum_threshold(s: np.ndarray, T: int, C: int, p: float) -> np.ndarray:
     """SST_c for c = 0..C-1 (Eq.5), float64, via numpy.percentile(method='linear')."""
     S = T // C
-    s = np.asarray(s, dtype=np.int64)
+    s = _metric(s)
     return np.array([np.percentile(s[c * S:(c + 1) * S], p) for c in range(C)], dtype=np.float64)
 
 
@@ -32,7 +52,7 @@ def keep_mask(s: np.ndarray, T: int, C: int, p: float) -> np.ndarray:
     if p == 0:
         return keep
     sst = spike_sum_threshold(s, T, C, p)
-    s = np.asarray(s, dtype=np.int64)
+    s = _metric(s)
     for c in range(C):
         for t in range(c * S + 1, (c + 1) * S):
             keep[t] = s[t] > sst[c]

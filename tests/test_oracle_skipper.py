@@ -136,3 +136,57 @@ def test_eq7_bounds_for_workloads():
     assert eq7_p_max(100, 10, 6) == pytest.approx(40.0)    # cfg 2 -> p=40
     assert eq7_p_max(200, 5, 11) == pytest.approx(72.5)    # cfg 3
     assert eq7_p_max(20, 2, 2) == pytest.approx(80.0)      # cfg 1
+
+
+# ---------------------------------------------------------------- NEXT-2: neuron-count-weighted SAM
+def test_sam_weighted_hand_example():
+    """Reading 22 on a hand-worked case: counts [[2,0,4],[1,3,0]], neurons [2, 4]."""
+    from oracle.skipper import sam_weighted
+    s = sam_weighted(np.array([[2, 0, 4], [1, 3, 0]]), [2, 4])
+    assert s.tolist() == [1.25, 0.75, 2.0]
+
+
+def test_sam_weighted_equal_sizes_reduces_to_spike_sum():
+    """With every layer the same (power-of-two) size the weighted metric is the spike sum / N, and the
+    percentile threshold and keep mask are scale-equivariant: the masks are identical."""
+    from oracle.skipper import sam_weighted
+    rng = np.random.default_rng(3)
+    for _ in range(200):
+        T, C = 40, 4
+        counts = rng.integers(0, 300, size=(3, T))
+        p = float(rng.choice([10, 25, 40, 50, 75]))
+        w = sam_weighted(counts, [64, 64, 64])
+        assert np.array_equal(keep_mask(w, T, C, p), keep_mask(counts.sum(0), T, C, p))
+
+
+def test_sam_weighted_network_brute_force():
+    """train_step(sam='weighted'): the policy metric equals the per-layer firing counts recorded in the
+    first pass divided by the layer sizes, and the mask is the Eq.5 rule applied to it."""
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net, seed=0)
+    x, y = synth.make_inputs(net, 12, 3, seed=1)
+    res = train_step(net, W, x, y, StepConfig(T=12, C=2, p=50.0, mode="skip", sam="weighted", record=True))
+    n0 = int(np.prod(x.shape[2:]))
+    brute = np.array([x[t].astype(np.int64).sum() / n0 +
+                      sum(res.first_o[l][t].astype(np.int64).sum() / res.first_o[l][t][0].size
+                          for l in range(len(res.first_o))) for t in range(12)])
+    assert np.allclose(res.sam, brute, rtol=1e-15, atol=0)
+    assert np.array_equal(res.keep, keep_mask(res.sam, 12, 2, 50.0))
+    assert res.counts.shape == (len(res.first_o) + 1, 12)
+    assert np.array_equal(res.counts.sum(0), res.s)
+
+
+def test_sam_weighted_changes_the_mask_somewhere():
+    """The variant is live: on the VGG-5 topology (layers of very different sizes) the weighted and
+    plain metrics select different steps for some seed."""
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net, seed=0)
+    differ = False
+    for seed in range(1, 8):
+        x, y = synth.make_inputs(net, 20, 2, seed=seed)
+        a = train_step(net, W, x, y, StepConfig(T=20, C=2, p=50.0, mode="skip"))
+        b = train_step(net, W, x, y, StepConfig(T=20, C=2, p=50.0, mode="skip", sam="weighted"))
+        differ |= not np.array_equal(a.keep, b.keep)
+        if differ:
+            break
+    assert differ
