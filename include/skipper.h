@@ -63,6 +63,12 @@ typedef enum { SKIPPER_MODE_FULL = 0, SKIPPER_MODE_CKPT = 1, SKIPPER_MODE_SKIP =
 typedef enum { SKIPPER_PASS_FIRST = 0, SKIPPER_PASS_RECOMPUTE = 1, SKIPPER_PASS_RECORD = 2 } skipper_pass;
 typedef enum { SKIPPER_LAYER_FC = 0, SKIPPER_LAYER_CONV3X3 = 1, SKIPPER_LAYER_READOUT = 2 } skipper_layer_kind;
 typedef enum { SKIPPER_SURR_TRIANGLE = 0, SKIPPER_SURR_FAST_SIGMOID = 1 } skipper_surrogate;
+/* Spike Activity Monitor metric the skip policy thresholds (Eq.5 takes the percentile of it):
+ * SPIKES   s_t = sum over the input and every spiking layer of the spikes at t (Eq.4);
+ * WEIGHTED s_t = sum_l count_l,t / N_l, N_l = neurons per sample of layer l (l = 0: the input), in
+ *          float64 in layer order - "the sum of spike counts weighted by the neuron count in each
+ *          layer" (reading 22). */
+typedef enum { SKIPPER_SAM_SPIKES = 0, SKIPPER_SAM_WEIGHTED = 1 } skipper_sam;
 
 /* One layer.  conv3x3: stride 1, zero pad 1, input and output h x w, optional 2x2
  * average pooling of the output spikes (pool = 2).  fc: h = w = 1.  The last layer
@@ -87,6 +93,7 @@ typedef struct {
     float surr_gamma;      /* triangle: peak; fast sigmoid: slope */
     float lr, beta1, beta2, eps;   /* Adam */
     int debug_record;      /* 1: keep per-step states for skipper_debug_copy (tests) */
+    int sam;               /* skipper_sam (0 = Eq.4 spike sum) */
 } skipper_config;
 
 /* Device-memory allocator used for every context allocation. */
@@ -151,6 +158,10 @@ skipper_status skipper_comm_init(skipper_ctx *ctx, const unsigned char id[128], 
 /* ---- introspection (host sync) ----------------------------------------------- */
 skipper_status skipper_get_loss(skipper_ctx *ctx, float *loss_host);
 skipper_status skipper_get_spike_sums(skipper_ctx *ctx, long long *s_host);      /* [T], global */
+/* per-layer spike counts of the last first pass, [L_n + 1][T] (row 0 = input spikes), global batch */
+skipper_status skipper_get_layer_spike_counts(skipper_ctx *ctx, long long *counts_host);
+/* the SAM values the keep mask was computed from (cfg.sam metric), [T] float64 */
+skipper_status skipper_get_sam(skipper_ctx *ctx, double *sam_host);
 skipper_status skipper_get_keep_mask(skipper_ctx *ctx, unsigned char *keep_host); /* [T] */
 skipper_status skipper_get_sst(skipper_ctx *ctx, double *sst_host);               /* [C]; NaN if p == 0 */
 skipper_status skipper_mem_stats(skipper_ctx *ctx, size_t *current_bytes, size_t *peak_bytes);

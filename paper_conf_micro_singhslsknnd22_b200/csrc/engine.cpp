@@ -114,7 +114,9 @@ struct skipper_ctx {
     unsigned char *x_stage = nullptr;
     int *y_stage = nullptr;
     // host-side step state
-    std::vector<long long> s_host;
+    std::vector<long long> s_host;         // Eq.4 spike sums [T]
+    std::vector<long long> counts_host;    // per-layer spike counts [(Ls + 1)][T], row 0 = input
+    std::vector<double> sam_host;          // the SAM metric thresholded by Eq.5 [T]
     std::vector<unsigned char> keep;
     std::vector<double> sst;
     std::vector<std::vector<int>> kept;
@@ -295,6 +297,24 @@ extern "C" double skipper_sst_host(const long long *s, int n, double p) {
     return a + (double)diff * g;
 }
 
+// the same on float64 values (the weighted SAM metric): lerp on doubles as numpy does
+static double sst_double(const double *s, int n, double p) {
+    if (n <= 0) return NAN;
+    std::vector<double> v(s, s + n);
+    std::sort(v.begin(), v.end());
+    const double q = p / 100.0;
+    const double vi = (double)(n - 1) * q;
+    const double lo_d = std::floor(vi);
+    long long lo = (long long)lo_d;
+    if (lo < 0) lo = 0;
+    if (lo > n - 1) lo = n - 1;
+    const long long hi = std::min<long long>(lo + 1, n - 1);
+    const double g = vi - lo_d;
+    const double diff = v[hi] - v[lo];
+    if (g >= 0.5) return v[hi] - diff * (1.0 - g);
+    return v[lo] + diff * g;
+}
+
 // ------------------------------------------------------------------------------------ create
 static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *layers, int n) {
     if (!layers || n < 2) return fail(c, SKIPPER_EINVAL, "need at least one spiking layer and a readout");
@@ -459,6 +479,8 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     if (cfg->mode < 0 || cfg->mode > 2) return bail(fail(c, SKIPPER_EINVAL, "unknown mode %d", cfg->mode));
     if (cfg->surrogate != SKIPPER_SURR_TRIANGLE && cfg->surrogate != SKIPPER_SURR_FAST_SIGMOID)
         return bail(fail(c, SKIPPER_EINVAL, "unknown surrogate %d", cfg->surrogate));
+    if (cfg->sam != SKIPPER_SAM_SPIKES && cfg->sam != SKIPPER_SAM_WEIGHTED)
+        return bail(fail(c, SKIPPER_EINVAL, "unknown SAM metric %d", cfg->sam));
     if (cfg->mode == SKIPPER_MODE_FULL) {
         c->C = 1;
     } else {
@@ -558,8 +580,8 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
             }
         }
     }
-    AL(c->s_part, (size_t)c->T * 32);
-    AL(c->s_dev, (size_t)c->T);
+    AL(c->s_part, (size_t)(c->Ls + 1) * c->T * 32);  // [layer group][T][32] partial counters
+    AL(c->s_dev, (size_t)(c->Ls + 1) * c->T);
     const Layer &last = c->L[c->Ls - 1];
     const Layer &ro = c->L.back();
     AL(c->cnt, (size_t)c->B * last.Nout);
@@ -582,6 +604,8 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     if (s != SKIPPER_OK) return bail(s);
     if (cudaStreamSynchronize(c->st) != cudaSuccess) return bail(fail(c, SKIPPER_ECUDA, "stream sync failed at create"));
     c->s_host.assign(c->T, 0);
+    c->counts_host.assign((size_t)(c->Ls + 1) * c->T, 0);
+    c->sam_host.assign(c->T, 0.0);
     c->keep.assign(c->T, 1);
     c->sst.assign(c->C, NAN);
     *out = c;
@@ -617,8 +641,8 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
     if (!c->L.empty() && c->Ls > 0) {
         const Layer &last = c->L[c->Ls - 1];
         const Layer &ro = c->L.back();
-        dev_free(c, c->s_part, (size_t)c->T * 32 * 4);
-        dev_free(c, c->s_dev, (size_t)c->T * 8);
+        dev_free(c, c->s_part, (size_t)(c->Ls + 1) * c->T * 32 * 4);
+        dev_free(c, c->s_dev, (size_t)(c->Ls + 1) * c->T * 8);
         dev_free(c, c->cnt, (size_t)c->B * last.Nout * 4);
         dev_free(c, c->cnt_kept, (size_t)c->B * last.Nout * 4);
         dev_free(c, c->g_last, (size_t)c->B * last.Nout * 4);
@@ -848,9 +872,12 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
 }
 
 // ------------------------------------------------------------------------------------ step pieces
+// SAM partial counters of one layer group (0 = input spikes, l + 1 = spiking layer l): [T][32]
+static unsigned *spart(skipper_ctx *c, int group) { return c->s_part + (size_t)group * c->T * 32; }
+
 static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
     if (c->prof_on) prof_resolve(c);
-    CKS(zero_dev(c, c->s_part, (size_t)c->T * 32 * 4));
+    CKS(zero_dev(c, c->s_part, (size_t)(c->Ls + 1) * c->T * 32 * 4));
     CKS(zero_dev(c, c->cnt, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
     CKS(zero_dev(c, c->cnt_kept, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
     CKS(zero_dev(c, c->loss_dev, 4));
@@ -898,7 +925,7 @@ static skipper_status stage_input(skipper_ctx *c, const int *rows, int t0, int R
     const double bytes = (double)R * c->B * (c->in_elems + c->in_row * 2);
     ProfScope ps(c, K_STAGE, bytes, 0);
     CK(sk::launch_stage_rows(c->x_cur, c->xg, rows, t0, R, c->B, c->in_h, c->in_w, c->in_c, kind, c->K0,
-                             c->in_elems, sam ? c->s_part : nullptr, c->st));
+                             c->in_elems, sam ? spart(c, 0) : nullptr, c->st));
     return SKIPPER_OK;
 }
 
@@ -929,7 +956,7 @@ static skipper_status forward_tail_first(skipper_ctx *c) {
         a.ckU = l.ckU;
         a.cko = l.cko;
         a.ck_every = c->S;
-        a.s_part = c->s_part;
+        a.s_part = spart(c, i + 1);
         a.t0 = 0;
         a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
         a.dbg_U = c->cfg.debug_record ? l.dbg[0] : nullptr;
@@ -974,7 +1001,8 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     a.Po_out = out;
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
-    a.s_part = restore ? nullptr : c->s_part;
+    a.s_part = restore ? nullptr : spart(c, 1);
+    a.s_part_in = restore ? nullptr : spart(c, 0);
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
     a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
     const double bytes = (double)R * c->B * (c->in_elems + l.Nout * 2 + (a.U_out ? l.N * 4 : 0)) + bn * 10;
@@ -1006,7 +1034,7 @@ static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16
     a.Po_out = out;
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
-    a.s_part = restore ? nullptr : c->s_part;
+    a.s_part = restore ? nullptr : spart(c, i + 1);
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
     a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
     a.lam = l.d.lambda;
@@ -1059,7 +1087,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         a.Po_out = out;
         a.ckU = record ? nullptr : l.ckU + (size_t)seg * c->B * l.N;
         a.cko = record ? nullptr : l.cko + (size_t)seg * c->B * l.N;
-        a.s_part = c->s_part;
+        a.s_part = spart(c, i + 1);
         a.row_t = nullptr;
         a.t0 = t0;
         a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
@@ -1083,7 +1111,8 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
 static skipper_status comm_allreduce_s(skipper_ctx *c) {
     if (c->comm.world > 1) {
         std::string e;
-        if (!c->comm.allreduce_i64(c->s_dev, c->T, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+        if (!c->comm.allreduce_i64(c->s_dev, (c->Ls + 1) * c->T, c->st, &e))  // per-layer counts
+            return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
     }
     return SKIPPER_OK;
 }
@@ -1092,25 +1121,41 @@ static skipper_status comm_allreduce_s(skipper_ctx *c) {
 static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     const Layer &last = c->L[c->Ls - 1];
     const Layer &ro = c->L.back();
-    ProfScope ps0(c, K_READOUT, (double)c->T * 32 * 4, 0);
-    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, c->T, c->st));
+    ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
+    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
     ProfScope ps1(c, K_READOUT, (double)c->B * last.Nout * 8 + (double)ro.wcount * 2, 4.0 * c->B * last.Nout * ro.Cout);
     c->launches += 2;  // z, cross-entropy and dL/da^{L-1} kernels
     CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
                                ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
     CKS(comm_allreduce_s(c));
-    CK(cudaMemcpyAsync(c->s_host.data(), c->s_dev, (size_t)c->T * 8, cudaMemcpyDeviceToHost, c->st));
+    CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
+                       c->st));
     CK(cudaStreamSynchronize(c->st));  // the one host sync of the step
+    // SAM (Eq.4) and the policy metric: Eq.4 totals, or the neuron-count-weighted sum (reading 22)
+    for (int t = 0; t < c->T; ++t) {
+        long long tot = 0;
+        double w = 0.0;
+        for (int g = 0; g <= c->Ls; ++g) {
+            const long long v = c->counts_host[(size_t)g * c->T + t];
+            tot += v;
+            w = w + (double)v / (double)(g == 0 ? c->in_elems : c->L[g - 1].N);
+        }
+        c->s_host[t] = tot;
+        c->sam_host[t] = c->cfg.sam == SKIPPER_SAM_WEIGHTED ? w : (double)tot;
+    }
     const int C = c->C, S = c->S;
     c->kept.assign(C, {});
     c->keep.assign(c->T, 1);
     c->sst.assign(C, NAN);
     const bool skip = c->cfg.mode == SKIPPER_MODE_SKIP && c->cfg.p != 0.0;
     for (int seg = 0; seg < C; ++seg) {
-        if (skip) c->sst[seg] = skipper_sst_host(c->s_host.data() + (size_t)seg * S, S, c->cfg.p);
+        if (skip)
+            c->sst[seg] = c->cfg.sam == SKIPPER_SAM_WEIGHTED
+                              ? sst_double(c->sam_host.data() + (size_t)seg * S, S, c->cfg.p)
+                              : skipper_sst_host(c->s_host.data() + (size_t)seg * S, S, c->cfg.p);
         for (int t = seg * S; t < (seg + 1) * S; ++t) {
             bool k = true;
-            if (skip && t != seg * S) k = (double)c->s_host[t] > c->sst[seg];
+            if (skip && t != seg * S) k = c->sam_host[t] > c->sst[seg];
             c->keep[t] = k ? 1 : 0;
             if (k) c->kept[seg].push_back(t);
         }
@@ -1475,6 +1520,18 @@ extern "C" skipper_status skipper_get_spike_sums(skipper_ctx *c, long long *s_ho
 extern "C" skipper_status skipper_get_keep_mask(skipper_ctx *c, unsigned char *keep_host) {
     CKS(check_ctx(c));
     std::copy(c->keep.begin(), c->keep.end(), keep_host);
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_get_layer_spike_counts(skipper_ctx *c, long long *counts_host) {
+    CKS(check_ctx(c));
+    if (!counts_host) return fail(c, SKIPPER_EINVAL, "null output");
+    std::copy(c->counts_host.begin(), c->counts_host.end(), counts_host);
+    return SKIPPER_OK;
+}
+extern "C" skipper_status skipper_get_sam(skipper_ctx *c, double *sam_host) {
+    CKS(check_ctx(c));
+    if (!sam_host) return fail(c, SKIPPER_EINVAL, "null output");
+    std::copy(c->sam_host.begin(), c->sam_host.end(), sam_host);
     return SKIPPER_OK;
 }
 extern "C" skipper_status skipper_get_sst(skipper_ctx *c, double *sst_host) {

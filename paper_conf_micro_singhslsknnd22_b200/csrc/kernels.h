@@ -77,7 +77,8 @@ struct L0FwdArgs {
     uint16_t *Po_out;      // [R][B*PH*PW*N] bf16
     float *ckU;            // FIRST: checkpoint slot (after row 0) or null
     uint8_t *cko;
-    unsigned *s_part;      // SAM partials (input + this layer) or null
+    unsigned *s_part;      // SAM partials [T][32] of this layer's spikes, or null
+    unsigned *s_part_in;   // SAM partials [T][32] of the input spikes (l = 0), or null
     float *dbg_U;
     uint8_t *dbg_o;
 };

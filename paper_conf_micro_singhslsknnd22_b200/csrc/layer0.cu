@@ -119,6 +119,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
     unsigned *row_cnt = reinterpret_cast<unsigned *>(smem_raw + (tmem_slot + 16 - raw));
     long long *s_rowt = reinterpret_cast<long long *>(smem_raw + ((tmem_slot + 16 + 4 * a.R + 7) & ~7u) - raw);
     uint2 *s_lut = reinterpret_cast<uint2 *>(s_rowt + a.R);  // 4 bits -> 4 bf16 {0, 1}
+    unsigned *row_cnt_in = reinterpret_cast<unsigned *>(s_lut + 16);  // input spike counts per row
     uint8_t *sB_ptr = smem_raw + (sB - raw);
     uint8_t *sA_ptr = smem_raw + (sA - raw);
 
@@ -134,6 +135,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
     }
     for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
         row_cnt[r] = 0;
+        row_cnt_in[r] = 0;
         s_rowt[r] = a.row_t ? a.row_t[r] : (long long)a.t0 + r;
     }
     if (threadIdx.x < 16) {
@@ -288,9 +290,9 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 const uint2 lo = s_lut[(m >> (8 * j)) & 15u], hi = s_lut[(m >> (8 * j + 4)) & 15u];
                 *reinterpret_cast<uint4 *>(dst + j * L0_PLANE_A) = make_uint4(lo.x, lo.y, hi.x, hi.y);
             }
-            if (a.s_part) {
+            if (a.s_part_in) {
                 const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
-                if (lane == 0 && v) atomicAdd(&row_cnt[cri], v);
+                if (lane == 0 && v) atomicAdd(&row_cnt_in[cri], v);
             }
             L0_T1(5); L0_T0; fence_async_shared(); L0_T1(6);
             __syncwarp();
@@ -481,11 +483,10 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
     tc_fence_after();
     if (warp == F0_MMA_WARP) tmem_dealloc<TMEM_COLS>(tmem_base);
     L0_STAT_DUMP;
-    if (a.s_part) {
-        for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
-            const unsigned v = row_cnt[r];
-            if (v) atomicAdd(a.s_part + row_time(r) * 32 + (blockIdx.x & 31), v);
-        }
+    for (int r = threadIdx.x; r < a.R; r += blockDim.x) {
+        const unsigned v = row_cnt[r], vi = row_cnt_in[r];
+        if (a.s_part && v) atomicAdd(a.s_part + row_time(r) * 32 + (blockIdx.x & 31), v);
+        if (a.s_part_in && vi) atomicAdd(a.s_part_in + row_time(r) * 32 + (blockIdx.x & 31), vi);
     }
 }
 
@@ -523,7 +524,7 @@ cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
     const int tiles = g.tiles_b * g.tiles_y * g.tiles_x;
     if (tiles == 0 || a.R == 0) return cudaSuccess;
     const uint32_t smem =
-        1024 + L0_STAGES * L0_A_BYTES + 4 * a.N * 16 + L0_PGROUPS * L0_RING_BYTES + 8 * (2 * L0_STAGES + 2 * L0_NACC) + 16 + 4 * a.R + 8 + 8 * a.R + 128;
+        1024 + L0_STAGES * L0_A_BYTES + 4 * a.N * 16 + L0_PGROUPS * L0_RING_BYTES + 8 * (2 * L0_STAGES + 2 * L0_NACC) + 16 + 4 * a.R + 8 + 8 * a.R + 128 + 4 * a.R;
     if (smem > 200 * 1024) return cudaErrorInvalidValue;
     const int grid = tiles < num_sms ? tiles : num_sms;
     if (a.W * a.C0 % 8) return cudaErrorInvalidValue;

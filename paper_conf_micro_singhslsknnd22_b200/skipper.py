@@ -38,7 +38,7 @@ class Config(ct.Structure):
     _fields_ = [("T", ct.c_int), ("C", ct.c_int), ("p", ct.c_double), ("mode", ct.c_int), ("batch", ct.c_int),
                 ("global_batch", ct.c_int), ("surrogate", ct.c_int), ("surr_gamma", ct.c_float),
                 ("lr", ct.c_float), ("beta1", ct.c_float), ("beta2", ct.c_float), ("eps", ct.c_float),
-                ("debug_record", ct.c_int)]
+                ("debug_record", ct.c_int), ("sam", ct.c_int)]
 
 
 ALLOC_FN = ct.CFUNCTYPE(ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
@@ -75,6 +75,8 @@ def _load():
         "skipper_comm_init": (I, [P, P, I, I]),
         "skipper_get_loss": (I, [P, P]),
         "skipper_get_spike_sums": (I, [P, P]),
+        "skipper_get_layer_spike_counts": (I, [P, P]),
+        "skipper_get_sam": (I, [P, P]),
         "skipper_get_keep_mask": (I, [P, P]),
         "skipper_get_sst": (I, [P, P]),
         "skipper_mem_stats": (I, [P, P, P]),
@@ -121,10 +123,13 @@ def make_layers(net):
     return arr
 
 
+SAM = {"spikes": 0, "weighted": 1}
+
+
 def make_config(T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle", gamma=0.3,
-                lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False):
+                lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, sam="spikes"):
     return Config(T, C, float(p), MODE[mode], batch, global_batch, SURROGATE[surrogate], gamma, lr, beta1, beta2,
-                  eps, 1 if debug_record else 0)
+                  eps, 1 if debug_record else 0, SAM[sam])
 
 
 def sst_host(values, p):
@@ -169,7 +174,7 @@ class SkipperNet:
 
     def __init__(self, net, T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle",
                  gamma=0.3, lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, stream=None,
-                 torch_allocator=True):
+                 torch_allocator=True, sam="spikes"):
         torch = _torch()
         self.net = net
         self.T, self.B = T, batch
@@ -178,7 +183,7 @@ class SkipperNet:
         self.device = torch.cuda.current_device()
         self.stream = stream if stream is not None else torch.cuda.current_stream()
         self.cfg = make_config(T, C, p, mode, batch, global_batch, surrogate, gamma, lr, beta1, beta2, eps,
-                               debug_record)
+                               debug_record, sam)
         self._layers = make_layers(net)
         self._alloc = TorchAllocator(self.device) if torch_allocator else None
         h = ct.c_void_p()
@@ -293,6 +298,18 @@ class SkipperNet:
     def spike_sums(self):
         a = np.zeros(self.T, np.int64)
         self._c(lib.skipper_get_spike_sums(self.ctx, a.ctypes.data))
+        return a
+
+    def layer_spike_counts(self):
+        """[L_n + 1][T] int64 per-layer spike counts of the last first pass (row 0 = input spikes)."""
+        a = np.zeros((len(self.spiking) + 1, self.T), np.int64)
+        self._c(lib.skipper_get_layer_spike_counts(self.ctx, a.ctypes.data))
+        return a
+
+    def sam_values(self):
+        """[T] float64: the SAM metric the keep mask was computed from."""
+        a = np.zeros(self.T, np.float64)
+        self._c(lib.skipper_get_sam(self.ctx, a.ctypes.data))
         return a
 
     def keep_mask(self):

@@ -19,10 +19,10 @@ def _cuda():
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
 
 
-def run_gpu(net, W, x, y, T, C, p, mode, steps=1):
+def run_gpu(net, W, x, y, T, C, p, mode, steps=1, sam="spikes"):
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
     B = x.shape[1]
-    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True)
+    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True, sam=sam)
     m.set_weights(W)
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     yd = torch.from_numpy(np.ascontiguousarray(y)).cuda()
@@ -41,15 +41,17 @@ def grad_ok(g, r, tol=1e-3):
     return rel <= tol and mx <= tol, f"normwise {rel:.2e} maxabs {mx:.2e}"
 
 
-def check_parity(name, T, B, C, p, mode, lam=None, seed=0):
+def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes"):
     net = synth.net_config(name, lam=lam)
     W = synth.make_weights(net, seed=seed)
     x, y = synth.make_inputs(net, T, B, seed=seed + 1)
-    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True))
-    m, loss = run_gpu(net, W, x, y, T, C, p, mode)
+    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True, sam=sam))
+    m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam)
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
     # SAM and mask (Eq.4, Eq.5)
     np.testing.assert_array_equal(m.spike_sums(), ref.s)
+    np.testing.assert_array_equal(m.layer_spike_counts(), ref.counts)
+    np.testing.assert_array_equal(m.sam_values(), np.asarray(ref.sam, np.float64))  # same fp64 arithmetic
     np.testing.assert_array_equal(m.keep_mask(), ref.keep)
     # first pass and recomputed states per layer
     for l in range(len(spk)):
@@ -179,3 +181,10 @@ def test_memory_ordering_full_ckpt_skip():
 def test_vgg11_reduced(mode):
     """cfg 3 topology (VGG-11: 8 conv incl. 256/512-channel layers down to 2x2, fc 512-4096-4096)."""
     check_parity("vgg11", T=24, B=2, C=2, p=50.0, mode=mode)
+
+
+@pytest.mark.parametrize("name,T,B,C,p", [("tiny_conv", 20, 3, 2, 50.0), ("vgg5", 20, 2, 2, 40.0),
+                                          ("fc784", 20, 4, 2, 50.0)])
+def test_sam_weighted(name, T, B, C, p):
+    """NEXT-2: the neuron-count-weighted SAM (reading 22) selects the same steps as the oracle."""
+    check_parity(name, T=T, B=B, C=C, p=p, mode="skip", sam="weighted")

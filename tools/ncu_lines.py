@@ -1,6 +1,6 @@
 """Per-source-line instruction / stall attribution from an ncu report (cuda,sass source view).
 
-usage: python tools/ncu_lines.py report.ncu-rep [top]
+usage: python tools/ncu_lines.py report.ncu-rep [top] [kernel-substring]
 """
 import csv
 import io
@@ -9,7 +9,7 @@ import sys
 from collections import defaultdict
 
 
-def main(rep, top=30):
+def main(rep, top=30, kfilter=None):
     out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                          capture_output=True, text=True).stdout
     fname, line, src = "?", None, ""
@@ -17,16 +17,22 @@ def main(rep, top=30):
     stall = defaultdict(float)
     text = {}
     hdr = None
+    keep = kfilter is None
     for r in csv.reader(io.StringIO(out)):
         if not r:
             continue
         if r[0] == "File Path":
             fname = r[1].split("/")[-1]
             continue
+        if r[0] == "Function Name":
+            keep = kfilter is None or kfilter in r[1]
+            continue
+        if not keep:
+            continue
         if r[0] == "Line No":
             hdr = r
             continue
-        if hdr is None or r[0] == "Function Name":
+        if hdr is None:
             continue
         if r[0]:
             line = (fname, int(r[0]))
@@ -45,4 +51,4 @@ def main(rep, top=30):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30)
+    main(sys.argv[1], int(sys.argv[2]) if len(sys.argv) > 2 else 30, sys.argv[3] if len(sys.argv) > 3 else None)
