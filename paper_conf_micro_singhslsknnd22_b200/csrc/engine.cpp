@@ -1005,7 +1005,10 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     a.s_part_in = restore ? nullptr : spart(c, 0);
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
     a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
-    const double bytes = (double)R * c->B * (c->in_elems + l.Nout * 2 + (a.U_out ? l.N * 4 : 0)) + bn * 10;
+    // stored passes also emit the im2col rows the layer-0 weight gradient reads (no staging kernel)
+    a.xg_out = (restore || record) && !c->l0_bwd_fused ? c->xg : nullptr;
+    const double bytes = (double)R * c->B * (c->in_elems + l.Nout * 2 + (a.U_out ? l.N * 4 : 0) +
+                                             (a.xg_out ? (double)l.H * l.W * c->K0 * 2 : 0)) + bn * 10;
     const double flops = 2.0 * R * c->B * l.H * l.W * l.Cout * 9 * l.Cin;
     ProfScope ps(c, K_L0_FWD, bytes, flops);
     CK(sk::launch_layer0_fwd(a, c->st, c->num_sms));
@@ -1054,7 +1057,8 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
     // the staged layer-0 operand is needed by the first pass unless layer 0 is fused (or part of the
     // whole-sequence fc tail), and by the layer-0 weight gradient of FULL mode
     const int iend = record ? c->Ls : c->tail0;
-    if ((record && !c->l0_bwd_fused) || (iend > 0 && !c->l0_fused)) CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
+    if ((record && !c->l0_bwd_fused && !c->l0_fused) || (iend > 0 && !c->l0_fused))
+        CKS(stage_input(c, nullptr, t0, R, !c->l0_fused));
     for (int i = 0; i < iend; ++i) {
         Layer &l = c->L[i];
         const uint16_t *in;
@@ -1173,7 +1177,8 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
 static skipper_status recompute_segment(skipper_ctx *c, int seg) {
     const int R = (int)c->kept[seg].size();
     const int *row_t = c->kept_dev + (size_t)seg * c->S;
-    if (!c->l0_bwd_fused) CKS(stage_input(c, row_t, 0, R, false));  // layer-0 weight-gradient operand
+    // layer-0 weight-gradient operand (written by the fused layer-0 kernel itself when it runs)
+    if (!c->l0_bwd_fused && !c->l0_fused) CKS(stage_input(c, row_t, 0, R, false));
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         if (i == 0 && c->l0_fused) {

@@ -81,6 +81,7 @@ struct L0FwdArgs {
     unsigned *s_part_in;   // SAM partials [T][32] of the input spikes (l = 0), or null
     float *dbg_U;
     uint8_t *dbg_o;
+    uint16_t *xg_out;      // or null: also write the bf16 im2col rows [R][B*H*W][32] (weight-gradient operand)
 };
 bool layer0_supported(int B, int H, int W, int C0, int N, int pool);
 

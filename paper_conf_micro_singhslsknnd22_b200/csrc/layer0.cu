@@ -240,12 +240,43 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 tile += gridDim.x;
             }
         int ptile = tile, pri = ri;  // fetch cursor, L0_PD rows (of this group) ahead
-        int cb = 0, cxx = 0;  // build cursor's pixel
+        int cb = 0, cxx = 0, cyy = 0;  // build cursor's pixel
+        // im2col row of (pixel, input row ri) -> the layer-0 weight-gradient operand xg [R][B*H*W][32]
+        auto store_xg = [&](int rr, uint32_t m) {
+            if (cb >= a.B) return;
+            uint4 *dst = reinterpret_cast<uint4 *>(a.xg_out + (((long long)rr * a.B + cb) * a.H * a.W +
+                                                               (long long)cyy * a.W + cxx) * 32);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const uint2 lo = s_lut[(m >> (8 * j)) & 15u], hi = s_lut[(m >> (8 * j + 4)) & 15u];
+                dst[j] = make_uint4(lo.x, lo.y, hi.x, hi.y);
+            }
+        };
+        // RECOMPUTE: row 0 (the checkpoint) has no MMA but its im2col row is part of the operand
+        auto xg_row0 = [&]() {
+            if (!(a.xg_out && a.restore && grp == 0) || cb >= a.B) return;
+            const long long t = s_rowt[0];
+            const int bstart = a.C0 * (cxx - 1), w0 = bstart >> 3, sh = bstart & 7;
+            const uint32_t wmask = (1u << (3 * a.C0)) - 1u;
+            uint32_t m = 0;
+#pragma unroll
+            for (int dy = 0; dy < 3; ++dy) {
+                const int y = cyy + dy - 1;
+                if (y < 0 || y >= a.H) continue;
+                const uint2 *rowp = reinterpret_cast<const uint2 *>(a.x + ((t * a.B + cb) * a.H + y) * (long long)rowbytes);
+                const uint2 c0 = (w0 >= 0 && w0 < rowchunks) ? __ldg(rowp + w0) : make_uint2(0u, 0u);
+                const uint2 c1 = (w0 + 1 >= 0 && w0 + 1 < rowchunks) ? __ldg(rowp + w0 + 1) : make_uint2(0u, 0u);
+                const uint32_t nib = byte_bits4(c0.x) | byte_bits4(c0.y) << 4 | byte_bits4(c1.x) << 8 | byte_bits4(c1.y) << 12;
+                m |= ((nib >> sh) & wmask) << (dy * 3 * a.C0);
+            }
+            store_xg(0, m);
+        };
         auto build_pixel = [&](int tile) {
             int b0, y0, x0;
             tile_origin(tile, b0, y0, x0);
             cb = b0 + bl;
             cxx = x0 + xl;
+            cyy = y0 + yl;
         };
         if (nit_tile > 0) {
             if (ptile < tiles) fetch_pixel(ptile);
@@ -294,6 +325,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
                 if (lane == 0 && v) atomicAdd(&row_cnt_in[cri], v);
             }
+            if (a.xg_out) store_xg(cri, m);
             L0_T1(5); L0_T0; fence_async_shared(); L0_T1(6);
             __syncwarp();
             if (lane == 0) mbar_arrive(full_bar(stage));
@@ -304,6 +336,12 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             }
         }
         cp_async_wait<0>();
+        if (a.xg_out && a.restore && grp == 0) {  // after the pipelined rows: every tile's row 0
+            for (int t2 = blockIdx.x; t2 < tiles; t2 += gridDim.x) {
+                build_pixel(t2);
+                xg_row0();
+            }
+        }
     } else if (warp == F0_MMA_WARP) {
         // ------------------------------------------------------------ MMA issuer
         if (lane == 0) {
