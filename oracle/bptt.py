@@ -19,7 +19,14 @@ PAPER.md citations (P:<line>):
 Readout and loss (reading 5, "loss ... at t=19"): non-spiking
 integrator z = (1/T) W^L sum_t a^{L-1}_t, softmax cross-entropy summed over the
 local batch and divided by the global batch.  Readout gradients run over the
-kept steps only (reading 15).
+kept steps only (reading 15).  A readout marked "gap" integrates the global
+average pool of a^{L-1} (the ResNet20 SNN, reading 23).
+
+ResNet layers (reading 8): a conv layer may have stride 2 (its h, w are the
+output = neuron dims) and a residual source "res" = index r of an earlier
+spiking layer: the option-A shortcut of a^r is added into the layer's current,
+I = W * a^{l-1} + S(a^r) (exact sum, rounded once to float32), and Eq.2's
+gradient wrt a^r gains S^T(delta^l).
 
 Arithmetic contract: forward currents are the exact
 sum of bf16 weights times spike inputs, rounded once to float32 (exact for the
@@ -33,7 +40,8 @@ from dataclasses import dataclass, field
 
 import numpy as np
 
-from .layers import conv3x3, conv3x3_input_grad, conv3x3_weight_grad, pool2, pool2_T
+from .layers import (conv3x3, conv3x3_input_grad, conv3x3_weight_grad, gap, gap_T, pool2, pool2_T,
+                     shortcut_a, shortcut_a_T)
 from .lif import lif_step, surrogate_grad
 from .numerics import bf16_round
 from .skipper import keep_mask, kept_lists, sam_weighted, spike_sum_threshold
@@ -97,11 +105,13 @@ def out_shape(layer) -> tuple:
     return neuron_shape(layer)
 
 
-def synaptic_current(layer, Wb, a_in) -> np.ndarray:
-    """I = W^l P(o^{l-1}) (Eq.1 second term): exact float64 sum, rounded once to float32."""
+def synaptic_current(layer, Wb, a_in, a_res=None) -> np.ndarray:
+    """I = W^l P(o^{l-1}) (Eq.1 second term) [+ S(a^r), reading 8]: exact float64 sum, rounded once to float32."""
     B = a_in.shape[0]
     if layer["kind"] == "conv":
-        I = conv3x3(a_in, Wb)
+        I = conv3x3(a_in, Wb, layer.get("stride", 1))
+        if a_res is not None:
+            I = I + shortcut_a(a_res, a_res.shape[1] // layer["h"], layer["cout"])
     else:
         I = a_in.reshape(B, -1) @ Wb.T
     return I.astype(np.float32)
@@ -121,7 +131,8 @@ def forward_step(net, Wb, x_t, U_prev, o_prev):
     a = [np.asarray(x_t, np.float64)]
     Us, os_ = [], []
     for l, layer in enumerate(spiking_layers(net)):
-        I = synaptic_current(layer, Wb[l], a[l])
+        r = layer.get("res")
+        I = synaptic_current(layer, Wb[l], a[l], None if r is None else a[r + 1])
         U, o = lif_step(U_prev[l], o_prev[l], I, layer["lam"], layer["theta"])
         Us.append(U)
         os_.append(o)
@@ -134,10 +145,15 @@ def spike_sum(x_t, os_) -> int:
     return int(np.asarray(x_t, np.int64).sum()) + sum(int(np.asarray(o, np.int64).sum()) for o in os_)
 
 
-def readout(WbL, cnt, y, T_norm: int, B_global: int):
+def readout_input(cnt, use_gap: bool) -> np.ndarray:
+    """What the readout integrates: the summed a^{L-1}, flattened, or its global average pool (reading 23)."""
+    return gap(cnt) if use_gap else np.asarray(cnt, np.float64).reshape(cnt.shape[0], -1)
+
+
+def readout(WbL, cnt, y, T_norm: int, B_global: int, use_gap: bool = False):
     """z = W^L cnt / T; loss = sum_b CE(z_b, y_b) / B_global; dz = (softmax - onehot) / B_global."""
     B = cnt.shape[0]
-    c2 = cnt.reshape(B, -1)
+    c2 = readout_input(cnt, use_gap)
     z = c2 @ WbL.T / T_norm
     zmax = z.max(axis=1, keepdims=True)
     e = np.exp(z - zmax)
@@ -240,17 +256,25 @@ def backward_segment(net, Wb, rows_state, dz, T_norm, carry, dW, cnt_kept, cfg: 
     K = len(rows_state)
     B = dz.shape[0]
     WbL = Wb[Ls]
+    use_gap = bool(net["layers"][-1].get("gap"))
     # readout input summed over the kept rows (readout gradients over kept t, reading 15)
     for j in reversed(range(K)):
         cnt_kept += rows_state[j][2][Ls]
-    # grad wrt the readout input, identical at every kept t: dz W^L / T
-    ga_const = (dz @ WbL / T_norm).reshape((B,) + out_shape(spk[-1]))
+    # grad wrt the readout input, identical at every kept t: dz W^L / T (through the GAP when present)
+    ga_const = dz @ WbL / T_norm
+    if use_gap:
+        ga_const = gap_T(ga_const, out_shape(spk[-1])[:2])
+    ga_const = ga_const.reshape((B,) + out_shape(spk[-1]))
     ga = [ga_const] * K
+    ga_res = {}                                                   # residual source r -> S^T(delta) per row
     new_carry = [None] * Ls
     for l in reversed(range(Ls)):
         layer = spk[l]
         lam = float(layer["lam"])
         pooled = layer["kind"] == "conv" and layer["pool"]
+        if l in ga_res:                                           # dL/da^l also flows through the shortcut
+            extra = ga_res.pop(l)
+            ga = [ga[j] + extra[j] for j in range(K)]
         g = [pool2_T(gj) if pooled else gj for gj in ga]           # dL/do^l_t (spatial path)
         delta = [None] * K
         nxt = carry[l]
@@ -260,16 +284,23 @@ def backward_segment(net, Wb, rows_state, dz, T_norm, carry, dW, cnt_kept, cfg: 
             nxt = delta[j]
         new_carry[l] = delta[0]
         db = [bf16_round(d) for d in delta] if cfg.emulate_bf16 else delta
+        stride = layer.get("stride", 1)
         for j in reversed(range(K)):                              # dW^l += delta_t^T a^{l-1}_t
             a_in = rows_state[j][2][l]
             if layer["kind"] == "conv":
-                dW[l] += conv3x3_weight_grad(db[j], a_in)
+                dW[l] += conv3x3_weight_grad(db[j], a_in, stride)
             else:
                 dW[l] += db[j].reshape(B, -1).T @ a_in.reshape(B, -1)
+        r = layer.get("res")
+        if r is not None:                                          # S^T delta^l into dL/da^r
+            a_r = rows_state[0][2][r + 1]
+            prev = ga_res.get(r, [0.0] * K)
+            ga_res[r] = [prev[j] + shortcut_a_T(db[j], a_r.shape[1] // layer["h"], a_r.shape[3], a_r.shape[1:3])
+                         for j in range(K)]
         if l > 0:                                                  # grad wrt a^{l-1}: W^{l T} delta^l
             a_shape = rows_state[0][2][l].shape
             if layer["kind"] == "conv":
-                ga = [conv3x3_input_grad(db[j], Wb[l]) for j in range(K)]
+                ga = [conv3x3_input_grad(db[j], Wb[l], stride, a_shape[1:3]) for j in range(K)]
             else:
                 ga = [(db[j].reshape(B, -1) @ Wb[l]).reshape(a_shape) for j in range(K)]
     if trace is not None and rows is not None:
@@ -301,7 +332,8 @@ def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
     first = forward_first_pass(net, Wb, x, T, S, store_all=(mode == "full"), ledger=ledger,
                                record=cfg.record, trace=trace)
     s = first["s"]
-    loss, z, dz = readout(Wb[Ls], first["cnt"], y, T_norm, B_global)
+    use_gap = bool(net["layers"][-1].get("gap"))
+    loss, z, dz = readout(Wb[Ls], first["cnt"], y, T_norm, B_global, use_gap)
     if trace is not None:
         trace.append(("loss", T - 1))
     if cfg.dz is not None:
@@ -358,7 +390,7 @@ def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
             if trace is not None:
                 trace.append(("release", c))
     # readout weight gradient once, over the kept rows of every segment
-    dW[Ls] += dz.T @ cnt_kept.reshape(B, -1) / T_norm
+    dW[Ls] += dz.T @ readout_input(cnt_kept, use_gap) / T_norm
     return StepResult(loss=loss, z=z, dz=dz, s=s, counts=first["counts"], sam=s_pol, sst=sst, keep=keep, kept=kept, dW=dW,
                       cnt=first["cnt"], cnt_kept=cnt_kept, ledger_peak=ledger.peak,
                       first_U=first["first_U"], first_o=first["first_o"],

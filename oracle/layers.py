@@ -2,8 +2,11 @@
 
 The paper's networks (Table I) use conv and linear layers; it
 does not fix padding or pooling.  Readings: 3x3 convolution,
-stride 1, zero padding 1, no bias (Eq.1 has none); 2x2 average
-pooling of output spikes (reading 7).  Layout NHWC; weights [Cout][3][3][Cin].
+zero padding 1, no bias (Eq.1 has none), stride 1 or 2 (the
+ResNet20 SNN of Table I downsamples; reading 8); 2x2 average pooling of output
+spikes (reading 7); ResNet shortcuts are option A (spatial subsample +
+channel zero pad, no parameters; reading 8); global average pooling feeds the
+ResNet readout (reading 23).  Layout NHWC; weights [Cout][3][3][Cin].
 All in float64.
 """
 from __future__ import annotations
@@ -11,45 +14,84 @@ from __future__ import annotations
 import numpy as np
 
 
-def conv3x3(a: np.ndarray, W: np.ndarray) -> np.ndarray:
-    """out[n,y,x,co] = sum_{dy,dx,ci} W[co,dy,dx,ci] * a[n, y+dy-1, x+dx-1, ci] (zero outside).
+def conv3x3(a: np.ndarray, W: np.ndarray, stride: int = 1) -> np.ndarray:
+    """out[n,y,x,co] = sum_{dy,dx,ci} W[co,dy,dx,ci] * a[n, s*y+dy-1, s*x+dx-1, ci] (zero outside),
+    output size ceil(H/s) x ceil(W/s).
 
     Written as one matmul per tap over the zero-padded input."""
     N, H, Wd, Ci = a.shape
     Co = W.shape[0]
-    ap = np.pad(np.asarray(a, np.float64), ((0, 0), (1, 1), (1, 1), (0, 0)))
-    out = np.zeros((N, H, Wd, Co), dtype=np.float64)
+    Ho, Wo = -(-H // stride), -(-Wd // stride)
+    ap = np.pad(np.asarray(a, np.float64), ((0, 0), (1, 1 + stride), (1, 1 + stride), (0, 0)))
+    out = np.zeros((N, Ho, Wo, Co), dtype=np.float64)
     for dy in range(3):
         for dx in range(3):
-            out += ap[:, dy:dy + H, dx:dx + Wd, :] @ np.asarray(W[:, dy, dx, :], np.float64).T
+            win = ap[:, dy:dy + stride * Ho:stride, dx:dx + stride * Wo:stride, :]
+            out += win @ np.asarray(W[:, dy, dx, :], np.float64).T
     return out
 
 
-def conv3x3_input_grad(d: np.ndarray, W: np.ndarray) -> np.ndarray:
-    """Adjoint of conv3x3 in its input:
-    ga[n,y,x,ci] = sum_{dy,dx,co} W[co,dy,dx,ci] * d[n, y-dy+1, x-dx+1, co]."""
-    N, H, Wd, Co = d.shape
+def conv3x3_input_grad(d: np.ndarray, W: np.ndarray, stride: int = 1, in_hw: tuple | None = None) -> np.ndarray:
+    """Adjoint of conv3x3 in its input (in_hw = the input's H, W; default the output's times s):
+    ga[n,yi,xi,ci] = sum over (y, x, dy, dx) with s*y+dy-1 = yi, s*x+dx-1 = xi of W[co,dy,dx,ci] d[n,y,x,co].
+
+    Written as a scatter of one matmul per tap into the zero-padded input."""
+    N, Ho, Wo, Co = d.shape
     Ci = W.shape[3]
-    dp = np.pad(np.asarray(d, np.float64), ((0, 0), (1, 1), (1, 1), (0, 0)))
-    out = np.zeros((N, H, Wd, Ci), dtype=np.float64)
+    H, Wd = in_hw if in_hw is not None else (Ho * stride, Wo * stride)
+    gp = np.zeros((N, H + 2 + stride, Wd + 2 + stride, Ci), dtype=np.float64)
+    d64 = np.asarray(d, np.float64)
     for dy in range(3):
         for dx in range(3):
-            out += dp[:, 2 - dy:2 - dy + H, 2 - dx:2 - dx + Wd, :] @ np.asarray(W[:, dy, dx, :], np.float64)
-    return out
+            gp[:, dy:dy + stride * Ho:stride, dx:dx + stride * Wo:stride, :] += d64 @ np.asarray(W[:, dy, dx, :], np.float64)
+    return gp[:, 1:1 + H, 1:1 + Wd, :]
 
 
-def conv3x3_weight_grad(d: np.ndarray, a: np.ndarray) -> np.ndarray:
+def conv3x3_weight_grad(d: np.ndarray, a: np.ndarray, stride: int = 1) -> np.ndarray:
     """Adjoint of conv3x3 in its weights:
-    gW[co,dy,dx,ci] = sum_{n,y,x} d[n,y,x,co] * a[n, y+dy-1, x+dx-1, ci]."""
-    N, H, Wd, Co = d.shape
+    gW[co,dy,dx,ci] = sum_{n,y,x} d[n,y,x,co] * a[n, s*y+dy-1, s*x+dx-1, ci]."""
+    N, Ho, Wo, Co = d.shape
     Ci = a.shape[3]
-    ap = np.pad(np.asarray(a, np.float64), ((0, 0), (1, 1), (1, 1), (0, 0)))
+    ap = np.pad(np.asarray(a, np.float64), ((0, 0), (1, 1 + stride), (1, 1 + stride), (0, 0)))
     d2 = np.asarray(d, np.float64).reshape(-1, Co)
     out = np.zeros((Co, 3, 3, Ci), dtype=np.float64)
     for dy in range(3):
         for dx in range(3):
-            out[:, dy, dx, :] = d2.T @ ap[:, dy:dy + H, dx:dx + Wd, :].reshape(-1, Ci)
+            win = ap[:, dy:dy + stride * Ho:stride, dx:dx + stride * Wo:stride, :]
+            out[:, dy, dx, :] = d2.T @ win.reshape(-1, Ci)
     return out
+
+
+def shortcut_a(a: np.ndarray, stride: int, cout: int) -> np.ndarray:
+    """Option-A ResNet shortcut (reading 8): out[n,y,x,c] = a[n, s*y, s*x, c - lo] for
+    lo <= c < lo + Cin with lo = (cout - Cin) // 2, zero elsewhere (no parameters)."""
+    N, H, Wd, Ci = a.shape
+    lo = (cout - Ci) // 2
+    sub = np.asarray(a, np.float64)[:, ::stride, ::stride, :]
+    out = np.zeros(sub.shape[:3] + (cout,), dtype=np.float64)
+    out[..., lo:lo + Ci] = sub
+    return out
+
+
+def shortcut_a_T(g: np.ndarray, stride: int, cin: int, in_hw: tuple) -> np.ndarray:
+    """Adjoint of shortcut_a: the channel window lo..lo+cin of g scattered back to the subsampled positions."""
+    N, Ho, Wo, Co = g.shape
+    lo = (Co - cin) // 2
+    out = np.zeros((N,) + tuple(in_hw) + (cin,), dtype=np.float64)
+    out[:, ::stride, ::stride, :] = np.asarray(g, np.float64)[..., lo:lo + cin]
+    return out
+
+
+def gap(a: np.ndarray) -> np.ndarray:
+    """Global average pooling over (h, w) of an NHWC array (reading 23)."""
+    return np.asarray(a, np.float64).mean(axis=(1, 2))
+
+
+def gap_T(g: np.ndarray, hw: tuple) -> np.ndarray:
+    """Adjoint of gap: g / (h w) broadcast over every position."""
+    H, Wd = hw
+    g = np.asarray(g, np.float64) / (H * Wd)
+    return np.broadcast_to(g[:, None, None, :], (g.shape[0], H, Wd, g.shape[1])).copy()
 
 
 def pool2(o: np.ndarray) -> np.ndarray:

@@ -19,9 +19,16 @@ LAM = 0.99
 THETA = 1.0
 
 
-def _conv(cin, cout, hw, pool=0, lam=LAM, theta=THETA):
-    return {"kind": "conv", "cin": cin, "cout": cout, "h": hw, "w": hw,
-            "pool": pool, "lam": lam, "theta": theta}
+def _conv(cin, cout, hw, pool=0, lam=LAM, theta=THETA, stride=1, res=None):
+    """3x3 conv LIF layer; hw = its OUTPUT (neuron) size, the input is hw*stride.
+    res = index of the spiking layer whose output spikes enter through the option-A shortcut."""
+    d = {"kind": "conv", "cin": cin, "cout": cout, "h": hw, "w": hw,
+         "pool": pool, "lam": lam, "theta": theta}
+    if stride != 1:
+        d["stride"] = stride
+    if res is not None:
+        d["res"] = res
+    return d
 
 
 def _fc(cin, cout, lam=LAM, theta=THETA):
@@ -29,9 +36,32 @@ def _fc(cin, cout, lam=LAM, theta=THETA):
             "pool": 0, "lam": lam, "theta": theta}
 
 
-def _readout(cin, classes):
-    return {"kind": "readout", "cin": cin, "cout": classes, "h": 1, "w": 1,
-            "pool": 0, "lam": 1.0, "theta": 0.0}
+def _readout(cin, classes, gap=False):
+    d = {"kind": "readout", "cin": cin, "cout": classes, "h": 1, "w": 1,
+         "pool": 0, "lam": 1.0, "theta": 0.0}
+    if gap:
+        d["gap"] = True
+    return d
+
+
+def _resnet(in_hw, in_c, widths, blocks, classes):
+    """ResNet-style SNN (SURVEY.md §8(a) cfg 4; Table I "ResNet20"): a stride-2 stem,
+    len(widths) stages of `blocks` basic blocks (two 3x3 conv LIF layers; the second one receives the
+    block input through the option-A shortcut, reading 8); stages after the first start with a stride-2
+    conv; global average pool into the readout (reading 23)."""
+    hw = in_hw // 2
+    layers = [_conv(in_c, widths[0], hw, stride=2)]
+    cin = widths[0]
+    for si, wd in enumerate(widths):
+        for bi in range(blocks):
+            stride = 2 if (si > 0 and bi == 0) else 1
+            hw //= stride
+            src = len(layers) - 1
+            layers.append(_conv(cin, wd, hw, stride=stride))
+            layers.append(_conv(wd, wd, hw, res=src))
+            cin = wd
+    layers.append(_readout(cin, classes, gap=True))
+    return layers
 
 
 def _vgg11(classes=100):
@@ -69,6 +99,11 @@ NETS = {
         _readout(192, 10),
     ]},
     "tiny_fc": {"input": ("flat", 40), "layers": [_fc(40, 24), _fc(24, 16), _readout(16, 5)]},
+    # cfg 4: ResNet-20-style SNN on DVS-Gesture-shaped event frames (2 x 128 x 128): stem 2-16 s2 -> 64^2,
+    # 3 stages x 3 basic blocks (16 @64^2, 32 @32^2, 64 @16^2), GAP -> 11 classes.  19 spiking layers + readout.
+    "resnet20_dvs": {"input": ("dvs", 128, 128, 2), "layers": _resnet(128, 2, (16, 32, 64), 3, 11)},
+    # small ResNet for tests: both shortcut kinds (identity, stride-2 + channel pad), narrow channels
+    "tiny_resnet": {"input": ("dvs", 16, 16, 2), "layers": _resnet(16, 2, (16, 32), 1, 5)},
 }
 
 
@@ -90,6 +125,7 @@ WORKLOADS = {
     "cfg1_fc784": {"net": "fc784", "T": 20, "B": 4, "C": 2, "p": 50.0, "classes": 10},
     "cfg2_vgg5": {"net": "vgg5", "T": 100, "B": 64, "C": 10, "p": 40.0, "classes": 10},
     "cfg3_vgg11": {"net": "vgg11", "T": 200, "B": 128, "C": 5, "p": 50.0, "classes": 100},
+    "cfg4_resnet_dvs": {"net": "resnet20_dvs", "T": 300, "B": 32, "C": 5, "p": 50.0, "classes": 11},
 }
 
 

@@ -43,7 +43,8 @@ def make_weights(net, seed: int = 0, gain: float = 0.6, bias: float = 0.0):
     """One float32 master weight array per layer (spiking layers and readout)."""
     rng = np.random.default_rng(seed)
     out = []
-    rate = 0.3  # Poisson input layer rate (envelope mean ~0.75 * E[x]=0.5 -> ~0.37)
+    # input firing rate: Poisson frames ~0.37 (envelope mean ~0.75 * E[x]=0.5); DVS events ~0.02
+    rate = 0.02 if net.get("input", ("",))[0] == "dvs" else 0.3
     for layer in net["layers"]:
         if layer["kind"] == "readout":
             out.append(grid_weights(layer, rng, rate_in=rate, gain=2.0, bias=0.0))
@@ -115,6 +116,10 @@ def make_inputs(net, T: int, B: int, classes: int | None = None, seed: int = 1,
     """(x u8 [T][B][*input], y int32 [B]) for a network."""
     if classes is None:
         classes = net["layers"][-1]["cout"]
-    x = poisson_frames(T, B, input_shape(net), seed=seed, rate_scale=rate_scale)
+    if net["input"][0] == "dvs":
+        _, H, W, _c = net["input"]
+        x = dvs_frames(T, B, H, W, seed=seed)
+    else:
+        x = poisson_frames(T, B, input_shape(net), seed=seed, rate_scale=rate_scale)
     y = labels(B, classes, seed=seed + 1)
     return x, y

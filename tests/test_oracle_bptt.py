@@ -32,10 +32,26 @@ class Spike(torch.autograd.Function):
         return g * sg, None, None
 
 
-def t_current(layer, W, a):
+def t_current(layer, W, a, a_res=None):
+    """Synaptic current; ResNet layers (reading 8): stride, plus the option-A shortcut of the residual
+    source written the classic CIFAR-ResNet way (subsample, zero-pad channels on both sides)."""
     if layer["kind"] == "conv":
-        return F.conv2d(a.permute(0, 3, 1, 2), W.permute(0, 3, 1, 2), padding=1).permute(0, 2, 3, 1)
+        I = F.conv2d(a.permute(0, 3, 1, 2), W.permute(0, 3, 1, 2), padding=1,
+                     stride=layer.get("stride", 1)).permute(0, 2, 3, 1)
+        if a_res is not None:
+            r = a_res.permute(0, 3, 1, 2)
+            if r.shape[2] != I.shape[1]:
+                r = r[:, :, ::2, ::2]
+            pad = (I.shape[3] - r.shape[1]) // 2
+            I = I + F.pad(r, (0, 0, 0, 0, pad, pad)).permute(0, 2, 3, 1)
+        return I
     return a.reshape(a.shape[0], -1) @ W.T
+
+
+def t_readin(net, cnt):
+    if net["layers"][-1].get("gap"):
+        return F.adaptive_avg_pool2d(cnt.permute(0, 3, 1, 2), 1).flatten(1)
+    return cnt.reshape(cnt.shape[0], -1)
 
 
 def t_out(layer, o):
@@ -53,16 +69,18 @@ def torch_full_bptt(net, W, x, y, gamma=0.3):
     cnt = 0
     for t in range(T):
         a = torch.tensor(x[t].astype(np.float64))
+        outs = []
         for l, L in enumerate(spk):
-            I = t_current(L, Wt[l], a)
+            I = t_current(L, Wt[l], a, outs[L["res"]] if "res" in L else None)
             if U[l] is None:
                 U[l] = I                                   # U_{-1} = o_{-1} = 0
             else:
                 U[l] = L["lam"] * U[l] + I - L["theta"] * o[l].detach()
             o[l] = Spike.apply(U[l], L["theta"], gamma)
             a = t_out(L, o[l])
+            outs.append(a)
         cnt = cnt + a
-    z = cnt.reshape(B, -1) @ Wt[-1].T / T
+    z = t_readin(net, cnt) @ Wt[-1].T / T
     loss = F.cross_entropy(z, torch.tensor(y, dtype=torch.long), reduction="sum") / B
     loss.backward()
     return float(loss.detach()), [w.grad.numpy() for w in Wt]
@@ -84,11 +102,13 @@ def torch_skip_bptt(net, W, x, kept, dz, T, gamma=0.3):
         starts = {int(k[0]) for k in kept}
         for t in range(T):
             a = torch.tensor(x[t].astype(np.float64))
+            outs = []
             for l, L in enumerate(spk):
-                I = t_current(L, Wt[l], a)
+                I = t_current(L, Wt[l], a, outs[L["res"]] if "res" in L else None)
                 U[l] = I if U[l] is None else L["lam"] * U[l] + I - L["theta"] * o[l]
                 o[l] = (U[l] > L["theta"]).double()
                 a = t_out(L, o[l])
+                outs.append(a)
             if t in starts:
                 ck[t] = [u.clone() for u in U]
     cnt = 0
@@ -98,8 +118,9 @@ def torch_skip_bptt(net, W, x, kept, dz, T, gamma=0.3):
         o = [None] * len(spk)
         for j, t in enumerate(rows):
             a = torch.tensor(x[t].astype(np.float64))
+            outs = []
             for l, L in enumerate(spk):
-                I = t_current(L, Wt[l], a)
+                I = t_current(L, Wt[l], a, outs[L["res"]] if "res" in L else None)
                 if j == 0:
                     u = ck[int(t)][l] + (I - I.detach())
                     if prev_last is not None:
@@ -109,9 +130,10 @@ def torch_skip_bptt(net, W, x, kept, dz, T, gamma=0.3):
                     U[l] = L["lam"] * U[l] + I - L["theta"] * o[l].detach()
                 o[l] = Spike.apply(U[l], L["theta"], gamma)
                 a = t_out(L, o[l])
+                outs.append(a)
             cnt = cnt + a
         prev_last = list(U)
-    z = cnt.reshape(B, -1) @ Wt[-1].T / T
+    z = t_readin(net, cnt) @ Wt[-1].T / T
     surrogate_loss = (torch.tensor(dz, dtype=torch.float64) * z).sum()
     surrogate_loss.backward()
     return [w.grad.numpy() for w in Wt]
@@ -128,7 +150,8 @@ def rel_err(a, b):
     return np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-300)
 
 
-@pytest.mark.parametrize("name,lam", [("tiny_fc", 1.0), ("tiny_fc", 0.5), ("tiny_conv", 0.75), ("tiny_conv", 1.0)])
+@pytest.mark.parametrize("name,lam", [("tiny_fc", 1.0), ("tiny_fc", 0.5), ("tiny_conv", 0.75), ("tiny_conv", 1.0),
+                                      ("tiny_resnet", 0.75), ("tiny_resnet", 1.0)])
 def test_full_bptt_equals_autograd(name, lam):
     T = 6
     net, W, x, y = dyadic_setup(name, T, 3, lam)
@@ -140,7 +163,7 @@ def test_full_bptt_equals_autograd(name, lam):
         assert rel_err(a, b) < 1e-12 or np.abs(a - b).max() < 1e-15, (l, rel_err(a, b))
 
 
-@pytest.mark.parametrize("name,lam,C", [("tiny_fc", 0.5, 2), ("tiny_conv", 1.0, 3)])
+@pytest.mark.parametrize("name,lam,C", [("tiny_fc", 0.5, 2), ("tiny_conv", 1.0, 3), ("tiny_resnet", 0.75, 2)])
 def test_ckpt_equals_full_bitwise(name, lam, C):
     """Checkpointing reaches exactly the BPTT gradient."""
     T = 12
@@ -163,7 +186,8 @@ def test_skip_p0_equals_ckpt_bitwise():
 
 
 @pytest.mark.parametrize("name,lam,C,seed", [("tiny_fc", 0.5, 1, 0), ("tiny_fc", 1.0, 3, 1),
-                                             ("tiny_conv", 0.5, 2, 2), ("tiny_conv", 1.0, 1, 3)])
+                                             ("tiny_conv", 0.5, 2, 2), ("tiny_conv", 1.0, 1, 3),
+                                             ("tiny_resnet", 0.5, 2, 4), ("tiny_resnet", 1.0, 3, 5)])
 def test_skip_equals_autograd_on_compacted_chain(name, lam, C, seed):
     T = 12
     net, W, x, y = dyadic_setup(name, T, 2, lam, seed=seed)

@@ -93,3 +93,70 @@ def test_bf16_grid_values_exact(rng):
     j = rng.integers(-255, 256, 1000)
     w = j * 2.0 ** -9
     np.testing.assert_array_equal(bf16_round(w), w)
+
+
+# ---- ResNet pieces (reading 8, reading 23): strided conv, option-A shortcut, global average pool
+
+def brute_conv_strided(a, W, s):
+    N, H, Wd, Ci = a.shape
+    Co = W.shape[0]
+    Ho, Wo = (H + s - 1) // s, (Wd + s - 1) // s
+    out = np.zeros((N, Ho, Wo, Co))
+    for n in range(N):
+        for y in range(Ho):
+            for x in range(Wo):
+                for dy in range(3):
+                    for dx in range(3):
+                        yy, xx = s * y + dy - 1, s * x + dx - 1
+                        if 0 <= yy < H and 0 <= xx < Wd:
+                            out[n, y, x] += W[:, dy, dx, :] @ a[n, yy, xx, :]
+    return out
+
+
+@pytest.mark.parametrize("shape", [(2, 8, 8, 3), (1, 6, 10, 2), (2, 5, 7, 4)])
+def test_conv_stride2_brute_and_torch(rng, shape):
+    a = rng.standard_normal(shape)
+    W = rng.standard_normal((5, 3, 3, shape[3]))
+    out = conv3x3(a, W, 2)
+    np.testing.assert_allclose(out, brute_conv_strided(a, W, 2), rtol=1e-12, atol=1e-12)
+    ref = torch.nn.functional.conv2d(torch.tensor(a).permute(0, 3, 1, 2), torch.tensor(W).permute(0, 3, 1, 2),
+                                     padding=1, stride=2).permute(0, 2, 3, 1)
+    np.testing.assert_allclose(out, ref.numpy(), rtol=1e-12, atol=1e-12)
+
+
+@pytest.mark.parametrize("stride", [1, 2])
+def test_conv_strided_adjoints(rng, stride):
+    a = rng.standard_normal((2, 8, 6, 3))
+    W = rng.standard_normal((4, 3, 3, 3))
+    y = conv3x3(a, W, stride)
+    d = rng.standard_normal(y.shape)
+    lhs = np.sum(y * d)
+    assert np.sum(a * conv3x3_input_grad(d, W, stride, a.shape[1:3])) == pytest.approx(lhs, rel=1e-12)
+    assert np.sum(W * conv3x3_weight_grad(d, a, stride)) == pytest.approx(lhs, rel=1e-12)
+
+
+def test_shortcut_option_a(rng):
+    from oracle.layers import shortcut_a, shortcut_a_T
+    a = (rng.random((2, 8, 8, 4)) < 0.5).astype(np.float64)
+    s = shortcut_a(a, 2, 8)                       # 4 -> 8 channels, 2 zero channels each side
+    assert s.shape == (2, 4, 4, 8)
+    np.testing.assert_array_equal(s[..., :2], 0)
+    np.testing.assert_array_equal(s[..., 6:], 0)
+    for y in range(4):
+        for x in range(4):
+            np.testing.assert_array_equal(s[:, y, x, 2:6], a[:, 2 * y, 2 * x, :])
+    # the classic CIFAR ResNet option-A: F.pad(x[:, :, ::2, ::2], (0, 0, 0, 0, c/4, c/4)) in NCHW
+    ref = torch.nn.functional.pad(torch.tensor(a).permute(0, 3, 1, 2)[:, :, ::2, ::2], (0, 0, 0, 0, 2, 2))
+    np.testing.assert_array_equal(s, ref.permute(0, 2, 3, 1).numpy())
+    np.testing.assert_array_equal(shortcut_a(a, 1, 4), a)                     # identity shortcut
+    g = rng.standard_normal(s.shape)
+    assert np.sum(s * g) == pytest.approx(np.sum(a * shortcut_a_T(g, 2, 4, (8, 8))), rel=1e-12)
+
+
+def test_gap_and_adjoint(rng):
+    from oracle.layers import gap, gap_T
+    o = (rng.random((3, 4, 4, 5)) < 0.3).astype(np.uint8)
+    p = gap(o)
+    np.testing.assert_array_equal(p * 16, o.sum(axis=(1, 2)))
+    g = rng.standard_normal(p.shape)
+    assert np.sum(p * g) == pytest.approx(np.sum(o * gap_T(g, (4, 4))), rel=1e-12)
