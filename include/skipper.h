@@ -70,16 +70,25 @@ typedef enum { SKIPPER_SURR_TRIANGLE = 0, SKIPPER_SURR_FAST_SIGMOID = 1 } skippe
  *          layer" (reading 22). */
 typedef enum { SKIPPER_SAM_SPIKES = 0, SKIPPER_SAM_WEIGHTED = 1 } skipper_sam;
 
-/* One layer.  conv3x3: stride 1, zero pad 1, input and output h x w, optional 2x2
- * average pooling of the output spikes (pool = 2).  fc: h = w = 1.  The last layer
- * must be the (non-spiking) readout; lambda/theta are ignored for it. */
+/* One layer.  conv3x3: zero pad 1, stride 1 or 2; h x w = the OUTPUT (neuron) size, the
+ * input is (stride*h) x (stride*w); optional 2x2 average pooling of the output spikes
+ * (pool = 2).  fc: h = w = 1.  The last layer must be the (non-spiking) readout;
+ * lambda/theta are ignored for it, and pool = 1 on the readout means it integrates the
+ * global average pool of the last conv layer's spikes (reading 23; then cin = that
+ * layer's cout).
+ * residual_from (ResNet SNN, Table I "ResNet20", reading 8): -1, or the index
+ * r = (this layer) - 2 of a spiking conv layer whose output spikes are added into this
+ * layer's current through the option-A shortcut: subsample by h_r / h (1 or 2) and
+ * zero-pad the channels (cout - cout_r) / 2 on each side.  Unpooled layers only. */
 typedef struct {
     int kind;        /* skipper_layer_kind */
     int cin, cout;
     int h, w;
-    int pool;        /* 0 or 2 */
+    int pool;        /* 0 or 2 (conv); 0 or 1 = GAP (readout) */
     float lambda;    /* leak, Eq.1 (lambda < 1; 1 = integrate-and-fire) */
     float theta;     /* firing threshold, Eq.1 */
+    int stride;      /* conv: 1 or 2 (0 is read as 1) */
+    int residual_from;  /* -1 or layer index - 2 (see above) */
 } skipper_layer;
 
 typedef struct {

@@ -32,6 +32,10 @@ struct Layer {
     skipper_layer d{};
     bool fc = false, conv = false, pool = false, readout = false;
     int H = 1, W = 1, Cin = 0, Cout = 0, PH = 1, PW = 1;
+    int stride = 1, Hin = 1, Win = 1;  // conv: output (neuron) H x W, input (stride H) x (stride W)
+    int res = -1, res_to = -1;          // ResNet: residual source layer (this = receiver) / receiver (this = source)
+    bool icol = false;                  // conv via explicit im2col + GEMM (narrow / strided layers)
+    bool gap = false;                   // readout integrates the global average pool (reading 23)
     long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
     size_t wcount = 0;
     float *w = nullptr, *dw = nullptr, *m = nullptr, *v = nullptr;
@@ -90,8 +94,8 @@ struct skipper_ctx {
     // side stream: the weight-gradient GEMM of layer l runs there, overlapping the dgrad of layer l
     // and the reverse scan of layer l-1 on the main stream (delta is double-buffered)
     cudaStream_t st2 = nullptr;
-    cudaEvent_t ev_ready[2] = {nullptr, nullptr}, ev_done[2] = {nullptr, nullptr};
-    bool w_pending[2] = {false, false};
+    cudaEvent_t ev_ready[3] = {nullptr, nullptr, nullptr}, ev_done[3] = {nullptr, nullptr, nullptr};
+    bool w_pending[3] = {false, false, false};
     int T = 0, C = 1, S = 0, B = 0, Bg = 0;
     int num_sms = 148;
     int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
@@ -127,8 +131,12 @@ struct skipper_ctx {
     size_t arena_bytes = 0;
     float *I_buf = nullptr;     // currents (fwd) and gradients wrt spikes (dgrad)
     uint16_t *d_buf = nullptr;  // delta (bf16)
-    uint16_t *d_buf2[2] = {nullptr, nullptr};
-    uint16_t *P2[2] = {nullptr, nullptr};
+    uint16_t *d_buf2[3] = {nullptr, nullptr, nullptr};  // delta ring (3 deep when residuals exist)
+    uint16_t *P2[3] = {nullptr, nullptr, nullptr};      // FIRST-pass output ring (3 deep when residuals exist)
+    int nD = 2, nP = 2;
+    uint16_t *cols[3] = {nullptr, nullptr, nullptr};    // im2col operands of icol layers (per delta slot)
+    float *dcols = nullptr;                             // icol dgrad output columns (fp32)
+    float *cnt_gap = nullptr, *g_gap = nullptr;         // GAP readout input / gradient [B][C]
     uint16_t *xg = nullptr;     // staged layer-0 operand rows of the current pass
     // schedule state
     int phase = PH_IDLE;
@@ -156,11 +164,11 @@ struct skipper_ctx {
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
-    K_L0_FWD, K_L0_BWD, K_CONV_LIF, K_NCLASS
+    K_L0_FWD, K_L0_BWD, K_CONV_LIF, K_IM2COL, K_NCLASS
 };
 static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
                                                "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad",
-                                               "layer0_fused_fwd", "layer0_fused_bwd", "gemm_lif_fwd"};
+                                               "layer0_fused_fwd", "layer0_fused_bwd", "gemm_lif_fwd", "im2col"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -333,6 +341,10 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
             l.W = d.w;
             l.Cin = d.cin;
             l.Cout = d.cout;
+            l.stride = d.stride == 0 ? 1 : d.stride;
+            if (l.stride != 1 && l.stride != 2) return fail(c, SKIPPER_EINVAL, "layer %d: stride must be 1 or 2", i);
+            l.Hin = d.h * l.stride;
+            l.Win = d.w * l.stride;
             l.pool = d.pool == 2;
             if (d.pool != 0 && d.pool != 2) return fail(c, SKIPPER_EINVAL, "layer %d: pool must be 0 or 2", i);
             if (l.pool && (d.h % 2 || d.w % 2)) return fail(c, SKIPPER_EINVAL, "layer %d: pooled size must be even", i);
@@ -340,11 +352,15 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
             l.PW = l.pool ? d.w / 2 : d.w;
             l.N = (long long)d.h * d.w * d.cout;
             l.Nout = (long long)l.PH * l.PW * d.cout;
-            l.Nin = (long long)d.h * d.w * d.cin;
+            l.Nin = (long long)l.Hin * l.Win * d.cin;
             l.wcount = (size_t)d.cout * 9 * d.cin;
         } else if (d.kind == SKIPPER_LAYER_FC || d.kind == SKIPPER_LAYER_READOUT) {
             l.fc = d.kind == SKIPPER_LAYER_FC;
             l.readout = d.kind == SKIPPER_LAYER_READOUT;
+            if (l.readout) {
+                if (d.pool != 0 && d.pool != 1) return fail(c, SKIPPER_EINVAL, "readout: pool must be 0 or 1 (GAP)");
+                l.gap = d.pool == 1;
+            }
             l.Cin = d.cin;
             l.Cout = d.cout;
             l.N = l.Nout = d.cout;
@@ -362,8 +378,8 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
     // chaining
     const Layer &f = c->L[0];
     if (f.conv) {
-        c->in_h = f.H;
-        c->in_w = f.W;
+        c->in_h = f.Hin;
+        c->in_w = f.Win;
         c->in_c = f.Cin;
     } else {
         c->in_h = c->in_w = 1;
@@ -384,12 +400,33 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
         const Layer &p = c->L[i - 1];
         const Layer &l = c->L[i];
         if (l.conv) {
-            if (!p.conv || l.H != p.PH || l.W != p.PW || l.Cin != p.Cout)
+            if (!p.conv || l.Hin != p.PH || l.Win != p.PW || l.Cin != p.Cout)
                 return fail(c, SKIPPER_EINVAL, "layer %d: conv input must be the %dx%dx%d output of layer %d", i, p.PH, p.PW,
                             p.Cout, i - 1);
+        } else if (l.gap) {
+            if (!p.conv || l.Cin != p.Cout)
+                return fail(c, SKIPPER_EINVAL, "GAP readout: cin %d must be the channels of conv layer %d", l.Cin, i - 1);
         } else if (l.Cin != p.Nout) {
             return fail(c, SKIPPER_EINVAL, "layer %d: cin %d != %lld outputs of layer %d", i, l.Cin, p.Nout, i - 1);
         }
+    }
+    // residual shortcuts (reading 8): source r = i - 2, option A
+    for (int i = 0; i < c->Ls; ++i) {
+        Layer &l = c->L[i];
+        const int r = layers[i].residual_from;
+        if (r == -1) continue;
+        if (!l.conv || r != i - 2 || r < 0)
+            return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: residual_from must be -1 or %d (a conv layer)", i, i - 2);
+        Layer &src = c->L[r];
+        if (!src.conv || src.pool || l.pool)
+            return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: residual between unpooled conv layers only", i);
+        const int rs = src.H / l.H;
+        if ((rs != 1 && rs != 2) || src.H != rs * l.H || src.W != rs * l.W || src.Cout > l.Cout ||
+            (l.Cout - src.Cout) % 8)
+            return fail(c, SKIPPER_EINVAL, "layer %d: option-A shortcut from %dx%dx%d to %dx%dx%d", i, src.H, src.W,
+                        src.Cout, l.H, l.W, l.Cout);
+        l.res = r;
+        src.res_to = i;
     }
     // kernel support per layer
     for (int i = 0; i < c->Ls; ++i) {
@@ -399,16 +436,20 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
             continue;
         }
         if (l.conv) {
-            if (l.Cin % 64) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: tensor-core conv needs cin %% 64 == 0", i);
-            if (l.Cout % 64 && i > 0) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: conv dgrad needs cout %% 64 == 0", i);
             auto boxok = [](int h, int w, int rows) {
                 if (w > rows || rows % w) return false;
                 int by = rows / w;
                 if (by <= h) return h % by == 0;
                 return by % h == 0;
             };
-            if (!boxok(l.H, l.W, 128) || !boxok(l.H, l.W, 64))
-                return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: %dx%d image does not tile 64/128-row TMA boxes", i, l.H, l.W);
+            const bool implicit = l.Cin % 64 == 0 && (l.Cout % 64 == 0 || i == 0) && l.stride == 1 &&
+                                  boxok(l.H, l.W, 128) && boxok(l.H, l.W, 64);
+            if (!implicit) {  // explicit im2col + GEMM (narrow channels, stride 2, small images)
+                if (i == 0) return fail(c, SKIPPER_EUNSUPPORTED, "layer 0: wide-input conv needs cin %% 64 == 0, stride 1");
+                if (l.Cin % 8 || l.Cout % 8)
+                    return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: im2col conv needs cin, cout %% 8 == 0", i);
+                l.icol = true;
+            }
         } else {
             if (l.Cin % 8 || l.Cout % 8) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: fc needs cin, cout %% 8 == 0", i);
         }
@@ -430,6 +471,12 @@ static long long max_nout(const skipper_ctx *c) {
 static long long max_n(const skipper_ctx *c) {
     long long m = 0;
     for (int i = 0; i < c->Ls; ++i) m = std::max(m, c->L[i].N);
+    return m;
+}
+static long long max_icol(const skipper_ctx *c) {  // im2col columns per sample-row (icol layers)
+    long long m = 0;
+    for (int i = 0; i < c->Ls; ++i)
+        if (c->L[i].icol) m = std::max(m, (long long)c->L[i].H * c->L[i].W * 9 * c->L[i].Cin);
     return m;
 }
 static long long max_gemm_io(const skipper_ctx *c) {  // fp32 I (fwd) and g (dgrad) per sample-row
@@ -503,14 +550,16 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     c->num_sms = sk::device_num_sms();
     if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess)
         return bail(fail(c, SKIPPER_ECUDA, "side stream creation failed"));
-    for (int k = 0; k < 2; ++k)
+    for (int i = 0; i < c->Ls; ++i)
+        if (c->L[i].res >= 0) c->nD = c->nP = 3;
+    for (int k = 0; k < 3; ++k)
         if (cudaEventCreateWithFlags(&c->ev_ready[k], cudaEventDisableTiming) != cudaSuccess ||
             cudaEventCreateWithFlags(&c->ev_done[k], cudaEventDisableTiming) != cudaSuccess)
             return bail(fail(c, SKIPPER_ECUDA, "event creation failed"));
     {
         const Layer &f = c->L[0];
         const char *e = getenv("SKIPPER_NO_L0_FUSION");
-        c->l0_fused = c->in_kind == 1 && c->K0 == 32 && c->Ls >= 2 && !(e && atoi(e)) &&
+        c->l0_fused = c->in_kind == 1 && c->K0 == 32 && c->Ls >= 2 && !(e && atoi(e)) && f.stride == 1 &&
                       sk::layer0_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
         // opt-in: measured slower than reverse scan + im2col wgrad GEMM on VGG-5
         const char *e2 = getenv("SKIPPER_L0_BWD_FUSION");
@@ -521,7 +570,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         const char *e3 = getenv("SKIPPER_NO_CONV_FUSION");
         for (int i = 1; i < c->Ls - 1; ++i) {
             Layer &l = c->L[i];
-            l.cfused = l.conv && !(e3 && atoi(e3)) &&
+            l.cfused = l.conv && !l.icol && l.res < 0 && !(e3 && atoi(e3)) &&
                        sk::conv_lif_supported(c->B, l.H, l.W, l.Cin, l.Cout, l.pool ? 1 : 0);
         }
     }
@@ -585,6 +634,10 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     const Layer &last = c->L[c->Ls - 1];
     const Layer &ro = c->L.back();
     AL(c->cnt, (size_t)c->B * last.Nout);
+    if (ro.gap) {
+        AL(c->cnt_gap, (size_t)c->B * ro.Cin);
+        AL(c->g_gap, (size_t)c->B * ro.Cin);
+    }
     AL(c->cnt_kept, (size_t)c->B * last.Nout);
     AL(c->g_last, (size_t)c->B * last.Nout);
     AL(c->z, (size_t)c->B * ro.Cout);
@@ -644,6 +697,8 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         dev_free(c, c->s_part, (size_t)(c->Ls + 1) * c->T * 32 * 4);
         dev_free(c, c->s_dev, (size_t)(c->Ls + 1) * c->T * 8);
         dev_free(c, c->cnt, (size_t)c->B * last.Nout * 4);
+        dev_free(c, c->cnt_gap, (size_t)c->B * ro.Cin * 4);
+        dev_free(c, c->g_gap, (size_t)c->B * ro.Cin * 4);
         dev_free(c, c->cnt_kept, (size_t)c->B * last.Nout * 4);
         dev_free(c, c->g_last, (size_t)c->B * last.Nout * 4);
         dev_free(c, c->z, (size_t)c->B * ro.Cout * 4);
@@ -659,7 +714,7 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         cudaStreamSynchronize(c->st2);
         cudaStreamDestroy(c->st2);
     }
-    for (int k = 0; k < 2; ++k) {
+    for (int k = 0; k < 3; ++k) {
         if (c->ev_ready[k]) cudaEventDestroy(c->ev_ready[k]);
         if (c->ev_done[k]) cudaEventDestroy(c->ev_done[k]);
     }
@@ -750,8 +805,8 @@ static skipper_status arena_free(skipper_ctx *c) {
     }
     c->I_buf = nullptr;
     c->d_buf = nullptr;
-    c->d_buf2[0] = c->d_buf2[1] = nullptr;
-    c->P2[0] = c->P2[1] = nullptr;
+    for (int k = 0; k < 3; ++k) c->d_buf2[k] = c->P2[k] = c->cols[k] = nullptr;
+    c->dcols = nullptr;
     c->xg = nullptr;
     c->tail_in = c->tailP[0] = c->tailP[1] = nullptr;
     c->tail_I = nullptr;
@@ -777,15 +832,17 @@ static skipper_status arena_first(skipper_ctx *c) {
         tp = al256(rowsT * mo * 2);
         ti = al256(rowsT * mi * 4);
     }
-    c->arena_bytes = 2 * pbytes + ibytes + xbytes + tin + 2 * tp + ti;
+    const size_t cbytes = al256(rowsB * max_icol(c) * 2);
+    const int nP = c->nP;
+    c->arena_bytes = nP * pbytes + ibytes + xbytes + tin + 2 * tp + ti + cbytes;
     c->arena = dev_alloc(c, c->arena_bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "first-pass arena of %zu bytes", c->arena_bytes);
     char *p = static_cast<char *>(c->arena);
-    c->P2[0] = reinterpret_cast<uint16_t *>(p);
-    c->P2[1] = reinterpret_cast<uint16_t *>(p + pbytes);
-    c->I_buf = reinterpret_cast<float *>(p + 2 * pbytes);
-    c->xg = reinterpret_cast<uint16_t *>(p + 2 * pbytes + ibytes);
-    char *q = p + 2 * pbytes + ibytes + xbytes;
+    for (int k = 0; k < nP; ++k) c->P2[k] = reinterpret_cast<uint16_t *>(p + k * pbytes);
+    c->I_buf = reinterpret_cast<float *>(p + nP * pbytes);
+    c->xg = reinterpret_cast<uint16_t *>(p + nP * pbytes + ibytes);
+    c->cols[0] = cbytes ? reinterpret_cast<uint16_t *>(p + nP * pbytes + ibytes + xbytes) : nullptr;
+    char *q = p + nP * pbytes + ibytes + xbytes + cbytes;
     c->tail_in = tin ? reinterpret_cast<uint16_t *>(q) : nullptr;
     c->tailP[0] = tp ? reinterpret_cast<uint16_t *>(q + tin) : nullptr;
     c->tailP[1] = tp ? reinterpret_cast<uint16_t *>(q + tin + tp) : nullptr;
@@ -801,7 +858,8 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t dbytes = al256(rowsB * max_n(c) * 2);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
-    bytes += ibytes + 2 * dbytes + xbytes;
+    const size_t cbytes = al256(rowsB * max_icol(c) * 2), dcbytes = al256(rowsB * max_icol(c) * 4);
+    bytes += ibytes + c->nD * (dbytes + cbytes) + xbytes + dcbytes;
     c->arena_bytes = bytes;
     c->arena = dev_alloc(c, bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "segment arena of %zu bytes (%d rows)", bytes, R);
@@ -816,10 +874,13 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     c->I_buf = reinterpret_cast<float *>(p);
     p += ibytes;
     c->d_buf = reinterpret_cast<uint16_t *>(p);
-    c->d_buf2[0] = c->d_buf;
-    c->d_buf2[1] = reinterpret_cast<uint16_t *>(p + dbytes);
-    p += 2 * dbytes;
+    for (int k = 0; k < c->nD; ++k) c->d_buf2[k] = reinterpret_cast<uint16_t *>(p + k * dbytes);
+    p += c->nD * dbytes;
     c->xg = reinterpret_cast<uint16_t *>(p);
+    p += xbytes;
+    for (int k = 0; k < c->nD; ++k) c->cols[k] = cbytes ? reinterpret_cast<uint16_t *>(p + k * cbytes) : nullptr;
+    p += c->nD * cbytes;
+    c->dcols = dcbytes ? reinterpret_cast<float *>(p) : nullptr;
     return SKIPPER_OK;
 }
 
@@ -857,7 +918,15 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
         ok = get_plan(c, {0, in, l.wbp, I, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 1}, g,
                       [&](sk::GemmLaunch *p) { return sk::plan_fc(p, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0); });
-    else if (l.conv)
+    else if (l.icol) {  // explicit im2col rows [nb*H*W][9*Cin] x weights [cout][9*Cin]
+        {
+            ProfScope ps(c, K_IM2COL, (double)nb * (l.Nin * 2 + (double)l.H * l.W * 9 * l.Cin * 2), 0);
+            CK(sk::launch_im2col_bf16(in, c->cols[0], nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
+        }
+        const int M = nb * l.H * l.W, K = 9 * l.Cin;
+        ok = get_plan(c, {4, c->cols[0], l.wb, I, M, l.Cout, K, 0, 0, 1}, g,
+                      [&](sk::GemmLaunch *p) { return sk::plan_fc(p, c->cols[0], l.wb, I, M, l.Cout, K); });
+    } else if (l.conv)
         ok = get_plan(c, {1, in, l.wb, I, nb, l.Cin, l.Cout, l.H, l.W, 1}, g, [&](sk::GemmLaunch *p) {
             return sk::plan_conv(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
         });
@@ -866,8 +935,9 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
             return sk::plan_fc(p, in, l.wb, I, nb, l.Cout, l.Cin, fsp);
         });
     if (ok && g.d.splits != (l.fc ? fsp : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
-    const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
-    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4 * (l.fc ? fsp : 1);
+    const double M = (double)nb * l.H * l.W, K = (double)l.Cin * (l.conv ? 9 : 1);
+    const double bytes = (l.icol ? M * K * 2 : (double)nb * l.Nin * 2) + (double)l.wcount * 2 +
+                         (double)nb * l.N * 4 * (l.fc ? fsp : 1);
     return run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, bytes, 2.0 * M * l.Cout * K);
 }
 
@@ -924,9 +994,23 @@ static skipper_status stage_input(skipper_ctx *c, const int *rows, int t0, int R
     const int kind = c->in_kind == 1 ? 1 : 0;
     const double bytes = (double)R * c->B * (c->in_elems + c->in_row * 2);
     ProfScope ps(c, K_STAGE, bytes, 0);
-    CK(sk::launch_stage_rows(c->x_cur, c->xg, rows, t0, R, c->B, c->in_h, c->in_w, c->in_c, kind, c->K0,
-                             c->in_elems, sam ? spart(c, 0) : nullptr, c->st));
+    const Layer &f = c->L[0];
+    CK(sk::launch_stage_rows(c->x_cur, c->xg, rows, t0, R, c->B, kind == 1 ? f.H : c->in_h, kind == 1 ? f.W : c->in_w,
+                             c->in_c, kind, c->K0, c->in_elems, sam ? spart(c, 0) : nullptr, c->st, f.stride));
     return SKIPPER_OK;
+}
+
+// Residual shortcut of layer i (reading 8): the source layer's bf16 output rows, same row order.
+static void set_res_fwd(const skipper_ctx *c, int i, sk::ScanFwdArgs &a, const uint16_t *src_rows) {
+    const Layer &l = c->L[i];
+    if (l.res < 0) return;
+    const Layer &src = c->L[l.res];
+    a.res = src_rows;
+    a.res_H = src.H;
+    a.res_W = src.W;
+    a.res_C = src.Cout;
+    a.res_stride = src.H / l.H;
+    a.res_lo = (l.Cout - src.Cout) / 2;
 }
 
 // First pass of the fc tail over all T rows (layer-major): GEMM with M = T*B, one scan per layer.
@@ -1067,8 +1151,8 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
             in = i == 0 ? c->xg : c->L[i - 1].Po;
             out = l.Po;
         } else {
-            in = i == 0 ? c->xg : c->P2[(i - 1) & 1];
-            out = (i == c->tail0 - 1) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i & 1];
+            in = i == 0 ? c->xg : c->P2[(i - 1) % c->nP];
+            out = (i == c->tail0 - 1) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i % c->nP];
         }
         if (i == 0 && c->l0_fused) {
             CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));
@@ -1104,6 +1188,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         a.pool = l.pool ? 1 : 0;
         a.lam = l.d.lambda;
         a.theta = l.d.theta;
+        if (l.res >= 0) set_res_fwd(c, i, a, record ? c->L[l.res].Po : c->P2[l.res % c->nP]);
         {
             ProfScope ps(c, K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
             CK(sk::launch_lif_fwd(a, c->st));
@@ -1129,8 +1214,17 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
     ProfScope ps1(c, K_READOUT, (double)c->B * last.Nout * 8 + (double)ro.wcount * 2, 4.0 * c->B * last.Nout * ro.Cout);
     c->launches += 2;  // z, cross-entropy and dL/da^{L-1} kernels
-    CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
-                               ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+    if (ro.gap) {  // readout of the global average pool (reading 23); dL/da^{L-1} spread back over the positions
+        const int P = (int)(last.Nout / last.Cout);
+        c->launches += 2;
+        CK(sk::launch_gap_reduce(c->cnt, c->cnt_gap, c->B, P, last.Cout, c->st));
+        CK(sk::launch_readout_loss(ro.wb, c->cnt_gap, labels, c->z, c->dz, c->loss_dev, c->g_gap, c->B, ro.Cin,
+                                   ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+        CK(sk::launch_gap_expand(c->g_gap, c->g_last, c->B, P, last.Cout, c->st));
+    } else {
+        CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
+                                   ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+    }
     CKS(comm_allreduce_s(c));
     CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
                        c->st));
@@ -1215,6 +1309,7 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
         a.pool = l.pool ? 1 : 0;
         a.lam = l.d.lambda;
         a.theta = l.d.theta;
+        if (l.res >= 0) set_res_fwd(c, i, a, c->L[l.res].Po);
         {
             ProfScope ps(c, K_SCAN_FWD, scan_fwd_bytes(c, l, a), 0);
             CK(sk::launch_lif_fwd(a, c->st));
@@ -1225,13 +1320,15 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
 
 // Eq.2 backward over the R stored rows of a segment (layer-major, reverse t inside the scan).
 static skipper_status join_wgrads(skipper_ctx *c) {
-    for (int k = 0; k < 2; ++k)
+    for (int k = 0; k < 3; ++k)
         if (c->w_pending[k]) {
             CK(cudaStreamWaitEvent(c->st, c->ev_done[k], 0));
             c->w_pending[k] = false;
         }
     return SKIPPER_OK;
 }
+
+static long long rcv_neurons(const skipper_ctx *c, int i) { return i >= 0 ? c->L[i].N : 0; }
 
 static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
     for (int i = c->Ls - 1; i >= 0; --i) {
@@ -1262,7 +1359,7 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             CK(sk::launch_layer0_bwd(b, c->st, c->num_sms));
             continue;
         }
-        const int par = i & 1;
+        const int par = i % c->nD;
         uint16_t *dcur = c->d_buf2[par];
         if (c->w_pending[par]) {  // the wgrad of layer i+2 still reads this delta buffer
             CK(cudaStreamWaitEvent(c->st, c->ev_done[par], 0));
@@ -1287,15 +1384,34 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         a.theta = l.d.theta;
         a.surr = c->cfg.surrogate;
         a.gamma = c->cfg.surr_gamma;
+        if (l.res_to >= 0) {  // shortcut source: S^T(delta of the receiving layer) joins g (reading 8)
+            const Layer &rcv = c->L[l.res_to];
+            a.res_delta = c->d_buf2[l.res_to % c->nD];
+            a.res_C = rcv.Cout;
+            a.res_stride = l.H / rcv.H;
+            a.res_lo = (rcv.Cout - l.Cout) / 2;
+        }
         {
-            ProfScope ps(c, K_SCAN_BWD, scan_bwd_bytes(c, l, a), 0);
+            double bytes = scan_bwd_bytes(c, l, a);
+            if (a.res_delta) bytes += (double)R * c->B * rcv_neurons(c, l.res_to) * 2;
+            ProfScope ps(c, K_SCAN_BWD, bytes, 0);
             CK(sk::launch_lif_bwd(a, c->st));
         }
         const int nb = R * c->B;
         const uint16_t *X = i == 0 ? c->xg : c->L[i - 1].Po;
         sk::GemmLaunch g;
         bool ok;
-        if (i == 0 && c->in_kind == 1)
+        const double Mw = (double)nb * l.H * l.W, Kw = (double)l.Cin * (l.conv ? 9 : 1);
+        if (l.icol) {  // the weight-gradient operand: im2col of the layer input, one slot per delta slot
+            ProfScope ps(c, K_IM2COL, (double)nb * l.Nin * 2 + Mw * Kw * 2, 0);
+            CK(sk::launch_im2col_bf16(X, c->cols[par], nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
+        }
+        if (l.icol)
+            ok = get_plan(c, {6, dcur, c->cols[par], l.dw, (long long)Mw, l.Cout, (int)Kw, 0, 0, 0}, g,
+                          [&](sk::GemmLaunch *p) {
+                              return sk::plan_fc_wgrad(p, dcur, c->cols[par], l.dw, (int)Mw, l.Cout, (int)Kw, c->num_sms);
+                          });
+        else if (i == 0 && c->in_kind == 1)
             ok = get_plan(c, {2, dcur, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
                           [&](sk::GemmLaunch *p) {
                               return sk::plan_fc_wgrad(p, dcur, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
@@ -1308,20 +1424,26 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             ok = get_plan(c, {2, dcur, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
                 return sk::plan_fc_wgrad(p, dcur, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
             });
+        const double wbytes = (double)nb * l.N * 2 + (l.icol ? Mw * Kw * 2 : (double)nb * l.Nin * 2) + (double)l.wcount * 8;
         if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
-            const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
-            const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
-            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K));
+            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw));
         } else {   // weight gradient on the side stream, after this layer's delta is written
             CK(cudaEventRecord(c->ev_ready[par], c->st));
             CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
-            const double M = (double)nb * l.H * l.W, K = (double)l.Nin / (l.H * l.W) * (l.conv ? 9 : 1);
-            const double bytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
-            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, bytes, 2.0 * M * l.Cout * K, c->st2));
+            CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw, c->st2));
             CK(cudaEventRecord(c->ev_done[par], c->st2));
             c->w_pending[par] = true;
         }
-        if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
+        if (i > 0 && l.icol) {  // dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
+            const int M = nb * l.H * l.W, N = 9 * l.Cin;
+            ok = get_plan(c, {5, dcur, l.wt, c->dcols, M, N, l.Cout, 0, 0, 1}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_fc(p, dcur, l.wt, c->dcols, M, N, l.Cout);
+            });
+            const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)M * N * 4;
+            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * N * l.Cout));
+            ProfScope ps(c, K_IM2COL, (double)M * N * 4 + (double)nb * l.Nin * 4, 0);
+            CK(sk::launch_col2im_f32(c->dcols, c->I_buf, nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
+        } else if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
             if (l.conv)
                 ok = get_plan(c, {1, dcur, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g,
                               [&](sk::GemmLaunch *p) {
@@ -1334,7 +1456,7 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
                               });
             const double M = (double)nb * l.H * l.W, K = (double)l.Cout * (l.conv ? 9 : 1);
             const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4 * l.dsplit;
-            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * (l.Nin / (l.H * l.W)) * K));
+            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * l.Cin * K));
         }
     }
     // the next segment reuses the arena (X operands, delta buffers): wait for the weight gradients
@@ -1414,8 +1536,15 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
         }
         ProfScope ps(c, K_READOUT, (double)c->B * (last.Nout + ro.Cout) * 4 + (double)ro.wcount * 4,
                      2.0 * c->B * last.Nout * ro.Cout);
-        CK(sk::launch_readout_wgrad(c->dz, full ? c->cnt : c->cnt_kept, ro.dw, c->B, (int)last.Nout, ro.Cout,
-                                    1.0f / c->T, c->st));
+        const float *cin = full ? c->cnt : c->cnt_kept;
+        int D = (int)last.Nout;
+        if (ro.gap) {
+            c->launches += 1;
+            CK(sk::launch_gap_reduce(cin, c->cnt_gap, c->B, (int)(last.Nout / last.Cout), last.Cout, c->st));
+            cin = c->cnt_gap;
+            D = ro.Cin;
+        }
+        CK(sk::launch_readout_wgrad(c->dz, cin, ro.dw, c->B, D, ro.Cout, 1.0f / c->T, c->st));
         if (c->cfg.debug_record && full)
             for (int i = 0; i < c->Ls; ++i) {
                 const size_t bn = (size_t)c->B * c->L[i].N * c->T;

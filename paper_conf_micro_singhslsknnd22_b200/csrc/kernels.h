@@ -31,6 +31,10 @@ struct ScanFwdArgs {
     uint8_t *dbg_o;
     int B, H, W, C, pool;
     float lam, theta;
+    // ResNet residual (reading 8): I += S(a^r), the option-A shortcut of the bf16 output rows of source
+    // layer r, [R][B][res_H][res_W][res_C] (row r of the segment reads row r); unpooled layers only
+    const uint16_t *res;
+    int res_H, res_W, res_C, res_stride, res_lo;
 };
 cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s);
 
@@ -49,6 +53,10 @@ struct ScanBwdArgs {
     float lam, theta;
     int surr;
     float gamma;
+    // ResNet residual (reading 8): this layer is the shortcut source of a later layer whose bf16 delta
+    // rows res_delta [R][B][H/res_stride][W/res_stride][res_C] add S^T(delta) to g (unpooled layers only)
+    const uint16_t *res_delta;
+    int res_C, res_stride, res_lo;
 };
 cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s);
 
@@ -56,8 +64,21 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s);
 // kind 0: bf16 copy of x[t] (D = elements per sample); kind 1: 3x3/pad-1 im2col of an
 // H x W x C0 image zero-padded to K0 columns.  rows: device list of t (or null -> t0 + r).
 // s_part != null adds the SAM term l = 0 (Eq.4).
+// kind 1 with stride 2: H x W are the OUTPUT pixels, the image is (2H) x (2W); SAM counts every input pixel.
 cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, int t0, int R, int B, int H, int W,
-                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s);
+                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s, int stride = 1);
+
+// Narrow / strided conv layers (ResNet SNN): explicit 3x3 im2col of bf16 NHWC rows,
+// cols[(n, y, x)][(dy*3+dx)*Cin + ci] = X[n][s*y+dy-1][s*x+dx-1][ci] (zero outside), Cin % 8 == 0.
+cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, int Hin, int Win, int Cin, int H,
+                               int W, int stride, cudaStream_t s);
+// Adjoint: G[n][yi][xi][ci] = sum_{dy,dx: s | (yi+1-dy), s | (xi+1-dx)} dcols[(n, y, x)][ci*9 + dy*3+dx]
+// (column order (ci, tap): the dgrad GEMM's B operand is the transposed shadow [cin][9][cout]).
+cudaError_t launch_col2im_f32(const float *dcols, float *G, long long nb, int Hin, int Win, int Cin, int H, int W,
+                              int stride, cudaStream_t s);
+// Global average pool of the readout input (reading 23): out[b][c] = sum_p in[b][p][c] / P, and its adjoint.
+cudaError_t launch_gap_reduce(const float *in, float *out, int B, int P, int C, cudaStream_t s);
+cudaError_t launch_gap_expand(const float *g, float *out, int B, int P, int C, cudaStream_t s);
 cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);

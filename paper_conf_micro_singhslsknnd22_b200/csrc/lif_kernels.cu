@@ -111,6 +111,17 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
             oidx = nidx[0];
         }
     }
+    // residual shortcut (reading 8): offset of this thread's 4 channels in a source row, or -1 (zero pad)
+    long long res_off = -1, res_rs = 0;
+    if (!POOL && a.res && active) {
+        const long long pix = p / C4;
+        const int x = (int)(pix % a.W), y = (int)((pix / a.W) % a.H);
+        const long long b = pix / HW;
+        const int cs = 4 * (int)(p % C4) - a.res_lo;
+        res_rs = (long long)a.B * a.res_H * a.res_W * a.res_C;
+        if (cs >= 0 && cs < a.res_C)
+            res_off = ((b * a.res_H + (long long)y * a.res_stride) * a.res_W + (long long)x * a.res_stride) * a.res_C + cs;
+    }
 
     float U[NP][4];
     uint32_t ob = 0;  // spike bits, bit 4k+i
@@ -175,6 +186,13 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
                 if (active && r < a.R) {
                     const float *src = a.I + (long long)r * rs + nidx[k];
                     Iv[j][k] = SPLIT ? ldg4_split(src, nspl, a.split_stride) : ldg4(src);
+                    if (!POOL && res_off >= 0) {  // I += S(a^r): exact (spikes added to the fp32 GEMM sum)
+                        const uint2 rv = __ldg(reinterpret_cast<const uint2 *>(a.res + (long long)r * res_rs + res_off));
+                        Iv[j][k].x = __fadd_rn(Iv[j][k].x, __uint_as_float(rv.x << 16));
+                        Iv[j][k].y = __fadd_rn(Iv[j][k].y, __uint_as_float(rv.x & 0xffff0000u));
+                        Iv[j][k].z = __fadd_rn(Iv[j][k].z, __uint_as_float(rv.y << 16));
+                        Iv[j][k].w = __fadd_rn(Iv[j][k].w, __uint_as_float(rv.y & 0xffff0000u));
+                    }
                 } else {
                     Iv[j][k] = make_float4(0.f, 0.f, 0.f, 0.f);
                 }
@@ -323,7 +341,8 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
 
 cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
-    if (!a.pool && a.H * a.W == 1 && (long long)a.B * a.C <= (1LL << 20)) {  // fc layers
+    if (a.res && (a.pool || a.H * a.W == 1 || a.res_C % 4 || a.res_lo % 4 || a.res_stride < 1)) return cudaErrorInvalidValue;
+    if (!a.pool && !a.res && a.H * a.W == 1 && (long long)a.B * a.C <= (1LL << 20)) {  // fc layers
         const long long rs = (long long)a.B * a.C;
         const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
         if (smem > 48 * 1024) return cudaErrorInvalidValue;
@@ -376,6 +395,18 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
     if (a.g_broadcast) grs = 0;
     const float gs = a.g_pooled ? 0.25f : 1.0f;
     const int nspl = SPLIT ? a.nsplit : 1;
+    // shortcut source (reading 8): S^T(delta of the receiving layer) joins g at this neuron, or not
+    long long rd_off = -1, rd_rs = 0;
+    if (a.res_delta) {
+        const int c = (int)(n0 % C);
+        const long long pixel = n0 / C;
+        const int x = (int)(pixel % a.W), y = (int)((pixel / a.W) % a.H);
+        const long long b = pixel / HW;
+        const int s = a.res_stride, Hr = a.H / s, Wr = a.W / s;
+        rd_rs = (long long)a.B * Hr * Wr * a.res_C;
+        if (y % s == 0 && x % s == 0)
+            rd_off = ((b * Hr + y / s) * Wr + x / s) * a.res_C + c + a.res_lo;
+    }
     float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
     // two chunks of CH rows in flight: loads of the next (earlier) chunk overlap the recurrence
     auto load = [&](float4 (&gv)[CH], float4 (&uv)[CH], int rb) {
@@ -386,6 +417,13 @@ __global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
                 const float *src = a.g + (long long)r * grs + gi;
                 gv[j] = SPLIT ? ldg4_split(src, nspl, a.split_stride) : ldg4(src);
                 uv[j] = ldg4(a.U + (long long)r * rs + n0);
+                if (rd_off >= 0) {
+                    const uint2 rv = __ldg(reinterpret_cast<const uint2 *>(a.res_delta + (long long)r * rd_rs + rd_off));
+                    gv[j].x = __fadd_rn(gv[j].x, __uint_as_float(rv.x << 16));  // unpooled: gs = 1
+                    gv[j].y = __fadd_rn(gv[j].y, __uint_as_float(rv.x & 0xffff0000u));  // unpooled: gs = 1
+                    gv[j].z = __fadd_rn(gv[j].z, __uint_as_float(rv.y << 16));  // unpooled: gs = 1
+                    gv[j].w = __fadd_rn(gv[j].w, __uint_as_float(rv.y & 0xffff0000u));  // unpooled: gs = 1
+                }
             }
         }
     };
@@ -453,7 +491,10 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     if (rs == 0 || a.R == 0) return cudaSuccess;
-    if (!a.g_pooled && a.H * a.W == 1 && rs <= (1LL << 20)) {  // fc layers
+    if (a.res_delta && (a.pool || a.H * a.W == 1 || a.res_lo % 4 || a.res_stride < 1 || a.H % a.res_stride ||
+                        a.W % a.res_stride))
+        return cudaErrorInvalidValue;
+    if (!a.g_pooled && !a.res_delta && a.H * a.W == 1 && rs <= (1LL << 20)) {  // fc layers
         if (a.nsplit > 1)
             lif_bwd_small_kernel<4, 1><<<(unsigned)((rs + 255) / 256), 256, 0, s>>>(a);
         else
@@ -474,7 +515,7 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
 // SAM term l = 0 (Eq.4) is counted when s_part is given (FIRST pass only).
 __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__restrict__ dst, const int *rows, int t0,
                                   int R, int B, int H, int W, int C0, int kind, int K0, long long D,
-                                  unsigned *s_part) {
+                                  unsigned *s_part, int stride) {
     const long long per_row = kind == 1 ? (long long)B * H * W : (long long)B * D;
     const long long total = (long long)R * per_row;
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -488,21 +529,26 @@ __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__res
             const int xx = (int)(e % W);
             const int yy = (int)((e / W) % H);
             const long long b = e / ((long long)H * W);
-            const uint8_t *xt = x + (t * B + b) * (long long)H * W * C0;
+            const int Hi = H * stride, Wi = W * stride;  // input image (H x W output pixels)
+            const uint8_t *xt = x + (t * B + b) * (long long)Hi * Wi * C0;
             uint64_t m = 0;  // bit k = im2col column k (registers only: no dynamically indexed arrays)
             for (int dy = 0; dy < 3; ++dy) {
-                const int y = yy + dy - 1;
-                if (y < 0 || y >= H) continue;
+                const int y = stride * yy + dy - 1;
+                if (y < 0 || y >= Hi) continue;
                 for (int dx = 0; dx < 3; ++dx) {
-                    const int xq = xx + dx - 1;
-                    if (xq < 0 || xq >= W) continue;
-                    const uint8_t *px = xt + ((long long)y * W + xq) * C0;
+                    const int xq = stride * xx + dx - 1;
+                    if (xq < 0 || xq >= Wi) continue;
+                    const uint8_t *px = xt + ((long long)y * Wi + xq) * C0;
                     for (int ci = 0; ci < C0; ++ci)
                         if (__ldg(px + ci)) m |= 1ull << ((dy * 3 + dx) * C0 + ci);
                 }
             }
-            const uint8_t *pc = xt + ((long long)yy * W + xx) * C0;
-            for (int ci = 0; ci < C0; ++ci) cnt += __ldg(pc + ci) ? 1u : 0u;
+            if (s_part)  // SAM l = 0: this output pixel's stride x stride block of input pixels
+                for (int sy = 0; sy < stride; ++sy)
+                    for (int sx = 0; sx < stride; ++sx) {
+                        const uint8_t *pc = xt + ((long long)(stride * yy + sy) * Wi + stride * xx + sx) * C0;
+                        for (int ci = 0; ci < C0; ++ci) cnt += __ldg(pc + ci) ? 1u : 0u;
+                    }
             uint4 *o = reinterpret_cast<uint4 *>(dst + i * K0);
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
@@ -536,13 +582,108 @@ __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__res
 }
 
 cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, int t0, int R, int B, int H, int W,
-                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s) {
+                              int C0, int kind, int K0, long long D, unsigned *s_part, cudaStream_t s, int stride) {
     const long long per_row = kind == 1 ? (long long)B * H * W : (long long)B * D;
     const long long total = (long long)R * per_row;
     if (total == 0) return cudaSuccess;
-    if (kind == 1 && (K0 % 8 || K0 > 64 || 9 * C0 > K0)) return cudaErrorInvalidValue;
+    if (kind == 1 && (K0 % 8 || K0 > 64 || 9 * C0 > K0 || stride < 1 || stride > 2)) return cudaErrorInvalidValue;
     stage_rows_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, dst, rows, t0, R, B, H, W, C0, kind, K0, D,
-                                                                     s_part);
+                                                                     s_part, stride);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------- narrow / strided convs
+// One thread per (output pixel, tap, 8-channel chunk): 16-byte load (or zero) -> 16-byte store.
+__global__ void im2col_bf16_kernel(const uint16_t *__restrict__ X, uint16_t *__restrict__ cols, long long total,
+                                   int Hin, int Win, int Cin, int H, int W, int stride) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= total) return;
+    const int C8 = Cin >> 3;
+    const int ch = (int)(i % C8);
+    const long long q = i / C8;
+    const int tap = (int)(q % 9);
+    const long long m = q / 9;
+    const int x = (int)(m % W), y = (int)((m / W) % H);
+    const long long n = m / ((long long)H * W);
+    const int yi = stride * y + tap / 3 - 1, xi = stride * x + tap % 3 - 1;
+    uint4 v = make_uint4(0u, 0u, 0u, 0u);
+    if (yi >= 0 && yi < Hin && xi >= 0 && xi < Win)
+        v = __ldg(reinterpret_cast<const uint4 *>(X + ((n * Hin + yi) * Win + xi) * Cin) + ch);
+    reinterpret_cast<uint4 *>(cols)[i] = v;
+}
+
+cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, int Hin, int Win, int Cin, int H,
+                               int W, int stride, cudaStream_t s) {
+    if (Cin % 8) return cudaErrorInvalidValue;
+    const long long total = nb * H * W * 9 * (Cin / 8);
+    if (total == 0) return cudaSuccess;
+    im2col_bf16_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(X, cols, total, Hin, Win, Cin, H, W, stride);
+    return cudaGetLastError();
+}
+
+// One thread per input neuron (n, yi, xi, ci): the <= 9 tap contributions in fixed order (deterministic).
+__global__ void col2im_f32_kernel(const float *__restrict__ dcols, float *__restrict__ G, long long total, int Hin,
+                                  int Win, int Cin, int H, int W, int stride) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= total) return;
+    const int ci = (int)(i % Cin);
+    const long long pix = i / Cin;
+    const int xi = (int)(pix % Win), yi = (int)((pix / Win) % Hin);
+    const long long n = pix / ((long long)Hin * Win);
+    float acc = 0.f;
+#pragma unroll
+    for (int dy = 0; dy < 3; ++dy) {
+        const int ys = yi + 1 - dy;
+        if (ys < 0 || ys % stride) continue;
+        const int y = ys / stride;
+        if (y >= H) continue;
+#pragma unroll
+        for (int dx = 0; dx < 3; ++dx) {
+            const int xs = xi + 1 - dx;
+            if (xs < 0 || xs % stride) continue;
+            const int x = xs / stride;
+            if (x >= W) continue;
+            acc = __fadd_rn(acc, __ldg(dcols + ((n * H + y) * W + x) * 9LL * Cin + ci * 9 + dy * 3 + dx));
+        }
+    }
+    G[i] = acc;
+}
+
+cudaError_t launch_col2im_f32(const float *dcols, float *G, long long nb, int Hin, int Win, int Cin, int H, int W,
+                              int stride, cudaStream_t s) {
+    const long long total = nb * Hin * Win * Cin;
+    if (total == 0) return cudaSuccess;
+    col2im_f32_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(dcols, G, total, Hin, Win, Cin, H, W, stride);
+    return cudaGetLastError();
+}
+
+// Global average pool (reading 23): one thread per (b, c), positions summed in order, then / P (exact for
+// spike counts: integers < 2^24 and P a power of two in the supported networks).
+__global__ void gap_reduce_kernel(const float *__restrict__ in, float *__restrict__ out, int B, int P, int C) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= B * C) return;
+    const int b = i / C, c = i % C;
+    float acc = 0.f;
+    for (int p = 0; p < P; ++p) acc += in[((long long)b * P + p) * C + c];
+    out[i] = acc / (float)P;
+}
+
+__global__ void gap_expand_kernel(const float *__restrict__ g, float *__restrict__ out, int B, int P, int C) {
+    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= (long long)B * P * C) return;
+    const int c = (int)(i % C);
+    const long long b = i / ((long long)P * C);
+    out[i] = g[b * C + c] / (float)P;
+}
+
+cudaError_t launch_gap_reduce(const float *in, float *out, int B, int P, int C, cudaStream_t s) {
+    gap_reduce_kernel<<<(B * C + 255) / 256, 256, 0, s>>>(in, out, B, P, C);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gap_expand(const float *g, float *out, int B, int P, int C, cudaStream_t s) {
+    const long long n = (long long)B * P * C;
+    gap_expand_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(g, out, B, P, C);
     return cudaGetLastError();
 }
 

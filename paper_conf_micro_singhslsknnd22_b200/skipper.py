@@ -31,7 +31,8 @@ class SkipperError(RuntimeError):
 
 class Layer(ct.Structure):
     _fields_ = [("kind", ct.c_int), ("cin", ct.c_int), ("cout", ct.c_int), ("h", ct.c_int), ("w", ct.c_int),
-                ("pool", ct.c_int), ("lam", ct.c_float), ("theta", ct.c_float)]
+                ("pool", ct.c_int), ("lam", ct.c_float), ("theta", ct.c_float), ("stride", ct.c_int),
+                ("residual_from", ct.c_int)]
 
 
 class Config(ct.Structure):
@@ -118,8 +119,11 @@ def _check(status, ctx=None):
 def make_layers(net):
     arr = (Layer * len(net["layers"]))()
     for i, L in enumerate(net["layers"]):
+        pool = (1 if L.get("gap") else 0) if L["kind"] == "readout" else L.get("pool", 0)
+        res = L.get("res")
         arr[i] = Layer(LAYER_KIND[L["kind"]], L["cin"], L["cout"], L.get("h", 1), L.get("w", 1),
-                       L.get("pool", 0), float(L.get("lam", 1.0)), float(L.get("theta", 1.0)))
+                       pool, float(L.get("lam", 1.0)), float(L.get("theta", 1.0)), int(L.get("stride", 1)),
+                       -1 if res is None else int(res))
     return arr
 
 

@@ -188,3 +188,17 @@ def test_vgg11_reduced(mode):
 def test_sam_weighted(name, T, B, C, p):
     """NEXT-2: the neuron-count-weighted SAM (reading 22) selects the same steps as the oracle."""
     check_parity(name, T=T, B=B, C=C, p=p, mode="skip", sam="weighted")
+
+
+@pytest.mark.parametrize("mode,lam", [("full", 0.99), ("ckpt", 1.0), ("skip", 0.99), ("skip", 0.75)])
+def test_tiny_resnet(mode, lam):
+    """ResNet SNN pieces (reading 8, 23): stride-2 stem from DVS events, narrow im2col convs, identity and
+    stride-2 / channel-padded option-A shortcuts, GAP readout."""
+    check_parity("tiny_resnet", T=12, B=3, C=2, p=50.0, mode=mode, lam=lam)
+
+
+@pytest.mark.parametrize("mode", ["skip", "full"])
+def test_resnet20_dvs_reduced(mode):
+    """cfg 4 topology (ResNet-20 SNN on 2x128x128 DVS frames) at reduced T and B: 19 spiking layers of
+    every conv kind (im2col 16/32 channels, stride 2, implicit 64-channel, fused conv+LIF), 9 shortcuts."""
+    check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode=mode)
