@@ -65,11 +65,12 @@ def describe(net):
     parts = []
     for L in net["layers"]:
         if L["kind"] == "conv":
-            parts.append(f"conv{L['cin']}-{L['cout']}@{L['h']}" + ("p" if L["pool"] else ""))
+            parts.append(f"conv{L['cin']}-{L['cout']}@{L['h']}" + ("p" if L["pool"] else "")
+                         + ("s2" if L.get("stride", 1) == 2 else "") + (f"+r{L['res']}" if "res" in L else ""))
         elif L["kind"] == "fc":
             parts.append(f"fc{L['cin']}-{L['cout']}")
         else:
-            parts.append(f"readout{L['cin']}-{L['cout']}")
+            parts.append(("gap-" if L.get("gap") else "") + f"readout{L['cin']}-{L['cout']}")
     return " ".join(parts)
 
 
@@ -162,7 +163,9 @@ def config_block(args, wl, net):
     return {"workload": args.workload, "net": describe(net), "T": wl["T"], "per_gpu_batch": wl["B"],
             "global_batch": wl["B"] * args.gpus, "C": wl["C"], "p": wl["p"], "mode": args.mode,
             "parallelism": f"dp{args.gpus}", "l2": "flushed between timed steps (512 MB write)",
-            "inputs": "Poisson rate-coded CIFAR-shaped frames, seeded; grid-quantised random weights"}
+            "inputs": ("DVS-Gesture-shaped event frames (2x128x128, moving blob, burst envelope)"
+                       if net["input"][0] == "dvs" else "Poisson rate-coded CIFAR-shaped frames")
+                      + ", seeded; grid-quantised random weights"}
 
 
 # ------------------------------------------------------------------------------------- GPU arm

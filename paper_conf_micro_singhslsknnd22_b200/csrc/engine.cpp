@@ -1152,7 +1152,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
             out = l.Po;
         } else {
             in = i == 0 ? c->xg : c->P2[(i - 1) % c->nP];
-            out = (i == c->tail0 - 1) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i % c->nP];
+            out = (i == c->tail0 - 1 && c->tail0 < c->Ls) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i % c->nP];
         }
         if (i == 0 && c->l0_fused) {
             CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));

@@ -90,13 +90,12 @@ def dvs_frames(T: int, B: int, H: int = 128, W: int = 128, seed: int = 1) -> np.
     phase = rng.random(B) * 2 * np.pi
     for t in range(T):
         burst = 0.5 + 0.5 * math.sin(math.pi * t / 40.0) ** 2
-        for b in range(B):
-            cy = H / 2 + H / 4 * math.sin(phase[b] + t / 20.0)
-            cx = W / 2 + W / 4 * math.cos(phase[b] + t / 20.0)
-            blob = np.exp(-((yy - cy) ** 2 + (xx - cx) ** 2) / (2 * (H / 8) ** 2))
-            prob = (0.005 + 0.12 * blob * burst).astype(np.float32)
-            u = rng.random((H, W, 2), dtype=np.float32)
-            out[t, b] = u < prob[..., None]
+        cy = (H / 2 + H / 4 * np.sin(phase + t / 20.0)).astype(np.float32)[:, None, None]
+        cx = (W / 2 + W / 4 * np.cos(phase + t / 20.0)).astype(np.float32)[:, None, None]
+        blob = np.exp(-((yy - cy) ** 2 + (xx - cx) ** 2) / np.float32(2 * (H / 8) ** 2))
+        prob = (0.005 + 0.12 * blob * burst).astype(np.float32)
+        u = rng.random((B, H, W, 2), dtype=np.float32)
+        out[t] = u < prob[..., None]
     return out
 
 

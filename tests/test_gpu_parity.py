@@ -41,11 +41,17 @@ def grad_ok(g, r, tol=1e-3):
     return rel <= tol and mx <= tol, f"normwise {rel:.2e} maxabs {mx:.2e}"
 
 
-def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes"):
+def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=False):
+    """deep=True (networks deeper than the 11 spiking layers of VGG-11): a layer's dW tolerance is
+    max(1e-3, the size of the bf16 contract's own effect on that layer), DESIGN.md §4 "deep networks"."""
     net = synth.net_config(name, lam=lam)
     W = synth.make_weights(net, seed=seed)
     x, y = synth.make_inputs(net, T, B, seed=seed + 1)
     ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True, sam=sam))
+    tols = [1e-3] * len(ref.dW)
+    if deep:
+        exact = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, sam=sam, emulate_bf16=False))
+        tols = [max(1e-3, np.linalg.norm(a - b) / max(np.linalg.norm(a), 1e-300)) for a, b in zip(ref.dW, exact.dW)]
     m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam)
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
     # SAM and mask (Eq.4, Eq.5)
@@ -66,8 +72,8 @@ def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes"):
     assert loss == pytest.approx(ref.loss, rel=1e-5)
     grads = m.grads()
     for l, (g, r) in enumerate(zip(grads, ref.dW)):
-        ok, msg = grad_ok(g.cpu().numpy(), r)
-        assert ok, f"layer {l} dW: {msg}"
+        ok, msg = grad_ok(g.cpu().numpy(), r, tols[l])
+        assert ok, f"layer {l} dW: {msg} (tolerance {tols[l]:.1e})"
     # one Adam step from the shared starting point
     w_new = m.weights()
     for l, (wn, w0, r, g) in enumerate(zip(w_new, W, ref.dW, grads)):
@@ -194,11 +200,11 @@ def test_sam_weighted(name, T, B, C, p):
 def test_tiny_resnet(mode, lam):
     """ResNet SNN pieces (reading 8, 23): stride-2 stem from DVS events, narrow im2col convs, identity and
     stride-2 / channel-padded option-A shortcuts, GAP readout."""
-    check_parity("tiny_resnet", T=12, B=3, C=2, p=50.0, mode=mode, lam=lam)
+    check_parity("tiny_resnet", T=16, B=3, C=2, p=50.0, mode=mode, lam=lam)
 
 
 @pytest.mark.parametrize("mode", ["skip", "full"])
 def test_resnet20_dvs_reduced(mode):
     """cfg 4 topology (ResNet-20 SNN on 2x128x128 DVS frames) at reduced T and B: 19 spiking layers of
     every conv kind (im2col 16/32 channels, stride 2, implicit 64-channel, fused conv+LIF), 9 shortcuts."""
-    check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode=mode)
+    check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode=mode, deep=True)
