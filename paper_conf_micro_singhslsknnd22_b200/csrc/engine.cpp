@@ -479,6 +479,17 @@ static long long max_icol(const skipper_ctx *c) {  // im2col columns per sample-
         if (c->L[i].icol) m = std::max(m, (long long)c->L[i].H * c->L[i].W * 9 * c->L[i].Cin);
     return m;
 }
+// icol layers run in chunks of sample-rows so that the im2col / dgrad column buffers stay bounded
+// (SKIPPER_ICOL_CHUNK_MB of bf16 columns, default 1024) however many rows a pass has.
+static long long icol_chunk(const skipper_ctx *c) {
+    static long long mb = -1;
+    if (mb < 0) {
+        const char *e = getenv("SKIPPER_ICOL_CHUNK_MB");
+        mb = e ? std::max(1, atoi(e)) : 1024;
+    }
+    const long long per = max_icol(c) * 2;
+    return per ? std::max(1LL, (mb << 20) / per) : 1;
+}
 static long long max_gemm_io(const skipper_ctx *c) {  // fp32 I (fwd) and g (dgrad) per sample-row
     long long m = 0;
     for (int i = 0; i < c->Ls; ++i) {
@@ -832,7 +843,7 @@ static skipper_status arena_first(skipper_ctx *c) {
         tp = al256(rowsT * mo * 2);
         ti = al256(rowsT * mi * 4);
     }
-    const size_t cbytes = al256(rowsB * max_icol(c) * 2);
+    const size_t cbytes = al256(std::min<long long>(rowsB, icol_chunk(c)) * max_icol(c) * 2);
     const int nP = c->nP;
     c->arena_bytes = nP * pbytes + ibytes + xbytes + tin + 2 * tp + ti + cbytes;
     c->arena = dev_alloc(c, c->arena_bytes);
@@ -858,7 +869,8 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t dbytes = al256(rowsB * max_n(c) * 2);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
-    const size_t cbytes = al256(rowsB * max_icol(c) * 2), dcbytes = al256(rowsB * max_icol(c) * 4);
+    const long long ch = std::min<long long>(rowsB, icol_chunk(c));
+    const size_t cbytes = al256(ch * max_icol(c) * 2), dcbytes = al256(ch * max_icol(c) * 4);
     bytes += ibytes + c->nD * (dbytes + cbytes) + xbytes + dcbytes;
     c->arena_bytes = bytes;
     c->arena = dev_alloc(c, bytes);
@@ -918,14 +930,25 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
         ok = get_plan(c, {0, in, l.wbp, I, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 1}, g,
                       [&](sk::GemmLaunch *p) { return sk::plan_fc(p, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0); });
-    else if (l.icol) {  // explicit im2col rows [nb*H*W][9*Cin] x weights [cout][9*Cin]
-        {
-            ProfScope ps(c, K_IM2COL, (double)nb * (l.Nin * 2 + (double)l.H * l.W * 9 * l.Cin * 2), 0);
-            CK(sk::launch_im2col_bf16(in, c->cols[0], nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
+    else if (l.icol) {  // explicit im2col rows [nb*H*W][9*Cin] x weights [cout][9*Cin], in sample-row chunks
+        const long long ch = icol_chunk(c);
+        const int K = 9 * l.Cin;
+        for (long long n0 = 0; n0 < nb; n0 += ch) {
+            const int nbc = (int)std::min<long long>(ch, nb - n0);
+            {
+                ProfScope ps(c, K_IM2COL, (double)nbc * (l.Nin * 2 + (double)l.H * l.W * K * 2), 0);
+                CK(sk::launch_im2col_bf16(in + n0 * l.Nin, c->cols[0], nbc, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride,
+                                          c->st));
+            }
+            const int M = nbc * l.H * l.W;
+            float *Ic = I + n0 * l.N;
+            ok = get_plan(c, {4, c->cols[0], l.wb, Ic, M, l.Cout, K, 0, 0, 1}, g,
+                          [&](sk::GemmLaunch *p) { return sk::plan_fc(p, c->cols[0], l.wb, Ic, M, l.Cout, K); });
+            const double Mf = M;
+            CKS(run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, Mf * K * 2 + (double)l.wcount * 2 + (double)nbc * l.N * 4,
+                         2.0 * Mf * l.Cout * K));
         }
-        const int M = nb * l.H * l.W, K = 9 * l.Cin;
-        ok = get_plan(c, {4, c->cols[0], l.wb, I, M, l.Cout, K, 0, 0, 1}, g,
-                      [&](sk::GemmLaunch *p) { return sk::plan_fc(p, c->cols[0], l.wb, I, M, l.Cout, K); });
+        return SKIPPER_OK;
     } else if (l.conv)
         ok = get_plan(c, {1, in, l.wb, I, nb, l.Cin, l.Cout, l.H, l.W, 1}, g, [&](sk::GemmLaunch *p) {
             return sk::plan_conv(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1);
@@ -1402,16 +1425,33 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
         sk::GemmLaunch g;
         bool ok;
         const double Mw = (double)nb * l.H * l.W, Kw = (double)l.Cin * (l.conv ? 9 : 1);
-        if (l.icol) {  // the weight-gradient operand: im2col of the layer input, one slot per delta slot
-            ProfScope ps(c, K_IM2COL, (double)nb * l.Nin * 2 + Mw * Kw * 2, 0);
-            CK(sk::launch_im2col_bf16(X, c->cols[par], nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
-        }
-        if (l.icol)
-            ok = get_plan(c, {6, dcur, c->cols[par], l.dw, (long long)Mw, l.Cout, (int)Kw, 0, 0, 0}, g,
-                          [&](sk::GemmLaunch *p) {
-                              return sk::plan_fc_wgrad(p, dcur, c->cols[par], l.dw, (int)Mw, l.Cout, (int)Kw, c->num_sms);
-                          });
-        else if (i == 0 && c->in_kind == 1)
+        if (l.icol) {  // im2col of the layer input + weight-gradient GEMM per chunk, one column slot per delta slot
+            cudaStream_t ws = c->prof_on ? c->st : c->st2;
+            if (!c->prof_on) {
+                CK(cudaEventRecord(c->ev_ready[par], c->st));
+                CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
+            }
+            const long long ch = icol_chunk(c);
+            for (long long n0 = 0; n0 < nb; n0 += ch) {
+                const int nbc = (int)std::min<long long>(ch, nb - n0);
+                const int M = nbc * l.H * l.W;
+                {
+                    ProfScope ps(c, K_IM2COL, (double)nbc * l.Nin * 2 + (double)M * Kw * 2, 0, ws);
+                    CK(sk::launch_im2col_bf16(X + n0 * l.Nin, c->cols[par], nbc, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride,
+                                              ws));
+                }
+                const uint16_t *Dc = dcur + n0 * l.N;
+                ok = get_plan(c, {6, Dc, c->cols[par], l.dw, M, l.Cout, (int)Kw, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
+                    return sk::plan_fc_wgrad(p, Dc, c->cols[par], l.dw, M, l.Cout, (int)Kw, c->num_sms);
+                });
+                CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, (double)nbc * l.N * 2 + (double)M * Kw * 2 + (double)l.wcount * 8,
+                             2.0 * M * l.Cout * Kw, ws));
+            }
+            if (!c->prof_on) {
+                CK(cudaEventRecord(c->ev_done[par], c->st2));
+                c->w_pending[par] = true;
+            }
+        } else if (i == 0 && c->in_kind == 1)
             ok = get_plan(c, {2, dcur, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
                           [&](sk::GemmLaunch *p) {
                               return sk::plan_fc_wgrad(p, dcur, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
@@ -1424,8 +1464,10 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             ok = get_plan(c, {2, dcur, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
                 return sk::plan_fc_wgrad(p, dcur, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
             });
-        const double wbytes = (double)nb * l.N * 2 + (l.icol ? Mw * Kw * 2 : (double)nb * l.Nin * 2) + (double)l.wcount * 8;
-        if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
+        const double wbytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
+        if (l.icol) {
+            // issued above
+        } else if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
             CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw));
         } else {   // weight gradient on the side stream, after this layer's delta is written
             CK(cudaEventRecord(c->ev_ready[par], c->st));
@@ -1434,15 +1476,22 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             CK(cudaEventRecord(c->ev_done[par], c->st2));
             c->w_pending[par] = true;
         }
-        if (i > 0 && l.icol) {  // dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
-            const int M = nb * l.H * l.W, N = 9 * l.Cin;
-            ok = get_plan(c, {5, dcur, l.wt, c->dcols, M, N, l.Cout, 0, 0, 1}, g, [&](sk::GemmLaunch *p) {
-                return sk::plan_fc(p, dcur, l.wt, c->dcols, M, N, l.Cout);
-            });
-            const double bytes = (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)M * N * 4;
-            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * N * l.Cout));
-            ProfScope ps(c, K_IM2COL, (double)M * N * 4 + (double)nb * l.Nin * 4, 0);
-            CK(sk::launch_col2im_f32(c->dcols, c->I_buf, nb, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride, c->st));
+        if (i > 0 && l.icol) {  // per chunk: dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
+            const long long ch = icol_chunk(c);
+            const int N = 9 * l.Cin;
+            for (long long n0 = 0; n0 < nb; n0 += ch) {
+                const int nbc = (int)std::min<long long>(ch, nb - n0);
+                const int M = nbc * l.H * l.W;
+                const uint16_t *Dc = dcur + n0 * l.N;
+                ok = get_plan(c, {5, Dc, l.wt, c->dcols, M, N, l.Cout, 0, 0, 1}, g, [&](sk::GemmLaunch *p) {
+                    return sk::plan_fc(p, Dc, l.wt, c->dcols, M, N, l.Cout);
+                });
+                const double bytes = (double)nbc * l.N * 2 + (double)l.wcount * 2 + (double)M * N * 4;
+                CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * N * l.Cout));
+                ProfScope ps(c, K_IM2COL, (double)M * N * 4 + (double)nbc * l.Nin * 4, 0);
+                CK(sk::launch_col2im_f32(c->dcols, c->I_buf + n0 * l.Nin, nbc, l.Hin, l.Win, l.Cin, l.H, l.W, l.stride,
+                                         c->st));
+            }
         } else if (i > 0) {  // g for layer i-1 = delta_i W_i  (gradient wrt its (pooled) output)
             if (l.conv)
                 ok = get_plan(c, {1, dcur, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g,
