@@ -48,7 +48,8 @@ def grad_ok(g, r, tol=(1e-3, 1e-3)):
 
 def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=False):
     """deep=True (networks deeper than the 11 spiking layers of VGG-11): a layer's dW tolerance is
-    max(1e-3, the size of the bf16 contract's own effect on that layer), DESIGN.md §4 "deep networks"."""
+    max(1e-3, the size of the bf16 contract's own effect on that layer: normwise, and twice it for the
+    max-abs measure), DESIGN.md §4 "deep networks"."""
     net = synth.net_config(name, lam=lam)
     W = synth.make_weights(net, seed=seed)
     x, y = synth.make_inputs(net, T, B, seed=seed + 1)
@@ -56,7 +57,10 @@ def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=Fa
     tols = [(1e-3, 1e-3)] * len(ref.dW)
     if deep:
         exact = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, sam=sam, emulate_bf16=False))
-        tols = [tuple(max(1e-3, e) for e in grad_errs(b, a)) for a, b in zip(ref.dW, exact.dW)]
+        tols = []
+        for a, b in zip(ref.dW, exact.dW):
+            en, em = grad_errs(b, a)
+            tols.append((max(1e-3, en), max(1e-3, 2 * em)))  # a single element's error is noisier than the norm
     m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam)
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
     # SAM and mask (Eq.4, Eq.5)
