@@ -169,13 +169,28 @@ def config_block(args, wl, net):
 
 
 # ------------------------------------------------------------------------------------- GPU arm
+_INPUT_CACHE = {}
+
+
+def cached_inputs(net, T, B, seed):
+    """Seeded inputs; frames are prefix-consistent in T (synth draws them in t order), so the longest
+    sequence generated so far for (net, B, seed) is reused by slicing."""
+    key = (json.dumps(net["input"]), net["layers"][-1]["cout"], B, seed)
+    hit = _INPUT_CACHE.get(key)
+    if hit is None or hit[0].shape[0] < T:
+        _INPUT_CACHE.clear()
+        hit = synth.make_inputs(net, T, B, seed=seed)
+        _INPUT_CACHE[key] = hit
+    return np.ascontiguousarray(hit[0][:T]), hit[1]
+
+
 def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=False, e2e=False, steps=None,
              warmup=None):
     steps = steps or args.steps
     warmup = warmup or args.warmup
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
     T, B, C, p = wl["T"], wl["B"], wl["C"], wl["p"]
-    x, y = synth.make_inputs(net, T, B, seed=1 + 1000 * rank)
+    x, y = cached_inputs(net, T, B, seed=1 + 1000 * rank)
     W = synth.make_weights(net)
     m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, global_batch=B * world)
     m.set_weights(W)
@@ -348,6 +363,39 @@ def run_ours(args):
                 except Exception as e:  # noqa: BLE001
                     row[mode] = {"error": str(e)[:160]}
             t_sweep[str(T)] = row
+    # the other BASELINE.json configs at N GPUs (per-GPU batch fixed): cfg 3 VGG-11, cfg 4 ResNet-DVS
+    other = {}
+    if not args.no_compare and args.workloads:
+        for name in [w for w in args.workloads.split(",") if w]:
+            w2 = synth.workload(name)
+            net2 = synth.net_config(w2["net"])
+            row = {"net": describe(net2), "T": w2["T"], "per_gpu_batch": w2["B"], "C": w2["C"], "p": w2["p"]}
+            for mode in ("skip", "ckpt", "full"):
+                try:
+                    r = run_mode(torch, dist, args, w2, net2, mode, rank, world, local_rank, steps=5, warmup=3)
+                    row[mode] = {"samples_per_s": w2["B"] * world * 5 / (r["total_ms"] / 1e3),
+                                 "ms_per_step": r["total_ms"] / 5, "peak_hbm_gb": r["peak_lib"] / 1e9,
+                                 "kept_fraction": r["kept_fraction"]}
+                except Exception as e:  # noqa: BLE001
+                    row[mode] = {"error": str(e)[:160]}
+            other[name] = row
+    # cfg 5: VGG-11 T sweep at per-GPU B = 128, C = 5, p = 50 (Fig. 14 setting): throughput and peak HBM
+    # per mode; FULL stops fitting in HBM as T grows (reported as its allocation error)
+    sweep11 = {}
+    if not args.no_compare and args.t_sweep_vgg11:
+        w5 = synth.workload("cfg3_vgg11")
+        net5 = synth.net_config(w5["net"])
+        for T in [int(v) for v in args.t_sweep_vgg11.split(",") if v]:
+            w2 = dict(w5, T=T, C=5)
+            row = {}
+            for mode in ("skip", "ckpt", "full"):
+                try:
+                    r = run_mode(torch, dist, args, w2, net5, mode, rank, world, local_rank, steps=3, warmup=3)
+                    row[mode] = {"samples_per_s": w2["B"] * world * 3 / (r["total_ms"] / 1e3),
+                                 "peak_hbm_gb": r["peak_lib"] / 1e9}
+                except Exception as e:  # noqa: BLE001
+                    row[mode] = {"error": str(e)[:120]}
+            sweep11[str(T)] = row
     if rank != 0:
         if world > 1:
             dist.barrier()
@@ -363,6 +411,10 @@ def run_ours(args):
     cfg["compare"] = compare
     if t_sweep:
         cfg["t_sweep"] = t_sweep
+    if other:
+        cfg["other_workloads"] = other
+    if sweep11:
+        cfg["t_sweep_vgg11_cfg5"] = sweep11
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": main["total_ms"] / args.steps, "higher_is_better": True,
@@ -402,6 +454,10 @@ def main():
     ap.add_argument("--no-compare", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--t-sweep", default="50,200,400", help="extra T values for peak-HBM / throughput vs T")
+    ap.add_argument("--workloads", default="cfg3_vgg11,cfg4_resnet_dvs",
+                    help="other BASELINE.json configs measured briefly in the same run (config.other_workloads)")
+    ap.add_argument("--t-sweep-vgg11", default="100,500,1000,2000",
+                    help="cfg 5: VGG-11 T values (B=128, C=5, p=50), all three modes")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

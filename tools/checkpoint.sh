@@ -8,7 +8,7 @@ timeout 900 python -m pytest tests -m gpu -q > $o/pytest_gpu.log 2>&1; tail -2 $
 timeout 600 python bench.py > $o/bench.json 2> $o/bench.err; tail -c 600 $o/bench.json
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > $o/bench_ref.json 2> $o/bench_ref.err; tail -c 300 $o/bench_ref.json
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file $o/launches.csv \
-    python bench.py --steps 2 --warmup 3 --no-compare --no-cpu-baseline --t-sweep "" > /dev/null 2>&1
+    python bench.py --steps 2 --warmup 3 --no-compare --no-cpu-baseline --t-sweep "" --workloads "" --t-sweep-vgg11 "" > /dev/null 2>&1
 python tools/launches.py $o/launches.csv > $o/launches.txt 2>&1; head -30 $o/launches.txt
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"conv_lif_kernel|gemm_tc_kernel|layer0_fwd|lif_bwd_kernel" -s 30 -c 8 \
     -o $o/full python tools/prof_step.py --steps 2 > $o/ncu_full.log 2>&1; tail -2 $o/ncu_full.log
