@@ -147,7 +147,8 @@ size_t skipper_weight_count(const skipper_ctx *ctx, int layer);
 skipper_status skipper_forward_segment(skipper_ctx *ctx, int seg, int pass,
                                        const unsigned char *x_dev, const int *labels_dev);
 skipper_status skipper_backward_segment(skipper_ctx *ctx, int seg);
-/* Allreduce dW over ranks (if skipper_comm_init was called) and apply Adam. */
+/* Join the dW allreduce (issued in buckets during backward_segment(0) when skipper_comm_init was
+ * called) and apply Adam. */
 skipper_status skipper_optimizer_step(skipper_ctx *ctx);
 
 /* One full training iteration on device-resident inputs.  loss_host may be NULL
@@ -160,9 +161,21 @@ skipper_status skipper_step(skipper_ctx *ctx, const unsigned char *x_dev, const 
 skipper_status skipper_step_host(skipper_ctx *ctx, const unsigned char *x_host, const int *labels_host,
                                  float *loss_host);
 
-/* ---- data parallelism (batch-sharded) ---------- */
+/* ---- data parallelism (batch-sharded) ----------
+ * comm_unique_id: rank 0 creates the NCCL id; the caller broadcasts it.  comm_init: every rank joins
+ * the library-owned communicator (world == 1 builds a one-rank communicator: the same schedule runs and
+ * the collectives are identities).  With a communicator, the per-layer spike counts are allreduced
+ * (int64) before Eq.5 so every rank computes the same keep mask, and dW is allreduced (fp32 sum) in
+ * layer buckets of SKIPPER_BUCKET_MB (default 25) on a dedicated stream as soon as segment 0's weight
+ * gradients of the bucket's layers have run, overlapping the rest of the backward.  ENCCL on failure
+ * (the context is then poisoned). */
 skipper_status skipper_comm_unique_id(unsigned char id_out[128]);
 skipper_status skipper_comm_init(skipper_ctx *ctx, const unsigned char id[128], int rank, int world);
+/* The bucket plan (host only): walking spiking layers n_spiking-1 .. 1, closes[i] = 1 where a bucket of
+ * >= bucket_bytes of fp32 gradients ends (layer 1 always ends the last one; layer 0 and the readout go
+ * after segment 0).  Returns the number of buckets, or -1 for null pointers or n_spiking < 1. */
+int skipper_plan_buckets(const unsigned long long *wcount, int n_spiking, unsigned long long bucket_bytes,
+                         int *closes);
 
 /* ---- introspection (host sync) ----------------------------------------------- */
 skipper_status skipper_get_loss(skipper_ctx *ctx, float *loss_host);

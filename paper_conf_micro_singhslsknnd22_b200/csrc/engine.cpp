@@ -148,8 +148,14 @@ struct skipper_ctx {
     size_t cur_bytes = 0, peak_bytes = 0;
     std::string err;
     bool poisoned = false;
-    // comm
+    // comm: one NCCL communicator (K5).  The dW allreduce runs in layer buckets on st3 while segment 0's
+    // backward continues (a bucket of layers hi..lo is final once lo's weight gradient has run in
+    // segment 0); layer 0 (unpadded at the end) and the readout follow on the same stream.
     sk::Comm comm;
+    cudaStream_t st3 = nullptr;
+    cudaEvent_t ev_w = nullptr, ev_comm = nullptr;
+    std::vector<int> bucket_lo;   // per spiking layer i >= 1: 1 if layer i closes a bucket
+    bool comm_pending = false;
     std::unordered_map<PlanKey, sk::GemmLaunch, PlanKeyHash> plans;
     // profiling (per kernel class: launches, device ms, algorithmic bytes and flops)
     bool prof_on = false;
@@ -729,6 +735,12 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         if (c->ev_ready[k]) cudaEventDestroy(c->ev_ready[k]);
         if (c->ev_done[k]) cudaEventDestroy(c->ev_done[k]);
     }
+    if (c->st3) {
+        cudaStreamSynchronize(c->st3);
+        cudaStreamDestroy(c->st3);
+    }
+    if (c->ev_w) cudaEventDestroy(c->ev_w);
+    if (c->ev_comm) cudaEventDestroy(c->ev_comm);
     c->comm.destroy();
     delete c;
 }
@@ -1221,7 +1233,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
 }
 
 static skipper_status comm_allreduce_s(skipper_ctx *c) {
-    if (c->comm.world > 1) {
+    if (c->comm.comm) {
         std::string e;
         if (!c->comm.allreduce_i64(c->s_dev, (c->Ls + 1) * c->T, c->st, &e))  // per-layer counts
             return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
@@ -1353,7 +1365,41 @@ static skipper_status join_wgrads(skipper_ctx *c) {
 
 static long long rcv_neurons(const skipper_ctx *c, int i) { return i >= 0 ? c->L[i].N : 0; }
 
-static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
+// Bucket plan for the overlapped dW allreduce: walking the spiking layers i = Ls-1 .. 1 (the order their
+// final weight gradients appear in segment 0), close a bucket once it holds >= bucket_bytes; returns the
+// 0/1 "closes a bucket" flags indexed by layer (layer 1 always closes the last one).
+extern "C" int skipper_plan_buckets(const unsigned long long *wcount, int n_spiking, unsigned long long bucket_bytes,
+                                    int *closes) {
+    if (!wcount || !closes || n_spiking < 1) return -1;
+    unsigned long long acc = 0;
+    int nb = 0;
+    for (int i = 0; i < n_spiking; ++i) closes[i] = 0;
+    for (int i = n_spiking - 1; i >= 1; --i) {
+        acc += wcount[i] * 4ULL;
+        if (acc >= bucket_bytes || i == 1) {
+            closes[i] = 1;
+            acc = 0;
+            ++nb;
+        }
+    }
+    return nb;
+}
+
+// segment 0 only: layer i's weight gradient has been issued on `ws`; launch the bucket it closes
+static skipper_status comm_after_wgrad(skipper_ctx *c, int i, cudaStream_t ws) {
+    if (!c->comm.comm || i < 1 || !c->bucket_lo[i]) return SKIPPER_OK;
+    int hi = i;
+    while (hi + 1 < c->Ls && !c->bucket_lo[hi + 1]) ++hi;
+    CK(cudaEventRecord(c->ev_w, ws));  // ws is in order: every wgrad of layers hi..i precedes this
+    CK(cudaStreamWaitEvent(c->st3, c->ev_w, 0));
+    const size_t cnt = (size_t)(c->L[hi].dw - c->L[i].dw) + c->L[hi].wcount;
+    std::string e;
+    if (!c->comm.allreduce_f32(c->L[i].dw, cnt, c->st3, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    c->comm_pending = true;
+    return SKIPPER_OK;
+}
+
+static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, bool last_seg) {
     for (int i = c->Ls - 1; i >= 0; --i) {
         Layer &l = c->L[i];
         if (i == 0 && c->l0_bwd_fused) {  // reverse scan + weight gradient in one kernel, no delta in HBM
@@ -1451,6 +1497,7 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
                 CK(cudaEventRecord(c->ev_done[par], c->st2));
                 c->w_pending[par] = true;
             }
+            if (last_seg) CKS(comm_after_wgrad(c, i, ws));
         } else if (i == 0 && c->in_kind == 1)
             ok = get_plan(c, {2, dcur, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
                           [&](sk::GemmLaunch *p) {
@@ -1469,12 +1516,14 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t) {
             // issued above
         } else if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
             CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw));
+            if (last_seg) CKS(comm_after_wgrad(c, i, c->st));
         } else {   // weight gradient on the side stream, after this layer's delta is written
             CK(cudaEventRecord(c->ev_ready[par], c->st));
             CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
             CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw, c->st2));
             CK(cudaEventRecord(c->ev_done[par], c->st2));
             c->w_pending[par] = true;
+            if (last_seg) CKS(comm_after_wgrad(c, i, c->st2));
         }
         if (i > 0 && l.icol) {  // per chunk: dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
             const long long ch = icol_chunk(c);
@@ -1573,7 +1622,7 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
     const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
     const int R = full ? c->T : (int)c->kept[seg].size();
     const int *row_t = full ? nullptr : c->kept_dev + (size_t)seg * c->S;
-    CKS(backward_rows(c, R, row_t));
+    CKS(backward_rows(c, R, row_t, seg == 0));
     if (seg == 0) {
         const Layer &last = c->L[c->Ls - 1];
         const Layer &ro = c->L.back();
@@ -1594,6 +1643,15 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
             D = ro.Cin;
         }
         CK(sk::launch_readout_wgrad(c->dz, cin, ro.dw, c->B, D, ro.Cout, 1.0f / c->T, c->st));
+        if (c->comm.comm) {  // the last buckets: layer 0 (final after the unpad above) and the readout
+            CK(cudaEventRecord(c->ev_w, c->st));
+            CK(cudaStreamWaitEvent(c->st3, c->ev_w, 0));
+            std::string e;
+            if (!c->comm.allreduce_f32(l0.dw, l0.wcount, c->st3, &e) ||
+                !c->comm.allreduce_f32(ro.dw, ro.wcount, c->st3, &e))
+                return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+            c->comm_pending = true;
+        }
         if (c->cfg.debug_record && full)
             for (int i = 0; i < c->Ls; ++i) {
                 const size_t bn = (size_t)c->B * c->L[i].N * c->T;
@@ -1614,9 +1672,10 @@ extern "C" skipper_status skipper_optimizer_step(skipper_ctx *c) {
     CKS(check_ctx(c));
     if (c->phase != PH_BWD_DONE || !c->grads_ready)
         return fail(c, SKIPPER_EORDER, "optimizer_step needs a completed backward");
-    if (c->comm.world > 1) {
-        std::string e;
-        if (!c->comm.allreduce_f32(c->dw_all, c->dw_total, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    if (c->comm_pending) {  // the bucketed dW allreduce issued during segment 0's backward
+        CK(cudaEventRecord(c->ev_comm, c->st3));
+        CK(cudaStreamWaitEvent(c->st, c->ev_comm, 0));
+        c->comm_pending = false;
     }
     c->adam_step += 1;
     const double b1 = c->cfg.beta1, b2 = c->cfg.beta2;
@@ -1781,9 +1840,22 @@ extern "C" skipper_status skipper_comm_unique_id(unsigned char id_out[128]) {
 extern "C" skipper_status skipper_comm_init(skipper_ctx *c, const unsigned char id[128], int rank, int world) {
     CKS(check_ctx(c));
     if (world < 1 || rank < 0 || rank >= world) return fail(c, SKIPPER_EINVAL, "bad rank/world");
-    if (world == 1) return SKIPPER_OK;
+    // world == 1 also builds a (one-rank) communicator: the bucketed path then runs as an identity
     std::string e;
     if (!c->comm.init(id, rank, world, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    if (!c->st3 && cudaStreamCreateWithFlags(&c->st3, cudaStreamNonBlocking) != cudaSuccess)
+        return fail(c, SKIPPER_ECUDA, "comm stream creation failed");
+    if ((!c->ev_w && cudaEventCreateWithFlags(&c->ev_w, cudaEventDisableTiming) != cudaSuccess) ||
+        (!c->ev_comm && cudaEventCreateWithFlags(&c->ev_comm, cudaEventDisableTiming) != cudaSuccess))
+        return fail(c, SKIPPER_ECUDA, "comm event creation failed");
+    std::vector<unsigned long long> wc(c->Ls);
+    for (int i = 0; i < c->Ls; ++i) wc[i] = c->L[i].wcount;
+    c->bucket_lo.assign(c->Ls, 0);
+    static const unsigned long long kBucket = [] {
+        const char *b = getenv("SKIPPER_BUCKET_MB");
+        return (unsigned long long)(b ? std::max(1, atoi(b)) : 25) << 20;
+    }();
+    skipper_plan_buckets(wc.data(), c->Ls, kBucket, c->bucket_lo.data());
     return SKIPPER_OK;
 }
 

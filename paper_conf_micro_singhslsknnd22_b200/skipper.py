@@ -99,6 +99,7 @@ def _load():
         "skipper_profile_class_name": (ct.c_char_p, [I]),
         "skipper_profile_num_classes": (I, []),
         "skipper_launch_count": (ct.c_longlong, [P]),
+        "skipper_plan_buckets": (I, [P, I, ct.c_ulonglong, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -140,6 +141,14 @@ def sst_host(values, p):
     """Eq.5 for one segment as implemented in the library (host code)."""
     a = np.ascontiguousarray(values, dtype=np.int64)
     return lib.skipper_sst_host(a.ctypes.data, a.size, float(p))
+
+
+def plan_buckets(wcounts, bucket_bytes):
+    """The library's dW-allreduce bucket plan: closes[i] = 1 where a bucket (walking layers n-1 .. 1) ends."""
+    wc = np.ascontiguousarray(wcounts, dtype=np.uint64)
+    closes = np.zeros(len(wc), dtype=np.int32)
+    nb = lib.skipper_plan_buckets(wc.ctypes.data, len(wc), int(bucket_bytes), closes.ctypes.data)
+    return nb, closes
 
 
 def workspace_bytes(net, cfg: Config, kept_max=-1):

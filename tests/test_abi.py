@@ -99,3 +99,35 @@ def test_status_strings_and_build_info():
     assert sk.lib.skipper_status_string(0) == b"ok"
     assert sk.lib.skipper_status_string(5) == b"call order violation"
     assert b"sm_100a" in sk.lib.skipper_build_info()
+
+
+def buckets_from_plan(closes):
+    """Layer ranges [lo, hi] of the buckets, in the order the library launches them (top layer first)."""
+    out, hi = [], len(closes) - 1
+    for i in range(len(closes) - 1, 0, -1):
+        if closes[i]:
+            out.append((i, hi))
+            hi = i - 1
+    return out
+
+
+@pytest.mark.parametrize("name", ["vgg5", "vgg11", "resnet20_dvs", "fc784", "tiny_fc"])
+@pytest.mark.parametrize("mb", [1, 25, 1000])
+def test_bucket_plan_partitions_layers(name, mb):
+    """K5 bucket plan: every spiking layer >= 1 in exactly one contiguous bucket, each
+    bucket but the last at least bucket_bytes, launched top-down (the order segment 0 finalises dW)."""
+    net = synth.net_config(name)
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    from synth.inputs import weight_shape
+    wc = [int(np.prod(weight_shape(L))) for L in spk]
+    nb, closes = sk.plan_buckets(wc, mb << 20)
+    if len(spk) == 1:
+        assert nb == 0 and not closes.any()
+        return
+    b = buckets_from_plan(closes)
+    assert nb == len(b) and b[-1][0] == 1 and b[0][1] == len(spk) - 1
+    covered = sorted(i for lo, hi in b for i in range(lo, hi + 1))
+    assert covered == list(range(1, len(spk)))
+    for lo, hi in b[:-1]:
+        assert 4 * sum(wc[lo:hi + 1]) >= mb << 20
+        assert 4 * sum(wc[lo + 1:hi + 1]) < mb << 20      # closed as soon as it was full

@@ -217,3 +217,31 @@ def test_resnet20_dvs_reduced(mode):
     """cfg 4 topology (ResNet-20 SNN on 2x128x128 DVS frames) at reduced T and B: 19 spiking layers of
     every conv kind (im2col 16/32 channels, stride 2, implicit 64-channel, fused conv+LIF), 9 shortcuts."""
     check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode=mode, deep=True)
+
+
+@pytest.mark.parametrize("name,T,C", [("vgg5", 14, 2), ("tiny_resnet", 16, 2)])
+def test_one_rank_nccl_bucketed_allreduce(name, T, C, monkeypatch):
+    """K5 on the device: with a (one-rank) NCCL communicator the s allreduce and the bucketed dW
+    allreduce on the comm stream run inside the step; the collectives are identities, so the
+    gradients and post-Adam weights equal the communicator-free run."""
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    monkeypatch.setenv("SKIPPER_BUCKET_MB", "1")        # several buckets even for small nets
+    net = synth.net_config(name)
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, T, 2)
+    xd, yd = torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda()
+    out = []
+    for comm in (False, True):
+        m = SkipperNet(net, T, C=C, p=50.0, mode="skip", batch=2)
+        m.set_weights(W)
+        if comm:
+            m.comm_init(SkipperNet.comm_unique_id(), 0, 1)
+        loss = m.step(xd, yd)
+        out.append((loss, [g.cpu() for g in m.grads()], [w.cpu() for w in m.weights()], m.keep_mask()))
+        m.close()
+    assert out[0][0] == out[1][0]
+    np.testing.assert_array_equal(out[0][3], out[1][3])
+    for a, b in zip(out[0][1], out[1][1]):
+        assert (a.double() - b.double()).norm() <= 1e-6 * b.double().norm() + 1e-12   # split-K atomics order
+    for a, b in zip(out[0][2], out[1][2]):
+        np.testing.assert_allclose(a.numpy(), b.numpy(), rtol=0, atol=1e-6)

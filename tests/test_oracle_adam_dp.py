@@ -72,3 +72,62 @@ def test_data_parallel_sharding_gloo():
     assert loss == pytest.approx(ref.loss, rel=1e-12)
     for a, b in zip(grads, ref.dW):
         np.testing.assert_allclose(a, b, rtol=1e-10, atol=1e-14)
+
+
+def _dp_bucket_worker(rank, world, port, out):
+    """The library's K5 schedule on the host: s allreduced before Eq.5, then dW allreduced in the
+    library's layer buckets (flat, top-down), layer 0 and the readout last."""
+    from paper_conf_micro_singhslsknnd22_b200 import skipper as sk
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    net = synth.net_config("tiny_resnet")
+    W = synth.make_weights(net)
+    T, B = 16, 4
+    x, y = synth.make_inputs(net, T, B)
+    shard = slice(rank * B // world, (rank + 1) * B // world)
+    r0 = train_step(net, W, x[:, shard], y[shard], StepConfig(T=T, C=2, mode="ckpt", global_batch=B))
+    s = torch.tensor(r0.s)
+    dist.all_reduce(s)
+    r = train_step(net, W, x[:, shard], y[shard], StepConfig(T=T, C=2, mode="skip", p=50.0, global_batch=B,
+                                                             s_global=s.numpy()))
+    Ls = len(r.dW) - 1
+    nb, closes = sk.plan_buckets([w.size for w in W[:Ls]], 8 << 10)   # small buckets: several of them
+    grads = [torch.tensor(g) for g in r.dW]
+    hi = Ls - 1
+    for i in range(Ls - 1, 0, -1):
+        if closes[i]:
+            flat = torch.cat([grads[j].flatten() for j in range(i, hi + 1)])
+            dist.all_reduce(flat)
+            off = 0
+            for j in range(i, hi + 1):
+                n = grads[j].numel()
+                grads[j] = flat[off:off + n].reshape(grads[j].shape)
+                off += n
+            hi = i - 1
+    for j in (0, Ls):
+        dist.all_reduce(grads[j])
+    if rank == 0:
+        out.put((nb, [g.numpy() for g in grads], r.keep.copy()))
+    dist.destroy_process_group()
+
+
+def test_data_parallel_bucketed_allreduce_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 30500 + os.getpid() % 1000
+    procs = [ctx.Process(target=_dp_bucket_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    nb, grads, keep = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert nb >= 2
+    net = synth.net_config("tiny_resnet")
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, 16, 4)
+    ref = train_step(net, W, x, y, StepConfig(T=16, C=2, mode="skip", p=50.0))
+    np.testing.assert_array_equal(keep, ref.keep)
+    for a, b in zip(grads, ref.dW):
+        np.testing.assert_allclose(a, b, rtol=1e-10, atol=1e-14)
