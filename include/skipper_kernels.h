@@ -32,6 +32,13 @@ int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, floa
                          int nb, int h, int w, int cin, int cout, void *stream);
 int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float *dW,
                          int nb, int h, int w, int cin, int cout, int accumulate, void *stream);
+/* Strided / narrow-channel implicit conv (ResNet layers, reading 8):
+ *   Y[nb,y,x,co] = sum_{dy,dx,ci} Wk[co][dy*3+dx][ci] X[nb, s*y+dy-1, s*x+dx-1, ci]   (pad 1, stride s)
+ * h x w is the OUTPUT size, X is [nb][s*h][s*w][cin]; cin in {16, 32} (one 32B/64B-swizzled TMA box per
+ * tap) or a multiple of 64; s in {1, 2} (TMA element strides).  With sign = -1 (stride 1 only) it is the
+ * dgrad of conv_dgrad above (X = D, Wk = Wt, cin = the layer's cout).  EUNSUPPORTED otherwise. */
+int skipper_k_conv_s(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w, int cin,
+                     int cout, int sign, int stride, void *stream);
 
 /* Fused 3x3 convolution + LIF over R timestep rows (Eq.1): for r = 0..R-1
  *   I_r = conv_fwd(X_r, Wk)  (bf16 x bf16 -> fp32, tensor cores, never written to memory)

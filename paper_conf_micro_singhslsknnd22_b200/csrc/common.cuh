@@ -149,6 +149,16 @@ SK_DEV uint64_t umma_desc_sw128(uint32_t saddr, uint32_t lbo_bytes, uint32_t sbo
     d |= (uint64_t)2 << 61;  // SWIZZLE_128B
     return d;
 }
+// K-major smem descriptor with a runtime swizzle (layout code: 2 = 128B, 4 = 64B, 6 = 32B); sbo = 8 rows
+SK_DEV uint64_t umma_desc_kmajor(uint32_t saddr, uint32_t sbo_bytes, uint32_t layout) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+    d |= (uint64_t)1 << 16;  // LBO (unused for swizzled K-major)
+    d |= (uint64_t)((sbo_bytes >> 4) & 0x3FFF) << 32;
+    d |= (uint64_t)1 << 46;
+    d |= (uint64_t)(layout & 7) << 61;
+    return d;
+}
 // instruction descriptor, kind::f16: D fp32, A/B bf16, majors, N, M
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(uint32_t M, uint32_t N, uint32_t a_mn_major, uint32_t b_mn_major) {
     return (1u << 4)            // D format: F32

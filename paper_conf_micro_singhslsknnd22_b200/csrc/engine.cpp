@@ -1959,6 +1959,13 @@ extern "C" int skipper_k_conv_wgrad(const unsigned short *D, const unsigned shor
     return kapi_run(g, ok, stream, "conv_wgrad");
 }
 
+extern "C" int skipper_k_conv_s(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w,
+                                int cin, int cout, int sign, int stride, void *stream) {
+    sk::GemmLaunch g;
+    const bool ok = sk::plan_conv_s(&g, X, Wk, Y, nb, h, w, cin, cout, sign, stride);
+    return kapi_run(g, ok, stream, "conv_s");
+}
+
 extern "C" int skipper_k_num_sms(void) { return sk::device_num_sms(); }
 
 // ------------------------------------------------------------------------------------ profiling API

@@ -38,6 +38,12 @@ struct GemmDev {
     int M, N;           // valid output extent (rows, columns of one tap block)
     int store_mode;
     unsigned long long *stats;  // optional pipeline wait statistics (null in production)
+    // narrow / strided implicit conv (plan_conv_s): K elements per K block (16 or 32 = one tap of a
+    // 16/32-channel image, 32B/64B-swizzled boxes; 0 = the 64-element 128B-swizzled default), the conv
+    // stride (TMA element strides) and the bytes one pipeline stage receives
+    int kblk;
+    int conv_stride;
+    uint32_t stage_tx;
 };
 
 struct GemmLaunch {
@@ -63,6 +69,11 @@ bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M
 // dgrad: G[nb,h,w,cin] from D[nb,h,w,cout] and Wt[cin][9][cout]
 bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
                int sign);
+// conv forward / dgrad with stride (1 or 2) and narrow channels (cin in {16, 32} or a multiple of 64):
+// Y[nb, h, w, cout] (h x w = OUTPUT size) from X[nb, s*h, s*w, cin]; pixels on M, non-transposed.
+// dgrad of a stride-1 conv: sign = -1 with D as X and Wt [cin][9][cout] as Wk (as plan_conv).
+bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
+                 int sign, int stride);
 // conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
                      int num_sms);

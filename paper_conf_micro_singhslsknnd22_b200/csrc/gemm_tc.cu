@@ -151,7 +151,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                     const uint32_t sb = sa + Cfg::A_BYTES;
                     const uint32_t fb = full_bar(stage);
-                    mbar_expect_tx(fb, Cfg::STAGE_BYTES);
+                    mbar_expect_tx(fb, g.kblk ? g.stage_tx : Cfg::STAGE_BYTES);
+                    const int kbe = g.kblk ? g.kblk : BK;  // K elements per block
                     // ---- A
                     if (g.a_kind == OP_K2D) {
                         tma_load_2d(sa, &ta, fb, kb * BK, tc.m_t * BM);
@@ -161,7 +162,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         const int m0 = tc.m_t * BM;
                         const int n0 = m0 / g.conv_hw;
                         const int y0 = (m0 % g.conv_hw) / g.conv_w;
-                        tma_load_4d(sa, &ta, fb, cblk * BK, g.conv_sign * dx, y0 + g.conv_sign * dy, n0);
+                        if (g.kblk)  // strided / narrow: input rows s*y0 + dy, element strides in the map
+                            tma_load_4d(sa, &ta, fb, cblk * kbe, g.conv_sign * dx,
+                                        g.conv_stride * y0 + g.conv_sign * dy, n0);
+                        else
+                            tma_load_4d(sa, &ta, fb, cblk * BK, g.conv_sign * dx, y0 + g.conv_sign * dy, n0);
                     } else {  // OP_MN2D: two 64-wide MN chunks
                         tma_load_2d(sa, &ta, fb, tc.m_t * BM, kb * BK);
                         tma_load_2d(sa + 8192u, &ta, fb, tc.m_t * BM + 64, kb * BK);
@@ -172,7 +177,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         tma_load_2d_mc(sb + (uint32_t)rank * SL * 128u, &tb, fb, kb * BK, tc.n_t * BN + rank * (int)SL,
                                        mc_mask);
                     } else if (g.b_kind == OP_K2D) {
-                        tma_load_2d(sb, &tb, fb, kb * BK, tc.n_t * BN);
+                        tma_load_2d(sb, &tb, fb, kb * kbe, tc.n_t * BN);
                     } else if (g.b_kind == OP_MN2D) {
 #pragma unroll
                         for (int i = 0; i < BN / 64; ++i)
@@ -231,6 +236,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                     tc_fence_after();
                     const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
                     const uint32_t sb = sa + Cfg::A_BYTES;
+                    if (!MN && g.kblk) {  // narrow K block: 16/32 elements, 32B/64B swizzle atoms
+                        const uint32_t rowb = (uint32_t)g.kblk * 2u, lay = g.kblk == 16 ? 6u : (g.kblk == 32 ? 4u : 2u);
+                        for (int k = 0; k < g.kblk / 16; ++k) {
+                            const uint64_t ad = umma_desc_kmajor(sa + k * 32u, 8u * rowb, lay);
+                            const uint64_t bd = umma_desc_kmajor(sb + k * 32u, 8u * rowb, lay);
+                            tc_mma_f16(d_tmem, ad, bd, idesc, (kb > tc.kb0 || k > 0) ? 1u : 0u);
+                        }
+                        tc_commit(empty_bar(stage));
+                        if (++stage == STAGES) {
+                            stage = 0;
+                            phase ^= 1u;
+                        }
+                        continue;
+                    }
 #pragma unroll
                     for (int k = 0; k < BK / 16; ++k) {
                         uint64_t ad, bd;
@@ -394,6 +413,40 @@ bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// 4D NHWC map with a box of `cin_box` channels (32/64/128 bytes -> matching swizzle) and element strides
+static bool make_map_conv_s(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint64_t H, uint64_t NB,
+                            uint32_t cin_box, uint32_t box_w, uint32_t box_h, uint32_t box_n, uint32_t stride) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    if ((C * 2) % 16 != 0 || (reinterpret_cast<uintptr_t>(ptr) & 15)) return false;
+    cuuint64_t dims[4] = {C, W, H, NB};
+    cuuint64_t strides[3] = {C * 2, W * C * 2, H * W * C * 2};
+    cuuint32_t box[4] = {cin_box, box_w * stride, box_h * stride, box_n};
+    cuuint32_t es[4] = {1, stride, stride, 1};
+    const CUtensorMapSwizzle sw = cin_box == 16 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                  : cin_box == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B;
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void *>(ptr), dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// 2D K-major map [outer][inner] with a box of `box_inner` elements and the matching swizzle
+static bool make_map_2d_sw(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer, uint32_t box_inner,
+                           uint32_t box_outer) {
+    auto fn = encode_fn();
+    if (!fn) return false;
+    if ((inner * 2) % 16 != 0 || (reinterpret_cast<uintptr_t>(ptr) & 15)) return false;
+    cuuint64_t dims[2] = {inner, outer};
+    cuuint64_t strides[1] = {inner * 2};
+    cuuint32_t box[2] = {box_inner, box_outer};
+    cuuint32_t es[2] = {1, 1};
+    const CUtensorMapSwizzle sw = box_inner == 16 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                  : box_inner == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B;
+    return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 static int pick_bn(int N) { return N <= 64 ? 64 : (N <= 128 ? 128 : 256); }
 
 // Cluster size for B multicast (K-major, unsplit GEMMs with enough M tiles).  SKIPPER_GEMM_CS
@@ -549,6 +602,52 @@ bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, i
     g->cs = pick_cs(d);
     return make_map_conv(&g->ta, X, cin, w, h, nb, bw, bh, bnn) && make_map_2d(&g->tb, Wk, 9ull * cin, cout, BK, g->bn / g->cs) &&
            make_map_out(&g->tc, Y, cout, 1, M, cout, cout);
+}
+
+bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
+                 int sign, int stride) {
+    if (cout % 8 || (stride != 1 && stride != 2) || (sign == -1 && stride != 1)) return false;
+    int kblk, cb;
+    if (cin == 16 || cin == 32) {
+        kblk = cin;
+        cb = 1;
+    } else if (cin % 64 == 0) {
+        kblk = 64;
+        cb = cin / 64;
+    } else {
+        return false;
+    }
+    uint32_t bw, bh, bnn;
+    if (!conv_box(h, w, BM, &bw, &bh, &bnn)) return false;
+    if (bw * stride > 256 || bh * stride > 256) return false;
+    const long long M = (long long)nb * h * w;
+    GemmDev &d = g->d;
+    d = GemmDev{};
+    g->bn = pick_bn(cout);
+    g->mn_major = 0;
+    g->cs = 1;
+    d.m_tiles = cdiv(M, BM);
+    d.n_tiles = cdiv(cout, g->bn);
+    d.taps = 1;
+    d.splits = 1;
+    d.conv_cb = cb;
+    d.num_kb = 9 * cb;
+    d.kb_per_split = d.num_kb;
+    d.a_kind = OP_KCONV;
+    d.b_kind = OP_K2D;
+    d.conv_hw = h * w;
+    d.conv_w = w;
+    d.conv_sign = sign;
+    d.conv_stride = stride;
+    d.kblk = kblk;
+    d.stage_tx = (uint32_t)(BM + g->bn) * kblk * 2;
+    d.C = Y;
+    d.ldc = cout;
+    d.M = (int)M;
+    d.N = cout;
+    d.store_mode = STORE_OVERWRITE;
+    return make_map_conv_s(&g->ta, X, cin, (uint64_t)w * stride, (uint64_t)h * stride, nb, kblk, bw, bh, bnn, stride) &&
+           make_map_2d_sw(&g->tb, Wk, 9ull * cin, cout, kblk, g->bn) && make_map_out(&g->tc, Y, cout, 1, M, cout, cout);
 }
 
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,

@@ -166,3 +166,36 @@ def test_conv_lif_exact(R, nb, h, w, cin, cout, pool, variant, monkeypatch):
         assert torch.equal(Uo[r].cpu(), refU[r]), f"row {r}: U max diff {(Uo[r].cpu() - refU[r]).abs().max()}"
     assert torch.equal(Us.cpu(), refU[-1])
     assert torch.equal(os_.cpu(), (refU[-1] > theta).to(torch.uint8))
+
+
+CONV_S_SHAPES = [  # nb, output h, w, cin, cout, stride  (ResNet-DVS layers and ragged / multi-image tiles)
+    (3, 64, 64, 16, 16, 1), (2, 32, 32, 16, 32, 2), (2, 32, 32, 32, 32, 1), (2, 16, 16, 32, 64, 2),
+    (3, 8, 8, 16, 16, 1), (5, 4, 4, 16, 32, 2), (3, 16, 16, 64, 64, 2), (2, 8, 8, 32, 16, 1)]
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout,stride", CONV_S_SHAPES)
+def test_conv_s_exact(nb, h, w, cin, cout, stride):
+    """Narrow-channel / strided implicit conv (per-tap 32B/64B-swizzled TMA boxes, TMA element strides)
+    against torch conv2d(stride, padding=1) in float64: exact for spikes x grid weights."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_s
+    g = torch.Generator().manual_seed(nb * 131 + h + cin + stride)
+    X = spikes((nb, h * stride, w * stride, cin), gen=g)
+    W = grid((cout, 3, 3, cin), gen=g)
+    ref = F.conv2d(X.permute(0, 3, 1, 2).double(), W.permute(0, 3, 1, 2).double(), padding=1,
+                   stride=stride).permute(0, 2, 3, 1).float()
+    out = k_conv_s(bf16_bits(X).cuda(), bf16_bits(W).cuda(), stride=stride).cpu()
+    assert torch.equal(out, ref), (out - ref).abs().max()
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout", [(3, 64, 64, 16, 16), (2, 32, 32, 32, 32), (2, 8, 8, 32, 16)])
+def test_conv_s_dgrad_exact(nb, h, w, cin, cout):
+    """Stride-1 dgrad through the narrow path: G = conv_transpose(D, W) = conv(D, flipped W^T)."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_conv_s
+    g = torch.Generator().manual_seed(nb + h + cin)
+    D = grid((nb, h, w, cout), e=10, gen=g)
+    W = grid((cout, 3, 3, cin), gen=g)
+    ref = F.conv_transpose2d(D.permute(0, 3, 1, 2).double(), W.permute(0, 3, 1, 2).double(),
+                             padding=1).permute(0, 2, 3, 1).float()
+    Wt = W.permute(3, 1, 2, 0).contiguous()          # [cin][3][3][cout]
+    out = k_conv_s(bf16_bits(D).cuda(), bf16_bits(Wt).cuda(), stride=1, sign=-1).cpu()
+    assert torch.equal(out, ref), (out - ref).abs().max()
