@@ -35,6 +35,7 @@ struct Layer {
     int stride = 1, Hin = 1, Win = 1;  // conv: output (neuron) H x W, input (stride H) x (stride W)
     int res = -1, res_to = -1;          // ResNet: residual source layer (this = receiver) / receiver (this = source)
     bool icol = false;                  // conv via explicit im2col + GEMM (narrow / strided layers)
+    bool fwd_s = false, dgrad_s = false;  // icol layer whose forward / dgrad runs as the narrow implicit conv
     bool gap = false;                   // readout integrates the global average pool (reading 23)
     long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
     size_t wcount = 0;
@@ -455,6 +456,14 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
                 if (l.Cin % 8 || l.Cout % 8)
                     return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: im2col conv needs cin, cout %% 8 == 0", i);
                 l.icol = true;
+                // the strided / narrow implicit conv (gemm_tc.cu plan_conv_s) where its boxes fit
+                auto narrow_ok = [](int ch) { return ch == 16 || ch == 32 || ch % 64 == 0; };
+                const bool tiles = boxok(l.H, l.W, 128) && l.W * l.stride <= 256 &&
+                                   (128 / l.W <= l.H ? 128 / l.W : l.H) * l.stride <= 256;
+                const char *en = getenv("SKIPPER_NO_NARROW_IMPLICIT");
+                const bool allow = !(en && atoi(en));
+                l.fwd_s = allow && tiles && narrow_ok(l.Cin);
+                l.dgrad_s = allow && tiles && l.stride == 1 && narrow_ok(l.Cout);
             }
         } else {
             if (l.Cin % 8 || l.Cout % 8) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: fc needs cin, cout %% 8 == 0", i);
@@ -942,6 +951,10 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
         ok = get_plan(c, {0, in, l.wbp, I, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 1}, g,
                       [&](sk::GemmLaunch *p) { return sk::plan_fc(p, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0); });
+    else if (l.icol && l.fwd_s)  // strided / narrow implicit conv: per-tap TMA boxes, no column buffer
+        ok = get_plan(c, {7, in, l.wb, I, nb, l.Cin, l.Cout, l.H, l.W, l.stride}, g, [&](sk::GemmLaunch *p) {
+            return sk::plan_conv_s(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1, l.stride);
+        });
     else if (l.icol) {  // explicit im2col rows [nb*H*W][9*Cin] x weights [cout][9*Cin], in sample-row chunks
         const long long ch = icol_chunk(c);
         const int K = 9 * l.Cin;
@@ -971,7 +984,7 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
         });
     if (ok && g.d.splits != (l.fc ? fsp : 1)) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: split mismatch", i);
     const double M = (double)nb * l.H * l.W, K = (double)l.Cin * (l.conv ? 9 : 1);
-    const double bytes = (l.icol ? M * K * 2 : (double)nb * l.Nin * 2) + (double)l.wcount * 2 +
+    const double bytes = (double)nb * l.Nin * 2 + (double)l.wcount * 2 +
                          (double)nb * l.N * 4 * (l.fc ? fsp : 1);
     return run_gemm(c, g, ok, "forward", i, K_GEMM_FWD, bytes, 2.0 * M * l.Cout * K);
 }
@@ -1525,7 +1538,14 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             c->w_pending[par] = true;
             if (last_seg) CKS(comm_after_wgrad(c, i, c->st2));
         }
-        if (i > 0 && l.icol) {  // per chunk: dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
+        if (i > 0 && l.icol && l.dgrad_s) {  // stride 1: g = conv(delta, flipped W^T) as a narrow implicit conv
+            ok = get_plan(c, {8, dcur, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_conv_s(p, dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1, 1);
+            });
+            const double M = (double)nb * l.H * l.W;
+            CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD,
+                         (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4, 2.0 * M * l.Cin * 9 * l.Cout));
+        } else if (i > 0 && l.icol) {  // per chunk: dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
             const long long ch = icol_chunk(c);
             const int N = 9 * l.Cin;
             for (long long n0 = 0; n0 < nb; n0 += ch) {
