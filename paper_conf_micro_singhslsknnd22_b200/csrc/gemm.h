@@ -44,6 +44,8 @@ struct GemmDev {
     int kblk;
     int conv_stride;
     uint32_t stage_tx;
+    int ring;               // narrow: smem ring depth (stages of stage_stride bytes)
+    uint32_t stage_stride;
 };
 
 struct GemmLaunch {

@@ -13,6 +13,7 @@
 #include "common.cuh"
 #include "gemm.h"
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <mutex>
@@ -31,7 +32,8 @@ struct GemmCfg {
     static constexpr int STAGES = (BN == 64) ? 8 : (BN == 128 ? 6 : 4);
     static constexpr uint32_t TMEM_COLS = (2 * BN <= 128) ? 128 : (2 * BN <= 256 ? 256 : 512);
     static constexpr uint32_t EPI_BYTES = 4 * 2 * 4096;  // 4 epilogue warps x 2 buffers x (32 x 32 fp32)
-    static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + EPI_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+    static constexpr int MAX_RING = 48;  // narrow K blocks (plan_conv_s) run a deeper ring of smaller stages
+    static constexpr uint32_t SMEM_BYTES = STAGES * STAGE_BYTES + EPI_BYTES + 1024 /*align*/ + 1024 /*barriers*/;
 };
 
 struct TileCoord {
@@ -98,10 +100,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t epi = base + STAGES * Cfg::STAGE_BYTES;  // 1024-aligned (stage bytes are multiples of 1 KB)
     const uint32_t bars = epi + Cfg::EPI_BYTES;
     auto full_bar = [&](int s) { return bars + 8u * s; };
-    auto empty_bar = [&](int s) { return bars + 8u * (STAGES + s); };
-    auto tfull_bar = [&](int a) { return bars + 8u * (2 * STAGES + a); };
-    auto tempty_bar = [&](int a) { return bars + 8u * (2 * STAGES + 2 + a); };
-    const uint32_t tmem_slot = bars + 8u * (2 * STAGES + 4);
+    constexpr int MR = Cfg::MAX_RING;
+    auto empty_bar = [&](int s) { return bars + 8u * (MR + s); };
+    auto tfull_bar = [&](int a) { return bars + 8u * (2 * MR + a); };
+    auto tempty_bar = [&](int a) { return bars + 8u * (2 * MR + 2 + a); };
+    const uint32_t tmem_slot = bars + 8u * (2 * MR + 4);
+    // ring geometry: the compile-time stages, or (narrow K blocks) g.ring stages of g.stage_stride bytes
+    const int nst = g.kblk ? g.ring : STAGES;
+    const uint32_t sstride = g.kblk ? g.stage_stride : Cfg::STAGE_BYTES;
+    const uint32_t a_bytes = g.kblk ? (uint32_t)BM * g.kblk * 2u : Cfg::A_BYTES;
     uint32_t *tmem_slot_ptr = reinterpret_cast<uint32_t *>(smem_raw + (tmem_slot - raw));
 
     const int warp = threadIdx.x >> 5;
@@ -113,7 +120,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         tma_prefetch(&ta);
         tma_prefetch(&tb);
         tma_prefetch(&tcm);
-        for (int s = 0; s < STAGES; ++s) {
+        for (int s = 0; s < nst; ++s) {
             mbar_init(full_bar(s), 1);
             mbar_init(empty_bar(s), CS);  // every CTA of the cluster frees the stage (multicast B)
         }
@@ -148,8 +155,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 const int tdy = tc.tap / 3 - 1, tdx = tc.tap % 3 - 1;
                 for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
                     mbar_wait_t(empty_bar(stage), phase ^ 1u, wst);
-                    const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
-                    const uint32_t sb = sa + Cfg::A_BYTES;
+                    const uint32_t sa = base + stage * sstride;
+                    const uint32_t sb = sa + a_bytes;
                     const uint32_t fb = full_bar(stage);
                     mbar_expect_tx(fb, g.kblk ? g.stage_tx : Cfg::STAGE_BYTES);
                     const int kbe = g.kblk ? g.kblk : BK;  // K elements per block
@@ -205,7 +212,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                             tma_load_4d(sb + 8192u * i, &tb, fb, ci0, ddx, y0 + ddy, n0);
                         }
                     }
-                    if (++stage == STAGES) {
+                    if (++stage == nst) {
                         stage = 0;
                         phase ^= 1u;
                     }
@@ -234,8 +241,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         mbar_wait(full_bar(stage), phase);
                     }
                     tc_fence_after();
-                    const uint32_t sa = base + stage * Cfg::STAGE_BYTES;
-                    const uint32_t sb = sa + Cfg::A_BYTES;
+                    const uint32_t sa = base + stage * sstride;
+                    const uint32_t sb = sa + a_bytes;
                     if (!MN && g.kblk) {  // narrow K block: 16/32 elements, 32B/64B swizzle atoms
                         const uint32_t rowb = (uint32_t)g.kblk * 2u, lay = g.kblk == 16 ? 6u : (g.kblk == 32 ? 4u : 2u);
                         for (int k = 0; k < g.kblk / 16; ++k) {
@@ -244,7 +251,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                             tc_mma_f16(d_tmem, ad, bd, idesc, (kb > tc.kb0 || k > 0) ? 1u : 0u);
                         }
                         tc_commit(empty_bar(stage));
-                        if (++stage == STAGES) {
+                        if (++stage == nst) {
                             stage = 0;
                             phase ^= 1u;
                         }
@@ -266,7 +273,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         tc_commit_mc(empty_bar(stage), mc_mask);
                     else
                         tc_commit(empty_bar(stage));
-                    if (++stage == STAGES) {
+                    if (++stage == nst) {
                         stage = 0;
                         phase ^= 1u;
                     }
@@ -641,6 +648,8 @@ bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb,
     d.conv_stride = stride;
     d.kblk = kblk;
     d.stage_tx = (uint32_t)(BM + g->bn) * kblk * 2;
+    d.stage_stride = (d.stage_tx + 1023u) & ~1023u;
+    d.ring = (int)std::min<uint32_t>(GemmCfg<64>::MAX_RING, (uint32_t)(192u * 1024u) / d.stage_stride);
     d.C = Y;
     d.ldc = cout;
     d.M = (int)M;
