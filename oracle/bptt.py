@@ -52,7 +52,7 @@ class StepConfig:
     T: int
     C: int = 1
     p: float = 0.0
-    mode: str = "full"            # "full" | "ckpt" | "skip"
+    mode: str = "full"            # "full" | "ckpt" | "skip" | "tbptt"
     surrogate: str = "triangle"
     gamma: float = 0.3
     global_batch: int | None = None
@@ -309,11 +309,73 @@ def backward_segment(net, Wb, rows_state, dz, T_norm, carry, dW, cnt_kept, cfg: 
     return new_carry
 
 
+def tbptt_step(net, W, x, y, cfg: StepConfig) -> StepResult:
+    """Truncated BPTT (Sec. III-C), NEXT-4 of SURVEY.md §8(f).
+
+    The network is unrolled over truncation windows of t' = T/C steps.  At the end of window w a loss
+    is computed from the readout integrated over that window, z_w = W^L (sum_{t in w} a^{L-1}_t) / t'
+    (reading 24), its derivatives are back-propagated through the window only (the graph of earlier
+    windows is discarded: delta after the window's last step is zero), and the weight gradients of all
+    windows are summed.  The neuron state (U, o) itself carries on across windows.  The
+    reported loss is the sum of the window losses, so the gradient is the (truncated) gradient of it."""
+    spk = spiking_layers(net)
+    Ls = len(spk)
+    T, C = cfg.T, cfg.C
+    if T % C:
+        raise ValueError("C must divide T")
+    S = T // C
+    B = x.shape[1]
+    B_global = cfg.global_batch or B
+    use_gap = bool(net["layers"][-1].get("gap"))
+    Wb = [bf16_round(w) for w in W]
+    ledger = _Ledger()
+    U = [np.zeros((B,) + neuron_shape(L), np.float32) for L in spk]
+    o = [np.zeros((B,) + neuron_shape(L), np.uint8) for L in spk]
+    s = np.zeros(T, np.int64)
+    counts = np.zeros((Ls + 1, T), np.int64)
+    dW = [np.zeros(w.shape, np.float64) for w in W]
+    loss_tot = 0.0
+    first_U = [np.zeros((T, B) + neuron_shape(L), np.float32) for L in spk] if cfg.record else []
+    first_o = [np.zeros((T, B) + neuron_shape(L), np.uint8) for L in spk] if cfg.record else []
+    cnt_all = np.zeros((B,) + out_shape(spk[-1]), np.float64)
+    z = dz = None
+    for w in range(C):
+        rows_state = []
+        cnt = np.zeros((B,) + out_shape(spk[-1]), np.float64)
+        for t in range(w * S, (w + 1) * S):
+            U, o, a = forward_step(net, Wb, x[t], U, o)
+            s[t] = spike_sum(x[t], o)
+            counts[0, t] = int(np.asarray(x[t], np.int64).sum())
+            for l in range(Ls):
+                counts[l + 1, t] = int(np.asarray(o[l], np.int64).sum())
+                if cfg.record:
+                    first_U[l][t] = U[l]
+                    first_o[l][t] = o[l]
+            cnt += a[-1]
+            rows_state.append((U, o, a))
+            ledger.add(U + o)
+        cnt_all += cnt
+        loss_w, z, dz = readout(Wb[Ls], cnt, y, S, B_global, use_gap)
+        loss_tot += loss_w
+        carry = [np.zeros((B,) + neuron_shape(L), np.float64) for L in spk]     # the graph is cut here
+        cnt_w = np.zeros_like(cnt)
+        backward_segment(net, Wb, rows_state, dz, S, carry, dW, cnt_w, cfg)
+        dW[Ls] += dz.T @ readout_input(cnt_w, use_gap) / S
+        for st in rows_state:                     # the window's graph is released (P:459-462)
+            ledger.sub(st[0] + st[1])
+    keep = np.ones(T, bool)
+    return StepResult(loss=loss_tot, z=z, dz=dz, s=s, counts=counts, sam=s, sst=None, keep=keep,
+                      kept=kept_lists(keep, T, C), dW=dW, cnt=cnt_all, cnt_kept=cnt_all, ledger_peak=ledger.peak,
+                      first_U=first_U, first_o=first_o, rec_U=first_U, rec_o=first_o)
+
+
 def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
     """One training iteration's gradients (no optimizer step; see oracle/adam.py).
 
     W: float32 master weights per layer (spiking layers then readout).
     x: uint8 [T][B][...] input spikes, y: int [B] labels."""
+    if cfg.mode == "tbptt":
+        return tbptt_step(net, W, x, y, cfg)
     spk = spiking_layers(net)
     Ls = len(spk)
     T = cfg.T

@@ -256,3 +256,69 @@ def test_bf16_emulation_changes_only_rounding():
     for a, b in zip(r1.dW[:-1], r0.dW[:-1]):
         assert rel_err(a, b) < 2e-2
     np.testing.assert_array_equal(r1.dW[-1], r0.dW[-1])
+
+
+# ---- TBPTT (Sec. III-C; NEXT-4, reading 24)
+
+def torch_tbptt(net, W, x, y, C, gamma=0.3):
+    """Truncated BPTT as an autograd graph: the state carries on across windows but is detached at
+    every window start; each window's loss is CE of its own readout integral / t'; loss = sum."""
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    Wt = [torch.tensor(w.astype(np.float64), dtype=torch.float64, requires_grad=True) for w in W]
+    T, B = x.shape[:2]
+    S = T // C
+    U = [None] * len(spk)
+    o = [None] * len(spk)
+    total = 0
+    for w in range(C):
+        U = [u.detach() if u is not None else None for u in U]
+        o = [v.detach() if v is not None else None for v in o]
+        cnt = 0
+        for t in range(w * S, (w + 1) * S):
+            a = torch.tensor(x[t].astype(np.float64))
+            outs = []
+            for l, L in enumerate(spk):
+                I = t_current(L, Wt[l], a, outs[L["res"]] if "res" in L else None)
+                U[l] = I if U[l] is None else L["lam"] * U[l] + I - L["theta"] * o[l].detach()
+                o[l] = Spike.apply(U[l], L["theta"], gamma)
+                a = t_out(L, o[l])
+                outs.append(a)
+            cnt = cnt + a
+        z = t_readin(net, cnt) @ Wt[-1].T / S
+        total = total + F.cross_entropy(z, torch.tensor(y, dtype=torch.long), reduction="sum") / B
+    total.backward()
+    return float(total.detach()), [w.grad.numpy() for w in Wt]
+
+
+@pytest.mark.parametrize("name,lam,C", [("tiny_fc", 0.5, 3), ("tiny_conv", 1.0, 2), ("tiny_resnet", 0.5, 2)])
+def test_tbptt_equals_autograd(name, lam, C):
+    T = 12
+    net, W, x, y = dyadic_setup(name, T, 3, lam)
+    r = train_step(net, W, x, y, StepConfig(T=T, C=C, mode="tbptt", emulate_bf16=False))
+    loss, grads = torch_tbptt(net, W, x, y, C)
+    assert r.loss == pytest.approx(loss, rel=1e-12)
+    for l, (a, b) in enumerate(zip(r.dW, grads)):
+        assert rel_err(a, b) < 1e-12 or np.abs(a - b).max() < 1e-15, (l, rel_err(a, b))
+
+
+def test_tbptt_one_window_is_full_bptt():
+    """t' = T (C = 1): TBPTT is plain BPTT."""
+    T = 10
+    net, W, x, y = dyadic_setup("tiny_conv", T, 2, 0.75)
+    rt = train_step(net, W, x, y, StepConfig(T=T, C=1, mode="tbptt"))
+    rf = train_step(net, W, x, y, StepConfig(T=T, mode="full"))
+    assert rt.loss == rf.loss
+    for a, b in zip(rt.dW, rf.dW):
+        np.testing.assert_array_equal(a, b)
+
+
+def test_tbptt_forward_state_is_not_truncated():
+    """Only the gradient is truncated: the spikes of every window equal full BPTT's forward."""
+    T = 12
+    net, W, x, y = dyadic_setup("tiny_conv", T, 2, 0.75)
+    rt = train_step(net, W, x, y, StepConfig(T=T, C=3, mode="tbptt", record=True))
+    rf = train_step(net, W, x, y, StepConfig(T=T, mode="full", record=True))
+    for a, b in zip(rt.first_o, rf.first_o):
+        np.testing.assert_array_equal(a, b)
+    np.testing.assert_array_equal(rt.s, rf.s)
+    assert rt.ledger_peak * 3 == rf.ledger_peak      # one window of t' = T/3 stored at a time
