@@ -351,7 +351,7 @@ def run_ours(args):
     main = run_mode(torch, dist, args, wl, net, args.mode, rank, world, local_rank, profile=True, e2e=True)
     compare = {}
     if not args.no_compare:
-        for mode in ("full", "ckpt"):
+        for mode in ("full", "ckpt", "tbptt"):   # tbptt: the paper's comparison algorithm (Sec. III-C), t' = T/C
             if mode == args.mode:
                 continue
             try:
@@ -463,7 +463,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="cfg2_vgg5")
-    ap.add_argument("--mode", default="skip", choices=["skip", "ckpt", "full"])
+    ap.add_argument("--mode", default="skip", choices=["skip", "ckpt", "full", "tbptt"])
     ap.add_argument("--T", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--C", type=int, default=0)

@@ -59,7 +59,12 @@ typedef enum {
     SKIPPER_EUNSUPPORTED = 7  /* layer geometry this build has no kernel for        */
 } skipper_status;
 
-typedef enum { SKIPPER_MODE_FULL = 0, SKIPPER_MODE_CKPT = 1, SKIPPER_MODE_SKIP = 2 } skipper_mode;
+/* TBPTT (Sec. III-C): C truncation windows of t' = T/C steps;
+ * each window integrates its own readout (z_w = W^L sum_{t in w} a_t / t'), adds its cross-entropy to the
+ * loss and back-propagates through the window only (delta is zero after the window's last step); the
+ * neuron state carries on; weight gradients are summed over windows.  Segment API order:
+ * forward_segment(w, FIRST, x, labels) then backward_segment(w) for w = 0..C-1, then optimizer_step. */
+typedef enum { SKIPPER_MODE_FULL = 0, SKIPPER_MODE_CKPT = 1, SKIPPER_MODE_SKIP = 2, SKIPPER_MODE_TBPTT = 3 } skipper_mode;
 typedef enum { SKIPPER_PASS_FIRST = 0, SKIPPER_PASS_RECOMPUTE = 1, SKIPPER_PASS_RECORD = 2 } skipper_pass;
 typedef enum { SKIPPER_LAYER_FC = 0, SKIPPER_LAYER_CONV3X3 = 1, SKIPPER_LAYER_READOUT = 2 } skipper_layer_kind;
 typedef enum { SKIPPER_SURR_TRIANGLE = 0, SKIPPER_SURR_FAST_SIGMOID = 1 } skipper_surrogate;

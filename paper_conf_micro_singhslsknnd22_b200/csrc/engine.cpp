@@ -549,13 +549,17 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     c->B = cfg->batch;
     c->Bg = cfg->global_batch > 0 ? cfg->global_batch : cfg->batch;
     if (c->T <= 0 || c->B <= 0) return bail(fail(c, SKIPPER_EINVAL, "T and batch must be positive"));
-    if (cfg->mode < 0 || cfg->mode > 2) return bail(fail(c, SKIPPER_EINVAL, "unknown mode %d", cfg->mode));
+    if (cfg->mode < 0 || cfg->mode > 3) return bail(fail(c, SKIPPER_EINVAL, "unknown mode %d", cfg->mode));
     if (cfg->surrogate != SKIPPER_SURR_TRIANGLE && cfg->surrogate != SKIPPER_SURR_FAST_SIGMOID)
         return bail(fail(c, SKIPPER_EINVAL, "unknown surrogate %d", cfg->surrogate));
     if (cfg->sam != SKIPPER_SAM_SPIKES && cfg->sam != SKIPPER_SAM_WEIGHTED)
         return bail(fail(c, SKIPPER_EINVAL, "unknown SAM metric %d", cfg->sam));
     if (cfg->mode == SKIPPER_MODE_FULL) {
         c->C = 1;
+    } else if (cfg->mode == SKIPPER_MODE_TBPTT) {
+        c->C = cfg->C;
+        if (c->C <= 0 || c->T % c->C)
+            return bail(fail(c, SKIPPER_EINVAL, "C=%d truncation windows must divide T=%d", c->C, c->T));
     } else {
         c->C = cfg->C;
         if (c->C <= 0 || c->T % c->C)
@@ -589,7 +593,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
                       sk::layer0_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
         // opt-in: measured slower than reverse scan + im2col wgrad GEMM on VGG-5
         const char *e2 = getenv("SKIPPER_L0_BWD_FUSION");
-        c->l0_bwd_fused = c->l0_fused && (e2 && atoi(e2)) &&
+        c->l0_bwd_fused = c->l0_fused && (e2 && atoi(e2)) && cfg->mode != SKIPPER_MODE_TBPTT &&
                           sk::layer0_bwd_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
         // conv layers after the first: tensor-core GEMM + LIF scan fused (not the last spiking layer,
         // whose scan also accumulates the readout counts)
@@ -613,7 +617,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     // recurrences still run in time order; checkpoints are written every S rows).
     c->tail0 = c->Ls;
     while (c->tail0 > 0 && c->L[c->tail0 - 1].fc) --c->tail0;
-    if (cfg->mode == SKIPPER_MODE_FULL) c->tail0 = c->Ls;
+    if (cfg->mode == SKIPPER_MODE_FULL || cfg->mode == SKIPPER_MODE_TBPTT) c->tail0 = c->Ls;
 
     // ---- persistent allocations
     c->dw_total = 0;
@@ -643,7 +647,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
             AL(l.U_run, bn);
             AL(l.o_run, bn);
             AL(l.carry, bn);
-            if (cfg->mode != SKIPPER_MODE_FULL) {
+            if (cfg->mode != SKIPPER_MODE_FULL && cfg->mode != SKIPPER_MODE_TBPTT) {
                 AL(l.ckU, bn * c->C);
                 AL(l.cko, bn * c->C);
             }
@@ -1255,11 +1259,11 @@ static skipper_status comm_allreduce_s(skipper_ctx *c) {
 }
 
 // After the last FIRST segment: loss, SAM totals, SST and keep lists (Eq.4, Eq.5).
-static skipper_status finish_first(skipper_ctx *c, const int *labels) {
+// Readout integrator + cross-entropy of cnt (normalised by 1/Tn): z, dz, loss += CE / B_global, and
+// dL/da^{L-1} into g_last (through the GAP when the readout has one).
+static skipper_status readout_forward(skipper_ctx *c, const int *labels, float invTn) {
     const Layer &last = c->L[c->Ls - 1];
     const Layer &ro = c->L.back();
-    ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
-    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
     ProfScope ps1(c, K_READOUT, (double)c->B * last.Nout * 8 + (double)ro.wcount * 2, 4.0 * c->B * last.Nout * ro.Cout);
     c->launches += 2;  // z, cross-entropy and dL/da^{L-1} kernels
     if (ro.gap) {  // readout of the global average pool (reading 23); dL/da^{L-1} spread back over the positions
@@ -1267,12 +1271,19 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
         c->launches += 2;
         CK(sk::launch_gap_reduce(c->cnt, c->cnt_gap, c->B, P, last.Cout, c->st));
         CK(sk::launch_readout_loss(ro.wb, c->cnt_gap, labels, c->z, c->dz, c->loss_dev, c->g_gap, c->B, ro.Cin,
-                                   ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+                                   ro.Cout, invTn, 1.0f / c->Bg, c->st));
         CK(sk::launch_gap_expand(c->g_gap, c->g_last, c->B, P, last.Cout, c->st));
     } else {
         CK(sk::launch_readout_loss(ro.wb, c->cnt, labels, c->z, c->dz, c->loss_dev, c->g_last, c->B, (int)last.Nout,
-                                   ro.Cout, 1.0f / c->T, 1.0f / c->Bg, c->st));
+                                   ro.Cout, invTn, 1.0f / c->Bg, c->st));
     }
+    return SKIPPER_OK;
+}
+
+static skipper_status finish_first(skipper_ctx *c, const int *labels) {
+    ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
+    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
+    if (c->cfg.mode != SKIPPER_MODE_TBPTT) CKS(readout_forward(c, labels, 1.0f / c->T));
     CKS(comm_allreduce_s(c));
     CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
                        c->st));
@@ -1294,6 +1305,7 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     c->keep.assign(c->T, 1);
     c->sst.assign(C, NAN);
     const bool skip = c->cfg.mode == SKIPPER_MODE_SKIP && c->cfg.p != 0.0;
+    if (c->cfg.mode == SKIPPER_MODE_TBPTT) return SKIPPER_OK;  // no keep mask: the counts are for reporting
     for (int seg = 0; seg < C; ++seg) {
         if (skip)
             c->sst[seg] = c->cfg.sam == SKIPPER_SAM_WEIGHTED
@@ -1581,6 +1593,62 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
     return join_wgrads(c);
 }
 
+// ------------------------------------------------------------------------------------ TBPTT (NEXT-4)
+// Window w of truncated BPTT (reading 24): forward from the running state storing U and the outputs of
+// its t' = S rows, then the window's own readout and loss (added to the step loss).
+static skipper_status tbptt_forward(skipper_ctx *c, int w, const int *labels) {
+    CKS(zero_dev(c, c->cnt, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
+    CKS(forward_rows_first(c, w, c->S, w * c->S, true));
+    return readout_forward(c, labels, 1.0f / c->S);
+}
+
+// Backward of window w: the graph is cut at the window's end (zero carry), weight gradients accumulate.
+static skipper_status tbptt_backward(skipper_ctx *c, int w) {
+    for (int i = 0; i < c->Ls; ++i) CKS(zero_dev(c, c->L[i].carry, (size_t)c->B * c->L[i].N * 4));
+    CKS(backward_rows(c, c->S, nullptr, w == c->C - 1));
+    const Layer &last = c->L[c->Ls - 1];
+    const Layer &ro = c->L.back();
+    ProfScope ps(c, K_READOUT, (double)c->B * (last.Nout + ro.Cout) * 4 + (double)ro.wcount * 8,
+                 2.0 * c->B * last.Nout * ro.Cout);
+    const float *cin = c->cnt;
+    int D = (int)last.Nout;
+    if (ro.gap) {
+        c->launches += 1;
+        CK(sk::launch_gap_reduce(c->cnt, c->cnt_gap, c->B, (int)(last.Nout / last.Cout), last.Cout, c->st));
+        cin = c->cnt_gap;
+        D = ro.Cin;
+    }
+    CK(sk::launch_readout_wgrad(c->dz, cin, ro.dw, c->B, D, ro.Cout, 1.0f / c->S, c->st, 1));
+    return SKIPPER_OK;
+}
+
+// After the last window: layer-0 unpad, the last dW buckets, SAM counts (reporting), debug copies.
+static skipper_status tbptt_finish(skipper_ctx *c) {
+    Layer &l0 = c->L[0];
+    const Layer &ro = c->L.back();
+    if (l0.dwp) {
+        const int cols = (int)(l0.wcount / l0.Cout);
+        ProfScope ps(c, K_UNPAD, (double)l0.Cout * (c->K0 + cols) * 4, 0);
+        CK(sk::launch_unpad_f32(l0.dwp, l0.dw, l0.Cout, cols, c->K0, c->st));
+    }
+    if (c->comm.comm) {
+        CK(cudaEventRecord(c->ev_w, c->st));
+        CK(cudaStreamWaitEvent(c->st3, c->ev_w, 0));
+        std::string e;
+        if (!c->comm.allreduce_f32(l0.dw, l0.wcount, c->st3, &e) || !c->comm.allreduce_f32(ro.dw, ro.wcount, c->st3, &e))
+            return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+        c->comm_pending = true;
+    }
+    CKS(finish_first(c, nullptr));
+    if (c->cfg.debug_record)
+        for (int i = 0; i < c->Ls; ++i) {
+            const size_t bn = (size_t)c->B * c->L[i].N * c->T;
+            CK(cudaMemcpyAsync(c->L[i].dbg[1], c->L[i].dbg[0], bn * 4, cudaMemcpyDeviceToDevice, c->st));
+            CK(cudaMemcpyAsync(c->L[i].dbgo[1], c->L[i].dbgo[0], bn, cudaMemcpyDeviceToDevice, c->st));
+        }
+    return SKIPPER_OK;
+}
+
 // ------------------------------------------------------------------------------------ public schedule
 extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int pass, const unsigned char *x_dev,
                                                   const int *labels_dev) {
@@ -1599,6 +1667,25 @@ extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int p
         return SKIPPER_OK;
     }
     if (full) return fail(c, SKIPPER_EORDER, "FULL mode uses the RECORD pass");
+    if (c->cfg.mode == SKIPPER_MODE_TBPTT) {  // window w: forward + its loss (then backward_segment(w))
+        if (pass != SKIPPER_PASS_FIRST) return fail(c, SKIPPER_EORDER, "TBPTT windows use the FIRST pass");
+        if (!labels_dev) return fail(c, SKIPPER_EINVAL, "every TBPTT window needs labels");
+        if (seg == 0) {
+            if (c->phase != PH_IDLE && c->phase != PH_BWD_DONE)
+                return fail(c, SKIPPER_EORDER, "FIRST(0) while an iteration is in flight");
+            CKS(begin_step(c, x_dev));
+            CKS(arena_rows(c, c->S));
+            c->phase = PH_FIRST;
+            c->next_seg = 0;
+        }
+        if (c->phase != PH_FIRST || seg != c->next_seg)
+            return fail(c, SKIPPER_EORDER, "TBPTT windows run FIRST(w), BACKWARD(w) for w = 0..C-1 (expected %d)",
+                        c->next_seg);
+        if (x_dev != c->x_cur) return fail(c, SKIPPER_EINVAL, "x_dev changed within an iteration");
+        CKS(tbptt_forward(c, seg, labels_dev));
+        c->phase = PH_RECOMPUTED;
+        return SKIPPER_OK;
+    }
     if (pass == SKIPPER_PASS_FIRST) {
         if (seg == 0) {
             if (c->phase != PH_IDLE && c->phase != PH_BWD_DONE && c->phase != PH_FIRST)
@@ -1639,6 +1726,19 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
     CKS(check_ctx(c));
     if (c->phase != PH_RECOMPUTED || seg != c->next_seg)
         return fail(c, SKIPPER_EORDER, "BACKWARD(%d) must follow RECOMPUTE(%d)", seg, c->next_seg);
+    if (c->cfg.mode == SKIPPER_MODE_TBPTT) {
+        CKS(tbptt_backward(c, seg));
+        if (seg == c->C - 1) {
+            CKS(tbptt_finish(c));
+            c->phase = PH_BWD_DONE;
+            c->grads_ready = true;
+            CKS(arena_free(c));
+        } else {
+            c->phase = PH_FIRST;
+            c->next_seg = seg + 1;
+        }
+        return SKIPPER_OK;
+    }
     const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
     const int R = full ? c->T : (int)c->kept[seg].size();
     const int *row_t = full ? nullptr : c->kept_dev + (size_t)seg * c->S;
@@ -1732,6 +1832,12 @@ extern "C" skipper_status skipper_step(skipper_ctx *c, const unsigned char *x_de
     if (c->cfg.mode == SKIPPER_MODE_FULL) {
         CKS(skipper_forward_segment(c, 0, SKIPPER_PASS_RECORD, x_dev, labels_dev));
         CKS(skipper_backward_segment(c, 0));
+    } else if (c->cfg.mode == SKIPPER_MODE_TBPTT) {
+        c->phase = PH_IDLE;
+        for (int w = 0; w < c->C; ++w) {
+            CKS(skipper_forward_segment(c, w, SKIPPER_PASS_FIRST, x_dev, labels_dev));
+            CKS(skipper_backward_segment(c, w));
+        }
     } else {
         c->phase = PH_IDLE;
         for (int seg = 0; seg < c->C; ++seg)
@@ -1846,6 +1952,7 @@ extern "C" size_t skipper_workspace_bytes(const skipper_layer *layers, int n, co
     const long long per_step = B * (Nsum * 4 + Nout_sum * 2);  // stored U fp32 + layer output bf16
     const long long per_ckpt = B * Nsum * 5;                   // checkpoint U fp32 + o u8
     if (cfg->mode == SKIPPER_MODE_FULL) return (size_t)(cfg->T * per_step);
+    if (cfg->mode == SKIPPER_MODE_TBPTT) return (size_t)((cfg->C > 0 ? cfg->T / cfg->C : cfg->T) * per_step);
     const int C = cfg->C > 0 ? cfg->C : 1;
     const int rows = kept_max >= 0 ? kept_max : cfg->T / C;
     return (size_t)(C * per_ckpt + (long long)rows * per_step);

@@ -130,7 +130,7 @@ cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int
                                 float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
                                 cudaStream_t s);
 cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K,
-                                 float invT, cudaStream_t s);
+                                 float invT, cudaStream_t s, int accumulate = 0);
 
 // Adam + bf16 shadow; transposed bf16 shadow for the dgrad GEMMs.
 cudaError_t launch_adam(float *w, const float *g, float *m, float *v, uint16_t *wb, size_t n, float lr, float b1,

@@ -787,19 +787,20 @@ cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int
     return cudaGetLastError();
 }
 
-__global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT) {
+__global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT,
+                                     int accumulate) {
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)K * D) return;
     const int k = (int)(i / D), n = (int)(i % D);
     float acc = 0.f;
     for (int b = 0; b < B; ++b) acc += dz[(long long)b * K + k] * cnt_kept[(long long)b * D + n];
-    dWL[i] = acc * invT;
+    dWL[i] = accumulate ? dWL[i] + acc * invT : acc * invT;
 }
 
 cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT,
-                                 cudaStream_t s) {
+                                 cudaStream_t s, int accumulate) {
     const long long n = (long long)K * D;
-    readout_wgrad_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(dz, cnt_kept, dWL, B, D, K, invT);
+    readout_wgrad_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(dz, cnt_kept, dWL, B, D, K, invT, accumulate);
     return cudaGetLastError();
 }
 

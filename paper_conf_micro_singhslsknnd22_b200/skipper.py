@@ -16,7 +16,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libskipper.so")
 
-MODE = {"full": 0, "ckpt": 1, "skip": 2}
+MODE = {"full": 0, "ckpt": 1, "skip": 2, "tbptt": 3}
 PASS_FIRST, PASS_RECOMPUTE, PASS_RECORD = 0, 1, 2
 LAYER_KIND = {"fc": 0, "conv": 1, "readout": 2}
 SURROGATE = {"triangle": 0, "fast_sigmoid": 1}

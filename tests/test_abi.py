@@ -131,3 +131,19 @@ def test_bucket_plan_partitions_layers(name, mb):
     for lo, hi in b[:-1]:
         assert 4 * sum(wc[lo:hi + 1]) >= mb << 20
         assert 4 * sum(wc[lo + 1:hi + 1]) < mb << 20      # closed as soon as it was full
+
+
+def test_workspace_model_tbptt():
+    """TBPTT stores one truncation window: T/C steps of U + outputs, independent of T at fixed t'."""
+    net = synth.net_config("vgg5")
+    full = sk.workspace_bytes(net, sk.make_config(T=100, mode="full", batch=8))
+    tb = [sk.workspace_bytes(net, sk.make_config(T=T, C=T // 10, mode="tbptt", batch=8)) for T in (100, 400)]
+    assert tb[0] == tb[1] == full // 10
+
+
+def test_tbptt_validation():
+    net = synth.net_config("tiny_fc")
+    st, msg = _create(net, T=12, C=5, mode="tbptt", batch=2)
+    assert st == 1 and "divide" in msg
+    st, _ = _create(net, T=12, C=12, mode="tbptt", batch=2)   # t' = 1 is a valid truncation window
+    assert st == 0 or st == 3   # 3 = no CUDA device on the CPU box

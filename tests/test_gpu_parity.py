@@ -245,3 +245,12 @@ def test_one_rank_nccl_bucketed_allreduce(name, T, C, monkeypatch):
         assert (a.double() - b.double()).norm() <= 1e-6 * b.double().norm() + 1e-12   # split-K atomics order
     for a, b in zip(out[0][2], out[1][2]):
         np.testing.assert_allclose(a.numpy(), b.numpy(), rtol=0, atol=1e-6)
+
+
+@pytest.mark.parametrize("name,T,B,C,lam", [("tiny_fc", 12, 3, 3, 0.5), ("tiny_conv", 12, 3, 2, 0.99),
+                                            ("vgg5", 14, 2, 2, None), ("tiny_resnet", 16, 3, 2, 0.75),
+                                            ("fc784", 20, 4, 4, None)])
+def test_tbptt(name, T, B, C, lam):
+    """NEXT-4: truncated BPTT (Sec. III-C) on the device - per-window loss and readout, graph cut at window
+    edges, state carried on - against the oracle (spikes exact, summed loss, dW)."""
+    check_parity(name, T=T, B=B, C=C, p=0.0, mode="tbptt", lam=lam)
