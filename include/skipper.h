@@ -72,8 +72,11 @@ typedef enum { SKIPPER_SURR_TRIANGLE = 0, SKIPPER_SURR_FAST_SIGMOID = 1 } skippe
  * SPIKES   s_t = sum over the input and every spiking layer of the spikes at t (Eq.4);
  * WEIGHTED s_t = sum_l count_l,t / N_l, N_l = neurons per sample of layer l (l = 0: the input), in
  *          float64 in layer order - "the sum of spike counts weighted by the neuron count in each
- *          layer" (reading 22). */
-typedef enum { SKIPPER_SAM_SPIKES = 0, SKIPPER_SAM_WEIGHTED = 1 } skipper_sam;
+ *          layer" (reading 22).
+ * L2TRACE  s_t = sqrt(sum over every spiking neuron of U_t^2), the l2 norm of the membrane trace at t (the
+ *          other variant P:1049-1061 names; reading 25), squares exact in float64, summed in
+ *          float64 (allreduced under DP); the mask then depends only on the order of the s_t. */
+typedef enum { SKIPPER_SAM_SPIKES = 0, SKIPPER_SAM_WEIGHTED = 1, SKIPPER_SAM_L2TRACE = 2 } skipper_sam;
 
 /* One layer.  conv3x3: zero pad 1, stride 1 or 2; h x w = the OUTPUT (neuron) size, the
  * input is (stride*h) x (stride*w); optional 2x2 average pooling of the output spikes

@@ -61,8 +61,9 @@ class StepConfig:
     dz: np.ndarray | None = None         # test hook: impose the readout gradient
     T_norm: int | None = None            # readout normalisation (default T)
     s_global: np.ndarray | None = None   # data-parallel: allreduced s (reading 19)
-    sam: str = "spikes"                  # SAM metric: "spikes" (Eq.4) | "weighted" (NEXT-2, reading 22)
+    sam: str = "spikes"                  # SAM metric: "spikes" (Eq.4) | "weighted" (reading 22) | "l2trace" (reading 25)
     counts_global: np.ndarray | None = None  # data-parallel: allreduced per-layer counts (weighted SAM)
+    u2_global: np.ndarray | None = None      # data-parallel: allreduced sum of U^2 per t (l2-trace SAM)
     record: bool = False
     trace: bool = False
 
@@ -194,6 +195,7 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
     o = [np.zeros((B,) + neuron_shape(L), np.uint8) for L in spk]
     s = np.zeros(T, np.int64)
     counts = np.zeros((len(spk) + 1, T), np.int64)
+    u2 = np.zeros(T, np.float64)          # sum over every spiking neuron of U_t^2 (l2-trace SAM, reading 25)
     cnt = np.zeros((B,) + out_shape(spk[-1]), np.float64)
     ckpt = {}
     stored = []          # FULL: list over t of (U list, o list, a list)
@@ -205,6 +207,7 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
         counts[0, t] = int(np.asarray(x[t], np.int64).sum())
         for l in range(len(spk)):
             counts[l + 1, t] = int(np.asarray(o[l], np.int64).sum())
+            u2[t] += float(np.sum(np.asarray(U[l], np.float64) ** 2))
         cnt += a[-1]
         if record:
             for l in range(len(spk)):
@@ -220,7 +223,7 @@ def forward_first_pass(net, Wb, x, T: int, S: int, store_all: bool, ledger: _Led
                 trace.append(("ckpt", t))
         if trace is not None:
             trace.append(("first", t))
-    return {"s": s, "counts": counts, "cnt": cnt, "ckpt": ckpt, "stored": stored,
+    return {"s": s, "counts": counts, "u2": u2, "cnt": cnt, "ckpt": ckpt, "stored": stored,
             "first_U": first_U, "first_o": first_o}
 
 
@@ -405,6 +408,9 @@ def train_step(net, W, x, y, cfg: StepConfig) -> StepResult:
         counts = first["counts"] if cfg.counts_global is None else np.asarray(cfg.counts_global, np.int64)
         neurons = [int(np.prod(x.shape[2:]))] + [int(np.prod(neuron_shape(L))) for L in spk]
         s_pol = sam_weighted(counts, neurons)
+    elif cfg.sam == "l2trace":
+        u2 = first["u2"] if cfg.u2_global is None else np.asarray(cfg.u2_global, np.float64)
+        s_pol = np.sqrt(u2)
     elif cfg.sam == "spikes":
         s_pol = s if cfg.s_global is None else np.asarray(cfg.s_global, np.int64)
     else:

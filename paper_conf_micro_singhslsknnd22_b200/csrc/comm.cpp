@@ -82,6 +82,11 @@ bool Comm::allreduce_i64(long long *buf, size_t cnt, cudaStream_t s, std::string
                  "ncclAllReduce(s)", err);
 }
 
+bool Comm::allreduce_f64(double *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    return check(nccl().allReduce(buf, buf, cnt, ncclFloat64, ncclSum, static_cast<ncclComm_t>(comm), s),
+                 "ncclAllReduce(u2)", err);
+}
+
 bool Comm::allreduce_f32(float *buf, size_t cnt, cudaStream_t s, std::string *err) {
     return check(nccl().allReduce(buf, buf, cnt, ncclFloat32, ncclSum, static_cast<ncclComm_t>(comm), s),
                  "ncclAllReduce(dW)", err);

@@ -17,6 +17,7 @@ struct Comm {
     bool init(const unsigned char id[128], int rank, int world, std::string *err);
     bool allreduce_i64(long long *buf, size_t n, cudaStream_t s, std::string *err);
     bool allreduce_f32(float *buf, size_t n, cudaStream_t s, std::string *err);
+    bool allreduce_f64(double *buf, size_t n, cudaStream_t s, std::string *err);
     void destroy();
 };
 

@@ -175,6 +175,13 @@ SK_DEV void red_add_v4(float *addr, float a, float b, float c, float d) {
                  : "memory");
 }
 
+// l2-trace SAM (reading 25): sum of the warp's U^2 (squares exact in fp64) into partial slot t*32 + blk%32
+SK_DEV void u2_warp_add(double *part, long long t, double q) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
+    if ((threadIdx.x & 31) == 0 && q != 0.0) atomicAdd(part + t * 32 + (blockIdx.x & 31), q);
+}
+
 SK_DEV uint32_t elect_one() {
     uint32_t pred = 0;
     asm volatile(

@@ -351,6 +351,14 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             auto emit = [&](int r) {
                 const long long t = row_time(r);
                 unsigned cnt = 0;
+                if (a.u2_part) {  // l2-trace SAM (reading 25): this thread's U^2, summed per warp
+                    double q2 = 0.0;
+                    if (valid) {
+#pragma unroll
+                        for (int c = 0; c < CW; ++c) q2 += (double)U[c] * (double)U[c];
+                    }
+                    u2_warp_add(a.u2_part, t, q2);
+                }
                 if (valid) {
 #pragma unroll
                     for (int j = 0; j < CW / 32; ++j) cnt += __popc(ob[j]);

@@ -111,6 +111,8 @@ struct skipper_ctx {
     long long in_row = 0;       // staged bf16 layer-0 operand elements per sample
     // persistent
     unsigned *s_part = nullptr;
+    double *u2_part = nullptr, *u2_dev = nullptr;  // l2-trace SAM: [T][32] partials, [T] totals
+    std::vector<double> u2_host;
     long long *s_dev = nullptr;
     float *cnt = nullptr, *cnt_kept = nullptr, *z = nullptr, *dz = nullptr, *loss_dev = nullptr, *g_last = nullptr;
     int *kept_dev = nullptr;
@@ -552,7 +554,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     if (cfg->mode < 0 || cfg->mode > 3) return bail(fail(c, SKIPPER_EINVAL, "unknown mode %d", cfg->mode));
     if (cfg->surrogate != SKIPPER_SURR_TRIANGLE && cfg->surrogate != SKIPPER_SURR_FAST_SIGMOID)
         return bail(fail(c, SKIPPER_EINVAL, "unknown surrogate %d", cfg->surrogate));
-    if (cfg->sam != SKIPPER_SAM_SPIKES && cfg->sam != SKIPPER_SAM_WEIGHTED)
+    if (cfg->sam != SKIPPER_SAM_SPIKES && cfg->sam != SKIPPER_SAM_WEIGHTED && cfg->sam != SKIPPER_SAM_L2TRACE)
         return bail(fail(c, SKIPPER_EINVAL, "unknown SAM metric %d", cfg->sam));
     if (cfg->mode == SKIPPER_MODE_FULL) {
         c->C = 1;
@@ -660,6 +662,10 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         }
     }
     AL(c->s_part, (size_t)(c->Ls + 1) * c->T * 32);  // [layer group][T][32] partial counters
+    if (cfg->sam == SKIPPER_SAM_L2TRACE) {
+        AL(c->u2_part, (size_t)c->T * 32);
+        AL(c->u2_dev, (size_t)c->T);
+    }
     AL(c->s_dev, (size_t)(c->Ls + 1) * c->T);
     const Layer &last = c->L[c->Ls - 1];
     const Layer &ro = c->L.back();
@@ -725,6 +731,8 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         const Layer &last = c->L[c->Ls - 1];
         const Layer &ro = c->L.back();
         dev_free(c, c->s_part, (size_t)(c->Ls + 1) * c->T * 32 * 4);
+        dev_free(c, c->u2_part, (size_t)c->T * 32 * 8);
+        dev_free(c, c->u2_dev, (size_t)c->T * 8);
         dev_free(c, c->s_dev, (size_t)(c->Ls + 1) * c->T * 8);
         dev_free(c, c->cnt, (size_t)c->B * last.Nout * 4);
         dev_free(c, c->cnt_gap, (size_t)c->B * ro.Cin * 4);
@@ -1000,6 +1008,7 @@ static unsigned *spart(skipper_ctx *c, int group) { return c->s_part + (size_t)g
 static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
     if (c->prof_on) prof_resolve(c);
     CKS(zero_dev(c, c->s_part, (size_t)(c->Ls + 1) * c->T * 32 * 4));
+    if (c->u2_part) CKS(zero_dev(c, c->u2_part, (size_t)c->T * 32 * 8));
     CKS(zero_dev(c, c->cnt, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
     CKS(zero_dev(c, c->cnt_kept, (size_t)c->B * c->L[c->Ls - 1].Nout * 4));
     CKS(zero_dev(c, c->loss_dev, 4));
@@ -1093,6 +1102,7 @@ static skipper_status forward_tail_first(skipper_ctx *c) {
         a.cko = l.cko;
         a.ck_every = c->S;
         a.s_part = spart(c, i + 1);
+        a.u2_part = c->u2_part;
         a.t0 = 0;
         a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
         a.dbg_U = c->cfg.debug_record ? l.dbg[0] : nullptr;
@@ -1139,6 +1149,7 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
     a.s_part = restore ? nullptr : spart(c, 1);
     a.s_part_in = restore ? nullptr : spart(c, 0);
+    a.u2_part = restore ? nullptr : c->u2_part;
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
     a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
     // stored passes also emit the im2col rows the layer-0 weight gradient reads (no staging kernel)
@@ -1174,6 +1185,7 @@ static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
     a.s_part = restore ? nullptr : spart(c, i + 1);
+    a.u2_part = restore ? nullptr : c->u2_part;
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
     a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
     a.lam = l.d.lambda;
@@ -1228,6 +1240,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         a.ckU = record ? nullptr : l.ckU + (size_t)seg * c->B * l.N;
         a.cko = record ? nullptr : l.cko + (size_t)seg * c->B * l.N;
         a.s_part = spart(c, i + 1);
+        a.u2_part = c->u2_part;
         a.row_t = nullptr;
         a.t0 = t0;
         a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
@@ -1283,6 +1296,15 @@ static skipper_status readout_forward(skipper_ctx *c, const int *labels, float i
 static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
     CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
+    if (c->u2_part) {
+        CK(sk::launch_sum32_f64(c->u2_part, c->u2_dev, c->T, c->st));
+        if (c->comm.comm) {
+            std::string e;
+            if (!c->comm.allreduce_f64(c->u2_dev, c->T, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+        }
+        c->u2_host.assign(c->T, 0.0);
+        CK(cudaMemcpyAsync(c->u2_host.data(), c->u2_dev, (size_t)c->T * 8, cudaMemcpyDeviceToHost, c->st));
+    }
     if (c->cfg.mode != SKIPPER_MODE_TBPTT) CKS(readout_forward(c, labels, 1.0f / c->T));
     CKS(comm_allreduce_s(c));
     CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
@@ -1298,7 +1320,8 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
             w = w + (double)v / (double)(g == 0 ? c->in_elems : c->L[g - 1].N);
         }
         c->s_host[t] = tot;
-        c->sam_host[t] = c->cfg.sam == SKIPPER_SAM_WEIGHTED ? w : (double)tot;
+        c->sam_host[t] = c->cfg.sam == SKIPPER_SAM_WEIGHTED ? w
+                         : c->cfg.sam == SKIPPER_SAM_L2TRACE ? std::sqrt(c->u2_host[t]) : (double)tot;
     }
     const int C = c->C, S = c->S;
     c->kept.assign(C, {});
@@ -1308,7 +1331,7 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     if (c->cfg.mode == SKIPPER_MODE_TBPTT) return SKIPPER_OK;  // no keep mask: the counts are for reporting
     for (int seg = 0; seg < C; ++seg) {
         if (skip)
-            c->sst[seg] = c->cfg.sam == SKIPPER_SAM_WEIGHTED
+            c->sst[seg] = c->cfg.sam != SKIPPER_SAM_SPIKES
                               ? sst_double(c->sam_host.data() + (size_t)seg * S, S, c->cfg.p)
                               : skipper_sst_host(c->s_host.data() + (size_t)seg * S, S, c->cfg.p);
         for (int t = seg * S; t < (seg + 1) * S; ++t) {

@@ -96,6 +96,7 @@ struct ConvLifArgs {
     float *ckU;
     uint8_t *cko;
     unsigned *s_part;
+    double *u2_part;  // l2-trace SAM partials [T][32] or null
     float *dbg_U;
     uint8_t *dbg_o;
     float lam, theta;

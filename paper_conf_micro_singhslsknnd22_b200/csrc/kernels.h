@@ -24,6 +24,7 @@ struct ScanFwdArgs {
     uint8_t *cko;
     int ck_every;          // >0: rows r % ck_every == 0 write checkpoint slot r / ck_every (whole-T scans)
     unsigned *s_part;      // SAM partials [T][32] or null (FIRST/RECORD only)
+    double *u2_part;       // l2-trace SAM (reading 25): sum of U^2 per row into [T][32] fp64 partials, or null
     const int *row_t;      // absolute t of each row (device) or null -> t0 + r
     int t0;
     float *cnt;            // readout accumulation [B*Nout] or null (last spiking layer)
@@ -82,6 +83,8 @@ cudaError_t launch_gap_expand(const float *g, float *out, int B, int P, int C, c
 cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);
+// u2[t] = sum of the 32 fp64 partials of row t, in slot order
+cudaError_t launch_sum32_f64(const double *part, double *out, int T, cudaStream_t st);
 
 // Fused first layer for narrow inputs (layer0.cu): im2col in smem + tcgen05 + LIF + pool + SAM.
 struct L0FwdArgs {
@@ -100,6 +103,7 @@ struct L0FwdArgs {
     uint8_t *cko;
     unsigned *s_part;      // SAM partials [T][32] of this layer's spikes, or null
     unsigned *s_part_in;   // SAM partials [T][32] of the input spikes (l = 0), or null
+    double *u2_part;       // l2-trace SAM: sum of U^2 per row into [T][32] fp64 partials, or null
     float *dbg_U;
     uint8_t *dbg_o;
     uint16_t *xg_out;      // or null: also write the bf16 im2col rows [R][B*H*W][32] (weight-gradient operand)

@@ -421,6 +421,14 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             auto emit = [&](int ri) {
                 const long long t = row_time(ri);
                 unsigned cnt = valid ? __popc(ob) : 0u;
+                if (a.u2_part) {  // l2-trace SAM (reading 25): this thread's U^2, summed per warp
+                    double q2 = 0.0;
+                    if (valid) {
+#pragma unroll
+                        for (int c = 0; c < CW; ++c) q2 += (double)U[c] * (double)U[c];
+                    }
+                    u2_warp_add(a.u2_part, t, q2);
+                }
                 if (a.pool) {  // 2x2 window = lanes 4k..4k+3
                     const int lb = lane & ~3;
                     const uint32_t w0 = __shfl_sync(0xffffffffu, ob, lb), w1 = __shfl_sync(0xffffffffu, ob, lb + 1);

@@ -203,6 +203,7 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
             const int r = rb + j;
             if (r >= a.R) break;  // block-uniform
             unsigned nspk = 0;
+            double q2 = 0.0;
             if (active) {
                 uint32_t nb = 0;
 #pragma unroll
@@ -212,6 +213,7 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
                     for (int i = 0; i < 4; ++i) {
                         U[k][i] = lif_update(U[k][i], Ii[i], bit(k, i), a.lam, a.theta);
                         nb |= (U[k][i] > a.theta ? 1u : 0u) << (4 * k + i);
+                        if (a.u2_part) q2 += (double)U[k][i] * (double)U[k][i];
                     }
                 }
                 ob = nb;
@@ -232,6 +234,7 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
                 const unsigned v = __reduce_add_sync(0xffffffffu, nspk);
                 if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
             }
+            if (a.u2_part) u2_warp_add(a.u2_part, a.row_t ? a.row_t[r] : a.t0 + r, q2);
         }
     }
     if (active) {
@@ -305,8 +308,10 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
             const int r = rb + j;
             if (r >= a.R) break;
             unsigned spk = 0;
+            double q2 = 0.0;
             if (active) {
                 U = lif_update(U, Iv[j], o, a.lam, a.theta);
+                q2 = (double)U * (double)U;
                 o = U > a.theta ? 1.f : 0.f;
                 spk = o != 0.f ? 1u : 0u;
                 emit(r);
@@ -320,6 +325,7 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
                 const unsigned v = __reduce_add_sync(0xffffffffu, spk);
                 if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
             }
+            if (a.u2_part) u2_warp_add(a.u2_part, a.row_t ? a.row_t[r] : a.t0 + r, q2);
         }
     }
     if (active) {
@@ -721,6 +727,19 @@ __global__ void sam_finalize_kernel(const unsigned *s_part, long long *s, int T)
     long long tot = 0;
     for (int i = 0; i < 32; ++i) tot += s_part[t * 32 + i];
     s[t] = tot;
+}
+
+__global__ void sum32_f64_kernel(const double *part, double *out, int T) {
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= T) return;
+    double tot = 0.0;
+    for (int i = 0; i < 32; ++i) tot += part[t * 32 + i];
+    out[t] = tot;
+}
+
+cudaError_t launch_sum32_f64(const double *part, double *out, int T, cudaStream_t st) {
+    sum32_f64_kernel<<<(T + 255) / 256, 256, 0, st>>>(part, out, T);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st) {

@@ -129,7 +129,7 @@ def make_layers(net):
     return arr
 
 
-SAM = {"spikes": 0, "weighted": 1}
+SAM = {"spikes": 0, "weighted": 1, "l2trace": 2}
 
 
 def make_config(T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle", gamma=0.3,

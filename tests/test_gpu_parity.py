@@ -66,7 +66,10 @@ def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=Fa
     # SAM and mask (Eq.4, Eq.5)
     np.testing.assert_array_equal(m.spike_sums(), ref.s)
     np.testing.assert_array_equal(m.layer_spike_counts(), ref.counts)
-    np.testing.assert_array_equal(m.sam_values(), np.asarray(ref.sam, np.float64))  # same fp64 arithmetic
+    if sam == "l2trace":  # float64 sums of exact squares: only the summation order differs
+        np.testing.assert_allclose(m.sam_values(), np.asarray(ref.sam, np.float64), rtol=1e-12)
+    else:
+        np.testing.assert_array_equal(m.sam_values(), np.asarray(ref.sam, np.float64))  # same fp64 arithmetic
     np.testing.assert_array_equal(m.keep_mask(), ref.keep)
     # first pass and recomputed states per layer
     for l in range(len(spk)):
@@ -254,3 +257,11 @@ def test_tbptt(name, T, B, C, lam):
     """NEXT-4: truncated BPTT (Sec. III-C) on the device - per-window loss and readout, graph cut at window
     edges, state carried on - against the oracle (spikes exact, summed loss, dW)."""
     check_parity(name, T=T, B=B, C=C, p=0.0, mode="tbptt", lam=lam)
+
+
+@pytest.mark.parametrize("name,T,B,C,p", [("tiny_conv", 20, 3, 2, 50.0), ("vgg5", 20, 2, 2, 40.0),
+                                          ("fc784", 20, 4, 2, 50.0), ("tiny_resnet", 16, 2, 2, 50.0)])
+def test_sam_l2trace(name, T, B, C, p):
+    """NEXT-2, second variant: the l2 norm of the membrane trace per step (reading 25), accumulated inside every
+    forward kernel (fused conv + LIF, layer 0, scans), selects the same steps as the oracle."""
+    check_parity(name, T=T, B=B, C=C, p=p, mode="skip", sam="l2trace")

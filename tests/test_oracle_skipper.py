@@ -190,3 +190,31 @@ def test_sam_weighted_changes_the_mask_somewhere():
         if differ:
             break
     assert differ
+
+
+def test_l2trace_sam_brute_force_and_mask():
+    """NEXT-2 second variant (reading 25): s_t = ||U_t||_2 over every spiking neuron of the
+    first pass; recomputed here from the recorded membranes, and the mask is the Eq.5 rule applied to it."""
+    import synth
+    from oracle import StepConfig, train_step
+    net = synth.net_config("tiny_conv")
+    W = synth.make_weights(net)
+    T, C, p = 20, 2, 50.0
+    x, y = synth.make_inputs(net, T, 3)
+    r = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode="skip", sam="l2trace", record=True))
+    brute = np.zeros(T)
+    for t in range(T):
+        tot = 0.0
+        for U in r.first_U:
+            for v in np.asarray(U[t], np.float64).ravel():
+                tot += v * v
+        brute[t] = np.sqrt(tot)
+    np.testing.assert_allclose(r.sam, brute, rtol=1e-13)
+    S = T // C
+    for c in range(C):
+        seg = brute[c * S:(c + 1) * S]
+        thr = np.percentile(seg, p)
+        keep = seg > thr
+        keep[0] = True
+        np.testing.assert_array_equal(r.keep[c * S:(c + 1) * S], keep)
+    assert 0 < r.keep.sum() < T
