@@ -169,6 +169,22 @@ skipper_status skipper_step(skipper_ctx *ctx, const unsigned char *x_dev, const 
 skipper_status skipper_step_host(skipper_ctx *ctx, const unsigned char *x_host, const int *labels_host,
                                  float *loss_host);
 
+/* ---- on-device input encoding ----------
+ * Poisson rate coding o0_t[b][d] = [u < x[b][d] * rates[t]] with u drawn from Philox4x32-10:
+ * element e of the row-major [T][B][D] output uses word e%4 of Philox(counter = (e/4 lo, e/4 hi, 0, 0),
+ * key = (seed lo, seed hi)), u = (word >> 8) * 2^-24; x * rates[t] is one fp32 product (reading 18;
+ * oracle/encoder.py draws the identical numbers).  x_dev: float32 [B][D] intensities in [0, 1] (D = the
+ * input elements per sample), rates_dev: float32 [T]; out_dev: uint8 [T][B][D].  All device pointers. */
+skipper_status skipper_encode_poisson(const float *x_dev, const float *rates_dev, unsigned long long seed, int T,
+                                      int B, long long D, unsigned char *out_dev, void *stream);
+/* One training iteration from intensities: encodes the spikes into a context-owned buffer on the context
+ * stream, then skipper_step.  skipper_step_host_encoded: the same from host buffers (H2D of x, rates and
+ * labels inside the call, then the loss D2H) - the end-to-end user call. */
+skipper_status skipper_step_encoded(skipper_ctx *ctx, const float *x_dev, const float *rates_dev, unsigned long long seed,
+                                    const int *labels_dev, float *loss_host);
+skipper_status skipper_step_host_encoded(skipper_ctx *ctx, const float *x_host, const float *rates_host,
+                                         unsigned long long seed, const int *labels_host, float *loss_host);
+
 /* ---- data parallelism (batch-sharded) ----------
  * comm_unique_id: rank 0 creates the NCCL id; the caller broadcasts it.  comm_init: every rank joins
  * the library-owned communicator (world == 1 builds a one-rank communicator: the same schedule runs and

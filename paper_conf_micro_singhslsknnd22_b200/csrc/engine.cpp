@@ -120,6 +120,8 @@ struct skipper_ctx {
     size_t dw_total = 0;
     unsigned char *x_stage = nullptr;
     int *y_stage = nullptr;
+    unsigned char *x_enc = nullptr;                           // on-device encoded spikes [T][B][D]
+    float *img_stage = nullptr, *rates_stage = nullptr;       // host-encoded path staging
     // host-side step state
     std::vector<long long> s_host;         // Eq.4 spike sums [T]
     std::vector<long long> counts_host;    // per-layer spike counts [(Ls + 1)][T], row 0 = input
@@ -745,6 +747,9 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         dev_free(c, c->kept_dev, (size_t)c->T * 4);
         dev_free(c, c->x_stage, (size_t)c->T * c->B * c->in_elems);
         dev_free(c, c->y_stage, (size_t)c->B * 4);
+        dev_free(c, c->x_enc, (size_t)c->T * c->B * c->in_elems);
+        dev_free(c, c->img_stage, (size_t)c->B * c->in_elems * 4);
+        dev_free(c, c->rates_stage, (size_t)c->T * 4);
     }
     if (c->st) cudaStreamSynchronize(c->st);
     for (auto e : c->ev_pool) cudaEventDestroy(e);
@@ -1885,12 +1890,52 @@ extern "C" skipper_status skipper_step_host(skipper_ctx *c, const unsigned char 
     const size_t xbytes = (size_t)c->T * c->B * c->in_elems;
     if (!c->x_stage) {
         CKS(alloc_arr(c, &c->x_stage, xbytes));
-        CKS(alloc_arr(c, &c->y_stage, (size_t)c->B));
     }
+    if (!c->y_stage) CKS(alloc_arr(c, &c->y_stage, (size_t)c->B));
     CK(cudaMemcpyAsync(c->x_stage, x_host, xbytes, cudaMemcpyHostToDevice, c->st));
     CK(cudaMemcpyAsync(c->y_stage, labels_host, (size_t)c->B * 4, cudaMemcpyHostToDevice, c->st));
     float loss = 0.f;
     CKS(skipper_step(c, c->x_stage, c->y_stage, &loss));
+    if (loss_host) *loss_host = loss;
+    return SKIPPER_OK;
+}
+
+// ------------------------------------------------------------------------------------ encoder (NEXT-3)
+extern "C" skipper_status skipper_encode_poisson(const float *x_dev, const float *rates_dev, unsigned long long seed,
+                                                 int T, int B, long long D, unsigned char *out_dev, void *stream) {
+    if (!x_dev || !rates_dev || !out_dev || T < 0 || B < 0 || D < 0)
+        return fail(nullptr, SKIPPER_EINVAL, "encode_poisson: bad arguments");
+    const cudaError_t e = sk::launch_poisson_encode(x_dev, rates_dev, seed, T, B, D, out_dev, static_cast<cudaStream_t>(stream));
+    if (e != cudaSuccess) return fail(nullptr, SKIPPER_ECUDA, "encode_poisson: %s", cudaGetErrorString(e));
+    return SKIPPER_OK;
+}
+
+extern "C" skipper_status skipper_step_encoded(skipper_ctx *c, const float *x_dev, const float *rates_dev,
+                                               unsigned long long seed, const int *labels_dev, float *loss_host) {
+    CKS(check_ctx(c));
+    if (!x_dev || !rates_dev || !labels_dev) return fail(c, SKIPPER_EINVAL, "null input");
+    if (!c->x_enc) CKS(alloc_arr(c, &c->x_enc, (size_t)c->T * c->B * c->in_elems));
+    {
+        ProfScope ps(c, K_STAGE, (double)c->B * c->in_elems * 4 + (double)c->T * c->B * c->in_elems, 0);
+        CK(sk::launch_poisson_encode(x_dev, rates_dev, seed, c->T, c->B, c->in_elems, c->x_enc, c->st));
+    }
+    return skipper_step(c, c->x_enc, labels_dev, loss_host);
+}
+
+extern "C" skipper_status skipper_step_host_encoded(skipper_ctx *c, const float *x_host, const float *rates_host,
+                                                    unsigned long long seed, const int *labels_host, float *loss_host) {
+    CKS(check_ctx(c));
+    if (!x_host || !rates_host || !labels_host) return fail(c, SKIPPER_EINVAL, "null host input");
+    if (!c->img_stage) {
+        CKS(alloc_arr(c, &c->img_stage, (size_t)c->B * c->in_elems));
+        CKS(alloc_arr(c, &c->rates_stage, (size_t)c->T));
+    }
+    if (!c->y_stage) CKS(alloc_arr(c, &c->y_stage, (size_t)c->B));
+    CK(cudaMemcpyAsync(c->img_stage, x_host, (size_t)c->B * c->in_elems * 4, cudaMemcpyHostToDevice, c->st));
+    CK(cudaMemcpyAsync(c->rates_stage, rates_host, (size_t)c->T * 4, cudaMemcpyHostToDevice, c->st));
+    CK(cudaMemcpyAsync(c->y_stage, labels_host, (size_t)c->B * 4, cudaMemcpyHostToDevice, c->st));
+    float loss = 0.f;
+    CKS(skipper_step_encoded(c, c->img_stage, c->rates_stage, seed, c->y_stage, &loss));
     if (loss_host) *loss_host = loss;
     return SKIPPER_OK;
 }

@@ -83,6 +83,9 @@ cudaError_t launch_gap_expand(const float *g, float *out, int B, int P, int C, c
 cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s);
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st);
+// Poisson rate encoder (NEXT-3): out[t][b][d] = [u < x[b][d] * rates[t]], u from Philox4x32-10
+cudaError_t launch_poisson_encode(const float *x, const float *rates, unsigned long long seed, int T, int B, long long D,
+                                  uint8_t *out, cudaStream_t s);
 // u2[t] = sum of the 32 fp64 partials of row t, in slot order
 cudaError_t launch_sum32_f64(const double *part, double *out, int T, cudaStream_t st);
 

@@ -729,6 +729,49 @@ __global__ void sam_finalize_kernel(const unsigned *s_part, long long *s, int T)
     s[t] = tot;
 }
 
+// ---------------------------------------------------------------------------- Poisson encoder (NEXT-3)
+// o0_t = [u_t < x * r_t].  u from Philox4x32-10 (counter = element index / 4, key = seed),
+// u = (word >> 8) * 2^-24; x * r_t rounded once in fp32 - the oracle (oracle/encoder.py) draws the same.
+SK_DEV void philox4x32_10(uint32_t c[4], uint32_t k0, uint32_t k1) {
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c[0]), lo0 = 0xD2511F53u * c[0];
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c[2]), lo1 = 0xCD9E8D57u * c[2];
+        const uint32_t n0 = hi1 ^ c[1] ^ k0, n2 = hi0 ^ c[3] ^ k1;
+        c[0] = n0;
+        c[1] = lo1;
+        c[2] = n2;
+        c[3] = lo0;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+}
+
+__global__ void poisson_encode_kernel(const float *__restrict__ x, const float *__restrict__ rates,
+                                      unsigned long long seed, long long n, long long BD, uint8_t *__restrict__ out) {
+    const long long q = (long long)blockIdx.x * blockDim.x + threadIdx.x;  // one Philox block = 4 elements
+    if (4 * q >= n) return;
+    uint32_t c[4] = {(uint32_t)q, (uint32_t)((unsigned long long)q >> 32), 0u, 0u};
+    philox4x32_10(c, (uint32_t)seed, (uint32_t)(seed >> 32));
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const long long e = 4 * q + j;
+        if (e >= n) break;
+        const float u = (float)(c[j] >> 8) * 5.9604644775390625e-08f;  // 2^-24
+        const float thr = __fmul_rn(__ldg(x + e % BD), __ldg(rates + e / BD));
+        out[e] = u < thr ? 1 : 0;
+    }
+}
+
+cudaError_t launch_poisson_encode(const float *x, const float *rates, unsigned long long seed, int T, int B, long long D,
+                                  uint8_t *out, cudaStream_t s) {
+    const long long n = (long long)T * B * D;
+    const long long blocks = (n + 4 * 256 - 1) / (4 * 256);
+    if (n == 0) return cudaSuccess;
+    poisson_encode_kernel<<<(unsigned)blocks, 256, 0, s>>>(x, rates, seed, n, (long long)B * D, out);
+    return cudaGetLastError();
+}
+
 __global__ void sum32_f64_kernel(const double *part, double *out, int T) {
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= T) return;

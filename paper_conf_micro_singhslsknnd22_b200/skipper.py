@@ -101,6 +101,9 @@ def _load():
         "skipper_profile_num_classes": (I, []),
         "skipper_launch_count": (ct.c_longlong, [P]),
         "skipper_plan_buckets": (I, [P, I, ct.c_ulonglong, P]),
+        "skipper_encode_poisson": (I, [P, P, ct.c_ulonglong, I, I, ct.c_longlong, P, P]),
+        "skipper_step_encoded": (I, [P, P, P, ct.c_ulonglong, P, P]),
+        "skipper_step_host_encoded": (I, [P, P, P, ct.c_ulonglong, P, P]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(lib, name)
@@ -282,6 +285,20 @@ class SkipperNet:
                                       ct.byref(loss)))
         return float(loss.value)
 
+    def step_encoded(self, x, rates, seed, y, want_loss=True):
+        """Poisson-encode x (float32 [B][...] intensities) with rates (float32 [T]) on the device, then step."""
+        loss = ct.c_float(0.0)
+        self._c(lib.skipper_step_encoded(self.ctx, ct.c_void_p(x.data_ptr()), ct.c_void_p(rates.data_ptr()),
+                                         int(seed), ct.c_void_p(y.data_ptr()), ct.byref(loss) if want_loss else None))
+        return float(loss.value) if want_loss else None
+
+    def step_host_encoded(self, x_host: np.ndarray, rates_host: np.ndarray, seed: int, y_host: np.ndarray):
+        loss = ct.c_float(0.0)
+        self._c(lib.skipper_step_host_encoded(self.ctx, ct.c_void_p(x_host.ctypes.data),
+                                              ct.c_void_p(rates_host.ctypes.data), int(seed),
+                                              ct.c_void_p(y_host.ctypes.data), ct.byref(loss)))
+        return float(loss.value)
+
     def forward_segment(self, seg, pass_, x, y=None):
         self._c(lib.skipper_forward_segment(self.ctx, seg, pass_, ct.c_void_p(x.data_ptr()),
                                             ct.c_void_p(y.data_ptr()) if y is not None else None))
@@ -417,6 +434,18 @@ def k_conv_fwd(X, Wk):
     cout = Wk.shape[0]
     out = torch.empty((nb, h, w, cout), dtype=torch.float32, device=X.device)
     _check(lib.skipper_k_conv_fwd(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, _stream_handle()))
+    return out
+
+
+def encode_poisson(x, rates, seed):
+    """Device Poisson encoder: x float32 [B][D...] (cuda), rates float32 [T] -> uint8 [T][B][D...]."""
+    torch = _torch()
+    B = x.shape[0]
+    D = x[0].numel()
+    T = rates.shape[0]
+    out = torch.empty((T,) + tuple(x.shape), dtype=torch.uint8, device=x.device)
+    _check(lib.skipper_encode_poisson(ct.c_void_p(x.data_ptr()), ct.c_void_p(rates.data_ptr()), int(seed), T, B, D,
+                                      ct.c_void_p(out.data_ptr()), _stream_handle()))
     return out
 
 

@@ -265,3 +265,51 @@ def test_sam_l2trace(name, T, B, C, p):
     """NEXT-2, second variant: the l2 norm of the membrane trace per step (reading 25), accumulated inside every
     forward kernel (fused conv + LIF, layer 0, scans), selects the same steps as the oracle."""
     check_parity(name, T=T, B=B, C=C, p=p, mode="skip", sam="l2trace")
+
+
+@pytest.mark.parametrize("T,B,shape,seed", [(7, 3, (32, 32, 3), 5), (20, 4, (784,), 123456789012),
+                                            (5, 2, (128, 128, 2), 1)])
+def test_poisson_encoder_bitexact(T, B, shape, seed):
+    """NEXT-3: the device Poisson encoder draws the oracle's Philox4x32-10 numbers: spikes bit-exact."""
+    from oracle.encoder import poisson_encode
+    from paper_conf_micro_singhslsknnd22_b200 import encode_poisson
+    rng = np.random.default_rng(seed % 1000)
+    x = rng.random((B,) + shape, dtype=np.float32)
+    rates = (0.5 + 0.5 * rng.random(T)).astype(np.float32)
+    ref = poisson_encode(x.reshape(B, -1), rates, seed).reshape((T, B) + shape)
+    out = encode_poisson(torch.from_numpy(x).cuda(), torch.from_numpy(rates).cuda(), seed).cpu().numpy()
+    np.testing.assert_array_equal(out, ref)
+
+
+def test_step_encoded_equals_step_on_encoded_spikes():
+    """skipper_step_encoded / step_host_encoded = skipper_step on the oracle-encoded spikes (same loss, dW)."""
+    from oracle.encoder import poisson_encode
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    net = synth.net_config("vgg5")
+    W = synth.make_weights(net)
+    T, B, seed = 14, 2, 99
+    rng = np.random.default_rng(0)
+    img = rng.random((B, 32, 32, 3), dtype=np.float32)
+    rates = synth.envelope(np.arange(T)).astype(np.float32)
+    x = poisson_encode(img.reshape(B, -1), rates, seed).reshape(T, B, 32, 32, 3)
+    y = synth.labels(B, 10)
+    ref = train_step(net, W, x, y, StepConfig(T=T, C=2, p=40.0, mode="skip"))
+    out = []
+    for how in ("spikes", "device", "host"):
+        m = SkipperNet(net, T, C=2, p=40.0, mode="skip", batch=B)
+        m.set_weights(W)
+        if how == "spikes":
+            loss = m.step(torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda())
+        elif how == "device":
+            loss = m.step_encoded(torch.from_numpy(img).cuda(), torch.from_numpy(rates).cuda(), seed,
+                                  torch.from_numpy(y).cuda())
+        else:
+            loss = m.step_host_encoded(img, rates, seed, y)
+        np.testing.assert_array_equal(m.spike_sums(), ref.s)
+        out.append((loss, [g.cpu().numpy() for g in m.grads()]))
+        m.close()
+    for loss, grads in out:
+        assert loss == pytest.approx(ref.loss, rel=1e-5)
+        for g, r in zip(grads, ref.dW):
+            ok, msg = grad_ok(g, r)
+            assert ok, msg
