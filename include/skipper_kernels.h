@@ -40,6 +40,11 @@ int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float
 int skipper_k_conv_s(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w, int cin,
                      int cout, int sign, int stride, void *stream);
 
+/* The same contraction as skipper_k_conv_s for narrow channels with a cp.async gather producer (the 9 taps
+ * re-read through L1; no 32-byte TMA box rows): cin in {16, 32, 48, 64}, cout a multiple of 16 up to 128. */
+int skipper_k_conv_narrow(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w, int cin,
+                          int cout, int sign, int stride, void *stream);
+
 /* Fused 3x3 convolution + LIF over R timestep rows (Eq.1): for r = 0..R-1
  *   I_r = conv_fwd(X_r, Wk)  (bf16 x bf16 -> fp32, tensor cores, never written to memory)
  *   U_r = ((lam * U_{r-1}) + I_r) - theta * o_{r-1},   o_r = [U_r > theta]

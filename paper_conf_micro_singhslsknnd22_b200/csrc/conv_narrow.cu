@@ -1,0 +1,259 @@
+// conv_narrow.cu - 3x3 / pad-1 convolutions of narrow-channel (16..64) images on tcgen05, for the ResNet
+// SNN layers (reading 8): forward with stride 1 or 2, and the stride-1 dgrad (flipped taps).
+//
+// A TMA box of a 16-channel image has 32-byte rows, and the TMA unit is row-issue bound on them
+// (tools/conv_s_bench.py).  Here the activation tile of each tap is instead gathered by
+// 128 producer threads with 16-byte cp.async (.ca: the 9 taps re-read the same pixels through L1),
+// written in the no-swizzle K-major UMMA layout (one 2 KB plane per 8 channels: 128 pixel rows x 16 B,
+// 8-row core matrices 128 B apart, planes LBO apart), so a pixel shift is just a different source address.
+// The weights of all 9 taps stay resident in shared memory for the kernel's lifetime.
+//
+//   warps 0-3   producers: thread p gathers tile row p (one output pixel) for every tap
+//   warp 4      TMEM allocator + MMA issuer (tcgen05.mma M=128, N=Cout, K=16 per instruction)
+//   warps 5-8   epilogue: tcgen05.ld 32x32b -> fp32 rows of the output (one pixel row per thread)
+//
+// Y[n, y, x, co] = sum_{tap, ci} Wk[co][tap][ci] X[n, s*y + dy - 1, s*x + dx - 1, ci]  (sign = +1)
+// G[n, y, x, ci] = sum_{tap, co} Wt[ci][tap][co] D[n, y - dy + 1, x - dx + 1, co]      (sign = -1, s = 1)
+#include <algorithm>
+
+#include "common.cuh"
+#include "gemm.h"
+
+namespace sk {
+
+static constexpr int CN_PROD = 128;       // producer threads (one per tile row)
+static constexpr int CN_MMA_WARP = 4;
+static constexpr int CN_EPI_WARP0 = 5;
+static constexpr int CN_THREADS = 32 * (CN_EPI_WARP0 + 4);
+static constexpr int CN_LAG = 3;          // stages each producer thread keeps in flight before signalling
+static constexpr int CN_MAX_RING = 16;
+
+SK_DEV void cp_async16(uint32_t dst, const void *src, uint32_t src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
+SK_DEV void cp_async_wait_dyn(int n) {
+    // wait until at most n groups are pending (n in 0..CN_LAG)
+    if (n <= 0) asm volatile("cp.async.wait_group 0;" ::: "memory");
+    else if (n == 1) asm volatile("cp.async.wait_group 1;" ::: "memory");
+    else if (n == 2) asm volatile("cp.async.wait_group 2;" ::: "memory");
+    else asm volatile("cp.async.wait_group 3;" ::: "memory");
+}
+
+// K-major, no swizzle: 8-row core matrices of 16 B rows, SBO = 128 B along M/N, LBO between 8-col K chunks
+SK_DEV uint64_t cn_desc(uint32_t saddr, uint32_t lbo_bytes) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+    d |= (uint64_t)((lbo_bytes >> 4) & 0x3FFF) << 16;
+    d |= (uint64_t)(128u >> 4) << 32;
+    d |= (uint64_t)1 << 46;
+    return d;
+}
+
+template <int N>  // output channels (16..128, multiple of 16)
+__global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const NarrowConvArgs a) {
+    constexpr uint32_t TMEM_COLS = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t raw = smem_u32(smem_raw);
+    const uint32_t base = (raw + 1023u) & ~1023u;
+    const int KP = a.Cin / 8;                                 // 16-byte K planes per tap
+    const uint32_t plane_a = 128u * 16u;                      // one plane of the A tile
+    const uint32_t stage_bytes = (uint32_t)KP * plane_a;
+    const uint32_t plane_b = (uint32_t)N * 16u;
+    const uint32_t sB = base;                                 // [9][KP][N][16 B] resident weights
+    const uint32_t b_bytes = 9u * KP * plane_b;
+    const uint32_t sA = (sB + b_bytes + 1023u) & ~1023u;      // ring of A stages
+    const int ring = a.ring;
+    const uint32_t bars = sA + (uint32_t)ring * stage_bytes;
+    auto full_bar = [&](int s) { return bars + 8u * s; };
+    auto empty_bar = [&](int s) { return bars + 8u * (CN_MAX_RING + s); };
+    auto tfull_bar = [&](int i) { return bars + 8u * (2 * CN_MAX_RING + i); };
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CN_MAX_RING + 2 + i); };
+    const uint32_t tmem_slot = bars + 8u * (2 * CN_MAX_RING + 4);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const long long HW = (long long)a.H * a.W;
+    const long long M = (long long)a.nb * HW;
+    const int tiles = (int)((M + 127) / 128);
+
+    // resident weights: chunk (co, tap, k8) of Wk[co][tap][Cin] -> sB + (tap*KP + k8)*plane_b + co*16
+    {
+        const int chunks = N * 9 * KP;
+        for (int e = threadIdx.x; e < chunks; e += blockDim.x) {
+            const int k8 = e % KP, tap = (e / KP) % 9, co = e / (9 * KP);
+            const uint4 v = *reinterpret_cast<const uint4 *>(a.Wk + ((long long)co * 9 + tap) * a.Cin + 8 * k8);
+            *reinterpret_cast<uint4 *>(smem_raw + (sB - raw) + ((uint32_t)tap * KP + k8) * plane_b + (uint32_t)co * 16u) = v;
+        }
+    }
+    fence_async_shared();
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < ring; ++s) {
+            mbar_init(full_bar(s), CN_PROD);
+            mbar_init(empty_bar(s), 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(tfull_bar(i), 1);
+            mbar_init(tempty_bar(i), 4);
+        }
+        fence_mbar_init();
+    }
+    if (warp == CN_MMA_WARP) tmem_alloc<TMEM_COLS>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *reinterpret_cast<volatile uint32_t *>(smem_raw + (tmem_slot - raw));
+
+    if (warp < 4) {
+        // ------------------------------------------------------------ producers
+        const int p = threadIdx.x;  // tile row
+        int stage = 0, issued = 0, signalled = 0;
+        uint32_t phase = 0;
+        int sig_stage = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            const long long m = (long long)tile * 128 + p;
+            const bool valid = m < M;
+            const long long n = valid ? m / HW : 0;
+            const int y = valid ? (int)((m / a.W) % a.H) : 0, x = valid ? (int)(m % a.W) : 0;
+            for (int tap = 0; tap < 9; ++tap) {
+                mbar_wait(empty_bar(stage), phase ^ 1u);
+                const int dy = tap / 3 - 1, dx = tap % 3 - 1;
+                const int yi = a.sign > 0 ? a.stride * y + dy : y - dy;
+                const int xi = a.sign > 0 ? a.stride * x + dx : x - dx;
+                const bool in = valid && yi >= 0 && yi < a.Hin && xi >= 0 && xi < a.Win;
+                const uint16_t *src = in ? a.X + ((n * a.Hin + yi) * a.Win + xi) * a.Cin : a.X;
+                const uint32_t dst = sA + (uint32_t)stage * stage_bytes + (uint32_t)p * 16u;
+                for (int j = 0; j < KP; ++j) cp_async16(dst + (uint32_t)j * plane_a, src + 8 * j, in ? 16u : 0u);
+                cp_async_commit();
+                ++issued;
+                if (++stage == ring) {
+                    stage = 0;
+                    phase ^= 1u;
+                }
+                if (issued - signalled > CN_LAG) {  // the oldest pending stage has landed: publish it
+                    cp_async_wait_dyn(CN_LAG);
+                    fence_async_shared();
+                    mbar_arrive(full_bar(sig_stage));
+                    ++signalled;
+                    if (++sig_stage == ring) sig_stage = 0;
+                }
+            }
+        }
+        cp_async_wait_dyn(0);
+        fence_async_shared();
+        while (signalled < issued) {
+            mbar_arrive(full_bar(sig_stage));
+            ++signalled;
+            if (++sig_stage == ring) sig_stage = 0;
+        }
+    } else if (warp == CN_MMA_WARP) {
+        if (lane == 0) {
+            // ------------------------------------------------------------ MMA issuer
+            constexpr uint32_t idesc = umma_idesc_bf16(128, N, 0, 0);
+            int stage = 0, acc = 0;
+            uint32_t phase = 0, acc_phase = 0;
+            for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+                mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + (uint32_t)acc * N;
+                for (int tap = 0; tap < 9; ++tap) {
+                    mbar_wait(full_bar(stage), phase);
+                    tc_fence_after();
+                    const uint32_t sa = sA + (uint32_t)stage * stage_bytes;
+                    const uint32_t sb = sB + (uint32_t)tap * KP * plane_b;
+                    for (int k = 0; k < KP / 2; ++k) {  // K = 16 per instruction = two 8-channel planes
+                        const uint64_t ad = cn_desc(sa + (uint32_t)k * 2u * plane_a, plane_a);
+                        const uint64_t bd = cn_desc(sb + (uint32_t)k * 2u * plane_b, plane_b);
+                        tc_mma_f16(d_tmem, ad, bd, idesc, (tap > 0 || k > 0) ? 1u : 0u);
+                    }
+                    tc_commit(empty_bar(stage));
+                    if (++stage == ring) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                }
+                tc_commit(tfull_bar(acc));
+                acc ^= 1;
+                if (acc == 0) acc_phase ^= 1u;
+            }
+        }
+    } else {
+        // ---------------------------------------------------------------- epilogue
+        const int q = warp & 3;  // TMEM lane quadrant (warps 5, 6, 7, 8 -> 1, 2, 3, 0)
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            mbar_wait(tfull_bar(acc), acc_phase);
+            tc_fence_after();
+            const long long m = (long long)tile * 128 + q * 32 + lane;
+            const bool valid = m < M;
+            float *dst = a.Y + (valid ? m : 0) * (long long)a.Cout;
+#pragma unroll
+            for (int c = 0; c < N / 16; ++c) {
+                uint32_t r[16];
+                tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)acc * N + c * 16, r);
+                tmem_ld_wait();
+                if (valid) {
+#pragma unroll
+                    for (int i = 0; i < 16; i += 4)
+                        *reinterpret_cast<float4 *>(dst + 16 * c + i) =
+                            make_float4(__uint_as_float(r[i]), __uint_as_float(r[i + 1]), __uint_as_float(r[i + 2]),
+                                        __uint_as_float(r[i + 3]));
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(tempty_bar(acc));
+            acc ^= 1;
+            if (acc == 0) acc_phase ^= 1u;
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    if (warp == CN_MMA_WARP) tmem_dealloc<TMEM_COLS>(tmem_base);
+}
+
+bool conv_narrow_supported(int cin, int cout, int stride, int sign) {
+    if (cin % 16 || cin < 16 || cin > 64) return false;
+    if (cout % 16 || cout < 16 || cout > 128) return false;
+    if (stride != 1 && stride != 2) return false;
+    if (sign == -1 && stride != 1) return false;
+    return true;
+}
+
+template <int N>
+static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
+    const int KP = a.Cin / 8;
+    const uint32_t stage_bytes = (uint32_t)KP * 2048u;
+    const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
+    const uint32_t budget = 200u * 1024u - b_bytes;
+    a.ring = (int)std::min<uint32_t>(CN_MAX_RING, budget / stage_bytes);
+    if (a.ring < CN_LAG + 2) return cudaErrorInvalidValue;
+    const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 4) + 16;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(conv_narrow_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    const long long M = (long long)a.nb * a.H * a.W;
+    const int tiles = (int)((M + 127) / 128);
+    const int grid = std::min(tiles, num_sms);
+    if (grid <= 0) return cudaSuccess;
+    conv_narrow_kernel<N><<<grid, CN_THREADS, smem, s>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_conv_narrow(const NarrowConvArgs &a, cudaStream_t s, int num_sms) {
+    if (!conv_narrow_supported(a.Cin, a.Cout, a.stride, a.sign)) return cudaErrorInvalidValue;
+    switch (a.Cout) {
+        case 16: return launch_n<16>(a, s, num_sms);
+        case 32: return launch_n<32>(a, s, num_sms);
+        case 48: return launch_n<48>(a, s, num_sms);
+        case 64: return launch_n<64>(a, s, num_sms);
+        case 96: return launch_n<96>(a, s, num_sms);
+        case 128: return launch_n<128>(a, s, num_sms);
+    }
+    return cudaErrorInvalidValue;
+}
+
+}  // namespace sk

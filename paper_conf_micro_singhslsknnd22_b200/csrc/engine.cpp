@@ -2161,6 +2161,33 @@ extern "C" int skipper_k_conv_s(const unsigned short *X, const unsigned short *W
     return kapi_run(g, ok, stream, "conv_s");
 }
 
+extern "C" int skipper_k_conv_narrow(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w,
+                                     int cin, int cout, int sign, int stride, void *stream) {
+    if (!sk::conv_narrow_supported(cin, cout, stride, sign)) {
+        g_last_error = "conv_narrow: unsupported shape";
+        return SKIPPER_EUNSUPPORTED;
+    }
+    sk::NarrowConvArgs a{};
+    a.X = X;
+    a.Wk = Wk;
+    a.Y = Y;
+    a.nb = nb;
+    a.H = h;
+    a.W = w;
+    a.Hin = h * stride;
+    a.Win = w * stride;
+    a.Cin = cin;
+    a.Cout = cout;
+    a.stride = stride;
+    a.sign = sign;
+    const cudaError_t e = sk::launch_conv_narrow(a, static_cast<cudaStream_t>(stream), sk::device_num_sms());
+    if (e != cudaSuccess) {
+        g_last_error = std::string("conv_narrow: ") + cudaGetErrorString(e);
+        return SKIPPER_ECUDA;
+    }
+    return SKIPPER_OK;
+}
+
 extern "C" int skipper_k_num_sms(void) { return sk::device_num_sms(); }
 
 // ------------------------------------------------------------------------------------ profiling API

@@ -76,6 +76,17 @@ bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, i
 // dgrad of a stride-1 conv: sign = -1 with D as X and Wt [cin][9][cout] as Wk (as plan_conv).
 bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
                  int sign, int stride);
+// Narrow-channel conv with a cp.async gather producer (conv_narrow.cu): cin in {16, 32, 48, 64},
+// cout a multiple of 16 up to 128, stride 1 or 2 (sign +1), or the stride-1 dgrad (sign -1, Wk = Wt).
+struct NarrowConvArgs {
+    const uint16_t *X;   // [nb][Hin][Win][Cin] bf16
+    const uint16_t *Wk;  // [Cout][9][Cin] bf16
+    float *Y;            // [nb][H][W][Cout] fp32
+    int nb, H, W, Hin, Win, Cin, Cout, stride, sign;
+    int ring;            // filled by the launcher
+};
+bool conv_narrow_supported(int cin, int cout, int stride, int sign);
+cudaError_t launch_conv_narrow(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
 // conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
                      int num_sms);

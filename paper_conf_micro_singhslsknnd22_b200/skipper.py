@@ -95,6 +95,7 @@ def _load():
         "skipper_k_conv_lif": (I, [P, P, P, P, P, P, I, I, I, I, I, I, I, ct.c_float, ct.c_float, P]),
         "skipper_k_num_sms": (I, []),
         "skipper_k_conv_s": (I, [P, P, P, I, I, I, I, I, I, I, P]),
+        "skipper_k_conv_narrow": (I, [P, P, P, I, I, I, I, I, I, I, P]),
         "skipper_profile": (I, [P, I]),
         "skipper_profile_read": (I, [P, I, P, P, P, P]),
         "skipper_profile_class_name": (ct.c_char_p, [I]),
@@ -449,16 +450,17 @@ def encode_poisson(x, rates, seed):
     return out
 
 
-def k_conv_s(X, Wk, stride=1, sign=1):
+def k_conv_s(X, Wk, stride=1, sign=1, narrow=False):
     """Strided / narrow implicit conv: X [nb][s*h][s*w][cin] bf16, Wk [cout][3][3][cin] bf16 ->
-    Y [nb][h][w][cout] fp32 (sign = -1: the stride-1 dgrad form, Wk = Wt)."""
+    Y [nb][h][w][cout] fp32 (sign = -1: the stride-1 dgrad form, Wk = Wt).  narrow=True: the cp.async
+    gather kernel (skipper_k_conv_narrow) instead of the TMA-box one."""
     torch = _torch()
     nb, hi, wi, cin = X.shape
     cout = Wk.shape[0]
     h, w = hi // stride, wi // stride
     out = torch.empty((nb, h, w, cout), dtype=torch.float32, device=X.device)
-    _check(lib.skipper_k_conv_s(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, sign, stride,
-                                _stream_handle()))
+    fn = lib.skipper_k_conv_narrow if narrow else lib.skipper_k_conv_s
+    _check(fn(_ptr(X, "bf16"), _ptr(Wk, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, sign, stride, _stream_handle()))
     return out
 
 

@@ -173,8 +173,9 @@ CONV_S_SHAPES = [  # nb, output h, w, cin, cout, stride  (ResNet-DVS layers and 
     (3, 8, 8, 16, 16, 1), (5, 4, 4, 16, 32, 2), (3, 16, 16, 64, 64, 2), (2, 8, 8, 32, 16, 1)]
 
 
+@pytest.mark.parametrize("narrow", [False, True])
 @pytest.mark.parametrize("nb,h,w,cin,cout,stride", CONV_S_SHAPES)
-def test_conv_s_exact(nb, h, w, cin, cout, stride):
+def test_conv_s_exact(nb, h, w, cin, cout, stride, narrow):
     """Narrow-channel / strided implicit conv (per-tap 32B/64B-swizzled TMA boxes, TMA element strides)
     against torch conv2d(stride, padding=1) in float64: exact for spikes x grid weights."""
     from paper_conf_micro_singhslsknnd22_b200 import k_conv_s
@@ -183,12 +184,14 @@ def test_conv_s_exact(nb, h, w, cin, cout, stride):
     W = grid((cout, 3, 3, cin), gen=g)
     ref = F.conv2d(X.permute(0, 3, 1, 2).double(), W.permute(0, 3, 1, 2).double(), padding=1,
                    stride=stride).permute(0, 2, 3, 1).float()
-    out = k_conv_s(bf16_bits(X).cuda(), bf16_bits(W).cuda(), stride=stride).cpu()
+    out = k_conv_s(bf16_bits(X).cuda(), bf16_bits(W).cuda(), stride=stride, narrow=narrow).cpu()
     assert torch.equal(out, ref), (out - ref).abs().max()
 
 
-@pytest.mark.parametrize("nb,h,w,cin,cout", [(3, 64, 64, 16, 16), (2, 32, 32, 32, 32), (2, 8, 8, 32, 16)])
-def test_conv_s_dgrad_exact(nb, h, w, cin, cout):
+@pytest.mark.parametrize("narrow", [False, True])
+@pytest.mark.parametrize("nb,h,w,cin,cout", [(3, 64, 64, 16, 16), (2, 32, 32, 32, 32), (2, 8, 8, 32, 16),
+                                             (2, 16, 16, 64, 64)])
+def test_conv_s_dgrad_exact(nb, h, w, cin, cout, narrow):
     """Stride-1 dgrad through the narrow path: G = conv_transpose(D, W) = conv(D, flipped W^T)."""
     from paper_conf_micro_singhslsknnd22_b200 import k_conv_s
     g = torch.Generator().manual_seed(nb + h + cin)
@@ -197,5 +200,5 @@ def test_conv_s_dgrad_exact(nb, h, w, cin, cout):
     ref = F.conv_transpose2d(D.permute(0, 3, 1, 2).double(), W.permute(0, 3, 1, 2).double(),
                              padding=1).permute(0, 2, 3, 1).float()
     Wt = W.permute(3, 1, 2, 0).contiguous()          # [cin][3][3][cout]
-    out = k_conv_s(bf16_bits(D).cuda(), bf16_bits(Wt).cuda(), stride=1, sign=-1).cpu()
+    out = k_conv_s(bf16_bits(D).cuda(), bf16_bits(Wt).cuda(), stride=1, sign=-1, narrow=narrow).cpu()
     assert torch.equal(out, ref), (out - ref).abs().max()

@@ -23,9 +23,11 @@ def r(shape):
 for (nb, h, w, cin, cout, s) in [(960, 64, 64, 16, 16, 1), (960, 32, 32, 16, 32, 2), (960, 32, 32, 32, 32, 1),
                                  (960, 16, 16, 32, 64, 2), (960, 16, 16, 64, 64, 1)]:
     X = r((nb, h * s, w * s, cin)); Wk = r((cout, 3, 3, cin))
-    ms = bench(lambda: k_conv_s(X, Wk, stride=s))
     byt = X.numel() * 2 + nb * h * w * cout * 4
-    print(f"conv_s {nb}x{h}x{w} {cin}->{cout} s{s}: {ms*1e3:9.1f} us  {byt/ms/1e6:7.1f} GB/s", flush=True)
+    for nw in (False, True):
+        ms = bench(lambda: k_conv_s(X, Wk, stride=s, narrow=nw))
+        print(f"conv_{'narrow' if nw else 's'} {nb}x{h}x{w} {cin}->{cout} s{s}: {ms*1e3:9.1f} us  {byt/ms/1e6:7.1f} GB/s",
+              flush=True)
 # the same work as an explicit-column GEMM (what the im2col path runs after staging)
 M = 960 * 64 * 64
 A = r((M, 144)); B = r((16, 144))
