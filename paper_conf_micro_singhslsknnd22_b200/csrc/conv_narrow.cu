@@ -25,18 +25,14 @@ static constexpr int CN_PROD = 128;       // producer threads (one per tile row)
 static constexpr int CN_MMA_WARP = 4;
 static constexpr int CN_EPI_WARP0 = 5;
 static constexpr int CN_THREADS = 32 * (CN_EPI_WARP0 + 4);
-static constexpr int CN_LAG = 3;          // stages each producer thread keeps in flight before signalling
 static constexpr int CN_MAX_RING = 16;
 
 SK_DEV void cp_async16(uint32_t dst, const void *src, uint32_t src_bytes) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
-SK_DEV void cp_async_wait_dyn(int n) {
-    // wait until at most n groups are pending (n in 0..CN_LAG)
-    if (n <= 0) asm volatile("cp.async.wait_group 0;" ::: "memory");
-    else if (n == 1) asm volatile("cp.async.wait_group 1;" ::: "memory");
-    else if (n == 2) asm volatile("cp.async.wait_group 2;" ::: "memory");
-    else asm volatile("cp.async.wait_group 3;" ::: "memory");
+template <int N>
+SK_DEV void cp_async_wait_n() {  // at most N groups still pending
+    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 
 // K-major, no swizzle: 8-row core matrices of 16 B rows, SBO = 128 B along M/N, LBO between 8-col K chunks
@@ -87,7 +83,7 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
     fence_async_shared();
     if (threadIdx.x == 0) {
         for (int s = 0; s < ring; ++s) {
-            mbar_init(full_bar(s), CN_PROD);
+            mbar_init(full_bar(s), CN_PROD / 32);  // one arrival per producer warp
             mbar_init(empty_bar(s), 1);
         }
         for (int i = 0; i < 2; ++i) {
@@ -106,6 +102,7 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
         // ------------------------------------------------------------ producers
         const int p = threadIdx.x;  // tile row
         int stage = 0, issued = 0, signalled = 0;
+        const int lag = ring >= 10 ? 8 : (ring >= 6 ? 4 : 2);  // stages in flight per thread (wait_group immediates)
         uint32_t phase = 0;
         int sig_stage = 0;
         for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
@@ -128,19 +125,23 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
                     stage = 0;
                     phase ^= 1u;
                 }
-                if (issued - signalled > CN_LAG) {  // the oldest pending stage has landed: publish it
-                    cp_async_wait_dyn(CN_LAG);
+                if (issued - signalled > lag) {  // the oldest pending stage has landed: publish it
+                    if (lag >= 8) cp_async_wait_n<8>();
+                    else if (lag >= 4) cp_async_wait_n<4>();
+                    else cp_async_wait_n<2>();
                     fence_async_shared();
-                    mbar_arrive(full_bar(sig_stage));
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(full_bar(sig_stage));
                     ++signalled;
                     if (++sig_stage == ring) sig_stage = 0;
                 }
             }
         }
-        cp_async_wait_dyn(0);
+        cp_async_wait_n<0>();
         fence_async_shared();
+        __syncwarp();
         while (signalled < issued) {
-            mbar_arrive(full_bar(sig_stage));
+            if (lane == 0) mbar_arrive(full_bar(sig_stage));
             ++signalled;
             if (++sig_stage == ring) sig_stage = 0;
         }
@@ -225,9 +226,10 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const int KP = a.Cin / 8;
     const uint32_t stage_bytes = (uint32_t)KP * 2048u;
     const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
-    const uint32_t budget = 200u * 1024u - b_bytes;
-    a.ring = (int)std::min<uint32_t>(CN_MAX_RING, budget / stage_bytes);
-    if (a.ring < CN_LAG + 2) return cudaErrorInvalidValue;
+    // a 64 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
+    // producer warps (not a deeper ring per CTA) is what feeds it
+    a.ring = (int)std::min<uint32_t>(CN_MAX_RING, (64u * 1024u) / stage_bytes);
+    if (a.ring < 4) return cudaErrorInvalidValue;
     const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 4) + 16;
     static bool attr = false;
     if (!attr) {
@@ -235,9 +237,15 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
         if (e != cudaSuccess) return e;
         attr = true;
     }
+    int per_sm = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_narrow_kernel<N>, CN_THREADS, smem) != cudaSuccess ||
+        per_sm < 1)
+        per_sm = 1;
+    constexpr int tmem_cols = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
+    per_sm = std::min(per_sm, 512 / tmem_cols);  // every resident CTA holds its TMEM accumulators
     const long long M = (long long)a.nb * a.H * a.W;
     const int tiles = (int)((M + 127) / 128);
-    const int grid = std::min(tiles, num_sms);
+    const int grid = (int)std::min<long long>(tiles, (long long)num_sms * per_sm);
     if (grid <= 0) return cudaSuccess;
     conv_narrow_kernel<N><<<grid, CN_THREADS, smem, s>>>(a);
     return cudaGetLastError();

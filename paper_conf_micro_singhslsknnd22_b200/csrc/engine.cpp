@@ -36,6 +36,7 @@ struct Layer {
     int res = -1, res_to = -1;          // ResNet: residual source layer (this = receiver) / receiver (this = source)
     bool icol = false;                  // conv via explicit im2col + GEMM (narrow / strided layers)
     bool fwd_s = false, dgrad_s = false;  // icol layer whose forward / dgrad runs as the narrow implicit conv
+    bool fwd_g = false, dgrad_g = false;  // ... through the cp.async gather kernel (conv_narrow.cu)
     bool gap = false;                   // readout integrates the global average pool (reading 23)
     long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
     size_t wcount = 0;
@@ -468,6 +469,15 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
                 const bool allow = !(en && atoi(en));
                 l.fwd_s = allow && tiles && narrow_ok(l.Cin);
                 l.dgrad_s = allow && tiles && l.stride == 1 && narrow_ok(l.Cout);
+                // the gather kernel where it measured faster than the TMA boxes (tools/conv_s_bench.py):
+                // 16-channel inputs, and 32 -> <= 32
+                auto gather_ok = [](int ci, int co, int st, int sg) {
+                    return sk::conv_narrow_supported(ci, co, st, sg) && (ci == 16 || (ci == 32 && co <= 32));
+                };
+                l.fwd_g = allow && gather_ok(l.Cin, l.Cout, l.stride, 1);
+                l.dgrad_g = allow && gather_ok(l.Cout, l.Cin, 1, -1) && l.stride == 1;
+                if (l.fwd_g) l.fwd_s = false;
+                if (l.dgrad_g) l.dgrad_s = false;
             }
         } else {
             if (l.Cin % 8 || l.Cout % 8) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: fc needs cin, cout %% 8 == 0", i);
@@ -957,6 +967,25 @@ static skipper_status run_gemm(skipper_ctx *c, const sk::GemmLaunch &g, bool ok,
     return SKIPPER_OK;
 }
 
+// conv_narrow.cu arguments for layer l: forward (X = the layer input, Wk = wb) or stride-1 dgrad (X = delta,
+// Wk = the transposed shadow wt, output channels = the layer's cin)
+static sk::NarrowConvArgs narrow_args(const Layer &l, const uint16_t *X, const uint16_t *Wk, float *Y, int nb, int sign) {
+    sk::NarrowConvArgs a{};
+    a.X = X;
+    a.Wk = Wk;
+    a.Y = Y;
+    a.nb = nb;
+    a.H = l.H;
+    a.W = l.W;
+    a.Hin = sign > 0 ? l.Hin : l.H;
+    a.Win = sign > 0 ? l.Win : l.W;
+    a.Cin = sign > 0 ? l.Cin : l.Cout;
+    a.Cout = sign > 0 ? l.Cout : l.Cin;
+    a.stride = sign > 0 ? l.stride : 1;
+    a.sign = sign;
+    return a;
+}
+
 // I rows = input rows x W^T for spiking layer i over `rows` timestep rows.
 static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, float *I, int rows, int splits = -1) {
     Layer &l = c->L[i];
@@ -968,7 +997,13 @@ static skipper_status gemm_forward(skipper_ctx *c, int i, const uint16_t *in, fl
     if (i == 0 && c->in_kind == 1)  // im2col rows [nb*H*W][K0] x padded weights [cout][K0]
         ok = get_plan(c, {0, in, l.wbp, I, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 1}, g,
                       [&](sk::GemmLaunch *p) { return sk::plan_fc(p, in, l.wbp, I, nb * l.H * l.W, l.Cout, c->K0); });
-    else if (l.icol && l.fwd_s)  // strided / narrow implicit conv: per-tap TMA boxes, no column buffer
+    else if (l.icol && l.fwd_g) {  // narrow conv, cp.async gather producer
+        const double M = (double)nb * l.H * l.W;
+        ProfScope ps(c, K_GEMM_FWD, (double)nb * l.Nin * 2 + (double)l.wcount * 2 + (double)nb * l.N * 4,
+                     2.0 * M * l.Cout * 9 * l.Cin);
+        CK(sk::launch_conv_narrow(narrow_args(l, in, l.wb, I, nb, +1), c->st, c->num_sms));
+        return SKIPPER_OK;
+    } else if (l.icol && l.fwd_s)  // strided / narrow implicit conv: per-tap TMA boxes, no column buffer
         ok = get_plan(c, {7, in, l.wb, I, nb, l.Cin, l.Cout, l.H, l.W, l.stride}, g, [&](sk::GemmLaunch *p) {
             return sk::plan_conv_s(p, in, l.wb, I, nb, l.H, l.W, l.Cin, l.Cout, +1, l.stride);
         });
@@ -1578,7 +1613,12 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             c->w_pending[par] = true;
             if (last_seg) CKS(comm_after_wgrad(c, i, c->st2));
         }
-        if (i > 0 && l.icol && l.dgrad_s) {  // stride 1: g = conv(delta, flipped W^T) as a narrow implicit conv
+        if (i > 0 && l.icol && l.dgrad_g) {  // stride 1: g = conv(delta, flipped W^T), cp.async gather kernel
+            const double M = (double)nb * l.H * l.W;
+            ProfScope ps(c, K_GEMM_DGRAD, (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4,
+                         2.0 * M * l.Cin * 9 * l.Cout);
+            CK(sk::launch_conv_narrow(narrow_args(l, dcur, l.wt, c->I_buf, nb, -1), c->st, c->num_sms));
+        } else if (i > 0 && l.icol && l.dgrad_s) {  // stride 1: g = conv(delta, flipped W^T) as a narrow implicit conv
             ok = get_plan(c, {8, dcur, l.wt, c->I_buf, nb, l.Cout, l.Cin, l.H, l.W, -1}, g, [&](sk::GemmLaunch *p) {
                 return sk::plan_conv_s(p, dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cout, l.Cin, -1, 1);
             });
