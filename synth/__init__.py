@@ -13,5 +13,5 @@ Both sides (oracle/ and the CUDA path) receive the exact same arrays.
 """
 from .configs import NETS, net_config, workload, WORKLOADS  # noqa: F401
 from .inputs import (  # noqa: F401
-    grid_weights, poisson_frames, dvs_frames, labels, make_inputs, make_weights,
+    grid_weights, poisson_frames, dvs_frames, labels, make_inputs, make_weights, envelope, weight_shape,
 )
