@@ -313,3 +313,79 @@ def test_step_encoded_equals_step_on_encoded_spikes():
         for g, r in zip(grads, ref.dW):
             ok, msg = grad_ok(g, r)
             assert ok, msg
+
+
+# ---- BASELINE.json full sizes, in the configuration bench.py times (sampled outputs + properties)
+
+def _full_size_gpu(wl):
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    net = synth.net_config(wl["net"])
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, wl["T"], wl["B"])
+    m = SkipperNet(net, wl["T"], C=wl["C"], p=wl["p"], mode="skip", batch=wl["B"], debug_record=True)
+    m.set_weights(W)
+    loss = m.step(torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda())
+    return net, W, x, y, m, loss
+
+
+def _check_sampled(net, W, x, y, m, wl, samples, keep):
+    """First-pass and recomputed states of sampled batch elements against the oracle run on those samples
+    alone with the keep mask imposed (the recompute of a sample depends only on its input and the mask)."""
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    ref = train_step(net, W, np.ascontiguousarray(x[:, samples]), y[samples],
+                     StepConfig(T=wl["T"], C=wl["C"], p=wl["p"], mode="skip", keep=keep, global_batch=wl["B"],
+                                record=True))
+    for l in range(len(spk)):
+        for which, arr, exact in ((1, ref.first_o, True), (3, ref.rec_o, True), (0, ref.first_U, False),
+                                  (2, ref.rec_U, False)):
+            got = m.debug(which, l)[:, samples].cpu().numpy()
+            if exact:
+                assert np.array_equal(got, arr[l]), f"layer {l} debug {which}: {np.count_nonzero(got != arr[l])} differ"
+            else:
+                np.testing.assert_allclose(got, arr[l], rtol=1e-5, atol=1e-6)
+    return ref
+
+
+@pytest.mark.parametrize("name,samples", [("cfg2_vgg5", [0, 31, 63]), ("cfg4_resnet_dvs", [0, 31])])
+def test_full_size_sampled_parity(name, samples):
+    """cfg 2 (VGG-5, T=100, B=64, C=10, p=40) and cfg 4 (ResNet-20 DVS, T=300, B=32, C=5, p=50) at full size:
+    s_t, per-layer counts, keep mask and loss against the oracle's full-batch first pass (computed in batch
+    slices on the host cores); first-pass and recomputed spikes / membranes of sampled batch elements."""
+    from _oracle_pool import full_batch_forward
+    from oracle.bptt import readout
+    from oracle.numerics import bf16_round
+    from oracle.skipper import keep_mask
+    wl = synth.workload(name)
+    net, W, x, y, m, loss = _full_size_gpu(wl)
+    counts, cnt = full_batch_forward(wl["net"], wl["T"], wl["B"], wl["C"])
+    s = counts.sum(axis=0)
+    np.testing.assert_array_equal(m.layer_spike_counts(), counts)
+    np.testing.assert_array_equal(m.spike_sums(), s)
+    keep = keep_mask(s, wl["T"], wl["C"], wl["p"])
+    np.testing.assert_array_equal(m.keep_mask(), keep)
+    ref_loss, _, _ = readout(bf16_round(W[-1]), cnt, y, wl["T"], wl["B"], bool(net["layers"][-1].get("gap")))
+    assert loss == pytest.approx(ref_loss, rel=1e-5)
+    _check_sampled(net, W, x, y, m, wl, samples, keep)
+    m.close()
+
+
+def test_full_size_sampled_vgg11():
+    """cfg 3 (VGG-11, T=200, B=128, C=5, p=50) at full size: sampled first-pass states exact against the
+    oracle (its full-batch first pass is too slow for a test), and properties at full size: the keep mask
+    is Eq.5 applied to the device's own s_t, and s_t equals the device's per-layer counts summed."""
+    from oracle.skipper import keep_mask
+    wl = synth.workload("cfg3_vgg11")
+    net, W, x, y, m, loss = _full_size_gpu(wl)
+    s = m.spike_sums()
+    np.testing.assert_array_equal(m.layer_spike_counts().sum(axis=0), s)
+    np.testing.assert_array_equal(m.keep_mask(), keep_mask(s, wl["T"], wl["C"], wl["p"]))
+    assert 0 < m.keep_mask().sum() < wl["T"] and np.isfinite(loss)
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    samples = [0, 127]
+    ref = train_step(net, W, np.ascontiguousarray(x[:, samples]), y[samples],
+                     StepConfig(T=wl["T"], C=wl["C"], p=0.0, mode="ckpt", record=True, global_batch=wl["B"]))
+    for l in range(len(spk)):
+        got = m.debug(1, l)[:, samples].cpu().numpy()
+        assert np.array_equal(got, ref.first_o[l]), f"layer {l}: {np.count_nonzero(got != ref.first_o[l])} differ"
+        np.testing.assert_allclose(m.debug(0, l)[:, samples].cpu().numpy(), ref.first_U[l], rtol=1e-5, atol=1e-6)
+    m.close()
