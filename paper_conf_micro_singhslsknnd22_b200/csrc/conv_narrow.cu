@@ -15,6 +15,8 @@
 // Y[n, y, x, co] = sum_{tap, ci} Wk[co][tap][ci] X[n, s*y + dy - 1, s*x + dx - 1, ci]  (sign = +1)
 // G[n, y, x, ci] = sum_{tap, co} Wt[ci][tap][co] D[n, y - dy + 1, x - dx + 1, co]      (sign = -1, s = 1)
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "gemm.h"
@@ -228,7 +230,7 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
     // a 64 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
     // producer warps (not a deeper ring per CTA) is what feeds it
-    a.ring = (int)std::min<uint32_t>(CN_MAX_RING, (64u * 1024u) / stage_bytes);
+    a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, (48u * 1024u) / stage_bytes));
     if (a.ring < 4) return cudaErrorInvalidValue;
     const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 4) + 16;
     static bool attr = false;
@@ -237,15 +239,18 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    int per_sm = 1;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_narrow_kernel<N>, CN_THREADS, smem) != cudaSuccess ||
-        per_sm < 1)
-        per_sm = 1;
+    // resident CTAs per SM from shared memory (228 KB per SM, 1 KB reserved per CTA), warps and registers
+    // (<= 4 x 288 threads x 48 registers); the occupancy API reports 1 here (launch bounds), so computed
+    int per_sm = (int)std::min<size_t>(4, (228u * 1024u) / (smem + 1024));
+    if (per_sm < 1) per_sm = 1;
     constexpr int tmem_cols = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
     per_sm = std::min(per_sm, 512 / tmem_cols);  // every resident CTA holds its TMEM accumulators
     const long long M = (long long)a.nb * a.H * a.W;
     const int tiles = (int)((M + 127) / 128);
     const int grid = (int)std::min<long long>(tiles, (long long)num_sms * per_sm);
+    if (getenv("SKIPPER_NARROW_DEBUG"))
+        fprintf(stderr, "[conv_narrow] N=%d cin=%d ring=%d smem=%zu per_sm=%d grid=%d tiles=%d\n", N, a.Cin, a.ring, smem,
+                per_sm, grid, tiles);
     if (grid <= 0) return cudaSuccess;
     conv_narrow_kernel<N><<<grid, CN_THREADS, smem, s>>>(a);
     return cudaGetLastError();
