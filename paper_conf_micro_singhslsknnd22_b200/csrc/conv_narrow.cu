@@ -47,8 +47,15 @@ SK_DEV uint64_t cn_desc(uint32_t saddr, uint32_t lbo_bytes) {
     return d;
 }
 
-template <int N>  // output channels (16..128, multiple of 16)
-__global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const NarrowConvArgs a) {
+SK_DEV float cn_lif(float U, float I, float o, float lam, float th) {  // Eq.1, no FMA (oracle order)
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+}
+
+// LIF = false: one conv over nb images (R = 1), fp32 output.  LIF = true: the tile is 128 pixels of one
+// timestep row; the CTA walks the segment's rows for it, and the epilogue runs Eq.1 with the membranes of
+// its pixel held in registers across the rows (conv_lif.cu's scheme for narrow layers).
+template <int N, bool LIF>  // output channels (16..128, multiple of 16; LIF: 16 or 32)
+__global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(const NarrowConvArgs a) {
     constexpr uint32_t TMEM_COLS = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
@@ -70,8 +77,11 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const long long HW = (long long)a.H * a.W;
-    const long long M = (long long)a.nb * HW;
+    const long long M = (long long)a.nb * HW;                 // output pixels per row
     const int tiles = (int)((M + 127) / 128);
+    const int R = LIF ? a.R : 1;
+    const int r_mma0 = (LIF && a.restore) ? 1 : 0;            // RECOMPUTE: row 0 is the checkpoint
+    const long long in_row = (long long)a.nb * a.Hin * a.Win * a.Cin;
 
     // resident weights: chunk (co, tap, k8) of Wk[co][tap][Cin] -> sB + (tap*KP + k8)*plane_b + co*16
     {
@@ -112,30 +122,33 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
             const bool valid = m < M;
             const long long n = valid ? m / HW : 0;
             const int y = valid ? (int)((m / a.W) % a.H) : 0, x = valid ? (int)(m % a.W) : 0;
-            for (int tap = 0; tap < 9; ++tap) {
-                mbar_wait(empty_bar(stage), phase ^ 1u);
-                const int dy = tap / 3 - 1, dx = tap % 3 - 1;
-                const int yi = a.sign > 0 ? a.stride * y + dy : y - dy;
-                const int xi = a.sign > 0 ? a.stride * x + dx : x - dx;
-                const bool in = valid && yi >= 0 && yi < a.Hin && xi >= 0 && xi < a.Win;
-                const uint16_t *src = in ? a.X + ((n * a.Hin + yi) * a.Win + xi) * a.Cin : a.X;
-                const uint32_t dst = sA + (uint32_t)stage * stage_bytes + (uint32_t)p * 16u;
-                for (int j = 0; j < KP; ++j) cp_async16(dst + (uint32_t)j * plane_a, src + 8 * j, in ? 16u : 0u);
-                cp_async_commit();
-                ++issued;
-                if (++stage == ring) {
-                    stage = 0;
-                    phase ^= 1u;
-                }
-                if (issued - signalled > lag) {  // the oldest pending stage has landed: publish it
-                    if (lag >= 8) cp_async_wait_n<8>();
-                    else if (lag >= 4) cp_async_wait_n<4>();
-                    else cp_async_wait_n<2>();
-                    fence_async_shared();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(full_bar(sig_stage));
-                    ++signalled;
-                    if (++sig_stage == ring) sig_stage = 0;
+            for (int r = r_mma0; r < R; ++r) {
+                const uint16_t *Xr = a.X + (long long)r * in_row;
+                for (int tap = 0; tap < 9; ++tap) {
+                    mbar_wait(empty_bar(stage), phase ^ 1u);
+                    const int dy = tap / 3 - 1, dx = tap % 3 - 1;
+                    const int yi = a.sign > 0 ? a.stride * y + dy : y - dy;
+                    const int xi = a.sign > 0 ? a.stride * x + dx : x - dx;
+                    const bool in = valid && yi >= 0 && yi < a.Hin && xi >= 0 && xi < a.Win;
+                    const uint16_t *src = in ? Xr + ((n * a.Hin + yi) * a.Win + xi) * a.Cin : a.X;
+                    const uint32_t dst = sA + (uint32_t)stage * stage_bytes + (uint32_t)p * 16u;
+                    for (int j = 0; j < KP; ++j) cp_async16(dst + (uint32_t)j * plane_a, src + 8 * j, in ? 16u : 0u);
+                    cp_async_commit();
+                    ++issued;
+                    if (++stage == ring) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                    if (issued - signalled > lag) {  // the oldest pending stage has landed: publish it
+                        if (lag >= 8) cp_async_wait_n<8>();
+                        else if (lag >= 4) cp_async_wait_n<4>();
+                        else cp_async_wait_n<2>();
+                        fence_async_shared();
+                        __syncwarp();
+                        if (lane == 0) mbar_arrive(full_bar(sig_stage));
+                        ++signalled;
+                        if (++sig_stage == ring) sig_stage = 0;
+                    }
                 }
             }
         }
@@ -154,32 +167,34 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
             int stage = 0, acc = 0;
             uint32_t phase = 0, acc_phase = 0;
             for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-                mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
-                tc_fence_after();
-                const uint32_t d_tmem = tmem_base + (uint32_t)acc * N;
-                for (int tap = 0; tap < 9; ++tap) {
-                    mbar_wait(full_bar(stage), phase);
+                for (int r = r_mma0; r < R; ++r) {
+                    mbar_wait(tempty_bar(acc), acc_phase ^ 1u);
                     tc_fence_after();
-                    const uint32_t sa = sA + (uint32_t)stage * stage_bytes;
-                    const uint32_t sb = sB + (uint32_t)tap * KP * plane_b;
-                    for (int k = 0; k < KP / 2; ++k) {  // K = 16 per instruction = two 8-channel planes
-                        const uint64_t ad = cn_desc(sa + (uint32_t)k * 2u * plane_a, plane_a);
-                        const uint64_t bd = cn_desc(sb + (uint32_t)k * 2u * plane_b, plane_b);
-                        tc_mma_f16(d_tmem, ad, bd, idesc, (tap > 0 || k > 0) ? 1u : 0u);
+                    const uint32_t d_tmem = tmem_base + (uint32_t)acc * N;
+                    for (int tap = 0; tap < 9; ++tap) {
+                        mbar_wait(full_bar(stage), phase);
+                        tc_fence_after();
+                        const uint32_t sa = sA + (uint32_t)stage * stage_bytes;
+                        const uint32_t sb = sB + (uint32_t)tap * KP * plane_b;
+                        for (int k = 0; k < KP / 2; ++k) {  // K = 16 per instruction = two 8-channel planes
+                            const uint64_t ad = cn_desc(sa + (uint32_t)k * 2u * plane_a, plane_a);
+                            const uint64_t bd = cn_desc(sb + (uint32_t)k * 2u * plane_b, plane_b);
+                            tc_mma_f16(d_tmem, ad, bd, idesc, (tap > 0 || k > 0) ? 1u : 0u);
+                        }
+                        tc_commit(empty_bar(stage));
+                        if (++stage == ring) {
+                            stage = 0;
+                            phase ^= 1u;
+                        }
                     }
-                    tc_commit(empty_bar(stage));
-                    if (++stage == ring) {
-                        stage = 0;
-                        phase ^= 1u;
-                    }
+                    tc_commit(tfull_bar(acc));
+                    acc ^= 1;
+                    if (acc == 0) acc_phase ^= 1u;
                 }
-                tc_commit(tfull_bar(acc));
-                acc ^= 1;
-                if (acc == 0) acc_phase ^= 1u;
             }
         }
-    } else {
-        // ---------------------------------------------------------------- epilogue
+    } else if (!LIF) {
+        // ---------------------------------------------------------------- epilogue (fp32 output)
         const int q = warp & 3;  // TMEM lane quadrant (warps 5, 6, 7, 8 -> 1, 2, 3, 0)
         int acc = 0;
         uint32_t acc_phase = 0;
@@ -208,6 +223,135 @@ __global__ void __launch_bounds__(CN_THREADS, 1) conv_narrow_kernel(const Narrow
             acc ^= 1;
             if (acc == 0) acc_phase ^= 1u;
         }
+    } else {
+        // ---------------------------------------------------------------- epilogue (Eq.1 over the rows)
+        constexpr int NW = (N + 31) / 32;
+        const int q = warp & 3;
+        const long long rs = M * N;  // neurons per row
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+            const long long m = (long long)tile * 128 + q * 32 + lane;
+            const bool valid = m < M;
+            const long long nidx = (valid ? m : 0) * N;
+            float U[N];
+            uint32_t ob[NW];
+#pragma unroll
+            for (int j = 0; j < NW; ++j) ob[j] = 0u;
+            if (valid) {
+#pragma unroll
+                for (int c = 0; c < N; c += 4) {
+                    const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nidx + c);
+                    U[c] = u.x; U[c + 1] = u.y; U[c + 2] = u.z; U[c + 3] = u.w;
+                    const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nidx + c);
+                    ob[c >> 5] |= ((o4.x ? 1u : 0u) | (o4.y ? 2u : 0u) | (o4.z ? 4u : 0u) | (o4.w ? 8u : 0u)) << (c & 31);
+                }
+            } else {
+#pragma unroll
+                for (int c = 0; c < N; ++c) U[c] = 0.f;
+            }
+            // residual source offset of this pixel (reading 8): channels [res_lo, res_lo + res_C)
+            long long roff = -1, rrs = 0;
+            if (a.res && valid) {
+                const long long n = m / HW;
+                const int y = (int)((m / a.W) % a.H), x = (int)(m % a.W);
+                rrs = (long long)a.nb * a.res_H * a.res_W * a.res_C;
+                roff = ((n * a.res_H + (long long)y * a.res_stride) * a.res_W + (long long)x * a.res_stride) * a.res_C;
+            }
+            auto bitf = [&](int c) { return (float)((ob[c >> 5] >> (c & 31)) & 1u); };
+            auto store_state = [&](float *Ud, uint8_t *od) {
+#pragma unroll
+                for (int c = 0; c < N; c += 4) {
+                    *reinterpret_cast<float4 *>(Ud + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    const uint32_t w = ob[c >> 5] >> (c & 31);
+                    *reinterpret_cast<uchar4 *>(od + c) = make_uchar4(w & 1u, (w >> 1) & 1u, (w >> 2) & 1u, (w >> 3) & 1u);
+                }
+            };
+            auto emit = [&](int r, bool counted) {
+                const long long t = a.row_t ? (long long)a.row_t[r] : (long long)a.t0 + r;
+                unsigned cnt = 0;
+                double q2 = 0.0;
+                if (valid) {
+#pragma unroll
+                    for (int j = 0; j < NW; ++j) cnt += __popc(ob[j]);
+                    uint16_t *po = a.Po_out + (long long)r * rs + nidx;
+#pragma unroll
+                    for (int c = 0; c < N; c += 8) {
+                        const uint32_t w = ob[c >> 5] >> (c & 31);
+                        uint32_t pk[4];
+#pragma unroll
+                        for (int e = 0; e < 4; ++e)
+                            pk[e] = (((w >> (2 * e)) & 1u) ? 0x3F80u : 0u) | (((w >> (2 * e + 1)) & 1u) ? 0x3F800000u : 0u);
+                        *reinterpret_cast<uint4 *>(po + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                    }
+                    if (a.U_out) {
+                        float *du = a.U_out + (long long)r * rs + nidx;
+#pragma unroll
+                        for (int c = 0; c < N; c += 4)
+                            *reinterpret_cast<float4 *>(du + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    }
+                    if (a.dbg_U) store_state(a.dbg_U + t * rs + nidx, a.dbg_o + t * rs + nidx);
+                    if (a.cnt) {  // readout input sum (last spiking layer): this thread owns these neurons
+#pragma unroll
+                        for (int c = 0; c < N; c += 4) {
+                            float4 *cp = reinterpret_cast<float4 *>(a.cnt + nidx + c);
+                            float4 v = *cp;
+                            v.x += bitf(c); v.y += bitf(c + 1); v.z += bitf(c + 2); v.w += bitf(c + 3);
+                            *cp = v;
+                        }
+                    }
+                    if (a.u2_part) {
+#pragma unroll
+                        for (int c = 0; c < N; ++c) q2 += (double)U[c] * (double)U[c];
+                    }
+                }
+                if (counted && a.s_part) {
+                    const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
+                    if (lane == 0 && v) atomicAdd(a.s_part + t * 32 + (blockIdx.x & 31), v);
+                }
+                if (counted && a.u2_part) u2_warp_add(a.u2_part, t, q2);
+            };
+            if (a.restore) emit(0, false);
+            for (int r = r_mma0; r < R; ++r) {
+                mbar_wait(tfull_bar(acc), acc_phase);
+                tc_fence_after();
+                float I[N];
+#pragma unroll
+                for (int c = 0; c < N / 16; ++c) {
+                    uint32_t rr[16];
+                    tmem_ld_32x32b_x16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)acc * N + c * 16, rr);
+                    tmem_ld_wait();
+#pragma unroll
+                    for (int i = 0; i < 16; ++i) I[16 * c + i] = __uint_as_float(rr[i]);
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(tempty_bar(acc));
+                acc ^= 1;
+                if (acc == 0) acc_phase ^= 1u;
+                if (roff >= 0) {  // I += S(a^r): exact (spikes added to the fp32 sum)
+                    const uint16_t *rp = a.res + (long long)r * rrs + roff;
+#pragma unroll
+                    for (int c = 0; c < N; ++c) {
+                        const int cs = c - a.res_lo;
+                        if (cs >= 0 && cs < a.res_C) I[c] = __fadd_rn(I[c], bf_bits2f(__ldg(rp + cs)));
+                    }
+                }
+                uint32_t nb[NW];
+#pragma unroll
+                for (int j = 0; j < NW; ++j) nb[j] = 0u;
+#pragma unroll
+                for (int c = 0; c < N; ++c) {
+                    U[c] = cn_lif(U[c], I[c], bitf(c), a.lam, a.theta);
+                    nb[c >> 5] |= (U[c] > a.theta ? 1u : 0u) << (c & 31);
+                }
+#pragma unroll
+                for (int j = 0; j < NW; ++j) ob[j] = nb[j];
+                emit(r, true);
+                if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
+            }
+            if (valid && !a.restore) store_state(a.U_state + nidx, a.o_state + nidx);
+        }
     }
     tc_fence_before();
     __syncthreads();
@@ -223,25 +367,25 @@ bool conv_narrow_supported(int cin, int cout, int stride, int sign) {
     return true;
 }
 
-template <int N>
+template <int N, bool LIF>
 static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const int KP = a.Cin / 8;
     const uint32_t stage_bytes = (uint32_t)KP * 2048u;
     const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
-    // a 64 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
+    // a 48 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
     // producer warps (not a deeper ring per CTA) is what feeds it
     a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, (48u * 1024u) / stage_bytes));
-    if (a.ring < 4) return cudaErrorInvalidValue;
     const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 4) + 16;
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(conv_narrow_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        cudaError_t e = cudaFuncSetAttribute(conv_narrow_kernel<N, LIF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             227 * 1024);
         if (e != cudaSuccess) return e;
         attr = true;
     }
-    // resident CTAs per SM from shared memory (228 KB per SM, 1 KB reserved per CTA), warps and registers
-    // (<= 4 x 288 threads x 48 registers); the occupancy API reports 1 here (launch bounds), so computed
-    int per_sm = (int)std::min<size_t>(4, (228u * 1024u) / (smem + 1024));
+    // resident CTAs per SM from shared memory (228 KB per SM, 1 KB reserved per CTA) and registers; the
+    // occupancy API reports 1 here (launch bounds), so computed
+    int per_sm = (int)std::min<size_t>(LIF ? 2 : 4, (228u * 1024u) / (smem + 1024));
     if (per_sm < 1) per_sm = 1;
     constexpr int tmem_cols = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
     per_sm = std::min(per_sm, 512 / tmem_cols);  // every resident CTA holds its TMEM accumulators
@@ -249,22 +393,38 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const int tiles = (int)((M + 127) / 128);
     const int grid = (int)std::min<long long>(tiles, (long long)num_sms * per_sm);
     if (getenv("SKIPPER_NARROW_DEBUG"))
-        fprintf(stderr, "[conv_narrow] N=%d cin=%d ring=%d smem=%zu per_sm=%d grid=%d tiles=%d\n", N, a.Cin, a.ring, smem,
-                per_sm, grid, tiles);
+        fprintf(stderr, "[conv_narrow%s] N=%d cin=%d ring=%d smem=%zu per_sm=%d grid=%d tiles=%d\n", LIF ? "_lif" : "",
+                N, a.Cin, a.ring, smem, per_sm, grid, tiles);
     if (grid <= 0) return cudaSuccess;
-    conv_narrow_kernel<N><<<grid, CN_THREADS, smem, s>>>(a);
+    conv_narrow_kernel<N, LIF><<<grid, CN_THREADS, smem, s>>>(a);
     return cudaGetLastError();
 }
 
 cudaError_t launch_conv_narrow(const NarrowConvArgs &a, cudaStream_t s, int num_sms) {
     if (!conv_narrow_supported(a.Cin, a.Cout, a.stride, a.sign)) return cudaErrorInvalidValue;
     switch (a.Cout) {
-        case 16: return launch_n<16>(a, s, num_sms);
-        case 32: return launch_n<32>(a, s, num_sms);
-        case 48: return launch_n<48>(a, s, num_sms);
-        case 64: return launch_n<64>(a, s, num_sms);
-        case 96: return launch_n<96>(a, s, num_sms);
-        case 128: return launch_n<128>(a, s, num_sms);
+        case 16: return launch_n<16, false>(a, s, num_sms);
+        case 32: return launch_n<32, false>(a, s, num_sms);
+        case 48: return launch_n<48, false>(a, s, num_sms);
+        case 64: return launch_n<64, false>(a, s, num_sms);
+        case 96: return launch_n<96, false>(a, s, num_sms);
+        case 128: return launch_n<128, false>(a, s, num_sms);
+    }
+    return cudaErrorInvalidValue;
+}
+
+bool conv_narrow_lif_supported(int cin, int cout, int stride) {
+    return conv_narrow_supported(cin, cout, stride, 1) && (cout == 16 || cout == 32);
+}
+
+cudaError_t launch_conv_narrow_lif(const NarrowConvArgs &a0, cudaStream_t s, int num_sms) {
+    NarrowConvArgs a = a0;
+    a.sign = 1;
+    if (!conv_narrow_lif_supported(a.Cin, a.Cout, a.stride) || a.R <= 0) return cudaErrorInvalidValue;
+    if (a.res && (a.res_C % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
+    switch (a.Cout) {
+        case 16: return launch_n<16, true>(a, s, num_sms);
+        case 32: return launch_n<32, true>(a, s, num_sms);
     }
     return cudaErrorInvalidValue;
 }

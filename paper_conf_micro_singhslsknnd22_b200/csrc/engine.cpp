@@ -37,6 +37,7 @@ struct Layer {
     bool icol = false;                  // conv via explicit im2col + GEMM (narrow / strided layers)
     bool fwd_s = false, dgrad_s = false;  // icol layer whose forward / dgrad runs as the narrow implicit conv
     bool fwd_g = false, dgrad_g = false;  // ... through the cp.async gather kernel (conv_narrow.cu)
+    bool nlif = false;                    // gather conv + LIF scan fused (conv_narrow.cu, LIF epilogue)
     bool gap = false;                   // readout integrates the global average pool (reading 23)
     long long N = 0, Nout = 0, Nin = 0;  // per sample: neurons, outputs (after pool), inputs
     size_t wcount = 0;
@@ -477,6 +478,8 @@ static skipper_status validate_and_shape(skipper_ctx *c, const skipper_layer *la
                 l.fwd_g = allow && gather_ok(l.Cin, l.Cout, l.stride, 1);
                 l.dgrad_g = allow && gather_ok(l.Cout, l.Cin, 1, -1) && l.stride == 1;
                 if (l.fwd_g) l.fwd_s = false;
+                const char *enl = getenv("SKIPPER_NO_NARROW_LIF");
+                l.nlif = l.fwd_g && !l.pool && sk::conv_narrow_lif_supported(l.Cin, l.Cout, l.stride) && !(enl && atoi(enl));
                 if (l.dgrad_g) l.dgrad_s = false;
             }
         } else {
@@ -1240,6 +1243,47 @@ static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16
     return SKIPPER_OK;
 }
 
+// Narrow conv layer i as one kernel: cp.async gather conv on tcgen05 + the LIF scan in its epilogue.
+static skipper_status narrow_lif_rows(skipper_ctx *c, int i, int seg, const uint16_t *in, int R, int t0,
+                                      const int *row_t, bool restore, bool record, uint16_t *out) {
+    Layer &l = c->L[i];
+    const size_t bn = (size_t)c->B * l.N;
+    sk::NarrowConvArgs a = narrow_args(l, in, l.wb, nullptr, c->B, +1);
+    a.R = R;
+    a.restore = restore ? 1 : 0;
+    a.t0 = t0;
+    a.row_t = row_t;
+    a.U_state = restore ? l.ckU + (size_t)seg * bn : l.U_run;
+    a.o_state = restore ? l.cko + (size_t)seg * bn : l.o_run;
+    a.U_out = (restore || record) ? l.Useg : nullptr;
+    a.Po_out = out;
+    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
+    a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.s_part = restore ? nullptr : spart(c, i + 1);
+    a.u2_part = restore ? nullptr : c->u2_part;
+    a.cnt = (i == c->Ls - 1) ? (restore ? c->cnt_kept : c->cnt) : nullptr;
+    a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
+    a.dbg_o = c->cfg.debug_record ? l.dbgo[restore ? 1 : 0] : nullptr;
+    a.lam = l.d.lambda;
+    a.theta = l.d.theta;
+    if (l.res >= 0) {
+        const Layer &src = c->L[l.res];
+        a.res = (restore || record) ? src.Po : c->P2[l.res % c->nP];
+        a.res_H = src.H;
+        a.res_W = src.W;
+        a.res_C = src.Cout;
+        a.res_stride = src.H / l.H;
+        a.res_lo = (l.Cout - src.Cout) / 2;
+    }
+    const double comp = R - (restore ? 1 : 0);
+    double bytes = comp * c->B * l.Nin * 2 + (double)l.wcount * 2 + (double)R * bn * 2 + bn * 10;
+    if (a.U_out) bytes += (double)R * bn * 4;
+    if (a.res) bytes += comp * c->B * c->L[l.res].N * 2;
+    ProfScope ps(c, K_CONV_LIF, bytes, 2.0 * comp * c->B * l.H * l.W * l.Cout * 9.0 * l.Cin);
+    CK(sk::launch_conv_narrow_lif(a, c->st, c->num_sms));
+    return SKIPPER_OK;
+}
+
 // Forward through all spiking layers for R rows starting at absolute time t0 (FIRST / RECORD).
 static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0, bool record) {
     // the staged layer-0 operand is needed by the first pass unless layer 0 is fused (or part of the
@@ -1264,6 +1308,10 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         }
         if (l.cfused) {
             CKS(conv_lif_rows(c, i, seg, in, R, t0, nullptr, false, record, out));
+            continue;
+        }
+        if (l.nlif) {
+            CKS(narrow_lif_rows(c, i, seg, in, R, t0, nullptr, false, record, out));
             continue;
         }
         CKS(gemm_forward(c, i, in, c->I_buf, R));
@@ -1405,6 +1453,10 @@ static skipper_status recompute_segment(skipper_ctx *c, int seg) {
         const uint16_t *in = i == 0 ? c->xg : c->L[i - 1].Po;
         if (l.cfused) {
             CKS(conv_lif_rows(c, i, seg, in, R, 0, row_t, true, false, l.Po));
+            continue;
+        }
+        if (l.nlif) {
+            CKS(narrow_lif_rows(c, i, seg, in, R, 0, row_t, true, false, l.Po));
             continue;
         }
         const size_t in_row = (size_t)c->B * (i == 0 ? c->in_row : c->L[i - 1].Nout);

@@ -79,14 +79,34 @@ bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb,
 // Narrow-channel conv with a cp.async gather producer (conv_narrow.cu): cin in {16, 32, 48, 64},
 // cout a multiple of 16 up to 128, stride 1 or 2 (sign +1), or the stride-1 dgrad (sign -1, Wk = Wt).
 struct NarrowConvArgs {
-    const uint16_t *X;   // [nb][Hin][Win][Cin] bf16
+    const uint16_t *X;   // [nb][Hin][Win][Cin] bf16 (LIF: [R][nb][Hin][Win][Cin], row r read by row r)
     const uint16_t *Wk;  // [Cout][9][Cin] bf16
-    float *Y;            // [nb][H][W][Cout] fp32
+    float *Y;            // [nb][H][W][Cout] fp32 (conv only)
     int nb, H, W, Hin, Win, Cin, Cout, stride, sign;
     int ring;            // filled by the launcher
+    // ---- fused LIF scan (launch_conv_narrow_lif): Eq.1 over the R rows of a segment in the epilogue, with
+    // the same state / output / checkpoint / SAM / residual semantics as ScanFwdArgs (kernels.h), unpooled
+    int R, restore, t0;
+    const int *row_t;
+    float *U_state;
+    uint8_t *o_state;
+    float *U_out;
+    uint16_t *Po_out;
+    float *ckU;
+    uint8_t *cko;
+    unsigned *s_part;
+    double *u2_part;
+    float *cnt;
+    float *dbg_U;
+    uint8_t *dbg_o;
+    const uint16_t *res;
+    int res_H, res_W, res_C, res_stride, res_lo;
+    float lam, theta;
 };
 bool conv_narrow_supported(int cin, int cout, int stride, int sign);
 cudaError_t launch_conv_narrow(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
+bool conv_narrow_lif_supported(int cin, int cout, int stride);
+cudaError_t launch_conv_narrow_lif(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
 // conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
                      int num_sms);
