@@ -56,7 +56,8 @@ SK_DEV float cn_lif(float U, float I, float o, float lam, float th) {  // Eq.1, 
 // its pixel held in registers across the rows (conv_lif.cu's scheme for narrow layers).
 template <int N, bool LIF>  // output channels (16..128, multiple of 16; LIF: 16 or 32)
 __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(const NarrowConvArgs a) {
-    constexpr uint32_t TMEM_COLS = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
+    constexpr int NACC = LIF ? 4 : 2;  // TMEM accumulator ring (the LIF epilogue is the slower consumer)
+    constexpr uint32_t TMEM_COLS = (NACC * N <= 32) ? 32 : (NACC * N <= 64 ? 64 : (NACC * N <= 128 ? 128 : 256));
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
     const uint32_t base = (raw + 1023u) & ~1023u;
@@ -72,8 +73,8 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(co
     auto full_bar = [&](int s) { return bars + 8u * s; };
     auto empty_bar = [&](int s) { return bars + 8u * (CN_MAX_RING + s); };
     auto tfull_bar = [&](int i) { return bars + 8u * (2 * CN_MAX_RING + i); };
-    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CN_MAX_RING + 2 + i); };
-    const uint32_t tmem_slot = bars + 8u * (2 * CN_MAX_RING + 4);
+    auto tempty_bar = [&](int i) { return bars + 8u * (2 * CN_MAX_RING + 4 + i); };
+    const uint32_t tmem_slot = bars + 8u * (2 * CN_MAX_RING + 8);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const long long HW = (long long)a.H * a.W;
@@ -98,7 +99,7 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(co
             mbar_init(full_bar(s), CN_PROD / 32);  // one arrival per producer warp
             mbar_init(empty_bar(s), 1);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < NACC; ++i) {
             mbar_init(tfull_bar(i), 1);
             mbar_init(tempty_bar(i), 4);
         }
@@ -188,8 +189,10 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(co
                         }
                     }
                     tc_commit(tfull_bar(acc));
-                    acc ^= 1;
-                    if (acc == 0) acc_phase ^= 1u;
+                    if (++acc == NACC) {
+                        acc = 0;
+                        acc_phase ^= 1u;
+                    }
                 }
             }
         }
@@ -220,8 +223,10 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(co
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(tempty_bar(acc));
-            acc ^= 1;
-            if (acc == 0) acc_phase ^= 1u;
+            if (++acc == NACC) {
+                acc = 0;
+                acc_phase ^= 1u;
+            }
         }
     } else {
         // ---------------------------------------------------------------- epilogue (Eq.1 over the rows)
@@ -327,8 +332,10 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(co
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(tempty_bar(acc));
-                acc ^= 1;
-                if (acc == 0) acc_phase ^= 1u;
+                if (++acc == NACC) {
+                    acc = 0;
+                    acc_phase ^= 1u;
+                }
                 if (roff >= 0) {  // I += S(a^r): exact (spikes added to the fp32 sum)
                     const uint16_t *rp = a.res + (long long)r * rrs + roff;
 #pragma unroll
@@ -374,8 +381,8 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
     // a 48 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
     // producer warps (not a deeper ring per CTA) is what feeds it
-    a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, (48u * 1024u) / stage_bytes));
-    const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 4) + 16;
+    a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, ((LIF ? 64u : 48u) * 1024u) / stage_bytes));
+    const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 8) + 16;
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(conv_narrow_kernel<N, LIF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -387,7 +394,8 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     // occupancy API reports 1 here (launch bounds), so computed
     int per_sm = (int)std::min<size_t>(LIF ? 2 : 4, (228u * 1024u) / (smem + 1024));
     if (per_sm < 1) per_sm = 1;
-    constexpr int tmem_cols = (2 * N <= 32) ? 32 : (2 * N <= 64 ? 64 : (2 * N <= 128 ? 128 : 256));
+    constexpr int nacc = LIF ? 4 : 2;
+    constexpr int tmem_cols = (nacc * N <= 32) ? 32 : (nacc * N <= 64 ? 64 : (nacc * N <= 128 ? 128 : 256));
     per_sm = std::min(per_sm, 512 / tmem_cols);  // every resident CTA holds its TMEM accumulators
     const long long M = (long long)a.nb * a.H * a.W;
     const int tiles = (int)((M + 127) / 128);
