@@ -614,10 +614,17 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
                           sk::layer0_bwd_supported(c->B, f.H, f.W, f.Cin, f.Cout, f.pool ? 1 : 0);
         // conv layers after the first: tensor-core GEMM + LIF scan fused (not the last spiking layer,
         // whose scan also accumulates the readout counts)
+        // The fused kernel's work unit is (128 pixels of one timestep, <= 128 channels) walking the rows of
+        // the segment in order, so its parallelism is the unit count alone: deep layers at small spatial
+        // size (VGG-11 at 4x4 / 2x2: 16-64 units) would leave most SMs idle for a long sequential K loop.
+        // Those run layer-major instead (one GEMM over all rows of the segment, then the scan).
         const char *e3 = getenv("SKIPPER_NO_CONV_FUSION");
+        const char *e4 = getenv("SKIPPER_CL_MIN_UNITS");
+        const int min_units = e4 ? atoi(e4) : (c->num_sms * 4) / 5;
         for (int i = 1; i < c->Ls - 1; ++i) {
             Layer &l = c->L[i];
-            l.cfused = l.conv && !l.icol && l.res < 0 && !(e3 && atoi(e3)) &&
+            const long long units = ((long long)c->B * l.H * l.W + 127) / 128 * (l.Cout == 64 ? 1 : l.Cout / 128);
+            l.cfused = l.conv && !l.icol && l.res < 0 && !(e3 && atoi(e3)) && units >= min_units &&
                        sk::conv_lif_supported(c->B, l.H, l.W, l.Cin, l.Cout, l.pool ? 1 : 0);
         }
     }

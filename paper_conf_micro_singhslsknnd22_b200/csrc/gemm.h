@@ -15,6 +15,9 @@ enum OperandKind {
     OP_KCONV = 1,   // K-major implicit im2col of an NHWC image, one 3x3 tap per K block
     OP_MN2D = 2,    // MN-major 2D matrix [K rows][MN], TMA boxes {64, 64}
     OP_MNCONV = 3,  // MN-major shifted NHWC image (wgrad input operand), boxes {64, W, bh, bn}
+    OP_MNSHIFT = 4, // MN-major shifted NHWC image as 2D boxes of the flattened pixels at row offset
+                    // dy*W + dx; rows whose shifted pixel leaves the image are zeroed in smem by the
+                    // MMA warp before the MMA reads them (4D boxes measured ~2x slower through TMA)
 };
 
 // OVERWRITE: plain store; ATOMIC_ADD: TMA reduce-add (split-K wgrad, accumulation over segments);

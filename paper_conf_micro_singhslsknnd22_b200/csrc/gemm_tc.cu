@@ -23,6 +23,9 @@ namespace sk {
 static constexpr int BM = 128;
 static constexpr int BK = 64;        // bf16 elements per K block = one 128-byte swizzle row
 static constexpr int NUM_THREADS = 192;
+// MN-major (weight-gradient) kernels carry a 7th warp that zero-fixes OP_MNSHIFT operand rows
+template <int MN>
+static constexpr int kThreads = MN ? 224 : 192;
 
 template <int BN>
 struct GemmCfg {
@@ -89,7 +92,7 @@ SK_DEV void mbar_wait_t(uint32_t bar, uint32_t parity, unsigned long long *acc) 
 }
 
 template <int BN, int MN, int CS>
-__global__ void __launch_bounds__(NUM_THREADS, 1)
+__global__ void __launch_bounds__(kThreads<MN>, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
                    const __grid_constant__ CUtensorMap tcm, const GemmDev g) {
     using Cfg = GemmCfg<BN>;
@@ -105,6 +108,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     auto tfull_bar = [&](int a) { return bars + 8u * (2 * MR + a); };
     auto tempty_bar = [&](int a) { return bars + 8u * (2 * MR + 2 + a); };
     const uint32_t tmem_slot = bars + 8u * (2 * MR + 4);
+    auto fixed_bar = [&](int s) { return bars + 8u * (2 * MR + 6 + s); };  // OP_MNSHIFT: rows fixed (s < STAGES)
     // ring geometry: the compile-time stages, or (narrow K blocks) g.ring stages of g.stage_stride bytes
     const int nst = g.kblk ? g.ring : STAGES;
     const uint32_t sstride = g.kblk ? g.stage_stride : Cfg::STAGE_BYTES;
@@ -124,6 +128,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
             mbar_init(full_bar(s), 1);
             mbar_init(empty_bar(s), CS);  // every CTA of the cluster frees the stage (multicast B)
         }
+        if (MN)
+            for (int s = 0; s < STAGES; ++s) mbar_init(fixed_bar(s), 1);
         for (int a = 0; a < 2; ++a) {
             mbar_init(tfull_bar(a), 1);
             mbar_init(tempty_bar(a), 4);
@@ -196,6 +202,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                         const int n0 = m0 / g.conv_hw;
                         const int y0 = (m0 % g.conv_hw) / g.conv_w;
                         tma_load_4d(sb, &tb, fb, cblk * BK, g.conv_sign * dx, y0 + g.conv_sign * dy, n0);
+                    } else if (g.b_kind == OP_MNSHIFT) {  // flattened pixels kb*64.. at the tap's row offset
+#pragma unroll
+                        for (int i = 0; i < BN / 64; ++i) {
+                            int ci0 = tc.n_t * BN + 64 * i;
+                            const int tp = ci0 / g.wg_cin;
+                            ci0 -= tp * g.wg_cin;
+                            tma_load_2d(sb + 8192u * i, &tb, fb, ci0, kb * BK + (tp / 3 - 1) * g.conv_w + (tp % 3 - 1));
+                        }
                     } else {  // OP_MNCONV: K rows kb*64.. of the image, shifted by the tap of each 64-chunk
                         const int m0 = kb * BK;
                         const int n0 = m0 / g.conv_hw;
@@ -223,6 +237,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
         if (lane == 0) {
             // ------------------------------------------------------------ MMA issuer
             constexpr uint32_t idesc = umma_idesc_bf16(BM, BN, MN, MN);
+            const bool fix = MN && g.b_kind == OP_MNSHIFT;  // stages pass through the fixer warp
             int stage = 0;
             uint32_t phase = 0;
             int acc = 0;
@@ -233,12 +248,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + acc * BN;
                 for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
+                    const uint32_t rb = fix ? fixed_bar(stage) : full_bar(stage);
                     if (wst) {  // MMA waiting on TMA data is accounted separately (slot 4)
                         unsigned long long f = 0;
-                        mbar_wait_t(full_bar(stage), phase, &f);
+                        mbar_wait_t(rb, phase, &f);
                         atomicAdd(g.stats + 4, f);
                     } else {
-                        mbar_wait(full_bar(stage), phase);
+                        mbar_wait(rb, phase);
                     }
                     tc_fence_after();
                     const uint32_t sa = base + stage * sstride;
@@ -281,6 +297,60 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                 tc_commit(tfull_bar(acc));
                 acc ^= 1;
                 if (acc == 0) acc_phase ^= 1u;
+            }
+        }
+    } else if (MN && warp == 6) {
+        // ------------------------------------------------------------ OP_MNSHIFT row fixer
+        // B chunk i of a stage holds 64 channels of one tap (dy, dx) for the 64 flattened pixels of the
+        // K block, loaded at row offset dy*W + dx: rows whose shifted pixel leaves its image hold a
+        // neighbour's pixel and are zeroed here (conv zero padding) before the MMA reads the stage.
+        if (g.b_kind == OP_MNSHIFT) {
+            const int W = g.conv_w, H = g.conv_hw / g.conv_w;
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int tile = it0; tile < total; tile += itstep) {
+                const TileCoord tc = tile_at<CS>(g, tile, rank);
+                int dxs[BN / 64], dys[BN / 64];
+#pragma unroll
+                for (int i = 0; i < BN / 64; ++i) {
+                    const int tp = (tc.n_t * BN + 64 * i) / g.wg_cin;
+                    dys[i] = tp / 3 - 1;
+                    dxs[i] = tp % 3 - 1;
+                }
+                for (int kb = tc.kb0; kb < tc.kb1; ++kb) {
+                    mbar_wait(full_bar(stage), phase);
+                    const uint32_t sb = base + stage * sstride + a_bytes;
+                    // rows lane and lane + 32: a lane zeroes its own row of every chunk whose tap moves the pixel
+                    // out of its image, 16-byte units in a lane-rotated order (the 8 lanes of a store phase hit
+                    // 8 different bank groups although their rows are 128 B apart)
+#pragma unroll
+                    for (int h2 = 0; h2 < 2; ++h2) {
+                        const int r = lane + 32 * h2;
+                        const unsigned p = (unsigned)kb * BK + (unsigned)r;
+                        const unsigned q = p / (unsigned)W;
+                        const int x = (int)(p - q * (unsigned)W);
+                        const int y = (int)(q % (unsigned)H);
+#pragma unroll
+                        for (int i = 0; i < BN / 64; ++i) {
+                            const int xs = x + dxs[i], ys = y + dys[i];
+                            if (xs < 0 || xs >= W || ys < 0 || ys >= H) {
+                                const uint32_t row = sb + 8192u * i + 128u * (uint32_t)r;
+#pragma unroll
+                                for (int j = 0; j < 8; ++j)
+                                    asm volatile("st.shared.v4.u32 [%0], {%1, %1, %1, %1};" ::"r"(row + 16u * (uint32_t)((j + lane) & 7)),
+                                                 "r"(0u)
+                                                 : "memory");
+                            }
+                        }
+                    }
+                    fence_async_shared();  // generic-proxy stores -> visible to the tensor core (async proxy)
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(fixed_bar(stage));
+                    if (++stage == nst) {
+                        stage = 0;
+                        phase ^= 1u;
+                    }
+                }
             }
         }
     } else {
@@ -513,8 +583,9 @@ bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N
            make_map_out(&g->tc, C, N, d.splits, M, (uint64_t)M * N, N);
 }
 
-static void choose_splits(GemmDev &d, int base_tiles, int num_sms) {
-    int target = 2 * num_sms;
+static void choose_splits(GemmDev &d, int base_tiles, int num_sms, int mult = 2) {
+    if (getenv("SKIPPER_SPLIT_MULT")) mult = atoi(getenv("SKIPPER_SPLIT_MULT"));  // experiments
+    int target = mult * num_sms;
     int splits = base_tiles >= target ? 1 : cdiv(target, base_tiles);
     if (splits > d.num_kb) splits = d.num_kb;
     if (splits < 1) splits = 1;
@@ -667,8 +738,11 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     const long long M = (long long)nb * h * w;
     GemmDev &d = g->d;
     d = GemmDev{};
-    // N = (tap, cin) = 9*cin columns in 256-wide tiles; each 64-column chunk is one tap's shifted box
-    g->bn = 256;
+    // N = (tap, cin) = 9*cin columns in 256-wide tiles (192-wide when that tiles 9*cin exactly and 256
+    // does not: cin = 64 -> 3 x 192 instead of 3 x 256 with a quarter-full last tile); each 64-column
+    // chunk is one tap's shifted box
+    g->bn = (9 * cin) % 256 && (9 * cin) % 192 == 0 ? 192 : 256;
+    if (getenv("SKIPPER_WG_BN")) g->bn = atoi(getenv("SKIPPER_WG_BN"));  // experiments
     g->mn_major = 1;
     g->cs = 1;
     d.m_tiles = cdiv(cout, BM);
@@ -676,9 +750,10 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     d.taps = 1;
     d.wg_cin = cin;
     d.num_kb = cdiv(M, BK);
-    choose_splits(d, d.m_tiles * d.n_tiles, num_sms);
+    choose_splits(d, d.m_tiles * d.n_tiles, num_sms, 4);  // ~4 units per CTA: measured +5-15 % over 2
     d.a_kind = OP_MN2D;
-    d.b_kind = OP_MNCONV;
+    static const bool box4d = getenv("SKIPPER_WG_4D") && atoi(getenv("SKIPPER_WG_4D"));  // experiments
+    d.b_kind = box4d ? OP_MNCONV : OP_MNSHIFT;
     d.conv_hw = h * w;
     d.conv_w = w;
     d.conv_sign = 1;
@@ -688,7 +763,9 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     d.M = cout;
     d.N = 9 * cin;
     d.store_mode = STORE_ATOMIC_ADD;
-    return make_map_2d(&g->ta, D, cout, M, 64, BK) && make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn) &&
+    const bool okb = box4d ? make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn)
+                           : make_map_2d(&g->tb, X, cin, (uint64_t)M, 64, BK);
+    return make_map_2d(&g->ta, D, cout, M, 64, BK) && okb &&
            make_map_out(&g->tc, dW, 9ull * cin, 1, cout, 9ull * cin, 9ull * cin);
 }
 
@@ -704,7 +781,7 @@ static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sm
         if (CS > 1) {
             cudaLaunchConfig_t qc{};
             qc.gridDim = dim3(CS * max_clusters);
-            qc.blockDim = dim3(NUM_THREADS);
+            qc.blockDim = dim3(kThreads<MN>);
             qc.dynamicSmemBytes = Cfg::SMEM_BYTES;
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeClusterDimension;
@@ -722,7 +799,7 @@ static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sm
     const int units = total < max_clusters ? total : max_clusters;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(units * CS);
-    cfg.blockDim = dim3(NUM_THREADS);
+    cfg.blockDim = dim3(kThreads<MN>);
     cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
     cfg.stream = stream;
     cudaLaunchAttribute attrs[1];
@@ -741,6 +818,7 @@ cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
     if (g.mn_major) {
         if (g.bn == 64) return launch_t<64, 1, 1>(g, stream, num_sms);
         if (g.bn == 128) return launch_t<128, 1, 1>(g, stream, num_sms);
+        if (g.bn == 192) return launch_t<192, 1, 1>(g, stream, num_sms);
         return launch_t<256, 1, 1>(g, stream, num_sms);
     }
     if (g.cs == 4) {
