@@ -348,7 +348,11 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
 cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
     if (a.res && (a.pool || a.H * a.W == 1 || a.res_C % 4 || a.res_lo % 4 || a.res_stride < 1)) return cudaErrorInvalidValue;
-    if (!a.pool && !a.res && a.H * a.W == 1 && (long long)a.B * a.C <= (1LL << 20)) {  // fc layers
+    // fc layers too small for 4 neurons per thread to fill the GPU (2 blocks of 256 per SM) run one neuron
+    // per thread; larger ones (VGG-11 fc4096 x B=128 over T=200 rows) take the vectorised kernel: the
+    // per-row overhead (SAM reduction, checkpoint test) is amortised over 4 neurons (cfg 3: the two
+    // 524-us fc-tail scans of the first pass drop by ~400 us together)
+    if (!a.pool && !a.res && a.H * a.W == 1 && (long long)a.B * a.C < 4LL * 2 * 148 * 256) {
         const long long rs = (long long)a.B * a.C;
         const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
         if (smem > 48 * 1024) return cudaErrorInvalidValue;
