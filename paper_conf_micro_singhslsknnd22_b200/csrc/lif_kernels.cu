@@ -381,10 +381,13 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
 }
 
 // ============================================================================ K4 reverse scan
-// One thread owns 4 neurons; CH rows of (g, U) are loaded ahead of the reverse recurrence.
+// One thread owns 4 neurons; the (g, U) loads of the next row are issued ahead of the reverse
+// recurrence of the current one.  One row per chunk at 8 resident blocks per SM measured faster than
+// two rows at 4 blocks (cfg 2 1.53 -> 1.33 ms, cfg 3 4.39 -> 3.72 ms, cfg 4 8.8 -> 7.8 ms per step):
+// the scan is latency-bound and more resident warps hide more of it than a deeper per-thread prefetch.
 template <int SPLIT>
-__global__ void __launch_bounds__(256, 4) lif_bwd_kernel(const ScanBwdArgs a) {
-    constexpr int CH = SPLIT ? 1 : 2;
+__global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanBwdArgs a) {
+    constexpr int CH = 1;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
     const long long rs = (long long)a.B * HW * C;
