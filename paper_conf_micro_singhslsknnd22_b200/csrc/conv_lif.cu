@@ -82,6 +82,7 @@ SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
 template <int BN, int POOL, int PAIR, int RESB, int HALO>
 __global__ void __launch_bounds__(CL_THREADS, 1)
     conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
+    pdl_enter();
     using Cfg = ClCfg<BN, PAIR>;
     constexpr int CW = Cfg::CW;
     constexpr int NW = BN / 32;  // spike words per pixel
@@ -529,13 +530,15 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvL
     cfg.blockDim = dim3(CL_THREADS);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = s;
-    cudaLaunchAttribute attrs[1];
+    cudaLaunchAttribute attrs[2];
     attrs[0].id = cudaLaunchAttributeClusterDimension;
     attrs[0].val.clusterDim.x = PAIR ? 2 : 1;
     attrs[0].val.clusterDim.y = 1;
     attrs[0].val.clusterDim.z = 1;
+    attrs[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attrs[1].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
     cfg.attrs = attrs;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = 2;
     return cudaLaunchKernelEx(&cfg, kern, ta, tb, a);
 }
 

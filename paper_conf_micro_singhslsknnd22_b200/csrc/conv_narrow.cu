@@ -55,7 +55,8 @@ SK_DEV float cn_lif(float U, float I, float o, float lam, float th) {  // Eq.1, 
 // timestep row; the CTA walks the segment's rows for it, and the epilogue runs Eq.1 with the membranes of
 // its pixel held in registers across the rows (conv_lif.cu's scheme for narrow layers).
 template <int N, bool LIF>  // output channels (16..128, multiple of 16; LIF: 16 or 32)
-__global__ void __launch_bounds__(CN_THREADS, LIF ? 2 : 1) conv_narrow_kernel(const NarrowConvArgs a) {
+__global__ void __launch_bounds__(CN_THREADS, LIF ? (N <= 16 ? 3 : 2) : 1) conv_narrow_kernel(const NarrowConvArgs a) {
+    pdl_enter();
     constexpr int NACC = LIF ? 4 : 2;  // TMEM accumulator ring (the LIF epilogue is the slower consumer)
     constexpr uint32_t TMEM_COLS = (NACC * N <= 32) ? 32 : (NACC * N <= 64 ? 64 : (NACC * N <= 128 ? 128 : 256));
     extern __shared__ uint8_t smem_raw[];
@@ -392,7 +393,8 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     }
     // resident CTAs per SM from shared memory (228 KB per SM, 1 KB reserved per CTA) and registers; the
     // occupancy API reports 1 here (launch bounds), so computed
-    int per_sm = (int)std::min<size_t>(LIF ? 2 : 4, (228u * 1024u) / (smem + 1024));
+    // (the 16-channel LIF variant fits 72 registers without spills: 3 resident CTAs)
+    int per_sm = (int)std::min<size_t>(LIF ? (N <= 16 ? 3 : 2) : 4, (228u * 1024u) / (smem + 1024));
     if (per_sm < 1) per_sm = 1;
     constexpr int nacc = LIF ? 4 : 2;
     constexpr int tmem_cols = (nacc * N <= 32) ? 32 : (nacc * N <= 64 ? 64 : (nacc * N <= 128 ? 128 : 256));
@@ -404,7 +406,7 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
         fprintf(stderr, "[conv_narrow%s] N=%d cin=%d ring=%d smem=%zu per_sm=%d grid=%d tiles=%d\n", LIF ? "_lif" : "",
                 N, a.Cin, a.ring, smem, per_sm, grid, tiles);
     if (grid <= 0) return cudaSuccess;
-    conv_narrow_kernel<N, LIF><<<grid, CN_THREADS, smem, s>>>(a);
+    sk_launch(conv_narrow_kernel<N, LIF>, grid, CN_THREADS, smem, s, a);
     return cudaGetLastError();
 }
 

@@ -95,6 +95,7 @@ template <int BN, int MN, int CS>
 __global__ void __launch_bounds__(kThreads<MN>, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb,
                    const __grid_constant__ CUtensorMap tcm, const GemmDev g) {
+    pdl_enter();
     using Cfg = GemmCfg<BN>;
     constexpr int STAGES = Cfg::STAGES;
     extern __shared__ uint8_t smem_raw[];
@@ -802,13 +803,15 @@ static cudaError_t launch_t(const GemmLaunch &g, cudaStream_t stream, int num_sm
     cfg.blockDim = dim3(kThreads<MN>);
     cfg.dynamicSmemBytes = Cfg::SMEM_BYTES;
     cfg.stream = stream;
-    cudaLaunchAttribute attrs[1];
+    cudaLaunchAttribute attrs[2];
     attrs[0].id = cudaLaunchAttributeClusterDimension;
     attrs[0].val.clusterDim.x = CS;
     attrs[0].val.clusterDim.y = 1;
     attrs[0].val.clusterDim.z = 1;
+    attrs[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attrs[1].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
     cfg.attrs = attrs;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = 2;
     return cudaLaunchKernelEx(&cfg, kern, g.ta, g.tb, g.tc, g.d);
 }
 
@@ -834,6 +837,11 @@ cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms) {
     if (g.bn == 64) return launch_t<64, 0, 1>(g, stream, num_sms);
     if (g.bn == 128) return launch_t<128, 0, 1>(g, stream, num_sms);
     return launch_t<256, 0, 1>(g, stream, num_sms);
+}
+
+bool pdl_enabled() {
+    static const bool on = !(getenv("SKIPPER_NO_PDL") && atoi(getenv("SKIPPER_NO_PDL")));
+    return on;
 }
 
 int device_num_sms() {

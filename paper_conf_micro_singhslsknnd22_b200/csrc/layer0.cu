@@ -100,6 +100,7 @@ SK_DEV void l0_row_pos(const L0Tile &g, int pool, int r, int &bl, int &yl, int &
 template <int NCH, int CW>
 __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
     layer0_fwd_kernel(const L0FwdArgs a, const L0Tile tg) {
+    pdl_enter();
     constexpr int N = 32 * NCH;
     constexpr int NEPI = 4 * N / CW;
     constexpr uint32_t PLANE_B = N * 16;
@@ -582,21 +583,21 @@ cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
             cudaFuncSetAttribute(layer0_fwd_kernel<2, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
             set = true;
         }
-        layer0_fwd_kernel<2, 32><<<grid, 32 * (F0_EPI_WARP0 + 8), smem, s>>>(a, g);
+        sk_launch(layer0_fwd_kernel<2, 32>, grid, 32 * (F0_EPI_WARP0 + 8), smem, s, a, g);
     } else if (a.N == 64) {
         static bool set = false;
         if (!set) {
             cudaFuncSetAttribute(layer0_fwd_kernel<2, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
             set = true;
         }
-        layer0_fwd_kernel<2, 16><<<grid, 32 * (F0_EPI_WARP0 + 16), smem, s>>>(a, g);
+        sk_launch(layer0_fwd_kernel<2, 16>, grid, 32 * (F0_EPI_WARP0 + 16), smem, s, a, g);
     } else if (a.N == 32) {
         static bool set = false;
         if (!set) {
             cudaFuncSetAttribute(layer0_fwd_kernel<1, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
             set = true;
         }
-        layer0_fwd_kernel<1, 16><<<grid, 32 * (F0_EPI_WARP0 + 8), smem, s>>>(a, g);
+        sk_launch(layer0_fwd_kernel<1, 16>, grid, 32 * (F0_EPI_WARP0 + 8), smem, s, a, g);
     } else {
         return cudaErrorInvalidValue;
     }
@@ -630,6 +631,7 @@ SK_DEV float surr_grad(float U, float th, int kind, float gamma) {
 static constexpr int LB_DWARPS = 16;  // delta warps: 4 lane quadrants x 4 chunks of 16 channels
 
 __global__ void __launch_bounds__(32 * (L0_EPI_WARP0 + LB_DWARPS), 1) layer0_bwd_kernel(const L0BwdArgs a, const L0Tile tg) {
+    pdl_enter();
     constexpr int N = 64;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t raw = smem_u32(smem_raw);
@@ -875,7 +877,7 @@ cudaError_t launch_layer0_bwd(const L0BwdArgs &a, cudaStream_t s, int num_sms) {
         set = true;
     }
     const int grid = tiles < num_sms ? tiles : num_sms;
-    layer0_bwd_kernel<<<grid, 32 * (L0_EPI_WARP0 + LB_DWARPS), smem, s>>>(a, g);
+    sk_launch(layer0_bwd_kernel, grid, 32 * (L0_EPI_WARP0 + LB_DWARPS), smem, s, a, g);
     return cudaGetLastError();
 }
 

@@ -74,6 +74,7 @@ SK_DEV float ldg_split(const float *p, int nsplit, long long stride) {
 // go through shared-memory atomics and one global atomic per row per block at the end.
 template <int POOL, int SPLIT>
 __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFwdArgs a) {
+    pdl_enter();
     constexpr int NP = POOL ? 4 : 1;
     constexpr int CH = POOL ? 2 : (SPLIT ? 4 : 8);
     extern __shared__ unsigned s_cnt[];  // [R] block spike count per row (when a.s_part)
@@ -268,6 +269,7 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
 // the split-K partial currents of CH rows are all in flight before the recurrence consumes them.
 template <int CH, int SPLIT>
 __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a) {
+    pdl_enter();
     extern __shared__ unsigned s_cnt[];
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -357,9 +359,9 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
         const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
         if (smem > 48 * 1024) return cudaErrorInvalidValue;
         if (a.nsplit > 1)
-            lif_fwd_small_kernel<4, 1><<<(unsigned)((rs + 255) / 256), 256, smem, s>>>(a);
+            sk_launch(lif_fwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         else
-            lif_fwd_small_kernel<16, 0><<<(unsigned)((rs + 255) / 256), 256, smem, s>>>(a);
+            sk_launch(lif_fwd_small_kernel<16, 0>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         return cudaGetLastError();
     }
     const long long HW = (long long)a.H * a.W;
@@ -371,11 +373,11 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
     if (smem > 48 * 1024) return cudaErrorInvalidValue;
     const bool split = a.nsplit > 1;
     if (a.pool) {
-        if (split) lif_fwd_kernel<1, 1><<<(unsigned)blocks, threads, smem, s>>>(a);
-        else lif_fwd_kernel<1, 0><<<(unsigned)blocks, threads, smem, s>>>(a);
+        if (split) sk_launch(lif_fwd_kernel<1, 1>, (unsigned)blocks, threads, smem, s, a);
+        else sk_launch(lif_fwd_kernel<1, 0>, (unsigned)blocks, threads, smem, s, a);
     } else {
-        if (split) lif_fwd_kernel<0, 1><<<(unsigned)blocks, threads, smem, s>>>(a);
-        else lif_fwd_kernel<0, 0><<<(unsigned)blocks, threads, smem, s>>>(a);
+        if (split) sk_launch(lif_fwd_kernel<0, 1>, (unsigned)blocks, threads, smem, s, a);
+        else sk_launch(lif_fwd_kernel<0, 0>, (unsigned)blocks, threads, smem, s, a);
     }
     return cudaGetLastError();
 }
@@ -387,6 +389,7 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
 // the scan is latency-bound and more resident warps hide more of it than a deeper per-thread prefetch.
 template <int SPLIT>
 __global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanBwdArgs a) {
+    pdl_enter();
     constexpr int CH = 1;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
@@ -471,6 +474,7 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanB
 // Small unpooled layers (fc): one thread per neuron (see lif_fwd_small_kernel).
 template <int CH, int SPLIT>
 __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a) {
+    pdl_enter();
     const long long rs = (long long)a.B * a.C;
     const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (n >= rs) return;
@@ -509,16 +513,16 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
         return cudaErrorInvalidValue;
     if (!a.g_pooled && !a.res_delta && a.H * a.W == 1 && rs <= (1LL << 20)) {  // fc layers
         if (a.nsplit > 1)
-            lif_bwd_small_kernel<4, 1><<<(unsigned)((rs + 255) / 256), 256, 0, s>>>(a);
+            sk_launch(lif_bwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
         else
-            lif_bwd_small_kernel<16, 0><<<(unsigned)((rs + 255) / 256), 256, 0, s>>>(a);
+            sk_launch(lif_bwd_small_kernel<16, 0>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
         return cudaGetLastError();
     }
     const long long P = rs / 4;
     if (a.nsplit > 1)
-        lif_bwd_kernel<1><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
+        sk_launch(lif_bwd_kernel<1>, (unsigned)((P + 255) / 256), 256, 0, s, a);
     else
-        lif_bwd_kernel<0><<<(unsigned)((P + 255) / 256), 256, 0, s>>>(a);
+        sk_launch(lif_bwd_kernel<0>, (unsigned)((P + 255) / 256), 256, 0, s, a);
     return cudaGetLastError();
 }
 
@@ -529,6 +533,7 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
 __global__ void stage_rows_kernel(const uint8_t *__restrict__ x, uint16_t *__restrict__ dst, const int *rows, int t0,
                                   int R, int B, int H, int W, int C0, int kind, int K0, long long D,
                                   unsigned *s_part, int stride) {
+    pdl_enter();
     const long long per_row = kind == 1 ? (long long)B * H * W : (long long)B * D;
     const long long total = (long long)R * per_row;
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -600,7 +605,7 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
     const long long total = (long long)R * per_row;
     if (total == 0) return cudaSuccess;
     if (kind == 1 && (K0 % 8 || K0 > 64 || 9 * C0 > K0 || stride < 1 || stride > 2)) return cudaErrorInvalidValue;
-    stage_rows_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(x, dst, rows, t0, R, B, H, W, C0, kind, K0, D,
+    sk_launch(stage_rows_kernel, (unsigned)((total + 255) / 256), 256, 0, s, x, dst, rows, t0, R, B, H, W, C0, kind, K0, D,
                                                                      s_part, stride);
     return cudaGetLastError();
 }
@@ -609,6 +614,7 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
 // One thread per (output pixel, tap, 8-channel chunk): 16-byte load (or zero) -> 16-byte store.
 __global__ void im2col_bf16_kernel(const uint16_t *__restrict__ X, uint16_t *__restrict__ cols, long long total,
                                    int Hin, int Win, int Cin, int H, int W, int stride) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= total) return;
     const int C8 = Cin >> 3;
@@ -630,13 +636,14 @@ cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, 
     if (Cin % 8) return cudaErrorInvalidValue;
     const long long total = nb * H * W * 9 * (Cin / 8);
     if (total == 0) return cudaSuccess;
-    im2col_bf16_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(X, cols, total, Hin, Win, Cin, H, W, stride);
+    sk_launch(im2col_bf16_kernel, (unsigned)((total + 255) / 256), 256, 0, s, X, cols, total, Hin, Win, Cin, H, W, stride);
     return cudaGetLastError();
 }
 
 // One thread per input neuron (n, yi, xi, ci): the <= 9 tap contributions in fixed order (deterministic).
 __global__ void col2im_f32_kernel(const float *__restrict__ dcols, float *__restrict__ G, long long total, int Hin,
                                   int Win, int Cin, int H, int W, int stride) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= total) return;
     const int ci = (int)(i % Cin);
@@ -666,13 +673,14 @@ cudaError_t launch_col2im_f32(const float *dcols, float *G, long long nb, int Hi
                               int stride, cudaStream_t s) {
     const long long total = nb * Hin * Win * Cin;
     if (total == 0) return cudaSuccess;
-    col2im_f32_kernel<<<(unsigned)((total + 255) / 256), 256, 0, s>>>(dcols, G, total, Hin, Win, Cin, H, W, stride);
+    sk_launch(col2im_f32_kernel, (unsigned)((total + 255) / 256), 256, 0, s, dcols, G, total, Hin, Win, Cin, H, W, stride);
     return cudaGetLastError();
 }
 
 // Global average pool (reading 23): one thread per (b, c), positions summed in order, then / P (exact for
 // spike counts: integers < 2^24 and P a power of two in the supported networks).
 __global__ void gap_reduce_kernel(const float *__restrict__ in, float *__restrict__ out, int B, int P, int C) {
+    pdl_enter();
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= B * C) return;
     const int b = i / C, c = i % C;
@@ -682,6 +690,7 @@ __global__ void gap_reduce_kernel(const float *__restrict__ in, float *__restric
 }
 
 __global__ void gap_expand_kernel(const float *__restrict__ g, float *__restrict__ out, int B, int P, int C) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)B * P * C) return;
     const int c = (int)(i % C);
@@ -690,18 +699,19 @@ __global__ void gap_expand_kernel(const float *__restrict__ g, float *__restrict
 }
 
 cudaError_t launch_gap_reduce(const float *in, float *out, int B, int P, int C, cudaStream_t s) {
-    gap_reduce_kernel<<<(B * C + 255) / 256, 256, 0, s>>>(in, out, B, P, C);
+    sk_launch(gap_reduce_kernel, (B * C + 255) / 256, 256, 0, s, in, out, B, P, C);
     return cudaGetLastError();
 }
 
 cudaError_t launch_gap_expand(const float *g, float *out, int B, int P, int C, cudaStream_t s) {
     const long long n = (long long)B * P * C;
-    gap_expand_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(g, out, B, P, C);
+    sk_launch(gap_expand_kernel, (unsigned)((n + 255) / 256), 256, 0, s, g, out, B, P, C);
     return cudaGetLastError();
 }
 
 // dst[r][c] = bf16(src[r][c]) for c < cols, 0 for cols <= c < ld   (layer-0 weights padded to K0)
 __global__ void cast_pad_bf16_kernel(const float *src, uint16_t *dst, int rows, int cols, int ld) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)rows * ld) return;
     const int r = (int)(i / ld), c = (int)(i % ld);
@@ -710,12 +720,13 @@ __global__ void cast_pad_bf16_kernel(const float *src, uint16_t *dst, int rows, 
 
 cudaError_t launch_cast_pad_bf16(const float *src, uint16_t *dst, int rows, int cols, int ld, cudaStream_t s) {
     const long long n = (long long)rows * ld;
-    cast_pad_bf16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(src, dst, rows, cols, ld);
+    sk_launch(cast_pad_bf16_kernel, (unsigned)((n + 255) / 256), 256, 0, s, src, dst, rows, cols, ld);
     return cudaGetLastError();
 }
 
 // dst[r][c] = src[r][c] for c < cols  (padded weight gradient back to [rows][cols])
 __global__ void unpad_f32_kernel(const float *src, float *dst, int rows, int cols, int ld) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)rows * cols) return;
     const int r = (int)(i / cols), c = (int)(i % cols);
@@ -724,11 +735,12 @@ __global__ void unpad_f32_kernel(const float *src, float *dst, int rows, int col
 
 cudaError_t launch_unpad_f32(const float *src, float *dst, int rows, int cols, int ld, cudaStream_t s) {
     const long long n = (long long)rows * cols;
-    unpad_f32_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(src, dst, rows, cols, ld);
+    sk_launch(unpad_f32_kernel, (unsigned)((n + 255) / 256), 256, 0, s, src, dst, rows, cols, ld);
     return cudaGetLastError();
 }
 
 __global__ void sam_finalize_kernel(const unsigned *s_part, long long *s, int T) {
+    pdl_enter();
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= T) return;
     long long tot = 0;
@@ -756,6 +768,7 @@ SK_DEV void philox4x32_10(uint32_t c[4], uint32_t k0, uint32_t k1) {
 
 __global__ void poisson_encode_kernel(const float *__restrict__ x, const float *__restrict__ rates,
                                       unsigned long long seed, long long n, long long BD, uint8_t *__restrict__ out) {
+    pdl_enter();
     const long long q = (long long)blockIdx.x * blockDim.x + threadIdx.x;  // one Philox block = 4 elements
     if (4 * q >= n) return;
     uint32_t c[4] = {(uint32_t)q, (uint32_t)((unsigned long long)q >> 32), 0u, 0u};
@@ -775,11 +788,12 @@ cudaError_t launch_poisson_encode(const float *x, const float *rates, unsigned l
     const long long n = (long long)T * B * D;
     const long long blocks = (n + 4 * 256 - 1) / (4 * 256);
     if (n == 0) return cudaSuccess;
-    poisson_encode_kernel<<<(unsigned)blocks, 256, 0, s>>>(x, rates, seed, n, (long long)B * D, out);
+    sk_launch(poisson_encode_kernel, (unsigned)blocks, 256, 0, s, x, rates, seed, n, (long long)B * D, out);
     return cudaGetLastError();
 }
 
 __global__ void sum32_f64_kernel(const double *part, double *out, int T) {
+    pdl_enter();
     const int t = blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= T) return;
     double tot = 0.0;
@@ -788,12 +802,12 @@ __global__ void sum32_f64_kernel(const double *part, double *out, int T) {
 }
 
 cudaError_t launch_sum32_f64(const double *part, double *out, int T, cudaStream_t st) {
-    sum32_f64_kernel<<<(T + 255) / 256, 256, 0, st>>>(part, out, T);
+    sk_launch(sum32_f64_kernel, (T + 255) / 256, 256, 0, st, part, out, T);
     return cudaGetLastError();
 }
 
 cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cudaStream_t st) {
-    sam_finalize_kernel<<<(T + 255) / 256, 256, 0, st>>>(s_part, s, T);
+    sk_launch(sam_finalize_kernel, (T + 255) / 256, 256, 0, st, s_part, s, T);
     return cudaGetLastError();
 }
 
@@ -801,6 +815,7 @@ cudaError_t launch_sam_finalize(const unsigned *s_part, long long *s, int T, cud
 // z[b][k] = (1/T) sum_n W^L[k][n] cnt[b][n]: one warp per (b, k)
 __global__ void readout_z_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ cnt, float *z, int B, int D,
                                  int K, float invT) {
+    pdl_enter();
     const long long w = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int lane = threadIdx.x & 31;
     if (w >= (long long)B * K) return;
@@ -815,6 +830,7 @@ __global__ void readout_z_kernel(const uint16_t *__restrict__ WbL, const float *
 
 // softmax cross-entropy per sample (one warp per sample): loss += CE / B_global, dz
 __global__ void readout_ce_kernel(const float *z, const int *labels, float *dz, float *loss, int B, int K, float invBg) {
+    pdl_enter();
     const int b = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     const int lane = threadIdx.x & 31;
     if (b >= B) return;
@@ -836,6 +852,7 @@ __global__ void readout_ce_kernel(const float *z, const int *labels, float *dz, 
 // g_last[b][n] = (1/T) sum_k dz[b][k] W^L[k][n]: the gradient wrt the readout input, same at every t
 __global__ void readout_g_kernel(const uint16_t *__restrict__ WbL, const float *__restrict__ dz, float *g_last, int B,
                                  int D, int K, float invT) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)B * D) return;
     const int b = (int)(i / D), n = (int)(i % D);
@@ -849,15 +866,16 @@ cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int
                                 float *loss, float *g_last, int B, int D, int K, float invT, float invBg,
                                 cudaStream_t s) {
     const long long warps = (long long)B * K;
-    readout_z_kernel<<<(unsigned)((warps * 32 + 255) / 256), 256, 0, s>>>(WbL, cnt, z, B, D, K, invT);
-    readout_ce_kernel<<<(B + 7) / 8, 256, 0, s>>>(z, labels, dz, loss, B, K, invBg);
+    sk_launch(readout_z_kernel, (unsigned)((warps * 32 + 255) / 256), 256, 0, s, WbL, cnt, z, B, D, K, invT);
+    sk_launch(readout_ce_kernel, (B + 7) / 8, 256, 0, s, z, labels, dz, loss, B, K, invBg);
     const long long n = (long long)B * D;
-    readout_g_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(WbL, dz, g_last, B, D, K, invT);
+    sk_launch(readout_g_kernel, (unsigned)((n + 255) / 256), 256, 0, s, WbL, dz, g_last, B, D, K, invT);
     return cudaGetLastError();
 }
 
 __global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT,
                                      int accumulate) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= (long long)K * D) return;
     const int k = (int)(i / D), n = (int)(i % D);
@@ -869,13 +887,14 @@ __global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, flo
 cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *dWL, int B, int D, int K, float invT,
                                  cudaStream_t s, int accumulate) {
     const long long n = (long long)K * D;
-    readout_wgrad_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(dz, cnt_kept, dWL, B, D, K, invT, accumulate);
+    sk_launch(readout_wgrad_kernel, (unsigned)((n + 255) / 256), 256, 0, s, dz, cnt_kept, dWL, B, D, K, invT, accumulate);
     return cudaGetLastError();
 }
 
 // ============================================================================ Adam + shadows
 __global__ void adam_kernel(float *w, const float *g, float *m, float *v, uint16_t *wb, long long n, float lr, float b1,
                             float b2, float eps, float bc1, float bc2_sqrt) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
     const float gi = g[i];
@@ -891,23 +910,25 @@ __global__ void adam_kernel(float *w, const float *g, float *m, float *v, uint16
 cudaError_t launch_adam(float *w, const float *g, float *m, float *v, uint16_t *wb, size_t n, float lr, float b1,
                         float b2, float eps, float bc1, float bc2_sqrt, cudaStream_t s) {
     if (n == 0) return cudaSuccess;
-    adam_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1, bc2_sqrt);
+    sk_launch(adam_kernel, (unsigned)((n + 255) / 256), 256, 0, s, w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1, bc2_sqrt);
     return cudaGetLastError();
 }
 
 __global__ void cast_bf16_kernel(const float *w, uint16_t *wb, long long n) {
+    pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i < n) wb[i] = f2bf_bits(w[i]);
 }
 
 cudaError_t launch_cast_bf16(const float *w, uint16_t *wb, size_t n, cudaStream_t s) {
     if (n == 0) return cudaSuccess;
-    cast_bf16_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(w, wb, (long long)n);
+    sk_launch(cast_bf16_kernel, (unsigned)((n + 255) / 256), 256, 0, s, w, wb, (long long)n);
     return cudaGetLastError();
 }
 
 // dst[c][t][a] = src[a][t][c]
 __global__ void transpose_bf16_kernel(const uint16_t *src, uint16_t *dst, int A, int Tp, int Cc) {
+    pdl_enter();
     __shared__ uint16_t tile[32][33];
     const int t = blockIdx.z;
     const int a0 = blockIdx.y * 32, c0 = blockIdx.x * 32;
@@ -924,7 +945,7 @@ __global__ void transpose_bf16_kernel(const uint16_t *src, uint16_t *dst, int A,
 
 cudaError_t launch_transpose_bf16(const uint16_t *src, uint16_t *dst, int A, int Tp, int Cc, cudaStream_t s) {
     dim3 grid((Cc + 31) / 32, (A + 31) / 32, Tp);
-    transpose_bf16_kernel<<<grid, dim3(32, 8), 0, s>>>(src, dst, A, Tp, Cc);
+    sk_launch(transpose_bf16_kernel, grid, dim3(32, 8), 0, s, src, dst, A, Tp, Cc);
     return cudaGetLastError();
 }
 
