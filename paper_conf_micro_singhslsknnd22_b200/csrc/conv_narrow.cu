@@ -55,7 +55,7 @@ SK_DEV float cn_lif(float U, float I, float o, float lam, float th) {  // Eq.1, 
 // timestep row; the CTA walks the segment's rows for it, and the epilogue runs Eq.1 with the membranes of
 // its pixel held in registers across the rows (conv_lif.cu's scheme for narrow layers).
 template <int N, bool LIF>  // output channels (16..128, multiple of 16; LIF: 16 or 32)
-__global__ void __launch_bounds__(CN_THREADS, LIF ? (N <= 16 ? 3 : 2) : 1) conv_narrow_kernel(const NarrowConvArgs a) {
+__global__ void __launch_bounds__(CN_THREADS, LIF ? (N <= 16 ? 4 : 2) : 1) conv_narrow_kernel(const NarrowConvArgs a) {
     pdl_enter();
     constexpr int NACC = LIF ? 4 : 2;  // TMEM accumulator ring (the LIF epilogue is the slower consumer)
     constexpr uint32_t TMEM_COLS = (NACC * N <= 32) ? 32 : (NACC * N <= 64 ? 64 : (NACC * N <= 128 ? 128 : 256));
@@ -382,7 +382,9 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     const uint32_t b_bytes = ((9u * KP * N * 16u) + 1023u) & ~1023u;
     // a 48 KB ring leaves room for several CTAs per SM: the gather is latency bound, so more resident
     // producer warps (not a deeper ring per CTA) is what feeds it
-    a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, ((LIF ? 64u : 48u) * 1024u) / stage_bytes));
+    static const int lif16_ctas = getenv("SKIPPER_NARROW_LIF_CTAS") ? atoi(getenv("SKIPPER_NARROW_LIF_CTAS")) : 4;
+    const int want = LIF ? (N <= 16 ? lif16_ctas : 2) : 4;  // resident CTAs per SM aimed for
+    a.ring = (int)std::max<uint32_t>(4u, std::min<uint32_t>(CN_MAX_RING, ((want >= 4 ? 48u : 64u) * 1024u) / stage_bytes));
     const size_t smem = 1024 + b_bytes + (size_t)a.ring * stage_bytes + 8 * (2 * CN_MAX_RING + 8) + 16;
     static bool attr = false;
     if (!attr) {
@@ -393,8 +395,8 @@ static cudaError_t launch_n(NarrowConvArgs a, cudaStream_t s, int num_sms) {
     }
     // resident CTAs per SM from shared memory (228 KB per SM, 1 KB reserved per CTA) and registers; the
     // occupancy API reports 1 here (launch bounds), so computed
-    // (the 16-channel LIF variant fits 72 registers without spills: 3 resident CTAs)
-    int per_sm = (int)std::min<size_t>(LIF ? (N <= 16 ? 3 : 2) : 4, (228u * 1024u) / (smem + 1024));
+    // (the 16-channel LIF variant fits 56 registers without spills: 4 resident CTAs with a 48 KB ring)
+    int per_sm = (int)std::min<size_t>(want, (228u * 1024u) / (smem + 1024));
     if (per_sm < 1) per_sm = 1;
     constexpr int nacc = LIF ? 4 : 2;
     constexpr int tmem_cols = (nacc * N <= 32) ? 32 : (nacc * N <= 64 ? 64 : (nacc * N <= 128 ? 128 : 256));

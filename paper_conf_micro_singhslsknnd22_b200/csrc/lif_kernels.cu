@@ -612,8 +612,32 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
 
 // ---------------------------------------------------------------------------- narrow / strided convs
 // One thread per (output pixel, tap, 8-channel chunk): 16-byte load (or zero) -> 16-byte store.
-__global__ void im2col_bf16_kernel(const uint16_t *__restrict__ X, uint16_t *__restrict__ cols, long long total,
+// One thread per 16-byte chunk (8 channels) of a column row.  32-bit index math with the channel-chunk
+// count as a template constant (the 64-bit div/mod chain of a generic version made this kernel
+// integer-issue bound, 0.34 of HBM on cfg 4).
+template <int C8>
+__global__ void im2col_bf16_kernel(const uint16_t *__restrict__ X, uint16_t *__restrict__ cols, unsigned total,
                                    int Hin, int Win, int Cin, int H, int W, int stride) {
+    pdl_enter();
+    const unsigned i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= total) return;
+    const int ch = (int)(i % C8);
+    const unsigned q = i / C8;
+    const int tap = (int)(q % 9u);
+    const unsigned m = q / 9u;
+    const unsigned my = m / (unsigned)W;
+    const int x = (int)(m - my * (unsigned)W);
+    const unsigned n = my / (unsigned)H;
+    const int y = (int)(my - n * (unsigned)H);
+    const int yi = stride * y + tap / 3 - 1, xi = stride * x + tap % 3 - 1;
+    uint4 v = make_uint4(0u, 0u, 0u, 0u);
+    if (yi >= 0 && yi < Hin && xi >= 0 && xi < Win)
+        v = __ldg(reinterpret_cast<const uint4 *>(X + (((long long)n * Hin + yi) * Win + xi) * Cin) + ch);
+    reinterpret_cast<uint4 *>(cols)[i] = v;
+}
+
+__global__ void im2col_bf16_kernel_l(const uint16_t *__restrict__ X, uint16_t *__restrict__ cols, long long total,
+                                     int Hin, int Win, int Cin, int H, int W, int stride) {
     pdl_enter();
     const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= total) return;
@@ -636,20 +660,33 @@ cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, 
     if (Cin % 8) return cudaErrorInvalidValue;
     const long long total = nb * H * W * 9 * (Cin / 8);
     if (total == 0) return cudaSuccess;
-    sk_launch(im2col_bf16_kernel, (unsigned)((total + 255) / 256), 256, 0, s, X, cols, total, Hin, Win, Cin, H, W, stride);
+    const unsigned blocks = (unsigned)((total + 255) / 256);
+    if (total < (1LL << 31)) {
+        const unsigned t = (unsigned)total;
+        switch (Cin / 8) {
+            case 2: sk_launch(im2col_bf16_kernel<2>, blocks, 256, 0, s, X, cols, t, Hin, Win, Cin, H, W, stride); return cudaGetLastError();
+            case 4: sk_launch(im2col_bf16_kernel<4>, blocks, 256, 0, s, X, cols, t, Hin, Win, Cin, H, W, stride); return cudaGetLastError();
+            case 8: sk_launch(im2col_bf16_kernel<8>, blocks, 256, 0, s, X, cols, t, Hin, Win, Cin, H, W, stride); return cudaGetLastError();
+        }
+    }
+    sk_launch(im2col_bf16_kernel_l, blocks, 256, 0, s, X, cols, total, Hin, Win, Cin, H, W, stride);
     return cudaGetLastError();
 }
 
 // One thread per input neuron (n, yi, xi, ci): the <= 9 tap contributions in fixed order (deterministic).
-__global__ void col2im_f32_kernel(const float *__restrict__ dcols, float *__restrict__ G, long long total, int Hin,
+template <typename IT>
+__global__ void col2im_f32_kernel(const float *__restrict__ dcols, float *__restrict__ G, IT total, int Hin,
                                   int Win, int Cin, int H, int W, int stride) {
     pdl_enter();
-    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const IT i = (IT)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= total) return;
-    const int ci = (int)(i % Cin);
-    const long long pix = i / Cin;
-    const int xi = (int)(pix % Win), yi = (int)((pix / Win) % Hin);
-    const long long n = pix / ((long long)Hin * Win);
+    const IT pix = i / (IT)Cin;
+    const int ci = (int)(i - pix * (IT)Cin);
+    const IT py = pix / (IT)Win;
+    const int xi = (int)(pix - py * (IT)Win);
+    const IT nn = py / (IT)Hin;
+    const int yi = (int)(py - nn * (IT)Hin);
+    const long long n = (long long)nn;
     float acc = 0.f;
 #pragma unroll
     for (int dy = 0; dy < 3; ++dy) {
@@ -673,7 +710,12 @@ cudaError_t launch_col2im_f32(const float *dcols, float *G, long long nb, int Hi
                               int stride, cudaStream_t s) {
     const long long total = nb * Hin * Win * Cin;
     if (total == 0) return cudaSuccess;
-    sk_launch(col2im_f32_kernel, (unsigned)((total + 255) / 256), 256, 0, s, dcols, G, total, Hin, Win, Cin, H, W, stride);
+    if (total < (1LL << 31))  // 32-bit index math (the 64-bit div/mod chain is integer-issue bound)
+        sk_launch(col2im_f32_kernel<unsigned>, (unsigned)((total + 255) / 256), 256, 0, s, dcols, G, (unsigned)total, Hin,
+                  Win, Cin, H, W, stride);
+    else
+        sk_launch(col2im_f32_kernel<long long>, (unsigned)((total + 255) / 256), 256, 0, s, dcols, G, total, Hin, Win, Cin,
+                  H, W, stride);
     return cudaGetLastError();
 }
 
