@@ -32,6 +32,15 @@ int skipper_k_conv_dgrad(const unsigned short *D, const unsigned short *Wt, floa
                          int nb, int h, int w, int cin, int cout, void *stream);
 int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float *dW,
                          int nb, int h, int w, int cin, int cout, int accumulate, void *stream);
+/* Weight gradient of a narrow-channel 3x3 conv (cin in {16, 32}, cout in {16, 32, 64}, stride 1 or 2,
+ * pad 1; the ResNet-DVS layers of cfg 4), Eq.2's weight term without a column buffer:
+ *   dW[co][dy*3+dx][ci] (+)= sum_{nb,y,x} D[nb,y,x,co] X[nb, s*y+dy-1, s*x+dx-1, ci]
+ * D [nb][h][w][cout] and X [nb][s*h][s*w][cin] bf16 device pointers, dW [cout][9][cin] fp32 device
+ * (zeroed first unless accumulate).  w must be a multiple of 16 dividing 128 and h a multiple of
+ * min(h, 128 / w).  fp32 atomics: the summation order is not fixed (rounding-level differences).
+ * EUNSUPPORTED for other shapes, ECUDA on a launch error. */
+int skipper_k_narrow_wgrad(const unsigned short *D, const unsigned short *X, float *dW, int nb, int h, int w,
+                           int cin, int cout, int stride, int accumulate, void *stream);
 /* Strided / narrow-channel implicit conv (ResNet layers, reading 8):
  *   Y[nb,y,x,co] = sum_{dy,dx,ci} Wk[co][dy*3+dx][ci] X[nb, s*y+dy-1, s*x+dx-1, ci]   (pad 1, stride s)
  * h x w is the OUTPUT size, X is [nb][s*h][s*w][cin]; cin in {16, 32} (one 32B/64B-swizzled TMA box per

@@ -1625,7 +1625,16 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
                 CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
             }
             const long long ch = icol_chunk(c);
-            for (long long n0 = 0; n0 < nb; n0 += ch) {
+            static const bool nw_off = getenv("SKIPPER_NO_NARROW_WGRAD") && atoi(getenv("SKIPPER_NO_NARROW_WGRAD"));
+            if (!nw_off && sk::narrow_wgrad_supported(l.Cin, l.Cout, l.stride, l.H, l.W)) {
+                // no column buffer: the delta tile and the input rows it reads staged per CTA (narrow_wgrad.cu)
+                const double M = (double)nb * l.H * l.W;
+                ProfScope ps(c, K_GEMM_WGRAD, (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8,
+                             2.0 * M * l.Cout * Kw, ws);
+                CK(sk::launch_narrow_wgrad(X, dcur, l.dw, nb, l.H, l.W, l.Cin, l.Cout, l.stride, ws, c->num_sms));
+            }
+            for (long long n0 = 0; n0 < nb && (nw_off || !sk::narrow_wgrad_supported(l.Cin, l.Cout, l.stride, l.H, l.W));
+                 n0 += ch) {
                 const int nbc = (int)std::min<long long>(ch, nb - n0);
                 const int M = nbc * l.H * l.W;
                 {
@@ -2251,6 +2260,22 @@ extern "C" int skipper_k_conv_wgrad(const unsigned short *D, const unsigned shor
     sk::GemmLaunch g;
     const bool ok = sk::plan_conv_wgrad(&g, D, X, dW, nb, h, w, cin, cout, sk::device_num_sms());
     return kapi_run(g, ok, stream, "conv_wgrad");
+}
+
+extern "C" int skipper_k_narrow_wgrad(const unsigned short *D, const unsigned short *X, float *dW, int nb, int h, int w,
+                                      int cin, int cout, int stride, int accumulate, void *stream) {
+    if (!sk::narrow_wgrad_supported(cin, cout, stride, h, w)) {
+        g_last_error = "narrow_wgrad: unsupported shape";
+        return SKIPPER_EUNSUPPORTED;
+    }
+    if (!accumulate && cudaMemsetAsync(dW, 0, (size_t)cout * 9 * cin * 4, static_cast<cudaStream_t>(stream)) != cudaSuccess)
+        return SKIPPER_ECUDA;
+    if (sk::launch_narrow_wgrad(reinterpret_cast<const uint16_t *>(X), reinterpret_cast<const uint16_t *>(D), dW, nb, h, w,
+                                cin, cout, stride, static_cast<cudaStream_t>(stream), sk::device_num_sms()) != cudaSuccess) {
+        g_last_error = "narrow_wgrad: launch failed";
+        return SKIPPER_ECUDA;
+    }
+    return SKIPPER_OK;
 }
 
 extern "C" int skipper_k_conv_s(const unsigned short *X, const unsigned short *Wk, float *Y, int nb, int h, int w,

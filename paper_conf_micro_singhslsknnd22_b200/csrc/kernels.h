@@ -71,6 +71,12 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
 
 // Narrow / strided conv layers (ResNet SNN): explicit 3x3 im2col of bf16 NHWC rows,
 // cols[(n, y, x)][(dy*3+dx)*Cin + ci] = X[n][s*y+dy-1][s*x+dx-1][ci] (zero outside), Cin % 8 == 0.
+// Narrow-channel (cin 16 / 32) 3x3 conv weight gradient without a column buffer (narrow_wgrad.cu):
+// dW[cout][9][cin] += sum over the nb*H*W output pixels of D[.][cout] X_shift[.][cin]; X is the layer
+// input [nb][H*stride][W*stride][cin], D [nb][H][W][cout], both bf16.
+bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W);
+cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
+                                int cout, int stride, cudaStream_t s, int num_sms);
 cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, int Hin, int Win, int Cin, int H,
                                int W, int stride, cudaStream_t s);
 // Adjoint: G[n][yi][xi][ci] = sum_{dy,dx: s | (yi+1-dy), s | (xi+1-dx)} dcols[(n, y, x)][ci*9 + dy*3+dx]

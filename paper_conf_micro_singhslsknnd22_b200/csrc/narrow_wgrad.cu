@@ -1,0 +1,229 @@
+// narrow_wgrad.cu - weight gradient of the narrow-channel (16 / 32 input channels) 3x3 convolutions of
+// the ResNet-DVS SNN (cfg 4), stride 1 or 2, without a column buffer:
+//     dW[co][tap][ci] += sum_p delta[p][co] * X[src(p, tap)][ci]          (Eq.2 weight term)
+// over every output pixel p of the segment's kept rows.  The explicit path (im2col of 18-36 B per
+// input pixel per tap into HBM, then a GEMM over the columns) moved ~9x the layer input through HBM;
+// here each CTA stages one (image, band of output rows) unit in shared memory - the delta tile and
+// the input rows it reads, zero rows for the padding - and its warps run bf16 m16n8k16 tensor-core
+// MMAs whose B operand rows are gathered by ldmatrix straight from the staged input (one row address
+// per output pixel and tap, so the shift / stride / zero padding costs nothing).  The work is
+// bandwidth-sized (K = pixels, M = cout, N = 9 cin), so the warp-level MMA is not the bound; the
+// accumulators stay in registers across all units of a persistent CTA and are reduced once at the end
+// (shared-memory atomics across warps, then one global fp32 atomic per weight per CTA).
+#include "common.cuh"
+#include "kernels.h"
+
+#include <algorithm>
+
+namespace sk {
+
+namespace {
+
+constexpr int NW_THREADS = 256;
+constexpr int NW_P = 128;  // output pixels per unit
+
+template <int CIN, int COUT>
+struct NwCfg {
+    static constexpr int MT = COUT / 16;                   // M tiles of 16 output channels
+    static constexpr int NTT = CIN / 8;                    // n tiles of 8 input channels per tap
+    static constexpr int NTG = CIN == 16 ? (MT == 4 ? 2 : 1) : 8 / MT;  // tap groups
+    static constexpr int COMBOS = MT * NTG;                // (M tile, tap group) work items
+    static constexpr int WPC = 8 / COMBOS;                 // warps per work item (split over k chunks)
+    static constexpr int MAXT = (9 + NTG - 1) / NTG;       // taps per group (max)
+    static_assert(8 % COMBOS == 0, "work items must divide the 8 warps");
+};
+
+SK_DEV void ldsm_x4_t(uint32_t addr, uint32_t &r0, uint32_t &r1, uint32_t &r2, uint32_t &r3) {
+    asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+                 : "r"(addr));
+}
+SK_DEV void ldsm_x2_t(uint32_t addr, uint32_t &r0, uint32_t &r1) {
+    asm volatile("ldmatrix.sync.aligned.m8n8.x2.trans.shared.b16 {%0, %1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(addr));
+}
+SK_DEV void mma_bf16(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3, uint32_t b0, uint32_t b1) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+        "{%0, %1, %2, %3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+}  // namespace
+
+// X [nb][Hin][Win][CIN] bf16, D [nb][H][W][COUT] bf16 (H = Hin / S), dW [COUT][9][CIN] fp32 (+=)
+template <int CIN, int COUT, int S>
+__global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t *__restrict__ X,
+                                                                   const uint16_t *__restrict__ D, float *dW, int nb,
+                                                                   int H, int W, int TH) {
+    pdl_enter();
+    using Cfg = NwCfg<CIN, COUT>;
+    extern __shared__ __align__(16) uint8_t smem[];
+    const int Hin = H * S, Win = W * S;
+    const int RX = S * (TH - 1) + 3;                      // staged input rows per unit
+    uint16_t *sD = reinterpret_cast<uint16_t *>(smem);    // [NW_P][COUT]
+    uint16_t *sX = sD + NW_P * COUT;                      // [RX][Win][CIN] then one zero row [CIN]
+    uint16_t *sZ = sX + (size_t)RX * Win * CIN;
+    float *sR = reinterpret_cast<float *>(sZ + CIN);      // [COUT * 9 * CIN] cross-warp reduction (WPC > 1)
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int combo = warp / Cfg::WPC, wk = warp % Cfg::WPC;
+    const int mt = combo / Cfg::NTG, tg = combo % Cfg::NTG;
+    const int tap0 = tg * 9 / Cfg::NTG, tap1 = (tg + 1) * 9 / Cfg::NTG;
+    if (threadIdx.x < CIN / 8) reinterpret_cast<uint4 *>(sZ)[threadIdx.x] = make_uint4(0u, 0u, 0u, 0u);
+    if (Cfg::WPC > 1)
+        for (int i = threadIdx.x; i < COUT * 9 * CIN; i += NW_THREADS) sR[i] = 0.f;
+
+    float acc[Cfg::MAXT][Cfg::NTT][4];
+#pragma unroll
+    for (int t = 0; t < Cfg::MAXT; ++t)
+#pragma unroll
+        for (int j = 0; j < Cfg::NTT; ++j) acc[t][j][0] = acc[t][j][1] = acc[t][j][2] = acc[t][j][3] = 0.f;
+
+    const int bands = H / TH;
+    const long long units = (long long)nb * bands;
+    const uint32_t sD_a = smem_u32(sD), sX_a = smem_u32(sX), sZ_a = smem_u32(sZ);
+    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
+        const long long n = u / bands;
+        const int y0 = (int)(u - n * bands) * TH;
+        __syncthreads();  // previous unit's readers are done
+        {   // stage delta rows y0 .. y0+TH-1 (contiguous) and input rows S*y0-1 .. (zero outside the image)
+            const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + y0) * (long long)W) * COUT);
+            const int nD = TH * W * COUT / 8;
+            for (int i = threadIdx.x; i < nD; i += NW_THREADS) reinterpret_cast<uint4 *>(sD)[i] = __ldg(src + i);
+            const int rowv = Win * CIN / 8;
+            const int nX = RX * rowv;
+            for (int i = threadIdx.x; i < nX; i += NW_THREADS) {
+                const int r = i / rowv, e = i - r * rowv;
+                const int yi = S * y0 - 1 + r;
+                uint4 v = make_uint4(0u, 0u, 0u, 0u);
+                if (yi >= 0 && yi < Hin)
+                    v = __ldg(reinterpret_cast<const uint4 *>(X + ((n * Hin + yi) * (long long)Win) * CIN) + e);
+                reinterpret_cast<uint4 *>(sX)[i] = v;
+            }
+        }
+        __syncthreads();
+        const int P = TH * W;
+        for (int kc = wk; kc < P / 16; kc += Cfg::WPC) {
+            // A = delta^T (m = output channel, k = pixel): 4 transposed 8x8 blocks of sD
+            uint32_t a0, a1, a2, a3;
+            {
+                const int j = lane >> 3, r = lane & 7;
+                const int k = kc * 16 + ((j & 2) ? 8 : 0) + r;
+                const int m = mt * 16 + ((j & 1) ? 8 : 0);
+                ldsm_x4_t(sD_a + (uint32_t)(k * COUT + m) * 2u, a0, a1, a2, a3);
+            }
+            // this lane's B row: output pixel kc*16 + (lane & 15)
+            const int p = kc * 16 + (lane & 15);
+            const int yl = p / W, x = p - yl * W;
+#pragma unroll
+            for (int t = 0; t < Cfg::MAXT; ++t) {
+                const int tap = tap0 + t;
+                if (tap >= tap1) break;
+                const int dy = tap / 3, dx = tap % 3;
+                const int xs = S * x + dx - 1;
+                const int ys = S * yl + dy;                       // staged row
+                const int yi = S * y0 - 1 + ys;                   // image row
+                const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
+                const uint32_t row = ok ? sX_a + (uint32_t)((ys * Win + xs) * CIN) * 2u : sZ_a;
+#pragma unroll
+                for (int j = 0; j < Cfg::NTT; ++j) {
+                    uint32_t b0, b1;
+                    ldsm_x2_t(row + (uint32_t)j * 16u, b0, b1);
+                    mma_bf16(acc[t][j], a0, a1, a2, a3, b0, b1);
+                }
+            }
+        }
+    }
+    // D fragment: rows (co) mt*16 + lane/4 (+8), cols (ci within n tile) 2*(lane%4) (+1)
+    const int co = mt * 16 + (lane >> 2), ci0 = 2 * (lane & 3);
+    if (Cfg::WPC > 1) {
+        __syncthreads();
+#pragma unroll
+        for (int t = 0; t < Cfg::MAXT; ++t) {
+            const int tap = tap0 + t;
+            if (tap >= tap1) break;
+#pragma unroll
+            for (int j = 0; j < Cfg::NTT; ++j) {
+                const int ci = j * 8 + ci0;
+                atomicAdd(&sR[(co * 9 + tap) * CIN + ci], acc[t][j][0]);
+                atomicAdd(&sR[(co * 9 + tap) * CIN + ci + 1], acc[t][j][1]);
+                atomicAdd(&sR[((co + 8) * 9 + tap) * CIN + ci], acc[t][j][2]);
+                atomicAdd(&sR[((co + 8) * 9 + tap) * CIN + ci + 1], acc[t][j][3]);
+            }
+        }
+        __syncthreads();
+        for (int i = threadIdx.x; i < COUT * 9 * CIN; i += NW_THREADS)
+            if (sR[i] != 0.f) atomicAdd(dW + i, sR[i]);
+    } else {
+#pragma unroll
+        for (int t = 0; t < Cfg::MAXT; ++t) {
+            const int tap = tap0 + t;
+            if (tap >= tap1) break;
+#pragma unroll
+            for (int j = 0; j < Cfg::NTT; ++j) {
+                const int ci = j * 8 + ci0;
+                atomicAdd(dW + (co * 9 + tap) * CIN + ci, acc[t][j][0]);
+                atomicAdd(dW + (co * 9 + tap) * CIN + ci + 1, acc[t][j][1]);
+                atomicAdd(dW + ((co + 8) * 9 + tap) * CIN + ci, acc[t][j][2]);
+                atomicAdd(dW + ((co + 8) * 9 + tap) * CIN + ci + 1, acc[t][j][3]);
+            }
+        }
+    }
+}
+
+bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W) {
+    if (!((cin == 16 || cin == 32) && (cout == 16 || cout == 32 || cout == 64) && (stride == 1 || stride == 2)))
+        return false;
+    if (W > NW_P || NW_P % W || W % 16) return false;  // 16-pixel k chunks inside one image row band
+    const int TH = std::min(H, NW_P / W);
+    return H % TH == 0;
+}
+
+template <int CIN, int COUT, int S>
+static cudaError_t launch_nw(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, cudaStream_t s,
+                             int num_sms) {
+    using Cfg = NwCfg<CIN, COUT>;
+    const int TH = std::min(H, NW_P / W);
+    const int RX = S * (TH - 1) + 3;
+    const size_t smem = (size_t)NW_P * COUT * 2 + (size_t)RX * W * S * CIN * 2 + CIN * 2 +
+                        (Cfg::WPC > 1 ? (size_t)COUT * 9 * CIN * 4 : 0);
+    auto kern = narrow_wgrad_kernel<CIN, COUT, S>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    if (smem > 200 * 1024) return cudaErrorInvalidValue;
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW_THREADS, smem) != cudaSuccess || per_sm < 1)
+        per_sm = 1;
+    const long long units = (long long)nb * (H / TH);
+    if (units == 0) return cudaSuccess;
+    const int grid = (int)std::min<long long>(units, (long long)num_sms * per_sm);
+    sk_launch(kern, grid, NW_THREADS, smem, s, X, D, dW, nb, H, W, TH);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
+                                int cout, int stride, cudaStream_t s, int num_sms) {
+    if (!narrow_wgrad_supported(cin, cout, stride, H, W)) return cudaErrorInvalidValue;
+#define NW_CASE(CI, CO, ST) \
+    if (cin == CI && cout == CO && stride == ST) return launch_nw<CI, CO, ST>(X, D, dW, nb, H, W, s, num_sms)
+    NW_CASE(16, 16, 1);
+    NW_CASE(16, 32, 1);
+    NW_CASE(16, 64, 1);
+    NW_CASE(32, 16, 1);
+    NW_CASE(32, 32, 1);
+    NW_CASE(32, 64, 1);
+    NW_CASE(16, 16, 2);
+    NW_CASE(16, 32, 2);
+    NW_CASE(16, 64, 2);
+    NW_CASE(32, 16, 2);
+    NW_CASE(32, 32, 2);
+    NW_CASE(32, 64, 2);
+#undef NW_CASE
+    return cudaErrorInvalidValue;
+}
+
+}  // namespace sk

@@ -92,6 +92,7 @@ def _load():
         "skipper_k_conv_fwd": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_wgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
+        "skipper_k_narrow_wgrad": (I, [P, P, P, I, I, I, I, I, I, I, P]),
         "skipper_k_conv_lif": (I, [P, P, P, P, P, P, I, I, I, I, I, I, I, ct.c_float, ct.c_float, P]),
         "skipper_k_num_sms": (I, []),
         "skipper_k_conv_s": (I, [P, P, P, I, I, I, I, I, I, I, P]),
@@ -489,6 +490,19 @@ def k_conv_dgrad(D, Wt):
     cin = Wt.shape[0]
     out = torch.empty((nb, h, w, cin), dtype=torch.float32, device=D.device)
     _check(lib.skipper_k_conv_dgrad(_ptr(D, "bf16"), _ptr(Wt, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, _stream_handle()))
+    return out
+
+
+def k_narrow_wgrad(D, X, stride=1, out=None):
+    """D [nb][h][w][cout], X [nb][stride*h][stride*w][cin] bf16 -> dW [cout][3][3][cin] fp32 (narrow channels)."""
+    torch = _torch()
+    nb, h, w, cout = D.shape
+    cin = X.shape[3]
+    acc = out is not None
+    if out is None:
+        out = torch.empty((cout, 3, 3, cin), dtype=torch.float32, device=D.device)
+    _check(lib.skipper_k_narrow_wgrad(_ptr(D, "bf16"), _ptr(X, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, stride,
+                                      1 if acc else 0, _stream_handle()))
     return out
 
 

@@ -113,6 +113,29 @@ def test_conv_wgrad(nb, h, w, cin, cout):
     assert (out - ref).abs().max() <= 1e-5 * ref.abs().max() + 1e-12
 
 
+NARROW_WGRAD_SHAPES = [(3, 64, 64, 16, 16, 1), (2, 32, 32, 32, 32, 1), (5, 16, 16, 16, 32, 1), (3, 32, 32, 16, 32, 2),
+                       (2, 16, 16, 32, 64, 2), (4, 16, 16, 32, 16, 1), (7, 4, 16, 16, 64, 1)]
+
+
+@pytest.mark.parametrize("nb,h,w,cin,cout,stride", NARROW_WGRAD_SHAPES)
+def test_narrow_wgrad(nb, h, w, cin, cout, stride):
+    """Narrow-channel weight gradient (ldmatrix row gathers, no column buffer) against the float64 conv
+    backward, for stride 1 and 2 and every (cin, cout) the ResNet layers use; h x w is the output size."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_narrow_wgrad
+    g = torch.Generator().manual_seed(nb * 7 + h + cout + stride)
+    D = grid((nb, h, w, cout), e=12, gen=g)
+    X = spikes((nb, stride * h, stride * w, cin), gen=g)
+    Wv = torch.zeros((cout, 3, 3, cin), dtype=torch.float64, requires_grad=True)
+    y = F.conv2d(X.permute(0, 3, 1, 2).double(), Wv.permute(0, 3, 1, 2), padding=1, stride=stride).permute(0, 2, 3, 1)
+    y.backward(D.double())
+    ref = Wv.grad
+    out = k_narrow_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda(), stride=stride).cpu().double()
+    assert (out - ref).abs().max() <= 1e-5 * ref.abs().max() + 1e-12
+    acc = out.float().cuda()
+    k_narrow_wgrad(bf16_bits(D).cuda(), bf16_bits(X).cuda(), stride=stride, out=acc)  # accumulates
+    assert (acc.cpu().double() - 2 * ref).abs().max() <= 2e-5 * ref.abs().max() + 1e-12
+
+
 def test_stream_ordering_with_torch():
     """The library's kernels are ordered with torch's work on the same stream: a long GEMM
     followed immediately by a torch copy of its output must see the finished result."""
