@@ -98,6 +98,9 @@ SK_DEV void tma_reduce_add_3d(const void *tmap, uint32_t src, int c0, int c1, in
 SK_DEV void cp_async4(uint32_t dst, const void *src, uint32_t src_bytes) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }
+SK_DEV void cp_async16_cg(uint32_t dst, const void *src, uint32_t src_bytes) {  // L2 only; src_bytes = 0: zero fill
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
+}
 SK_DEV void cp_async8(uint32_t dst, const void *src, uint32_t src_bytes) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(dst), "l"(src), "r"(src_bytes) : "memory");
 }

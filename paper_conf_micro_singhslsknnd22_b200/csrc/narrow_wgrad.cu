@@ -4,7 +4,8 @@
 // over every output pixel p of the segment's kept rows.  The explicit path (im2col of 18-36 B per
 // input pixel per tap into HBM, then a GEMM over the columns) moved ~9x the layer input through HBM;
 // here each CTA stages one (image, band of output rows) unit in shared memory - the delta tile and
-// the input rows it reads, zero rows for the padding - and its warps run bf16 m16n8k16 tensor-core
+// the input rows it reads, zero rows for the padding; cp.async, double-buffered so the next unit
+// streams in while this one computes - and its warps run bf16 m16n8k16 tensor-core
 // MMAs whose B operand rows are gathered by ldmatrix straight from the staged input (one row address
 // per output pixel and tap, so the shift / stride / zero padding costs nothing).  The work is
 // bandwidth-sized (K = pixels, M = cout, N = 9 cin), so the warp-level MMA is not the bound; the
@@ -61,9 +62,9 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
     extern __shared__ __align__(16) uint8_t smem[];
     const int Hin = H * S, Win = W * S;
     const int RX = S * (TH - 1) + 3;                      // staged input rows per unit
-    uint16_t *sD = reinterpret_cast<uint16_t *>(smem);    // [NW_P][COUT]
-    uint16_t *sX = sD + NW_P * COUT;                      // [RX][Win][CIN] then one zero row [CIN]
-    uint16_t *sZ = sX + (size_t)RX * Win * CIN;
+    const int BUF = NW_P * COUT + RX * Win * CIN;         // bf16 elements of one staging buffer
+    uint16_t *sB = reinterpret_cast<uint16_t *>(smem);    // 2 x { delta [NW_P][COUT], input [RX][Win][CIN] }
+    uint16_t *sZ = sB + 2 * (size_t)BUF;                  // one zero row [CIN]
     float *sR = reinterpret_cast<float *>(sZ + CIN);      // [COUT * 9 * CIN] cross-warp reduction (WPC > 1)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int combo = warp / Cfg::WPC, wk = warp % Cfg::WPC;
@@ -81,30 +82,43 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
 
     const int bands = H / TH;
     const long long units = (long long)nb * bands;
-    const uint32_t sD_a = smem_u32(sD), sX_a = smem_u32(sX), sZ_a = smem_u32(sZ);
-    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
+    const uint32_t sB_a = smem_u32(sB), sZ_a = smem_u32(sZ);
+    // stage unit u into buffer b with cp.async (16-byte pieces; rows outside the image are zero-filled)
+    auto stage = [&](long long u, int b) {
         const long long n = u / bands;
         const int y0 = (int)(u - n * bands) * TH;
-        __syncthreads();  // previous unit's readers are done
-        {   // stage delta rows y0 .. y0+TH-1 (contiguous) and input rows S*y0-1 .. (zero outside the image)
-            const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + y0) * (long long)W) * COUT);
-            const int nD = TH * W * COUT / 8;
-            for (int i = threadIdx.x; i < nD; i += NW_THREADS) reinterpret_cast<uint4 *>(sD)[i] = __ldg(src + i);
-            const int rowv = Win * CIN / 8;
-            const int nX = RX * rowv;
-            for (int i = threadIdx.x; i < nX; i += NW_THREADS) {
-                const int r = i / rowv, e = i - r * rowv;
-                const int yi = S * y0 - 1 + r;
-                uint4 v = make_uint4(0u, 0u, 0u, 0u);
-                if (yi >= 0 && yi < Hin)
-                    v = __ldg(reinterpret_cast<const uint4 *>(X + ((n * Hin + yi) * (long long)Win) * CIN) + e);
-                reinterpret_cast<uint4 *>(sX)[i] = v;
-            }
+        const uint32_t dD = sB_a + (uint32_t)(b * BUF) * 2u, dX = dD + (uint32_t)(NW_P * COUT) * 2u;
+        const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + y0) * (long long)W) * COUT);
+        const int nD = TH * W * COUT / 8;
+        for (int i = threadIdx.x; i < nD; i += NW_THREADS) cp_async16_cg(dD + 16u * i, src + i, 16u);
+        const int rowv = Win * CIN / 8;
+        const int nX = RX * rowv;
+        for (int i = threadIdx.x; i < nX; i += NW_THREADS) {
+            const int r = i / rowv, e = i - r * rowv;
+            const int yi = S * y0 - 1 + r;
+            const bool in = yi >= 0 && yi < Hin;
+            const uint4 *xs = reinterpret_cast<const uint4 *>(X + ((n * Hin + (in ? yi : 0)) * (long long)Win) * CIN) + e;
+            cp_async16_cg(dX + 16u * i, xs, in ? 16u : 0u);
+        }
+        cp_async_commit();
+    };
+    if ((long long)blockIdx.x < units) stage(blockIdx.x, 0);
+    int b = 0;
+    for (long long u = blockIdx.x; u < units; u += gridDim.x, b ^= 1) {
+        const long long n = u / bands;
+        const int y0 = (int)(u - n * bands) * TH;
+        const long long un = u + gridDim.x;
+        if (un < units) {
+            stage(un, b ^ 1);   // the buffer the previous unit read (released by the barrier below)
+            cp_async_wait<1>(); // this unit's pieces have landed (the next unit's may still be in flight)
+        } else {
+            cp_async_wait<0>();
         }
         __syncthreads();
+        const uint32_t sD_a = sB_a + (uint32_t)(b * BUF) * 2u, sX_a = sD_a + (uint32_t)(NW_P * COUT) * 2u;
         const int P = TH * W;
         for (int kc = wk; kc < P / 16; kc += Cfg::WPC) {
-            // A = delta^T (m = output channel, k = pixel): 4 transposed 8x8 blocks of sD
+            // A = delta^T (m = output channel, k = pixel): 4 transposed 8x8 blocks of the delta tile
             uint32_t a0, a1, a2, a3;
             {
                 const int j = lane >> 3, r = lane & 7;
@@ -133,6 +147,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
                 }
             }
         }
+        __syncthreads();  // buffer b is free for the unit after next
     }
     // D fragment: rows (co) mt*16 + lane/4 (+8), cols (ci within n tile) 2*(lane%4) (+1)
     const int co = mt * 16 + (lane >> 2), ci0 = 2 * (lane & 3);
@@ -185,7 +200,7 @@ static cudaError_t launch_nw(const uint16_t *X, const uint16_t *D, float *dW, in
     using Cfg = NwCfg<CIN, COUT>;
     const int TH = std::min(H, NW_P / W);
     const int RX = S * (TH - 1) + 3;
-    const size_t smem = (size_t)NW_P * COUT * 2 + (size_t)RX * W * S * CIN * 2 + CIN * 2 +
+    const size_t smem = 2 * ((size_t)NW_P * COUT * 2 + (size_t)RX * W * S * CIN * 2) + CIN * 2 +
                         (Cfg::WPC > 1 ? (size_t)COUT * 9 * CIN * 4 : 0);
     auto kern = narrow_wgrad_kernel<CIN, COUT, S>;
     static bool attr = false;
