@@ -542,12 +542,13 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvL
     return cudaLaunchKernelEx(&cfg, kern, ta, tb, a);
 }
 
-// CTA pairs (SKIPPER_CL_PAIR=1 enables) when the pixel tiles of a channel tile pair up
+// CTA pairs (SKIPPER_CL_PAIR=0 disables) when the pixel tiles of a channel tile pair up
 static bool cl_use_pair(int m_tiles) {
     const char *e = getenv("SKIPPER_CL_PAIR");  // read per launch so tests can cover both variants
-    // default off: pairs measured ~2 % slower (the kernel is bound by per-SM TMA processing of the
-    // 4D activation boxes, not by shared-memory bandwidth or the MMA)
-    return e && atoi(e) != 0 && m_tiles % 2 == 0;
+    // default on since the halo boxes and PDL: pairs with resident weight halves measured ~0.4 % faster
+    // per step on cfg 2 and cfg 3 (two alternating repetitions); before the halo boxes they were ~2 %
+    // slower.  The kernel stays bound by its TMA producer skeleton either way.
+    return (!e || atoi(e) != 0) && m_tiles % 2 == 0;
 }
 
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms) {
