@@ -8,7 +8,7 @@ exists.
 """
 _EXPORTS = (
     "SkipperNet", "SkipperError", "lib", "sst_host", "workspace_bytes", "make_config", "make_layers",
-    "k_fc_fwd", "k_fc_wgrad", "k_conv_fwd", "k_conv_dgrad", "k_conv_wgrad", "k_narrow_wgrad", "k_conv_lif", "k_conv_s", "encode_poisson",
+    "k_fc_fwd", "k_fc_wgrad", "k_conv_fwd", "k_conv_dgrad", "k_conv_wgrad", "k_narrow_wgrad", "k_narrow_dgrad", "k_conv_lif", "k_conv_s", "encode_poisson",
     "PASS_FIRST", "PASS_RECOMPUTE", "PASS_RECORD",
 )
 __all__ = list(_EXPORTS)

@@ -186,6 +186,152 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
     }
 }
 
+namespace {
+SK_DEV void ldsm_x4(uint32_t addr, uint32_t &r0, uint32_t &r1, uint32_t &r2, uint32_t &r3) {
+    asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+                 : "r"(addr));
+}
+SK_DEV void ldsm_x2(uint32_t addr, uint32_t &r0, uint32_t &r1) {
+    asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0, %1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(addr));
+}
+}  // namespace
+
+// Stride-1 dgrad of a narrow 3x3 conv (Eq.2's g = W^T delta):
+//     G[n, y, x, ci] = sum_{dy, dx, co} W[co][dy*3+dx][ci] D[n, y+1-dy, x+1-dx, co]
+// M = pixels of a band (8 warps x 16), N = ci, K = (tap, co).  The band's delta rows plus a one-row halo
+// are staged by cp.async (double-buffered), the transposed weights Wt [ci][9][co] stay resident, and the
+// A rows (one per pixel and tap, or a zero row) are gathered by ldmatrix.
+template <int CI, int CO>
+__global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t *__restrict__ D,
+                                                                   const uint16_t *__restrict__ Wt, float *G, int nb,
+                                                                   int H, int W, int TH) {
+    pdl_enter();
+    extern __shared__ __align__(16) uint8_t smem[];
+    const int RD = TH + 2;                                // staged delta rows per band
+    const int BUF = RD * W * CO;                          // bf16 elements of one staging buffer
+    uint16_t *sW = reinterpret_cast<uint16_t *>(smem);   // [CI][9][CO]
+    uint16_t *sB = sW + 9 * CI * CO;                      // 2 x [RD][W][CO]
+    uint16_t *sZ = sB + 2 * (size_t)BUF;                  // zero row [CO]
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < 9 * CI * CO / 8; i += NW_THREADS)
+        reinterpret_cast<uint4 *>(sW)[i] = __ldg(reinterpret_cast<const uint4 *>(Wt) + i);
+    if (threadIdx.x < CO / 8) reinterpret_cast<uint4 *>(sZ)[threadIdx.x] = make_uint4(0u, 0u, 0u, 0u);
+    const int bands = H / TH;
+    const long long units = (long long)nb * bands;
+    const uint32_t sW_a = smem_u32(sW), sB_a = smem_u32(sB), sZ_a = smem_u32(sZ);
+    auto stage = [&](long long u, int b) {
+        const long long n = u / bands;
+        const int y0 = (int)(u - n * bands) * TH;
+        const uint32_t dst = sB_a + (uint32_t)(b * BUF) * 2u;
+        const int rowv = W * CO / 8;
+        for (int i = threadIdx.x; i < RD * rowv; i += NW_THREADS) {
+            const int r = i / rowv, e = i - r * rowv;
+            const int y = y0 - 1 + r;
+            const bool in = y >= 0 && y < H;
+            const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + (in ? y : 0)) * (long long)W) * CO) + e;
+            cp_async16_cg(dst + 16u * i, src, in ? 16u : 0u);
+        }
+        cp_async_commit();
+    };
+    if ((long long)blockIdx.x < units) stage(blockIdx.x, 0);
+    int b = 0;
+    for (long long u = blockIdx.x; u < units; u += gridDim.x, b ^= 1) {
+        const long long n = u / bands;
+        const int y0 = (int)(u - n * bands) * TH;
+        const long long un = u + gridDim.x;
+        if (un < units) {
+            stage(un, b ^ 1);
+            cp_async_wait<1>();
+        } else {
+            cp_async_wait<0>();
+        }
+        __syncthreads();
+        const uint32_t sD_a = sB_a + (uint32_t)(b * BUF) * 2u;
+        if (warp * 16 < TH * W) {
+            float acc[CI / 8][4];
+#pragma unroll
+            for (int j = 0; j < CI / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+            // this lane's A row: pixel warp*16 + (lane&7) + ((lane>>3)&1)*8, k half (lane>>4)*8
+            const int pa = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
+            const int ya = pa / W, xa = pa - ya * W;
+            const int kh = (lane >> 4) * 8;
+#pragma unroll
+            for (int tap = 0; tap < 9; ++tap) {
+                const int dy = tap / 3, dx = tap % 3;
+                const int xs = xa + 1 - dx, ys = ya + 1 - dy;  // staged row ys + 1 - 1 (halo row 0 = y0 - 1)
+                const int yi = y0 + ys;
+                const bool ok = xs >= 0 && xs < W && yi >= 0 && yi < H;
+                const uint32_t arow = ok ? sD_a + (uint32_t)(((ys + 1) * W + xs) * CO) * 2u : sZ_a;
+#pragma unroll
+                for (int ks = 0; ks < CO / 16; ++ks) {
+                    uint32_t a0, a1, a2, a3;
+                    ldsm_x4(arow + (uint32_t)(ks * 16 + kh) * 2u, a0, a1, a2, a3);
+#pragma unroll
+                    for (int nt = 0; nt < CI / 8; ++nt) {
+                        uint32_t b0, b1;
+                        const int ci = nt * 8 + (lane & 7), co = ks * 16 + ((lane >> 3) & 1) * 8;
+                        ldsm_x2(sW_a + (uint32_t)((ci * 9 + tap) * CO + co) * 2u, b0, b1);
+                        mma_bf16(acc[nt], a0, a1, a2, a3, b0, b1);
+                    }
+                }
+            }
+            // D fragment: pixel warp*16 + lane/4 (+8), ci nt*8 + 2*(lane%4) (+1)
+            const int p0 = warp * 16 + (lane >> 2);
+#pragma unroll
+            for (int h2 = 0; h2 < 2; ++h2) {
+                const int p = p0 + 8 * h2;
+                const int yy = y0 + p / W, xx = p % W;
+                float *dst = G + (((n * H + yy) * (long long)W + xx) * CI) + 2 * (lane & 3);
+#pragma unroll
+                for (int nt = 0; nt < CI / 8; ++nt)
+                    *reinterpret_cast<float2 *>(dst + nt * 8) = make_float2(acc[nt][2 * h2], acc[nt][2 * h2 + 1]);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+bool narrow_dgrad_supported(int cin, int cout, int H, int W) {
+    if (!((cin == 16 || cin == 32) && (cout == 16 || cout == 32))) return false;
+    if (W > NW_P || NW_P % W || W % 16) return false;
+    const int TH = std::min(H, NW_P / W);
+    return H % TH == 0;
+}
+
+template <int CI, int CO>
+static cudaError_t launch_nd(const uint16_t *D, const uint16_t *Wt, float *G, int nb, int H, int W, cudaStream_t s,
+                             int num_sms) {
+    const int TH = std::min(H, NW_P / W);
+    const size_t smem = (size_t)9 * CI * CO * 2 + 2 * (size_t)(TH + 2) * W * CO * 2 + CO * 2;
+    auto kern = narrow_dgrad_kernel<CI, CO>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW_THREADS, smem) != cudaSuccess || per_sm < 1)
+        per_sm = 1;
+    const long long units = (long long)nb * (H / TH);
+    if (units == 0) return cudaSuccess;
+    const int grid = (int)std::min<long long>(units, (long long)num_sms * per_sm);
+    sk_launch(kern, grid, NW_THREADS, smem, s, D, Wt, G, nb, H, W, TH);
+    return cudaGetLastError();
+}
+
+// G [nb][H][W][cin] fp32 = stride-1 dgrad of D [nb][H][W][cout] through Wt [cin][9][cout] (bf16)
+cudaError_t launch_narrow_dgrad(const uint16_t *D, const uint16_t *Wt, float *G, int nb, int H, int W, int cin, int cout,
+                                cudaStream_t s, int num_sms) {
+    if (!narrow_dgrad_supported(cin, cout, H, W)) return cudaErrorInvalidValue;
+    if (cin == 16 && cout == 16) return launch_nd<16, 16>(D, Wt, G, nb, H, W, s, num_sms);
+    if (cin == 16 && cout == 32) return launch_nd<16, 32>(D, Wt, G, nb, H, W, s, num_sms);
+    if (cin == 32 && cout == 16) return launch_nd<32, 16>(D, Wt, G, nb, H, W, s, num_sms);
+    if (cin == 32 && cout == 32) return launch_nd<32, 32>(D, Wt, G, nb, H, W, s, num_sms);
+    return cudaErrorInvalidValue;
+}
+
 bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W) {
     if (!((cin == 16 || cin == 32) && (cout == 16 || cout == 32 || cout == 64) && (stride == 1 || stride == 2)))
         return false;

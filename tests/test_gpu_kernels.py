@@ -136,6 +136,23 @@ def test_narrow_wgrad(nb, h, w, cin, cout, stride):
     assert (acc.cpu().double() - 2 * ref).abs().max() <= 2e-5 * ref.abs().max() + 1e-12
 
 
+@pytest.mark.parametrize("nb,h,w,cin,cout", [(3, 64, 64, 16, 16), (2, 32, 32, 32, 32), (5, 16, 16, 16, 32),
+                                              (4, 16, 16, 32, 16), (7, 4, 16, 16, 16), (2, 8, 32, 32, 32)])
+def test_narrow_dgrad(nb, h, w, cin, cout):
+    """Stride-1 narrow dgrad (staged halo, ldmatrix gathers) against the float64 conv input gradient;
+    spike-like delta and grid weights make every fp32 sum exact."""
+    from paper_conf_micro_singhslsknnd22_b200 import k_narrow_dgrad
+    g = torch.Generator().manual_seed(nb * 11 + h + cin + cout)
+    W = grid((cout, 3, 3, cin), gen=g)
+    D = spikes((nb, h, w, cout), gen=g)
+    X = torch.zeros((nb, h, w, cin), dtype=torch.float64, requires_grad=True)
+    conv_ref(X, W).backward(D.double())
+    ref = X.grad
+    Wt = W.permute(3, 1, 2, 0).contiguous()  # [cin][3][3][cout]
+    out = k_narrow_dgrad(bf16_bits(D).cuda(), bf16_bits(Wt).cuda()).cpu().double()
+    assert torch.equal(out, ref)
+
+
 def test_stream_ordering_with_torch():
     """The library's kernels are ordered with torch's work on the same stream: a long GEMM
     followed immediately by a torch copy of its output must see the finished result."""
