@@ -23,7 +23,7 @@ NVCC_FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-
                      "-I" + os.path.join(ROOT, "include")] + os.environ.get("SKIPPER_NVCC_EXTRA", "").split()
 CXX_FLAGS = ["-O2", "-fPIC", "-std=c++17", "-I" + os.path.join(CUDA, "include"), "-I" + os.path.join(ROOT, "include")]
 
-CU_SOURCES = ["gemm_tc.cu", "conv_lif.cu", "lif_kernels.cu", "layer0.cu", "conv_narrow.cu", "narrow_wgrad.cu"]
+CU_SOURCES = ["gemm_tc.cu", "conv_lif.cu", "lif_kernels.cu", "layer0.cu", "conv_narrow.cu", "narrow_wgrad.cu", "narrow_lif.cu"]
 CXX_SOURCES = ["engine.cpp", "comm.cpp"]
 
 

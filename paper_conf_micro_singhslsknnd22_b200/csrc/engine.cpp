@@ -1287,7 +1287,11 @@ static skipper_status narrow_lif_rows(skipper_ctx *c, int i, int seg, const uint
     if (a.U_out) bytes += (double)R * bn * 4;
     if (a.res) bytes += comp * c->B * c->L[l.res].N * 2;
     ProfScope ps(c, K_CONV_LIF, bytes, 2.0 * comp * c->B * l.H * l.W * l.Cout * 9.0 * l.Cin);
-    CK(sk::launch_conv_narrow_lif(a, c->st, c->num_sms));
+    static const bool nl_off = getenv("SKIPPER_NO_NARROW_LIF_MMA") && atoi(getenv("SKIPPER_NO_NARROW_LIF_MMA"));
+    if (!nl_off && sk::narrow_lif_mma_supported(a.Cin, a.Cout, a.stride, a.H, a.W))
+        CK(sk::launch_narrow_lif_mma(a, c->st, c->num_sms));
+    else
+        CK(sk::launch_conv_narrow_lif(a, c->st, c->num_sms));
     return SKIPPER_OK;
 }
 

@@ -110,6 +110,10 @@ bool conv_narrow_supported(int cin, int cout, int stride, int sign);
 cudaError_t launch_conv_narrow(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
 bool conv_narrow_lif_supported(int cin, int cout, int stride);
 cudaError_t launch_conv_narrow_lif(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
+// The same fused conv + LIF on warp-level bf16 MMAs over staged input rows (narrow_lif.cu): cin 16,
+// cout 16 / 32, stride 1 / 2, output width a multiple of 16 dividing 128
+bool narrow_lif_mma_supported(int cin, int cout, int stride, int H, int W);
+cudaError_t launch_narrow_lif_mma(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
 // conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
                      int num_sms);
