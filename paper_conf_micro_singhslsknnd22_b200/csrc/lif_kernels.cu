@@ -922,7 +922,8 @@ __global__ void readout_wgrad_kernel(const float *dz, const float *cnt_kept, flo
     if (i >= (long long)K * D) return;
     const int k = (int)(i / D), n = (int)(i % D);
     float acc = 0.f;
-    for (int b = 0; b < B; ++b) acc += dz[(long long)b * K + k] * cnt_kept[(long long)b * D + n];
+#pragma unroll 16
+    for (int b = 0; b < B; ++b) acc += dz[(long long)b * K + k] * cnt_kept[(long long)b * D + n];  // b ascending
     dWL[i] = accumulate ? dWL[i] + acc * invT : acc * invT;
 }
 
@@ -934,25 +935,57 @@ cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *
 }
 
 // ============================================================================ Adam + shadows
+template <int VEC>
 __global__ void adam_kernel(float *w, const float *g, float *m, float *v, uint16_t *wb, long long n, float lr, float b1,
                             float b2, float eps, float bc1, float bc2_sqrt) {
     pdl_enter();
-    const long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x;
-    if (i >= n) return;
-    const float gi = g[i];
-    const float mi = b1 * m[i] + (1.f - b1) * gi;
-    const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
-    m[i] = mi;
-    v[i] = vi;
-    const float wi = w[i] - (lr / bc1) * mi / (sqrtf(vi) / bc2_sqrt + eps);
-    w[i] = wi;
-    wb[i] = f2bf_bits(wi);
+    // VEC: 4 parameters per thread (16-byte loads / stores); the per-element arithmetic is the same
+    const long long i4 = ((long long)blockIdx.x * blockDim.x + threadIdx.x) * (VEC ? 4 : 1);
+    if (i4 >= n) return;
+    auto upd = [&](float wi, float gi, float &mi, float &vi) {
+        mi = b1 * mi + (1.f - b1) * gi;
+        vi = b2 * vi + (1.f - b2) * gi * gi;
+        return wi - (lr / bc1) * mi / (sqrtf(vi) / bc2_sqrt + eps);
+    };
+    if (VEC && i4 + 4 <= n) {
+        float4 w4 = *reinterpret_cast<const float4 *>(w + i4);
+        const float4 g4 = *reinterpret_cast<const float4 *>(g + i4);
+        float4 m4 = *reinterpret_cast<const float4 *>(m + i4);
+        float4 v4 = *reinterpret_cast<const float4 *>(v + i4);
+        w4.x = upd(w4.x, g4.x, m4.x, v4.x);
+        w4.y = upd(w4.y, g4.y, m4.y, v4.y);
+        w4.z = upd(w4.z, g4.z, m4.z, v4.z);
+        w4.w = upd(w4.w, g4.w, m4.w, v4.w);
+        *reinterpret_cast<float4 *>(m + i4) = m4;
+        *reinterpret_cast<float4 *>(v + i4) = v4;
+        *reinterpret_cast<float4 *>(w + i4) = w4;
+        *reinterpret_cast<uint2 *>(wb + i4) = make_uint2(f2bf_bits(w4.x) | ((uint32_t)f2bf_bits(w4.y) << 16),
+                                                         f2bf_bits(w4.z) | ((uint32_t)f2bf_bits(w4.w) << 16));
+    } else {
+        for (long long i = i4; i < n && i < i4 + (VEC ? 4 : 1); ++i) {
+            float mi = m[i], vi = v[i];
+            const float wi = upd(w[i], g[i], mi, vi);
+            m[i] = mi;
+            v[i] = vi;
+            w[i] = wi;
+            wb[i] = f2bf_bits(wi);
+        }
+    }
 }
 
 cudaError_t launch_adam(float *w, const float *g, float *m, float *v, uint16_t *wb, size_t n, float lr, float b1,
                         float b2, float eps, float bc1, float bc2_sqrt, cudaStream_t s) {
     if (n == 0) return cudaSuccess;
-    sk_launch(adam_kernel, (unsigned)((n + 255) / 256), 256, 0, s, w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1, bc2_sqrt);
+    const bool aligned = ((reinterpret_cast<uintptr_t>(w) | reinterpret_cast<uintptr_t>(g) | reinterpret_cast<uintptr_t>(m) |
+                           reinterpret_cast<uintptr_t>(v)) & 15) == 0 && (reinterpret_cast<uintptr_t>(wb) & 7) == 0;
+    if (aligned) {
+        const long long t = ((long long)n + 3) / 4;
+        sk_launch(adam_kernel<1>, (unsigned)((t + 255) / 256), 256, 0, s, w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1,
+                  bc2_sqrt);
+    } else {  // a layer's slice of the flat gradient buffer need not be 16-byte aligned
+        sk_launch(adam_kernel<0>, (unsigned)((n + 255) / 256), 256, 0, s, w, g, m, v, wb, (long long)n, lr, b1, b2, eps, bc1,
+                  bc2_sqrt);
+    }
     return cudaGetLastError();
 }
 
