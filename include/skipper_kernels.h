@@ -41,12 +41,14 @@ int skipper_k_conv_wgrad(const unsigned short *D, const unsigned short *X, float
  * EUNSUPPORTED for other shapes, ECUDA on a launch error. */
 int skipper_k_narrow_wgrad(const unsigned short *D, const unsigned short *X, float *dW, int nb, int h, int w,
                            int cin, int cout, int stride, int accumulate, void *stream);
-/* Stride-1 dgrad of a narrow-channel 3x3 conv (cin, cout in {16, 32}; pad 1), Eq.2's g term:
- *   G[nb,y,x,ci] = sum_{dy,dx,co} Wt[ci][dy*3+dx][co] D[nb, y+1-dy, x+1-dx, co]
- * D [nb][h][w][cout] and Wt [cin][9][cout] bf16, G [nb][h][w][cin] fp32 (overwritten), device pointers;
- * w a multiple of 16 dividing 128.  EUNSUPPORTED for other shapes, ECUDA on a launch error. */
+/* dgrad of a narrow-channel 3x3 conv (pad 1, stride s in {1, 2}), Eq.2's g term:
+ *   G[nb,yi,xi,ci] = sum_{dy,dx,co} Wt[ci][dy*3+dx][co] D[nb, (yi+1-dy)/s, (xi+1-dx)/s, co]
+ * (terms whose offsets are not multiples of s vanish).  h x w is the OUTPUT (delta) size: D [nb][h][w][cout]
+ * and Wt [cin][9][cout] bf16, G [nb][s*h][s*w][cin] fp32 (overwritten), device pointers.  cin 16 with
+ * cout 16 / 32, or cin 32 with cout 16 / 32 (64 at s = 2); s*w a multiple of 16 dividing 128.
+ * EUNSUPPORTED for other shapes, ECUDA on a launch error. */
 int skipper_k_narrow_dgrad(const unsigned short *D, const unsigned short *Wt, float *G, int nb, int h, int w,
-                           int cin, int cout, void *stream);
+                           int cin, int cout, int stride, void *stream);
 /* Strided / narrow-channel implicit conv (ResNet layers, reading 8):
  *   Y[nb,y,x,co] = sum_{dy,dx,ci} Wk[co][dy*3+dx][ci] X[nb, s*y+dy-1, s*x+dx-1, ci]   (pad 1, stride s)
  * h x w is the OUTPUT size, X is [nb][s*h][s*w][cin]; cin in {16, 32} (one 32B/64B-swizzled TMA box per

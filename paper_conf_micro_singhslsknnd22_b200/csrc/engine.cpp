@@ -1690,8 +1690,8 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             ProfScope ps(c, K_GEMM_DGRAD, (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4,
                          2.0 * M * l.Cin * 9 * l.Cout);
             static const bool nd_off = getenv("SKIPPER_NO_NARROW_DGRAD") && atoi(getenv("SKIPPER_NO_NARROW_DGRAD"));
-            if (!nd_off && sk::narrow_dgrad_supported(l.Cin, l.Cout, l.H, l.W))  // staged halo + ldmatrix gathers
-                CK(sk::launch_narrow_dgrad(dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cin, l.Cout, c->st, c->num_sms));
+            if (!nd_off && sk::narrow_dgrad_supported(l.Cin, l.Cout, l.H, l.W, 1))  // staged halo + ldmatrix gathers
+                CK(sk::launch_narrow_dgrad(dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cin, l.Cout, 1, c->st, c->num_sms));
             else
                 CK(sk::launch_conv_narrow(narrow_args(l, dcur, l.wt, c->I_buf, nb, -1), c->st, c->num_sms));
         } else if (i > 0 && l.icol && l.dgrad_s) {  // stride 1: g = conv(delta, flipped W^T) as a narrow implicit conv
@@ -1701,6 +1701,12 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             const double M = (double)nb * l.H * l.W;
             CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD,
                          (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4, 2.0 * M * l.Cin * 9 * l.Cout));
+        } else if (i > 0 && l.icol && !(getenv("SKIPPER_NO_NARROW_DGRAD") && atoi(getenv("SKIPPER_NO_NARROW_DGRAD"))) &&
+                   sk::narrow_dgrad_supported(l.Cin, l.Cout, l.H, l.W, l.stride)) {  // strided: no column buffer
+            const double M = (double)nb * l.H * l.W;
+            ProfScope ps(c, K_GEMM_DGRAD, (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4,
+                         2.0 * M * l.Cin * 9 * l.Cout);
+            CK(sk::launch_narrow_dgrad(dcur, l.wt, c->I_buf, nb, l.H, l.W, l.Cin, l.Cout, l.stride, c->st, c->num_sms));
         } else if (i > 0 && l.icol) {  // per chunk: dcols = delta_i W_i (columns (ci, tap)), then the col2im gather into g
             const long long ch = icol_chunk(c);
             const int N = 9 * l.Cin;
@@ -2287,13 +2293,13 @@ extern "C" int skipper_k_narrow_wgrad(const unsigned short *D, const unsigned sh
 }
 
 extern "C" int skipper_k_narrow_dgrad(const unsigned short *D, const unsigned short *Wt, float *G, int nb, int h, int w,
-                                      int cin, int cout, void *stream) {
-    if (!sk::narrow_dgrad_supported(cin, cout, h, w)) {
+                                      int cin, int cout, int stride, void *stream) {
+    if (!sk::narrow_dgrad_supported(cin, cout, h, w, stride)) {
         g_last_error = "narrow_dgrad: unsupported shape";
         return SKIPPER_EUNSUPPORTED;
     }
     if (sk::launch_narrow_dgrad(reinterpret_cast<const uint16_t *>(D), reinterpret_cast<const uint16_t *>(Wt), G, nb, h, w,
-                                cin, cout, static_cast<cudaStream_t>(stream), sk::device_num_sms()) != cudaSuccess) {
+                                cin, cout, stride, static_cast<cudaStream_t>(stream), sk::device_num_sms()) != cudaSuccess) {
         g_last_error = "narrow_dgrad: launch failed";
         return SKIPPER_ECUDA;
     }

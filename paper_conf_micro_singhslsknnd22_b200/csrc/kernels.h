@@ -77,11 +77,12 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
 bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W);
 cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
                                 int cout, int stride, cudaStream_t s, int num_sms);
-// Stride-1 dgrad of a narrow 3x3 conv (cin, cout in {16, 32}): G [nb][H][W][cin] fp32 from the layer's
-// delta D [nb][H][W][cout] and the transposed weights Wt [cin][9][cout] (narrow_wgrad.cu)
-bool narrow_dgrad_supported(int cin, int cout, int H, int W);
+// dgrad of a narrow 3x3 conv, stride 1 or 2 (narrow_wgrad.cu): G [nb][s*H][s*W][cin] fp32 from the layer's
+// delta D [nb][H][W][cout] and the transposed weights Wt [cin][9][cout]; cin 16 / 32, cout 16 / 32 (64 for
+// cin 32 at stride 2)
+bool narrow_dgrad_supported(int cin, int cout, int H, int W, int stride);
 cudaError_t launch_narrow_dgrad(const uint16_t *D, const uint16_t *Wt, float *G, int nb, int H, int W, int cin, int cout,
-                                cudaStream_t s, int num_sms);
+                                int stride, cudaStream_t s, int num_sms);
 cudaError_t launch_im2col_bf16(const uint16_t *X, uint16_t *cols, long long nb, int Hin, int Win, int Cin, int H,
                                int W, int stride, cudaStream_t s);
 // Adjoint: G[n][yi][xi][ci] = sum_{dy,dx: s | (yi+1-dy), s | (xi+1-dx)} dcols[(n, y, x)][ci*9 + dy*3+dx]

@@ -197,18 +197,21 @@ SK_DEV void ldsm_x2(uint32_t addr, uint32_t &r0, uint32_t &r1) {
 }
 }  // namespace
 
-// Stride-1 dgrad of a narrow 3x3 conv (Eq.2's g = W^T delta):
-//     G[n, y, x, ci] = sum_{dy, dx, co} W[co][dy*3+dx][ci] D[n, y+1-dy, x+1-dx, co]
-// M = pixels of a band (8 warps x 16), N = ci, K = (tap, co).  The band's delta rows plus a one-row halo
-// are staged by cp.async (double-buffered), the transposed weights Wt [ci][9][co] stay resident, and the
-// A rows (one per pixel and tap, or a zero row) are gathered by ldmatrix.
-template <int CI, int CO>
+// dgrad of a narrow 3x3 conv, stride S in {1, 2} (Eq.2's g = W^T delta):
+//     G[n, yi, xi, ci] = sum_{dy, dx, co} W[co][dy*3+dx][ci] D[n, (yi+1-dy)/S, (xi+1-dx)/S, co]
+// (terms whose (yi+1-dy, xi+1-dx) is not a multiple of S or leaves the image vanish).  M = pixels of a
+// band of G (8 warps x 16), N = ci, K = (tap, co).  The delta rows the band reads are staged by cp.async
+// (double-buffered), the transposed weights Wt [ci][9][co] stay resident, and the A rows (one per pixel
+// and tap, or a zero row) are gathered by ldmatrix.  Replaces conv_narrow's dgrad (S = 1) and the
+// GEMM-into-columns + col2im of the stride-2 layers.
+template <int CI, int CO, int S>
 __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t *__restrict__ D,
                                                                    const uint16_t *__restrict__ Wt, float *G, int nb,
                                                                    int H, int W, int TH) {
     pdl_enter();
     extern __shared__ __align__(16) uint8_t smem[];
-    const int RD = TH + 2;                                // staged delta rows per band
+    const int Hg = S * H, Wg = S * W;                     // G (layer input) size
+    const int RD = TH / S + 2;                            // staged delta rows per band (max)
     const int BUF = RD * W * CO;                          // bf16 elements of one staging buffer
     uint16_t *sW = reinterpret_cast<uint16_t *>(smem);   // [CI][9][CO]
     uint16_t *sB = sW + 9 * CI * CO;                      // 2 x [RD][W][CO]
@@ -217,17 +220,19 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
     for (int i = threadIdx.x; i < 9 * CI * CO / 8; i += NW_THREADS)
         reinterpret_cast<uint4 *>(sW)[i] = __ldg(reinterpret_cast<const uint4 *>(Wt) + i);
     if (threadIdx.x < CO / 8) reinterpret_cast<uint4 *>(sZ)[threadIdx.x] = make_uint4(0u, 0u, 0u, 0u);
-    const int bands = H / TH;
+    const int bands = Hg / TH;
     const long long units = (long long)nb * bands;
     const uint32_t sW_a = smem_u32(sW), sB_a = smem_u32(sB), sZ_a = smem_u32(sZ);
+    auto fdiv = [](int a) { return a >= 0 ? a / S : -((-a + S - 1) / S); };  // floor(a / S)
     auto stage = [&](long long u, int b) {
         const long long n = u / bands;
         const int y0 = (int)(u - n * bands) * TH;
+        const int ylo = fdiv(y0 - 1);
         const uint32_t dst = sB_a + (uint32_t)(b * BUF) * 2u;
         const int rowv = W * CO / 8;
         for (int i = threadIdx.x; i < RD * rowv; i += NW_THREADS) {
             const int r = i / rowv, e = i - r * rowv;
-            const int y = y0 - 1 + r;
+            const int y = ylo + r;
             const bool in = y >= 0 && y < H;
             const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + (in ? y : 0)) * (long long)W) * CO) + e;
             cp_async16_cg(dst + 16u * i, src, in ? 16u : 0u);
@@ -239,6 +244,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
     for (long long u = blockIdx.x; u < units; u += gridDim.x, b ^= 1) {
         const long long n = u / bands;
         const int y0 = (int)(u - n * bands) * TH;
+        const int ylo = fdiv(y0 - 1);
         const long long un = u + gridDim.x;
         if (un < units) {
             stage(un, b ^ 1);
@@ -248,21 +254,21 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
         }
         __syncthreads();
         const uint32_t sD_a = sB_a + (uint32_t)(b * BUF) * 2u;
-        if (warp * 16 < TH * W) {
+        if (warp * 16 < TH * Wg) {
             float acc[CI / 8][4];
 #pragma unroll
             for (int j = 0; j < CI / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
-            // this lane's A row: pixel warp*16 + (lane&7) + ((lane>>3)&1)*8, k half (lane>>4)*8
+            // this lane's A row: G pixel warp*16 + (lane&7) + ((lane>>3)&1)*8, k half (lane>>4)*8
             const int pa = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
-            const int ya = pa / W, xa = pa - ya * W;
+            const int ya = pa / Wg, xa = pa - ya * Wg;
             const int kh = (lane >> 4) * 8;
 #pragma unroll
             for (int tap = 0; tap < 9; ++tap) {
                 const int dy = tap / 3, dx = tap % 3;
-                const int xs = xa + 1 - dx, ys = ya + 1 - dy;  // staged row ys + 1 - 1 (halo row 0 = y0 - 1)
-                const int yi = y0 + ys;
-                const bool ok = xs >= 0 && xs < W && yi >= 0 && yi < H;
-                const uint32_t arow = ok ? sD_a + (uint32_t)(((ys + 1) * W + xs) * CO) * 2u : sZ_a;
+                const int ty = y0 + ya + 1 - dy, tx = xa + 1 - dx;  // S * (delta pixel) when it exists
+                const int ys = fdiv(ty), xs = fdiv(tx);
+                const bool ok = ys * S == ty && xs * S == tx && ys >= 0 && ys < H && xs >= 0 && xs < W;
+                const uint32_t arow = ok ? sD_a + (uint32_t)(((ys - ylo) * W + xs) * CO) * 2u : sZ_a;
 #pragma unroll
                 for (int ks = 0; ks < CO / 16; ++ks) {
                     uint32_t a0, a1, a2, a3;
@@ -281,8 +287,8 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
 #pragma unroll
             for (int h2 = 0; h2 < 2; ++h2) {
                 const int p = p0 + 8 * h2;
-                const int yy = y0 + p / W, xx = p % W;
-                float *dst = G + (((n * H + yy) * (long long)W + xx) * CI) + 2 * (lane & 3);
+                const int yy = y0 + p / Wg, xx = p % Wg;
+                float *dst = G + (((n * Hg + yy) * (long long)Wg + xx) * CI) + 2 * (lane & 3);
 #pragma unroll
                 for (int nt = 0; nt < CI / 8; ++nt)
                     *reinterpret_cast<float2 *>(dst + nt * 8) = make_float2(acc[nt][2 * h2], acc[nt][2 * h2 + 1]);
@@ -292,19 +298,24 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
     }
 }
 
-bool narrow_dgrad_supported(int cin, int cout, int H, int W) {
-    if (!((cin == 16 || cin == 32) && (cout == 16 || cout == 32))) return false;
-    if (W > NW_P || NW_P % W || W % 16) return false;
-    const int TH = std::min(H, NW_P / W);
-    return H % TH == 0;
+// H x W is the delta (output) size; G is (S*H) x (S*W)
+bool narrow_dgrad_supported(int cin, int cout, int H, int W, int stride) {
+    if (!((cin == 16 && (cout == 16 || cout == 32)) || (cin == 32 && (cout == 16 || cout == 32 || cout == 64))))
+        return false;
+    if (stride != 1 && stride != 2) return false;
+    const int Wg = stride * W, Hg = stride * H;
+    if (Wg > NW_P || NW_P % Wg || Wg % 16) return false;
+    const int TH = std::min(Hg, NW_P / Wg);
+    return Hg % TH == 0 && TH % stride == 0;
 }
 
-template <int CI, int CO>
+template <int CI, int CO, int S>
 static cudaError_t launch_nd(const uint16_t *D, const uint16_t *Wt, float *G, int nb, int H, int W, cudaStream_t s,
                              int num_sms) {
-    const int TH = std::min(H, NW_P / W);
-    const size_t smem = (size_t)9 * CI * CO * 2 + 2 * (size_t)(TH + 2) * W * CO * 2 + CO * 2;
-    auto kern = narrow_dgrad_kernel<CI, CO>;
+    const int Hg = S * H, Wg = S * W;
+    const int TH = std::min(Hg, NW_P / Wg);
+    const size_t smem = (size_t)9 * CI * CO * 2 + 2 * (size_t)(TH / S + 2) * W * CO * 2 + CO * 2;
+    auto kern = narrow_dgrad_kernel<CI, CO, S>;
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
@@ -314,21 +325,28 @@ static cudaError_t launch_nd(const uint16_t *D, const uint16_t *Wt, float *G, in
     int per_sm = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW_THREADS, smem) != cudaSuccess || per_sm < 1)
         per_sm = 1;
-    const long long units = (long long)nb * (H / TH);
+    const long long units = (long long)nb * (Hg / TH);
     if (units == 0) return cudaSuccess;
     const int grid = (int)std::min<long long>(units, (long long)num_sms * per_sm);
     sk_launch(kern, grid, NW_THREADS, smem, s, D, Wt, G, nb, H, W, TH);
     return cudaGetLastError();
 }
 
-// G [nb][H][W][cin] fp32 = stride-1 dgrad of D [nb][H][W][cout] through Wt [cin][9][cout] (bf16)
+// G [nb][S*H][S*W][cin] fp32 = dgrad of D [nb][H][W][cout] through Wt [cin][9][cout] (bf16)
 cudaError_t launch_narrow_dgrad(const uint16_t *D, const uint16_t *Wt, float *G, int nb, int H, int W, int cin, int cout,
-                                cudaStream_t s, int num_sms) {
-    if (!narrow_dgrad_supported(cin, cout, H, W)) return cudaErrorInvalidValue;
-    if (cin == 16 && cout == 16) return launch_nd<16, 16>(D, Wt, G, nb, H, W, s, num_sms);
-    if (cin == 16 && cout == 32) return launch_nd<16, 32>(D, Wt, G, nb, H, W, s, num_sms);
-    if (cin == 32 && cout == 16) return launch_nd<32, 16>(D, Wt, G, nb, H, W, s, num_sms);
-    if (cin == 32 && cout == 32) return launch_nd<32, 32>(D, Wt, G, nb, H, W, s, num_sms);
+                                int stride, cudaStream_t s, int num_sms) {
+    if (!narrow_dgrad_supported(cin, cout, H, W, stride)) return cudaErrorInvalidValue;
+#define ND_CASE(CI_, CO_, S_) \
+    if (cin == CI_ && cout == CO_ && stride == S_) return launch_nd<CI_, CO_, S_>(D, Wt, G, nb, H, W, s, num_sms)
+    ND_CASE(16, 16, 1);
+    ND_CASE(16, 32, 1);
+    ND_CASE(32, 16, 1);
+    ND_CASE(32, 32, 1);
+    ND_CASE(16, 16, 2);
+    ND_CASE(16, 32, 2);
+    ND_CASE(32, 32, 2);
+    ND_CASE(32, 64, 2);
+#undef ND_CASE
     return cudaErrorInvalidValue;
 }
 

@@ -93,7 +93,7 @@ def _load():
         "skipper_k_conv_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
         "skipper_k_conv_wgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
         "skipper_k_narrow_wgrad": (I, [P, P, P, I, I, I, I, I, I, I, P]),
-        "skipper_k_narrow_dgrad": (I, [P, P, P, I, I, I, I, I, P]),
+        "skipper_k_narrow_dgrad": (I, [P, P, P, I, I, I, I, I, I, P]),
         "skipper_k_conv_lif": (I, [P, P, P, P, P, P, I, I, I, I, I, I, I, ct.c_float, ct.c_float, P]),
         "skipper_k_num_sms": (I, []),
         "skipper_k_conv_s": (I, [P, P, P, I, I, I, I, I, I, I, P]),
@@ -507,13 +507,13 @@ def k_narrow_wgrad(D, X, stride=1, out=None):
     return out
 
 
-def k_narrow_dgrad(D, Wt):
-    """D [nb][h][w][cout], Wt [cin][3][3][cout] bf16 -> G [nb][h][w][cin] fp32 (stride-1 narrow dgrad)."""
+def k_narrow_dgrad(D, Wt, stride=1):
+    """D [nb][h][w][cout], Wt [cin][3][3][cout] bf16 -> G [nb][stride*h][stride*w][cin] fp32 (narrow dgrad)."""
     torch = _torch()
     nb, h, w, cout = D.shape
     cin = Wt.shape[0]
-    out = torch.empty((nb, h, w, cin), dtype=torch.float32, device=D.device)
-    _check(lib.skipper_k_narrow_dgrad(_ptr(D, "bf16"), _ptr(Wt, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout,
+    out = torch.empty((nb, stride * h, stride * w, cin), dtype=torch.float32, device=D.device)
+    _check(lib.skipper_k_narrow_dgrad(_ptr(D, "bf16"), _ptr(Wt, "bf16"), _ptr(out, "f32"), nb, h, w, cin, cout, stride,
                                       _stream_handle()))
     return out
 

@@ -136,20 +136,22 @@ def test_narrow_wgrad(nb, h, w, cin, cout, stride):
     assert (acc.cpu().double() - 2 * ref).abs().max() <= 2e-5 * ref.abs().max() + 1e-12
 
 
-@pytest.mark.parametrize("nb,h,w,cin,cout", [(3, 64, 64, 16, 16), (2, 32, 32, 32, 32), (5, 16, 16, 16, 32),
-                                              (4, 16, 16, 32, 16), (7, 4, 16, 16, 16), (2, 8, 32, 32, 32)])
-def test_narrow_dgrad(nb, h, w, cin, cout):
-    """Stride-1 narrow dgrad (staged halo, ldmatrix gathers) against the float64 conv input gradient;
-    spike-like delta and grid weights make every fp32 sum exact."""
+@pytest.mark.parametrize("nb,h,w,cin,cout,stride", [(3, 64, 64, 16, 16, 1), (2, 32, 32, 32, 32, 1), (5, 16, 16, 16, 32, 1),
+                                                     (4, 16, 16, 32, 16, 1), (7, 4, 16, 16, 16, 1), (2, 8, 32, 32, 32, 1),
+                                                     (3, 32, 32, 16, 32, 2), (2, 16, 16, 32, 64, 2), (5, 8, 8, 16, 16, 2)])
+def test_narrow_dgrad(nb, h, w, cin, cout, stride):
+    """Narrow dgrad (staged delta rows, ldmatrix gathers; stride 1 and 2) against the float64 conv input
+    gradient; h x w is the output size.  Spike-like delta and grid weights make every fp32 sum exact."""
     from paper_conf_micro_singhslsknnd22_b200 import k_narrow_dgrad
-    g = torch.Generator().manual_seed(nb * 11 + h + cin + cout)
+    g = torch.Generator().manual_seed(nb * 11 + h + cin + cout + stride)
     W = grid((cout, 3, 3, cin), gen=g)
     D = spikes((nb, h, w, cout), gen=g)
-    X = torch.zeros((nb, h, w, cin), dtype=torch.float64, requires_grad=True)
-    conv_ref(X, W).backward(D.double())
+    X = torch.zeros((nb, stride * h, stride * w, cin), dtype=torch.float64, requires_grad=True)
+    y = F.conv2d(X.permute(0, 3, 1, 2), W.permute(0, 3, 1, 2).double(), padding=1, stride=stride).permute(0, 2, 3, 1)
+    y.backward(D.double())
     ref = X.grad
     Wt = W.permute(3, 1, 2, 0).contiguous()  # [cin][3][3][cout]
-    out = k_narrow_dgrad(bf16_bits(D).cuda(), bf16_bits(Wt).cuda()).cpu().double()
+    out = k_narrow_dgrad(bf16_bits(D).cuda(), bf16_bits(Wt).cuda(), stride=stride).cpu().double()
     assert torch.equal(out, ref)
 
 
