@@ -545,9 +545,9 @@ static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvL
 // CTA pairs (SKIPPER_CL_PAIR=0 disables) when the pixel tiles of a channel tile pair up
 static bool cl_use_pair(int m_tiles) {
     const char *e = getenv("SKIPPER_CL_PAIR");  // read per launch so tests can cover both variants
-    // default on since the halo boxes and PDL: pairs with resident weight halves measured ~0.4 % faster
-    // per step on cfg 2 and cfg 3 (two alternating repetitions); before the halo boxes they were ~2 %
-    // slower.  The kernel stays bound by its TMA producer skeleton either way.
+    // default on since the halo boxes and PDL: pairs measured ~0.4-0.7 % faster per step on cfg 2 and
+    // cfg 3 (alternating repetitions); before the halo boxes they were ~2 % slower.  The kernel stays
+    // bound by its TMA producer skeleton either way.
     return (!e || atoi(e) != 0) && m_tiles % 2 == 0;
 }
 
@@ -587,7 +587,10 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
     }
     if (!make_map_2d(&tb, Wk, 9ull * a.Cin, a.Cout, CL_BK, pair ? bn / 2 : bn)) return cudaErrorInvalidValue;
     // resident weights when this CTA's half fits next to >= 4 activation stages
-    const int resb_env = getenv("SKIPPER_CL_RESB") ? atoi(getenv("SKIPPER_CL_RESB")) : 1;
+    // resident weight halves: opt-in (SKIPPER_CL_RESB=1); streaming them measured ~0.3 % faster per step on
+    // cfg 2 and cfg 3 (alternating repetitions): the resident halves leave room for only ~one row of
+    // activation stages
+    const int resb_env = getenv("SKIPPER_CL_RESB") ? atoi(getenv("SKIPPER_CL_RESB")) : 0;
     const uint32_t half_bytes = (uint32_t)a.num_kb * (uint32_t)(bn / 2) * CL_BK * 2;
     const bool resb = pair && resb_env && half_bytes + 3u * CL_AH_MAX + 8192u + 4u * a.R <= 226u * 1024u;
 #define CL_LAUNCH(BN_, PAIR_, RESB_, HALO_)                                                                    \
