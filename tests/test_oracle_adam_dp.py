@@ -26,6 +26,24 @@ def test_adam_matches_torch():
         np.testing.assert_allclose(w, p.detach().numpy(), rtol=1e-14, atol=1e-15)
 
 
+def test_adam_closed_forms():
+    """Closed forms of the bias-corrected update (reading 17): with a constant gradient g the
+    corrected moments are exactly g and g^2 at every step, so each step moves w by
+    -lr * g / (|g| + eps) (eps = 0: -lr * sign(g)); a zero gradient leaves w and the moments at 0."""
+    rng = np.random.default_rng(1)
+    w0 = rng.standard_normal(11)
+    g = rng.standard_normal(11) * 10 ** rng.uniform(-3, 2, 11)
+    lr, eps = 2e-3, 1e-8
+    w, m, v = w0.copy(), np.zeros(11), np.zeros(11)
+    for step in range(1, 40):
+        w, m, v = adam_update(w, g, m, v, step, lr=lr, eps=eps)
+        np.testing.assert_allclose(w, w0 - step * lr * g / (np.abs(g) + eps), rtol=1e-12, atol=1e-14)
+    w1, _, _ = adam_update(w0, g, np.zeros(11), np.zeros(11), 1, lr=lr, eps=0.0)
+    np.testing.assert_allclose(w1, w0 - lr * np.sign(g), rtol=0, atol=1e-15)
+    wz, mz, vz = adam_update(w0, np.zeros(11), np.zeros(11), np.zeros(11), 3, lr=lr, eps=eps)
+    assert np.array_equal(wz, w0) and not mz.any() and not vz.any()
+
+
 def _dp_worker(rank, world, port, out):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
