@@ -48,7 +48,7 @@ struct Layer {
     uint16_t *Po = nullptr;    // arena rows
     float *Useg = nullptr;     // arena rows
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
-    int fsplitT = 1;             // forward split-K of the whole-sequence first pass (fc tail layers)
+    int fsplitT = 1;             // forward split-K of the chunked first pass (fc tail layers, tail_G*S rows)
     bool cfused = false;         // conv layer: GEMM + LIF scan as one kernel (conv_lif.cu)
     uint16_t *wbp = nullptr;   // layer 0 im2col: bf16 weights zero-padded to [cout][K0]
     float *dwp = nullptr;      // layer 0 im2col: padded weight gradient
@@ -105,7 +105,9 @@ struct skipper_ctx {
     int K0 = 0;                 // im2col width (32 or 64)
     bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
     bool l0_bwd_fused = false;  // layer 0 backward: fused reverse scan + tcgen05 weight gradient
-    int tail0 = 0;              // first layer of the fc tail: the first pass runs it over all T at once
+    int tail0 = 0;              // first layer of the fc tail: the first pass runs it per chunk of tail_G segments
+    int tail_G = 1;             // segments per fc-tail chunk (fixed, independent of T: the tail's first-pass
+                                // buffers are O(tail_G * S) rows, keeping Eq.3's O(C) + O(S) law)
     uint16_t *tail_in = nullptr, *tailP[2] = {nullptr, nullptr};
     float *tail_I = nullptr;
     int in_h = 1, in_w = 1, in_c = 0;
@@ -633,15 +635,25 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         if (!l.fc) continue;
         const int rowsM = c->S * c->B;
         l.fsplit = fc_splits(rowsM, l.Cout, l.Cin, c->num_sms);
-        l.fsplitT = fc_splits(c->T * c->B, l.Cout, l.Cin, c->num_sms);
         if (i > 0) l.dsplit = fc_splits(rowsM, l.Cin, l.Cout, c->num_sms);
     }
     // The fc tail (a few thousand neurons per sample) would run as tiny latency-bound launches per
-    // segment; in the first pass it is evaluated layer-major over the whole sequence instead (its
-    // recurrences still run in time order; checkpoints are written every S rows).
+    // segment; in the first pass it is evaluated layer-major over chunks of tail_G segments instead (its
+    // recurrences still run in time order; checkpoints are written every S rows).  tail_G is the fewest
+    // segments whose rows reach a GEMM M of SKIPPER_TAIL_ROWS (default 4096 sample-rows): a constant
+    // number of rows, so the tail's buffers do not grow with T (a whole-sequence tail held an
+    // O(T * B) activation term that checkpointing never released).
     c->tail0 = c->Ls;
     while (c->tail0 > 0 && c->L[c->tail0 - 1].fc) --c->tail0;
     if (cfg->mode == SKIPPER_MODE_FULL || cfg->mode == SKIPPER_MODE_TBPTT) c->tail0 = c->Ls;
+    {
+        const char *e = getenv("SKIPPER_TAIL_ROWS");
+        const long long target = e ? std::max(1, atoi(e)) : 4096;
+        const long long sb = (long long)c->S * c->B;
+        c->tail_G = (int)std::min<long long>(c->C, std::max<long long>(1, (target + sb - 1) / sb));
+        for (int i = c->tail0; i < c->Ls; ++i)
+            c->L[i].fsplitT = fc_splits(c->tail_G * c->S * c->B, c->L[i].Cout, c->L[i].Cin, c->num_sms);
+    }
 
     // ---- persistent allocations
     c->dw_total = 0;
@@ -888,10 +900,10 @@ static skipper_status arena_first(skipper_ctx *c) {
     const size_t pbytes = al256(rowsB * max_nout(c) * 2);
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
-    // fc tail over all T rows: its input rows, ping-pong outputs, currents (with split partials)
+    // fc tail over one chunk of tail_G * S rows: its input rows, ping-pong outputs, currents (with split partials)
     size_t tin = 0, tp = 0, ti = 0;
     if (c->tail0 < c->Ls) {
-        const size_t rowsT = (size_t)c->T * c->B;
+        const size_t rowsT = (size_t)c->tail_G * c->S * c->B;
         tin = al256(rowsT * (c->tail0 == 0 ? c->in_row : c->L[c->tail0 - 1].Nout) * 2);
         long long mo = 0, mi = 0;
         for (int i = c->tail0; i < c->Ls; ++i) {
@@ -1124,36 +1136,38 @@ static void set_res_fwd(const skipper_ctx *c, int i, sk::ScanFwdArgs &a, const u
     a.res_lo = (l.Cout - src.Cout) / 2;
 }
 
-// First pass of the fc tail over all T rows (layer-major): GEMM with M = T*B, one scan per layer.
-static skipper_status forward_tail_first(skipper_ctx *c) {
+// First pass of the fc tail over segments g0 .. g0+nseg-1 (layer-major): GEMM with M = nseg*S*B, one scan
+// per layer; tail_in holds the chunk's input rows (written by the last conv layer, or staged here).
+static skipper_status forward_tail_chunk(skipper_ctx *c, int g0, int nseg) {
     if (c->tail0 >= c->Ls) return SKIPPER_OK;
-    const int T = c->T;
+    const int R = nseg * c->S, t0 = g0 * c->S;
     if (c->tail0 == 0) {
         uint16_t *save = c->xg;
         c->xg = c->tail_in;
-        skipper_status st = stage_input(c, nullptr, 0, T, true);
+        skipper_status st = stage_input(c, nullptr, t0, R, true);
         c->xg = save;
         CKS(st);
     }
     for (int i = c->tail0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
+        const size_t bn = (size_t)c->B * l.N;
         const uint16_t *in = i == c->tail0 ? c->tail_in : c->tailP[(i - c->tail0 - 1) & 1];
         uint16_t *out = c->tailP[(i - c->tail0) & 1];
-        CKS(gemm_forward(c, i, in, c->tail_I, T, l.fsplitT));
+        CKS(gemm_forward(c, i, in, c->tail_I, R, l.fsplitT));
         sk::ScanFwdArgs a{};
         a.I = c->tail_I;
         a.nsplit = l.fsplitT;
-        a.split_stride = (long long)T * c->B * l.N;
-        a.R = T;
+        a.split_stride = (long long)R * c->B * l.N;
+        a.R = R;
         a.U_state = l.U_run;
         a.o_state = l.o_run;
         a.Po_out = out;
-        a.ckU = l.ckU;
-        a.cko = l.cko;
+        a.ckU = l.ckU + (size_t)g0 * bn;
+        a.cko = l.cko + (size_t)g0 * bn;
         a.ck_every = c->S;
         a.s_part = spart(c, i + 1);
         a.u2_part = c->u2_part;
-        a.t0 = 0;
+        a.t0 = t0;
         a.cnt = (i == c->Ls - 1) ? c->cnt : nullptr;
         a.dbg_U = c->cfg.debug_record ? l.dbg[0] : nullptr;
         a.dbg_o = c->cfg.debug_record ? l.dbgo[0] : nullptr;
@@ -1311,7 +1325,9 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
             out = l.Po;
         } else {
             in = i == 0 ? c->xg : c->P2[(i - 1) % c->nP];
-            out = (i == c->tail0 - 1 && c->tail0 < c->Ls) ? c->tail_in + (size_t)t0 * c->B * l.Nout : c->P2[i % c->nP];
+            out = (i == c->tail0 - 1 && c->tail0 < c->Ls)
+                      ? c->tail_in + (size_t)(seg % c->tail_G) * c->S * c->B * l.Nout  // row in the tail chunk
+                      : c->P2[i % c->nP];
         }
         if (i == 0 && c->l0_fused) {
             CKS(layer0_fused(c, seg, R, t0, nullptr, false, record, out));
@@ -1848,11 +1864,13 @@ extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int p
         if (c->phase != PH_FIRST || seg != c->next_seg)
             return fail(c, SKIPPER_EORDER, "FIRST segments must run 0..C-1 in order (expected %d)", c->next_seg);
         if (x_dev != c->x_cur) return fail(c, SKIPPER_EINVAL, "x_dev changed within an iteration");
+        // checked before any work or state change, so a retry with labels can continue from here
+        if (seg == c->C - 1 && !labels_dev) return fail(c, SKIPPER_EINVAL, "the last FIRST segment needs labels");
         CKS(forward_rows_first(c, seg, c->S, seg * c->S, false));
         c->next_seg = seg + 1;
+        if ((seg + 1) % c->tail_G == 0 || seg == c->C - 1)  // the fc tail of the chunk that ends here
+            CKS(forward_tail_chunk(c, seg - seg % c->tail_G, seg % c->tail_G + 1));
         if (seg == c->C - 1) {
-            if (!labels_dev) return fail(c, SKIPPER_EINVAL, "the last FIRST segment needs labels");
-            CKS(forward_tail_first(c));
             CKS(finish_first(c, labels_dev));
             CKS(arena_rows(c, c->Kmax));
             c->phase = PH_READY_BWD;

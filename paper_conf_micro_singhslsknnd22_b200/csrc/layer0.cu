@@ -243,10 +243,12 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
         int ptile = tile, pri = ri;  // fetch cursor, L0_PD rows (of this group) ahead
         int cb = 0, cxx = 0, cyy = 0;  // build cursor's pixel
         // im2col row of (pixel, input row ri) -> the layer-0 weight-gradient operand xg [R][B*H*W][32]
-        auto store_xg = [&](int rr, uint32_t m) {
-            if (cb >= a.B) return;
-            uint4 *dst = reinterpret_cast<uint4 *>(a.xg_out + (((long long)rr * a.B + cb) * a.H * a.W +
-                                                               (long long)cyy * a.W + cxx) * 32);
+        // (b, yy, xx): the pixel the row was BUILT for - the build cursor may already have moved on to the
+        // next tile when the row is stored
+        auto store_xg = [&](int rr, uint32_t m, int b, int yy, int xx) {
+            if (b >= a.B) return;
+            uint4 *dst = reinterpret_cast<uint4 *>(a.xg_out + (((long long)rr * a.B + b) * a.H * a.W +
+                                                               (long long)yy * a.W + xx) * 32);
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
                 const uint2 lo = s_lut[(m >> (8 * j)) & 15u], hi = s_lut[(m >> (8 * j + 4)) & 15u];
@@ -270,7 +272,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 const uint32_t nib = byte_bits4(c0.x) | byte_bits4(c0.y) << 4 | byte_bits4(c1.x) << 8 | byte_bits4(c1.y) << 12;
                 m |= ((nib >> sh) & wmask) << (dy * 3 * a.C0);
             }
-            store_xg(0, m);
+            store_xg(0, m, cb, cyy, cxx);
         };
         auto build_pixel = [&](int tile) {
             int b0, y0, x0;
@@ -292,6 +294,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
         while (tile < tiles && nit_tile > 0) {
             L0_T0; cp_async_wait<L0_PD - 1>(); L0_T1(1); L0_T0;  // this row's group has landed
             const bool cok = cb < a.B;
+            const int xb = cb, xy = cyy, xx = cxx;  // this row's pixel (the cursor advances below)
             const int cshift = (a.C0 * (cxx - 1)) & 7;  // window offset in its first chunk
             const int cri = ri;
             // build the im2col row: bit (dy*3+dx)*C0+ci <- window byte dx*C0+ci of row dy
@@ -326,7 +329,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
                 if (lane == 0 && v) atomicAdd(&row_cnt_in[cri], v);
             }
-            if (a.xg_out) store_xg(cri, m);
+            if (a.xg_out) store_xg(cri, m, xb, xy, xx);
             L0_T1(5); L0_T0; fence_async_shared(); L0_T1(6);
             __syncwarp();
             if (lane == 0) mbar_arrive(full_bar(stage));

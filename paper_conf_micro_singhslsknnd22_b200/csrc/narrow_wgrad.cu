@@ -299,10 +299,16 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
 }
 
 // H x W is the delta (output) size; G is (S*H) x (S*W)
+// exactly the (cin, cout, stride) instantiations of launch_narrow_dgrad below: a layer this predicate
+// rejects takes the GEMM + col2im branch of the engine instead of failing the step
+static bool nd_instantiated(int cin, int cout, int stride) {
+    if (stride == 1) return (cin == 16 && (cout == 16 || cout == 32)) || (cin == 32 && (cout == 16 || cout == 32));
+    if (stride == 2) return (cin == 16 && (cout == 16 || cout == 32)) || (cin == 32 && (cout == 32 || cout == 64));
+    return false;
+}
+
 bool narrow_dgrad_supported(int cin, int cout, int H, int W, int stride) {
-    if (!((cin == 16 && (cout == 16 || cout == 32)) || (cin == 32 && (cout == 16 || cout == 32 || cout == 64))))
-        return false;
-    if (stride != 1 && stride != 2) return false;
+    if (!nd_instantiated(cin, cout, stride)) return false;
     const int Wg = stride * W, Hg = stride * H;
     if (Wg > NW_P || NW_P % Wg || Wg % 16) return false;
     const int TH = std::min(Hg, NW_P / Wg);

@@ -19,10 +19,11 @@ def _cuda():
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
 
 
-def run_gpu(net, W, x, y, T, C, p, mode, steps=1, sam="spikes"):
+def run_gpu(net, W, x, y, T, C, p, mode, steps=1, sam="spikes", surrogate="triangle", gamma=0.3):
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
     B = x.shape[1]
-    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True, sam=sam)
+    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True, sam=sam, surrogate=surrogate,
+                   gamma=gamma)
     m.set_weights(W)
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     yd = torch.from_numpy(np.ascontiguousarray(y)).cuda()
@@ -46,22 +47,29 @@ def grad_ok(g, r, tol=(1e-3, 1e-3)):
     return rel <= tol[0] and mx <= tol[1], f"normwise {rel:.2e} maxabs {mx:.2e}"
 
 
-def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=False):
+def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=False, theta=None, wscale=1.0,
+                 surrogate="triangle", gamma=0.3, x_fn=None):
     """deep=True (networks deeper than the 11 spiking layers of VGG-11): a layer's dW tolerance is
     max(1e-3, twice the size of the bf16 contract's own effect on that layer), normwise and max-abs,
-    DESIGN.md §4 "deep networks"."""
-    net = synth.net_config(name, lam=lam)
+    DESIGN.md §4 "deep networks".  theta / wscale: threshold of every spiking layer and a power-of-two
+    scale of their (grid) weights; surrogate / gamma: reading 4; x_fn: transforms the seeded input."""
+    net = synth.net_config(name, lam=lam, theta=theta)
     W = synth.make_weights(net, seed=seed)
+    W = [w * np.float32(wscale) if L["kind"] != "readout" else w for w, L in zip(W, net["layers"])]
     x, y = synth.make_inputs(net, T, B, seed=seed + 1)
-    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True, sam=sam))
+    if x_fn is not None:
+        x = np.ascontiguousarray(x_fn(x))
+    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, record=True, sam=sam, surrogate=surrogate,
+                                              gamma=gamma))
     tols = [(1e-3, 1e-3)] * len(ref.dW)
     if deep:
-        exact = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, sam=sam, emulate_bf16=False))
+        exact = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode=mode, sam=sam, emulate_bf16=False,
+                                                     surrogate=surrogate, gamma=gamma))
         tols = []
         for a, b in zip(ref.dW, exact.dW):
             en, em = grad_errs(b, a)
             tols.append((max(1e-3, 2 * en), max(1e-3, 2 * em)))
-    m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam)
+    m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam, surrogate=surrogate, gamma=gamma)
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
     # SAM and mask (Eq.4, Eq.5)
     np.testing.assert_array_equal(m.spike_sums(), ref.s)
@@ -117,6 +125,44 @@ def test_tiny_fc(mode, lam):
 @pytest.mark.parametrize("mode,lam", [("full", 0.99), ("ckpt", 1.0), ("skip", 0.99), ("skip", 0.75)])
 def test_tiny_conv(mode, lam):
     check_parity("tiny_conv", T=12, B=3, C=2, p=50.0, mode=mode, lam=lam)
+
+
+@pytest.mark.parametrize("name,T,B,theta,wscale,surrogate,gamma", [
+    ("tiny_conv", 12, 3, 2.0, 2.0, "triangle", 0.3), ("tiny_conv", 12, 3, 0.5, 1.0, "triangle", 0.3),
+    ("tiny_fc", 12, 3, 0.5, 0.5, "fast_sigmoid", 2.0), ("tiny_conv", 12, 3, 1.0, 1.0, "fast_sigmoid", 4.0),
+    ("vgg5", 14, 2, 2.0, 2.0, "fast_sigmoid", 1.0), ("tiny_resnet", 16, 3, 0.5, 0.5, "triangle", 0.5),
+    ("fc784", 20, 4, 2.0, 2.0, "triangle", 0.3)])
+def test_theta_and_surrogate(name, T, B, theta, wscale, surrogate, gamma):
+    """theta != 1 (the /theta of the triangle surrogate and the theta*o reset, reading 1 and 4) and the
+    fast-sigmoid surrogate (reading 4) on the device, every kernel kind that evaluates sigma'."""
+    check_parity(name, T=T, B=B, C=2, p=50.0, mode="skip", theta=theta, wscale=wscale, surrogate=surrogate,
+                 gamma=gamma)
+
+
+@pytest.mark.parametrize("name,T,B,C,p,pulse", [("tiny_conv", 12, 3, 2, 90.0, True), ("tiny_conv", 12, 3, 2, 99.0, False),
+                                                ("vgg5", 24, 2, 2, 95.0, True), ("tiny_fc", 12, 3, 2, 99.0, True),
+                                                ("tiny_resnet", 16, 2, 2, 99.0, True), ("fc784", 20, 4, 2, 99.0, True)])
+def test_high_p_single_row_segments(name, T, B, C, p, pulse):
+    """p above the Eq.7 rule of thumb (accepted with a warning, reading 20).  pulse: the input fires only at the
+    segment starts t = cS, so s_{cS} is each segment's maximum and every other step falls below SST_c: the
+    segments shrink to K_c = 1 (only the checkpoint row is recomputed and back-propagated)."""
+    S = T // C
+    fn = (lambda x: np.where((np.arange(x.shape[0]) % S == 0).reshape((-1,) + (1,) * (x.ndim - 1)), x, 0)) if pulse else None
+    _, ref = check_parity(name, T=T, B=B, C=C, p=p, mode="skip", x_fn=fn)
+    if pulse:
+        assert all(len(k) == 1 for k in ref.kept), [len(k) for k in ref.kept]
+
+
+@pytest.mark.parametrize("name,how", [("tiny_conv", "zeros"), ("tiny_conv", "frozen"), ("vgg5", "zeros"),
+                                      ("tiny_fc", "frozen")])
+def test_tied_spike_sums(name, how):
+    """Ties in s_t (reading 13: strict '>', ties skipped).  'zeros': an all-zero input keeps every layer silent,
+    s_t = 0 for all t, every step ties the SST and only checkpoint rows are kept (all-zero gradients).
+    'frozen': one input frame repeated, so s_t saturates into repeated values within a segment."""
+    fn = (lambda x: np.zeros_like(x)) if how == "zeros" else (lambda x: np.repeat(x[:1], x.shape[0], axis=0))
+    _, ref = check_parity(name, T=12 if name != "vgg5" else 14, B=2, C=2, p=40.0, mode="skip", x_fn=fn)
+    if how == "zeros":
+        assert (ref.s == 0).all() and all(len(k) == 1 for k in ref.kept)
 
 
 @pytest.mark.parametrize("mode", ["full", "skip"])
@@ -193,6 +239,36 @@ def test_memory_ordering_full_ckpt_skip():
         peaks[mode] = m.mem_stats()[1]
         m.close()
     assert peaks["full"] > peaks["ckpt"] > peaks["skip"], peaks
+
+
+@pytest.mark.parametrize("name,B", [("vgg5", 8), ("fc784", 64)])
+def test_measured_peak_sublinear_in_T(name, B):
+    """Eq.3 / Eq.6 on the device's allocator (not the analytic model): at C = sqrt(T) the peak device memory
+    of CKPT and SKIP grows like sqrt(T) (x4 over a x16 range of T, plus T-independent weights / buffers)
+    while FULL BPTT's grows linearly.  Covers the fc tail's chunked first pass."""
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    net = synth.net_config(name)
+    W = synth.make_weights(net)
+    Ts = (64, 256, 1024)
+    x, y = synth.make_inputs(net, Ts[-1], B)
+    xd, yd = torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda()
+    peak = {}
+    for mode, p in (("ckpt", 0.0), ("skip", 50.0), ("full", 0.0)):
+        for T in Ts:
+            C = int(round(T ** 0.5))
+            m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B)
+            m.set_weights(W)
+            m.step(xd[:T].contiguous(), yd)
+            peak[mode, T] = m.mem_stats()[1]
+            m.close()
+    # T grows x4 per point: stored state ~ sqrt(T) grows its INCREMENT x2 per point, linear growth x4 (the
+    # T-independent part - weights, Adam moments, shadows, running state - cancels in the increments)
+    inc = {mode: (peak[mode, Ts[2]] - peak[mode, Ts[1]]) / (peak[mode, Ts[1]] - peak[mode, Ts[0]])
+           for mode in ("ckpt", "skip", "full")}
+    print(name, {k: round(v / 1e6, 1) for k, v in peak.items()}, inc)
+    assert inc["ckpt"] < 2.6 and inc["skip"] < 2.6, (inc, peak)
+    assert inc["full"] > 3.0, (inc, peak)
+    assert peak["skip", Ts[-1]] <= peak["ckpt", Ts[-1]] < peak["full", Ts[-1]], peak
 
 
 @pytest.mark.parametrize("mode", ["skip", "full"])
@@ -372,23 +448,66 @@ def test_full_size_sampled_parity(name, samples):
     m.close()
 
 
-def test_full_size_sampled_vgg11():
-    """cfg 3 (VGG-11, T=200, B=128, C=5, p=50) at full size: sampled first-pass states exact against the
-    oracle (its full-batch first pass is too slow for a test), and properties at full size: the keep mask
-    is Eq.5 applied to the device's own s_t, and s_t equals the device's per-layer counts summed."""
+def test_full_size_vgg11_forward():
+    """cfg 3 (VGG-11, T=200, B=128, C=5, p=50) at full size: s_t, per-layer counts, keep mask and loss against
+    the oracle's full-batch first pass (batch slices on the host cores); first-pass and recomputed spikes /
+    membranes of sampled batch elements against the oracle with its own mask imposed."""
+    from _oracle_pool import full_batch_forward
+    from oracle.bptt import readout
+    from oracle.numerics import bf16_round
     from oracle.skipper import keep_mask
     wl = synth.workload("cfg3_vgg11")
     net, W, x, y, m, loss = _full_size_gpu(wl)
-    s = m.spike_sums()
-    np.testing.assert_array_equal(m.layer_spike_counts().sum(axis=0), s)
-    np.testing.assert_array_equal(m.keep_mask(), keep_mask(s, wl["T"], wl["C"], wl["p"]))
-    assert 0 < m.keep_mask().sum() < wl["T"] and np.isfinite(loss)
-    spk = [L for L in net["layers"] if L["kind"] != "readout"]
-    samples = [0, 127]
-    ref = train_step(net, W, np.ascontiguousarray(x[:, samples]), y[samples],
-                     StepConfig(T=wl["T"], C=wl["C"], p=0.0, mode="ckpt", record=True, global_batch=wl["B"]))
-    for l in range(len(spk)):
-        got = m.debug(1, l)[:, samples].cpu().numpy()
-        assert np.array_equal(got, ref.first_o[l]), f"layer {l}: {np.count_nonzero(got != ref.first_o[l])} differ"
-        np.testing.assert_allclose(m.debug(0, l)[:, samples].cpu().numpy(), ref.first_U[l], rtol=1e-5, atol=1e-6)
+    counts, cnt = full_batch_forward(wl["net"], wl["T"], wl["B"], wl["C"])
+    s = counts.sum(axis=0)
+    np.testing.assert_array_equal(m.layer_spike_counts(), counts)
+    np.testing.assert_array_equal(m.spike_sums(), s)
+    keep = keep_mask(s, wl["T"], wl["C"], wl["p"])
+    np.testing.assert_array_equal(m.keep_mask(), keep)
+    assert 0 < keep.sum() < wl["T"]
+    ref_loss, _, _ = readout(bf16_round(W[-1]), cnt, y, wl["T"], wl["B"], False)
+    assert loss == pytest.approx(ref_loss, rel=1e-5)
+    _check_sampled(net, W, x, y, m, wl, [0, 77, 127], keep)
     m.close()
+
+
+@pytest.mark.parametrize("name,T,C,mode", [("cfg2_vgg5", 0, 0, "skip"), ("cfg2_vgg5", 0, 0, "full"),
+                                           ("cfg3_vgg11", 24, 2, "skip"), ("cfg4_resnet_dvs", 0, 0, "skip")])
+def test_full_size_backward_parity(name, T, C, mode):
+    """Weight gradients at the BASELINE.json batch sizes in bench.py's launch configuration (no debug
+    recording): cfg 2 at full size (T=100, B=64, C=10, p=40), cfg 3 at its full batch B=128 (the batch decides
+    the kernel paths: fused conv+LIF, split-K counts of the fc GEMMs) with T=24, C=2, and cfg 4 at full size
+    (T=300, B=32).  The oracle's dW is the sum of batch-slice training steps with the global keep mask (from its
+    own full-batch first pass) and the global batch size imposed.  Tolerances as check_parity (cfg 4: deep)."""
+    from _oracle_pool import full_batch_forward, full_batch_train
+    from oracle.skipper import keep_mask
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    wl = synth.workload(name)
+    if T:
+        wl["T"], wl["C"] = T, C
+    net = synth.net_config(wl["net"])
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, wl["T"], wl["B"])
+    m = SkipperNet(net, wl["T"], C=wl["C"], p=wl["p"], mode=mode, batch=wl["B"])
+    m.set_weights(W)
+    loss = m.step(torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda())
+    grads = [g.cpu().numpy() for g in m.grads()]
+    keep = None
+    if mode == "skip":
+        counts, _ = full_batch_forward(wl["net"], wl["T"], wl["B"], wl["C"])
+        keep = keep_mask(counts.sum(axis=0), wl["T"], wl["C"], wl["p"])
+        np.testing.assert_array_equal(m.keep_mask(), keep)
+    m.close()
+    dW, ref_loss = full_batch_train(wl["net"], wl["T"], wl["B"], wl["C"], wl["p"], mode, keep)
+    assert loss == pytest.approx(ref_loss, rel=1e-5)
+    deep = name.startswith("cfg4")
+    tols = [(1e-3, 1e-3)] * len(dW)
+    if deep:   # DESIGN.md §4 "deep networks": twice the bf16 contract's own effect, per layer
+        exact, _ = full_batch_train(wl["net"], wl["T"], wl["B"], wl["C"], wl["p"], mode + "_exact", keep)
+        tols = [(max(1e-3, 2 * grad_errs(b, a)[0]), max(1e-3, 2 * grad_errs(b, a)[1])) for a, b in zip(dW, exact)]
+    report = []
+    for l, (g, r) in enumerate(zip(grads, dW)):
+        ok, msg = grad_ok(g, r, tols[l])
+        report.append(f"layer {l}: {msg}")
+        assert ok, f"layer {l} dW: {msg} (tolerance {tols[l][0]:.1e}, {tols[l][1]:.1e})"
+    print(name, mode, "; ".join(report))

@@ -149,3 +149,23 @@ def test_data_parallel_bucketed_allreduce_gloo():
     np.testing.assert_array_equal(keep, ref.keep)
     for a, b in zip(grads, ref.dW):
         np.testing.assert_allclose(a, b, rtol=1e-10, atol=1e-14)
+
+
+def test_batch_slice_pool_equals_full_batch():
+    """tests/_oracle_pool.full_batch_train (the full-size backward parity reference): slices with the global
+    keep mask and batch size imposed sum to the full-batch oracle step."""
+    from _oracle_pool import full_batch_forward, full_batch_train
+    from oracle.skipper import keep_mask
+    name, T, B, C, p = "tiny_conv", 12, 5, 2, 50.0
+    net = synth.net_config(name)
+    W = synth.make_weights(net)
+    x, y = synth.make_inputs(net, T, B)
+    ref = train_step(net, W, x, y, StepConfig(T=T, C=C, p=p, mode="skip"))
+    counts, _ = full_batch_forward(name, T, B, C, workers=2)
+    np.testing.assert_array_equal(counts, ref.counts)
+    keep = keep_mask(counts.sum(axis=0), T, C, p)
+    np.testing.assert_array_equal(keep, ref.keep)
+    dW, loss = full_batch_train(name, T, B, C, p, "skip", keep, workers=3)
+    assert loss == pytest.approx(ref.loss, rel=1e-12)
+    for a, b in zip(dW, ref.dW):
+        np.testing.assert_allclose(a, b, rtol=1e-12, atol=1e-15)

@@ -322,3 +322,85 @@ def test_tbptt_forward_state_is_not_truncated():
         np.testing.assert_array_equal(a, b)
     np.testing.assert_array_equal(rt.s, rf.s)
     assert rt.ledger_peak * 3 == rf.ledger_peak      # one window of t' = T/3 stored at a time
+
+
+# ---- the surrogate's threshold scaling and the fast-sigmoid branch (reading 4), pinned by autograd
+# on the surrogate's ANTIDERIVATIVE: the spike is Heaviside in the forward value and F(U - theta) in the
+# backward (straight-through, F - F.detach()), so torch differentiates F itself and nothing of sigma' is
+# retyped here.  Triangle: F(x) = gamma (x - x|x| / (2 theta)) on |x| <= theta, constant outside, whose
+# derivative is gamma max(0, 1 - |x| / theta).  Fast sigmoid: F(x) = x / (1 + kappa |x|), the fast sigmoid
+# itself, whose derivative is 1 / (1 + kappa |x|)^2.
+
+def st_spike(U, theta, kind, gamma):
+    x = U - theta
+    if kind == "triangle":
+        xc = torch.clamp(x, -theta, theta)
+        Fx = gamma * (xc - xc * xc.abs() / (2.0 * theta))
+    else:
+        Fx = x / (1.0 + gamma * x.abs())
+    return (x > 0).to(U.dtype) + (Fx - Fx.detach())
+
+
+def torch_full_bptt_st(net, W, x, y, kind, gamma):
+    spk = [L for L in net["layers"] if L["kind"] != "readout"]
+    Wt = [torch.tensor(w.astype(np.float64), dtype=torch.float64, requires_grad=True) for w in W]
+    T, B = x.shape[:2]
+    U = [None] * len(spk)
+    o = [None] * len(spk)
+    cnt = 0
+    nspk = 0
+    for t in range(T):
+        a = torch.tensor(x[t].astype(np.float64))
+        outs = []
+        for l, L in enumerate(spk):
+            I = t_current(L, Wt[l], a, outs[L["res"]] if "res" in L else None)
+            U[l] = I if U[l] is None else L["lam"] * U[l] + I - L["theta"] * o[l].detach()
+            o[l] = st_spike(U[l], L["theta"], kind, gamma)
+            nspk += int(o[l].detach().sum())
+            a = t_out(L, o[l])
+            outs.append(a)
+        cnt = cnt + a
+    z = t_readin(net, cnt) @ Wt[-1].T / T
+    loss = F.cross_entropy(z, torch.tensor(y, dtype=torch.long), reduction="sum") / B
+    loss.backward()
+    return float(loss.detach()), [w.grad.numpy() for w in Wt], nspk
+
+
+@pytest.mark.parametrize("name,lam,theta,wscale,kind,gamma", [
+    ("tiny_fc", 0.5, 2.0, 2.0, "triangle", 0.3),
+    ("tiny_fc", 1.0, 0.5, 1.0, "triangle", 0.3),
+    ("tiny_conv", 0.75, 2.0, 2.0, "triangle", 0.3),
+    ("tiny_conv", 1.0, 0.5, 0.5, "triangle", 0.5),
+    ("tiny_resnet", 0.75, 0.5, 1.0, "triangle", 0.3),
+    ("tiny_fc", 0.5, 1.0, 1.0, "fast_sigmoid", 2.0),
+    ("tiny_conv", 0.75, 2.0, 2.0, "fast_sigmoid", 4.0),
+    ("tiny_resnet", 1.0, 0.5, 0.5, "fast_sigmoid", 1.0),
+])
+def test_full_bptt_surrogate_theta_and_kind_equal_autograd(name, lam, theta, wscale, kind, gamma):
+    """theta != 1 and the fast-sigmoid surrogate: the oracle's sigma' (oracle/lif.py surrogate_grad) against
+    autograd through the antiderivative.  Weights are scaled by a power of two (exact on the grid) so the
+    network fires at theta != 1."""
+    T = 6
+    net = synth.net_config(name, lam=lam, theta=theta)
+    W = [w * np.float32(wscale) if L["kind"] != "readout" else w for w, L in zip(synth.make_weights(net), net["layers"])]
+    x, y = synth.make_inputs(net, T, 3, seed=1)
+    r = train_step(net, W, x, y, StepConfig(T=T, mode="full", emulate_bf16=False, surrogate=kind, gamma=gamma))
+    loss, grads, nspk = torch_full_bptt_st(net, W, x, y, kind, gamma)
+    assert nspk > 0, "the network never fired"
+    assert r.loss == pytest.approx(loss, rel=1e-12)
+    assert all(np.abs(g).max() > 0 for g in grads[:-1]), "a spiking layer received no gradient"
+    for l, (a, b) in enumerate(zip(r.dW, grads)):
+        assert rel_err(a, b) < 1e-12 or np.abs(a - b).max() < 1e-15, (l, rel_err(a, b))
+
+
+def test_st_spike_derivatives_match_reading4_shapes():
+    """The antiderivatives above differentiate to reading 4's shapes at sample points (a check of the
+    test's own F, so that the pin above is not vacuous)."""
+    U = torch.linspace(-3.0, 5.0, 801, dtype=torch.float64, requires_grad=True)
+    for theta in (0.5, 1.0, 2.0):
+        g, = torch.autograd.grad(st_spike(U, theta, "triangle", 0.3).sum(), U)
+        x = U.detach() - theta
+        want = 0.3 * torch.clamp(1.0 - x.abs() / theta, min=0.0)
+        assert torch.allclose(g, want, atol=1e-14)
+        g, = torch.autograd.grad(st_spike(U, theta, "fast_sigmoid", 2.0).sum(), U)
+        assert torch.allclose(g, 1.0 / (1.0 + 2.0 * x.abs()) ** 2, atol=1e-14)
