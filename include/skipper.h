@@ -232,6 +232,12 @@ skipper_status skipper_profile_read(skipper_ctx *ctx, int cls, long long *launch
                                     double *flops);
 const char *skipper_profile_class_name(int cls);
 int skipper_profile_num_classes(void);
+/* The profiled scopes since the last skipper_profile() call, in launch order: kernel class, number of
+ * kernels the scope launched, algorithmic bytes and FLOPs, device ms.  Host arrays of `cap` entries (any
+ * may be NULL); synchronises the stream; returns the total number of scopes (-1 on a null context).  Used
+ * to attribute an ncu launch list to kernel classes (tools/ncu_classes.py). */
+long long skipper_profile_records(skipper_ctx *ctx, int *cls, long long *n_kernels, double *bytes, double *flops,
+                                  float *ms, long long cap);
 /* Kernel launches issued by this context since creation (always counted). */
 long long skipper_launch_count(const skipper_ctx *ctx);
 

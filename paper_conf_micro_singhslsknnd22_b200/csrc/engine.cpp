@@ -50,6 +50,13 @@ struct Layer {
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
     int fsplitT = 1;             // forward split-K of the chunked first pass (fc tail layers, tail_G*S rows)
     bool cfused = false;         // conv layer: GEMM + LIF scan as one kernel (conv_lif.cu)
+    // deterministic split-K weight gradient: wsl > 0 -> the wgrad launches add into slice s of dws
+    // [wsl][wg_count] (one writer per slice per launch), summed in slice order into dW (or dwp) after the
+    // layer's last weight-gradient launch of the step (launch_reduce_slices)
+    float *dws = nullptr;
+    int wsl = 0;
+    bool wsl_narrow = false;   // the slices are narrow_wgrad's per-CTA partials
+    size_t wg_count = 0;
     uint16_t *wbp = nullptr;   // layer 0 im2col: bf16 weights zero-padded to [cout][K0]
     float *dwp = nullptr;      // layer 0 im2col: padded weight gradient
     float *dbg[2] = {nullptr, nullptr};     // first / recompute U
@@ -106,8 +113,8 @@ struct skipper_ctx {
     bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
     bool l0_bwd_fused = false;  // layer 0 backward: fused reverse scan + tcgen05 weight gradient
     int tail0 = 0;              // first layer of the fc tail: the first pass runs it per chunk of tail_G segments
-    int tail_G = 1;             // segments per fc-tail chunk (fixed, independent of T: the tail's first-pass
-                                // buffers are O(tail_G * S) rows, keeping Eq.3's O(C) + O(S) law)
+    int tail_G = 1;             // segments per fc-tail chunk (tail_G * S * B <= max(SKIPPER_TAIL_ROWS, S * B) rows,
+                                // independent of T: keeps Eq.3's O(C) + O(S) law)
     uint16_t *tail_in = nullptr, *tailP[2] = {nullptr, nullptr};
     float *tail_I = nullptr;
     int in_h = 1, in_w = 1, in_c = 0;
@@ -170,8 +177,10 @@ struct skipper_ctx {
     bool prof_on = false;
     std::vector<cudaEvent_t> ev_pool;
     size_t ev_used = 0;
-    struct ProfRec { int cls; cudaEvent_t a, b; double bytes, flops; };
+    struct ProfRec { int cls; cudaEvent_t a, b; double bytes, flops; long long k0, nk; };
     std::vector<ProfRec> prof_recs;
+    struct ProfLog { int cls; long long nk; double bytes, flops; float ms; };
+    std::vector<ProfLog> prof_log;   // every profiled scope in launch order (ncu attribution, tools/ncu_classes.py)
     long long prof_n[16] = {0};
     double prof_ms[16] = {0}, prof_bytes[16] = {0}, prof_flops[16] = {0};
     long long launches = 0;
@@ -202,15 +211,17 @@ struct ProfScope {
     int rec = -1;
     ProfScope(skipper_ctx *c_, int cls, double bytes, double flops, cudaStream_t s_ = nullptr) : c(c_), s(s_) {
         if (!s) s = c->st;
-        c->launches++;
+        const long long k0 = c->launches++;
         if (!c->prof_on) return;
         cudaEvent_t a = ev_get(c), b = ev_get(c);
         cudaEventRecord(a, s);
-        c->prof_recs.push_back({cls, a, b, bytes, flops});
+        c->prof_recs.push_back({cls, a, b, bytes, flops, k0, 1});
         rec = (int)c->prof_recs.size() - 1;
     }
     ~ProfScope() {
-        if (rec >= 0) cudaEventRecord(c->prof_recs[rec].b, s);
+        if (rec < 0) return;
+        cudaEventRecord(c->prof_recs[rec].b, s);
+        c->prof_recs[rec].nk = c->launches - c->prof_recs[rec].k0;  // kernels launched inside the scope
     }
 };
 
@@ -225,6 +236,7 @@ static void prof_resolve(skipper_ctx *c) {
             c->prof_bytes[r.cls] += r.bytes;
             c->prof_flops[r.cls] += r.flops;
         }
+        c->prof_log.push_back({r.cls, r.nk, r.bytes, r.flops, ms});
     }
     c->prof_recs.clear();
     c->ev_used = 0;
@@ -639,18 +651,19 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     // The fc tail (a few thousand neurons per sample) would run as tiny latency-bound launches per
     // segment; in the first pass it is evaluated layer-major over chunks of tail_G segments instead (its
-    // recurrences still run in time order; checkpoints are written every S rows).  tail_G is the fewest
-    // segments whose rows reach a GEMM M of SKIPPER_TAIL_ROWS (default 4096 sample-rows): a constant
-    // number of rows, so the tail's buffers do not grow with T (a whole-sequence tail held an
+    // recurrences still run in time order; checkpoints are written every S rows).  The T*B rows are cut into
+    // ceil(T*B / SKIPPER_TAIL_ROWS) balanced chunks of whole segments (default 8192 sample-rows: the whole
+    // sequence at cfg 2): at most max(8192, S*B) rows, so the tail's buffers do not grow with T (a whole-sequence tail held an
     // O(T * B) activation term that checkpointing never released).
     c->tail0 = c->Ls;
     while (c->tail0 > 0 && c->L[c->tail0 - 1].fc) --c->tail0;
     if (cfg->mode == SKIPPER_MODE_FULL || cfg->mode == SKIPPER_MODE_TBPTT) c->tail0 = c->Ls;
     {
         const char *e = getenv("SKIPPER_TAIL_ROWS");
-        const long long target = e ? std::max(1, atoi(e)) : 4096;
-        const long long sb = (long long)c->S * c->B;
-        c->tail_G = (int)std::min<long long>(c->C, std::max<long long>(1, (target + sb - 1) / sb));
+        const long long target = e ? std::max(1, atoi(e)) : 8192;
+        const long long rows = (long long)c->T * c->B;
+        const long long nchunks = std::max<long long>(1, (rows + target - 1) / target);
+        c->tail_G = (int)std::max<long long>(1, (c->C + nchunks - 1) / nchunks);  // balanced chunks
         for (int i = c->tail0; i < c->Ls; ++i)
             c->L[i].fsplitT = fc_splits(c->tail_G * c->S * c->B, c->L[i].Cout, c->L[i].Cin, c->num_sms);
     }
@@ -714,6 +727,45 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     AL(c->dz, (size_t)c->B * ro.Cout);
     AL(c->loss_dev, 1);
     AL(c->kept_dev, (size_t)c->T);
+    // split-K slices of the weight gradients: the split count of every wgrad launch is at most the count the
+    // plan chooses at the layer's largest reduction (T rows in FULL mode, S otherwise), which sizes the slices
+    {
+        const long long Rmax = cfg->mode == SKIPPER_MODE_FULL ? c->T : c->S;
+        const long long nbmax = Rmax * c->B;
+        const bool nw_off = getenv("SKIPPER_NO_NARROW_WGRAD") && atoi(getenv("SKIPPER_NO_NARROW_WGRAD"));
+        // experiments: SKIPPER_WGRAD_ATOMIC=1 = the round-1 nondeterministic reduce-add into dW
+        const bool atomic_wg = getenv("SKIPPER_WGRAD_ATOMIC") && atoi(getenv("SKIPPER_WGRAD_ATOMIC"));
+        for (int i = 0; i < c->Ls; ++i) {
+            Layer &l = c->L[i];
+            l.wg_count = l.wcount;
+            int ns = 0;
+            if (i == 0 && c->l0_bwd_fused) {
+                ns = 0;
+            } else if (l.icol && !nw_off && sk::narrow_wgrad_supported(l.Cin, l.Cout, l.stride, l.H, l.W)) {
+                ns = sk::narrow_wgrad_slices(l.Cin, l.Cout, l.stride, l.H, l.W, c->num_sms);
+                l.wsl_narrow = true;
+                if (ns < 1) return bail(fail(c, SKIPPER_ECUDA, "narrow weight-gradient occupancy query failed"));
+            } else if (l.icol) {
+                ns = sk::fc_wgrad_splits(std::min<long long>(nbmax, icol_chunk(c)) * l.H * l.W, l.Cout, 9 * l.Cin,
+                                         c->num_sms);
+            } else if (i == 0 && c->in_kind == 1) {
+                ns = sk::fc_wgrad_splits(nbmax * l.H * l.W, l.Cout, c->K0, c->num_sms);
+                l.wg_count = (size_t)l.Cout * c->K0;
+            } else if (l.conv) {
+                ns = sk::conv_wgrad_splits(nbmax * l.H * l.W, l.Cin, l.Cout, c->num_sms);
+            } else {
+                ns = sk::fc_wgrad_splits(nbmax, l.Cout, l.Cin, c->num_sms);
+            }
+            if (atomic_wg && !l.wsl_narrow) ns = 0;   // legacy: split-K reduce-add straight into dW
+            l.wsl = ns;                               // 1: unsplit, reduce-add into dW (one writer per launch)
+            if (ns > 1 || l.wsl_narrow) {
+                l.wsl = ns;
+                AL(l.dws, (size_t)ns * l.wg_count);
+                s = zero_dev(c, l.dws, (size_t)ns * l.wg_count * 4);
+                if (s != SKIPPER_OK) return bail(s);
+            }
+        }
+    }
 #undef AL
     for (auto &l : c->L) {
         s = zero_dev(c, l.w, l.wcount * 4);
@@ -752,6 +804,7 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
             dev_free(c, l.U_run, bn * 4);
             dev_free(c, l.o_run, bn);
             dev_free(c, l.carry, bn * 4);
+            dev_free(c, l.dws, (size_t)l.wsl * l.wg_count * 4);
             dev_free(c, l.ckU, bn * c->C * 4);
             dev_free(c, l.cko, bn * c->C);
             for (int k = 0; k < 2; ++k) {
@@ -1566,6 +1619,17 @@ static skipper_status comm_after_wgrad(skipper_ctx *c, int i, cudaStream_t ws) {
     return SKIPPER_OK;
 }
 
+// segment 0 only: layer i's weight-gradient slices are final; sum them (slice order) into dW, on the stream
+// that ran the weight gradients
+static skipper_status reduce_wslices(skipper_ctx *c, int i, cudaStream_t ws) {
+    Layer &l = c->L[i];
+    if (!l.dws) return SKIPPER_OK;
+    float *dst = (i == 0 && l.dwp) ? l.dwp : l.dw;
+    ProfScope ps(c, K_GEMM_WGRAD, (double)l.wsl * l.wg_count * 8 + (double)l.wg_count * 8, 0, ws);
+    CK(sk::launch_reduce_slices(l.dws, l.wsl, dst, l.wg_count, ws));
+    return SKIPPER_OK;
+}
+
 static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, bool last_seg) {
     for (int i = c->Ls - 1; i >= 0; --i) {
         Layer &l = c->L[i];
@@ -1651,7 +1715,8 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
                 const double M = (double)nb * l.H * l.W;
                 ProfScope ps(c, K_GEMM_WGRAD, (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8,
                              2.0 * M * l.Cout * Kw, ws);
-                CK(sk::launch_narrow_wgrad(X, dcur, l.dw, nb, l.H, l.W, l.Cin, l.Cout, l.stride, ws, c->num_sms));
+                CK(sk::launch_narrow_wgrad(X, dcur, l.dws ? l.dws : l.dw, nb, l.H, l.W, l.Cin, l.Cout, l.stride, ws,
+                                           c->num_sms));
             }
             for (long long n0 = 0; n0 < nb && (nw_off || !sk::narrow_wgrad_supported(l.Cin, l.Cout, l.stride, l.H, l.W));
                  n0 += ch) {
@@ -1663,40 +1728,49 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
                                               ws));
                 }
                 const uint16_t *Dc = dcur + n0 * l.N;
-                ok = get_plan(c, {6, Dc, c->cols[par], l.dw, M, l.Cout, (int)Kw, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
-                    return sk::plan_fc_wgrad(p, Dc, c->cols[par], l.dw, M, l.Cout, (int)Kw, c->num_sms);
+                float *dwo = l.dws ? l.dws : l.dw;
+                ok = get_plan(c, {6, Dc, c->cols[par], dwo, M, l.Cout, (int)Kw, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
+                    return sk::plan_fc_wgrad(p, Dc, c->cols[par], dwo, M, l.Cout, (int)Kw, c->num_sms, l.wsl);
                 });
                 CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, (double)nbc * l.N * 2 + (double)M * Kw * 2 + (double)l.wcount * 8,
                              2.0 * M * l.Cout * Kw, ws));
             }
+            if (last_seg) CKS(reduce_wslices(c, i, ws));
             if (!c->prof_on) {
                 CK(cudaEventRecord(c->ev_done[par], c->st2));
                 c->w_pending[par] = true;
             }
             if (last_seg) CKS(comm_after_wgrad(c, i, ws));
-        } else if (i == 0 && c->in_kind == 1)
-            ok = get_plan(c, {2, dcur, X, l.dwp, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
+        } else if (i == 0 && c->in_kind == 1) {
+            float *dwo = l.dws ? l.dws : l.dwp;
+            ok = get_plan(c, {2, dcur, X, dwo, (long long)nb * l.H * l.W, l.Cout, c->K0, 0, 0, 0}, g,
                           [&](sk::GemmLaunch *p) {
-                              return sk::plan_fc_wgrad(p, dcur, X, l.dwp, nb * l.H * l.W, l.Cout, c->K0, c->num_sms);
+                              return sk::plan_fc_wgrad(p, dcur, X, dwo, nb * l.H * l.W, l.Cout, c->K0, c->num_sms,
+                                                       l.wsl);
                           });
-        else if (l.conv)
-            ok = get_plan(c, {3, dcur, X, l.dw, nb, l.Cin, l.Cout, l.H, l.W, 0}, g, [&](sk::GemmLaunch *p) {
-                return sk::plan_conv_wgrad(p, dcur, X, l.dw, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms);
+        } else if (l.conv) {
+            float *dwo = l.dws ? l.dws : l.dw;
+            ok = get_plan(c, {3, dcur, X, dwo, nb, l.Cin, l.Cout, l.H, l.W, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_conv_wgrad(p, dcur, X, dwo, nb, l.H, l.W, l.Cin, l.Cout, c->num_sms, l.wsl);
             });
-        else
-            ok = get_plan(c, {2, dcur, X, l.dw, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
-                return sk::plan_fc_wgrad(p, dcur, X, l.dw, nb, l.Cout, l.Cin, c->num_sms);
+        } else {
+            float *dwo = l.dws ? l.dws : l.dw;
+            ok = get_plan(c, {2, dcur, X, dwo, nb, l.Cout, l.Cin, 0, 0, 0}, g, [&](sk::GemmLaunch *p) {
+                return sk::plan_fc_wgrad(p, dcur, X, dwo, nb, l.Cout, l.Cin, c->num_sms, l.wsl);
             });
+        }
         const double wbytes = (double)nb * l.N * 2 + (double)nb * l.Nin * 2 + (double)l.wcount * 8;
         if (l.icol) {
             // issued above
         } else if (c->prof_on) {  // profiling: serialise so each kernel's events bracket only itself
             CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw));
+            if (last_seg) CKS(reduce_wslices(c, i, c->st));
             if (last_seg) CKS(comm_after_wgrad(c, i, c->st));
         } else {   // weight gradient on the side stream, after this layer's delta is written
             CK(cudaEventRecord(c->ev_ready[par], c->st));
             CK(cudaStreamWaitEvent(c->st2, c->ev_ready[par], 0));
             CKS(run_gemm(c, g, ok, "wgrad", i, K_GEMM_WGRAD, wbytes, 2.0 * Mw * l.Cout * Kw, c->st2));
+            if (last_seg) CKS(reduce_wslices(c, i, c->st2));
             CK(cudaEventRecord(c->ev_done[par], c->st2));
             c->w_pending[par] = true;
             if (last_seg) CKS(comm_after_wgrad(c, i, c->st2));
@@ -2300,10 +2374,22 @@ extern "C" int skipper_k_narrow_wgrad(const unsigned short *D, const unsigned sh
         g_last_error = "narrow_wgrad: unsupported shape";
         return SKIPPER_EUNSUPPORTED;
     }
-    if (!accumulate && cudaMemsetAsync(dW, 0, (size_t)cout * 9 * cin * 4, static_cast<cudaStream_t>(stream)) != cudaSuccess)
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const size_t cnt = (size_t)cout * 9 * cin;
+    if (!accumulate && cudaMemsetAsync(dW, 0, cnt * 4, st) != cudaSuccess) return SKIPPER_ECUDA;
+    // the kernel writes one dW slice per CTA; sum them in slice order (as the engine does)
+    const int ns = sk::narrow_wgrad_slices(cin, cout, stride, h, w, sk::device_num_sms());
+    float *sl = nullptr;
+    if (ns < 1 || cudaMallocAsync(reinterpret_cast<void **>(&sl), (size_t)ns * cnt * 4, st) != cudaSuccess ||
+        cudaMemsetAsync(sl, 0, (size_t)ns * cnt * 4, st) != cudaSuccess) {
+        g_last_error = "narrow_wgrad: slice allocation failed";
         return SKIPPER_ECUDA;
-    if (sk::launch_narrow_wgrad(reinterpret_cast<const uint16_t *>(X), reinterpret_cast<const uint16_t *>(D), dW, nb, h, w,
-                                cin, cout, stride, static_cast<cudaStream_t>(stream), sk::device_num_sms()) != cudaSuccess) {
+    }
+    const bool ok = sk::launch_narrow_wgrad(reinterpret_cast<const uint16_t *>(X), reinterpret_cast<const uint16_t *>(D), sl,
+                                            nb, h, w, cin, cout, stride, st, sk::device_num_sms()) == cudaSuccess &&
+                    sk::launch_reduce_slices(sl, ns, dW, cnt, st) == cudaSuccess;
+    cudaFreeAsync(sl, st);
+    if (!ok) {
         g_last_error = "narrow_wgrad: launch failed";
         return SKIPPER_ECUDA;
     }
@@ -2365,6 +2451,7 @@ extern "C" skipper_status skipper_profile(skipper_ctx *c, int enable) {
     CKS(check_ctx(c));
     prof_resolve(c);
     c->prof_on = enable != 0;
+    c->prof_log.clear();
     for (int k = 0; k < 16; ++k) {
         c->prof_n[k] = 0;
         c->prof_ms[k] = c->prof_bytes[k] = c->prof_flops[k] = 0;
@@ -2382,6 +2469,24 @@ extern "C" skipper_status skipper_profile_read(skipper_ctx *c, int cls, long lon
     if (bytes) *bytes = c->prof_bytes[cls];
     if (flops) *flops = c->prof_flops[cls];
     return SKIPPER_OK;
+}
+
+// The profiled scopes since skipper_profile() in launch order: class, kernels launched in the scope,
+// algorithmic bytes / FLOPs, device ms (CUDA events).  Fills up to cap entries; returns the total count.
+extern "C" long long skipper_profile_records(skipper_ctx *c, int *cls, long long *nk, double *bytes, double *flops,
+                                            float *ms, long long cap) {
+    if (!c) return -1;
+    prof_resolve(c);
+    const long long n = (long long)c->prof_log.size();
+    for (long long i = 0; i < n && i < cap; ++i) {
+        const auto &r = c->prof_log[i];
+        if (cls) cls[i] = r.cls;
+        if (nk) nk[i] = r.nk;
+        if (bytes) bytes[i] = r.bytes;
+        if (flops) flops[i] = r.flops;
+        if (ms) ms[i] = r.ms;
+    }
+    return n;
 }
 
 extern "C" const char *skipper_profile_class_name(int cls) {

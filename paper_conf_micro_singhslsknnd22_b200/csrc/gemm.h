@@ -20,10 +20,14 @@ enum OperandKind {
                     // MMA warp before the MMA reads them (4D boxes measured ~2x slower through TMA)
 };
 
-// OVERWRITE: plain store; ATOMIC_ADD: TMA reduce-add (split-K wgrad, accumulation over segments);
+// OVERWRITE: plain store; ATOMIC_ADD: TMA reduce-add (unsplit weight gradients accumulating over the
+// segments: one writer per element per launch, launches in stream order -> deterministic);
 // SPLIT: split s stores its partial sum into slice s of [splits][M][N] (summed in fixed order by the
-// consuming scan - deterministic split-K for the forward / dgrad GEMMs).
-enum StoreMode { STORE_OVERWRITE = 0, STORE_ATOMIC_ADD = 1, STORE_SPLIT = 2 };
+// consuming scan - deterministic split-K for the forward / dgrad GEMMs);
+// SLICE_ADD: split s reduce-adds into slice s of [slices][M][N] (split-K weight gradients: every slice has
+// one writer per launch and the launches are stream-ordered, so each slice accumulates the segments in a
+// fixed order; launch_reduce_slices sums the slices in slice order - deterministic split-K wgrad).
+enum StoreMode { STORE_OVERWRITE = 0, STORE_ATOMIC_ADD = 1, STORE_SPLIT = 2, STORE_SLICE_ADD = 3 };
 
 // Passed by value to the kernel.
 struct GemmDev {
@@ -68,8 +72,14 @@ bool make_map_conv(CUtensorMap *m, const void *ptr, uint64_t C, uint64_t W, uint
 // Plans (return false on unsupported geometry).  All pointers are device pointers.
 // C[M][N] = A[M][K] . B[N][K]^T
 bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N, int K, int splits = 1);
-// dW[N][K] (+)= D[M][N]^T . X[M][K]   (reduction over the M rows)
-bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms);
+// dW[N][K] (+)= D[M][N]^T . X[M][K]   (reduction over the M rows).  slices > 0: dW is the slice buffer
+// [slices][N][K] and split s reduce-adds into slice s (STORE_SLICE_ADD); needs fc_wgrad_splits(M) <= slices.
+bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms,
+                   int slices = 0);
+// split-K factor plan_fc_wgrad / plan_conv_wgrad choose for a reduction of M rows (monotone in M, so the
+// value at the largest M of a layer bounds every launch of that layer)
+int fc_wgrad_splits(long long M, int N, int K, int num_sms);
+int conv_wgrad_splits(long long M, int cin, int cout, int num_sms);
 // conv forward / dgrad: Y[nb,h,w,cout] from X[nb,h,w,cin] and Wk[cout][9][cin];
 // dgrad: G[nb,h,w,cin] from D[nb,h,w,cout] and Wt[cin][9][cout]
 bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
@@ -116,7 +126,7 @@ bool narrow_lif_mma_supported(int cin, int cout, int stride, int H, int W);
 cudaError_t launch_narrow_lif_mma(const NarrowConvArgs &a, cudaStream_t s, int num_sms);
 // conv wgrad: dW[cout][9][cin] (+)= sum D[.,cout] X_shift[.,cin]
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
-                     int num_sms);
+                     int num_sms, int slices = 0);
 
 cudaError_t gemm_run(const GemmLaunch &g, cudaStream_t stream, int num_sms);
 

@@ -401,6 +401,8 @@ __global__ void __launch_bounds__(kThreads<MN>, 1)
                     const int col0 = tc.n_t * BN + c * 32;
                     if (g.store_mode == STORE_ATOMIC_ADD)
                         tma_reduce_add_3d(&tcm, buf, col0, tc.tap, row0);
+                    else if (g.store_mode == STORE_SLICE_ADD)
+                        tma_reduce_add_3d(&tcm, buf, col0, tc.split, row0);
                     else
                         tma_store_3d(&tcm, buf, col0, g.store_mode == STORE_SPLIT ? tc.split : tc.tap, row0);
                     bulk_commit();
@@ -584,17 +586,53 @@ bool plan_fc(GemmLaunch *g, const void *A, const void *B, float *C, int M, int N
            make_map_out(&g->tc, C, N, d.splits, M, (uint64_t)M * N, N);
 }
 
-static void choose_splits(GemmDev &d, int base_tiles, int num_sms, int mult = 2) {
+// fit = true: at most mult * num_sms units (floor), so a one-unit-per-CTA launch has no second wave
+static void choose_splits(GemmDev &d, int base_tiles, int num_sms, int mult = 2, bool fit = false) {
     if (getenv("SKIPPER_SPLIT_MULT")) mult = atoi(getenv("SKIPPER_SPLIT_MULT"));  // experiments
     int target = mult * num_sms;
-    int splits = base_tiles >= target ? 1 : cdiv(target, base_tiles);
+    int splits = base_tiles >= target ? 1 : (fit ? target / base_tiles : cdiv(target, base_tiles));
     if (splits > d.num_kb) splits = d.num_kb;
     if (splits < 1) splits = 1;
     d.kb_per_split = cdiv(d.num_kb, splits);
     d.splits = cdiv(d.num_kb, d.kb_per_split);
 }
 
-bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms) {
+// split-K units per SM of the deterministic (slice) weight gradients: every split adds its whole output
+// tile into its own slice, so the slice bytes grow with the split count (SKIPPER_WG_SLICE_MULT, experiments)
+static int slice_mult(int dflt) {
+    static int m = -1;
+    if (m < 0) {
+        const char *e = getenv("SKIPPER_WG_SLICE_MULT");
+        m = e ? std::max(1, atoi(e)) : 0;
+    }
+    return m ? m : dflt;
+}
+
+// The bound on the split count before choose_splits rounds it to whole K blocks per split (the rounded
+// count is not monotone in M; this bound is, and every launch at a smaller M splits at most this often)
+static int splits_bound(long long M, int base_tiles, int num_sms, int mult) {
+    if (getenv("SKIPPER_SPLIT_MULT")) mult = atoi(getenv("SKIPPER_SPLIT_MULT"));
+    const int target = mult * num_sms;
+    int s = base_tiles >= target ? 1 : target / base_tiles;
+    return std::max(1, (int)std::min<long long>(s, cdiv(M, BK)));
+}
+
+int fc_wgrad_splits(long long M, int N, int K, int num_sms) {
+    return splits_bound(M, cdiv(N, BM) * cdiv(K, pick_bn(K)), num_sms, slice_mult(1));
+}
+
+static int conv_wgrad_bn(int cin) {
+    int bn = (9 * cin) % 256 && (9 * cin) % 192 == 0 ? 192 : 256;
+    if (getenv("SKIPPER_WG_BN")) bn = atoi(getenv("SKIPPER_WG_BN"));  // experiments
+    return bn;
+}
+
+int conv_wgrad_splits(long long M, int cin, int cout, int num_sms) {
+    return splits_bound(M, cdiv(cout, BM) * cdiv(9LL * cin, conv_wgrad_bn(cin)), num_sms, slice_mult(1));
+}
+
+bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M, int N, int K, int num_sms,
+                   int slices) {
     // GEMM rows = N (output neurons), GEMM cols = K (inputs), reduction over M rows.
     if (M <= 0 || N <= 0 || K <= 0 || N % 8 || K % 8) return false;
     GemmDev &d = g->d;
@@ -606,16 +644,17 @@ bool plan_fc_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int M
     d.n_tiles = cdiv(K, g->bn);
     d.taps = 1;
     d.num_kb = cdiv(M, BK);
-    choose_splits(d, d.m_tiles * d.n_tiles, num_sms);
+    choose_splits(d, d.m_tiles * d.n_tiles, num_sms, slices > 0 ? slice_mult(1) : 2, slices > 0);
+    if (slices > 0 && d.splits > slices) return false;
     d.a_kind = OP_MN2D;
     d.b_kind = OP_MN2D;
     d.C = dW;
     d.ldc = K;
     d.M = N;
     d.N = K;
-    d.store_mode = STORE_ATOMIC_ADD;
+    d.store_mode = slices > 0 ? STORE_SLICE_ADD : STORE_ATOMIC_ADD;
     return make_map_2d(&g->ta, D, N, M, 64, BK) && make_map_2d(&g->tb, X, K, M, 64, BK) &&
-           make_map_out(&g->tc, dW, K, 1, N, K, K);
+           make_map_out(&g->tc, dW, K, slices > 0 ? slices : 1, N, (uint64_t)N * K, K);
 }
 
 bool plan_conv(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb, int h, int w, int cin, int cout,
@@ -732,7 +771,7 @@ bool plan_conv_s(GemmLaunch *g, const void *X, const void *Wk, float *Y, int nb,
 }
 
 bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int nb, int h, int w, int cin, int cout,
-                     int num_sms) {
+                     int num_sms, int slices) {
     if (cin % 64 || cout % 8) return false;
     uint32_t bw, bh, bnn;
     if (!conv_box(h, w, BK, &bw, &bh, &bnn)) return false;
@@ -742,8 +781,7 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     // N = (tap, cin) = 9*cin columns in 256-wide tiles (192-wide when that tiles 9*cin exactly and 256
     // does not: cin = 64 -> 3 x 192 instead of 3 x 256 with a quarter-full last tile); each 64-column
     // chunk is one tap's shifted box
-    g->bn = (9 * cin) % 256 && (9 * cin) % 192 == 0 ? 192 : 256;
-    if (getenv("SKIPPER_WG_BN")) g->bn = atoi(getenv("SKIPPER_WG_BN"));  // experiments
+    g->bn = conv_wgrad_bn(cin);
     g->mn_major = 1;
     g->cs = 1;
     d.m_tiles = cdiv(cout, BM);
@@ -751,7 +789,9 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     d.taps = 1;
     d.wg_cin = cin;
     d.num_kb = cdiv(M, BK);
-    choose_splits(d, d.m_tiles * d.n_tiles, num_sms, 4);  // ~4 units per CTA: measured +5-15 % over 2
+    // ~4 units per CTA with reduce-add into one dW: measured +5-15 % over 2; slices: slice_mult
+    choose_splits(d, d.m_tiles * d.n_tiles, num_sms, slices > 0 ? slice_mult(1) : 4, slices > 0);
+    if (slices > 0 && d.splits > slices) return false;
     d.a_kind = OP_MN2D;
     static const bool box4d = getenv("SKIPPER_WG_4D") && atoi(getenv("SKIPPER_WG_4D"));  // experiments
     d.b_kind = box4d ? OP_MNCONV : OP_MNSHIFT;
@@ -763,11 +803,11 @@ bool plan_conv_wgrad(GemmLaunch *g, const void *D, const void *X, float *dW, int
     d.ldc = 9ll * cin;
     d.M = cout;
     d.N = 9 * cin;
-    d.store_mode = STORE_ATOMIC_ADD;
+    d.store_mode = slices > 0 ? STORE_SLICE_ADD : STORE_ATOMIC_ADD;
     const bool okb = box4d ? make_map_conv(&g->tb, X, cin, w, h, nb, bw, bh, bnn)
                            : make_map_2d(&g->tb, X, cin, (uint64_t)M, 64, BK);
     return make_map_2d(&g->ta, D, cout, M, 64, BK) && okb &&
-           make_map_out(&g->tc, dW, 9ull * cin, 1, cout, 9ull * cin, 9ull * cin);
+           make_map_out(&g->tc, dW, 9ull * cin, slices > 0 ? slices : 1, cout, 9ull * cin * cout, 9ull * cin);
 }
 
 template <int BN, int MN, int CS>

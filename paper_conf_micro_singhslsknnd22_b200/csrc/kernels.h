@@ -75,6 +75,11 @@ cudaError_t launch_stage_rows(const uint8_t *x, uint16_t *dst, const int *rows, 
 // dW[cout][9][cin] += sum over the nb*H*W output pixels of D[.][cout] X_shift[.][cin]; X is the layer
 // input [nb][H*stride][W*stride][cin], D [nb][H][W][cout], both bf16.
 bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W);
+// dW slices the narrow weight gradient writes: CTA b adds its partial into dW + b * |dW| (deterministic; sum
+// the slices with launch_reduce_slices)
+int narrow_wgrad_slices(int cin, int cout, int stride, int H, int W, int num_sms);
+// dst[i] += sum_{s < nslices} slices[s * count + i] in slice order, then slices[s * count + i] = 0
+cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s);
 cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
                                 int cout, int stride, cudaStream_t s, int num_sms);
 // dgrad of a narrow 3x3 conv, stride 1 or 2 (narrow_wgrad.cu): G [nb][s*H][s*W][cin] fp32 from the layer's

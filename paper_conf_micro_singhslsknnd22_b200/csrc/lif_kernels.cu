@@ -870,25 +870,33 @@ __global__ void readout_z_kernel(const uint16_t *__restrict__ WbL, const float *
     if (lane == 0) z[w] = acc * invT;
 }
 
-// softmax cross-entropy per sample (one warp per sample): loss += CE / B_global, dz
+// softmax cross-entropy, one block: warp w takes samples w, w + 8, ...; dz per sample, and loss += the
+// per-sample CE / B_global summed in sample order by one thread (deterministic, no float atomics)
 __global__ void readout_ce_kernel(const float *z, const int *labels, float *dz, float *loss, int B, int K, float invBg) {
     pdl_enter();
-    const int b = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    extern __shared__ float s_ce[];  // [B]
     const int lane = threadIdx.x & 31;
-    if (b >= B) return;
-    const float *zb = z + (long long)b * K;
-    float mx = -INFINITY;
-    for (int k = lane; k < K; k += 32) mx = fmaxf(mx, zb[k]);
-    for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-    float se = 0.f;
-    for (int k = lane; k < K; k += 32) se += expf(zb[k] - mx);
-    for (int o = 16; o; o >>= 1) se += __shfl_xor_sync(0xffffffffu, se, o);
-    const int y = labels[b];
-    for (int k = lane; k < K; k += 32) {
-        const float pr = expf(zb[k] - mx) / se;
-        dz[(long long)b * K + k] = (pr - (k == y ? 1.f : 0.f)) * invBg;
+    for (int b = threadIdx.x >> 5; b < B; b += blockDim.x >> 5) {
+        const float *zb = z + (long long)b * K;
+        float mx = -INFINITY;
+        for (int k = lane; k < K; k += 32) mx = fmaxf(mx, zb[k]);
+        for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        float se = 0.f;
+        for (int k = lane; k < K; k += 32) se += expf(zb[k] - mx);
+        for (int o = 16; o; o >>= 1) se += __shfl_xor_sync(0xffffffffu, se, o);
+        const int y = labels[b];
+        for (int k = lane; k < K; k += 32) {
+            const float pr = expf(zb[k] - mx) / se;
+            dz[(long long)b * K + k] = (pr - (k == y ? 1.f : 0.f)) * invBg;
+        }
+        if (lane == 0) s_ce[b] = (logf(se) + mx - zb[y]) * invBg;
     }
-    if (lane == 0) atomicAdd(loss, (logf(se) + mx - zb[y]) * invBg);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float acc = 0.f;
+        for (int b = 0; b < B; ++b) acc += s_ce[b];
+        *loss += acc;
+    }
 }
 
 // g_last[b][n] = (1/T) sum_k dz[b][k] W^L[k][n]: the gradient wrt the readout input, same at every t
@@ -909,7 +917,8 @@ cudaError_t launch_readout_loss(const uint16_t *WbL, const float *cnt, const int
                                 cudaStream_t s) {
     const long long warps = (long long)B * K;
     sk_launch(readout_z_kernel, (unsigned)((warps * 32 + 255) / 256), 256, 0, s, WbL, cnt, z, B, D, K, invT);
-    sk_launch(readout_ce_kernel, (B + 7) / 8, 256, 0, s, z, labels, dz, loss, B, K, invBg);
+    if ((size_t)B * 4 > 48 * 1024) return cudaErrorInvalidValue;
+    sk_launch(readout_ce_kernel, 1, 256, (size_t)B * 4, s, z, labels, dz, loss, B, K, invBg);
     const long long n = (long long)B * D;
     sk_launch(readout_g_kernel, (unsigned)((n + 255) / 256), 256, 0, s, WbL, dz, g_last, B, D, K, invT);
     return cudaGetLastError();
@@ -931,6 +940,37 @@ cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *
                                  cudaStream_t s, int accumulate) {
     const long long n = (long long)K * D;
     sk_launch(readout_wgrad_kernel, (unsigned)((n + 255) / 256), 256, 0, s, dz, cnt_kept, dWL, B, D, K, invT, accumulate);
+    return cudaGetLastError();
+}
+
+// ============================================================================ split-K weight-gradient slices
+// dst += sum of the nslices partial weight gradients in slice order (deterministic split-K, STORE_SLICE_ADD /
+// narrow_wgrad), and the slices are zeroed for the next step.  4 elements per thread.
+__global__ void reduce_slices_kernel(float4 *slices, int nslices, float4 *dst, long long count4) {
+    pdl_enter();
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count4;
+         i += (long long)gridDim.x * blockDim.x) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int s = 0; s < nslices; ++s) {
+            float4 *p = slices + (long long)s * count4 + i;
+            const float4 v = *p;
+            acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+            *p = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+        float4 d = dst[i];
+        d.x += acc.x; d.y += acc.y; d.z += acc.z; d.w += acc.w;
+        dst[i] = d;
+    }
+}
+
+cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s) {
+    if (count % 4 || (reinterpret_cast<uintptr_t>(slices) & 15) || (reinterpret_cast<uintptr_t>(dst) & 15))
+        return cudaErrorInvalidValue;
+    const long long c4 = (long long)(count / 4);
+    if (c4 == 0 || nslices <= 0) return cudaSuccess;
+    const int blocks = (int)std::min<long long>((c4 + 255) / 256, 148LL * 8);
+    sk_launch(reduce_slices_kernel, blocks, 256, 0, s, reinterpret_cast<float4 *>(slices), nslices,
+              reinterpret_cast<float4 *>(dst), c4);
     return cudaGetLastError();
 }
 

@@ -9,8 +9,9 @@
 // MMAs whose B operand rows are gathered by ldmatrix straight from the staged input (one row address
 // per output pixel and tap, so the shift / stride / zero padding costs nothing).  The work is
 // bandwidth-sized (K = pixels, M = cout, N = 9 cin), so the warp-level MMA is not the bound; the
-// accumulators stay in registers across all units of a persistent CTA and are reduced once at the end
-// (shared-memory atomics across warps, then one global fp32 atomic per weight per CTA).
+// accumulators stay in registers across all units of a persistent CTA and are reduced once at the end,
+// in a fixed order (warps in turn into shared memory, then the CTA's own dW slice; the slices are summed in
+// slice order by launch_reduce_slices), so the weight gradient is deterministic.
 #include "common.cuh"
 #include "kernels.h"
 
@@ -150,26 +151,34 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
         __syncthreads();  // buffer b is free for the unit after next
     }
     // D fragment: rows (co) mt*16 + lane/4 (+8), cols (ci within n tile) 2*(lane%4) (+1)
+    // Deterministic reduction: the WPC warps of a work item add their partials into sR in turn (wk order),
+    // then the CTA adds its sum into its own slice dW + blockIdx.x * |dW| - one writer per slice per launch,
+    // launches in stream order - and launch_reduce_slices sums the slices in slice order.
     const int co = mt * 16 + (lane >> 2), ci0 = 2 * (lane & 3);
+    float *dst = dW + (size_t)blockIdx.x * (COUT * 9 * CIN);
     if (Cfg::WPC > 1) {
         __syncthreads();
+        for (int turn = 0; turn < Cfg::WPC; ++turn) {
+            if (wk == turn) {
 #pragma unroll
-        for (int t = 0; t < Cfg::MAXT; ++t) {
-            const int tap = tap0 + t;
-            if (tap >= tap1) break;
+                for (int t = 0; t < Cfg::MAXT; ++t) {
+                    const int tap = tap0 + t;
+                    if (tap >= tap1) break;
 #pragma unroll
-            for (int j = 0; j < Cfg::NTT; ++j) {
-                const int ci = j * 8 + ci0;
-                atomicAdd(&sR[(co * 9 + tap) * CIN + ci], acc[t][j][0]);
-                atomicAdd(&sR[(co * 9 + tap) * CIN + ci + 1], acc[t][j][1]);
-                atomicAdd(&sR[((co + 8) * 9 + tap) * CIN + ci], acc[t][j][2]);
-                atomicAdd(&sR[((co + 8) * 9 + tap) * CIN + ci + 1], acc[t][j][3]);
+                    for (int j = 0; j < Cfg::NTT; ++j) {
+                        const int ci = j * 8 + ci0;
+                        sR[(co * 9 + tap) * CIN + ci] += acc[t][j][0];
+                        sR[(co * 9 + tap) * CIN + ci + 1] += acc[t][j][1];
+                        sR[((co + 8) * 9 + tap) * CIN + ci] += acc[t][j][2];
+                        sR[((co + 8) * 9 + tap) * CIN + ci + 1] += acc[t][j][3];
+                    }
+                }
             }
+            __syncthreads();
         }
-        __syncthreads();
         for (int i = threadIdx.x; i < COUT * 9 * CIN; i += NW_THREADS)
-            if (sR[i] != 0.f) atomicAdd(dW + i, sR[i]);
-    } else {
+            if (sR[i] != 0.f) dst[i] += sR[i];
+    } else {  // every element has one owner (warp, lane) in the CTA
 #pragma unroll
         for (int t = 0; t < Cfg::MAXT; ++t) {
             const int tap = tap0 + t;
@@ -177,10 +186,10 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
 #pragma unroll
             for (int j = 0; j < Cfg::NTT; ++j) {
                 const int ci = j * 8 + ci0;
-                atomicAdd(dW + (co * 9 + tap) * CIN + ci, acc[t][j][0]);
-                atomicAdd(dW + (co * 9 + tap) * CIN + ci + 1, acc[t][j][1]);
-                atomicAdd(dW + ((co + 8) * 9 + tap) * CIN + ci, acc[t][j][2]);
-                atomicAdd(dW + ((co + 8) * 9 + tap) * CIN + ci + 1, acc[t][j][3]);
+                dst[(co * 9 + tap) * CIN + ci] += acc[t][j][0];
+                dst[(co * 9 + tap) * CIN + ci + 1] += acc[t][j][1];
+                dst[((co + 8) * 9 + tap) * CIN + ci] += acc[t][j][2];
+                dst[((co + 8) * 9 + tap) * CIN + ci + 1] += acc[t][j][3];
             }
         }
     }
@@ -365,29 +374,67 @@ bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W) {
 }
 
 template <int CIN, int COUT, int S>
-static cudaError_t launch_nw(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, cudaStream_t s,
-                             int num_sms) {
+static size_t nw_smem(int H, int W) {
     using Cfg = NwCfg<CIN, COUT>;
     const int TH = std::min(H, NW_P / W);
     const int RX = S * (TH - 1) + 3;
-    const size_t smem = 2 * ((size_t)NW_P * COUT * 2 + (size_t)RX * W * S * CIN * 2) + CIN * 2 +
-                        (Cfg::WPC > 1 ? (size_t)COUT * 9 * CIN * 4 : 0);
+    return 2 * ((size_t)NW_P * COUT * 2 + (size_t)RX * W * S * CIN * 2) + CIN * 2 +
+           (Cfg::WPC > 1 ? (size_t)COUT * 9 * CIN * 4 : 0);
+}
+
+// the persistent grid's size = the number of dW slices (fixed per layer shape, independent of nb)
+template <int CIN, int COUT, int S>
+static int nw_grid_max(int H, int W, int num_sms) {
     auto kern = narrow_wgrad_kernel<CIN, COUT, S>;
     static bool attr = false;
     if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-        if (e != cudaSuccess) return e;
+        if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess)
+            return 0;
         attr = true;
     }
-    if (smem > 200 * 1024) return cudaErrorInvalidValue;
     int per_sm = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW_THREADS, smem) != cudaSuccess || per_sm < 1)
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NW_THREADS, nw_smem<CIN, COUT, S>(H, W)) !=
+            cudaSuccess || per_sm < 1)
         per_sm = 1;
+    return num_sms * per_sm;
+}
+
+template <int CIN, int COUT, int S>
+static cudaError_t launch_nw(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, cudaStream_t s,
+                             int num_sms) {
+    const int TH = std::min(H, NW_P / W);
+    const size_t smem = nw_smem<CIN, COUT, S>(H, W);
+    if (smem > 200 * 1024) return cudaErrorInvalidValue;
+    const int gmax = nw_grid_max<CIN, COUT, S>(H, W, num_sms);
+    if (gmax < 1) return cudaErrorInvalidValue;
     const long long units = (long long)nb * (H / TH);
     if (units == 0) return cudaSuccess;
-    const int grid = (int)std::min<long long>(units, (long long)num_sms * per_sm);
-    sk_launch(kern, grid, NW_THREADS, smem, s, X, D, dW, nb, H, W, TH);
+    const int grid = (int)std::min<long long>(units, (long long)gmax);
+    sk_launch(narrow_wgrad_kernel<CIN, COUT, S>, grid, NW_THREADS, smem, s, X, D, dW, nb, H, W, TH);
     return cudaGetLastError();
+}
+
+#define NW_CASES(X_)  \
+    X_(16, 16, 1);    \
+    X_(16, 32, 1);    \
+    X_(16, 64, 1);    \
+    X_(32, 16, 1);    \
+    X_(32, 32, 1);    \
+    X_(32, 64, 1);    \
+    X_(16, 16, 2);    \
+    X_(16, 32, 2);    \
+    X_(16, 64, 2);    \
+    X_(32, 16, 2);    \
+    X_(32, 32, 2);    \
+    X_(32, 64, 2)
+
+int narrow_wgrad_slices(int cin, int cout, int stride, int H, int W, int num_sms) {
+    if (!narrow_wgrad_supported(cin, cout, stride, H, W)) return 0;
+#define NWS_CASE(CI, CO, ST) \
+    if (cin == CI && cout == CO && stride == ST) return nw_grid_max<CI, CO, ST>(H, W, num_sms)
+    NW_CASES(NWS_CASE);
+#undef NWS_CASE
+    return 0;
 }
 
 cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
@@ -395,18 +442,7 @@ cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW,
     if (!narrow_wgrad_supported(cin, cout, stride, H, W)) return cudaErrorInvalidValue;
 #define NW_CASE(CI, CO, ST) \
     if (cin == CI && cout == CO && stride == ST) return launch_nw<CI, CO, ST>(X, D, dW, nb, H, W, s, num_sms)
-    NW_CASE(16, 16, 1);
-    NW_CASE(16, 32, 1);
-    NW_CASE(16, 64, 1);
-    NW_CASE(32, 16, 1);
-    NW_CASE(32, 32, 1);
-    NW_CASE(32, 64, 1);
-    NW_CASE(16, 16, 2);
-    NW_CASE(16, 32, 2);
-    NW_CASE(16, 64, 2);
-    NW_CASE(32, 16, 2);
-    NW_CASE(32, 32, 2);
-    NW_CASE(32, 64, 2);
+    NW_CASES(NW_CASE);
 #undef NW_CASE
     return cudaErrorInvalidValue;
 }

@@ -103,6 +103,7 @@ def _load():
         "skipper_profile_class_name": (ct.c_char_p, [I]),
         "skipper_profile_num_classes": (I, []),
         "skipper_launch_count": (ct.c_longlong, [P]),
+        "skipper_profile_records": (ct.c_longlong, [P, P, P, P, P, P, ct.c_longlong]),
         "skipper_plan_buckets": (I, [P, I, ct.c_ulonglong, P]),
         "skipper_encode_poisson": (I, [P, P, ct.c_ulonglong, I, I, ct.c_longlong, P, P]),
         "skipper_step_encoded": (I, [P, P, P, ct.c_ulonglong, P, P]),
@@ -376,6 +377,19 @@ class SkipperNet:
             out[lib.skipper_profile_class_name(k).decode()] = {
                 "launches": n.value, "ms": ms.value, "bytes": b.value, "flops": f.value}
         return out
+
+    def profile_records(self):
+        """Every profiled scope since profile() in launch order: [(class name, kernels, bytes, flops, ms)]."""
+        n = lib.skipper_profile_records(self.ctx, None, None, None, None, None, 0)
+        if n < 0:
+            raise SkipperError(-1, "profile_records on a null context")
+        cls = (ct.c_int * n)()
+        nk = (ct.c_longlong * n)()
+        by = (ct.c_double * n)()
+        fl = (ct.c_double * n)()
+        ms = (ct.c_float * n)()
+        lib.skipper_profile_records(self.ctx, cls, nk, by, fl, ms, n)
+        return [(lib.skipper_profile_class_name(cls[i]).decode(), nk[i], by[i], fl[i], ms[i]) for i in range(n)]
 
     def launch_count(self):
         return lib.skipper_launch_count(self.ctx)
