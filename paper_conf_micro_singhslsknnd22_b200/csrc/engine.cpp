@@ -1462,10 +1462,15 @@ static skipper_status readout_forward(skipper_ctx *c, const int *labels, float i
 }
 
 static skipper_status finish_first(skipper_ctx *c, const int *labels) {
-    ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
-    CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
+    {
+        ProfScope ps0(c, K_READOUT, (double)(c->Ls + 1) * c->T * 32 * 4, 0);
+        CK(sk::launch_sam_finalize(c->s_part, c->s_dev, (c->Ls + 1) * c->T, c->st));
+    }
     if (c->u2_part) {
-        CK(sk::launch_sum32_f64(c->u2_part, c->u2_dev, c->T, c->st));
+        {
+            ProfScope ps(c, K_READOUT, (double)c->T * 32 * 8 + (double)c->T * 8, 0);
+            CK(sk::launch_sum32_f64(c->u2_part, c->u2_dev, c->T, c->st));
+        }
         if (c->comm.comm) {
             std::string e;
             if (!c->comm.allreduce_f64(c->u2_dev, c->T, c->st, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());

@@ -1,7 +1,8 @@
 """ncu evidence for every kernel class of one training step.
 
   run:        python tools/ncu_classes.py run --workload cfg2_vgg5 --out gpurun_out/ncu_cfg2
-              (under `ncu --set full --profile-from-start off ... -o <rep>`: two warm-up steps, then
+              (under `ncu --metrics $(python tools/ncu_classes.py metrics) --profile-from-start off
+              --clock-control none -o <rep>`: two warm-up steps, then
               cudaProfilerStart, ONE profiled step whose every scope is logged by the engine
               (skipper_profile_records: class, kernels, algorithmic bytes / FLOPs), cudaProfilerStop)
   summarise:  python tools/ncu_classes.py summarise <rep.ncu-rep> <records.json> > profiles/r2_ncu_<cfg>.md
@@ -60,6 +61,7 @@ METRICS = {
     "sm": "sm__throughput.avg.pct_of_peak_sustained_elapsed",
     "dram_pct": "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
     "l1": "l1tex__throughput.avg.pct_of_peak_sustained_active",
+    "tma": "sm__pipe_tma_cycles_active.avg.pct_of_peak_sustained_active",
     "l2": "lts__throughput.avg.pct_of_peak_sustained_elapsed",
     "issue": "sm__inst_issued.avg.pct_of_peak_sustained_active",
 }
@@ -107,17 +109,17 @@ def summarise(a):
             c["kernels"][r["name"]] += 1
             c["t"] += r["t_us"]
             c["dram"] += r["dram_rd"] + r["dram_wr"]
-            tens = r["tc"] if r["tc"] == r["tc"] else r["tensor"]
+            tens = r["tensor"] if r["tensor"] == r["tensor"] else r["tc"]   # hmma subpipe counts UTCHMMA
             c["tensor_t"] += (tens if tens == tens else 0.0) * r["t_us"]
             c["occ_t"] += (r["occ"] if r["occ"] == r["occ"] else 0.0) * r["t_us"]
             units = {"DRAM": r["dram_pct"], "L1/TEX": r["l1"], "L2": r["l2"], "SM issue": r["issue"],
-                     "tensor": tens}
+                     "tensor": tens, "TMA": r["tma"]}
             units = {u: v for u, v in units.items() if v == v}
             if units:
                 top = max(units, key=units.get)
                 c["lim"][f"{top} {units[top]:.0f}%"] += r["t_us"]
         i += k
-    print(f"ncu --set full --clock-control none, one {meta['mode'].upper()} training step of {meta['workload']} "
+    print(f"ncu --clock-control none (the metrics of `tools/ncu_classes.py metrics`), one {meta['mode'].upper()} training step of {meta['workload']} "
           f"(tools/ncu_classes.py; kernels serialised and cold-cache under replay, so absolute times run long).  "
           f"`alg` = the engine's algorithmic bytes (DESIGN.md §7); `DRAM/alg` > 1.2 flags wasted traffic.  "
           f"HBM peak {peaks['hbm_gbs']:.0f} GB/s, sustained bf16 {peaks['bf16_tflops_sustained']:.0f} TF/s "
@@ -144,7 +146,7 @@ def summarise(a):
         if meta["workload"] == "cfg2_vgg5" and meta["mode"] == "skip":
             old.update(traffic)   # the bench's default workload: unprefixed keys, read by bench.py
         old["_note"] = ("dram__bytes_read.sum + dram__bytes_write.sum per launch of the class (mean over the "
-                        "class's launches in one ncu --set full capture of a training step, tools/ncu_classes.py)")
+                        "class's launches in one ncu metrics capture of a training step, tools/ncu_classes.py)")
         json.dump(old, open(tf, "w"), indent=1, sort_keys=True)
 
 
@@ -159,8 +161,12 @@ def main():
     s.add_argument("rep")
     s.add_argument("records")
     s.add_argument("--traffic", action="store_true")
+    sp.add_parser("metrics")
     a = ap.parse_args()
-    run(a) if a.cmd == "run" else summarise(a)
+    if a.cmd == "metrics":
+        print(",".join(METRICS.values()))
+    else:
+        run(a) if a.cmd == "run" else summarise(a)
 
 
 if __name__ == "__main__":
