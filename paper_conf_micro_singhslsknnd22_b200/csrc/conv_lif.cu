@@ -316,12 +316,16 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             const bool valid = uvalid && pg < BHW;
             const int ch0 = nt * BN + h * CW;
             const long long nidx = (long long)(valid ? pg : 0) * a.Cout + ch0;
+            // state / checkpoint element of channel c (multiple of 4): NHWC, or thread-major (a.state_tm:
+            // [unit][half][c/4][pixel of the tile][4], so a warp's float4 / uchar4 accesses are contiguous)
+            const long long tm0 = ((((long long)mt * a.n_tiles + nt) * 2 + h) * (CW / 4) * CL_BM + p) * 4;
+            auto sidx = [&](int c) -> long long { return a.state_tm ? tm0 + (long long)(c >> 2) * (CL_BM * 4) : nidx + c; };
             float U[CW];
             uint32_t ob[CW / 32];
-            if (valid) {
+            if (valid && !(a.diag & 32)) {  // diag 32: no state load / store (timing experiment)
 #pragma unroll
                 for (int c = 0; c < CW; c += 4) {
-                    const float4 v = *reinterpret_cast<const float4 *>(a.U_state + nidx + c);
+                    const float4 v = *reinterpret_cast<const float4 *>(a.U_state + sidx(c));
                     U[c] = v.x; U[c + 1] = v.y; U[c + 2] = v.z; U[c + 3] = v.w;
                 }
 #pragma unroll
@@ -329,7 +333,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     uint32_t w = 0;
 #pragma unroll
                     for (int c = 0; c < 32; c += 4) {
-                        const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nidx + 32 * j + c);
+                        const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + sidx(32 * j + c));
                         w |= (o4.x ? 1u : 0u) << c | (o4.y ? 1u : 0u) << (c + 1) | (o4.z ? 1u : 0u) << (c + 2) |
                              (o4.w ? 1u : 0u) << (c + 3);
                     }
@@ -341,12 +345,14 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
 #pragma unroll
                 for (int j = 0; j < CW / 32; ++j) ob[j] = 0u;
             }
-            auto store_state = [&](float *Ud, uint8_t *od) {
+            // state-layout stores (running state, checkpoint) when tm, else NHWC at nidx (debug record)
+            auto store_state = [&](float *Ud, uint8_t *od, bool tm) {
 #pragma unroll
                 for (int c = 0; c < CW; c += 4) {
-                    *reinterpret_cast<float4 *>(Ud + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    const long long e = tm ? sidx(c) : nidx + c;
+                    *reinterpret_cast<float4 *>(Ud + e) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
                     const uint32_t w = ob[c >> 5] >> (c & 31);
-                    *reinterpret_cast<uchar4 *>(od + c) = make_uchar4(w & 1u, (w >> 1) & 1u, (w >> 2) & 1u, (w >> 3) & 1u);
+                    *reinterpret_cast<uchar4 *>(od + e) = make_uchar4(w & 1u, (w >> 1) & 1u, (w >> 2) & 1u, (w >> 3) & 1u);
                 }
             };
             auto emit = [&](int r) {
@@ -369,7 +375,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         for (int c = 0; c < CW; c += 4)
                             *reinterpret_cast<float4 *>(dst + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
                     }
-                    if (a.dbg_U) store_state(a.dbg_U + t * rs + nidx, a.dbg_o + t * rs + nidx);
+                    if (a.dbg_U) store_state(a.dbg_U + t * rs, a.dbg_o + t * rs, false);
                     if (!POOL) {
                         uint16_t *dst = a.Po_out + (long long)r * rs + nidx;
 #pragma unroll
@@ -463,9 +469,9 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 CL_T0;
                 if (!(a.diag & 1)) emit(r);
                 CL_T1(3);
-                if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
+                if (a.ckU && r == 0 && valid) store_state(a.ckU, a.cko, true);
             }
-            if (!a.restore && valid) store_state(a.U_state + nidx, a.o_state + nidx);
+            if (!a.restore && valid && !(a.diag & 32)) store_state(a.U_state, a.o_state, true);
         }
     }
     tc_fence_before();
@@ -485,6 +491,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             if (v) atomicAdd(a.s_part + row_time(r) * 32 + (blockIdx.x & 31), v);
         }
     }
+}
+
+long long conv_lif_state_count(int B, int H, int W, int cout) {
+    return ((long long)B * H * W + CL_BM - 1) / CL_BM * CL_BM * cout;
 }
 
 bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {

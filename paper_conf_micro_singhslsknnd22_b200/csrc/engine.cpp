@@ -12,6 +12,7 @@
 #include "kernels.h"
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -50,6 +51,8 @@ struct Layer {
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
     int fsplitT = 1;             // forward split-K of the chunked first pass (fc tail layers, tail_G*S rows)
     bool cfused = false;         // conv layer: GEMM + LIF scan as one kernel (conv_lif.cu)
+    size_t sbn = 0;              // elements of one running-state / checkpoint slot (B*N, or conv_lif's
+                                 // thread-major layout, conv_lif_state_count, when cfused)
     // deterministic split-K weight gradient: wsl > 0 -> the wgrad launches add into slice s of dws
     // [wsl][wg_count] (one writer per slice per launch), summed in slice order into dW (or dwp) after the
     // layer's last weight-gradient launch of the step (launch_reduce_slices)
@@ -184,7 +187,16 @@ struct skipper_ctx {
     long long prof_n[16] = {0};
     double prof_ms[16] = {0}, prof_bytes[16] = {0}, prof_flops[16] = {0};
     long long launches = 0;
+    // host-side phase timing (SKIPPER_HOST_PROFILE=1, printed at destroy): issue of the first pass, the
+    // mask sync wait, issue of recompute + backward + optimizer
+    bool host_prof = false;
+    double hp_first = 0, hp_sync = 0, hp_bwd = 0;
+    long long hp_steps = 0;
 };
+
+static double now_ms() {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
@@ -609,6 +621,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     c->S = c->T / c->C;
     c->num_sms = sk::device_num_sms();
+    c->host_prof = getenv("SKIPPER_HOST_PROFILE") && atoi(getenv("SKIPPER_HOST_PROFILE"));
     if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess)
         return bail(fail(c, SKIPPER_ECUDA, "side stream creation failed"));
     for (int i = 0; i < c->Ls; ++i)
@@ -693,12 +706,15 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
                 AL(l.dwp, (size_t)l.Cout * c->K0);
             }
             const size_t bn = (size_t)c->B * l.N;
-            AL(l.U_run, bn);
-            AL(l.o_run, bn);
+            l.sbn = l.cfused ? (size_t)sk::conv_lif_state_count(c->B, l.H, l.W, l.Cout)
+                    : (i == 0 && c->l0_fused) ? (size_t)sk::layer0_state_count(c->B, l.H, l.W, l.Cout, l.pool ? 1 : 0)
+                                              : bn;
+            AL(l.U_run, l.sbn);
+            AL(l.o_run, l.sbn);
             AL(l.carry, bn);
             if (cfg->mode != SKIPPER_MODE_FULL && cfg->mode != SKIPPER_MODE_TBPTT) {
-                AL(l.ckU, bn * c->C);
-                AL(l.cko, bn * c->C);
+                AL(l.ckU, l.sbn * c->C);
+                AL(l.cko, l.sbn * c->C);
             }
             if (cfg->debug_record) {
                 for (int k = 0; k < 2; ++k) {
@@ -789,6 +805,10 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
 
 extern "C" void skipper_destroy(skipper_ctx *c) {
     if (!c) return;
+    if (c->host_prof && c->hp_steps)
+        fprintf(stderr, "skipper host profile: %lld steps, per step: first-pass issue %.3f ms, mask sync wait %.3f ms, "
+                        "recompute+backward issue %.3f ms\n", c->hp_steps, c->hp_first / c->hp_steps,
+                c->hp_sync / c->hp_steps, c->hp_bwd / c->hp_steps);
     if (c->st) cudaStreamSynchronize(c->st);
     if (c->arena) dev_free(c, c->arena, c->arena_bytes);
     for (auto &l : c->L) {
@@ -801,12 +821,12 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         dev_free(c, l.dwp, (size_t)l.Cout * c->K0 * 4);
         if (!l.readout) {
             const size_t bn = (size_t)c->B * l.N;
-            dev_free(c, l.U_run, bn * 4);
-            dev_free(c, l.o_run, bn);
+            dev_free(c, l.U_run, l.sbn * 4);
+            dev_free(c, l.o_run, l.sbn);
             dev_free(c, l.carry, bn * 4);
             dev_free(c, l.dws, (size_t)l.wsl * l.wg_count * 4);
-            dev_free(c, l.ckU, bn * c->C * 4);
-            dev_free(c, l.cko, bn * c->C);
+            dev_free(c, l.ckU, l.sbn * c->C * 4);
+            dev_free(c, l.cko, l.sbn * c->C);
             for (int k = 0; k < 2; ++k) {
                 dev_free(c, l.dbg[k], bn * c->T * 4);
                 dev_free(c, l.dbgo[k], bn * c->T);
@@ -1131,8 +1151,8 @@ static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
         const size_t bn = (size_t)c->B * l.N;
-        CKS(zero_dev(c, l.U_run, bn * 4));
-        CKS(zero_dev(c, l.o_run, bn));
+        CKS(zero_dev(c, l.U_run, l.sbn * 4));
+        CKS(zero_dev(c, l.o_run, l.sbn));
         CKS(zero_dev(c, l.carry, bn * 4));
         if (c->cfg.debug_record)
             for (int k = 0; k < 2; ++k) {
@@ -1258,12 +1278,13 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     a.pool = l.pool ? 1 : 0;
     a.lam = l.d.lambda;
     a.theta = l.d.theta;
-    a.U_state = restore ? l.ckU + (size_t)seg * bn : l.U_run;
-    a.o_state = restore ? l.cko + (size_t)seg * bn : l.o_run;
+    a.state_tm = 1;  // running state and checkpoints in the kernel's coalesced thread-major layout
+    a.U_state = restore ? l.ckU + (size_t)seg * l.sbn : l.U_run;
+    a.o_state = restore ? l.cko + (size_t)seg * l.sbn : l.o_run;
     a.U_out = (restore || record) ? l.Useg : nullptr;
     a.Po_out = out;
-    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
-    a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * l.sbn : nullptr;
+    a.cko = (!restore && !record) ? l.cko + (size_t)seg * l.sbn : nullptr;
     a.s_part = restore ? nullptr : spart(c, 1);
     a.s_part_in = restore ? nullptr : spart(c, 0);
     a.u2_part = restore ? nullptr : c->u2_part;
@@ -1295,12 +1316,13 @@ static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16
     a.restore = restore ? 1 : 0;
     a.t0 = t0;
     a.row_t = row_t;
-    a.U_state = restore ? l.ckU + (size_t)seg * bn : l.U_run;
-    a.o_state = restore ? l.cko + (size_t)seg * bn : l.o_run;
+    a.state_tm = 1;  // running state and checkpoints in the kernel's coalesced thread-major layout
+    a.U_state = restore ? l.ckU + (size_t)seg * l.sbn : l.U_run;
+    a.o_state = restore ? l.cko + (size_t)seg * l.sbn : l.o_run;
     a.U_out = (restore || record) ? l.Useg : nullptr;
     a.Po_out = out;
-    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
-    a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * l.sbn : nullptr;
+    a.cko = (!restore && !record) ? l.cko + (size_t)seg * l.sbn : nullptr;
     a.s_part = restore ? nullptr : spart(c, i + 1);
     a.u2_part = restore ? nullptr : c->u2_part;
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
@@ -1482,7 +1504,9 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     CKS(comm_allreduce_s(c));
     CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
                        c->st));
+    const double hs0 = c->host_prof ? now_ms() : 0.0;
     CK(cudaStreamSynchronize(c->st));  // the one host sync of the step
+    if (c->host_prof) c->hp_sync += now_ms() - hs0;
     // SAM (Eq.4) and the policy metric: Eq.4 totals, or the neuron-count-weighted sum (reading 22)
     for (int t = 0; t < c->T; ++t) {
         long long tot = 0;
@@ -2087,11 +2111,19 @@ extern "C" skipper_status skipper_step(skipper_ctx *c, const unsigned char *x_de
         }
     } else {
         c->phase = PH_IDLE;
+        const double h0 = c->host_prof ? now_ms() : 0.0;
+        const double s0 = c->hp_sync;
         for (int seg = 0; seg < c->C; ++seg)
             CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_FIRST, x_dev, seg == c->C - 1 ? labels_dev : nullptr));
+        const double h1 = c->host_prof ? now_ms() : 0.0;
         for (int seg = c->C - 1; seg >= 0; --seg) {
             CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_RECOMPUTE, x_dev, nullptr));
             CKS(skipper_backward_segment(c, seg));
+        }
+        if (c->host_prof) {
+            c->hp_first += (h1 - h0) - (c->hp_sync - s0);
+            c->hp_bwd += now_ms() - h1;
+            c->hp_steps++;
         }
     }
     CKS(skipper_optimizer_step(c));

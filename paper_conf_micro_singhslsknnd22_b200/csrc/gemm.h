@@ -148,6 +148,10 @@ struct ConvLifArgs {
     float *dbg_U;
     uint8_t *dbg_o;
     float lam, theta;
+    // 1: U_state / o_state / ckU / cko in the kernel's thread-major layout (conv_lif_state_count elements:
+    // [unit][channel half][channel / 4][pixel of the 128-pixel tile][4]) - coalesced state loads / stores;
+    // 0: NHWC [B][H][W][Cout] (the kernel-level test API)
+    int state_tm;
     // filled by launch_conv_lif
     int m_tiles, n_tiles, num_kb, conv_cb;
     int stages;      // smem ring depth
@@ -155,6 +159,8 @@ struct ConvLifArgs {
     int diag;  // SKIPPER_CL_DIAG timing experiments: 1 = no epilogue work, 2 = no MMA
 };
 bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool);
+// elements of one state / checkpoint slot in the thread-major layout (>= B*H*W*Cout: whole 128-pixel tiles)
+long long conv_lif_state_count(int B, int H, int W, int cout);
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms);
 
 int device_num_sms();

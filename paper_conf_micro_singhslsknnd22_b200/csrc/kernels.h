@@ -127,8 +127,11 @@ struct L0FwdArgs {
     float *dbg_U;
     uint8_t *dbg_o;
     uint16_t *xg_out;      // or null: also write the bf16 im2col rows [R][B*H*W][32] (weight-gradient operand)
+    int state_tm;          // 1: U_state / o_state / ckU / cko in the kernel's thread-major layout
+                           // (layer0_state_count elements: [tile][channel chunk][c/4][tile row][4]), 0: NHWC
 };
 bool layer0_supported(int B, int H, int W, int C0, int N, int pool);
+long long layer0_state_count(int B, int H, int W, int N, int pool);
 
 // Fused layer-0 backward (layer0.cu): Eq.2 reverse scan + weight gradient on the tensor cores.
 struct L0BwdArgs {

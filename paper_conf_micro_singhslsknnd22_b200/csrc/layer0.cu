@@ -399,14 +399,18 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             const long long pix = ((long long)(valid ? b : 0) * a.H + yy) * a.W + xx;
             const long long opix = a.pool ? ((long long)(valid ? b : 0) * PH + (yy >> 1)) * PW + (xx >> 1) : pix;
             const long long nbase = pix * N + c0;
+            // state / checkpoint element of channel c (multiple of 4): NHWC, or thread-major (a.state_tm:
+            // [tile][channel chunk][c/4][tile row][4]; a warp's float4 / uchar4 accesses are contiguous)
+            const long long tm0 = (((long long)tile * (N / CW) + h) * (CW / 4) * 128 + row) * 4;
+            auto sidx = [&](int c) -> long long { return a.state_tm ? tm0 + (long long)(c >> 2) * 512 : nbase + c; };
             float U[CW];
             uint32_t ob = 0;
             if (valid) {
 #pragma unroll
                 for (int c = 0; c < CW; c += 4) {
-                    const float4 u = *reinterpret_cast<const float4 *>(a.U_state + nbase + c);
+                    const float4 u = *reinterpret_cast<const float4 *>(a.U_state + sidx(c));
                     U[c] = u.x; U[c + 1] = u.y; U[c + 2] = u.z; U[c + 3] = u.w;
-                    const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + nbase + c);
+                    const uchar4 o4 = *reinterpret_cast<const uchar4 *>(a.o_state + sidx(c));
                     ob |= (o4.x ? 1u : 0u) << c | (o4.y ? 1u : 0u) << (c + 1) | (o4.z ? 1u : 0u) << (c + 2) |
                           (o4.w ? 1u : 0u) << (c + 3);
                 }
@@ -414,11 +418,13 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
 #pragma unroll
                 for (int c = 0; c < CW; ++c) U[c] = 0.f;
             }
-            auto store_state = [&](float *Ud, uint8_t *od) {
+            // tm: the state layout (running state, checkpoint), else NHWC at nbase (debug record)
+            auto store_state = [&](float *Ud, uint8_t *od, bool tm) {
 #pragma unroll
                 for (int c = 0; c < CW; c += 4) {
-                    *reinterpret_cast<float4 *>(Ud + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
-                    *reinterpret_cast<uchar4 *>(od + c) =
+                    const long long e = tm ? sidx(c) : nbase + c;
+                    *reinterpret_cast<float4 *>(Ud + e) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                    *reinterpret_cast<uchar4 *>(od + e) =
                         make_uchar4((ob >> c) & 1u, (ob >> (c + 1)) & 1u, (ob >> (c + 2)) & 1u, (ob >> (c + 3)) & 1u);
                 }
             };
@@ -485,7 +491,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                             *reinterpret_cast<float4 *>(a.U_out + (long long)ri * rs + nbase + c) =
                                 make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
                     }
-                    if (a.dbg_U) store_state(a.dbg_U + t * rs + nbase, a.dbg_o + t * rs + nbase);
+                    if (a.dbg_U) store_state(a.dbg_U + t * rs, a.dbg_o + t * rs, false);
                 }
                 if (a.s_part) {
                     const unsigned v = __reduce_add_sync(0xffffffffu, cnt);
@@ -520,11 +526,11 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 }
                 ob = nb; L0_T1(7); L0_T0;
                 emit(ri); L0_T1(3); L0_T0;
-                if (a.ckU && ri == 0 && valid) store_state(a.ckU + nbase, a.cko + nbase);
+                if (a.ckU && ri == 0 && valid) store_state(a.ckU, a.cko, true);
                 L0_T1(2);
             }
             L0_T0;
-            if (!a.restore && valid) store_state(a.U_state + nbase, a.o_state + nbase);
+            if (!a.restore && valid) store_state(a.U_state, a.o_state, true);
             L0_T1(4);
         }
     }
@@ -566,6 +572,12 @@ static bool l0_tiling(int B, int H, int W, int pool, L0Tile *g) {
 bool layer0_supported(int B, int H, int W, int C0, int N, int pool) {
     L0Tile g;
     return 9 * C0 <= 32 && (N == 32 || N == 64) && (W * C0) % 8 == 0 && l0_tiling(B, H, W, pool, &g);
+}
+
+long long layer0_state_count(int B, int H, int W, int N, int pool) {
+    L0Tile g;
+    if (!l0_tiling(B, H, W, pool, &g)) return (long long)B * H * W * N;
+    return (long long)g.tiles_b * g.tiles_y * g.tiles_x * 128 * N;
 }
 
 cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {

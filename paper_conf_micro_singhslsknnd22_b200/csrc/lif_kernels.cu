@@ -15,13 +15,15 @@ SK_DEV float lif_update(float U, float I, float o, float lam, float th) {
     return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
 }
 
-SK_DEV float surrogate(float U, float th, int kind, float gamma) {
+// sigma'(U) of reading 4; inv_th = 1 / theta computed once per thread (the reverse scan is issue-bound:
+// a multiply instead of an IEEE division per neuron-step; within 1 ulp of |U - theta| / theta)
+SK_DEV float surrogate(float U, float th, float inv_th, int kind, float gamma) {
     if (kind == SURR_TRIANGLE) {
-        const float v = 1.0f - fabsf(U - th) / th;
+        const float v = 1.0f - fabsf(U - th) * inv_th;
         return v > 0.0f ? gamma * v : 0.0f;
     }
     const float d = 1.0f + gamma * fabsf(U - th);
-    return 1.0f / (d * d);
+    return __frcp_rn(d * d);
 }
 
 SK_DEV uint2 pack_bf16x4(float a, float b, float c, float d) {
@@ -424,6 +426,7 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanB
             rd_off = ((b * Hr + y / s) * Wr + x / s) * a.res_C + c + a.res_lo;
     }
     float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
+    const float inv_th = 1.0f / a.theta;
     // two chunks of CH rows in flight: loads of the next (earlier) chunk overlap the recurrence
     auto load = [&](float4 (&gv)[CH], float4 (&uv)[CH], int rb) {
 #pragma unroll
@@ -448,10 +451,10 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanB
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
             if (r >= 0) {
-                d.x = surrogate(uv[j].x, a.theta, a.surr, a.gamma) * (gs * gv[j].x) + a.lam * d.x;
-                d.y = surrogate(uv[j].y, a.theta, a.surr, a.gamma) * (gs * gv[j].y) + a.lam * d.y;
-                d.z = surrogate(uv[j].z, a.theta, a.surr, a.gamma) * (gs * gv[j].z) + a.lam * d.z;
-                d.w = surrogate(uv[j].w, a.theta, a.surr, a.gamma) * (gs * gv[j].w) + a.lam * d.w;
+                d.x = surrogate(uv[j].x, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].x) + a.lam * d.x;
+                d.y = surrogate(uv[j].y, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].y) + a.lam * d.y;
+                d.z = surrogate(uv[j].z, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].z) + a.lam * d.z;
+                d.w = surrogate(uv[j].w, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].w) + a.lam * d.w;
                 if (a.delta)
                     *reinterpret_cast<uint2 *>(a.delta + (long long)r * rs + n0) = pack_bf16x4(d.x, d.y, d.z, d.w);
             }
@@ -479,6 +482,7 @@ __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a)
     const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (n >= rs) return;
     const long long grs = a.g_broadcast ? 0 : rs;
+    const float inv_th = 1.0f / a.theta;
     float d = a.carry[n];
     for (int rb = a.R - 1; rb >= 0; rb -= CH) {
         float gv[CH], uv[CH];
@@ -496,7 +500,7 @@ __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a)
         for (int j = 0; j < CH; ++j) {
             const int r = rb - j;
             if (r >= 0) {
-                d = surrogate(uv[j], a.theta, a.surr, a.gamma) * gv[j] + a.lam * d;
+                d = surrogate(uv[j], a.theta, inv_th, a.surr, a.gamma) * gv[j] + a.lam * d;
                 if (a.delta) a.delta[(long long)r * rs + n] = f2bf_bits(d);
             }
         }

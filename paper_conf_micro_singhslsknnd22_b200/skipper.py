@@ -183,6 +183,8 @@ class TorchAllocator:
                 return None
 
         def _free(ptr, nbytes, stream, user):
+            if torch is None or getattr(torch, "cuda", None) is None:  # interpreter teardown: memory goes with it
+                return
             torch.cuda.caching_allocator_delete(ptr)
 
         self._a = ALLOC_FN(_alloc)
