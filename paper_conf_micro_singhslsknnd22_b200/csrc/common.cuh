@@ -21,6 +21,20 @@ namespace sk {
 // attribute the wait is a no-op.
 SK_DEV void pdl_enter() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
+// 256-bit global store (sm_100: STG.E.256): one full 32-byte sector per lane, so a thread-per-pixel
+// epilogue writing a pixel's channels emits whole sectors instead of half-sector 16-byte pieces.
+// p must be 32-byte aligned.
+SK_DEV void st_global_v8u(void *p, uint4 a, uint4 b) {
+    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "r"(a.x), "r"(a.y), "r"(a.z),
+                 "r"(a.w), "r"(b.x), "r"(b.y), "r"(b.z), "r"(b.w)
+                 : "memory");
+}
+SK_DEV void st_global_v8(float *p, const float *v) {
+    asm volatile("st.global.v8.f32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "f"(v[0]), "f"(v[1]), "f"(v[2]),
+                 "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7])
+                 : "memory");
+}
+
 bool pdl_enabled();  // SKIPPER_NO_PDL=1 turns the launch attribute off (engine.cpp)
 
 template <typename... KArgs, typename... Args>

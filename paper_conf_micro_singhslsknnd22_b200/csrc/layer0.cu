@@ -247,13 +247,15 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
         // next tile when the row is stored
         auto store_xg = [&](int rr, uint32_t m, int b, int yy, int xx) {
             if (b >= a.B) return;
-            uint4 *dst = reinterpret_cast<uint4 *>(a.xg_out + (((long long)rr * a.B + b) * a.H * a.W +
-                                                               (long long)yy * a.W + xx) * 32);
+            uint16_t *dst = a.xg_out + (((long long)rr * a.B + b) * a.H * a.W + (long long)yy * a.W + xx) * 32;
+            uint4 q[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
                 const uint2 lo = s_lut[(m >> (8 * j)) & 15u], hi = s_lut[(m >> (8 * j + 4)) & 15u];
-                dst[j] = make_uint4(lo.x, lo.y, hi.x, hi.y);
+                q[j] = make_uint4(lo.x, lo.y, hi.x, hi.y);
             }
+            st_global_v8u(dst, q[0], q[1]);  // two whole 32-byte sectors
+            st_global_v8u(dst + 16, q[2], q[3]);
         };
         // RECOMPUTE: row 0 (the checkpoint) has no MMA but its im2col row is part of the operand
         auto xg_row0 = [&]() {
@@ -487,9 +489,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 if (valid) {
                     if (a.U_out) {
 #pragma unroll
-                        for (int c = 0; c < CW; c += 4)
-                            *reinterpret_cast<float4 *>(a.U_out + (long long)ri * rs + nbase + c) =
-                                make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                        for (int c = 0; c < CW; c += 8) st_global_v8(a.U_out + (long long)ri * rs + nbase + c, U + c);
                     }
                     if (a.dbg_U) store_state(a.dbg_U + t * rs, a.dbg_o + t * rs, false);
                 }
