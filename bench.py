@@ -209,7 +209,7 @@ def run_mode(torch, dist, args, wl, net, mode, rank, world, local_rank, profile=
     T, B, C, p = wl["T"], wl["B"], wl["C"], wl["p"]
     x, y = cached_inputs(net, T, B, seed=1 + 1000 * rank)
     W = synth.make_weights(net)
-    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, global_batch=B * world)
+    m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, global_batch=B * world, group=args.group)
     m.set_weights(W)
     if world > 1:
         obj = [m.comm_unique_id() if rank == 0 else None]
@@ -373,6 +373,90 @@ def roofline(prof, peaks, steps):
     return rf, breakdown, roof_ms
 
 
+def sqrt_divisor(T, L_n):
+    """C for the C ~ sqrt(T) leg of cfg 5: the divisor of T nearest sqrt(T) whose segment length T/C exceeds
+    the layer count - Eq.3's minimum of C + T/C."""
+    cands = [C for C in range(1, T + 1) if T % C == 0 and T // C > L_n]
+    return min(cands, key=lambda C: (abs(C - T ** 0.5), C))
+
+
+def sweep_sqrt_c(torch, dist, args, rank, world, local_rank):
+    """cfg 5, C ~ sqrt(T) leg: peak HBM and throughput of CKPT and SKIP with C chosen per T as above; the stored
+    state is O(C + T/C) = O(sqrt(T)) (Eq.3 / Eq.6), so peak HBM should grow like sqrt(T), not T."""
+    w5 = synth.workload("cfg3_vgg11")
+    net5 = synth.net_config(w5["net"])
+    L_n = len(net5["layers"])
+    out = {}
+    for T in [int(v) for v in args.t_sweep_vgg11.split(",") if v]:
+        C = sqrt_divisor(T, L_n)
+        w2 = dict(w5, T=T, C=C)
+        row = {"C": C}
+        for mode in ("skip", "ckpt"):
+            try:
+                r = run_mode(torch, dist, args, w2, net5, mode, rank, world, local_rank, steps=3, warmup=3)
+                row[mode] = {"samples_per_s": w2["B"] * world * 3 / (r["total_ms"] / 1e3),
+                             "peak_hbm_gb": r["peak_lib"] / 1e9}
+            except Exception as e:  # noqa: BLE001
+                row[mode] = {"error": str(e)[:120]}
+        out[str(T)] = row
+    Ts = sorted(int(t) for t in out)
+    for mode in ("skip", "ckpt"):
+        try:   # growth exponent of the peak between the smallest and largest T (1 = linear, 0.5 = sqrt)
+            a, b = out[str(Ts[0])][mode]["peak_hbm_gb"], out[str(Ts[-1])][mode]["peak_hbm_gb"]
+            out[f"{mode}_growth_exponent"] = float(np.log(b / a) / np.log(Ts[-1] / Ts[0]))
+        except Exception:  # noqa: BLE001
+            pass
+    return out
+
+
+def max_t_search(torch, dist, args, rank, world, local_rank, sweep11):
+    """cfg 5 / Fig. 14: the largest T (multiple of 100) each mode trains at C = 5, p = 50 within a
+    memory budget - the A100's 80 GB and this device's whole HBM.  Peak HBM at fixed C is affine in T, so T_max is
+    predicted from the two largest T of the C = 5 sweep and then CHECKED by one training step at the predicted T
+    (stepping down by 100 while the step's measured peak exceeds the budget or it does not fit)."""
+    w5 = synth.workload("cfg3_vgg11")
+    net5 = synth.net_config(w5["net"])
+    total = torch.cuda.mem_get_info()[1]
+    budgets = {"80GB": 80e9, "device_hbm": float(total)}
+    out = {"budgets_gb": {k: v / 1e9 for k, v in budgets.items()}, "C": 5, "p": w5["p"],
+           "peak": "library allocator high-water mark (the stored-state + workspace bytes of the step)"}
+    for bname, budget in budgets.items():
+        res = {}
+        for mode in ("full", "ckpt", "skip"):
+            pts = sorted((int(T), row[mode]["peak_hbm_gb"] * 1e9) for T, row in sweep11.items()
+                         if "peak_hbm_gb" in row.get(mode, {}))
+            if len(pts) < 2:
+                res[mode] = {"error": "fewer than two sweep points"}
+                continue
+            (t1, p1), (t2, p2) = pts[-2], pts[-1]
+            slope = (p2 - p1) / (t2 - t1)
+            Tm = int((t2 + (budget - p2) / slope) // 100 * 100)
+            entry = {"predicted_T_max": Tm}
+            for _ in range(4):
+                if Tm < 100:
+                    break
+                try:
+                    r = run_mode(torch, dist, args, dict(w5, T=Tm, C=5), net5, mode, rank, world, local_rank, steps=1,
+                                 warmup=1)
+                    if r["peak_lib"] <= budget:
+                        entry.update({"T_max": Tm, "peak_hbm_gb": r["peak_lib"] / 1e9,
+                                      "samples_per_s": w5["B"] * world / (r["total_ms"] / 1e3)})
+                        break
+                    entry.setdefault("over_budget", []).append([Tm, r["peak_lib"] / 1e9])
+                except Exception as e:  # noqa: BLE001
+                    entry.setdefault("failed", []).append([Tm, str(e)[:80]])
+                Tm -= 100
+            res[mode] = entry
+        for mode in ("ckpt", "skip"):
+            try:
+                res[f"{mode}_over_full"] = res[mode]["T_max"] / res["full"]["T_max"]
+            except Exception:  # noqa: BLE001
+                pass
+        out[bname] = res
+    out["paper"] = "A100 80 GB, VGG11/CIFAR100: BPTT T_max 200, checkpointed 4.5x (T=900), Skipper 9x (T=1800)"
+    return out
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -403,6 +487,17 @@ def run_ours(args):
                                  "ms_per_step": r["total_ms"] / args.steps, "peak_hbm_gb": r["peak_lib"] / 1e9}
             except Exception as e:  # noqa: BLE001
                 compare[mode] = {"error": str(e)[:200]}
+        # backward groups (skipper_config.group): G segments per layer-major backward pass, G x the segment arena
+        if args.mode in ("skip", "ckpt"):
+            for G in sorted({2, wl["C"]} - {args.group}):
+                try:
+                    a2 = argparse.Namespace(**dict(vars(args), group=G))
+                    r = run_mode(torch, dist, a2, wl, net, args.mode, rank, world, local_rank)
+                    compare[f"{args.mode}_group{G}"] = {
+                        "samples_per_s": wl["B"] * world * args.steps / (r["total_ms"] / 1e3),
+                        "ms_per_step": r["total_ms"] / args.steps, "peak_hbm_gb": r["peak_lib"] / 1e9}
+                except Exception as e:  # noqa: BLE001
+                    compare[f"{args.mode}_group{G}"] = {"error": str(e)[:200]}
     # peak HBM and throughput vs T (the metric's "vs T"): Skipper vs full BPTT, segment length S fixed
     t_sweep = {}
     if not args.no_compare and args.t_sweep:
@@ -453,6 +548,11 @@ def run_ours(args):
                 except Exception as e:  # noqa: BLE001
                     row[mode] = {"error": str(e)[:120]}
             sweep11[str(T)] = row
+    sqrt_leg, max_t = {}, {}
+    if not args.no_compare and args.t_sweep_vgg11:
+        sqrt_leg = sweep_sqrt_c(torch, dist, args, rank, world, local_rank)
+        if args.max_t:
+            max_t = max_t_search(torch, dist, args, rank, world, local_rank, sweep11)
     if rank != 0:
         if world > 1:
             dist.barrier()
@@ -478,6 +578,10 @@ def run_ours(args):
         cfg["other_workloads"] = other
     if sweep11:
         cfg["t_sweep_vgg11_cfg5"] = sweep11
+    if sqrt_leg:
+        cfg["t_sweep_vgg11_cfg5_c_sqrt_t"] = sqrt_leg
+    if max_t:
+        cfg["max_t_vgg11_cfg5"] = max_t
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": main["total_ms"] / args.steps, "higher_is_better": True,
@@ -526,13 +630,16 @@ def main():
     ap.add_argument("--C", type=int, default=0)
     ap.add_argument("--p", type=float, default=None)
     ap.add_argument("--ref-batch", type=int, default=1)
+    ap.add_argument("--group", type=int, default=1,
+                    help="CKPT/SKIP backward groups (skipper_config.group): 1 = the paper's per-segment schedule")
     ap.add_argument("--no-compare", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--t-sweep", default="50,200,400", help="extra T values for peak-HBM / throughput vs T")
     ap.add_argument("--workloads", default="cfg3_vgg11,cfg4_resnet_dvs",
                     help="other BASELINE.json configs measured briefly in the same run (config.other_workloads)")
     ap.add_argument("--t-sweep-vgg11", default="100,500,1000,2000",
-                    help="cfg 5: VGG-11 T values (B=128, C=5, p=50), all three modes")
+                    help="cfg 5: VGG-11 T values (B=128, C=5, p=50), all three modes; plus the C ~ sqrt(T) leg")
+    ap.add_argument("--max-t", type=int, default=1, help="cfg 5: max-T search per mode (80 GB and device HBM)")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

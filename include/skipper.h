@@ -111,6 +111,12 @@ typedef struct {
     float lr, beta1, beta2, eps;   /* Adam */
     int debug_record;      /* 1: keep per-step states for skipper_debug_copy (tests) */
     int sam;               /* skipper_sam (0 = Eq.4 spike sum) */
+    int group;             /* CKPT / SKIP backward groups: segments recomputed (one at a time) into one arena and
+                              back-propagated as one layer-major pass over their concatenated rows.  0 or 1 =
+                              the paper's schedule (one segment at a time); G > 1 trades a G-times
+                              larger segment arena (still O(T/C), Eq.6) for fewer, longer backward launches.
+                              The gradients are those of the per-segment schedule (the reverse scan carries
+                              delta across segment borders exactly as the per-segment carry does). */
 } skipper_config;
 
 /* Device-memory allocator used for every context allocation. */

@@ -145,6 +145,15 @@ struct skipper_ctx {
     std::vector<std::vector<int>> kept;
     std::vector<int> kept_flat;
     int Kmax = 0;
+    // backward groups (skipper_config.group = G): segments c_lo..c_lo+G-1 are recomputed one at a time into
+    // consecutive rows of one arena (ascending time) and back-propagated as ONE layer-major pass over the
+    // concatenated kept rows (the carry rule of Eq.2 across the segment border is the reverse scan's own)
+    int G = 1;
+    std::vector<int> seg_lo, seg_off, grp_R, grp_start;  // per segment: its group's lowest segment, row offset;
+                                                         // per lowest segment: group rows, start in grp_dev
+    std::vector<int> grp_flat;
+    int *grp_dev = nullptr;
+    int Rgrp = 0;                                        // arena rows: max over groups of the kept rows
     // arenas
     void *arena = nullptr;
     size_t arena_bytes = 0;
@@ -620,6 +629,7 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         }
     }
     c->S = c->T / c->C;
+    c->G = (cfg->mode == SKIPPER_MODE_CKPT || cfg->mode == SKIPPER_MODE_SKIP) ? std::max(1, std::min(cfg->group, c->C)) : 1;
     c->num_sms = sk::device_num_sms();
     c->host_prof = getenv("SKIPPER_HOST_PROFILE") && atoi(getenv("SKIPPER_HOST_PROFILE"));
     if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess)
@@ -743,10 +753,11 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     AL(c->dz, (size_t)c->B * ro.Cout);
     AL(c->loss_dev, 1);
     AL(c->kept_dev, (size_t)c->T);
+    AL(c->grp_dev, (size_t)c->T);
     // split-K slices of the weight gradients: the split count of every wgrad launch is at most the count the
-    // plan chooses at the layer's largest reduction (T rows in FULL mode, S otherwise), which sizes the slices
+    // plan chooses at the layer's largest reduction (T rows in FULL mode, G*S otherwise), which sizes the slices
     {
-        const long long Rmax = cfg->mode == SKIPPER_MODE_FULL ? c->T : c->S;
+        const long long Rmax = cfg->mode == SKIPPER_MODE_FULL ? c->T : (long long)c->S * c->G;  // rows per backward
         const long long nbmax = Rmax * c->B;
         const bool nw_off = getenv("SKIPPER_NO_NARROW_WGRAD") && atoi(getenv("SKIPPER_NO_NARROW_WGRAD"));
         // experiments: SKIPPER_WGRAD_ATOMIC=1 = the round-1 nondeterministic reduce-add into dW
@@ -850,6 +861,7 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         dev_free(c, c->dz, (size_t)c->B * ro.Cout * 4);
         dev_free(c, c->loss_dev, 4);
         dev_free(c, c->kept_dev, (size_t)c->T * 4);
+        dev_free(c, c->grp_dev, (size_t)c->T * 4);
         dev_free(c, c->x_stage, (size_t)c->T * c->B * c->in_elems);
         dev_free(c, c->y_stage, (size_t)c->B * 4);
         dev_free(c, c->x_enc, (size_t)c->T * c->B * c->in_elems);
@@ -1545,10 +1557,55 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
         c->Kmax = std::max<int>(c->Kmax, (int)c->kept[seg].size());
     }
     CK(cudaMemcpyAsync(c->kept_dev, c->kept_flat.data(), (size_t)C * S * 4, cudaMemcpyHostToDevice, c->st));
+    // backward groups of G segments from the top: [C-G, C-1], [C-2G, C-G-1], ... (the lowest may be smaller)
+    c->seg_lo.assign(C, 0);
+    c->seg_off.assign(C, 0);
+    c->grp_R.assign(C, 0);
+    c->grp_start.assign(C, 0);
+    c->grp_flat.clear();
+    c->Rgrp = 0;
+    for (int hi = C - 1; hi >= 0; hi -= c->G) {
+        const int lo = std::max(0, hi - c->G + 1);
+        c->grp_start[lo] = (int)c->grp_flat.size();
+        int R = 0;
+        for (int seg = lo; seg <= hi; ++seg) {
+            c->seg_lo[seg] = lo;
+            c->seg_off[seg] = R;
+            R += (int)c->kept[seg].size();
+            c->grp_flat.insert(c->grp_flat.end(), c->kept[seg].begin(), c->kept[seg].end());
+        }
+        c->grp_R[lo] = R;
+        c->Rgrp = std::max(c->Rgrp, R);
+    }
+    if (c->G > 1)
+        CK(cudaMemcpyAsync(c->grp_dev, c->grp_flat.data(), c->grp_flat.size() * 4, cudaMemcpyHostToDevice, c->st));
     return SKIPPER_OK;
 }
 
+static skipper_status recompute_segment_rows(skipper_ctx *c, int seg);
+
+// RECOMPUTE of segment seg into rows seg_off[seg].. of its group's arena: the per-layer arena bases (stored
+// membranes, layer outputs, layer-0 operand rows) are shifted for the duration of the segment
 static skipper_status recompute_segment(skipper_ctx *c, int seg) {
+    const size_t off = c->G > 1 ? (size_t)c->seg_off[seg] : 0;
+    if (!off) return recompute_segment_rows(c, seg);
+    for (auto &l : c->L) {
+        if (l.readout) continue;
+        l.Useg += off * c->B * l.N;
+        l.Po += off * c->B * l.Nout;
+    }
+    c->xg += off * c->B * c->in_row;
+    const skipper_status st = recompute_segment_rows(c, seg);
+    for (auto &l : c->L) {
+        if (l.readout) continue;
+        l.Useg -= off * c->B * l.N;
+        l.Po -= off * c->B * l.Nout;
+    }
+    c->xg -= off * c->B * c->in_row;
+    return st;
+}
+
+static skipper_status recompute_segment_rows(skipper_ctx *c, int seg) {
     const int R = (int)c->kept[seg].size();
     const int *row_t = c->kept_dev + (size_t)seg * c->S;
     // layer-0 weight-gradient operand (written by the fused layer-0 kernel itself when it runs)
@@ -1975,7 +2032,7 @@ extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int p
             CKS(forward_tail_chunk(c, seg - seg % c->tail_G, seg % c->tail_G + 1));
         if (seg == c->C - 1) {
             CKS(finish_first(c, labels_dev));
-            CKS(arena_rows(c, c->Kmax));
+            CKS(arena_rows(c, std::max(c->Kmax, c->Rgrp)));
             c->phase = PH_READY_BWD;
             c->next_seg = c->C - 1;
         }
@@ -2011,8 +2068,13 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
         return SKIPPER_OK;
     }
     const bool full = c->cfg.mode == SKIPPER_MODE_FULL;
-    const int R = full ? c->T : (int)c->kept[seg].size();
-    const int *row_t = full ? nullptr : c->kept_dev + (size_t)seg * c->S;
+    if (!full && c->G > 1 && c->seg_lo[seg] != seg) {  // grouped: the group's backward runs at its lowest segment
+        c->phase = PH_READY_BWD;
+        c->next_seg = seg - 1;
+        return SKIPPER_OK;
+    }
+    const int R = full ? c->T : c->G > 1 ? c->grp_R[seg] : (int)c->kept[seg].size();
+    const int *row_t = full ? nullptr : c->G > 1 ? c->grp_dev + c->grp_start[seg] : c->kept_dev + (size_t)seg * c->S;
     CKS(backward_rows(c, R, row_t, seg == 0));
     if (seg == 0) {
         const Layer &last = c->L[c->Ls - 1];

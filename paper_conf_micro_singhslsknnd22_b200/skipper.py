@@ -39,7 +39,7 @@ class Config(ct.Structure):
     _fields_ = [("T", ct.c_int), ("C", ct.c_int), ("p", ct.c_double), ("mode", ct.c_int), ("batch", ct.c_int),
                 ("global_batch", ct.c_int), ("surrogate", ct.c_int), ("surr_gamma", ct.c_float),
                 ("lr", ct.c_float), ("beta1", ct.c_float), ("beta2", ct.c_float), ("eps", ct.c_float),
-                ("debug_record", ct.c_int), ("sam", ct.c_int)]
+                ("debug_record", ct.c_int), ("sam", ct.c_int), ("group", ct.c_int)]
 
 
 ALLOC_FN = ct.CFUNCTYPE(ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
@@ -140,9 +140,9 @@ SAM = {"spikes": 0, "weighted": 1, "l2trace": 2}
 
 
 def make_config(T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle", gamma=0.3,
-                lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, sam="spikes"):
+                lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, sam="spikes", group=1):
     return Config(T, C, float(p), MODE[mode], batch, global_batch, SURROGATE[surrogate], gamma, lr, beta1, beta2,
-                  eps, 1 if debug_record else 0, SAM[sam])
+                  eps, 1 if debug_record else 0, SAM[sam], int(group))
 
 
 def sst_host(values, p):
@@ -197,7 +197,7 @@ class SkipperNet:
 
     def __init__(self, net, T, C=1, p=0.0, mode="skip", batch=1, global_batch=0, surrogate="triangle",
                  gamma=0.3, lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, debug_record=False, stream=None,
-                 torch_allocator=True, sam="spikes"):
+                 torch_allocator=True, sam="spikes", group=1):
         torch = _torch()
         self.net = net
         self.T, self.B = T, batch
@@ -206,7 +206,7 @@ class SkipperNet:
         self.device = torch.cuda.current_device()
         self.stream = stream if stream is not None else torch.cuda.current_stream()
         self.cfg = make_config(T, C, p, mode, batch, global_batch, surrogate, gamma, lr, beta1, beta2, eps,
-                               debug_record, sam)
+                               debug_record, sam, group)
         self._layers = make_layers(net)
         self._alloc = TorchAllocator(self.device) if torch_allocator else None
         h = ct.c_void_p()

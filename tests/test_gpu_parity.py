@@ -19,11 +19,11 @@ def _cuda():
     assert torch.cuda.is_available(), "GPU tests need a CUDA device"
 
 
-def run_gpu(net, W, x, y, T, C, p, mode, steps=1, sam="spikes", surrogate="triangle", gamma=0.3):
+def run_gpu(net, W, x, y, T, C, p, mode, steps=1, sam="spikes", surrogate="triangle", gamma=0.3, group=1):
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
     B = x.shape[1]
     m = SkipperNet(net, T, C=C, p=p, mode=mode, batch=B, debug_record=True, sam=sam, surrogate=surrogate,
-                   gamma=gamma)
+                   gamma=gamma, group=group)
     m.set_weights(W)
     xd = torch.from_numpy(np.ascontiguousarray(x)).cuda()
     yd = torch.from_numpy(np.ascontiguousarray(y)).cuda()
@@ -48,7 +48,7 @@ def grad_ok(g, r, tol=(1e-3, 1e-3)):
 
 
 def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=False, theta=None, wscale=1.0,
-                 surrogate="triangle", gamma=0.3, x_fn=None):
+                 surrogate="triangle", gamma=0.3, x_fn=None, group=1):
     """deep=True (networks deeper than the 11 spiking layers of VGG-11): a layer's dW tolerance is
     max(1e-3, twice the size of the bf16 contract's own effect on that layer), normwise and max-abs,
     DESIGN.md §4 "deep networks".  theta / wscale: threshold of every spiking layer and a power-of-two
@@ -69,7 +69,7 @@ def check_parity(name, T, B, C, p, mode, lam=None, seed=0, sam="spikes", deep=Fa
         for a, b in zip(ref.dW, exact.dW):
             en, em = grad_errs(b, a)
             tols.append((max(1e-3, 2 * en), max(1e-3, 2 * em)))
-    m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam, surrogate=surrogate, gamma=gamma)
+    m, loss = run_gpu(net, W, x, y, T, C, p, mode, sam=sam, surrogate=surrogate, gamma=gamma, group=group)
     spk = [L for L in net["layers"] if L["kind"] != "readout"]
     # SAM and mask (Eq.4, Eq.5)
     np.testing.assert_array_equal(m.spike_sums(), ref.s)
@@ -163,6 +163,16 @@ def test_tied_spike_sums(name, how):
     _, ref = check_parity(name, T=12 if name != "vgg5" else 14, B=2, C=2, p=40.0, mode="skip", x_fn=fn)
     if how == "zeros":
         assert (ref.s == 0).all() and all(len(k) == 1 for k in ref.kept)
+
+
+@pytest.mark.parametrize("name,T,B,C,mode,group", [("tiny_conv", 24, 3, 4, "skip", 2), ("tiny_conv", 24, 3, 4, "ckpt", 3),
+                                                  ("vgg5", 28, 2, 4, "skip", 4), ("tiny_resnet", 32, 2, 4, "skip", 2),
+                                                  ("fc784", 20, 4, 2, "skip", 2), ("tiny_fc", 24, 3, 3, "skip", 3)])
+def test_backward_groups(name, T, B, C, mode, group):
+    """skipper_config.group = G: G segments recomputed into one arena and back-propagated as one layer-major pass
+    (the reverse scan carries delta across the segment border as the per-segment carry does): the oracle's
+    per-segment Skipper / checkpointed gradients, spikes of every recomputed row exact."""
+    check_parity(name, T=T, B=B, C=C, p=50.0 if mode == "skip" else 0.0, mode=mode, group=group)
 
 
 @pytest.mark.parametrize("mode", ["full", "skip"])
