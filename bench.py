@@ -412,8 +412,9 @@ def sweep_sqrt_c(torch, dist, args, rank, world, local_rank):
 def max_t_search(torch, dist, args, rank, world, local_rank, sweep11):
     """cfg 5 / Fig. 14: the largest T (multiple of 100) each mode trains at C = 5, p = 50 within a
     memory budget - the A100's 80 GB and this device's whole HBM.  Peak HBM at fixed C is affine in T, so T_max is
-    predicted from the two largest T of the C = 5 sweep and then CHECKED by one training step at the predicted T
-    (stepping down by 100 while the step's measured peak exceeds the budget or it does not fit)."""
+    predicted from the two largest T of the C = 5 sweep and then CHECKED by training steps: bisection (multiples
+    of 100) between the largest sweep T that fit and the prediction, each probe one step whose measured peak must
+    stay within the budget (an allocation failure counts as not fitting)."""
     w5 = synth.workload("cfg3_vgg11")
     net5 = synth.net_config(w5["net"])
     total = torch.cuda.mem_get_info()[1]
@@ -432,20 +433,42 @@ def max_t_search(torch, dist, args, rank, world, local_rank, sweep11):
             slope = (p2 - p1) / (t2 - t1)
             Tm = int((t2 + (budget - p2) / slope) // 100 * 100)
             entry = {"predicted_T_max": Tm}
-            for _ in range(4):
-                if Tm < 100:
-                    break
+
+            def fits(T):
                 try:
-                    r = run_mode(torch, dist, args, dict(w5, T=Tm, C=5), net5, mode, rank, world, local_rank, steps=1,
+                    r = run_mode(torch, dist, args, dict(w5, T=T, C=5), net5, mode, rank, world, local_rank, steps=1,
                                  warmup=1)
-                    if r["peak_lib"] <= budget:
-                        entry.update({"T_max": Tm, "peak_hbm_gb": r["peak_lib"] / 1e9,
-                                      "samples_per_s": w5["B"] * world / (r["total_ms"] / 1e3)})
-                        break
-                    entry.setdefault("over_budget", []).append([Tm, r["peak_lib"] / 1e9])
                 except Exception as e:  # noqa: BLE001
-                    entry.setdefault("failed", []).append([Tm, str(e)[:80]])
-                Tm -= 100
+                    entry.setdefault("failed", []).append([T, str(e)[:80]])
+                    return None
+                if r["peak_lib"] > budget:
+                    entry.setdefault("over_budget", []).append([T, r["peak_lib"] / 1e9])
+                    return None
+                return r
+            # bisection on multiples of 100 between the largest sweep T known to fit and the prediction
+            lo, hi = (t2 // 100) * 100 if p2 <= budget else 0, Tm + 100
+            best = None
+            r = fits(Tm) if Tm >= 100 else None
+            if r is not None:
+                lo, best = Tm, (Tm, r)
+            else:
+                hi = Tm
+            for _ in range(6):
+                if hi - lo <= 100:
+                    break
+                mid = (lo + hi) // 200 * 100
+                r = fits(mid)
+                if r is not None:
+                    lo, best = mid, (mid, r)
+                else:
+                    hi = mid
+            if best is None and lo >= 100 and lo == (t2 // 100) * 100:
+                best = (lo, None)
+            if best is not None:
+                entry["T_max"] = best[0]
+                if best[1] is not None:
+                    entry.update({"peak_hbm_gb": best[1]["peak_lib"] / 1e9,
+                                  "samples_per_s": w5["B"] * world / (best[1]["total_ms"] / 1e3)})
             res[mode] = entry
         for mode in ("ckpt", "skip"):
             try:

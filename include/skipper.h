@@ -201,6 +201,13 @@ skipper_status skipper_step_host_encoded(skipper_ctx *ctx, const float *x_host, 
  * (the context is then poisoned). */
 skipper_status skipper_comm_unique_id(unsigned char id_out[128]);
 skipper_status skipper_comm_init(skipper_ctx *ctx, const unsigned char id[128], int rank, int world);
+/* The same data-parallel schedule with the collectives delegated to a host callback instead of NCCL:
+ * fn(buf_dev, count, dtype (0 f32, 1 f64, 2 int64), stream, user) must sum `count` elements at buf_dev
+ * over all ranks in place, ordered after the work already issued to `stream` (a cudaStream_t) and complete
+ * when it returns; it returns 0 on success (else the call fails with ENCCL).  For process groups NCCL cannot
+ * serve - several ranks on one GPU (tests: torch.distributed gloo), or a host-side transport. */
+typedef int (*skipper_allreduce_fn)(void *buf_dev, size_t count, int dtype, void *stream, void *user);
+skipper_status skipper_comm_init_callback(skipper_ctx *ctx, skipper_allreduce_fn fn, void *user, int rank, int world);
 /* The bucket plan (host only): walking spiking layers n_spiking-1 .. 1, closes[i] = 1 where a bucket of
  * >= bucket_bytes of fp32 gradients ends (layer 1 always ends the last one; layer 0 and the readout go
  * after segment 0).  Returns the number of buckets, or -1 for null pointers or n_spiking < 1. */

@@ -77,24 +77,49 @@ bool Comm::init(const unsigned char id[128], int r, int w, std::string *err) {
     return true;
 }
 
+bool Comm::init_callback(AllreduceFn fn, void *user, int r, int w, std::string *err) {
+    if (!fn) {
+        if (err) *err = "null allreduce callback";
+        return false;
+    }
+    cb = fn;
+    cb_user = user;
+    comm = this;
+    rank = r;
+    world = w;
+    return true;
+}
+
+static bool run_cb(const Comm &c, void *buf, size_t cnt, int dtype, cudaStream_t s, const char *what,
+                   std::string *err) {
+    if (c.cb(buf, cnt, dtype, s, c.cb_user) == 0) return true;
+    if (err) *err = std::string(what) + ": allreduce callback failed";
+    return false;
+}
+
 bool Comm::allreduce_i64(long long *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    if (cb) return run_cb(*this, buf, cnt, 2, s, "allreduce(s)", err);
     return check(nccl().allReduce(buf, buf, cnt, ncclInt64, ncclSum, static_cast<ncclComm_t>(comm), s),
                  "ncclAllReduce(s)", err);
 }
 
 bool Comm::allreduce_f64(double *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    if (cb) return run_cb(*this, buf, cnt, 1, s, "allreduce(u2)", err);
     return check(nccl().allReduce(buf, buf, cnt, ncclFloat64, ncclSum, static_cast<ncclComm_t>(comm), s),
                  "ncclAllReduce(u2)", err);
 }
 
 bool Comm::allreduce_f32(float *buf, size_t cnt, cudaStream_t s, std::string *err) {
+    if (cb) return run_cb(*this, buf, cnt, 0, s, "allreduce(dW)", err);
     return check(nccl().allReduce(buf, buf, cnt, ncclFloat32, ncclSum, static_cast<ncclComm_t>(comm), s),
                  "ncclAllReduce(dW)", err);
 }
 
 void Comm::destroy() {
-    if (comm && nccl().ok) nccl().commDestroy(static_cast<ncclComm_t>(comm));
+    if (comm && !cb && nccl().ok) nccl().commDestroy(static_cast<ncclComm_t>(comm));
     comm = nullptr;
+    cb = nullptr;
+    cb_user = nullptr;
     world = 1;
     rank = 0;
 }

@@ -2345,12 +2345,28 @@ extern "C" skipper_status skipper_comm_unique_id(unsigned char id_out[128]) {
     return SKIPPER_OK;
 }
 
+static skipper_status comm_setup(skipper_ctx *c);
+
 extern "C" skipper_status skipper_comm_init(skipper_ctx *c, const unsigned char id[128], int rank, int world) {
     CKS(check_ctx(c));
     if (world < 1 || rank < 0 || rank >= world) return fail(c, SKIPPER_EINVAL, "bad rank/world");
     // world == 1 also builds a (one-rank) communicator: the bucketed path then runs as an identity
     std::string e;
     if (!c->comm.init(id, rank, world, &e)) return fail(c, SKIPPER_ENCCL, "%s", e.c_str());
+    return comm_setup(c);
+}
+
+extern "C" skipper_status skipper_comm_init_callback(skipper_ctx *c, skipper_allreduce_fn fn, void *user, int rank,
+                                                     int world) {
+    CKS(check_ctx(c));
+    if (world < 1 || rank < 0 || rank >= world) return fail(c, SKIPPER_EINVAL, "bad rank/world");
+    std::string e;
+    if (!c->comm.init_callback(fn, user, rank, world, &e)) return fail(c, SKIPPER_EINVAL, "%s", e.c_str());
+    return comm_setup(c);
+}
+
+// comm stream, events and the dW bucket plan (both communicator kinds)
+static skipper_status comm_setup(skipper_ctx *c) {
     if (!c->st3 && cudaStreamCreateWithFlags(&c->st3, cudaStreamNonBlocking) != cudaSuccess)
         return fail(c, SKIPPER_ECUDA, "comm stream creation failed");
     if ((!c->ev_w && cudaEventCreateWithFlags(&c->ev_w, cudaEventDisableTiming) != cudaSuccess) ||

@@ -46,6 +46,17 @@ ALLOC_FN = ct.CFUNCTYPE(ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
 FREE_FN = ct.CFUNCTYPE(None, ct.c_void_p, ct.c_size_t, ct.c_void_p, ct.c_void_p)
 
 
+ALLREDUCE_FN = ct.CFUNCTYPE(ct.c_int, ct.c_void_p, ct.c_size_t, ct.c_int, ct.c_void_p, ct.c_void_p)
+
+
+class _DevArray:
+    """__cuda_array_interface__ view of a raw device buffer (torch.as_tensor wraps it without a copy)."""
+
+    def __init__(self, ptr, n, typestr):
+        self.__cuda_array_interface__ = {"shape": (int(n),), "typestr": typestr, "data": (int(ptr), False),
+                                         "version": 3, "strides": None}
+
+
 class Allocator(ct.Structure):
     _fields_ = [("alloc", ALLOC_FN), ("free", FREE_FN), ("user", ct.c_void_p)]
 
@@ -74,6 +85,7 @@ def _load():
         "skipper_step_host": (I, [P, P, P, P]),
         "skipper_comm_unique_id": (I, [P]),
         "skipper_comm_init": (I, [P, P, I, I]),
+        "skipper_comm_init_callback": (I, [P, ALLREDUCE_FN, P, I, I]),
         "skipper_get_loss": (I, [P, P]),
         "skipper_get_spike_sums": (I, [P, P]),
         "skipper_get_layer_spike_counts": (I, [P, P]),
@@ -325,6 +337,37 @@ class SkipperNet:
     def comm_init(self, uid: bytes, rank: int, world: int):
         buf = (ct.c_ubyte * 128).from_buffer_copy(uid)
         self._c(lib.skipper_comm_init(self.ctx, buf, rank, world))
+
+    def comm_init_host(self, rank: int, world: int, group=None):
+        """Data parallelism with the collectives on a torch.distributed process group (e.g. gloo) through
+        skipper_comm_init_callback: the library issues the same schedule (spike-count allreduce before Eq.5,
+        bucketed dW allreduce on its comm stream) and the callback reduces each buffer on the host (stream
+        synchronised, device -> host, all_reduce, host -> device).  For several ranks on one GPU, where NCCL
+        cannot run; the production path is comm_init (NCCL)."""
+        torch = _torch()
+        import torch.distributed as dist
+        dtypes = {0: (torch.float32, "<f4"), 1: (torch.float64, "<f8"), 2: (torch.int64, "<i8")}
+
+        def _cb(buf, count, dtype, stream, user):
+            try:
+                if stream:
+                    torch.cuda.ExternalStream(stream).synchronize()
+                else:
+                    torch.cuda.synchronize()
+                tdt, ts = dtypes[dtype]
+                dev = torch.as_tensor(_DevArray(buf, count, ts), device="cuda")
+                host = dev.cpu()
+                dist.all_reduce(host, group=group)
+                dev.copy_(host)
+                torch.cuda.current_stream().synchronize()
+                return 0
+            except Exception:  # noqa: BLE001 - reported to the library as a failed collective
+                import traceback
+                traceback.print_exc()
+                return 1
+
+        self._allreduce_cb = ALLREDUCE_FN(_cb)   # keep the trampoline alive with the context
+        self._c(lib.skipper_comm_init_callback(self.ctx, self._allreduce_cb, None, rank, world))
 
     # ------------------------------------------------------------------ introspection
     def loss(self):
