@@ -199,7 +199,8 @@ struct skipper_ctx {
     // host-side phase timing (SKIPPER_HOST_PROFILE=1, printed at destroy): issue of the first pass, the
     // mask sync wait, issue of recompute + backward + optimizer
     bool host_prof = false;
-    double hp_first = 0, hp_sync = 0, hp_bwd = 0;
+    double hp_first = 0, hp_sync = 0, hp_bwd = 0, hp_gap = 0;
+    cudaEvent_t hp_ev[2] = {nullptr, nullptr};  // device timeline: the mask D2H done / the first RECOMPUTE work
     long long hp_steps = 0;
 };
 
@@ -816,10 +817,12 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
 
 extern "C" void skipper_destroy(skipper_ctx *c) {
     if (!c) return;
+    if (c->hp_ev[0]) cudaEventDestroy(c->hp_ev[0]);
+    if (c->hp_ev[1]) cudaEventDestroy(c->hp_ev[1]);
     if (c->host_prof && c->hp_steps)
         fprintf(stderr, "skipper host profile: %lld steps, per step: first-pass issue %.3f ms, mask sync wait %.3f ms, "
-                        "recompute+backward issue %.3f ms\n", c->hp_steps, c->hp_first / c->hp_steps,
-                c->hp_sync / c->hp_steps, c->hp_bwd / c->hp_steps);
+                        "recompute+backward issue %.3f ms, device idle at the mask sync %.4f ms\n", c->hp_steps,
+                c->hp_first / c->hp_steps, c->hp_sync / c->hp_steps, c->hp_bwd / c->hp_steps, c->hp_gap / c->hp_steps);
     if (c->st) cudaStreamSynchronize(c->st);
     if (c->arena) dev_free(c, c->arena, c->arena_bytes);
     for (auto &l : c->L) {
@@ -1517,6 +1520,13 @@ static skipper_status finish_first(skipper_ctx *c, const int *labels) {
     CK(cudaMemcpyAsync(c->counts_host.data(), c->s_dev, (size_t)(c->Ls + 1) * c->T * 8, cudaMemcpyDeviceToHost,
                        c->st));
     const double hs0 = c->host_prof ? now_ms() : 0.0;
+    if (c->host_prof) {
+        if (!c->hp_ev[0]) {
+            cudaEventCreate(&c->hp_ev[0]);
+            cudaEventCreate(&c->hp_ev[1]);
+        }
+        cudaEventRecord(c->hp_ev[0], c->st);
+    }
     CK(cudaStreamSynchronize(c->st));  // the one host sync of the step
     if (c->host_prof) c->hp_sync += now_ms() - hs0;
     // SAM (Eq.4) and the policy metric: Eq.4 totals, or the neuron-count-weighted sum (reading 22)
@@ -2178,6 +2188,7 @@ extern "C" skipper_status skipper_step(skipper_ctx *c, const unsigned char *x_de
         for (int seg = 0; seg < c->C; ++seg)
             CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_FIRST, x_dev, seg == c->C - 1 ? labels_dev : nullptr));
         const double h1 = c->host_prof ? now_ms() : 0.0;
+        if (c->host_prof && c->hp_ev[1]) cudaEventRecord(c->hp_ev[1], c->st);  // after the kept-list H2D copy
         for (int seg = c->C - 1; seg >= 0; --seg) {
             CKS(skipper_forward_segment(c, seg, SKIPPER_PASS_RECOMPUTE, x_dev, nullptr));
             CKS(skipper_backward_segment(c, seg));
@@ -2186,6 +2197,10 @@ extern "C" skipper_status skipper_step(skipper_ctx *c, const unsigned char *x_de
             c->hp_first += (h1 - h0) - (c->hp_sync - s0);
             c->hp_bwd += now_ms() - h1;
             c->hp_steps++;
+            float gap = 0.f;
+            if (c->hp_ev[1] && cudaEventSynchronize(c->hp_ev[1]) == cudaSuccess &&
+                cudaEventElapsedTime(&gap, c->hp_ev[0], c->hp_ev[1]) == cudaSuccess)
+                c->hp_gap += gap;
         }
     }
     CKS(skipper_optimizer_step(c));
