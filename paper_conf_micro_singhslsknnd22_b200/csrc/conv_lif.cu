@@ -468,7 +468,10 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 CL_T0;
                 if (!(a.diag & 1)) emit(r);
                 CL_T1(3);
-                if (a.ckU && r == 0 && valid) store_state(a.ckU, a.cko, true);
+                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0) && valid) {
+                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * a.ck_stride : 0;
+                    store_state(a.ckU + slot, a.cko + slot, true);
+                }
             }
             if (!a.restore && valid && !(a.diag & 32)) store_state(a.U_state, a.o_state, true);
         }

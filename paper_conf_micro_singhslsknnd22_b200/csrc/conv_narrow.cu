@@ -356,7 +356,10 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? (N <= 16 ? 4 : 2) : 1) conv_
 #pragma unroll
                 for (int j = 0; j < NW; ++j) ob[j] = nb[j];
                 emit(r, true);
-                if (a.ckU && r == 0 && valid) store_state(a.ckU + nidx, a.cko + nidx);
+                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0) && valid) {
+                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * a.ck_stride : 0;
+                    store_state(a.ckU + slot + nidx, a.cko + slot + nidx);
+                }
             }
             if (valid && !a.restore) store_state(a.U_state + nidx, a.o_state + nidx);
         }

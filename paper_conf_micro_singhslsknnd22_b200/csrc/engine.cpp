@@ -116,6 +116,8 @@ struct skipper_ctx {
     bool l0_fused = false;      // layer 0 runs as the fused im2col+tcgen05+LIF kernel (layer0.cu)
     bool l0_bwd_fused = false;  // layer 0 backward: fused reverse scan + tcgen05 weight gradient
     int tail0 = 0;              // first layer of the fc tail: the first pass runs it per chunk of tail_G segments
+    int F = 1;                  // segments per first-pass launch of the layers before the fc tail
+    int fp_s0 = 0;              // first segment of the first-pass chunk in progress
     int tail_G = 1;             // segments per fc-tail chunk (tail_G * S * B <= max(SKIPPER_TAIL_ROWS, S * B) rows,
                                 // independent of T: keeps Eq.3's O(C) + O(S) law)
     uint16_t *tail_in = nullptr, *tailP[2] = {nullptr, nullptr};
@@ -580,6 +582,55 @@ static int fc_splits(int M, int N, int K, int num_sms) {
     return std::max(s, 1);
 }
 
+// First-pass arena layout for F segments per launch: only what the layers before the tail use - the output
+// ring (the last of them writes into the tail's input rows), fp32 currents of the layers that run as GEMM +
+// scan, the staged layer-0 operand when layer 0 is not the fused kernel, the im2col columns of icol layers -
+// and the fc tail's chunk buffers (input rows, ping-pong outputs, currents with split partials).
+struct FirstLayout {
+    size_t pbytes = 0, ibytes = 0, xbytes = 0, cbytes = 0, tin = 0, tp = 0, ti = 0, total = 0;
+};
+static FirstLayout first_layout(const skipper_ctx *c, int F) {
+    FirstLayout f;
+    const size_t rowsB = (size_t)F * c->S * c->B;
+    long long mo = 0, mio = 0, mic = 0;
+    for (int i = 0; i < c->tail0; ++i) {
+        const Layer &l = c->L[i];
+        if (i < c->tail0 - 1 || c->tail0 == c->Ls) mo = std::max(mo, l.Nout);
+        const bool kernel_lif = l.cfused || l.nlif || (i == 0 && c->l0_fused);
+        if (!kernel_lif) mio = std::max(mio, l.N * l.fsplit);
+        if (l.icol) mic = std::max(mic, (long long)l.H * l.W * 9 * l.Cin);
+    }
+    f.pbytes = al256(rowsB * mo * 2);
+    f.ibytes = al256(rowsB * mio * 4);
+    f.xbytes = (c->tail0 > 0 && !c->l0_fused) ? al256(rowsB * c->in_row * 2) : 0;
+    if (c->tail0 < c->Ls) {
+        const size_t rowsT = (size_t)c->tail_G * c->S * c->B;
+        f.tin = al256(rowsT * (c->tail0 == 0 ? c->in_row : c->L[c->tail0 - 1].Nout) * 2);
+        long long to = 0, ti = 0;
+        for (int i = c->tail0; i < c->Ls; ++i) {
+            to = std::max(to, c->L[i].Nout);
+            ti = std::max(ti, c->L[i].N * c->L[i].fsplitT);
+        }
+        f.tp = al256(rowsT * to * 2);
+        f.ti = al256(rowsT * ti * 4);
+    }
+    f.cbytes = al256(std::min<long long>(rowsB, icol_chunk(c)) * mic * 2);
+    f.total = c->nP * f.pbytes + f.ibytes + f.xbytes + f.cbytes + f.tin + 2 * f.tp + f.ti;
+    return f;
+}
+
+// RECOMPUTE / RECORD arena for R rows: per-layer stored U and outputs, fp32 I/g, bf16 delta ring, staged
+// layer-0 operand, icol columns
+static size_t rows_bytes(const skipper_ctx *c, int R) {
+    const size_t rowsB = (size_t)R * c->B;
+    size_t bytes = 0;
+    for (int i = 0; i < c->Ls; ++i) bytes += al256(rowsB * c->L[i].Nout * 2) + al256(rowsB * c->L[i].N * 4);
+    const long long ch = std::min<long long>(rowsB, icol_chunk(c));
+    bytes += al256(rowsB * max_gemm_io(c) * 4) + c->nD * (al256(rowsB * max_n(c) * 2) + al256(ch * max_icol(c) * 2)) +
+             al256(rowsB * c->in_row * 2) + al256(ch * max_icol(c) * 4);
+    return bytes;
+}
+
 extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_layers, const skipper_config *cfg,
                                          const skipper_allocator *alloc, void *cuda_stream, skipper_ctx **out) {
     if (out) *out = nullptr;
@@ -690,6 +741,25 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
         c->tail_G = (int)std::max<long long>(1, (c->C + nchunks - 1) / nchunks);  // balanced chunks
         for (int i = c->tail0; i < c->Ls; ++i)
             c->L[i].fsplitT = fc_splits(c->tail_G * c->S * c->B, c->L[i].Cout, c->L[i].Cin, c->num_sms);
+        // The first pass of the layers before the tail runs F segments per launch (checkpoints every S rows
+        // inside the kernels): fewer launches, each amortising its fixed cost (prologue, pipeline fill, state
+        // load / store) over more rows.  F * S * B <= SKIPPER_FIRST_ROWS (default 4096) sample-rows of
+        // first-pass buffers - a constant, so Eq.3's O(C) + O(S) law is kept.
+        // Bounded also so that the first-pass arena stays below the recompute arena of the expected kept rows
+        // ((1 - p/100)(S - 1) + 1): the step's peak memory stays the paper's (Eq.3 / Eq.6), F only spends
+        // memory the backward would claim anyway.
+        const char *ef = getenv("SKIPPER_FIRST_ROWS");
+        const long long frows = ef ? std::max(1, atoi(ef)) : 4096;
+        if (cfg->mode == SKIPPER_MODE_CKPT || cfg->mode == SKIPPER_MODE_SKIP) {
+            const int kexp = cfg->mode == SKIPPER_MODE_SKIP
+                                 ? std::min(c->S, 1 + (int)std::ceil((1.0 - cfg->p / 100.0) * (c->S - 1)))
+                                 : c->S;
+            const size_t cap = rows_bytes(c, kexp);
+            c->F = 1;
+            while (c->F < c->C && (long long)(c->F + 1) * c->S * c->B <= frows &&
+                   first_layout(c, c->F + 1).total <= cap)
+                ++c->F;
+        }
     }
 
     // ---- persistent allocations
@@ -982,40 +1052,30 @@ static skipper_status arena_free(skipper_ctx *c) {
     return SKIPPER_OK;
 }
 
+// [s0, end) of the first-pass chunk starting at segment s0: F segments, never across an fc-tail chunk border
+static int first_chunk_end(const skipper_ctx *c, int s0) {
+    int end = std::min(c->C, s0 + c->F);
+    if (c->tail0 < c->Ls) end = std::min(end, (s0 / c->tail_G + 1) * c->tail_G);
+    return end;
+}
+
 static skipper_status arena_first(skipper_ctx *c) {
     arena_free(c);
-    const size_t rowsB = (size_t)c->S * c->B;
-    const size_t pbytes = al256(rowsB * max_nout(c) * 2);
-    const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
-    const size_t xbytes = al256(rowsB * c->in_row * 2);
-    // fc tail over one chunk of tail_G * S rows: its input rows, ping-pong outputs, currents (with split partials)
-    size_t tin = 0, tp = 0, ti = 0;
-    if (c->tail0 < c->Ls) {
-        const size_t rowsT = (size_t)c->tail_G * c->S * c->B;
-        tin = al256(rowsT * (c->tail0 == 0 ? c->in_row : c->L[c->tail0 - 1].Nout) * 2);
-        long long mo = 0, mi = 0;
-        for (int i = c->tail0; i < c->Ls; ++i) {
-            mo = std::max(mo, c->L[i].Nout);
-            mi = std::max(mi, c->L[i].N * c->L[i].fsplitT);
-        }
-        tp = al256(rowsT * mo * 2);
-        ti = al256(rowsT * mi * 4);
-    }
-    const size_t cbytes = al256(std::min<long long>(rowsB, icol_chunk(c)) * max_icol(c) * 2);
+    const FirstLayout f = first_layout(c, c->F);
     const int nP = c->nP;
-    c->arena_bytes = nP * pbytes + ibytes + xbytes + tin + 2 * tp + ti + cbytes;
+    c->arena_bytes = f.total;
     c->arena = dev_alloc(c, c->arena_bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "first-pass arena of %zu bytes", c->arena_bytes);
     char *p = static_cast<char *>(c->arena);
-    for (int k = 0; k < nP; ++k) c->P2[k] = reinterpret_cast<uint16_t *>(p + k * pbytes);
-    c->I_buf = reinterpret_cast<float *>(p + nP * pbytes);
-    c->xg = reinterpret_cast<uint16_t *>(p + nP * pbytes + ibytes);
-    c->cols[0] = cbytes ? reinterpret_cast<uint16_t *>(p + nP * pbytes + ibytes + xbytes) : nullptr;
-    char *q = p + nP * pbytes + ibytes + xbytes + cbytes;
-    c->tail_in = tin ? reinterpret_cast<uint16_t *>(q) : nullptr;
-    c->tailP[0] = tp ? reinterpret_cast<uint16_t *>(q + tin) : nullptr;
-    c->tailP[1] = tp ? reinterpret_cast<uint16_t *>(q + tin + tp) : nullptr;
-    c->tail_I = ti ? reinterpret_cast<float *>(q + tin + 2 * tp) : nullptr;
+    for (int k = 0; k < nP; ++k) c->P2[k] = reinterpret_cast<uint16_t *>(p + k * f.pbytes);
+    c->I_buf = reinterpret_cast<float *>(p + nP * f.pbytes);
+    c->xg = reinterpret_cast<uint16_t *>(p + nP * f.pbytes + f.ibytes);
+    c->cols[0] = f.cbytes ? reinterpret_cast<uint16_t *>(p + nP * f.pbytes + f.ibytes + f.xbytes) : nullptr;
+    char *q = p + nP * f.pbytes + f.ibytes + f.xbytes + f.cbytes;
+    c->tail_in = f.tin ? reinterpret_cast<uint16_t *>(q) : nullptr;
+    c->tailP[0] = f.tp ? reinterpret_cast<uint16_t *>(q + f.tin) : nullptr;
+    c->tailP[1] = f.tp ? reinterpret_cast<uint16_t *>(q + f.tin + f.tp) : nullptr;
+    c->tail_I = f.ti ? reinterpret_cast<float *>(q + f.tin + 2 * f.tp) : nullptr;
     return SKIPPER_OK;
 }
 
@@ -1300,6 +1360,8 @@ static skipper_status layer0_fused(skipper_ctx *c, int seg, int R, int t0, const
     a.Po_out = out;
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * l.sbn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * l.sbn : nullptr;
+    a.ck_every = (a.ckU && R > c->S) ? c->S : 0;  // several segments per launch: a checkpoint every S rows
+    a.ck_stride = (long long)l.sbn;
     a.s_part = restore ? nullptr : spart(c, 1);
     a.s_part_in = restore ? nullptr : spart(c, 0);
     a.u2_part = restore ? nullptr : c->u2_part;
@@ -1338,6 +1400,8 @@ static skipper_status conv_lif_rows(skipper_ctx *c, int i, int seg, const uint16
     a.Po_out = out;
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * l.sbn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * l.sbn : nullptr;
+    a.ck_every = (a.ckU && R > c->S) ? c->S : 0;
+    a.ck_stride = (long long)l.sbn;
     a.s_part = restore ? nullptr : spart(c, i + 1);
     a.u2_part = restore ? nullptr : c->u2_part;
     a.dbg_U = c->cfg.debug_record ? l.dbg[restore ? 1 : 0] : nullptr;
@@ -1370,6 +1434,8 @@ static skipper_status narrow_lif_rows(skipper_ctx *c, int i, int seg, const uint
     a.Po_out = out;
     a.ckU = (!restore && !record) ? l.ckU + (size_t)seg * bn : nullptr;
     a.cko = (!restore && !record) ? l.cko + (size_t)seg * bn : nullptr;
+    a.ck_every = (a.ckU && R > c->S) ? c->S : 0;
+    a.ck_stride = (long long)bn;
     a.s_part = restore ? nullptr : spart(c, i + 1);
     a.u2_part = restore ? nullptr : c->u2_part;
     a.cnt = (i == c->Ls - 1) ? (restore ? c->cnt_kept : c->cnt) : nullptr;
@@ -1444,6 +1510,7 @@ static skipper_status forward_rows_first(skipper_ctx *c, int seg, int R, int t0,
         a.Po_out = out;
         a.ckU = record ? nullptr : l.ckU + (size_t)seg * c->B * l.N;
         a.cko = record ? nullptr : l.cko + (size_t)seg * c->B * l.N;
+        a.ck_every = (!record && R > c->S) ? c->S : 0;  // slots r / S, B*N apart
         a.s_part = spart(c, i + 1);
         a.u2_part = c->u2_part;
         a.row_t = nullptr;
@@ -2036,7 +2103,12 @@ extern "C" skipper_status skipper_forward_segment(skipper_ctx *c, int seg, int p
         if (x_dev != c->x_cur) return fail(c, SKIPPER_EINVAL, "x_dev changed within an iteration");
         // checked before any work or state change, so a retry with labels can continue from here
         if (seg == c->C - 1 && !labels_dev) return fail(c, SKIPPER_EINVAL, "the last FIRST segment needs labels");
-        CKS(forward_rows_first(c, seg, c->S, seg * c->S, false));
+        if (seg == 0) c->fp_s0 = 0;
+        const int end = first_chunk_end(c, c->fp_s0);
+        if (seg + 1 == end) {  // the chunk's last segment: its layers before the tail run now, F segments at once
+            CKS(forward_rows_first(c, c->fp_s0, (end - c->fp_s0) * c->S, c->fp_s0 * c->S, false));
+            c->fp_s0 = end;
+        }
         c->next_seg = seg + 1;
         if ((seg + 1) % c->tail_G == 0 || seg == c->C - 1)  // the fc tail of the chunk that ends here
             CKS(forward_tail_chunk(c, seg - seg % c->tail_G, seg % c->tail_G + 1));

@@ -107,6 +107,8 @@ struct NarrowConvArgs {
     uint16_t *Po_out;
     float *ckU;
     uint8_t *cko;
+    int ck_every;          // >0: rows r % ck_every == 0 write checkpoint slot r / ck_every (ck_stride elements
+    long long ck_stride;   // apart); 0: row 0 writes slot 0 (one segment per launch)
     unsigned *s_part;
     double *u2_part;
     float *cnt;
@@ -143,6 +145,8 @@ struct ConvLifArgs {
     uint16_t *Po_out;
     float *ckU;
     uint8_t *cko;
+    int ck_every;          // as NarrowConvArgs
+    long long ck_stride;
     unsigned *s_part;
     double *u2_part;  // l2-trace SAM partials [T][32] or null
     float *dbg_U;

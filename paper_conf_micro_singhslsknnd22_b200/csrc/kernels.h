@@ -121,6 +121,8 @@ struct L0FwdArgs {
     uint16_t *Po_out;      // [R][B*PH*PW*N] bf16
     float *ckU;            // FIRST: checkpoint slot (after row 0) or null
     uint8_t *cko;
+    int ck_every;          // >0: rows r % ck_every == 0 write checkpoint slot r / ck_every, ck_stride elements
+    long long ck_stride;   // apart (several segments per launch); 0: row 0 only
     unsigned *s_part;      // SAM partials [T][32] of this layer's spikes, or null
     unsigned *s_part_in;   // SAM partials [T][32] of the input spikes (l = 0), or null
     double *u2_part;       // l2-trace SAM: sum of U^2 per row into [T][32] fp64 partials, or null

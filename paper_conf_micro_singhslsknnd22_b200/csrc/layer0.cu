@@ -526,7 +526,10 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 }
                 ob = nb; L0_T1(7); L0_T0;
                 emit(ri); L0_T1(3); L0_T0;
-                if (a.ckU && ri == 0 && valid) store_state(a.ckU, a.cko, true);
+                if (a.ckU && (a.ck_every ? ri % a.ck_every == 0 : ri == 0) && valid) {
+                    const long long slot = a.ck_every ? (long long)(ri / a.ck_every) * a.ck_stride : 0;
+                    store_state(a.ckU + slot, a.cko + slot, true);
+                }
                 L0_T1(2);
             }
             L0_T0;

@@ -237,7 +237,10 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
 #pragma unroll
                 for (int j = 0; j < NW; ++j) ob[j] = nb[j];
                 emit(r, true);
-                if (a.ckU && r == 0) store_state(a.ckU + nidx, a.cko + nidx);
+                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0)) {
+                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * a.ck_stride : 0;
+                    store_state(a.ckU + slot + nidx, a.cko + slot + nidx);
+                }
             }
         }
         if (epi && !a.restore) store_state(a.U_state + nidx, a.o_state + nidx);
