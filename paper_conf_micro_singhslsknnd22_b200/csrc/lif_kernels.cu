@@ -385,14 +385,22 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
 }
 
 // ============================================================================ K4 reverse scan
-// One thread owns 4 neurons; the (g, U) loads of the next row are issued ahead of the reverse
-// recurrence of the current one.  One row per chunk at 8 resident blocks per SM measured faster than
-// two rows at 4 blocks (cfg 2 1.53 -> 1.33 ms, cfg 3 4.39 -> 3.72 ms, cfg 4 8.8 -> 7.8 ms per step):
-// the scan is latency-bound and more resident warps hide more of it than a deeper per-thread prefetch.
-template <int SPLIT>
-__global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanBwdArgs a) {
+// One thread owns 4 neurons (a float4 of channels of one pixel) and walks the rows downwards:
+//     delta_r = sigma'(U_r) * (gs * g_r) + lam * delta_{r+1}          (Eq.2, carry = delta after the last row)
+// The loop body is lean on purpose - the round-1 version was issue-bound (ncu: 80 % issue slots, 315 warp
+// instructions per row, a third of them 64-bit address arithmetic, branches and local-memory spills of
+// the prefetch arrays): row pointers walk down by a per-row stride, the surrogate kind is a template
+// parameter, gs * gamma is folded, and rows are consumed in unrolled chunks of CH with a scalar tail.
+#ifndef SK_BWD_CH
+#define SK_BWD_CH 2
+#endif
+#ifndef SK_BWD_MINB
+#define SK_BWD_MINB 8
+#endif
+template <int SPLIT, int KIND>
+__global__ void __launch_bounds__(256, SPLIT ? 4 : SK_BWD_MINB) lif_bwd_kernel(const ScanBwdArgs a) {
     pdl_enter();
-    constexpr int CH = 1;
+    constexpr int CH = SK_BWD_CH;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
     const long long rs = (long long)a.B * HW * C;
@@ -414,62 +422,70 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : 8) lif_bwd_kernel(const ScanB
     const float gs = a.g_pooled ? 0.25f : 1.0f;
     const int nspl = SPLIT ? a.nsplit : 1;
     // shortcut source (reading 8): S^T(delta of the receiving layer) joins g at this neuron, or not
-    long long rd_off = -1, rd_rs = 0;
+    const uint2 *rdp = nullptr;
+    long long rd_rs = 0;
     if (a.res_delta) {
         const int c = (int)(n0 % C);
         const long long pixel = n0 / C;
         const int x = (int)(pixel % a.W), y = (int)((pixel / a.W) % a.H);
         const long long b = pixel / HW;
-        const int s = a.res_stride, Hr = a.H / s, Wr = a.W / s;
+        const int sr = a.res_stride, Hr = a.H / sr, Wr = a.W / sr;
         rd_rs = (long long)a.B * Hr * Wr * a.res_C;
-        if (y % s == 0 && x % s == 0)
-            rd_off = ((b * Hr + y / s) * Wr + x / s) * a.res_C + c + a.res_lo;
+        if (y % sr == 0 && x % sr == 0)
+            rdp = reinterpret_cast<const uint2 *>(a.res_delta + ((b * Hr + y / sr) * Wr + x / sr) * a.res_C + c + a.res_lo);
     }
+    const float th = a.theta, inv_th = 1.0f / a.theta, lam = a.lam;
+    const float ggs = a.gamma * gs;  // triangle: gs * sigma' = (gs * gamma) * max(0, 1 - |U - theta| / theta)
+    auto sgm = [&](float u) -> float {  // gs * sigma'(u), reading 4
+        if (KIND == SURR_TRIANGLE) return ggs * fmaxf(0.0f, 1.0f - fabsf(u - th) * inv_th);
+        const float dd = 1.0f + a.gamma * fabsf(u - th);
+        return gs * __frcp_rn(dd * dd);
+    };
+    int r = a.R - 1;
+    const float *Up = a.U + (long long)r * rs + n0;
+    const float *Gp = a.g + (long long)r * grs + gi;
+    uint2 *Dp = a.delta ? reinterpret_cast<uint2 *>(a.delta + (long long)r * rs + n0) : nullptr;
+    const uint2 *Rp = rdp ? rdp + (long long)r * (rd_rs / 4) : nullptr;
+    const long long rs4 = rs / 4, rd4 = rd_rs / 4;   // uint2 = 4 bf16
     float4 d = *reinterpret_cast<const float4 *>(a.carry + n0);
-    const float inv_th = 1.0f / a.theta;
-    // two chunks of CH rows in flight: loads of the next (earlier) chunk overlap the recurrence
-    auto load = [&](float4 (&gv)[CH], float4 (&uv)[CH], int rb) {
+    auto load_g = [&](const float *gp, const uint2 *rp) -> float4 {
+        float4 g = SPLIT ? ldg4_split(gp, nspl, a.split_stride) : ldg4(gp);
+        if (rp) {  // unpooled layers only: gs = 1
+            const uint2 rv = __ldg(rp);
+            g.x = __fadd_rn(g.x, __uint_as_float(rv.x << 16));
+            g.y = __fadd_rn(g.y, __uint_as_float(rv.x & 0xffff0000u));
+            g.z = __fadd_rn(g.z, __uint_as_float(rv.y << 16));
+            g.w = __fadd_rn(g.w, __uint_as_float(rv.y & 0xffff0000u));
+        }
+        return g;
+    };
+    auto step = [&](const float4 &u, const float4 &g, uint2 *dp) {
+        d.x = sgm(u.x) * g.x + lam * d.x;
+        d.y = sgm(u.y) * g.y + lam * d.y;
+        d.z = sgm(u.z) * g.z + lam * d.z;
+        d.w = sgm(u.w) * g.w + lam * d.w;
+        if (dp) *dp = pack_bf16x4(d.x, d.y, d.z, d.w);
+    };
+    for (; r >= CH - 1; r -= CH) {
+        float4 uv[CH], gv[CH];
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
-            const int r = rb - j;
-            if (r >= 0) {
-                const float *src = a.g + (long long)r * grs + gi;
-                gv[j] = SPLIT ? ldg4_split(src, nspl, a.split_stride) : ldg4(src);
-                uv[j] = ldg4(a.U + (long long)r * rs + n0);
-                if (rd_off >= 0) {
-                    const uint2 rv = __ldg(reinterpret_cast<const uint2 *>(a.res_delta + (long long)r * rd_rs + rd_off));
-                    gv[j].x = __fadd_rn(gv[j].x, __uint_as_float(rv.x << 16));  // unpooled: gs = 1
-                    gv[j].y = __fadd_rn(gv[j].y, __uint_as_float(rv.x & 0xffff0000u));  // unpooled: gs = 1
-                    gv[j].z = __fadd_rn(gv[j].z, __uint_as_float(rv.y << 16));  // unpooled: gs = 1
-                    gv[j].w = __fadd_rn(gv[j].w, __uint_as_float(rv.y & 0xffff0000u));  // unpooled: gs = 1
-                }
-            }
+            uv[j] = ldg4(Up - j * rs);
+            gv[j] = load_g(Gp - j * grs, Rp ? Rp - j * rd4 : nullptr);
         }
-    };
-    auto consume = [&](const float4 (&gv)[CH], const float4 (&uv)[CH], int rb) {
 #pragma unroll
-        for (int j = 0; j < CH; ++j) {
-            const int r = rb - j;
-            if (r >= 0) {
-                d.x = surrogate(uv[j].x, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].x) + a.lam * d.x;
-                d.y = surrogate(uv[j].y, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].y) + a.lam * d.y;
-                d.z = surrogate(uv[j].z, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].z) + a.lam * d.z;
-                d.w = surrogate(uv[j].w, a.theta, inv_th, a.surr, a.gamma) * (gs * gv[j].w) + a.lam * d.w;
-                if (a.delta)
-                    *reinterpret_cast<uint2 *>(a.delta + (long long)r * rs + n0) = pack_bf16x4(d.x, d.y, d.z, d.w);
-            }
-        }
-    };
-    {
-        float4 gA[CH], uA[CH], gB[CH], uB[CH];
-        load(gA, uA, a.R - 1);
-        for (int rb = a.R - 1; rb >= 0; rb -= 2 * CH) {
-            if (rb - CH >= 0) load(gB, uB, rb - CH);
-            consume(gA, uA, rb);
-            if (rb - CH < 0) break;
-            if (rb - 2 * CH >= 0) load(gA, uA, rb - 2 * CH);
-            consume(gB, uB, rb - CH);
-        }
+        for (int j = 0; j < CH; ++j) step(uv[j], gv[j], Dp ? Dp - j * rs4 : nullptr);
+        Up -= CH * rs;
+        Gp -= CH * grs;
+        if (Dp) Dp -= CH * rs4;
+        if (Rp) Rp -= CH * rd4;
+    }
+    for (; r >= 0; --r) {
+        step(ldg4(Up), load_g(Gp, Rp), Dp);
+        Up -= rs;
+        Gp -= grs;
+        if (Dp) Dp -= rs4;
+        if (Rp) Rp -= rd4;
     }
     *reinterpret_cast<float4 *>(a.carry + n0) = d;
 }
@@ -523,10 +539,15 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
         return cudaGetLastError();
     }
     const long long P = rs / 4;
-    if (a.nsplit > 1)
-        sk_launch(lif_bwd_kernel<1>, (unsigned)((P + 255) / 256), 256, 0, s, a);
-    else
-        sk_launch(lif_bwd_kernel<0>, (unsigned)((P + 255) / 256), 256, 0, s, a);
+    const unsigned grid = (unsigned)((P + 255) / 256);
+    const bool tri = a.surr == SURR_TRIANGLE;
+    if (a.nsplit > 1) {
+        if (tri) sk_launch(lif_bwd_kernel<1, SURR_TRIANGLE>, grid, 256, 0, s, a);
+        else sk_launch(lif_bwd_kernel<1, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+    } else {
+        if (tri) sk_launch(lif_bwd_kernel<0, SURR_TRIANGLE>, grid, 256, 0, s, a);
+        else sk_launch(lif_bwd_kernel<0, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+    }
     return cudaGetLastError();
 }
 
