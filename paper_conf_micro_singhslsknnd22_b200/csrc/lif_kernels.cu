@@ -524,6 +524,72 @@ __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a)
     a.carry[n] = d;
 }
 
+// fc layers with long row ranges (FULL / CKPT / TBPTT segments): Eq.2's reverse recurrence is affine in delta,
+//     delta_r = c_r + lam * delta_{r+1},   c_r = sigma'(U_r) g_r,
+// so a segment of rows maps the delta after it to the delta at its first row by (A, Bv) = (lam^len, sum_k
+// lam^(k - lo) c_k), and segments compose.  A warp holds 8 neurons x 4 row chunks (lane = chunk * 8 +
+// neuron, so each row's 8 neurons are one 32-byte sector): every lane folds its chunk to (A, Bv), the four
+// chunk maps of a neuron are exchanged with __shfl_sync and composed from the carry down to chunk 0, and
+// each lane re-walks its chunk from its exact incoming delta, writing delta_r - the serial depth drops from
+// R to R/4 + 4.  (Rounding differs from the serial walk only in the composed incoming deltas.)
+template <int SPLIT, int KIND>
+__global__ void __launch_bounds__(256) lif_bwd_warp_kernel(const ScanBwdArgs a) {
+    pdl_enter();
+    constexpr int NCH = 4, NPW = 32 / NCH;   // row chunks, neurons per warp
+    const long long rs = (long long)a.B * a.C;
+    const int lane = threadIdx.x & 31, q = lane % NPW, j = lane / NPW;
+    const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const long long n = warp * NPW + q;
+    const bool act = n < rs;
+    const long long nn = act ? n : 0;
+    const long long grs = a.g_broadcast ? 0 : rs;
+    const float th = a.theta, inv_th = 1.0f / a.theta, lam = a.lam;
+    auto c_at = [&](int r) -> float {  // sigma'(U_r) g_r
+        const float *gp = a.g + (long long)r * grs + nn;
+        const float g = SPLIT ? ldg_split(gp, a.nsplit, a.split_stride) : __ldg(gp);
+        const float u = __ldg(a.U + (long long)r * rs + nn);
+        float sg;
+        if (KIND == SURR_TRIANGLE) {
+            sg = a.gamma * fmaxf(0.0f, 1.0f - fabsf(u - th) * inv_th);
+        } else {
+            const float dd = 1.0f + a.gamma * fabsf(u - th);
+            sg = __frcp_rn(dd * dd);
+        }
+        return sg * g;
+    };
+    const int L = (a.R + NCH - 1) / NCH;
+    const int lo = min(a.R, j * L), hi = min(a.R, lo + L);
+    // 1. this chunk's map: delta_lo = A * delta_hi + Bv
+    float A = 1.0f, Bv = 0.0f;
+    if (act)
+        for (int r = hi - 1; r >= lo; --r) {
+            Bv = c_at(r) + lam * Bv;
+            A *= lam;
+        }
+    // 2. compose the four maps of this neuron from the carry (after the last row) down to chunk 0
+    float Ak[NCH], Bk[NCH];
+#pragma unroll
+    for (int k = 0; k < NCH; ++k) {
+        Ak[k] = __shfl_sync(0xffffffffu, A, k * NPW + q);
+        Bk[k] = __shfl_sync(0xffffffffu, Bv, k * NPW + q);
+    }
+    float din = act ? a.carry[nn] : 0.0f;   // delta after chunk NCH-1
+    float mine = din;
+#pragma unroll
+    for (int k = NCH - 1; k >= 0; --k) {
+        if (k == j) mine = din;             // delta after this lane's chunk
+        din = Ak[k] * din + Bk[k];
+    }
+    // 3. re-walk the chunk from its incoming delta, emitting every delta_r
+    float d = mine;
+    if (act)
+        for (int r = hi - 1; r >= lo; --r) {
+            d = c_at(r) + lam * d;
+            if (a.delta) a.delta[(long long)r * rs + n] = f2bf_bits(d);
+        }
+    if (act && j == 0) a.carry[n] = lo < hi ? d : mine;
+}
+
 cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     if (a.C % 4) return cudaErrorInvalidValue;
     const long long rs = (long long)a.B * a.H * a.W * a.C;
@@ -532,6 +598,19 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
                         a.W % a.res_stride))
         return cudaErrorInvalidValue;
     if (!a.g_pooled && !a.res_delta && a.H * a.W == 1 && rs <= (1LL << 20)) {  // fc layers
+        static const bool warp_off = getenv("SKIPPER_NO_WARP_SCAN") && atoi(getenv("SKIPPER_NO_WARP_SCAN"));
+        if (a.R >= 16 && !warp_off) {   // long segments: the warp-parallel affine scan
+            const unsigned grid = (unsigned)((rs + 63) / 64);   // 8 warps x 8 neurons per block
+            const bool tri = a.surr == SURR_TRIANGLE;
+            if (a.nsplit > 1) {
+                if (tri) sk_launch(lif_bwd_warp_kernel<1, SURR_TRIANGLE>, grid, 256, 0, s, a);
+                else sk_launch(lif_bwd_warp_kernel<1, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+            } else {
+                if (tri) sk_launch(lif_bwd_warp_kernel<0, SURR_TRIANGLE>, grid, 256, 0, s, a);
+                else sk_launch(lif_bwd_warp_kernel<0, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+            }
+            return cudaGetLastError();
+        }
         if (a.nsplit > 1)
             sk_launch(lif_bwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
         else

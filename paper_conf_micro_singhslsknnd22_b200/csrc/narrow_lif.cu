@@ -130,18 +130,18 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
             for (int j = 0; j < NW; ++j) cnt += __popc(ob[j]);
             uint16_t *po = a.Po_out + (long long)r * rs + nidx;
 #pragma unroll
-            for (int c = 0; c < N; c += 8) {
+            for (int c = 0; c < N; c += 16) {  // 16 bf16 spikes = one 32-byte sector per store
                 const uint32_t w = ob[c >> 5] >> (c & 31);
-                uint32_t pk[4];
+                uint32_t pk[8];
 #pragma unroll
-                for (int e = 0; e < 4; ++e)
+                for (int e = 0; e < 8; ++e)
                     pk[e] = (((w >> (2 * e)) & 1u) ? 0x3F80u : 0u) | (((w >> (2 * e + 1)) & 1u) ? 0x3F800000u : 0u);
-                *reinterpret_cast<uint4 *>(po + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+                st_global_v8u(po + c, make_uint4(pk[0], pk[1], pk[2], pk[3]), make_uint4(pk[4], pk[5], pk[6], pk[7]));
             }
             if (a.U_out) {
                 float *du = a.U_out + (long long)r * rs + nidx;
 #pragma unroll
-                for (int c = 0; c < N; c += 4) *reinterpret_cast<float4 *>(du + c) = make_float4(U[c], U[c + 1], U[c + 2], U[c + 3]);
+                for (int c = 0; c < N; c += 8) st_global_v8(du + c, U + c);
             }
             if (a.dbg_U) store_state(a.dbg_U + t * rs + nidx, a.dbg_o + t * rs + nidx);
             if (a.cnt) {

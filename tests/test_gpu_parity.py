@@ -175,6 +175,16 @@ def test_backward_groups(name, T, B, C, mode, group):
     check_parity(name, T=T, B=B, C=C, p=50.0 if mode == "skip" else 0.0, mode=mode, group=group)
 
 
+@pytest.mark.parametrize("name,T,B,C,mode", [("fc784", 64, 4, 1, "full"), ("tiny_fc", 40, 3, 1, "full"),
+                                            ("tiny_fc", 48, 3, 2, "ckpt"), ("fc784", 60, 4, 3, "tbptt"),
+                                            ("tiny_conv", 36, 2, 1, "full")])
+def test_warp_parallel_fc_scan(name, T, B, C, mode):
+    """The warp-parallel affine reverse scan of fc layers (lif_bwd_warp_kernel: 4 row chunks per neuron folded
+    to (lam^len, partial) maps, composed with __shfl_sync, re-walked) on segments of >= 16 rows, against the
+    oracle's serial Eq.2 recurrence."""
+    check_parity(name, T=T, B=B, C=C, p=0.0, mode=mode)
+
+
 @pytest.mark.parametrize("mode", ["full", "skip"])
 def test_vgg5_reduced(mode):
     """cfg 2 topology (VGG-5) at reduced T and B: every kernel kind, several tiles, ragged tails."""
