@@ -49,14 +49,19 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
     const int Hin = a.Hin, Win = a.Win;
     const int RX = S * (TH - 1) + 3;                       // staged input rows per band
     const int XBUF = RX * Win * CIN;                       // bf16 elements of one staging buffer
-    uint16_t *sW = reinterpret_cast<uint16_t *>(smem);    // [N][9][CIN] resident weights
-    uint16_t *sX = sW + N * 9 * CIN;                       // 2 x [RX][Win][CIN]
+    // resident weights [9][N][WP]: row pitch WP = CIN + 8 (48 bytes for CIN = 16), so the 8 output-channel
+    // rows an ldmatrix reads land in 8 distinct 16-byte bank groups (the [N][9][CIN] layout was 2-way)
+    constexpr int WP = CIN + 8;
+    uint16_t *sW = reinterpret_cast<uint16_t *>(smem);
+    uint16_t *sX = sW + 9 * N * WP;                        // 2 x [RX][Win][CIN] (stride 1: chunk-swizzled)
     uint16_t *sZ = sX + 2 * (size_t)XBUF;                  // zero row [CIN]
     float *sI = reinterpret_cast<float *>(sZ + CIN);      // [NL_P][N + 1] currents of the row
     constexpr int IP = N + 1;                              // padded pitch (conflict-free column writes)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    for (int i = threadIdx.x; i < N * 9 * CIN / 8; i += NL_THREADS)
-        reinterpret_cast<uint4 *>(sW)[i] = __ldg(reinterpret_cast<const uint4 *>(a.Wk) + i);
+    for (int i = threadIdx.x; i < N * 9 * CIN / 8; i += NL_THREADS) {  // Wk [N][9][CIN] -> [9][N][WP]
+        const int co = i / (9 * CIN / 8), rem = i - co * (9 * CIN / 8), tap = rem / (CIN / 8), cc = rem % (CIN / 8);
+        *reinterpret_cast<uint4 *>(sW + (tap * N + co) * WP + cc * 8) = __ldg(reinterpret_cast<const uint4 *>(a.Wk) + i);
+    }
     if (threadIdx.x < CIN / 8) reinterpret_cast<uint4 *>(sZ)[threadIdx.x] = make_uint4(0u, 0u, 0u, 0u);
 
     const long long HW = (long long)a.H * a.W;
@@ -66,6 +71,12 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
     const int r_mma0 = a.restore ? 1 : 0;
     const long long in_row = (long long)a.nb * Hin * Win * CIN;
     const uint32_t sW_a = smem_u32(sW), sX_a = smem_u32(sX), sZ_a = smem_u32(sZ);
+    // stride 1, CIN = 16: a staged pixel is two 16-byte chunks; chunk k of pixel q sits at chunk slot
+    // 2q + (k ^ ((q >> 2) & 1)), so ANY 8 consecutive pixels' chunk k (the rows of one ldmatrix 8x8 matrix,
+    // whatever the tap shift) fall in 8 distinct bank groups - unswizzled the 32-byte pixel pitch made them
+    // 2-way conflicting (ncu: 48 % of the shared-load wavefronts excessive)
+    constexpr bool SWZ = (S == 1 && CIN == 16);
+    auto xswz = [&](int c) -> int { return SWZ ? (c ^ ((c >> 3) & 1)) : c; };   // chunk index c = 2q + k
     const int P = TH * a.W;                                  // == NL_P
 
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
@@ -81,7 +92,7 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
                 const int yi = S * y0 - 1 + rr;
                 const bool in = yi >= 0 && yi < Hin;
                 const uint4 *src = reinterpret_cast<const uint4 *>(Xr + ((n * Hin + (in ? yi : 0)) * (long long)Win) * CIN) + e;
-                cp_async16_cg(dst + 16u * i, src, in ? 16u : 0u);
+                cp_async16_cg(dst + 16u * (uint32_t)xswz(i), src, in ? 16u : 0u);
             }
             cp_async_commit();
         };
@@ -190,16 +201,18 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
                     const int xs = S * xa + dx - 1, ys = S * ya + dy;
                     const int yi = S * y0 - 1 + ys;
                     const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
-                    const uint32_t arow = ok ? xb + (uint32_t)((ys * Win + xs) * CIN) * 2u : sZ_a;
+                    const int q = ys * Win + xs;   // staged pixel
 #pragma unroll
                     for (int ks = 0; ks < CIN / 16; ++ks) {
                         uint32_t a0, a1, a2, a3;
-                        nl_ldsm_x4(arow + (uint32_t)(ks * 16 + kh) * 2u, a0, a1, a2, a3);
+                        const int chunk = q * (CIN / 8) + (ks * 16 + kh) / 8;
+                        const uint32_t aaddr = ok ? xb + 16u * (uint32_t)xswz(chunk) : sZ_a + (uint32_t)kh * 2u;
+                        nl_ldsm_x4(aaddr, a0, a1, a2, a3);
 #pragma unroll
                         for (int nt = 0; nt < N / 8; ++nt) {
                             uint32_t b0, b1;
                             const int co = nt * 8 + (lane & 7), ci = ks * 16 + ((lane >> 3) & 1) * 8;
-                            nl_ldsm_x2(sW_a + (uint32_t)((co * 9 + tap) * CIN + ci) * 2u, b0, b1);
+                            nl_ldsm_x2(sW_a + (uint32_t)((tap * N + co) * WP + ci) * 2u, b0, b1);
                             nl_mma(acc[nt], a0, a1, a2, a3, b0, b1);
                         }
                     }
@@ -260,7 +273,7 @@ template <int CIN, int N, int S>
 static cudaError_t launch_nl(const NarrowConvArgs &a, cudaStream_t s, int num_sms) {
     const int TH = NL_P / a.W;
     const int RX = S * (TH - 1) + 3;
-    const size_t smem = (size_t)N * 9 * CIN * 2 + 2 * (size_t)RX * a.Win * CIN * 2 + CIN * 2 + (size_t)NL_P * (N + 1) * 4;
+    const size_t smem = (size_t)9 * N * (CIN + 8) * 2 + 2 * (size_t)RX * a.Win * CIN * 2 + CIN * 2 + (size_t)NL_P * (N + 1) * 4;
     auto kern = narrow_lif_kernel<CIN, N, S>;
     static bool attr = false;
     if (!attr) {
