@@ -71,12 +71,12 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
     const int r_mma0 = a.restore ? 1 : 0;
     const long long in_row = (long long)a.nb * Hin * Win * CIN;
     const uint32_t sW_a = smem_u32(sW), sX_a = smem_u32(sX), sZ_a = smem_u32(sZ);
-    // stride 1, CIN = 16: a staged pixel is two 16-byte chunks; chunk k of pixel q sits at chunk slot
+    // CIN = 16: a staged pixel is two 16-byte chunks; chunk k of pixel q sits at chunk slot
     // 2q + (k ^ ((q >> 2) & 1)), so ANY 8 consecutive pixels' chunk k (the rows of one ldmatrix 8x8 matrix,
     // whatever the tap shift) fall in 8 distinct bank groups - unswizzled the 32-byte pixel pitch made them
     // 2-way conflicting (ncu: 48 % of the shared-load wavefronts excessive)
-    constexpr bool SWZ = (S == 1 && CIN == 16);
-    auto xswz = [&](int c) -> int { return SWZ ? (c ^ ((c >> 3) & 1)) : c; };   // chunk index c = 2q + k
+    // (stride 2 reads every other pixel: the swizzle halves that 4-way conflict to 2-way)
+    auto xswz = [&](int c) -> int { return c ^ ((c >> 3) & (CIN / 8 - 1)); };   // chunk index c = (CIN/8) q + k
     const int P = TH * a.W;                                  // == NL_P
 
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {

@@ -35,6 +35,15 @@ struct NwCfg {
     static_assert(8 % COMBOS == 0, "work items must divide the 8 warps");
 };
 
+// Staged [pixel][C] bf16 rows are ldmatrix'ed as 8 consecutive pixels' 16-byte chunk k.  With CP = C / 8
+// chunks per pixel that is 8 rows at a CP x 16-byte pitch: 2- (C = 16), 4- (32) or 8-way (64) bank conflicts.
+// Chunk c (= CP * pixel + k) is stored at slot c ^ ((c >> 3) & (CP - 1)): the 8 rows of any 8 consecutive
+// pixels land in 8 distinct 16-byte bank groups.
+template <int C>
+SK_DEV uint32_t xswz(uint32_t c) {
+    return c ^ ((c >> 3) & (uint32_t)(C / 8 - 1));
+}
+
 SK_DEV void ldsm_x4_t(uint32_t addr, uint32_t &r0, uint32_t &r1, uint32_t &r2, uint32_t &r3) {
     asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0, %1, %2, %3}, [%4];"
                  : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
@@ -91,7 +100,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
         const uint32_t dD = sB_a + (uint32_t)(b * BUF) * 2u, dX = dD + (uint32_t)(NW_P * COUT) * 2u;
         const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + y0) * (long long)W) * COUT);
         const int nD = TH * W * COUT / 8;
-        for (int i = threadIdx.x; i < nD; i += NW_THREADS) cp_async16_cg(dD + 16u * i, src + i, 16u);
+        for (int i = threadIdx.x; i < nD; i += NW_THREADS) cp_async16_cg(dD + 16u * xswz<COUT>(i), src + i, 16u);
         const int rowv = Win * CIN / 8;
         const int nX = RX * rowv;
         for (int i = threadIdx.x; i < nX; i += NW_THREADS) {
@@ -99,7 +108,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
             const int yi = S * y0 - 1 + r;
             const bool in = yi >= 0 && yi < Hin;
             const uint4 *xs = reinterpret_cast<const uint4 *>(X + ((n * Hin + (in ? yi : 0)) * (long long)Win) * CIN) + e;
-            cp_async16_cg(dX + 16u * i, xs, in ? 16u : 0u);
+            cp_async16_cg(dX + 16u * xswz<CIN>(i), xs, in ? 16u : 0u);
         }
         cp_async_commit();
     };
@@ -125,7 +134,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
                 const int j = lane >> 3, r = lane & 7;
                 const int k = kc * 16 + ((j & 2) ? 8 : 0) + r;
                 const int m = mt * 16 + ((j & 1) ? 8 : 0);
-                ldsm_x4_t(sD_a + (uint32_t)(k * COUT + m) * 2u, a0, a1, a2, a3);
+                ldsm_x4_t(sD_a + 16u * xswz<COUT>((uint32_t)(k * (COUT / 8) + m / 8)), a0, a1, a2, a3);
             }
             // this lane's B row: output pixel kc*16 + (lane & 15)
             const int p = kc * 16 + (lane & 15);
@@ -139,11 +148,11 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_wgrad_kernel(const uint16_t
                 const int ys = S * yl + dy;                       // staged row
                 const int yi = S * y0 - 1 + ys;                   // image row
                 const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
-                const uint32_t row = ok ? sX_a + (uint32_t)((ys * Win + xs) * CIN) * 2u : sZ_a;
+                const uint32_t c0 = (uint32_t)((ys * Win + xs) * (CIN / 8));
 #pragma unroll
                 for (int j = 0; j < Cfg::NTT; ++j) {
                     uint32_t b0, b1;
-                    ldsm_x2_t(row + (uint32_t)j * 16u, b0, b1);
+                    ldsm_x2_t(ok ? sX_a + 16u * xswz<CIN>(c0 + j) : sZ_a + (uint32_t)j * 16u, b0, b1);
                     mma_bf16(acc[t][j], a0, a1, a2, a3, b0, b1);
                 }
             }
@@ -222,12 +231,15 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
     const int Hg = S * H, Wg = S * W;                     // G (layer input) size
     const int RD = TH / S + 2;                            // staged delta rows per band (max)
     const int BUF = RD * W * CO;                          // bf16 elements of one staging buffer
-    uint16_t *sW = reinterpret_cast<uint16_t *>(smem);   // [CI][9][CO]
-    uint16_t *sB = sW + 9 * CI * CO;                      // 2 x [RD][W][CO]
+    constexpr int WP = CO + 8;                            // weight row pitch: conflict-free ldmatrix rows
+    uint16_t *sW = reinterpret_cast<uint16_t *>(smem);   // [9][CI][WP]
+    uint16_t *sB = sW + 9 * CI * WP;                      // 2 x [RD][W][CO] (chunk-swizzled)
     uint16_t *sZ = sB + 2 * (size_t)BUF;                  // zero row [CO]
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    for (int i = threadIdx.x; i < 9 * CI * CO / 8; i += NW_THREADS)
-        reinterpret_cast<uint4 *>(sW)[i] = __ldg(reinterpret_cast<const uint4 *>(Wt) + i);
+    for (int i = threadIdx.x; i < 9 * CI * CO / 8; i += NW_THREADS) {  // Wt [CI][9][CO] -> [9][CI][WP]
+        const int ci = i / (9 * CO / 8), rem = i - ci * (9 * CO / 8), tap = rem / (CO / 8), cc = rem % (CO / 8);
+        *reinterpret_cast<uint4 *>(sW + (tap * CI + ci) * WP + cc * 8) = __ldg(reinterpret_cast<const uint4 *>(Wt) + i);
+    }
     if (threadIdx.x < CO / 8) reinterpret_cast<uint4 *>(sZ)[threadIdx.x] = make_uint4(0u, 0u, 0u, 0u);
     const int bands = Hg / TH;
     const long long units = (long long)nb * bands;
@@ -244,7 +256,7 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
             const int y = ylo + r;
             const bool in = y >= 0 && y < H;
             const uint4 *src = reinterpret_cast<const uint4 *>(D + ((n * H + (in ? y : 0)) * (long long)W) * CO) + e;
-            cp_async16_cg(dst + 16u * i, src, in ? 16u : 0u);
+            cp_async16_cg(dst + 16u * xswz<CO>(i), src, in ? 16u : 0u);
         }
         cp_async_commit();
     };
@@ -277,16 +289,17 @@ __global__ void __launch_bounds__(NW_THREADS) narrow_dgrad_kernel(const uint16_t
                 const int ty = y0 + ya + 1 - dy, tx = xa + 1 - dx;  // S * (delta pixel) when it exists
                 const int ys = fdiv(ty), xs = fdiv(tx);
                 const bool ok = ys * S == ty && xs * S == tx && ys >= 0 && ys < H && xs >= 0 && xs < W;
-                const uint32_t arow = ok ? sD_a + (uint32_t)(((ys - ylo) * W + xs) * CO) * 2u : sZ_a;
+                const uint32_t c0 = (uint32_t)(((ys - ylo) * W + xs) * (CO / 8));
 #pragma unroll
                 for (int ks = 0; ks < CO / 16; ++ks) {
                     uint32_t a0, a1, a2, a3;
-                    ldsm_x4(arow + (uint32_t)(ks * 16 + kh) * 2u, a0, a1, a2, a3);
+                    ldsm_x4(ok ? sD_a + 16u * xswz<CO>(c0 + (ks * 16 + kh) / 8) : sZ_a + (uint32_t)(ks * 16 + kh) * 2u, a0,
+                            a1, a2, a3);
 #pragma unroll
                     for (int nt = 0; nt < CI / 8; ++nt) {
                         uint32_t b0, b1;
                         const int ci = nt * 8 + (lane & 7), co = ks * 16 + ((lane >> 3) & 1) * 8;
-                        ldsm_x2(sW_a + (uint32_t)((ci * 9 + tap) * CO + co) * 2u, b0, b1);
+                        ldsm_x2(sW_a + (uint32_t)((tap * CI + ci) * WP + co) * 2u, b0, b1);
                         mma_bf16(acc[nt], a0, a1, a2, a3, b0, b1);
                     }
                 }
@@ -329,7 +342,7 @@ static cudaError_t launch_nd(const uint16_t *D, const uint16_t *Wt, float *G, in
                              int num_sms) {
     const int Hg = S * H, Wg = S * W;
     const int TH = std::min(Hg, NW_P / Wg);
-    const size_t smem = (size_t)9 * CI * CO * 2 + 2 * (size_t)(TH / S + 2) * W * CO * 2 + CO * 2;
+    const size_t smem = (size_t)9 * CI * (CO + 8) * 2 + 2 * (size_t)(TH / S + 2) * W * CO * 2 + CO * 2;
     auto kern = narrow_dgrad_kernel<CI, CO, S>;
     static bool attr = false;
     if (!attr) {
