@@ -43,7 +43,7 @@ SK_DEV float nl_lif(float U, float I, float o, float lam, float th) {  // Eq.1, 
 }  // namespace
 
 template <int CIN, int N, int S>
-__global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConvArgs a, int TH) {
+__global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel(const NarrowConvArgs a, int TH) {
     pdl_enter();
     extern __shared__ __align__(16) uint8_t smem[];
     const int Hin = a.Hin, Win = a.Win;
@@ -176,6 +176,22 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
         };
         if (a.restore && epi) emit(0, false);
 
+        // this lane's A-row byte offset in a staging buffer for each tap (or ~0u: the zero padding row) - the
+        // same for every row of the tile, so the bounds checks and address math leave the row loop
+        uint32_t aoff[9];
+        {
+            const int pa = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
+            const int ya = pa / a.W, xa = pa - ya * a.W;
+            const int kh = (lane >> 4) * 8;
+#pragma unroll
+            for (int tap = 0; tap < 9; ++tap) {
+                const int dy = tap / 3, dx = tap % 3;
+                const int xs = S * xa + dx - 1, ys = S * ya + dy;
+                const int yi = S * y0 - 1 + ys;
+                const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
+                aoff[tap] = ok ? 16u * (uint32_t)xswz((ys * Win + xs) * (CIN / 8) + kh / 8) : ~0u;
+            }
+        }
         if (r_mma0 < R) stage(r_mma0, 0);
         int b = 0;
         for (int r = r_mma0; r < R; ++r, b ^= 1) {
@@ -192,22 +208,14 @@ __global__ void __launch_bounds__(NL_THREADS) narrow_lif_kernel(const NarrowConv
 #pragma unroll
                 for (int j = 0; j < N / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
                 const uint32_t xb = sX_a + (uint32_t)(b * XBUF) * 2u;
-                const int pa = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
-                const int ya = pa / a.W, xa = pa - ya * a.W;
-                const int kh = (lane >> 4) * 8;
+                const uint32_t zrow = sZ_a + (uint32_t)((lane >> 4) * 8) * 2u;
+                static_assert(CIN == 16, "one 16-channel K step per tap");
 #pragma unroll
                 for (int tap = 0; tap < 9; ++tap) {
-                    const int dy = tap / 3, dx = tap % 3;
-                    const int xs = S * xa + dx - 1, ys = S * ya + dy;
-                    const int yi = S * y0 - 1 + ys;
-                    const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
-                    const int q = ys * Win + xs;   // staged pixel
 #pragma unroll
                     for (int ks = 0; ks < CIN / 16; ++ks) {
                         uint32_t a0, a1, a2, a3;
-                        const int chunk = q * (CIN / 8) + (ks * 16 + kh) / 8;
-                        const uint32_t aaddr = ok ? xb + 16u * (uint32_t)xswz(chunk) : sZ_a + (uint32_t)kh * 2u;
-                        nl_ldsm_x4(aaddr, a0, a1, a2, a3);
+                        nl_ldsm_x4(aoff[tap] != ~0u ? xb + aoff[tap] : zrow, a0, a1, a2, a3);
 #pragma unroll
                         for (int nt = 0; nt < N / 8; ++nt) {
                             uint32_t b0, b1;
