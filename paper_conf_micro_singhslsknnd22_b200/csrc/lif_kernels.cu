@@ -1048,21 +1048,46 @@ cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *
 }
 
 // ============================================================================ split-K weight-gradient slices
-// dst += sum of the nslices partial weight gradients in slice order (deterministic split-K, STORE_SLICE_ADD /
-// narrow_wgrad), and the slices are zeroed for the next step.  4 elements per thread.
-__global__ void reduce_slices_kernel(float4 *slices, int nslices, float4 *dst, long long count4) {
+// dst += sum of the nslices partial weight gradients (deterministic split-K, STORE_SLICE_ADD / narrow_wgrad),
+// and the slices are zeroed for the next step.  A block owns 32 float4 columns; its 8 warps each sum a fixed
+// contiguous range of the slices (independent loads, in slice order), and warp 0 adds the 8 partials in
+// warp order - a fixed summation tree, so the result does not depend on scheduling.
+__global__ void __launch_bounds__(256) reduce_slices_kernel(float4 *__restrict__ slices, int nslices,
+                                                            float4 *__restrict__ dst, long long count4) {
     pdl_enter();
-    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count4;
-         i += (long long)gridDim.x * blockDim.x) {
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-        for (int s = 0; s < nslices; ++s) {
-            float4 *p = slices + (long long)s * count4 + i;
-            const float4 v = *p;
+    __shared__ float4 part[8][32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const long long i = (long long)blockIdx.x * 32 + lane;
+    const int per = (nslices + 7) / 8, s0 = w * per, s1 = min(nslices, s0 + per);
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (i < count4) {
+        int s = s0;
+        for (; s + 4 <= s1; s += 4) {  // four independent loads in flight, then the ordered adds
+            float4 v[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) v[k] = slices[(long long)(s + k) * count4 + i];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                acc.x += v[k].x; acc.y += v[k].y; acc.z += v[k].z; acc.w += v[k].w;
+                slices[(long long)(s + k) * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+        }
+        for (; s < s1; ++s) {
+            const float4 v = slices[(long long)s * count4 + i];
             acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-            *p = make_float4(0.f, 0.f, 0.f, 0.f);
+            slices[(long long)s * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
+    }
+    part[w][lane] = acc;
+    __syncthreads();
+    if (w == 0 && i < count4) {
+        float4 t = part[0][lane];
+#pragma unroll
+        for (int k = 1; k < 8; ++k) {
+            t.x += part[k][lane].x; t.y += part[k][lane].y; t.z += part[k][lane].z; t.w += part[k][lane].w;
         }
         float4 d = dst[i];
-        d.x += acc.x; d.y += acc.y; d.z += acc.z; d.w += acc.w;
+        d.x += t.x; d.y += t.y; d.z += t.z; d.w += t.w;
         dst[i] = d;
     }
 }
@@ -1072,8 +1097,7 @@ cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t 
         return cudaErrorInvalidValue;
     const long long c4 = (long long)(count / 4);
     if (c4 == 0 || nslices <= 0) return cudaSuccess;
-    const int blocks = (int)std::min<long long>((c4 + 255) / 256, 148LL * 8);
-    sk_launch(reduce_slices_kernel, blocks, 256, 0, s, reinterpret_cast<float4 *>(slices), nslices,
+    sk_launch(reduce_slices_kernel, (unsigned)((c4 + 31) / 32), 256, 0, s, reinterpret_cast<float4 *>(slices), nslices,
               reinterpret_cast<float4 *>(dst), c4);
     return cudaGetLastError();
 }
