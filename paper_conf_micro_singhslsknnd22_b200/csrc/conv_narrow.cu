@@ -338,10 +338,20 @@ __global__ void __launch_bounds__(CN_THREADS, LIF ? (N <= 16 ? 4 : 2) : 1) conv_
                 }
                 if (roff >= 0) {  // I += S(a^r): exact (spikes added to the fp32 sum)
                     const uint16_t *rp = a.res + (long long)r * rrs + roff;
+// 8 channels (16 bytes) per load: res_lo and res_C are multiples of 8 (launch check), so a chunk is
+                    // wholly in or out
 #pragma unroll
-                    for (int c = 0; c < N; ++c) {
-                        const int cs = c - a.res_lo;
-                        if (cs >= 0 && cs < a.res_C) I[c] = __fadd_rn(I[c], bf_bits2f(__ldg(rp + cs)));
+                    for (int c8 = 0; c8 < N; c8 += 8) {
+                        const int cs = c8 - a.res_lo;
+                        if (cs >= 0 && cs < a.res_C) {
+                            const uint4 v = __ldg(reinterpret_cast<const uint4 *>(rp + cs));
+                            const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                I[c8 + 2 * e] = __fadd_rn(I[c8 + 2 * e], __uint_as_float(w[e] << 16));
+                                I[c8 + 2 * e + 1] = __fadd_rn(I[c8 + 2 * e + 1], __uint_as_float(w[e] & 0xffff0000u));
+                            }
+                        }
                     }
                 }
                 uint32_t nb[NW];
@@ -435,7 +445,7 @@ cudaError_t launch_conv_narrow_lif(const NarrowConvArgs &a0, cudaStream_t s, int
     NarrowConvArgs a = a0;
     a.sign = 1;
     if (!conv_narrow_lif_supported(a.Cin, a.Cout, a.stride) || a.R <= 0) return cudaErrorInvalidValue;
-    if (a.res && (a.res_C % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
+    if (a.res && (a.res_C % 8 || a.res_lo % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
     switch (a.Cout) {
         case 16: return launch_n<16, true>(a, s, num_sms);
         case 32: return launch_n<32, true>(a, s, num_sms);

@@ -241,10 +241,20 @@ __global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel
                 for (int c = 0; c < N; ++c) I[c] = sI[threadIdx.x * IP + c];
                 if (roff >= 0) {  // I += S(a^r): exact (spikes added to the fp32 sum)
                     const uint16_t *rp = a.res + (long long)r * rrs + roff;
+// 8 channels (16 bytes) per load: res_lo and res_C are multiples of 8 (launch check), so a chunk is
+                    // wholly in or out
 #pragma unroll
-                    for (int c = 0; c < N; ++c) {
-                        const int cs = c - a.res_lo;
-                        if (cs >= 0 && cs < a.res_C) I[c] = __fadd_rn(I[c], bf_bits2f(__ldg(rp + cs)));
+                    for (int c8 = 0; c8 < N; c8 += 8) {
+                        const int cs = c8 - a.res_lo;
+                        if (cs >= 0 && cs < a.res_C) {
+                            const uint4 v = __ldg(reinterpret_cast<const uint4 *>(rp + cs));
+                            const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                I[c8 + 2 * e] = __fadd_rn(I[c8 + 2 * e], __uint_as_float(w[e] << 16));
+                                I[c8 + 2 * e + 1] = __fadd_rn(I[c8 + 2 * e + 1], __uint_as_float(w[e] & 0xffff0000u));
+                            }
+                        }
                     }
                 }
                 uint32_t nb[NW];
@@ -304,7 +314,7 @@ static cudaError_t launch_nl(const NarrowConvArgs &a, cudaStream_t s, int num_sm
 
 cudaError_t launch_narrow_lif_mma(const NarrowConvArgs &a, cudaStream_t s, int num_sms) {
     if (!narrow_lif_mma_supported(a.Cin, a.Cout, a.stride, a.H, a.W) || a.R <= 0) return cudaErrorInvalidValue;
-    if (a.res && (a.res_C % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
+    if (a.res && (a.res_C % 8 || a.res_lo % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
     if (a.Cout == 16 && a.stride == 1) return launch_nl<16, 16, 1>(a, s, num_sms);
     if (a.Cout == 32 && a.stride == 1) return launch_nl<16, 32, 1>(a, s, num_sms);
     if (a.Cout == 16 && a.stride == 2) return launch_nl<16, 16, 2>(a, s, num_sms);
