@@ -243,17 +243,27 @@ __global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel
                     const uint16_t *rp = a.res + (long long)r * rrs + roff;
 // 8 channels (16 bytes) per load: res_lo and res_C are multiples of 8 (launch check), so a chunk is
                     // wholly in or out
+auto add8 = [&](int c8, const uint4 &v) {
+                        const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                    for (int c8 = 0; c8 < N; c8 += 8) {
-                        const int cs = c8 - a.res_lo;
-                        if (cs >= 0 && cs < a.res_C) {
-                            const uint4 v = __ldg(reinterpret_cast<const uint4 *>(rp + cs));
-                            const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+                        for (int e = 0; e < 4; ++e) {
+                            I[c8 + 2 * e] = __fadd_rn(I[c8 + 2 * e], __uint_as_float(w[e] << 16));
+                            I[c8 + 2 * e + 1] = __fadd_rn(I[c8 + 2 * e + 1], __uint_as_float(w[e] & 0xffff0000u));
+                        }
+                    };
+                    if (a.res_lo == 0 && a.res_C == N && N % 16 == 0) {  // identity shortcut: 32-byte loads (whole sectors)
 #pragma unroll
-                            for (int e = 0; e < 4; ++e) {
-                                I[c8 + 2 * e] = __fadd_rn(I[c8 + 2 * e], __uint_as_float(w[e] << 16));
-                                I[c8 + 2 * e + 1] = __fadd_rn(I[c8 + 2 * e + 1], __uint_as_float(w[e] & 0xffff0000u));
-                            }
+                        for (int c16 = 0; c16 < N; c16 += 16) {
+                            uint4 v0, v1;
+                            ldg_v8u(rp + c16, v0, v1);
+                            add8(c16, v0);
+                            add8(c16 + 8, v1);
+                        }
+                    } else {
+#pragma unroll
+                        for (int c8 = 0; c8 < N; c8 += 8) {
+                            const int cs = c8 - a.res_lo;
+                            if (cs >= 0 && cs < a.res_C) add8(c8, __ldg(reinterpret_cast<const uint4 *>(rp + cs)));
                         }
                     }
                 }
