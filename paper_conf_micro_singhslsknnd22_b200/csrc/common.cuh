@@ -20,6 +20,12 @@ namespace sk {
 // then hold SM resources the side-stream weight-gradient kernels could use.  Without the launch
 // attribute the wait is a no-op.
 SK_DEV void pdl_enter() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// early trigger for small latency-bound kernels (fc scans): lets the dependent launch start its prologue
+SK_DEV void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+#ifndef SK_PDL_EARLY
+#define SK_PDL_EARLY 1
+#endif
+#define sk_pdl_early() (SK_PDL_EARLY)
 
 // 256-bit global store (sm_100: STG.E.256): one full 32-byte sector per lane, so a thread-per-pixel
 // epilogue writing a pixel's channels emits whole sectors instead of half-sector 16-byte pieces.

@@ -272,6 +272,7 @@ __global__ void __launch_bounds__(256, POOL ? 3 : 4) lif_fwd_kernel(const ScanFw
 template <int CH, int SPLIT>
 __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a) {
     pdl_enter();
+    if (sk_pdl_early()) pdl_trigger();
     extern __shared__ unsigned s_cnt[];
     const long long rs = (long long)a.B * a.H * a.W * a.C;
     const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
@@ -494,6 +495,7 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : SK_BWD_MINB) lif_bwd_kernel(c
 template <int CH, int SPLIT>
 __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a) {
     pdl_enter();
+    if (sk_pdl_early()) pdl_trigger();
     const long long rs = (long long)a.B * a.C;
     const long long n = (long long)blockIdx.x * blockDim.x + threadIdx.x;
     if (n >= rs) return;
@@ -535,6 +537,7 @@ __global__ void __launch_bounds__(256) lif_bwd_small_kernel(const ScanBwdArgs a)
 template <int SPLIT, int KIND>
 __global__ void __launch_bounds__(256) lif_bwd_warp_kernel(const ScanBwdArgs a) {
     pdl_enter();
+    if (sk_pdl_early()) pdl_trigger();
     constexpr int NCH = 4, NPW = 32 / NCH;   // row chunks, neurons per warp
     const long long rs = (long long)a.B * a.C;
     const int lane = threadIdx.x & 31, q = lane % NPW, j = lane / NPW;
