@@ -300,14 +300,16 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
         r0 = 1;
     }
     const int lane = threadIdx.x & 31;
-    for (int rb = r0; rb < a.R; rb += CH) {
-        float Iv[CH];
+    // two chunks of CH rows in flight: the loads of chunk k+1 are issued before the recurrence of chunk k
+    auto load = [&](float (&Iv)[CH], int rb) {
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb + j;
             const float *src = a.I + (long long)r * rs + n;
             Iv[j] = (active && r < a.R) ? (SPLIT ? ldg_split(src, a.nsplit, a.split_stride) : __ldg(src)) : 0.f;
         }
+    };
+    auto consume = [&](const float (&Iv)[CH], int rb) {
 #pragma unroll
         for (int j = 0; j < CH; ++j) {
             const int r = rb + j;
@@ -331,6 +333,20 @@ __global__ void __launch_bounds__(256) lif_fwd_small_kernel(const ScanFwdArgs a)
                 if (lane == 0 && v) atomicAdd(&s_cnt[r], v);
             }
             if (a.u2_part) u2_warp_add(a.u2_part, a.row_t ? a.row_t[r] : a.t0 + r, q2);
+        }
+    };
+    {
+        float IA[CH], IB[CH];
+        int rb = r0;
+        if (rb < a.R) load(IA, rb);
+        while (rb < a.R) {
+            if (rb + CH < a.R) load(IB, rb + CH);
+            consume(IA, rb);
+            rb += CH;
+            if (rb >= a.R) break;
+            if (rb + CH < a.R) load(IA, rb + CH);
+            consume(IB, rb);
+            rb += CH;
         }
     }
     if (active) {
@@ -364,7 +380,7 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
         if (a.nsplit > 1)
             sk_launch(lif_fwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         else
-            sk_launch(lif_fwd_small_kernel<16, 0>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
+            sk_launch(lif_fwd_small_kernel<8, 0>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         return cudaGetLastError();
     }
     const long long HW = (long long)a.H * a.W;
