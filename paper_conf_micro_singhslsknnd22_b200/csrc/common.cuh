@@ -83,6 +83,32 @@ SK_DEV void mbar_wait(uint32_t bar, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
+// checkpoint rows of a launch: every ck_every-th row (or row 0 when ck_every = 0) from r0 on, walked
+// with a running cursor instead of a per-row modulo
+struct CkCursor {
+    int next, every;
+    SK_DEV CkCursor(int r0, int ck_every) : every(ck_every) {
+        next = ck_every ? ((r0 + ck_every - 1) / ck_every) * ck_every : (r0 == 0 ? 0 : 0x7fffffff);
+    }
+    // true at a checkpoint row; slot = its index (row / every) and the cursor moves on
+    SK_DEV bool hit(int r, int &slot) {
+        if (r != next) return false;
+        slot = every ? r / every : 0;
+        next = every ? next + every : 0x7fffffff;
+        return true;
+    }
+};
+// mbarrier wait that suspends the waiting thread (up to hint_ns) instead of spinning on try_wait:
+// for waits that are usually long (a producer waiting for a stage the consumers still hold)
+SK_DEV void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "WAITS_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAITS_%=;\n\t}" ::"r"(bar),
+        "r"(parity), "r"(1000000u)
+        : "memory");
+}
 SK_DEV void mbar_arrive(uint32_t bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }

@@ -62,7 +62,7 @@ struct ClCfg {
 };
 
 SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
-    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), o != 0.f ? th : 0.f);  // theta * o, o in {0, 1}: exact select
 }
 
 // PAIR = 1: a cluster of two CTAs on the two SMs of a TPC runs M = 256 MMAs (tcgen05 cta_group::2):
@@ -431,6 +431,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             };
 
             if (a.restore && !(a.diag & 1)) emit(0);
+            CkCursor ck(r_mma0, a.ck_every);
             for (int r = r_mma0; r < a.R; ++r) {
                 CL_T0;
                 mbar_wait(tfull_bar(acc), acc_phase);
@@ -468,8 +469,9 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                 CL_T0;
                 if (!(a.diag & 1)) emit(r);
                 CL_T1(3);
-                if (a.ckU && (a.ck_every ? r % a.ck_every == 0 : r == 0) && valid) {
-                    const long long slot = a.ck_every ? (long long)(r / a.ck_every) * a.ck_stride : 0;
+                int ck_slot;
+                if (ck.hit(r, ck_slot) && a.ckU && valid) {
+                    const long long slot = (long long)ck_slot * a.ck_stride;
                     store_state(a.ckU + slot, a.cko + slot, true);
                 }
             }

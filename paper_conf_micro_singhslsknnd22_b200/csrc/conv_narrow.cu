@@ -48,7 +48,7 @@ SK_DEV uint64_t cn_desc(uint32_t saddr, uint32_t lbo_bytes) {
 }
 
 SK_DEV float cn_lif(float U, float I, float o, float lam, float th) {  // Eq.1, no FMA (oracle order)
-    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), o != 0.f ? th : 0.f);  // theta * o, o in {0, 1}: exact select
 }
 
 // LIF = false: one conv over nb images (R = 1), fp32 output.  LIF = true: the tile is 128 pixels of one

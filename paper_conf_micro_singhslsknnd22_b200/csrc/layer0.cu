@@ -60,8 +60,15 @@ static constexpr uint32_t L0_RING_BYTES = L0_PD * 6 * 128 * 8;  // 6 window chun
 // bit 0 of each byte of w -> 4-bit mask (byte i -> bit i); exact for bytes in {0,1}
 SK_DEV uint32_t byte_bits4(uint32_t w) { return ((w & 0x01010101u) * 0x10204080u) >> 28; }
 
+// bit i of x (i < 8) -> bit 4i
+SK_DEV uint32_t spread_bits_nibbles(uint32_t x) {
+    uint32_t t = (x | (x << 12)) & 0x000F000Fu;
+    t = (t | (t << 6)) & 0x03030303u;
+    return (t | (t << 3)) & 0x11111111u;
+}
+
 SK_DEV float lif_step0(float U, float I, float o, float lam, float th) {
-    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), o != 0.f ? th : 0.f);  // theta * o, o in {0, 1}: exact select
 }
 
 // UMMA descriptor, no swizzle, K-major: 16-byte rows (8 bf16 of K) contiguous within an 8-row core
@@ -320,7 +327,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             if (advance(ptile, pri) && ptile < tiles) fetch_pixel(ptile);
             if (++slot == L0_PD) slot = 0;
             if (advance(tile, ri) && tile < tiles) build_pixel(tile);
-            L0_T1(4); L0_T0; mbar_wait(empty_bar(stage), phase ^ 1u); L0_T1(2); L0_T0;
+            L0_T1(4); L0_T0; mbar_wait_sleep(empty_bar(stage), phase ^ 1u); L0_T1(2); L0_T0;
             uint8_t *dst = sA_ptr + stage * L0_A_BYTES + r * 16;
 #pragma unroll
             for (int j = 0; j < 4; ++j) {  // 8 K columns per 16-byte core-matrix row, via the nibble table
@@ -454,17 +461,16 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                     const uint32_t msk = (1u << PL) - 1u;
                     const uint32_t o8 = (ones >> (sub * PL)) & msk, t8 = (twos >> (sub * PL)) & msk;
                     const uint32_t f8 = (fours >> (sub * PL)) & msk;
+                    // window count n = o + 2t + 4f of channel k as nibble k of sel, then the bf16 of n/4
+                    // ({0, 0x3E80, 0x3F00, 0x3F40, 0x3F80}) by byte permutes of two byte tables
+                    const uint32_t sel = spread_bits_nibbles(o8) | spread_bits_nibbles(t8) << 1 | spread_bits_nibbles(f8) << 2;
 #pragma unroll
-                    for (int e = 0; e < PL / 2; ++e) {
-                        uint32_t v2 = 0;
-#pragma unroll
-                        for (int hh = 0; hh < 2; ++hh) {
-                            const int ch = 2 * e + hh;
-                            const uint32_t n = ((o8 >> ch) & 1u) + 2u * ((t8 >> ch) & 1u) + 4u * ((f8 >> ch) & 1u);
-                            // n/4 is exact in bf16: its bits are the top half of the fp32 bits
-                            v2 |= (__float_as_uint(__uint2float_rn(n) * 0.25f) >> 16) << (16 * hh);
-                        }
-                        pk[e] = v2;
+                    for (int g4 = 0; g4 < PL / 4; ++g4) {
+                        const uint32_t sg = sel >> (16 * g4);
+                        const uint32_t lo = __byte_perm(0x40008000u, 0x00000080u, sg);
+                        const uint32_t hi = __byte_perm(0x3F3F3E00u, 0x0000003Fu, sg);
+                        pk[2 * g4] = __byte_perm(lo, hi, 0x5140);
+                        pk[2 * g4 + 1] = __byte_perm(lo, hi, 0x7362);
                     }
                     if (valid) {
                         uint16_t *po = a.Po_out + (long long)ri * ors + opix * N + c0 + sub * PL;
@@ -501,6 +507,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
 
             if (a.restore) emit(0);
             L0_T1(1);
+            CkCursor ck(r_mma0, a.ck_every);
             for (int ri = r_mma0; ri < a.R; ++ri) {
                 L0_T0; mbar_wait(tfull_bar(acc), acc_phase); L0_T1(5); L0_T0;
                 tc_fence_after();
@@ -526,8 +533,9 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
                 }
                 ob = nb; L0_T1(7); L0_T0;
                 emit(ri); L0_T1(3); L0_T0;
-                if (a.ckU && (a.ck_every ? ri % a.ck_every == 0 : ri == 0) && valid) {
-                    const long long slot = a.ck_every ? (long long)(ri / a.ck_every) * a.ck_stride : 0;
+                int ck_slot;
+                if (ck.hit(ri, ck_slot) && a.ckU && valid) {
+                    const long long slot = (long long)ck_slot * a.ck_stride;
                     store_state(a.ckU + slot, a.cko + slot, true);
                 }
                 L0_T1(2);

@@ -12,7 +12,7 @@
 namespace sk {
 
 SK_DEV float lif_update(float U, float I, float o, float lam, float th) {
-    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), o != 0.f ? th : 0.f);  // theta * o, o in {0, 1}: exact select
 }
 
 // sigma'(U) of reading 4; inv_th = 1 / theta computed once per thread (the reverse scan is issue-bound:

@@ -38,7 +38,7 @@ SK_DEV void nl_mma(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_
         : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
 }
 SK_DEV float nl_lif(float U, float I, float o, float lam, float th) {  // Eq.1, no FMA (oracle order)
-    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), __fmul_rn(th, o));
+    return __fsub_rn(__fadd_rn(__fmul_rn(lam, U), I), o != 0.f ? th : 0.f);  // theta * o, o in {0, 1}: exact select
 }
 }  // namespace
 
