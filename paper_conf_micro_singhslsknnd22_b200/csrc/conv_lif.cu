@@ -79,7 +79,13 @@ SK_DEV float cl_lif(float U, float I, float o, float lam, float th) {
 // loaded together with the weights of the three vertical taps; the three dy taps read the same box at
 // descriptor offsets of dy * W rows (multiples of the 1024-byte swizzle atom).  Activation boxes per
 // row: 3 * Cin/64 instead of 9 * Cin/64 (the kernel is bound by per-SM TMA box processing).
-template <int BN, int POOL, int PAIR, int RESB, int HALO>
+// BWD = 1 / 2 (NEXT-1 backward half, K2 + K4): the same implicit-GEMM mainloop computes the weight-gradient
+// input g^{l-1}_t = conv(delta^l_t, W^l flipped) of a stride-1 3x3 layer (A = delta^l rows, taps shifted as in
+// the forward, weights [Cin][9][Cout] read at the flipped tap 8 - tap), walking the rows DOWNWARDS, and the
+// epilogue runs the reverse surrogate scan of layer l-1 (Eq.2; triangle (1) / fast-sigmoid (2)
+// surrogate) on the accumulator:  delta_t = sigma'(U_t) * g_t + lam * delta_{t+1}  (carry in / out), writing
+// the bf16 delta rows - g never reaches HBM.
+template <int BN, int POOL, int PAIR, int RESB, int HALO, int BWD = 0>
 __global__ void __launch_bounds__(CL_THREADS, 1)
     conv_lif_kernel(const __grid_constant__ CUtensorMap ta, const __grid_constant__ CUtensorMap tb, const ConvLifArgs a) {
     pdl_enter();
@@ -109,9 +115,11 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
     uint32_t *s_spk = reinterpret_cast<uint32_t *>(smem_raw + (spk - raw));
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int r_mma0 = a.restore ? 1 : 0;
+    const int r_mma0 = (!BWD && a.restore) ? 1 : 0;
     const int HW = a.H * a.W;
     const int BHW = a.B * HW;
+    auto row_of = [&](int r) -> int { return BWD ? a.R - 1 - r : r; };  // backward: rows downwards
+    auto wtap = [&](int tap) -> int { return BWD ? 8 - tap : tap; };    // backward: flipped weight taps
     // work decomposition: PAIR -> pair index / rank; unit = (pixel-tile group, channel tile)
     const int rank = PAIR ? (int)cluster_ctarank() : 0;
     const int grp_tiles = PAIR ? a.m_tiles / 2 : a.m_tiles;  // pixel-tile groups per channel tile
@@ -173,7 +181,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                         tma_load_2d_2sm(bres + kb * Cfg::B_BYTES, &tb, bfull_bar, kb * CL_BK, nt * BN + rank * (BN / 2));
                 }
                 for (int r = r_mma0; r < a.R; ++r) {
-                    const long long m0 = (long long)r * BHW + (long long)mt * CL_BM;  // flat input pixel
+                    const long long m0 = (long long)row_of(r) * BHW + (long long)mt * CL_BM;  // flat input pixel
                     const int n0 = (int)(m0 / HW);
                     const int y0 = (int)((m0 % HW) / a.W);
                     for (int kb = 0; kb < steps; ++kb) {
@@ -198,7 +206,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                             if (!RESB) {
 #pragma unroll
                                 for (int dyi = 0; dyi < 3; ++dyi) {
-                                    const int kc = ((dyi * 3 + dxi) * a.conv_cb + hc) * CL_BK;
+                                    const int kc = (wtap(dyi * 3 + dxi) * a.conv_cb + hc) * CL_BK;
                                     if (PAIR)
                                         tma_load_2d_2sm(sa + CL_AH_MAX + dyi * Cfg::B_BYTES, &tb, fb, kc,
                                                         nt * BN + rank * (BN / 2));
@@ -211,7 +219,8 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                             if (rank == 0) mbar_expect_tx(fb, 2 * SBYTES);
                             tma_load_4d_2sm(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
                             if (!RESB)
-                                tma_load_2d_2sm(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN + rank * (BN / 2));
+                                tma_load_2d_2sm(sa + Cfg::A_BYTES, &tb, fb, (wtap(tap) * a.conv_cb + cblk) * CL_BK,
+                                                nt * BN + rank * (BN / 2));
                         } else {
                             mbar_expect_tx(fb, Cfg::STAGE_BYTES);
                             if (a.diag & 8)  // diagnostic: A as a 2D box of the flat [pixels][cin] view
@@ -220,7 +229,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                                 tma_load_4d(sa, &ta, fb, cblk * CL_BK, 0, y0, n0);
                             else
                                 tma_load_4d(sa, &ta, fb, cblk * CL_BK, tap % 3 - 1, y0 + tap / 3 - 1, n0);
-                            tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, kb * CL_BK, nt * BN);
+                            tma_load_2d(sa + Cfg::A_BYTES, &tb, fb, (wtap(tap) * a.conv_cb + cblk) * CL_BK, nt * BN);
                         }
                         if (++stage == STAGES) {
                             stage = 0;
@@ -293,6 +302,98 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     }
                 }
                 if (RESB) tc_commit_2sm_mc(bempty_bar, 3);  // this unit's weights may be replaced
+            }
+        }
+    } else if constexpr (BWD != 0) {
+        // ---------------------------------------------------------------- epilogue: reverse scan (Eq.2)
+        // thread = pixel p of the tile, CW channels; delta of the unit in registers across the rows (the
+        // carry), U of the next row prefetched while this row's accumulator is awaited
+        const int q = warp & 3;
+        const int h = (warp - 2) >> 2;
+        const int p = q * 32 + lane;
+        const long long rs = (long long)BHW * a.Cout;  // neurons per row
+        const float th = a.theta, inv_th = 1.0f / a.theta, lam = a.lam, gam = a.gamma;
+        auto sgm = [&](float u) -> float {  // sigma'(u), reading 4 (as lif_bwd_kernel with gs = 1)
+            if (BWD == 1) return gam * fmaxf(0.0f, 1.0f - fabsf(u - th) * inv_th);
+            const float dd = 1.0f + gam * fabsf(u - th);
+            return __frcp_rn(dd * dd);
+        };
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int it = 0; it < niter; ++it) {
+            int mt, nt;
+            const bool uvalid = unit_tile(it, mt, nt);
+            const int pg = mt * CL_BM + p;
+            const bool valid = uvalid && pg < BHW;
+            const int ch0 = nt * BN + h * CW;
+            const long long nidx = (long long)(valid ? pg : 0) * a.Cout + ch0;
+            float d[CW];
+            auto load8 = [&](const float *src, float *dst) {
+                uint4 x0, x1;
+                ldg_v8u(src, x0, x1);
+                dst[0] = __uint_as_float(x0.x); dst[1] = __uint_as_float(x0.y); dst[2] = __uint_as_float(x0.z);
+                dst[3] = __uint_as_float(x0.w); dst[4] = __uint_as_float(x1.x); dst[5] = __uint_as_float(x1.y);
+                dst[6] = __uint_as_float(x1.z); dst[7] = __uint_as_float(x1.w);
+            };
+#pragma unroll
+            for (int c = 0; c < CW; ++c) d[c] = 0.f;
+            if (valid) {
+#pragma unroll
+                for (int c = 0; c < CW; c += 8) load8(a.bcarry + nidx + c, d + c);
+            }
+            for (int r = 0; r < a.R; ++r) {
+                const int rr = a.R - 1 - r;
+                const float *Ur = a.bU + (long long)rr * rs + nidx;
+                // U of this row, 32 channels at a time: chunk 0 is requested before the accumulator wait
+                float u[32];
+#pragma unroll
+                for (int c = 0; c < 32; ++c) u[c] = 0.f;
+                if (valid) {
+#pragma unroll
+                    for (int c = 0; c < 32; c += 8) load8(Ur + c, u + c);
+                }
+                mbar_wait(tfull_bar(acc), acc_phase);
+                tc_fence_after();
+#pragma unroll
+                for (int j = 0; j < CW / 32; ++j) {
+                    if (j > 0 && valid) {
+#pragma unroll
+                        for (int c = 0; c < 32; c += 8) load8(Ur + 32 * j + c, u + c);
+                    }
+                    uint32_t v[32];
+                    tmem_ld_32x32b_x32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + h * CW + j * 32, v);
+                    tmem_ld_wait();
+#pragma unroll
+                    for (int c = 0; c < 32; ++c)
+                        d[32 * j + c] = __fmaf_rn(sgm(u[c]), __uint_as_float(v[c]), __fmul_rn(lam, d[32 * j + c]));
+                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if (PAIR)
+                        mbar_arrive_leader(tempty_bar(acc));
+                    else
+                        mbar_arrive(tempty_bar(acc));
+                }
+                if (++acc == NACC) {
+                    acc = 0;
+                    acc_phase ^= 1u;
+                }
+                if (valid) {  // bf16 delta, 16 channels (one 32-byte sector) per store
+                    uint16_t *dst = a.bdelta + (long long)rr * rs + nidx;
+#pragma unroll
+                    for (int c = 0; c < CW; c += 16) {
+                        uint32_t pk[8];
+#pragma unroll
+                        for (int e = 0; e < 8; ++e)
+                            pk[e] = (uint32_t)f2bf_bits(d[c + 2 * e]) | ((uint32_t)f2bf_bits(d[c + 2 * e + 1]) << 16);
+                        st_global_v8u(dst + c, make_uint4(pk[0], pk[1], pk[2], pk[3]), make_uint4(pk[4], pk[5], pk[6], pk[7]));
+                    }
+                }
+            }
+            if (valid) {
+#pragma unroll
+                for (int c = 0; c < CW; c += 8) st_global_v8(a.bcarry + nidx + c, d + c);
             }
         }
     } else {
@@ -517,11 +618,11 @@ bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool) {
     return true;
 }
 
-template <int BN, int POOL, int PAIR, int RESB, int HALO>
+template <int BN, int POOL, int PAIR, int RESB, int HALO, int BWD = 0>
 static cudaError_t launch_cl(const CUtensorMap &ta, const CUtensorMap &tb, ConvLifArgs a, cudaStream_t s,
                              int num_sms) {
     using Cfg = ClCfg<BN, PAIR>;
-    auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB, HALO>;
+    auto kern = conv_lif_kernel<BN, POOL, PAIR, RESB, HALO, BWD>;
     uint32_t smem = Cfg::FIXED_BYTES + 4u * (uint32_t)a.R + 16;
     const uint32_t resb = RESB ? (uint32_t)a.num_kb * Cfg::B_BYTES : 0u;
     const uint32_t sbytes = (HALO ? CL_AH_MAX : Cfg::A_BYTES) + (RESB ? 0u : (HALO ? 3u : 1u) * Cfg::B_BYTES);
@@ -625,6 +726,60 @@ cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifA
     if (halo) CL_LAUNCH(128, 0, 0, 1);
     CL_LAUNCH(128, 0, 0, 0);
 #undef CL_LAUNCH
+}
+
+bool conv_lif_bwd_supported(int B, int H, int W, int cin, int cout) {
+    return cout % 64 == 0 && conv_lif_supported(B, H, W, cin, cout, 0);
+}
+
+cudaError_t launch_conv_lif_bwd(const void *D, int rows_in, const void *Wt, ConvLifArgs a, cudaStream_t s, int num_sms) {
+    if (!conv_lif_bwd_supported(a.B, a.H, a.W, a.Cin, a.Cout) || !a.bU || !a.bcarry || !a.bdelta)
+        return cudaErrorInvalidValue;
+    if (a.R <= 0) return cudaSuccess;
+    if (rows_in < a.R) return cudaErrorInvalidValue;
+    // 128-channel tiles (64 channels per epilogue thread: carry + one 32-channel U chunk + accumulator chunk
+    // in registers) halve the activation ingress per MMA against 64-channel tiles (SKIPPER_CLB_BN64=1)
+    const char *e64 = getenv("SKIPPER_CLB_BN64");
+    const int bn = (a.Cout % 128 == 0 && !(e64 && atoi(e64))) ? 128 : 64;
+    const int HW = a.H * a.W;
+    uint32_t bhh, bnn;
+    if (HW >= CL_BM) {
+        bhh = CL_BM / a.W;
+        bnn = 1;
+    } else {
+        bhh = a.H;
+        bnn = CL_BM / HW;
+    }
+    a.pool = 0;
+    a.restore = 0;
+    a.conv_cb = a.Cin / 64;
+    a.num_kb = 9 * a.conv_cb;
+    a.m_tiles = (a.B * HW + CL_BM - 1) / CL_BM;
+    a.n_tiles = a.Cout / bn;
+    a.diag = 0;
+    const bool pair = cl_use_pair(a.m_tiles);
+    const char *he = getenv("SKIPPER_CL_HALO");
+    const bool halo = !(he && atoi(he) == 0) && HW >= CL_BM && a.W >= 8 && a.W <= 32;
+    a.halo_bytes = halo ? (int)((bhh + 2) * (uint32_t)a.W * 128u) : 0;
+    CUtensorMap ta, tb;
+    if (!make_map_conv(&ta, D, a.Cin, a.W, a.H, (uint64_t)rows_in * a.B, a.W, halo ? bhh + 2 : bhh, bnn))
+        return cudaErrorInvalidValue;
+    if (!make_map_2d(&tb, Wt, 9ull * a.Cin, a.Cout, CL_BK, pair ? bn / 2 : bn)) return cudaErrorInvalidValue;
+    const bool tri = a.surr == 0;
+#define CLB_LAUNCH(BN_, PAIR_, HALO_)                                          \
+    return tri ? launch_cl<BN_, 0, PAIR_, 0, HALO_, 1>(ta, tb, a, s, num_sms) \
+               : launch_cl<BN_, 0, PAIR_, 0, HALO_, 2>(ta, tb, a, s, num_sms)
+    if (bn == 128) {
+        if (pair && halo) CLB_LAUNCH(128, 1, 1);
+        if (pair) CLB_LAUNCH(128, 1, 0);
+        if (halo) CLB_LAUNCH(128, 0, 1);
+        CLB_LAUNCH(128, 0, 0);
+    }
+    if (pair && halo) CLB_LAUNCH(64, 1, 1);
+    if (pair) CLB_LAUNCH(64, 1, 0);
+    if (halo) CLB_LAUNCH(64, 0, 1);
+    CLB_LAUNCH(64, 0, 0);
+#undef CLB_LAUNCH
 }
 
 }  // namespace sk

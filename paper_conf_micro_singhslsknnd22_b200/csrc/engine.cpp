@@ -47,10 +47,13 @@ struct Layer {
     float *U_run = nullptr, *ckU = nullptr, *carry = nullptr;
     uint8_t *o_run = nullptr, *cko = nullptr;
     uint16_t *Po = nullptr;    // arena rows
+    uint16_t *PoS[2] = {nullptr, nullptr};  // the two slots of Po (ctx.wdb)
     float *Useg = nullptr;     // arena rows
     int fsplit = 1, dsplit = 1;  // split-K factors of the forward / dgrad GEMMs (fc layers, fixed per layer)
     int fsplitT = 1;             // forward split-K of the chunked first pass (fc tail layers, tail_G*S rows)
     bool cfused = false;         // conv layer: GEMM + LIF scan as one kernel (conv_lif.cu)
+    bool dlif = false;           // this layer's dgrad runs with layer i-1's reverse scan in its epilogue
+                                 // (conv_lif.cu BWD, NEXT-1 backward half): g^{i-1} never reaches HBM
     size_t sbn = 0;              // elements of one running-state / checkpoint slot (B*N, or conv_lif's
                                  // thread-major layout, conv_lif_state_count, when cfused)
     // deterministic split-K weight gradient: wsl > 0 -> the wgrad launches add into slice s of dws
@@ -109,6 +112,14 @@ struct skipper_ctx {
     cudaStream_t st2 = nullptr;
     cudaEvent_t ev_ready[3] = {nullptr, nullptr, nullptr}, ev_done[3] = {nullptr, nullptr, nullptr};
     bool w_pending[3] = {false, false, false};
+    // weight gradients across segment borders (per-segment SKIP / CKPT schedule): the layer outputs and the
+    // layer-0 operand rows - the weight gradients' X operands - alternate between two arena slots by
+    // segment parity, so segment c's weight gradients run on under the recompute of c-1 instead of being
+    // joined before it (the slot is waited for only when segment c-2 reuses it)
+    bool wdb = false;
+    int cur_slot = 0;
+    cudaEvent_t ev_slot[2] = {nullptr, nullptr};
+    bool slot_rec[2] = {false, false};
     int T = 0, C = 1, S = 0, B = 0, Bg = 0;
     int num_sms = 148;
     int in_kind = 0;            // layer-0 operand: 0 fc rows, 1 3x3 im2col rows (K0 cols), 2 NHWC image
@@ -168,6 +179,7 @@ struct skipper_ctx {
     float *dcols = nullptr;                             // icol dgrad output columns (fp32)
     float *cnt_gap = nullptr, *g_gap = nullptr;         // GAP readout input / gradient [B][C]
     uint16_t *xg = nullptr;     // staged layer-0 operand rows of the current pass
+    uint16_t *xgS[2] = {nullptr, nullptr};  // the two slots of xg (wdb)
     // schedule state
     int phase = PH_IDLE;
     int next_seg = 0;
@@ -212,11 +224,12 @@ static double now_ms() {
 
 enum KClass {
     K_STAGE = 0, K_GEMM_FWD, K_SCAN_FWD, K_READOUT, K_SCAN_BWD, K_GEMM_WGRAD, K_GEMM_DGRAD, K_ADAM, K_UNPAD,
-    K_L0_FWD, K_L0_BWD, K_CONV_LIF, K_IM2COL, K_NCLASS
+    K_L0_FWD, K_L0_BWD, K_CONV_LIF, K_IM2COL, K_DGRAD_LIF, K_NCLASS
 };
 static const char *k_class_names[K_NCLASS] = {"stage_input", "gemm_fwd", "lif_fwd_scan", "readout_loss",
                                                "lif_bwd_scan", "gemm_wgrad", "gemm_dgrad", "adam", "unpad",
-                                               "layer0_fused_fwd", "layer0_fused_bwd", "gemm_lif_fwd", "im2col"};
+                                               "layer0_fused_fwd", "layer0_fused_bwd", "gemm_lif_fwd", "im2col",
+                                               "gemm_lif_bwd"};
 
 static cudaEvent_t ev_get(skipper_ctx *c) {
     if (c->ev_used < c->ev_pool.size()) return c->ev_pool[c->ev_used++];
@@ -682,6 +695,13 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     }
     c->S = c->T / c->C;
     c->G = (cfg->mode == SKIPPER_MODE_CKPT || cfg->mode == SKIPPER_MODE_SKIP) ? std::max(1, std::min(cfg->group, c->C)) : 1;
+    {
+        // opt-in (SKIPPER_WGRAD_OVERLAP=1): measured +0.4 % on cfg 2 and -2 % on cfg 3 for one
+        // more copy of the layer outputs - the GPU is saturated, the weight gradients cost SM time wherever they run
+        const char *e = getenv("SKIPPER_WGRAD_OVERLAP");
+        c->wdb = (cfg->mode == SKIPPER_MODE_CKPT || cfg->mode == SKIPPER_MODE_SKIP) && c->G == 1 && c->C > 1 &&
+                 (e && atoi(e));
+    }
     c->num_sms = sk::device_num_sms();
     c->host_prof = getenv("SKIPPER_HOST_PROFILE") && atoi(getenv("SKIPPER_HOST_PROFILE"));
     if (cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking) != cudaSuccess)
@@ -691,6 +711,9 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
     for (int k = 0; k < 3; ++k)
         if (cudaEventCreateWithFlags(&c->ev_ready[k], cudaEventDisableTiming) != cudaSuccess ||
             cudaEventCreateWithFlags(&c->ev_done[k], cudaEventDisableTiming) != cudaSuccess)
+            return bail(fail(c, SKIPPER_ECUDA, "event creation failed"));
+    for (int k = 0; k < 2; ++k)
+        if (cudaEventCreateWithFlags(&c->ev_slot[k], cudaEventDisableTiming) != cudaSuccess)
             return bail(fail(c, SKIPPER_ECUDA, "event creation failed"));
     {
         const Layer &f = c->L[0];
@@ -715,6 +738,21 @@ extern "C" skipper_status skipper_create(const skipper_layer *layers, int n_laye
             const long long units = ((long long)c->B * l.H * l.W + 127) / 128 * (l.Cout == 64 ? 1 : l.Cout / 128);
             l.cfused = l.conv && !l.icol && l.res < 0 && !(e3 && atoi(e3)) && units >= min_units &&
                        sk::conv_lif_supported(c->B, l.H, l.W, l.Cin, l.Cout, l.pool ? 1 : 0);
+        }
+        // dgrad of layer i with layer i-1's reverse scan fused (conv_lif.cu BWD): stride-1 3x3 layer i whose
+        // input is layer i-1's unpooled output, layer i-1 neither a shortcut source nor layer 0's fused
+        // backward; units = (128-pixel tile, 64 channels of C_{i-1}) as the forward's fill rule
+        // opt-in (SKIPPER_BWD_FUSION=1): the fused kernel is faster than the dgrad GEMM + reverse scan it replaces
+        // (cfg 2: 0.45 vs 0.72 ms per step serialised) but the step is not (the backward's
+        // critical path is shared with the side-stream weight gradients)
+        const char *e5 = getenv("SKIPPER_BWD_FUSION");
+        for (int i = 1; i < c->Ls; ++i) {
+            Layer &l = c->L[i];
+            const Layer &pv = c->L[i - 1];
+            const long long units = ((long long)c->B * l.H * l.W + 127) / 128 * (pv.Cout % 128 ? pv.Cout / 64 : pv.Cout / 128);
+            l.dlif = (e5 && atoi(e5)) && l.conv && !l.icol && l.stride == 1 && pv.conv && !pv.icol && !pv.pool &&
+                     pv.res_to < 0 && !(i == 1 && c->l0_bwd_fused) && pv.H == l.H && pv.W == l.W &&
+                     units >= min_units && sk::conv_lif_bwd_supported(c->B, l.H, l.W, l.Cout, l.Cin);
         }
     }
     for (int i = 0; i < c->Ls; ++i) {
@@ -951,6 +989,8 @@ extern "C" void skipper_destroy(skipper_ctx *c) {
         if (c->ev_ready[k]) cudaEventDestroy(c->ev_ready[k]);
         if (c->ev_done[k]) cudaEventDestroy(c->ev_done[k]);
     }
+    for (int k = 0; k < 2; ++k)
+        if (c->ev_slot[k]) cudaEventDestroy(c->ev_slot[k]);
     if (c->st3) {
         cudaStreamSynchronize(c->st3);
         cudaStreamDestroy(c->st3);
@@ -1039,9 +1079,12 @@ static skipper_status arena_free(skipper_ctx *c) {
     c->arena = nullptr;
     c->arena_bytes = 0;
     for (auto &l : c->L) {
-        l.Po = nullptr;
+        l.Po = l.PoS[0] = l.PoS[1] = nullptr;
         l.Useg = nullptr;
     }
+    c->xgS[0] = c->xgS[1] = nullptr;
+    c->slot_rec[0] = c->slot_rec[1] = false;
+    c->cur_slot = 0;
     c->I_buf = nullptr;
     c->d_buf = nullptr;
     for (int k = 0; k < 3; ++k) c->d_buf2[k] = c->P2[k] = c->cols[k] = nullptr;
@@ -1083,21 +1126,25 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     arena_free(c);
     const size_t rowsB = (size_t)R * c->B;
     size_t bytes = 0;
-    for (int i = 0; i < c->Ls; ++i) bytes += al256(rowsB * c->L[i].Nout * 2) + al256(rowsB * c->L[i].N * 4);
+    const int nslot = c->wdb ? 2 : 1;
+    for (int i = 0; i < c->Ls; ++i) bytes += nslot * al256(rowsB * c->L[i].Nout * 2) + al256(rowsB * c->L[i].N * 4);
     const size_t ibytes = al256(rowsB * max_gemm_io(c) * 4);
     const size_t dbytes = al256(rowsB * max_n(c) * 2);
     const size_t xbytes = al256(rowsB * c->in_row * 2);
     const long long ch = std::min<long long>(rowsB, icol_chunk(c));
     const size_t cbytes = al256(ch * max_icol(c) * 2), dcbytes = al256(ch * max_icol(c) * 4);
-    bytes += ibytes + c->nD * (dbytes + cbytes) + xbytes + dcbytes;
+    bytes += ibytes + c->nD * (dbytes + cbytes) + nslot * xbytes + dcbytes;
     c->arena_bytes = bytes;
     c->arena = dev_alloc(c, bytes);
     if (!c->arena) return fail(c, SKIPPER_ENOMEM, "segment arena of %zu bytes (%d rows)", bytes, R);
     char *p = static_cast<char *>(c->arena);
     for (int i = 0; i < c->Ls; ++i) {
         Layer &l = c->L[i];
-        l.Po = reinterpret_cast<uint16_t *>(p);
-        p += al256(rowsB * l.Nout * 2);
+        for (int k = 0; k < nslot; ++k) {
+            l.PoS[k] = reinterpret_cast<uint16_t *>(p);
+            p += al256(rowsB * l.Nout * 2);
+        }
+        l.Po = l.PoS[0];
         l.Useg = reinterpret_cast<float *>(p);
         p += al256(rowsB * l.N * 4);
     }
@@ -1106,8 +1153,11 @@ static skipper_status arena_rows(skipper_ctx *c, int R) {
     c->d_buf = reinterpret_cast<uint16_t *>(p);
     for (int k = 0; k < c->nD; ++k) c->d_buf2[k] = reinterpret_cast<uint16_t *>(p + k * dbytes);
     p += c->nD * dbytes;
-    c->xg = reinterpret_cast<uint16_t *>(p);
-    p += xbytes;
+    for (int k = 0; k < nslot; ++k) {
+        c->xgS[k] = reinterpret_cast<uint16_t *>(p);
+        p += xbytes;
+    }
+    c->xg = c->xgS[0];
     for (int k = 0; k < c->nD; ++k) c->cols[k] = cbytes ? reinterpret_cast<uint16_t *>(p + k * cbytes) : nullptr;
     p += c->nD * cbytes;
     c->dcols = dcbytes ? reinterpret_cast<float *>(p) : nullptr;
@@ -1132,6 +1182,10 @@ static skipper_status run_gemm(skipper_ctx *c, const sk::GemmLaunch &g, bool ok,
                                int cls, double bytes, double flops, cudaStream_t s = nullptr) {
     if (!ok) return fail(c, SKIPPER_EUNSUPPORTED, "layer %d: cannot plan %s GEMM (tensor map)", layer, what);
     if (!s) s = c->st;
+    // timing experiment only (gradients are wrong when set): SKIPPER_DIAG_NO_WGRAD=1 skips the weight-gradient
+    // GEMMs, to measure how much of the step they hold on the critical path
+    static const bool no_wgrad = getenv("SKIPPER_DIAG_NO_WGRAD") && atoi(getenv("SKIPPER_DIAG_NO_WGRAD"));
+    if (no_wgrad && cls == K_GEMM_WGRAD) return SKIPPER_OK;
     ProfScope ps(c, cls, bytes, flops, s);
     CK(sk::gemm_run(g, s, c->num_sms));
     return SKIPPER_OK;
@@ -1663,7 +1717,21 @@ static skipper_status recompute_segment_rows(skipper_ctx *c, int seg);
 
 // RECOMPUTE of segment seg into rows seg_off[seg].. of its group's arena: the per-layer arena bases (stored
 // membranes, layer outputs, layer-0 operand rows) are shifted for the duration of the segment
+// ctx.wdb: point the layer outputs and the layer-0 operand rows at segment seg's slot
+static void select_slot(skipper_ctx *c, int seg) {
+    if (!c->wdb || !c->xgS[1]) return;
+    const int s = seg & 1;
+    for (auto &l : c->L) l.Po = l.PoS[s];
+    c->xg = c->xgS[s];
+    c->cur_slot = s;
+}
+
 static skipper_status recompute_segment(skipper_ctx *c, int seg) {
+    if (c->wdb && c->xgS[1]) {
+        select_slot(c, seg);
+        // the weight gradients of segment seg + 2 read this slot's X operands
+        if (c->slot_rec[c->cur_slot]) CK(cudaStreamWaitEvent(c->st, c->ev_slot[c->cur_slot], 0));
+    }
     const size_t off = c->G > 1 ? (size_t)c->seg_off[seg] : 0;
     if (!off) return recompute_segment_rows(c, seg);
     for (auto &l : c->L) {
@@ -1854,7 +1922,7 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             a.res_stride = l.H / rcv.H;
             a.res_lo = (rcv.Cout - l.Cout) / 2;
         }
-        {
+        if (!(i + 1 < c->Ls && c->L[i + 1].dlif)) {  // else delta_i came from layer i+1's fused dgrad
             double bytes = scan_bwd_bytes(c, l, a);
             if (a.res_delta) bytes += (double)R * c->B * rcv_neurons(c, l.res_to) * 2;
             ProfScope ps(c, K_SCAN_BWD, bytes, 0);
@@ -1938,7 +2006,32 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             c->w_pending[par] = true;
             if (last_seg) CKS(comm_after_wgrad(c, i, c->st2));
         }
-        if (i > 0 && l.icol && l.dgrad_g) {  // stride 1: g = conv(delta, flipped W^T), cp.async gather kernel
+        if (i > 0 && l.dlif) {  // g^{i-1} = conv(delta_i, flipped W_i) and layer i-1's reverse scan in one kernel
+            Layer &pv = c->L[i - 1];
+            const int ppar = (i - 1) % c->nD;
+            if (c->w_pending[ppar]) {  // the wgrad of layer i+1 may still read layer i-1's delta buffer
+                CK(cudaStreamWaitEvent(c->st, c->ev_done[ppar], 0));
+                c->w_pending[ppar] = false;
+            }
+            sk::ConvLifArgs b{};
+            b.B = c->B;
+            b.H = l.H;
+            b.W = l.W;
+            b.Cin = l.Cout;
+            b.Cout = l.Cin;
+            b.R = R;
+            b.lam = pv.d.lambda;
+            b.theta = pv.d.theta;
+            b.bU = pv.Useg;
+            b.bcarry = pv.carry;
+            b.bdelta = c->d_buf2[ppar];
+            b.surr = c->cfg.surrogate;
+            b.gamma = c->cfg.surr_gamma;
+            const double M = (double)nb * l.H * l.W;
+            ProfScope ps(c, K_DGRAD_LIF, (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * pv.N * (4 + 2) +
+                         (double)c->B * pv.N * 8, 2.0 * M * l.Cin * 9 * l.Cout);
+            CK(sk::launch_conv_lif_bwd(dcur, R, l.wt, b, c->st, c->num_sms));
+        } else if (i > 0 && l.icol && l.dgrad_g) {  // stride 1: g = conv(delta, flipped W^T), cp.async gather kernel
             const double M = (double)nb * l.H * l.W;
             ProfScope ps(c, K_GEMM_DGRAD, (double)nb * l.N * 2 + (double)l.wcount * 2 + (double)nb * l.Nin * 4,
                          2.0 * M * l.Cin * 9 * l.Cout);
@@ -1992,7 +2085,14 @@ static skipper_status backward_rows(skipper_ctx *c, int R, const int *row_t, boo
             CKS(run_gemm(c, g, ok, "dgrad", i, K_GEMM_DGRAD, bytes, 2.0 * M * l.Cin * K));
         }
     }
-    // the next segment reuses the arena (X operands, delta buffers): wait for the weight gradients
+    // the next segment reuses the arena (X operands, delta buffers): wait for the weight gradients - or, with
+    // the two X slots (ctx.wdb), only mark this slot busy until they finish (the delta buffers keep their
+    // per-buffer w_pending waits)
+    if (c->wdb && c->xgS[1] && !last_seg && !c->prof_on) {
+        CK(cudaEventRecord(c->ev_slot[c->cur_slot], c->st2));
+        c->slot_rec[c->cur_slot] = true;
+        return SKIPPER_OK;
+    }
     return join_wgrads(c);
 }
 
@@ -2155,6 +2255,7 @@ extern "C" skipper_status skipper_backward_segment(skipper_ctx *c, int seg) {
         c->next_seg = seg - 1;
         return SKIPPER_OK;
     }
+    select_slot(c, seg);
     const int R = full ? c->T : c->G > 1 ? c->grp_R[seg] : (int)c->kept[seg].size();
     const int *row_t = full ? nullptr : c->G > 1 ? c->grp_dev + c->grp_start[seg] : c->kept_dev + (size_t)seg * c->S;
     CKS(backward_rows(c, R, row_t, seg == 0));

@@ -161,11 +161,25 @@ struct ConvLifArgs {
     int stages;      // smem ring depth
     int halo_bytes;  // bytes of one halo activation box (HALO variant)
     int diag;  // SKIPPER_CL_DIAG timing experiments: 1 = no epilogue work, 2 = no MMA
+    // backward (launch_conv_lif_bwd): U rows [R][B][H][W][Cout] fp32 of the layer whose delta is computed,
+    // its carry [B][H][W][Cout] (delta after the last row in, delta at row 0 out), the bf16 delta rows out,
+    // surrogate kind (SURR_*) and gamma
+    const float *bU;
+    float *bcarry;
+    uint16_t *bdelta;
+    int surr;
+    float gamma;
 };
 bool conv_lif_supported(int B, int H, int W, int cin, int cout, int pool);
 // elements of one state / checkpoint slot in the thread-major layout (>= B*H*W*Cout: whole 128-pixel tiles)
 long long conv_lif_state_count(int B, int H, int W, int cout);
 cudaError_t launch_conv_lif(const void *X, int rows_in, const void *Wk, ConvLifArgs a, cudaStream_t s, int num_sms);
+// NEXT-1 backward half (K2 + K4 fused): for a stride-1 3x3 layer l with Cin = C_l (the delta operand's
+// channels) and Cout = C_{l-1} (multiple of 64), g = conv(delta^l, W^l flipped) with the reverse scan of layer l-1
+// in the epilogue.  D: delta^l rows [rows_in][B][H][W][Cin] bf16 (row r = kept row r), Wt: W^l as
+// [Cout][9][Cin] bf16 (the dgrad layout [C_{l-1}][3][3][C_l]); writes a.bdelta rows and a.bcarry.
+bool conv_lif_bwd_supported(int B, int H, int W, int cin, int cout);
+cudaError_t launch_conv_lif_bwd(const void *D, int rows_in, const void *Wt, ConvLifArgs a, cudaStream_t s, int num_sms);
 
 int device_num_sms();
 

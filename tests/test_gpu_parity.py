@@ -191,6 +191,49 @@ def test_vgg5_reduced(mode):
     check_parity("vgg5", T=14, B=2, C=2, p=40.0, mode=mode)
 
 
+@pytest.mark.parametrize("name,T,B,mode,surrogate,gamma,pair,halo", [
+    ("vgg5", 14, 3, "skip", "triangle", 0.3, "1", "1"), ("vgg5", 14, 3, "full", "fast_sigmoid", 1.0, "0", "1"),
+    ("vgg5", 14, 3, "skip", "triangle", 0.3, "0", "0"), ("vgg5", 14, 2, "ckpt", "triangle", 0.3, "1", "0"),
+    ("tiny_conv", 12, 3, "skip", "fast_sigmoid", 2.0, "1", "1"), ("vgg11", 24, 8, "skip", "triangle", 0.3, "1", "1")])
+def test_fused_dgrad_reverse_scan(name, T, B, mode, surrogate, gamma, pair, halo, monkeypatch):
+    """NEXT-1 backward half (conv_lif.cu BWD): the dgrad of a stride-1 conv layer with the previous layer's
+    reverse surrogate scan (Eq.2) in its epilogue, forced on at reduced sizes (SKIPPER_CL_MIN_UNITS=0) for
+    the CTA-pair / single-CTA and halo / per-tap producer variants and both surrogates (opt-in,
+    SKIPPER_BWD_FUSION=1); the step matches the oracle and the fused class really ran."""
+    monkeypatch.setenv("SKIPPER_BWD_FUSION", "1")
+    monkeypatch.setenv("SKIPPER_CL_MIN_UNITS", "0")
+    monkeypatch.setenv("SKIPPER_CL_PAIR", pair)
+    monkeypatch.setenv("SKIPPER_CL_HALO", halo)
+    check_parity(name, T=T, B=B, C=2, p=40.0, mode=mode, surrogate=surrogate, gamma=gamma)
+    from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    net = synth.net_config(name)
+    x, y = synth.make_inputs(net, T, B, seed=1)
+    m = SkipperNet(net, T, C=2, p=40.0, mode=mode, batch=B, surrogate=surrogate, gamma=gamma)
+    m.set_weights(synth.make_weights(net, seed=0))
+    m.profile(True)
+    m.step(torch.from_numpy(np.ascontiguousarray(x)).cuda(), torch.from_numpy(np.ascontiguousarray(y)).cuda())
+    assert m.profile_read()["gemm_lif_bwd"]["launches"] > 0
+
+
+@pytest.mark.parametrize("pair", ["0", "1"])
+def test_fused_dgrad_reverse_scan_bn64(pair, monkeypatch):
+    """The 64-channel-tile variant of the fused dgrad + reverse scan (SKIPPER_CLB_BN64=1)."""
+    monkeypatch.setenv("SKIPPER_BWD_FUSION", "1")
+    monkeypatch.setenv("SKIPPER_CL_MIN_UNITS", "0")
+    monkeypatch.setenv("SKIPPER_CLB_BN64", "1")
+    monkeypatch.setenv("SKIPPER_CL_PAIR", pair)
+    check_parity("vgg5", T=14, B=3, C=2, p=40.0, mode="skip")
+
+
+@pytest.mark.parametrize("name,T,B,C,mode", [("vgg5", 14, 3, 2, "skip"), ("tiny_conv", 24, 3, 4, "ckpt"),
+                                              ("tiny_resnet", 24, 2, 3, "skip"), ("tiny_fc", 24, 3, 6, "skip")])
+def test_wgrad_overlap_slots(name, T, B, C, mode, monkeypatch):
+    """SKIPPER_WGRAD_OVERLAP=1: the weight gradients' X operands alternate between two arena slots by
+    segment parity and are no longer joined at each segment border - same gradients as the oracle."""
+    monkeypatch.setenv("SKIPPER_WGRAD_OVERLAP", "1")
+    check_parity(name, T=T, B=B, C=C, p=40.0, mode=mode)
+
+
 @pytest.mark.parametrize("env", ["SKIPPER_L0_BWD_FUSION", "SKIPPER_NO_L0_FUSION"])
 def test_vgg5_layer0_variants(env, monkeypatch):
     """The alternative first-layer paths (fused reverse scan + wgrad; unfused im2col GEMM) agree too."""
