@@ -535,7 +535,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
             CkCursor ck(r_mma0, a.ck_every);
             for (int r = r_mma0; r < a.R; ++r) {
                 CL_T0;
-                mbar_wait(tfull_bar(acc), acc_phase);
+                mbar_wait_sleep(tfull_bar(acc), acc_phase);
                 CL_T1(1);
                 CL_T0;
                 tc_fence_after();

@@ -365,8 +365,8 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             uint32_t acc_phase = 0;
             for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
                 for (int ri = r_mma0; ri < a.R; ++ri) {
-                    L0_T0; mbar_wait(tempty_bar(acc), acc_phase ^ 1u); L0_T1(3);
-                    L0_T0; mbar_wait(full_bar(stage), phase); L0_T1(4);
+                    L0_T0; mbar_wait_sleep(tempty_bar(acc), acc_phase ^ 1u); L0_T1(3);
+                    L0_T0; mbar_wait_sleep(full_bar(stage), phase); L0_T1(4);
                     tc_fence_after();
                     const uint32_t a0 = sA + stage * L0_A_BYTES;
 #pragma unroll
@@ -509,7 +509,7 @@ __global__ void __launch_bounds__(32 * (F0_EPI_WARP0 + 4 * NCH * 32 / CW), 1)
             L0_T1(1);
             CkCursor ck(r_mma0, a.ck_every);
             for (int ri = r_mma0; ri < a.R; ++ri) {
-                L0_T0; mbar_wait(tfull_bar(acc), acc_phase); L0_T1(5); L0_T0;
+                L0_T0; mbar_wait_sleep(tfull_bar(acc), acc_phase); L0_T1(5); L0_T0;
                 tc_fence_after();
                 uint32_t r[CW];
                 if constexpr (CW == 32)

@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel
 
         // this lane's A-row byte offset in a staging buffer for each tap (or ~0u: the zero padding row) - the
         // same for every row of the tile, so the bounds checks and address math leave the row loop
-        uint32_t aoff[9];
+        uint32_t aoff[9][CIN / 16];
         {
             const int pa = warp * 16 + (lane & 7) + ((lane >> 3) & 1) * 8;
             const int ya = pa / a.W, xa = pa - ya * a.W;
@@ -189,7 +189,9 @@ __global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel
                 const int xs = S * xa + dx - 1, ys = S * ya + dy;
                 const int yi = S * y0 - 1 + ys;
                 const bool ok = xs >= 0 && xs < Win && yi >= 0 && yi < Hin;
-                aoff[tap] = ok ? 16u * (uint32_t)xswz((ys * Win + xs) * (CIN / 8) + kh / 8) : ~0u;
+#pragma unroll
+                for (int ks = 0; ks < CIN / 16; ++ks)  // K step ks = channels 16 ks .. 16 ks + 15 (chunks 2 ks, 2 ks + 1)
+                    aoff[tap][ks] = ok ? 16u * (uint32_t)xswz((ys * Win + xs) * (CIN / 8) + 2 * ks + kh / 8) : ~0u;
             }
         }
         if (r_mma0 < R) stage(r_mma0, 0);
@@ -209,13 +211,13 @@ __global__ void __launch_bounds__(NL_THREADS, N == 16 ? 3 : 2) narrow_lif_kernel
                 for (int j = 0; j < N / 8; ++j) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
                 const uint32_t xb = sX_a + (uint32_t)(b * XBUF) * 2u;
                 const uint32_t zrow = sZ_a + (uint32_t)((lane >> 4) * 8) * 2u;
-                static_assert(CIN == 16, "one 16-channel K step per tap");
+                static_assert(CIN == 16 || CIN == 32, "16-channel K steps per tap");
 #pragma unroll
                 for (int tap = 0; tap < 9; ++tap) {
 #pragma unroll
                     for (int ks = 0; ks < CIN / 16; ++ks) {
                         uint32_t a0, a1, a2, a3;
-                        nl_ldsm_x4(aoff[tap] != ~0u ? xb + aoff[tap] : zrow, a0, a1, a2, a3);
+                        nl_ldsm_x4(aoff[tap][ks] != ~0u ? xb + aoff[tap][ks] : zrow, a0, a1, a2, a3);
 #pragma unroll
                         for (int nt = 0; nt < N / 8; ++nt) {
                             uint32_t b0, b1;
@@ -290,8 +292,13 @@ auto add8 = [&](int c8, const uint4 &v) {
 }
 
 bool narrow_lif_mma_supported(int cin, int cout, int stride, int H, int W) {
-    // 32 -> 32 measured slower here than conv_narrow.cu (128 registers: 2 CTAs per SM); it stays there
-    if (!(cin == 16 && (cout == 16 || cout == 32) && (stride == 1 || stride == 2))) return false;
+    // 32 -> 32 (stride 1): two 16-channel K steps per tap; with the conflict-free staging it beats
+    // conv_narrow.cu's tcgen05 gather kernel (cfg 4 SKIP 428.7 -> 444.7 samples/s; round 1, before the
+    // swizzled staging, it measured slower).  SKIPPER_NO_NL32=1 restores the gather kernel.
+    const char *e = getenv("SKIPPER_NO_NL32");  // read per call so tests can cover both paths in one process
+    const bool nl32 = !(e && atoi(e));
+    const bool c32 = nl32 && cin == 32 && cout == 32 && stride == 1;
+    if (!(c32 || (cin == 16 && (cout == 16 || cout == 32) && (stride == 1 || stride == 2)))) return false;
     if (W > NL_P || NL_P % W || W % 16) return false;
     const int TH = NL_P / W;
     return H % TH == 0 && TH <= H;
@@ -325,6 +332,7 @@ static cudaError_t launch_nl(const NarrowConvArgs &a, cudaStream_t s, int num_sm
 cudaError_t launch_narrow_lif_mma(const NarrowConvArgs &a, cudaStream_t s, int num_sms) {
     if (!narrow_lif_mma_supported(a.Cin, a.Cout, a.stride, a.H, a.W) || a.R <= 0) return cudaErrorInvalidValue;
     if (a.res && (a.res_C % 8 || a.res_lo % 8 || a.res_lo < 0 || a.res_lo + a.res_C > a.Cout)) return cudaErrorInvalidValue;
+    if (a.Cin == 32) return launch_nl<32, 32, 1>(a, s, num_sms);
     if (a.Cout == 16 && a.stride == 1) return launch_nl<16, 16, 1>(a, s, num_sms);
     if (a.Cout == 32 && a.stride == 1) return launch_nl<16, 32, 1>(a, s, num_sms);
     if (a.Cout == 16 && a.stride == 2) return launch_nl<16, 16, 2>(a, s, num_sms);

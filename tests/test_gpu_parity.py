@@ -379,6 +379,13 @@ def test_resnet20_dvs_reduced(mode):
     check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode=mode, deep=True)
 
 
+def test_resnet20_dvs_gather_lif_32(monkeypatch):
+    """SKIPPER_NO_NL32=1: the 32 -> 32 ResNet layers' fused conv + LIF on the tcgen05 gather kernel
+    (conv_narrow.cu) instead of the default warp-level MMA kernel (narrow_lif.cu, two 16-channel K steps)."""
+    monkeypatch.setenv("SKIPPER_NO_NL32", "1")
+    check_parity("resnet20_dvs", T=44, B=1, C=2, p=50.0, mode="skip", deep=True)
+
+
 @pytest.mark.parametrize("name,T,C", [("vgg5", 14, 2), ("tiny_resnet", 16, 2)])
 def test_one_rank_nccl_bucketed_allreduce(name, T, C, monkeypatch):
     """K5 on the device: with a (one-rank) NCCL communicator the s allreduce and the bucketed dW
