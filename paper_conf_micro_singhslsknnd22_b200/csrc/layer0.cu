@@ -601,8 +601,11 @@ cudaError_t launch_layer0_fwd(const L0FwdArgs &a, cudaStream_t s, int num_sms) {
     if (smem > 200 * 1024) return cudaErrorInvalidValue;
     const int grid = tiles < num_sms ? tiles : num_sms;
     if (a.W * a.C0 % 8) return cudaErrorInvalidValue;
-    // epilogue warps own 32 channels each (fewer, longer warps measured faster than 16-channel ones)
-    static const bool cw32 = !(getenv("SKIPPER_L0_CW16") && atoi(getenv("SKIPPER_L0_CW16")));
+    // epilogue warps own 16 channels each (16 epilogue warps): with the byte-permute pooling the per-warp fixed
+    // cost dropped and the extra warps hide more latency (cfg 2 step 6.008 -> 5.981 ms in alternating runs;
+    // before it, 32-channel warps measured faster).  SKIPPER_L0_CW32=1 selects 32-channel warps.
+    const char *ecw = getenv("SKIPPER_L0_CW32");  // read per launch so tests can cover both variants
+    const bool cw32 = ecw && atoi(ecw);
     if (a.N == 64 && cw32) {
         static bool set = false;
         if (!set) {

@@ -215,6 +215,17 @@ def test_fused_dgrad_reverse_scan(name, T, B, mode, surrogate, gamma, pair, halo
     assert m.profile_read()["gemm_lif_bwd"]["launches"] > 0
 
 
+def test_fused_dgrad_reverse_scan_single_row_segments(monkeypatch):
+    """The fused dgrad + reverse scan on segments shrunk to K_c = 1 (one kept row per segment: the kernel's
+    row walk is the carry in, one row, the carry out)."""
+    monkeypatch.setenv("SKIPPER_BWD_FUSION", "1")
+    monkeypatch.setenv("SKIPPER_CL_MIN_UNITS", "0")
+    T, C = 24, 2
+    S = T // C
+    fn = lambda x: np.where((np.arange(x.shape[0]) % S == 0).reshape((-1,) + (1,) * (x.ndim - 1)), x, 0)  # noqa: E731
+    check_parity("vgg5", T=T, B=2, C=C, p=95.0, mode="skip", x_fn=fn)
+
+
 @pytest.mark.parametrize("pair", ["0", "1"])
 def test_fused_dgrad_reverse_scan_bn64(pair, monkeypatch):
     """The 64-channel-tile variant of the fused dgrad + reverse scan (SKIPPER_CLB_BN64=1)."""
@@ -234,7 +245,7 @@ def test_wgrad_overlap_slots(name, T, B, C, mode, monkeypatch):
     check_parity(name, T=T, B=B, C=C, p=40.0, mode=mode)
 
 
-@pytest.mark.parametrize("env", ["SKIPPER_L0_BWD_FUSION", "SKIPPER_NO_L0_FUSION"])
+@pytest.mark.parametrize("env", ["SKIPPER_L0_BWD_FUSION", "SKIPPER_NO_L0_FUSION", "SKIPPER_L0_CW32"])
 def test_vgg5_layer0_variants(env, monkeypatch):
     """The alternative first-layer paths (fused reverse scan + wgrad; unfused im2col GEMM) agree too."""
     monkeypatch.setenv(env, "1")
@@ -555,9 +566,13 @@ def test_full_size_vgg11_forward():
     m.close()
 
 
-@pytest.mark.parametrize("name,T,C,mode", [("cfg2_vgg5", 0, 0, "skip"), ("cfg2_vgg5", 0, 0, "full"),
-                                           ("cfg3_vgg11", 24, 2, "skip"), ("cfg4_resnet_dvs", 0, 0, "skip")])
-def test_full_size_backward_parity(name, T, C, mode):
+@pytest.mark.parametrize("name,T,C,mode,env", [
+    ("cfg2_vgg5", 0, 0, "skip", None), ("cfg2_vgg5", 0, 0, "full", None), ("cfg3_vgg11", 24, 2, "skip", None),
+    ("cfg4_resnet_dvs", 0, 0, "skip", None),
+    # the opt-in round-2 paths at full size: fused dgrad + reverse scan, two X-operand slots
+    ("cfg2_vgg5", 0, 0, "skip", "SKIPPER_BWD_FUSION"), ("cfg3_vgg11", 24, 2, "skip", "SKIPPER_BWD_FUSION"),
+    ("cfg2_vgg5", 0, 0, "skip", "SKIPPER_WGRAD_OVERLAP")])
+def test_full_size_backward_parity(name, T, C, mode, env, monkeypatch):
     """Weight gradients at the BASELINE.json batch sizes in bench.py's launch configuration (no debug
     recording): cfg 2 at full size (T=100, B=64, C=10, p=40), cfg 3 at its full batch B=128 (the batch decides
     the kernel paths: fused conv+LIF, split-K counts of the fc GEMMs) with T=24, C=2, and cfg 4 at full size
@@ -566,6 +581,8 @@ def test_full_size_backward_parity(name, T, C, mode):
     from _oracle_pool import full_batch_forward, full_batch_train
     from oracle.skipper import keep_mask
     from paper_conf_micro_singhslsknnd22_b200 import SkipperNet
+    if env:
+        monkeypatch.setenv(env, "1")
     wl = synth.workload(name)
     if T:
         wl["T"], wl["C"] = T, C
