@@ -1290,6 +1290,19 @@ static skipper_status begin_step(skipper_ctx *c, const unsigned char *x) {
             }
     }
     if (c->L[0].dwp) CKS(zero_dev(c, c->L[0].dwp, (size_t)c->L[0].Cout * c->K0 * 4));
+    // the split-K weight-gradient slices the previous step summed: cleared on the weight-gradient stream, in
+    // order after that step's reduction and before this step's first weight gradient, while the first pass
+    // runs on the main stream (the reduction at the end of the step, on the critical path, only reads them)
+    {
+        cudaStream_t ws = c->prof_on ? c->st : c->st2;
+        if (ws != c->st) {  // after everything the previous step issued on the main stream (its reduction
+                            // ran there when it was profiled)
+            CK(cudaEventRecord(c->ev_ready[0], c->st));
+            CK(cudaStreamWaitEvent(ws, c->ev_ready[0], 0));
+        }
+        for (auto &l : c->L)
+            if (l.dws) CK(cudaMemsetAsync(l.dws, 0, (size_t)l.wsl * l.wg_count * 4, ws));
+    }
     c->x_cur = x;
     c->grads_ready = false;
     return SKIPPER_OK;
@@ -1856,8 +1869,8 @@ static skipper_status reduce_wslices(skipper_ctx *c, int i, cudaStream_t ws) {
     Layer &l = c->L[i];
     if (!l.dws) return SKIPPER_OK;
     float *dst = (i == 0 && l.dwp) ? l.dwp : l.dw;
-    ProfScope ps(c, K_GEMM_WGRAD, (double)l.wsl * l.wg_count * 8 + (double)l.wg_count * 8, 0, ws);
-    CK(sk::launch_reduce_slices(l.dws, l.wsl, dst, l.wg_count, ws));
+    ProfScope ps(c, K_GEMM_WGRAD, (double)l.wsl * l.wg_count * 4 + (double)l.wg_count * 8, 0, ws);
+    CK(sk::launch_reduce_slices(l.dws, l.wsl, dst, l.wg_count, ws, 0));  // cleared by begin_step
     return SKIPPER_OK;
 }
 

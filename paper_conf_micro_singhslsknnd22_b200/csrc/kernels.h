@@ -79,7 +79,9 @@ bool narrow_wgrad_supported(int cin, int cout, int stride, int H, int W);
 // the slices with launch_reduce_slices)
 int narrow_wgrad_slices(int cin, int cout, int stride, int H, int W, int num_sms);
 // dst[i] += sum_{s < nslices} slices[s * count + i] in slice order, then slices[s * count + i] = 0
-cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s);
+// zero = 0: the slices are left as they are (the engine clears them at the start of the next step, off the
+// critical path)
+cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s, int zero = 1);
 cudaError_t launch_narrow_wgrad(const uint16_t *X, const uint16_t *D, float *dW, int nb, int H, int W, int cin,
                                 int cout, int stride, cudaStream_t s, int num_sms);
 // dgrad of a narrow 3x3 conv, stride 1 or 2 (narrow_wgrad.cu): G [nb][s*H][s*W][cin] fp32 from the layer's

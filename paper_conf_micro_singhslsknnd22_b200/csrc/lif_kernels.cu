@@ -1073,7 +1073,7 @@ cudaError_t launch_readout_wgrad(const float *dz, const float *cnt_kept, float *
 // contiguous range of the slices (independent loads, in slice order), and warp 0 adds the 8 partials in
 // warp order - a fixed summation tree, so the result does not depend on scheduling.
 __global__ void __launch_bounds__(256) reduce_slices_kernel(float4 *__restrict__ slices, int nslices,
-                                                            float4 *__restrict__ dst, long long count4) {
+                                                            float4 *__restrict__ dst, long long count4, int zero) {
     pdl_enter();
     __shared__ float4 part[8][32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -1089,13 +1089,13 @@ __global__ void __launch_bounds__(256) reduce_slices_kernel(float4 *__restrict__
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
                 acc.x += v[k].x; acc.y += v[k].y; acc.z += v[k].z; acc.w += v[k].w;
-                slices[(long long)(s + k) * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (zero) slices[(long long)(s + k) * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
             }
         }
         for (; s < s1; ++s) {
             const float4 v = slices[(long long)s * count4 + i];
             acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
-            slices[(long long)s * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (zero) slices[(long long)s * count4 + i] = make_float4(0.f, 0.f, 0.f, 0.f);
         }
     }
     part[w][lane] = acc;
@@ -1112,13 +1112,13 @@ __global__ void __launch_bounds__(256) reduce_slices_kernel(float4 *__restrict__
     }
 }
 
-cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s) {
+cudaError_t launch_reduce_slices(float *slices, int nslices, float *dst, size_t count, cudaStream_t s, int zero) {
     if (count % 4 || (reinterpret_cast<uintptr_t>(slices) & 15) || (reinterpret_cast<uintptr_t>(dst) & 15))
         return cudaErrorInvalidValue;
     const long long c4 = (long long)(count / 4);
     if (c4 == 0 || nslices <= 0) return cudaSuccess;
     sk_launch(reduce_slices_kernel, (unsigned)((c4 + 31) / 32), 256, 0, s, reinterpret_cast<float4 *>(slices), nslices,
-              reinterpret_cast<float4 *>(dst), c4);
+              reinterpret_cast<float4 *>(dst), c4, zero);
     return cudaGetLastError();
 }
 
