@@ -50,7 +50,10 @@ static constexpr int L0_NACC = 4;  // TMEM accumulator ring (rows in flight betw
 static constexpr uint32_t L0_A_BYTES = 128 * 32 * 2;  // 128 rows x K=32 bf16
 static constexpr uint32_t L0_PLANE_A = 128 * 16;      // one 8-column K chunk of all 128 rows
 // forward kernel: warps 0-7 producers (two groups alternating rows), warp 8 MMA, warps 9..: epilogue
-static constexpr int L0_PGROUPS = 2;
+#ifndef SK_L0_PGROUPS
+#define SK_L0_PGROUPS 2
+#endif
+static constexpr int L0_PGROUPS = SK_L0_PGROUPS;  // producer groups (rows alternate between them)
 static constexpr int F0_PROD_WARPS = 4 * L0_PGROUPS;
 static constexpr int F0_MMA_WARP = F0_PROD_WARPS;
 static constexpr int F0_EPI_WARP0 = F0_PROD_WARPS + 1;
