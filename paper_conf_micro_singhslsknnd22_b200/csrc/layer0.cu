@@ -45,8 +45,14 @@ namespace sk {
 static constexpr int L0_PROD_WARPS = 4;
 static constexpr int L0_MMA_WARP = 4;
 static constexpr int L0_EPI_WARP0 = 5;
-static constexpr int L0_STAGES = 6;
-static constexpr int L0_NACC = 4;  // TMEM accumulator ring (rows in flight between MMA and epilogue)
+#ifndef SK_L0_STAGES
+#define SK_L0_STAGES 6
+#endif
+static constexpr int L0_STAGES = SK_L0_STAGES;
+#ifndef SK_L0_NACC
+#define SK_L0_NACC 4
+#endif
+static constexpr int L0_NACC = SK_L0_NACC;  // TMEM accumulator ring (rows in flight between MMA and epilogue)
 static constexpr uint32_t L0_A_BYTES = 128 * 32 * 2;  // 128 rows x K=32 bf16
 static constexpr uint32_t L0_PLANE_A = 128 * 16;      // one 8-column K chunk of all 128 rows
 // forward kernel: warps 0-7 producers (two groups alternating rows), warp 8 MMA, warps 9..: epilogue

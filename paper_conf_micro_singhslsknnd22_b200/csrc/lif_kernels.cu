@@ -414,10 +414,12 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
 #ifndef SK_BWD_MINB
 #define SK_BWD_MINB 8
 #endif
-template <int SPLIT, int KIND>
+#ifndef SK_BWD_CH1_MAX_R
+#define SK_BWD_CH1_MAX_R 12
+#endif
+template <int SPLIT, int KIND, int CH>
 __global__ void __launch_bounds__(256, SPLIT ? 4 : SK_BWD_MINB) lif_bwd_kernel(const ScanBwdArgs a) {
     pdl_enter();
-    constexpr int CH = SK_BWD_CH;
     const int C = a.C;
     const long long HW = (long long)a.H * a.W;
     const long long rs = (long long)a.B * HW * C;
@@ -640,13 +642,23 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
     const long long P = rs / 4;
     const unsigned grid = (unsigned)((P + 255) / 256);
     const bool tri = a.surr == SURR_TRIANGLE;
+    // rows per unrolled chunk: 1 for short segments (per-segment SKIP schedules of a few kept rows: cfg 2 step
+    // 5.867 -> 5.832 ms in alternating runs, the leaner loop co-resides better with the side-stream weight
+    // gradients), 2 for long ones (cfg 4's 30-row segments measured 1 % slower with 1)
+    const bool ch1 = a.R <= SK_BWD_CH1_MAX_R;
+#define BWD_LAUNCH(SPL, KND)                                                         \
+    do {                                                                             \
+        if (ch1) sk_launch(lif_bwd_kernel<SPL, KND, 1>, grid, 256, 0, s, a);        \
+        else sk_launch(lif_bwd_kernel<SPL, KND, SK_BWD_CH>, grid, 256, 0, s, a);   \
+    } while (0)
     if (a.nsplit > 1) {
-        if (tri) sk_launch(lif_bwd_kernel<1, SURR_TRIANGLE>, grid, 256, 0, s, a);
-        else sk_launch(lif_bwd_kernel<1, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+        if (tri) BWD_LAUNCH(1, SURR_TRIANGLE);
+        else BWD_LAUNCH(1, SURR_FAST_SIGMOID);
     } else {
-        if (tri) sk_launch(lif_bwd_kernel<0, SURR_TRIANGLE>, grid, 256, 0, s, a);
-        else sk_launch(lif_bwd_kernel<0, SURR_FAST_SIGMOID>, grid, 256, 0, s, a);
+        if (tri) BWD_LAUNCH(0, SURR_TRIANGLE);
+        else BWD_LAUNCH(0, SURR_FAST_SIGMOID);
     }
+#undef BWD_LAUNCH
     return cudaGetLastError();
 }
 
