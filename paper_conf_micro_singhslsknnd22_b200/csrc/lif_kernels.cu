@@ -9,6 +9,13 @@
 #include "common.cuh"
 #include "kernels.h"
 
+#ifndef SK_FS_CH_SPLIT
+#define SK_FS_CH_SPLIT 4  // rows per chunk of the fc forward scan over split-K partial currents
+#endif
+#ifndef SK_BS_CH_SPLIT
+#define SK_BS_CH_SPLIT 4  // rows per chunk of the fc reverse scan over split-K partial gradients
+#endif
+
 namespace sk {
 
 SK_DEV float lif_update(float U, float I, float o, float lam, float th) {
@@ -378,7 +385,7 @@ cudaError_t launch_lif_fwd(const ScanFwdArgs &a, cudaStream_t s) {
         const size_t smem = a.s_part ? (size_t)a.R * sizeof(unsigned) : 0;
         if (smem > 48 * 1024) return cudaErrorInvalidValue;
         if (a.nsplit > 1)
-            sk_launch(lif_fwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
+            sk_launch(lif_fwd_small_kernel<SK_FS_CH_SPLIT, 1>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         else
             sk_launch(lif_fwd_small_kernel<8, 0>, (unsigned)((rs + 255) / 256), 256, smem, s, a);
         return cudaGetLastError();
@@ -634,7 +641,7 @@ cudaError_t launch_lif_bwd(const ScanBwdArgs &a, cudaStream_t s) {
             return cudaGetLastError();
         }
         if (a.nsplit > 1)
-            sk_launch(lif_bwd_small_kernel<4, 1>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
+            sk_launch(lif_bwd_small_kernel<SK_BS_CH_SPLIT, 1>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
         else
             sk_launch(lif_bwd_small_kernel<16, 0>, (unsigned)((rs + 255) / 256), 256, 0, s, a);
         return cudaGetLastError();
