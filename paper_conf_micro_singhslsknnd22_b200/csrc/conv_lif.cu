@@ -365,7 +365,7 @@ __global__ void __launch_bounds__(CL_THREADS, 1)
                     tmem_ld_wait();
 #pragma unroll
                     for (int c = 0; c < 32; ++c)
-                        d[32 * j + c] = __fmaf_rn(sgm(u[c]), __uint_as_float(v[c]), __fmul_rn(lam, d[32 * j + c]));
+                        d[32 * j + c] = sgm(u[c]) * __uint_as_float(v[c]) + lam * d[32 * j + c];  // as lif_bwd_kernel
                 }
                 tc_fence_before();
                 __syncwarp();

@@ -486,11 +486,10 @@ __global__ void __launch_bounds__(256, SPLIT ? 4 : SK_BWD_MINB) lif_bwd_kernel(c
         return g;
     };
     auto step = [&](const float4 &u, const float4 &g, uint2 *dp) {
-        // explicit rounding (sigma' g + (lam d)), as the fused dgrad + scan epilogue (conv_lif.cu, BWD)
-        d.x = __fmaf_rn(sgm(u.x), g.x, __fmul_rn(lam, d.x));
-        d.y = __fmaf_rn(sgm(u.y), g.y, __fmul_rn(lam, d.y));
-        d.z = __fmaf_rn(sgm(u.z), g.z, __fmul_rn(lam, d.z));
-        d.w = __fmaf_rn(sgm(u.w), g.w, __fmul_rn(lam, d.w));
+        d.x = sgm(u.x) * g.x + lam * d.x;
+        d.y = sgm(u.y) * g.y + lam * d.y;
+        d.z = sgm(u.z) * g.z + lam * d.z;
+        d.w = sgm(u.w) * g.w + lam * d.w;
         if (dp) *dp = pack_bf16x4(d.x, d.y, d.z, d.w);
     };
     for (; r >= CH - 1; r -= CH) {
